@@ -1,0 +1,207 @@
+/*
+ * eirene.h -- C ABI of the B200-native Eirene batched B+tree.
+ *
+ * The library processes batches of Query / Update / Insert / Delete requests
+ * on a B+tree resident in GPU global memory and returns linearizable results
+ * (PAPER.md, Zhang et al., PPoPP'23).  Citations: P:N = /root/reference/PAPER.md
+ * line N, Alg.1:k = line k of Algorithm 1, SURVEY §x = SURVEY.md.
+ *
+ * Problem statement the calls follow:
+ *   - requests are buffered by the host and shipped to the GPU in batches
+ *     (P:167-171);
+ *   - each request carries a key, a value and a type: query, or one of the
+ *     update requests update / insertion / deletion;
+ *   - the logical timestamp of a request is its position in the buffer
+ *     (P:718-722); batches are linearized in submission order;
+ *   - results are linearizable: result[i] is the value the key
+ *     held immediately before request i in timestamp order, or
+ *     EIRENE_NOT_FOUND if it was absent.  Writes return the prior value too
+ *     (SURVEY §8(c) reading 1).  UPDATE and INSERT are both blind upserts,
+ *     DELETE erases (no-op on an absent key) (§8(c) readings 2-3).
+ *
+ * Conventions: pointers named *_dev are CUDA device pointers, *_host are host
+ * pointers (pinned memory recommended).  All calls return EIRENE_OK (0) or a
+ * negative error code; eirene_strerror() names it.  A handle is bound to one
+ * device, is single-stream and is NOT thread-safe.  No call allocates device
+ * memory after eirene_create except eirene_scan / eirene_check_invariants
+ * (quiescent utilities).
+ */
+#ifndef EIRENE_H
+#define EIRENE_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct CUstream_st* eirene_stream_t;   /* == cudaStream_t; NULL = legacy default stream */
+
+/* Result sentinel (null).  UINT64_MAX is also reserved as a key and
+ * as a written value; requests using it are rejected with EIRENE_EINVAL. */
+#define EIRENE_NOT_FOUND UINT64_MAX
+
+enum {
+  EIRENE_OK = 0,
+  EIRENE_EINVAL = -1,   /* bad argument or invalid request in a batch          */
+  EIRENE_ENOMEM = -2,   /* device allocation failed in create                  */
+  EIRENE_EFULL = -3,    /* node pools lack headroom for the batch's worst case */
+  EIRENE_ESTATE = -4,   /* call not valid in the handle's state / stale ticket */
+  EIRENE_ECUDA = -5,    /* a CUDA runtime error; eirene_last_cuda_error()      */
+  EIRENE_EINTERNAL = -6 /* device watchdog fired (a bug: no forward progress); the
+                           tree must be discarded                              */
+};
+
+/* Request types. */
+enum { EIRENE_QUERY = 0, EIRENE_UPDATE = 1, EIRENE_INSERT = 2, EIRENE_DELETE = 3 };
+
+/* eirene_config.flags */
+enum {
+  EIRENE_F_REGROUP = 1u << 0,   /* leaf-bucketed warp regrouping in the update kernel;
+                                   off = one warp per issued write (ablation, exercises retries) */
+  EIRENE_F_STATS = 1u << 1,     /* count retries / STM fallbacks / splits on the device           */
+  EIRENE_F_FORCE_STM = 1u << 2, /* every traversal in the update kernel is STM-protected
+                                   (equivalent to retry_threshold = 0, Alg.1:28-33)               */
+  EIRENE_F_TIMING = 1u << 3     /* record per-stage CUDA events (eirene_batch_stats.stage_ms)     */
+};
+
+typedef struct {
+  int device;                 /* CUDA device ordinal                                           */
+  uint32_t fanout;            /* node capacity; must be 16 (SURVEY §8(c) reading 12)           */
+  uint64_t max_keys;          /* sizes the node pools (keys the tree may hold)                 */
+  uint32_t max_batch;         /* largest n accepted by submit (sizes all scratch), <= 2^30     */
+  uint32_t retry_threshold;   /* THRESHOLD of Alg.1:28; attempts before the STM fallback       */
+  uint32_t flags;             /* EIRENE_F_*                                                    */
+  uint64_t key_lo, key_hi;    /* key range owned by this tree (shard), [key_lo, key_hi);
+                                 0 .. UINT64_MAX for a single GPU                              */
+} eirene_config;
+
+/* Fills *cfg with the defaults: device 0, fanout 16, max_keys 2^24,
+ * max_batch 2^20, retry_threshold 4, flags REGROUP|STATS, range [0, UINT64_MAX). */
+void eirene_default_config(eirene_config* cfg);
+
+typedef struct eirene_tree* eirene_handle;
+
+typedef struct {
+  int32_t status;             /* EIRENE_OK, EIRENE_EINVAL (invalid request: tree untouched),
+                                 EIRENE_EFULL (no headroom: tree untouched)                    */
+  uint32_t n;                 /* requests in the batch                                         */
+  uint64_t distinct;          /* distinct keys == issued requests                  */
+  uint64_t issued_q;          /* issued queries  (query kernel, Alg.1:4)                       */
+  uint64_t issued_w;          /* issued writes   (update kernel, Alg.1:5)                      */
+  uint64_t leaf_runs;         /* leaf runs processed by the update kernel (regrouping)         */
+  uint64_t retries;           /* failed optimistic / transactional attempts (Alg.1:41)         */
+  uint64_t stm_fallbacks;     /* attempts made with STM-protected traversal (Alg.1:30-33)      */
+  uint64_t leaf_splits;       /* leaves split                                    */
+  uint64_t inner_splits;      /* inner nodes split                                             */
+  uint64_t new_leaves, new_inner;
+  uint32_t height;            /* tree height after the batch (1 = root is a leaf)              */
+  uint32_t launches;          /* kernels launched for this batch                               */
+  float stage_ms[8];          /* EIRENE_F_TIMING: sort, combine, partition, query, update,
+                                 result, (unused), total                                       */
+} eirene_batch_stats;
+
+/* Creates a tree (one empty leaf) on cfg->device and allocates every pool and
+ * scratch buffer up front.  Errors: EINVAL (null / fanout != 16 / sizes),
+ * ENOMEM, ECUDA. */
+int eirene_create(const eirene_config* cfg, eirene_handle* out);
+
+/* Builds the tree bottom-up from n key/value pairs in device memory (the RF /
+ * tree construction step).  keys_dev must be strictly increasing,
+ * inside [key_lo, key_hi) and != UINT64_MAX; vals_dev != UINT64_MAX.  leaf_fill
+ * in (0, 1] sets the initial keys per leaf (round(16*fill)); it changes shape
+ * and speed only (§8(c) reading 13).  Valid only on a freshly created tree
+ * (ESTATE otherwise).  Synchronous with respect to `stream`; EINVAL if the
+ * device check of the keys fails (tree left empty). */
+int eirene_bulk_load(eirene_handle h, const uint64_t* keys_dev, const uint64_t* vals_dev,
+                     uint64_t n, float leaf_fill, eirene_stream_t stream);
+
+/* Submits one batch of n requests (Alg.1:1-7): ops_dev[n] (u8, EIRENE_*),
+ * keys_dev[n], vals_dev[n] (ignored for queries and deletes) and writes
+ * results_dev[n] (u64, timestamp = index order).  Asynchronous on `stream`;
+ * the caller keeps every buffer alive until eirene_results(ticket) returns.
+ * Pipeline: stable radix sort by key (Alg.1:10), combine/resolve (Alg.1:11,
+ * P:724-758), partition (Alg.1:3), query kernel (Alg.1:15-21), update kernel
+ * with optimistic retry and STM fallback (Alg.1:23-46), RESULT_CAL (Alg.1:6).
+ * Synchronous errors: EINVAL (null pointers, n == 0 or n > max_batch), ESTATE.
+ * Invalid requests (op > 3, key == UINT64_MAX or outside [key_lo, key_hi),
+ * upsert value == UINT64_MAX) are detected on the device: the batch then
+ * leaves the tree untouched and eirene_results reports EINVAL. */
+int eirene_submit_batch(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev,
+                        const uint64_t* vals_dev, uint32_t n, uint64_t* results_dev,
+                        eirene_stream_t stream, uint64_t* ticket);
+
+/* Same batch from HOST buffers: copies the requests host->device into
+ * handle-owned staging buffers, runs the pipeline, copies results device->host,
+ * all on `stream`.  The copies run at full speed only from pinned memory.
+ * Results are valid after eirene_results(ticket). */
+int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops_host, const uint64_t* keys_host,
+                             const uint64_t* vals_host, uint32_t n, uint64_t* results_host,
+                             eirene_stream_t stream, uint64_t* ticket);
+
+/* Waits for batch `ticket` and returns its status (EIRENE_OK, EINVAL, EFULL);
+ * fills *stats if non-NULL.  ESTATE if the ticket is unknown or too old (the
+ * handle remembers the last 64 batches). */
+int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats);
+
+/* In-order scan of the quiescent tree: pairs with lo <= key <= hi (inclusive,
+ * §8(c) reading 23) in ascending key order.  Writes min(count, cap) pairs to
+ * keys_out_dev / vals_out_dev (either may be NULL when cap == 0) and the total
+ * to *count.  Synchronous with respect to `stream`.  Used for parity and as
+ * the save half of save/restore (bulk_load is the restore half). */
+int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out_dev,
+                uint64_t* vals_out_dev, uint64_t cap, uint64_t* count, eirene_stream_t stream);
+
+/* Debug: copies the node pools to the host and checks the structural
+ * invariants of the quiescent tree: keys strictly increasing in every node,
+ * counts <= 16, children inside their parent's fences, uniform leaf depth,
+ * leaf chain == in-order leaves, fences contiguous, no node locked.  Returns
+ * 0 when they hold, else a positive code; *n_keys = keys in the tree. */
+int eirene_check_invariants(eirene_handle h, uint64_t* n_keys);
+
+typedef struct {
+  uint32_t height;            /* 1 = the root is a leaf */
+  uint32_t root;
+  uint64_t leaves, inner;     /* allocated nodes */
+  uint64_t leaf_cap, inner_cap;
+  uint64_t launches;          /* kernels launched by this handle so far */
+  uint64_t device_bytes;      /* device memory owned by the handle */
+} eirene_tree_info;
+
+/* Synchronous snapshot of the tree's size counters. */
+int eirene_get_info(eirene_handle h, eirene_tree_info* info);
+
+/* Frees every device and host resource of the handle (waits for pending work). */
+int eirene_destroy(eirene_handle h);
+
+const char* eirene_strerror(int code);
+/* Text of the last CUDA error seen by any handle in this process. */
+const char* eirene_last_cuda_error(void);
+
+/* ---- multi-GPU key-range routing; the collective itself is
+ * torch.distributed all_to_all_single (NCCL) issued by the caller ----------- */
+
+/* Stable partition of n requests by destination shard,
+ * dest(k) = #{ s in splitters[0..P-2] : s <= k } (upper_bound), so shard r
+ * owns [splitters[r-1], splitters[r]).  splitters_dev holds P-1 increasing
+ * keys (device), 1 <= P <= 64.  Writes send_ops/keys/vals_dev[n] grouped by
+ * destination in input (timestamp) order, perm_dev[n] (perm[j] = input index
+ * of send slot j) and counts_dev[P] (u32).  `h` provides scratch only.
+ * Asynchronous on `stream`. */
+int eirene_route_partition(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev,
+                           const uint64_t* vals_dev, uint32_t n, const uint64_t* splitters_dev,
+                           int P, uint8_t* send_ops_dev, uint64_t* send_keys_dev,
+                           uint64_t* send_vals_dev, uint32_t* perm_dev, uint32_t* counts_dev,
+                           eirene_stream_t stream);
+
+/* Inverse of the partition for the returned results:
+ * results_dev[perm_dev[j]] = recv_results_dev[j] for j < n.  Asynchronous. */
+int eirene_route_unpermute(eirene_handle h, const uint64_t* recv_results_dev,
+                           const uint32_t* perm_dev, uint32_t n, uint64_t* results_dev,
+                           eirene_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EIRENE_H */

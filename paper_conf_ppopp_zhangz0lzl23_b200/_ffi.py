@@ -1,0 +1,109 @@
+"""ctypes binding of include/eirene.h (argument marshalling only).
+
+Every function of the C ABI is exposed under the same name.  The library is
+the in-tree libeirene.so built by `build.py`; importing this module never
+falls back to anything else: if the library is missing or cannot be loaded,
+`lib()` raises.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import re
+
+PKG = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(PKG)
+LIB_PATH = os.path.join(PKG, "libeirene.so")
+HEADER = os.path.join(ROOT, "include", "eirene.h")
+
+EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECUDA = 0, -1, -2, -3, -4, -5
+EIRENE_QUERY, EIRENE_UPDATE, EIRENE_INSERT, EIRENE_DELETE = 0, 1, 2, 3
+EIRENE_F_REGROUP, EIRENE_F_STATS, EIRENE_F_FORCE_STM, EIRENE_F_TIMING = 1, 2, 4, 8
+NOT_FOUND = 0xFFFFFFFFFFFFFFFF
+
+_u64 = ctypes.c_uint64
+_u32 = ctypes.c_uint32
+_vp = ctypes.c_void_p
+_int = ctypes.c_int
+
+
+class eirene_config(ctypes.Structure):
+    _fields_ = [("device", ctypes.c_int), ("fanout", _u32), ("max_keys", _u64), ("max_batch", _u32),
+                ("retry_threshold", _u32), ("flags", _u32), ("key_lo", _u64), ("key_hi", _u64)]
+
+
+class eirene_batch_stats(ctypes.Structure):
+    _fields_ = [("status", ctypes.c_int32), ("n", _u32), ("distinct", _u64), ("issued_q", _u64),
+                ("issued_w", _u64), ("leaf_runs", _u64), ("retries", _u64), ("stm_fallbacks", _u64),
+                ("leaf_splits", _u64), ("inner_splits", _u64), ("new_leaves", _u64), ("new_inner", _u64),
+                ("height", _u32), ("launches", _u32), ("stage_ms", ctypes.c_float * 8)]
+
+    def to_dict(self) -> dict:
+        d = {f: getattr(self, f) for f, _ in self._fields_ if f != "stage_ms"}
+        d["stage_ms"] = list(self.stage_ms)
+        return d
+
+
+class eirene_tree_info(ctypes.Structure):
+    _fields_ = [("height", _u32), ("root", _u32), ("leaves", _u64), ("inner", _u64), ("leaf_cap", _u64),
+                ("inner_cap", _u64), ("launches", _u64), ("device_bytes", _u64)]
+
+
+_SIGS = {
+    "eirene_default_config": (None, [ctypes.POINTER(eirene_config)]),
+    "eirene_create": (_int, [ctypes.POINTER(eirene_config), ctypes.POINTER(_vp)]),
+    "eirene_bulk_load": (_int, [_vp, _vp, _vp, _u64, ctypes.c_float, _vp]),
+    "eirene_submit_batch": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _vp, ctypes.POINTER(_u64)]),
+    "eirene_submit_batch_host": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _vp, ctypes.POINTER(_u64)]),
+    "eirene_results": (_int, [_vp, _u64, ctypes.POINTER(eirene_batch_stats)]),
+    "eirene_scan": (_int, [_vp, _u64, _u64, _vp, _vp, _u64, ctypes.POINTER(_u64), _vp]),
+    "eirene_check_invariants": (_int, [_vp, ctypes.POINTER(_u64)]),
+    "eirene_get_info": (_int, [_vp, ctypes.POINTER(eirene_tree_info)]),
+    "eirene_destroy": (_int, [_vp]),
+    "eirene_strerror": (ctypes.c_char_p, [_int]),
+    "eirene_last_cuda_error": (ctypes.c_char_p, []),
+    "eirene_route_partition": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _int, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "eirene_route_unpermute": (_int, [_vp, _vp, _vp, _u32, _vp, _vp]),
+}
+
+_lib = None
+
+
+def header_functions() -> list[str]:
+    """Names of the functions include/eirene.h declares."""
+    with open(HEADER) as f:
+        text = f.read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    return sorted(set(re.findall(r"\b(eirene_[a-z_]+)\s*\(", text)))
+
+
+def lib() -> ctypes.CDLL:
+    """Load libeirene.so (raises if it was not built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise RuntimeError(f"{LIB_PATH} is missing: run `python -m paper_conf_ppopp_zhangz0lzl23_b200.build` "
+                               "(there is no CPU fallback)")
+        L = ctypes.CDLL(LIB_PATH)
+        for name, (res, args) in _SIGS.items():
+            fn = getattr(L, name)
+            fn.restype = res
+            fn.argtypes = args
+        _lib = L
+    return _lib
+
+
+class EireneError(RuntimeError):
+    def __init__(self, code: int, where: str):
+        L = lib()
+        msg = L.eirene_strerror(code).decode()
+        if code == EIRENE_ECUDA:
+            msg += ": " + L.eirene_last_cuda_error().decode()
+        super().__init__(f"{where}: {msg} ({code})")
+        self.code = code
+
+
+def check(code: int, where: str) -> int:
+    if code != EIRENE_OK:
+        raise EireneError(code, where)
+    return code

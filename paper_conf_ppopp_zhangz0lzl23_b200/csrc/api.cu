@@ -1,0 +1,559 @@
+// api.cu -- the C ABI (include/eirene.h): handle, pools, batch sequencing.
+//
+// A batch (Alg.1:1-7) is a fixed chain of kernels on the caller's stream:
+//   memset(batch scratch) -> sort upsweep + 8 digit passes (Alg.1:10)
+//   -> combine (Alg.1:11) -> partition (Alg.1:3) -> query + write-locate
+//   (Alg.1:4) -> update (Alg.1:5) -> RESULT_CAL (Alg.1:6) -> finalize
+// followed by an async copy of the batch's device scalars into a pinned ring
+// slot and an event; eirene_results() waits on that event.  No allocation and
+// no host synchronisation happen inside submit.
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "eirene_internal.cuh"
+
+using namespace eirene;
+
+namespace {
+
+constexpr int RING = 64;
+constexpr int NSTAGE = 7;
+
+std::mutex g_err_mu;
+std::string g_last_cuda_error = "no error";
+
+int cuda_fail(cudaError_t e, const char* where) {
+  std::lock_guard<std::mutex> lk(g_err_mu);
+  g_last_cuda_error = std::string(where) + ": " + cudaGetErrorString(e);
+  return EIRENE_ECUDA;
+}
+
+#define CK(expr)                                    \
+  do {                                              \
+    cudaError_t _e = (expr);                        \
+    if (_e != cudaSuccess) return cuda_fail(_e, #expr); \
+  } while (0)
+
+__global__ void finalize_kernel(BatchCtl* ctl, const TreeHdr* hdr) {
+  if (threadIdx.x == 0) {
+    if (ctl->invalid) ctl->status = EIRENE_EINVAL;
+    ctl->height = (uint32_t)(hdr->root_word >> 32);
+  }
+}
+
+__global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
+  const int i = threadIdx.x;
+  if (i < FAN) {
+    t.lkeys[i] = KEY_MAX;
+    t.lvals[i] = 0;
+  }
+  if (i == 0) {
+    NodeMeta m;
+    m.version = 0;
+    m.next = NIL;
+    m.lo = key_lo;
+    m.hi = key_hi;
+    m.count = 0;
+    m.level = 0;
+    t.lmeta[0] = m;
+    TreeHdr* h = t.hdr;
+    h->root_word = (1ull << 32) | 0ull;
+    h->leaf_count = 1;
+    h->inner_count = 0;
+    for (int l = 0; l < MAX_LEVELS; ++l) h->level_count[l] = 0;
+    h->level_count[0] = 1;
+  }
+}
+
+struct Rec {
+  uint64_t ticket = 0;
+  bool used = false;
+  bool timing = false;
+  uint32_t n = 0;
+  int launches = 0;
+  cudaEvent_t done = nullptr;
+  cudaEvent_t st[NSTAGE] = {};
+};
+
+}  // namespace
+
+struct eirene_tree {
+  eirene_config cfg{};
+  int num_sms = 148;
+  Tree t{};
+  SortBufs sb{};
+  CombBufs cb{};
+  UpdParams up{};
+  unsigned char* zero_region = nullptr;
+  size_t zero_bytes = 0;
+  BatchCtl* ctl = nullptr;
+  BatchCtl* host_ctl = nullptr;   // pinned [RING]
+  uint8_t* st_ops = nullptr;
+  uint64_t* st_keys = nullptr;
+  uint64_t* st_vals = nullptr;
+  uint64_t* st_res = nullptr;
+  unsigned long long* route_lb = nullptr;
+  uint32_t* route_ctr = nullptr;
+  uint32_t route_epoch = 0;
+  Rec ring[RING];
+  uint64_t next_ticket = 1;
+  uint32_t batch_seq = 0;
+  bool loaded = false;
+  bool modified = false;
+  uint64_t launches = 0;
+  size_t device_bytes = 0;
+  std::vector<void*> allocs;
+
+  template <class T>
+  cudaError_t dalloc(T** p, size_t count) {
+    size_t bytes = sizeof(T) * (count ? count : 1);
+    cudaError_t e = cudaMalloc(reinterpret_cast<void**>(p), bytes);
+    if (e == cudaSuccess) {
+      allocs.push_back(*p);
+      device_bytes += bytes;
+    }
+    return e;
+  }
+};
+
+extern "C" {
+
+void eirene_default_config(eirene_config* c) {
+  if (!c) return;
+  std::memset(c, 0, sizeof(*c));
+  c->device = 0;
+  c->fanout = 16;
+  c->max_keys = 1ull << 24;
+  c->max_batch = 1u << 20;
+  c->retry_threshold = 4;
+  c->flags = EIRENE_F_REGROUP | EIRENE_F_STATS;
+  c->key_lo = 0;
+  c->key_hi = UINT64_MAX;
+}
+
+const char* eirene_strerror(int code) {
+  switch (code) {
+    case EIRENE_OK: return "ok";
+    case EIRENE_EINVAL: return "invalid argument or invalid request";
+    case EIRENE_ENOMEM: return "device allocation failed";
+    case EIRENE_EFULL: return "node pools lack headroom for the batch";
+    case EIRENE_ESTATE: return "call not valid in this state (or stale ticket)";
+    case EIRENE_ECUDA: return "CUDA error (see eirene_last_cuda_error)";
+    default: return "unknown error";
+  }
+}
+
+const char* eirene_last_cuda_error(void) {
+  std::lock_guard<std::mutex> lk(g_err_mu);
+  static thread_local std::string copy;
+  copy = g_last_cuda_error;
+  return copy.c_str();
+}
+
+int eirene_destroy(eirene_handle h);
+
+int eirene_create(const eirene_config* cfg, eirene_handle* out) {
+  if (!cfg || !out) return EIRENE_EINVAL;
+  *out = nullptr;
+  if (cfg->fanout != 16 || cfg->max_batch == 0 || cfg->max_batch > (1u << 29) || cfg->key_lo >= cfg->key_hi ||
+      cfg->max_keys == 0)
+    return EIRENE_EINVAL;
+  CK(cudaSetDevice(cfg->device));
+  eirene_tree* h = new (std::nothrow) eirene_tree();
+  if (!h) return EIRENE_ENOMEM;
+  h->cfg = *cfg;
+  cudaDeviceGetAttribute(&h->num_sms, cudaDevAttrMultiProcessorCount, cfg->device);
+  const uint64_t nb = cfg->max_batch;
+  // Pools: leaves for max_keys at >= half fill plus one batch of worst-case
+  // splits; inner nodes: a 1/4 of that (every inner node keeps >= 8 children
+  // after a split) plus a batch of root growth.
+  uint64_t leaf_cap = cfg->max_keys / 8 + 2 * nb + 1024;
+  uint64_t inner_cap = leaf_cap / 4 + nb + 1024;
+  if (leaf_cap > 0x7FFFFFF0ull || inner_cap > 0x7FFFFFF0ull) {
+    delete h;
+    return EIRENE_EINVAL;
+  }
+  cudaError_t e = cudaSuccess;
+  Tree& t = h->t;
+  t.leaf_cap = (uint32_t)leaf_cap;
+  t.inner_cap = (uint32_t)inner_cap;
+  const size_t sort_tiles = (nb + SORT_TILE - 1) / SORT_TILE;
+  const size_t comb_tiles = (nb + COMB_TILE - 1) / COMB_TILE;
+#define AL(p, n)                                 \
+  if (e == cudaSuccess) e = h->dalloc(&(p), (n));
+  AL(t.lkeys, leaf_cap * FAN);
+  AL(t.lvals, leaf_cap * FAN);
+  AL(t.lmeta, leaf_cap);
+  AL(t.ikeys, inner_cap * FAN);
+  AL(t.ichild, inner_cap * FAN);
+  AL(t.imeta, inner_cap);
+  AL(t.hdr, 1);
+  AL(h->sb.kA, nb);
+  AL(h->sb.kB, nb);
+  AL(h->sb.pA, nb);
+  AL(h->sb.pB, nb);
+  AL(h->sb.lookback, sort_tiles * 256);
+  AL(h->cb.pinfo, nb);
+  AL(h->cb.ikey, nb);
+  AL(h->cb.iop, nb);
+  AL(h->cb.ival, nb);
+  AL(h->cb.qkey, nb);
+  AL(h->cb.qseg, nb);
+  AL(h->cb.wkey, nb);
+  AL(h->cb.wop, nb);
+  AL(h->cb.wval, nb);
+  AL(h->cb.wseg, nb);
+  AL(h->cb.wleaf, nb);
+  AL(h->cb.old, nb);
+  AL(h->up.entA_key, nb + 64);
+  AL(h->up.entA_child, nb + 64);
+  AL(h->up.entB_key, nb + 64);
+  AL(h->up.entB_child, nb + 64);
+  AL(h->st_ops, nb);
+  AL(h->st_keys, nb);
+  AL(h->st_vals, nb);
+  AL(h->st_res, nb);
+  AL(h->route_lb, ((nb + 2047) / 2048) * 64);
+  AL(h->route_ctr, 1);
+  // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
+  {
+    size_t off = 0;
+    auto bump = [&](size_t bytes) {
+      size_t o = off;
+      off += (bytes + 255) & ~size_t(255);
+      return o;
+    };
+    const size_t o_ctl = bump(sizeof(BatchCtl));
+    const size_t o_gh = bump(sizeof(uint32_t) * 8 * 256);
+    const size_t o_cs = bump(sizeof(unsigned long long) * comb_tiles);
+    const size_t o_ps = bump(sizeof(unsigned long long) * comb_tiles);
+    h->zero_bytes = off;
+    AL(h->zero_region, off);
+    if (e == cudaSuccess) {
+      h->ctl = reinterpret_cast<BatchCtl*>(h->zero_region + o_ctl);
+      h->sb.ghist = reinterpret_cast<uint32_t*>(h->zero_region + o_gh);
+      h->cb.comb_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_cs);
+      h->cb.part_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_ps);
+    }
+  }
+#undef AL
+  if (e == cudaSuccess) e = cudaMallocHost(reinterpret_cast<void**>(&h->host_ctl), sizeof(BatchCtl) * RING);
+  for (int i = 0; i < RING && e == cudaSuccess; ++i) {
+    e = cudaEventCreateWithFlags(&h->ring[i].done, cudaEventDisableTiming);
+    for (int s = 0; s < NSTAGE && e == cudaSuccess; ++s) e = cudaEventCreate(&h->ring[i].st[s]);
+  }
+  if (e == cudaSuccess) e = cudaMemset(h->sb.lookback, 0, sizeof(unsigned long long) * sort_tiles * 256);
+  if (e == cudaSuccess) e = cudaMemset(h->route_lb, 0, sizeof(unsigned long long) * ((nb + 2047) / 2048) * 64);
+  if (e == cudaSuccess) {
+    init_empty_kernel<<<1, 32>>>(t, cfg->key_lo, cfg->key_hi);
+    e = cudaGetLastError();
+    if (e == cudaSuccess) e = cudaDeviceSynchronize();
+  }
+  if (e != cudaSuccess) {
+    int rc = (e == cudaErrorMemoryAllocation) ? EIRENE_ENOMEM : cuda_fail(e, "eirene_create");
+    eirene_destroy(h);
+    return rc;
+  }
+  h->up.threshold = cfg->retry_threshold;
+  h->up.flags = cfg->flags;
+  *out = h;
+  return EIRENE_OK;
+}
+
+int eirene_destroy(eirene_handle h) {
+  if (!h) return EIRENE_EINVAL;
+  cudaSetDevice(h->cfg.device);
+  cudaDeviceSynchronize();
+  for (int i = 0; i < RING; ++i) {
+    if (h->ring[i].done) cudaEventDestroy(h->ring[i].done);
+    for (int s = 0; s < NSTAGE; ++s)
+      if (h->ring[i].st[s]) cudaEventDestroy(h->ring[i].st[s]);
+  }
+  for (void* p : h->allocs) cudaFree(p);
+  if (h->host_ctl) cudaFreeHost(h->host_ctl);
+  delete h;
+  return EIRENE_OK;
+}
+
+int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals, uint64_t n, float leaf_fill,
+                     eirene_stream_t stream) {
+  if (!h) return EIRENE_EINVAL;
+  if (h->loaded || h->modified) return EIRENE_ESTATE;
+  if (n == 0) return EIRENE_OK;
+  if (!keys || !vals || !(leaf_fill > 0.f) || leaf_fill > 1.f) return EIRENE_EINVAL;
+  CK(cudaSetDevice(h->cfg.device));
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  int per = (int)(16.f * leaf_fill + 0.5f);
+  if (per < 1) per = 1;
+  if (per > 16) per = 16;
+  if ((n + per - 1) / per > h->t.leaf_cap) return EIRENE_EFULL;
+  int launches = 0;
+  uint32_t* flag = &h->ctl->invalid;
+  CK(cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, st));
+  launch_validate_bulk(keys, vals, n, h->cfg.key_lo, h->cfg.key_hi, flag, st, &launches);
+  uint32_t bad = 0;
+  CK(cudaMemcpyAsync(&bad, flag, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  if (bad) return EIRENE_EINVAL;
+  uint32_t height = 0;
+  int rc = build_tree(h->t, keys, vals, n, per, h->cfg.key_lo, h->cfg.key_hi, st, &launches, &height);
+  h->launches += launches;
+  CK(cudaGetLastError());
+  if (rc == EIRENE_OK) h->loaded = true;
+  return rc;
+}
+
+static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
+                       uint64_t* results, cudaStream_t st, uint64_t* results_host, uint64_t* ticket) {
+  CK(cudaSetDevice(h->cfg.device));
+  const uint64_t tk = h->next_ticket++;
+  Rec& r = h->ring[tk % RING];
+  r.ticket = tk;
+  r.used = true;
+  r.n = n;
+  r.timing = (h->cfg.flags & EIRENE_F_TIMING) != 0;
+  int launches = 0;
+  const uint32_t seq = ++h->batch_seq;
+  BatchCtl* ctl = h->ctl;
+  static const bool dbg = std::getenv("EIRENE_DEBUG_SYNC") != nullptr;
+  auto stage = [&](const char* name) {
+    if (!dbg) return;
+    cudaError_t e = cudaStreamSynchronize(st);
+    std::fprintf(stderr, "[eirene] batch %u stage %s done: %s\n", seq, name, cudaGetErrorString(e));
+  };
+  if (r.timing) cudaEventRecord(r.st[0], st);
+  CK(cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, st));
+  uint64_t* skey;
+  uint32_t* spay;
+  launch_sort(keys, ops, nullptr, vals, n, h->cfg.key_lo, h->cfg.key_hi, h->sb, ctl, seq * 8u, st, &launches, &skey,
+              &spay);
+  stage("sort");
+  if (r.timing) cudaEventRecord(r.st[1], st);
+  launch_combine(skey, spay, vals, results, n, h->cb, ctl, st, &launches);
+  stage("combine");
+  if (r.timing) cudaEventRecord(r.st[2], st);
+  launch_partition(n, h->cb, h->t, ctl, st, &launches);
+  stage("partition");
+  if (r.timing) cudaEventRecord(r.st[3], st);
+  launch_query(n, h->cb, h->t, ctl, h->num_sms, st, &launches);
+  stage("query");
+  if (r.timing) cudaEventRecord(r.st[4], st);
+  launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, st, &launches);
+  stage("update");
+  if (r.timing) cudaEventRecord(r.st[5], st);
+  launch_result(spay, n, h->cb, results, ctl, st, &launches);
+  stage("result");
+  finalize_kernel<<<1, 32, 0, st>>>(ctl, h->t.hdr);
+  ++launches;
+  if (r.timing) cudaEventRecord(r.st[6], st);
+  CK(cudaGetLastError());
+  if (results_host) CK(cudaMemcpyAsync(results_host, results, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, st));
+  CK(cudaMemcpyAsync(&h->host_ctl[tk % RING], ctl, sizeof(BatchCtl), cudaMemcpyDeviceToHost, st));
+  CK(cudaEventRecord(r.done, st));
+  r.launches = launches;
+  h->launches += launches;
+  h->modified = true;
+  *ticket = tk;
+  return EIRENE_OK;
+}
+
+int eirene_submit_batch(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
+                        uint64_t* results, eirene_stream_t stream, uint64_t* ticket) {
+  if (!h || !ops || !keys || !vals || !results || !ticket) return EIRENE_EINVAL;
+  if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
+  return submit_impl(h, ops, keys, vals, n, results, reinterpret_cast<cudaStream_t>(stream), nullptr, ticket);
+}
+
+int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
+                             uint32_t n, uint64_t* results, eirene_stream_t stream, uint64_t* ticket) {
+  if (!h || !ops || !keys || !vals || !results || !ticket) return EIRENE_EINVAL;
+  if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(cudaSetDevice(h->cfg.device));
+  CK(cudaMemcpyAsync(h->st_ops, ops, n, cudaMemcpyHostToDevice, st));
+  CK(cudaMemcpyAsync(h->st_keys, keys, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, st));
+  CK(cudaMemcpyAsync(h->st_vals, vals, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, st));
+  return submit_impl(h, h->st_ops, h->st_keys, h->st_vals, n, h->st_res, st, results, ticket);
+}
+
+int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) {
+  if (!h) return EIRENE_EINVAL;
+  Rec& r = h->ring[ticket % RING];
+  if (!r.used || r.ticket != ticket) return EIRENE_ESTATE;
+  CK(cudaEventSynchronize(r.done));
+  const BatchCtl& c = h->host_ctl[ticket % RING];
+  if (stats) {
+    std::memset(stats, 0, sizeof(*stats));
+    stats->status = c.status;
+    stats->n = r.n;
+    stats->distinct = c.nseg;
+    stats->issued_q = c.nq;
+    stats->issued_w = c.nw;
+    stats->leaf_runs = c.leaf_runs;
+    stats->retries = c.retries;
+    stats->stm_fallbacks = c.stm_fallbacks;
+    stats->leaf_splits = c.leaf_splits;
+    stats->inner_splits = c.inner_splits;
+    stats->new_leaves = c.new_leaves;
+    stats->new_inner = c.new_inner;
+    stats->height = c.height;
+    stats->launches = (uint32_t)r.launches;
+    if (r.timing) {
+      for (int s = 0; s + 1 < NSTAGE; ++s) cudaEventElapsedTime(&stats->stage_ms[s], r.st[s], r.st[s + 1]);
+      cudaEventElapsedTime(&stats->stage_ms[7], r.st[0], r.st[NSTAGE - 1]);
+    }
+  }
+  return c.status;
+}
+
+int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out, uint64_t* vals_out, uint64_t cap,
+                uint64_t* count, eirene_stream_t stream) {
+  if (!h || !count) return EIRENE_EINVAL;
+  if (cap > 0 && !keys_out && !vals_out) return EIRENE_EINVAL;
+  CK(cudaSetDevice(h->cfg.device));
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  TreeHdr hdr;
+  CK(cudaMemcpyAsync(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));
+  int launches = 0;
+  int rc = scan_tree(h->t, hdr.leaf_count, lo, hi, keys_out, vals_out, cap, count, st, &launches);
+  h->launches += launches;
+  if (rc == EIRENE_ECUDA) return cuda_fail(cudaGetLastError(), "eirene_scan");
+  return rc;
+}
+
+int eirene_get_info(eirene_handle h, eirene_tree_info* info) {
+  if (!h || !info) return EIRENE_EINVAL;
+  CK(cudaSetDevice(h->cfg.device));
+  TreeHdr hdr;
+  CK(cudaMemcpy(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost));
+  info->height = (uint32_t)(hdr.root_word >> 32);
+  info->root = (uint32_t)hdr.root_word;
+  info->leaves = hdr.leaf_count;
+  info->inner = hdr.inner_count;
+  info->leaf_cap = h->t.leaf_cap;
+  info->inner_cap = h->t.inner_cap;
+  info->launches = h->launches;
+  info->device_bytes = h->device_bytes;
+  return EIRENE_OK;
+}
+
+// ---------------------------------------------------------------- invariants
+// Host-side structural check of a quiescent tree (debug utility).
+int eirene_check_invariants(eirene_handle h, uint64_t* n_keys) {
+  if (!h) return EIRENE_EINVAL;
+  CK(cudaSetDevice(h->cfg.device));
+  CK(cudaDeviceSynchronize());
+  TreeHdr hdr;
+  CK(cudaMemcpy(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost));
+  const uint32_t L = hdr.leaf_count, I = hdr.inner_count;
+  std::vector<uint64_t> lk((size_t)L * FAN), ik((size_t)I * FAN);
+  std::vector<uint32_t> ic((size_t)I * FAN);
+  std::vector<NodeMeta> lm(L), im(I);
+  CK(cudaMemcpy(lk.data(), h->t.lkeys, lk.size() * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy(lm.data(), h->t.lmeta, lm.size() * sizeof(NodeMeta), cudaMemcpyDeviceToHost));
+  if (I) {
+    CK(cudaMemcpy(ik.data(), h->t.ikeys, ik.size() * 8, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(ic.data(), h->t.ichild, ic.size() * 4, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(im.data(), h->t.imeta, im.size() * sizeof(NodeMeta), cudaMemcpyDeviceToHost));
+  }
+  const uint32_t height = (uint32_t)(hdr.root_word >> 32), root = (uint32_t)hdr.root_word;
+  if (height == 0 || height > MAX_LEVELS) return 10;
+  std::vector<uint32_t> inorder;
+  uint64_t total = 0;
+  // iterative DFS: (node, level, lo, hi)
+  struct Fr { uint32_t node, level; uint64_t lo, hi; };
+  std::vector<Fr> stack{{root, height - 1, h->cfg.key_lo, h->cfg.key_hi}};
+  std::vector<uint8_t> seen_leaf(L, 0);
+  while (!stack.empty()) {
+    Fr f = stack.back();
+    stack.pop_back();
+    if (f.level == 0) {
+      if (f.node >= L) return 11;
+      if (seen_leaf[f.node]++) return 12;
+      const NodeMeta& m = lm[f.node];
+      if (m.version & 1u) return 13;
+      if (m.lo != f.lo || m.hi != f.hi) return 14;
+      uint64_t prev = 0;
+      bool first = true, ended = false;
+      for (int s = 0; s < FAN; ++s) {
+        const uint64_t k = lk[(size_t)f.node * FAN + s];
+        if (k == KEY_MAX) { ended = true; continue; }
+        if (ended) return 15;               // key after padding
+        if (!first && !(prev < k)) return 16;   // strictly increasing
+        if (k < m.lo || k >= m.hi) return 17;   // inside fences
+        prev = k;
+        first = false;
+        ++total;
+      }
+      inorder.push_back(f.node);
+      continue;
+    }
+    if (f.node >= I) return 18;
+    const NodeMeta& m = im[f.node];
+    if (m.version & 1u) return 13;
+    if (m.level != f.level) return 19;
+    if (m.lo != f.lo || m.hi != f.hi) return 14;
+    const uint32_t c = m.count;
+    if (c < 1 || c > FAN) return 20;
+    const uint64_t* K = &ik[(size_t)f.node * FAN];
+    const uint32_t* Cc = &ic[(size_t)f.node * FAN];
+    for (uint32_t i = 0; i + 1 < c; ++i) {
+      if (K[i] == KEY_MAX) return 21;
+      if (i > 0 && !(K[i - 1] < K[i])) return 16;
+      if (K[i] <= f.lo || K[i] >= f.hi) return 17;
+    }
+    for (uint32_t i = c - 1; i < FAN; ++i)
+      if (K[i] != KEY_MAX) return 21;
+    // push children right-to-left so the leftmost is visited first
+    for (int i = (int)c - 1; i >= 0; --i) {
+      const uint64_t clo = i == 0 ? f.lo : K[i - 1];
+      const uint64_t chi = (uint32_t)i + 1 < c ? K[i] : f.hi;
+      stack.push_back({Cc[i], f.level - 1, clo, chi});
+    }
+  }
+  // leaf chain == in-order leaves; every allocated leaf is reachable
+  if (inorder.size() != L) return 22;
+  for (size_t i = 0; i < inorder.size(); ++i) {
+    const uint32_t want = i + 1 < inorder.size() ? inorder[i + 1] : NIL;
+    if (lm[inorder[i]].next != want) return 23;
+  }
+  if (n_keys) *n_keys = total;
+  return 0;
+}
+
+// ---------------------------------------------------------------- routing
+int eirene_route_partition(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
+                           const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
+                           uint32_t* perm, uint32_t* counts, eirene_stream_t stream) {
+  if (!h || P < 1 || P > 64 || !counts) return EIRENE_EINVAL;
+  if (n > h->cfg.max_batch) return EIRENE_EINVAL;
+  if (n > 0 && (!ops || !keys || !vals || !sops || !skeys || !svals || !perm)) return EIRENE_EINVAL;
+  if (P > 1 && !splitters) return EIRENE_EINVAL;
+  CK(cudaSetDevice(h->cfg.device));
+  int launches = 0;
+  launch_route_partition(ops, keys, vals, n, splitters, P, sops, skeys, svals, perm, counts, h->route_lb,
+                         h->route_ctr, ++h->route_epoch, reinterpret_cast<cudaStream_t>(stream), &launches);
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+int eirene_route_unpermute(eirene_handle h, const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,
+                           eirene_stream_t stream) {
+  if (!h) return EIRENE_EINVAL;
+  if (n > 0 && (!recv || !perm || !results)) return EIRENE_EINVAL;
+  CK(cudaSetDevice(h->cfg.device));
+  int launches = 0;
+  launch_route_unpermute(recv, perm, n, results, reinterpret_cast<cudaStream_t>(stream), &launches);
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+}  // extern "C"

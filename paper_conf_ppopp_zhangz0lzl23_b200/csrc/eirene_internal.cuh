@@ -1,0 +1,223 @@
+// eirene_internal.cuh -- device layout and helpers shared by the sm_100a kernels
+// of the Eirene batched B+tree (never included by oracle/).
+//
+// Citations: P:N = /root/reference/PAPER.md line N; Alg.1:k = Algorithm 1 line k.
+//
+// Tree layout in HBM (SoA node pools):
+//   leaves : lkeys[cap][16] u64 (one 128 B line), lvals[cap][16] u64 (128 B),
+//            lmeta[cap] (32 B).  Unused key slots hold KEY_MAX (sorted to the end).
+//   inner  : ikeys[cap][16] u64 separators (child i covers [key[i-1], key[i]),
+//            key[c-1..15] = KEY_MAX), ichild[cap][16] u32, imeta[cap] (32 B).
+//   The B+tree of P:327-330 / P:1622-1628, plus B-link right links and [lo, hi)
+//   fences on every node (P:1363-1366 leaf links; "key in range(leaf)",
+//   Alg.1:38) and a version word per node.
+#pragma once
+#include <algorithm>
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "eirene.h"
+
+namespace eirene {
+
+constexpr int FAN = 16;
+constexpr uint64_t KEY_MAX = ~0ull;
+constexpr uint32_t NIL = 0xFFFFFFFFu;
+constexpr int MAX_LEVELS = 32;
+constexpr uint32_t DONE_BIT = 0x80000000u;
+constexpr uint32_t FULL = 0xFFFFFFFFu;
+
+enum { OP_QUERY = 0, OP_UPDATE = 1, OP_INSERT = 2, OP_DELETE = 3 };
+
+// Version word (D2, SURVEY §8(c) reading 18): bit 0 = lock (eager write
+// ownership of the STM), bits 1.. = modification counter.
+// Leaves: +2 on split only; inner nodes: +2 on every change.
+struct NodeMeta {
+  uint32_t version;
+  uint32_t next;    // right sibling at the same level (B-link / leaf chain)
+  uint64_t lo;      // fences: every key k below this node has lo <= k < hi
+  uint64_t hi;
+  uint32_t count;   // inner: number of children; leaf: informational
+  uint32_t level;   // 0 = leaf
+};
+static_assert(sizeof(NodeMeta) == 32, "meta is 32 B");
+
+struct TreeHdr {
+  unsigned long long root_word;          // (height << 32) | root id; height 1 = leaf root
+  uint32_t leaf_count, inner_count;      // pool allocation counters
+  uint32_t level_count[MAX_LEVELS];      // nodes per level (EFULL bound)
+};
+
+// Per-batch device scalars; zeroed (cudaMemsetAsync) before every batch.
+struct BatchCtl {
+  int32_t status;
+  uint32_t invalid;
+  uint32_t tile_ctr[16];
+  uint32_t nseg, nq, nw, height;
+  unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
+  uint32_t dbg[8];   // watchdog diagnostics
+};
+
+// Device watchdog: spin / retry loops give up after this long and report
+// EIRENE_EINTERNAL instead of hanging the GPU.
+constexpr unsigned long long WATCHDOG_NS = 4000000000ull;
+__device__ __forceinline__ unsigned long long gtime_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// Decoupled look-back spin guard: a predecessor tile that never publishes is a
+// bug; give up after the watchdog period instead of hanging.
+struct SpinGuard {
+  unsigned long long t0 = 0;
+  __device__ __forceinline__ bool stuck(BatchCtl* ctl) {
+    const unsigned long long now = gtime_ns();
+    if (t0 == 0) {
+      t0 = now;
+      return false;
+    }
+    if (now - t0 > WATCHDOG_NS) {
+      if (ctl) atomicExch(reinterpret_cast<int*>(&ctl->status), EIRENE_EINTERNAL);
+      return true;
+    }
+    return false;
+  }
+};
+
+// tile counters
+enum { TC_SORT0 = 0, TC_COMB = 8, TC_PART = 9, TC_ROUTE = 10, TC_SCAN = 11 };
+
+struct Tree {
+  uint64_t* lkeys;
+  uint64_t* lvals;
+  NodeMeta* lmeta;
+  uint64_t* ikeys;
+  uint32_t* ichild;
+  NodeMeta* imeta;
+  TreeHdr* hdr;
+  uint32_t leaf_cap, inner_cap;
+};
+
+// ------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t lanemask_lt() {
+  uint32_t m;
+  asm volatile("mov.u32 %0, %%lanemask_lt;" : "=r"(m));
+  return m;
+}
+__device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31; }
+
+// L2-coherent loads for data concurrently written by other SMs (the update kernel).
+__device__ __forceinline__ uint64_t ld_cg(const uint64_t* p) {
+  return __ldcg(reinterpret_cast<const unsigned long long*>(p));
+}
+__device__ __forceinline__ uint32_t ld_cg(const uint32_t* p) { return __ldcg(p); }
+__device__ __forceinline__ uint32_t ld_acquire(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ unsigned long long ld_acquire64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
+  asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
+}
+__device__ __forceinline__ unsigned long long ld_relaxed64(const unsigned long long* p) {
+  unsigned long long v;
+  asm volatile("ld.relaxed.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_relaxed64(unsigned long long* p, unsigned long long v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+
+__device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
+  return __shfl_sync(FULL, (unsigned long long)v, src);
+}
+
+__host__ __device__ __forceinline__ bool is_write(uint32_t op) { return op != OP_QUERY; }
+
+// ------------------------------------------------------------ host-side launchers
+// (defined in the .cu files; called from api.cu)
+struct SortBufs {
+  uint64_t* kA;
+  uint32_t* pA;
+  uint64_t* kB;
+  uint32_t* pB;
+  unsigned long long* lookback;   // [tiles * 256]
+  uint32_t* ghist;                // [8 * 256]
+};
+constexpr int SORT_THREADS = 256;
+constexpr int SORT_ITEMS = 16;
+constexpr int SORT_TILE = SORT_THREADS * SORT_ITEMS;
+constexpr int SORT_PASSES = 8;
+
+// Sort (key, payload) pairs by key, stable.  If ops != nullptr the payload of
+// element i is (i << 2) | ops[i] (logical timestamp + type),
+// otherwise pay_in[i].  Returns (via *kout/*pout) which buffer holds the result.
+// Also validates requests when ops != nullptr (sets ctl->invalid).
+void launch_sort(const uint64_t* keys, const uint8_t* ops, const uint32_t* pay_in, const uint64_t* vals,
+                 uint32_t n, uint64_t key_lo, uint64_t key_hi, const SortBufs& b, BatchCtl* ctl,
+                 uint32_t epoch_base, cudaStream_t st, int* launches, uint64_t** kout, uint32_t** pout);
+
+size_t sort_lookback_words(uint32_t max_n);
+
+struct CombBufs {
+  uint32_t* pinfo;            // [n] seg | DONE
+  uint64_t* ikey;             // [n] issued key per segment
+  uint8_t* iop;               // [n]
+  uint64_t* ival;             // [n]
+  unsigned long long* comb_status;  // [tiles]  (zeroed per batch)
+  unsigned long long* part_status;  // [tiles]  (zeroed per batch)
+  uint64_t* qkey;
+  uint32_t* qseg;
+  uint64_t* wkey;
+  uint8_t* wop;
+  uint64_t* wval;
+  uint32_t* wseg;
+  uint32_t* wleaf;
+  uint64_t* old;              // [n] old value per segment
+};
+constexpr int COMB_THREADS = 256;
+constexpr int COMB_ITEMS = 8;
+constexpr int COMB_TILE = COMB_THREADS * COMB_ITEMS;
+
+void launch_combine(const uint64_t* skey, const uint32_t* spay, const uint64_t* vals, uint64_t* results,
+                    uint32_t n, const CombBufs& c, BatchCtl* ctl, cudaStream_t st, int* launches);
+void launch_partition(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, cudaStream_t st, int* launches);
+void launch_query(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, int num_sms, cudaStream_t st,
+                  int* launches);
+
+struct UpdParams {
+  uint32_t threshold;
+  uint32_t flags;
+  uint64_t* entA_key;
+  uint32_t* entA_child;
+  uint64_t* entB_key;
+  uint32_t* entB_child;
+};
+void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms,
+                   cudaStream_t st, int* launches);
+void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, uint64_t* results, BatchCtl* ctl,
+                   cudaStream_t st, int* launches);
+
+// bulk build / scan
+int build_tree(Tree t, const uint64_t* keys, const uint64_t* vals, uint64_t n, int per_leaf, uint64_t key_lo,
+               uint64_t key_hi, cudaStream_t st, int* launches, uint32_t* height_out);
+void launch_validate_bulk(const uint64_t* keys, const uint64_t* vals, uint64_t n, uint64_t key_lo, uint64_t key_hi,
+                          uint32_t* flag, cudaStream_t st, int* launches);
+int scan_tree(Tree t, uint32_t leaf_count, uint64_t lo, uint64_t hi, uint64_t* keys_out, uint64_t* vals_out,
+              uint64_t cap, uint64_t* count, cudaStream_t st, int* launches);
+
+// routing
+void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
+                            const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
+                            uint32_t* perm, uint32_t* counts, unsigned long long* lookback, uint32_t* tile_ctr,
+                            uint32_t epoch, cudaStream_t st, int* launches);
+void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,
+                            cudaStream_t st, int* launches);
+
+}  // namespace eirene

@@ -1,0 +1,84 @@
+// query.cu -- QUERY_KERNEL (Alg.1:15-21) and leaf locate for the issued writes.
+//
+// Issued queries run with no concurrency control: the tree is
+// quiescent (the update kernel of the previous batch has finished, and this
+// batch's update kernel runs after this one).  Each thread owns
+// one issued request; the issued list is key-sorted, so the 32 lanes of a warp
+// walk overlapping root-to-leaf paths and their 128-bit loads of shared upper
+// nodes coalesce into one L1/L2 request per distinct node (the B200 analogue
+// of Harmonia's path sharing / NTG).  Inner levels (<= 18 MB at
+// 2^24 keys) stay L2-resident across batches; leaves (256 MiB) come from HBM:
+// one 128 B key line plus one 32 B value sector per issued query.
+//
+// The same traversal gives each issued write its target leaf (a4, the input
+// of the leaf-run regrouping in the update kernel).
+#include "eirene_internal.cuh"
+
+namespace eirene {
+
+namespace {
+
+// Count of separators <= k in a 16-key node line (key[c-1..15] == KEY_MAX,
+// and k < KEY_MAX, so the count is the child index).
+__device__ __forceinline__ uint32_t route16(const uint64_t* __restrict__ line, uint64_t k) {
+  const ulonglong2* l2 = reinterpret_cast<const ulonglong2*>(line);
+  ulonglong2 v[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) v[i] = __ldg(l2 + i);
+  uint32_t c = 0;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) c += (v[i].x <= k) + (v[i].y <= k);
+  return c;
+}
+
+__device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_t k) {
+  const ulonglong2* l2 = reinterpret_cast<const ulonglong2*>(line);
+  ulonglong2 v[8];
+#pragma unroll
+  for (int i = 0; i < 8; ++i) v[i] = __ldg(l2 + i);
+  int s = -1;
+#pragma unroll
+  for (int i = 0; i < 8; ++i) {
+    if (v[i].x == k) s = 2 * i;
+    if (v[i].y == k) s = 2 * i + 1;
+  }
+  return s;
+}
+
+__global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__ qkey,
+                                                     const uint32_t* __restrict__ qseg,
+                                                     const uint64_t* __restrict__ wkey, uint32_t* __restrict__ wleaf,
+                                                     uint64_t* __restrict__ old, Tree t,
+                                                     const BatchCtl* __restrict__ ctl) {
+  if (ctl->invalid || ctl->status != 0) return;
+  const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
+  const unsigned long long rw = t.hdr->root_word;
+  const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += stride) {
+    const bool isq = i < nq;
+    const uint64_t k = isq ? qkey[i] : wkey[i - nq];
+    uint32_t node = root;
+    for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
+      const uint32_t c = route16(t.ikeys + (size_t)node * FAN, k);
+      node = __ldg(t.ichild + (size_t)node * FAN + c);
+    }
+    if (isq) {
+      const int s = slot16(t.lkeys + (size_t)node * FAN, k);
+      old[qseg[i]] = s >= 0 ? __ldg(t.lvals + (size_t)node * FAN + s) : KEY_MAX;
+    } else {
+      wleaf[i - nq] = node;
+    }
+  }
+}
+
+}  // namespace
+
+void launch_query(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
+  int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
+  if (blocks < 1) blocks = 1;
+  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wleaf, c.old, t, ctl);
+  ++*launches;
+}
+
+}  // namespace eirene

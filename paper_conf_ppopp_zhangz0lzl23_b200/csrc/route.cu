@@ -1,0 +1,202 @@
+// route.cu -- key-range routing for the multi-GPU mode.
+//
+// Each rank owns the contiguous timestamp slice r of the global batch; a request
+// goes to shard dest(k) = #{splitters <= k}.  The stable partition keeps each
+// destination's requests in timestamp order, so after the all-to-all (NCCL,
+// issued by the caller) the receiver's concatenation in source-rank order is
+// timestamp-ordered and the per-shard stable sort preserves linearizability
+// (§8(c) reading 7; per-key locality of linearizability, P:2487-2492 / [17]).
+// Same single-pass-per-digit design as sort.cu with <= 64 destinations.
+#include "eirene_internal.cuh"
+
+namespace eirene {
+
+namespace {
+
+constexpr int RT_THREADS = 256;
+constexpr int RT_ITEMS = 8;
+constexpr int RT_TILE = RT_THREADS * RT_ITEMS;
+constexpr int RT_MAXP = 64;
+constexpr int RT_WARPS = RT_THREADS / 32;
+constexpr unsigned long long LB_AGG = 1ull << 30;
+constexpr unsigned long long LB_INC = 2ull << 30;
+constexpr unsigned long long LB_VAL = (1ull << 30) - 1;
+
+__device__ __forceinline__ uint32_t dest_of(uint64_t k, const uint64_t* sp, int P) {
+  uint32_t d = 0;
+  for (int i = 0; i < P - 1; ++i) d += (sp[i] <= k) ? 1u : 0u;
+  return d;
+}
+
+__global__ void __launch_bounds__(RT_THREADS) route_count_kernel(const uint64_t* __restrict__ keys, uint32_t n,
+                                                                 const uint64_t* __restrict__ splitters, int P,
+                                                                 uint32_t* __restrict__ counts) {
+  __shared__ uint64_t sp[RT_MAXP];
+  __shared__ uint32_t h[RT_MAXP];
+  const int tid = threadIdx.x;
+  if (tid < RT_MAXP) {
+    sp[tid] = tid < P - 1 ? splitters[tid] : KEY_MAX;
+    h[tid] = 0;
+  }
+  __syncthreads();
+  for (uint32_t i = blockIdx.x * RT_THREADS + tid; i < n; i += gridDim.x * RT_THREADS) {
+    atomicAdd(&h[dest_of(keys[i], sp, P)], 1u);
+  }
+  __syncthreads();
+  if (tid < P && h[tid]) atomicAdd(&counts[tid], h[tid]);
+}
+
+struct RtSmem {
+  uint64_t keys[RT_TILE];
+  uint64_t vals[RT_TILE];
+  uint32_t idx[RT_TILE];
+  uint8_t ops[RT_TILE];
+  uint64_t sp[RT_MAXP];
+  uint32_t wh[RT_WARPS][RT_MAXP];
+  uint32_t tile_off[RT_MAXP];
+  uint32_t cnt[RT_MAXP];
+  uint32_t bin_base[RT_MAXP];
+  uint32_t bin_start[RT_MAXP];
+  uint32_t tile_id;
+};
+
+__global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
+    const uint8_t* __restrict__ ops, const uint64_t* __restrict__ keys, const uint64_t* __restrict__ vals, uint32_t n,
+    const uint64_t* __restrict__ splitters, int P, const uint32_t* __restrict__ counts, uint8_t* __restrict__ sops,
+    uint64_t* __restrict__ skeys, uint64_t* __restrict__ svals, uint32_t* __restrict__ perm,
+    unsigned long long* __restrict__ lookback, uint32_t epoch, uint32_t* __restrict__ tile_ctr) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  RtSmem& S = *reinterpret_cast<RtSmem*>(smem_raw);
+  const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+  if (tid == 0) {
+    S.tile_id = atomicAdd(tile_ctr, 1u);
+    uint32_t run = 0;
+    for (int d = 0; d < P; ++d) {
+      S.bin_start[d] = run;
+      run += counts[d];
+    }
+  }
+  for (int i = tid; i < RT_WARPS * RT_MAXP; i += RT_THREADS) (&S.wh[0][0])[i] = 0;
+  if (tid < RT_MAXP) S.sp[tid] = tid < P - 1 ? splitters[tid] : KEY_MAX;
+  __syncthreads();
+  const uint32_t tile = S.tile_id, base = tile * RT_TILE;
+  const uint32_t wbase = base + warp * (RT_ITEMS * 32);
+  uint64_t k[RT_ITEMS];
+  uint32_t d[RT_ITEMS], r[RT_ITEMS];
+#pragma unroll
+  for (int j = 0; j < RT_ITEMS; ++j) {
+    const uint32_t i = wbase + j * 32 + lane;
+    const bool act = i < n;
+    k[j] = act ? keys[i] : 0;
+    d[j] = act ? dest_of(k[j], S.sp, P) : RT_MAXP;
+    const uint32_t peers = __match_any_sync(FULL, d[j]);
+    const uint32_t before = act ? S.wh[warp][d[j]] : 0;
+    r[j] = before + __popc(peers & lanemask_lt());
+    __syncwarp();
+    if (act && lane == 31 - __clz(peers)) S.wh[warp][d[j]] = before + __popc(peers);
+    __syncwarp();
+  }
+  __syncthreads();
+  if (tid < RT_MAXP) {
+    uint32_t run = 0;
+    for (int w = 0; w < RT_WARPS; ++w) {
+      const uint32_t c = S.wh[w][tid];
+      S.wh[w][tid] = run;
+      run += c;
+    }
+    S.cnt[tid] = run;
+  }
+  __syncthreads();
+  if (tid == 0) {
+    uint32_t run = 0;
+    for (int dd = 0; dd < RT_MAXP; ++dd) {
+      S.tile_off[dd] = run;
+      run += S.cnt[dd];
+    }
+  }
+  __syncthreads();
+  if (tid < P) {
+    const uint32_t cnt_ok = S.cnt[tid];
+    unsigned long long* my = lookback + (size_t)tile * RT_MAXP + tid;
+    const unsigned long long ep = (unsigned long long)epoch << 32;
+    uint32_t excl = 0;
+    if (tile == 0) {
+      st_relaxed64(my, ep | LB_INC | cnt_ok);
+    } else {
+      st_relaxed64(my, ep | LB_AGG | cnt_ok);
+      SpinGuard sg;
+      int32_t pt = (int32_t)tile - 1;
+      while (pt >= 0) {
+        const unsigned long long w = ld_relaxed64(lookback + (size_t)pt * RT_MAXP + tid);
+        if ((w >> 32) != epoch || (w & (3ull << 30)) == 0) {
+          if (sg.stuck(nullptr)) break;
+          continue;
+        }
+        excl += (uint32_t)(w & LB_VAL);
+        if (w & LB_INC) break;
+        --pt;
+      }
+      st_relaxed64(my, ep | LB_INC | (excl + cnt_ok));
+    }
+    S.bin_base[tid] = S.bin_start[tid] + excl - S.tile_off[tid];
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < RT_ITEMS; ++j) {
+    const uint32_t i = wbase + j * 32 + lane;
+    if (i < n) {
+      const uint32_t pos = S.tile_off[d[j]] + S.wh[warp][d[j]] + r[j];
+      S.keys[pos] = k[j];
+      S.vals[pos] = vals[i];
+      S.ops[pos] = ops[i];
+      S.idx[pos] = i;
+    }
+  }
+  __syncthreads();
+  const uint32_t tile_n = min((uint32_t)RT_TILE, n - base);
+  for (uint32_t i = tid; i < tile_n; i += RT_THREADS) {
+    const uint64_t key = S.keys[i];
+    const uint32_t o = S.bin_base[dest_of(key, S.sp, P)] + i;
+    skeys[o] = key;
+    svals[o] = S.vals[i];
+    sops[o] = S.ops[i];
+    perm[o] = S.idx[i];
+  }
+}
+
+__global__ void unpermute_kernel(const uint64_t* __restrict__ recv, const uint32_t* __restrict__ perm, uint32_t n,
+                                 uint64_t* __restrict__ out) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) out[perm[j]] = recv[j];
+}
+
+}  // namespace
+
+void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
+                            const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
+                            uint32_t* perm, uint32_t* counts, unsigned long long* lookback, uint32_t* tile_ctr,
+                            uint32_t epoch, cudaStream_t st, int* launches) {
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(route_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(RtSmem));
+    attr = true;
+  }
+  cudaMemsetAsync(counts, 0, sizeof(uint32_t) * P, st);
+  cudaMemsetAsync(tile_ctr, 0, sizeof(uint32_t), st);
+  if (n == 0) return;
+  int blocks = (int)std::min<uint32_t>((n + RT_THREADS * 8 - 1) / (RT_THREADS * 8), 148u * 4u);
+  route_count_kernel<<<blocks, RT_THREADS, 0, st>>>(keys, n, splitters, P, counts);
+  const uint32_t tiles = (n + RT_TILE - 1) / RT_TILE;
+  route_scatter_kernel<<<tiles, RT_THREADS, sizeof(RtSmem), st>>>(ops, keys, vals, n, splitters, P, counts, sops,
+                                                                  skeys, svals, perm, lookback, epoch, tile_ctr);
+  *launches += 2;
+}
+
+void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,
+                            cudaStream_t st, int* launches) {
+  if (n == 0) return;
+  int blocks = (int)std::min<uint32_t>((n + 255) / 256, 148u * 8u);
+  unpermute_kernel<<<blocks, 256, 0, st>>>(recv, perm, n, results);
+  ++*launches;
+}
+
+}  // namespace eirene

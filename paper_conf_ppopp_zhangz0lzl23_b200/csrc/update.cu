@@ -1,0 +1,726 @@
+// update.cu -- UPDATE_KERNEL (Alg.1:23-46) with leaf-bucketed warp regrouping
+// (P:1334-1416), optimistic traversal, version validation and an
+// eager-conflict-detection STM fallback past THRESHOLD (Alg.1:28-33).
+//
+// Work unit (regrouping, a4): the issued writes are key-sorted and carry the
+// leaf the query-kernel traversal located (an unprotected findLeaf, Alg.1:29).
+// Equal leaf ids are contiguous, so each warp takes whole LEAF RUNS: a run is
+// merged into its leaf by one warp in one transaction, and no two warps ever
+// target the same leaf (the B200 form of the paper's iteration warps: the
+// locality is exploited by construction instead of by a horizontal walk).
+// With EIRENE_F_REGROUP off every issued write is its own run (one warp per
+// request, as in Alg.1:24), and leaf conflicts + retries appear.
+//
+// Per run (Alg.1:27-45):
+//   RETRY: leaf = hint (first try) | findLeaf optimistic (retry < THRESHOLD)
+//                                 | TX{findLeaf} with a read log (otherwise)
+//          leafvers = leaf.version                                  (Alg.1:35)
+//          TX_BEGIN: eager write ownership = CAS(version, v, v|1)    (Alg.1:37)
+//          if key in [leaf.lo, leaf.hi): merge the run (upsert/erase), split
+//            into ceil(t/16) leaves if it overflows, version += 2 on split
+//          else abort: retry_count++, goto RETRY                     (Alg.1:40-43)
+// Structure changes propagate upward (B-link tree: every node has a right link
+// and [lo, hi) fences, so a warp holds at most one lock at a time and never
+// waits while holding one -> no deadlock).  Inserting separators into a parent
+// repeats the same optimistic / STM protocol at the parent level; a root split
+// installs the new root while the old root is still owned.
+#include <cstdio>
+#include <cstdlib>
+
+#include "eirene_internal.cuh"
+
+namespace eirene {
+
+namespace {
+
+struct Ctx {
+  Tree t;
+  const uint64_t* wkey;
+  const uint8_t* wop;
+  const uint64_t* wval;
+  const uint32_t* wseg;
+  const uint32_t* wleaf;
+  uint64_t* old;
+  uint64_t* eK[2];    // entry ping-pong buffers: separators to insert at the next level
+  uint32_t* eC[2];
+  uint32_t threshold;
+  bool force_stm;
+  bool regroup;
+  bool stats;
+  BatchCtl* ctl;
+};
+
+struct WarpStats {
+  unsigned long long runs = 0, retries = 0, stm = 0, leaf_splits = 0, inner_splits = 0, new_leaves = 0,
+                     new_inner = 0;
+  unsigned long long t0 = 0;
+  bool dead = false;
+};
+
+// Watchdog (see eirene_internal.cuh): true if this warp must give up.
+__device__ bool watchdog(const Ctx& C, WarpStats& ws, uint32_t where, uint32_t a, uint32_t b, uint32_t c,
+                         uint32_t d) {
+  if (ws.dead) return true;
+  if (*(volatile int32_t*)&C.ctl->status == EIRENE_EINTERNAL || gtime_ns() - ws.t0 > WATCHDOG_NS) {
+    ws.dead = true;
+    if ((threadIdx.x & 31) == 0 && atomicCAS(reinterpret_cast<int*>(&C.ctl->status), 0, EIRENE_EINTERNAL) == 0) {
+      C.ctl->dbg[0] = where;
+      C.ctl->dbg[1] = a;
+      C.ctl->dbg[2] = b;
+      C.ctl->dbg[3] = c;
+      C.ctl->dbg[4] = d;
+      C.ctl->dbg[5] = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+      printf("eirene watchdog: where=%u a=%u b=%u c=%u d=%u warp=%u\n", where, a, b, c, d, C.ctl->dbg[5]);
+    }
+    return true;
+  }
+  return false;
+}
+
+constexpr uint32_t LEAF_TAG = 0x80000000u;
+
+__device__ __forceinline__ void backoff(uint32_t retry) {
+  uint32_t ns = 32u << (retry < 8 ? retry : 8);
+  __nanosleep(ns);
+}
+
+__device__ __forceinline__ uint32_t shfl32(uint32_t v, int src) { return __shfl_sync(FULL, v, src); }
+
+__device__ __forceinline__ NodeMeta* meta_of(const Tree& t, uint32_t node, bool leaf) {
+  return leaf ? t.lmeta + node : t.imeta + node;
+}
+
+// Warp-collective lock acquisition: TX_BEGIN with eager conflict detection.
+// Returns true and the pre-lock version in *v if the node was free.
+__device__ __forceinline__ bool try_lock(uint32_t* vp, uint32_t* v_out) {
+  uint32_t v = 0, ok = 0;
+  if (lane_id() == 0) {
+    v = ld_acquire(vp);
+    ok = (!(v & 1u) && atomicCAS(vp, v, v | 1u) == v) ? 1u : 0u;
+  }
+  ok = shfl32(ok, 0);
+  v = shfl32(v, 0);
+  __threadfence();
+  *v_out = v;
+  return ok != 0;
+}
+
+__device__ __forceinline__ void unlock(uint32_t* vp, uint32_t newv) {
+  __threadfence();
+  __syncwarp();
+  if (lane_id() == 0) st_release(vp, newv);
+  __syncwarp();
+}
+
+// findLeaf / find-node-at-level (warp-collective, uniform arguments).
+// Optimistic mode reads without any protection (Alg.1:29).  STM mode (Alg.1:31-33)
+// is a read-only transaction: every node read records (node, version) in a
+// per-lane read log, aborts eagerly on a node owned by a writer (odd version)
+// or a version change during the read, and validates the whole log at TX_END.
+// B-link move-right (k >= hi -> follow next) keeps descents correct across
+// concurrent splits whose separators are not yet in the parent.
+__device__ uint32_t descend(const Ctx& C, uint64_t k, uint32_t target, bool stm) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  const unsigned long long rw = ld_acquire64(&t.hdr->root_word);
+  const uint32_t height = (uint32_t)(rw >> 32);
+  uint32_t node = (uint32_t)rw;
+  if (height == 0 || target + 1 > height) return NIL;
+  uint32_t lvl = height - 1;
+  uint32_t log_node = NIL, log_ver = 0;
+  int nlog = 0;
+  for (int steps = 0; steps < 1024; ++steps) {
+    const bool leaf = (lvl == 0);
+    if (node >= (leaf ? t.leaf_cap : t.inner_cap)) return NIL;
+    NodeMeta* m = meta_of(t, node, leaf);
+    uint32_t v1 = 0;
+    if (stm) {
+      v1 = ld_acquire(&m->version);
+      if (v1 & 1u) return NIL;   // eager conflict: the node is owned by a writer
+    }
+    const uint64_t hi = ld_cg(&m->hi);
+    const uint32_t nxt = ld_cg(&m->next);
+    const bool right = (k >= hi) && nxt != NIL;
+    uint32_t child = NIL;
+    if (!right && lvl > target) {
+      const size_t nb = (size_t)node * FAN;
+      const uint64_t key = lane < FAN ? ld_cg(t.ikeys + nb + lane) : KEY_MAX;
+      const uint32_t ch = lane < FAN ? ld_cg(t.ichild + nb + lane) : NIL;
+      const uint32_t idx = __popc(__ballot_sync(FULL, lane < FAN - 1 && key <= k));
+      child = shfl32(ch, idx);
+    }
+    if (stm) {
+      __threadfence();
+      const uint32_t v2 = ld_acquire(&m->version);
+      if (v2 != v1 || nlog >= 32) return NIL;
+      if (lane == nlog) {
+        log_node = node | (leaf ? LEAF_TAG : 0u);
+        log_ver = v1;
+      }
+      ++nlog;
+    }
+    if (right) {
+      node = nxt;
+      continue;
+    }
+    if (lvl == target) {
+      if (stm) {   // TX_END of the traversal: validate the read set
+        bool okl = true;
+        if (lane < nlog) {
+          const bool lf = (log_node & LEAF_TAG) != 0;
+          okl = ld_acquire(&meta_of(t, log_node & ~LEAF_TAG, lf)->version) == log_ver;
+        }
+        if (!__all_sync(FULL, okl)) return NIL;
+      }
+      return node;
+    }
+    if (child == NIL) return NIL;
+    node = child;
+    --lvl;
+  }
+  return NIL;
+}
+
+__device__ __forceinline__ bool is_root(const Tree& t, uint32_t node, uint32_t level) {
+  const unsigned long long rw = ld_acquire64(&t.hdr->root_word);
+  return (uint32_t)rw == node && (uint32_t)(rw >> 32) == level + 1;
+}
+
+__device__ __forceinline__ uint32_t warp_alloc(uint32_t* ctr, uint32_t n) {
+  uint32_t f = 0;
+  if (lane_id() == 0) f = atomicAdd(ctr, n);
+  return shfl32(f, 0);
+}
+
+// New root level(s) above a list of nodes at level L: element 0 is (id0, lo0),
+// elements 1..m are the entries (K, Ch)[eb ..].  Called while the old root is
+// still owned, so the root word cannot change underneath (P:1196-1202 regions).
+__device__ void build_root(const Ctx& C, uint32_t L, uint32_t id0, uint64_t lo0, uint64_t hi_all, uint64_t* K,
+                           uint32_t* Ch, uint64_t* K2, uint32_t* Ch2, uint32_t eb, uint32_t m, WarpStats& ws) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  uint32_t cnt = m + 1;
+  for (;;) {
+    const uint32_t nn = (cnt + FAN - 1) / FAN;
+    const uint32_t first = warp_alloc(&t.hdr->inner_count, nn);
+    if (lane == 0) atomicAdd(&t.hdr->level_count[L + 1], nn);
+    const uint32_t bs = cnt / nn, rem = cnt % nn;
+    for (uint32_t q0 = 0; q0 < nn; q0 += 2) {
+      const uint32_t q = q0 + (lane >> 4), i = lane & 15;
+      if (q < nn) {
+        const uint32_t size = bs + (q < rem ? 1u : 0u);
+        const uint32_t start = q * bs + min(q, rem);
+        const uint32_t g = start + i;
+        const uint32_t id = first + q;
+        const uint32_t child = i < size ? (g == 0 ? id0 : ld_cg(Ch + eb + g - 1)) : NIL;
+        const uint64_t key = (i + 1 < size) ? ld_cg(K + eb + g) : KEY_MAX;
+        t.ichild[(size_t)id * FAN + i] = child;
+        t.ikeys[(size_t)id * FAN + i] = key;
+        if (i == 0) {
+          NodeMeta mt;
+          mt.version = 0;
+          mt.lo = g == 0 ? lo0 : ld_cg(K + eb + g - 1);
+          const uint32_t nstart = (q + 1) * bs + min(q + 1, rem);
+          mt.hi = (q + 1 < nn) ? ld_cg(K + eb + nstart - 1) : hi_all;
+          mt.next = (q + 1 < nn) ? id + 1 : NIL;
+          mt.count = size;
+          mt.level = L + 1;
+          t.imeta[id] = mt;
+          if (q >= 1) {
+            K2[eb + q - 1] = mt.lo;
+            Ch2[eb + q - 1] = id;
+          }
+        }
+      }
+    }
+    __threadfence();
+    __syncwarp();
+    ws.new_inner += nn;
+    if (nn == 1) {
+      if (lane == 0) atomicExch(&t.hdr->root_word, ((unsigned long long)(L + 2) << 32) | first);
+      __threadfence();
+      __syncwarp();
+      return;
+    }
+    id0 = first;
+    cnt = nn;
+    ++L;
+    uint64_t* tk = K; K = K2; K2 = tk;
+    uint32_t* tc = Ch; Ch = Ch2; Ch2 = tc;
+  }
+}
+
+// Merge writes [b, e) (key-sorted, all inside the locked leaf X's fences) into
+// X.  Every write returns the value X held for its key (old[seg]), NOT_FOUND if
+// absent.  Result t keys; t <= 16 stays in X, else an even multi-way split into
+// k = ceil(t/16) leaves (X + k-1 fresh), entries (first key, leaf) for the
+// parent written to (Ek, Ec)[b .. b+k-2].  Returns k.
+__device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e, uint64_t X_hi, uint32_t X_next,
+                               uint64_t* Ek, uint32_t* Ec, WarpStats& ws) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  const size_t xb = (size_t)X * FAN;
+  const uint64_t okey = lane < FAN ? ld_cg(t.lkeys + xb + lane) : KEY_MAX;
+  const uint64_t oval = lane < FAN ? ld_cg(t.lvals + xb + lane) : 0;
+  const uint32_t c = __popc(__ballot_sync(FULL, okey != KEY_MAX));
+
+  uint32_t mmask = 0, U = 0, ups_before = 0;
+  bool inplace = true;
+  for (uint32_t base = b; base < e; base += 32) {
+    const uint32_t j = base + lane;
+    const bool act = j < e;
+    const uint64_t wk = act ? C.wkey[j] : KEY_MAX;
+    const uint32_t wo = act ? C.wop[j] : 0;
+    uint32_t lo = 0;
+#pragma unroll
+    for (int i = 0; i < FAN; ++i) lo += shfl64(okey, i) < wk ? 1u : 0u;
+    const uint64_t at = shfl64(okey, lo);
+    const uint64_t ov = shfl64(oval, lo);
+    const bool match = act && lo < c && at == wk;
+    if (act) C.old[C.wseg[j]] = match ? ov : KEY_MAX;   // the issued write retrieves the old value
+    const bool ups = act && wo != OP_DELETE;
+    mmask |= __reduce_or_sync(FULL, match ? (1u << lo) : 0u);
+    const uint32_t um = __ballot_sync(FULL, ups);
+    U += __popc(um);
+    if (__any_sync(FULL, act && !(match && ups))) inplace = false;
+    if (c > 0 && um) {
+      for (uint32_t i = 0; i < c; ++i) {
+        const uint64_t oi = shfl64(okey, i);
+        const uint32_t bm = __ballot_sync(FULL, ups && wk < oi);
+        if (lane == (int)i) ups_before += __popc(bm);
+      }
+    }
+  }
+  if (inplace) {   // only value overwrites of present keys: no structural change
+    for (uint32_t base = b; base < e; base += 32) {
+      const uint32_t j = base + lane;
+      const bool act = j < e;
+      const uint64_t wk = act ? C.wkey[j] : KEY_MAX;
+      uint32_t lo = 0;
+#pragma unroll
+      for (int i = 0; i < FAN; ++i) lo += shfl64(okey, i) < wk ? 1u : 0u;
+      if (act) t.lvals[xb + lo] = C.wval[j];
+    }
+    __threadfence();
+    __syncwarp();
+    return 1;
+  }
+  const uint32_t tout = c - __popc(mmask) + U;
+  const uint32_t k = tout <= FAN ? 1u : (tout + FAN - 1) / FAN;
+  const uint32_t first = k > 1 ? warp_alloc(&t.hdr->leaf_count, k - 1) : 0u;
+  if (k > 1 && lane == 0) atomicAdd(&t.hdr->level_count[0], k - 1);
+  const uint32_t bs = tout / k, rem = tout % k, big = rem * (bs + 1);
+  auto place = [&](uint32_t f, uint64_t key, uint64_t val) {
+    uint32_t q, start;
+    if (f < big) {
+      q = f / (bs + 1);
+      start = q * (bs + 1);
+    } else {
+      q = rem + (f - big) / bs;
+      start = big + (q - rem) * bs;
+    }
+    const uint32_t slot = f - start;
+    const uint32_t id = q == 0 ? X : first + q - 1;
+    t.lkeys[(size_t)id * FAN + slot] = key;
+    t.lvals[(size_t)id * FAN + slot] = val;
+    if (q > 0 && slot == 0) {
+      Ek[b + q - 1] = key;
+      Ec[b + q - 1] = id;
+    }
+  };
+  if (lane < (int)c && !((mmask >> lane) & 1u))
+    place(lane - __popc(mmask & ((1u << lane) - 1u)) + ups_before, okey, oval);
+  uint32_t urun = 0;
+  for (uint32_t base = b; base < e; base += 32) {
+    const uint32_t j = base + lane;
+    const bool act = j < e;
+    const uint64_t wk = act ? C.wkey[j] : KEY_MAX;
+    const uint32_t wo = act ? C.wop[j] : 0;
+    uint32_t lo = 0;
+#pragma unroll
+    for (int i = 0; i < FAN; ++i) lo += shfl64(okey, i) < wk ? 1u : 0u;
+    const bool ups = act && wo != OP_DELETE;
+    const uint32_t um = __ballot_sync(FULL, ups);
+    if (ups) place(lo - __popc(mmask & ((1u << lo) - 1u)) + urun + __popc(um & lanemask_lt()), wk, C.wval[j]);
+    urun += __popc(um);
+  }
+  for (uint32_t q0 = 0; q0 < k; q0 += 2) {   // pad unused slots with KEY_MAX
+    const uint32_t q = q0 + (lane >> 4), s = lane & 15;
+    if (q < k) {
+      const uint32_t sz = bs + (q < rem ? 1u : 0u);
+      if (s >= sz) t.lkeys[(size_t)(q == 0 ? X : first + q - 1) * FAN + s] = KEY_MAX;
+    }
+  }
+  __threadfence();
+  __syncwarp();
+  if (k > 1) {
+    for (uint32_t q = 1 + lane; q < k; q += 32) {
+      const uint32_t id = first + q - 1;
+      NodeMeta mt;
+      mt.version = 0;
+      mt.lo = ld_cg(Ek + b + q - 1);
+      mt.hi = (q + 1 < k) ? ld_cg(Ek + b + q) : X_hi;
+      mt.next = (q + 1 < k) ? id + 1 : X_next;
+      mt.count = bs + (q < rem ? 1u : 0u);
+      mt.level = 0;
+      t.lmeta[id] = mt;
+    }
+    __threadfence();
+    __syncwarp();
+    if (lane == 0) {
+      t.lmeta[X].hi = ld_cg(Ek + b);
+      t.lmeta[X].next = first;
+      t.lmeta[X].count = bs + (rem > 0 ? 1u : 0u);
+    }
+    ws.leaf_splits += 1;
+    ws.new_leaves += k - 1;
+  } else if (lane == 0) {
+    t.lmeta[X].count = tout;
+  }
+  __threadfence();
+  __syncwarp();
+  return k;
+}
+
+// Merge m entries (K, Ch)[eb ..] (sorted separators, all inside [plo, phi))
+// into the locked parent P (level L, snapshot pk/pc in lanes 0..15) by key:
+// the children of P and the new nodes form one sequence sorted by their left
+// separator ("lowsep"; P's first child has lowsep plo < every entry).  t <= 16
+// elements stay in P; otherwise an even multi-way split into ceil(t/16) nodes
+// whose (lo, id) entries for P's parent are written to (K2, Ch2)[eb ..].
+// Returns the number of those entries (0 if P did not split).
+__device__ uint32_t inner_apply(const Ctx& C, uint32_t P, uint32_t L, uint64_t pk, uint32_t pc, uint32_t cP,
+                                uint64_t plo, uint64_t phi, uint32_t pnext, const uint64_t* K, const uint32_t* Ch,
+                                uint64_t* K2, uint32_t* Ch2, uint32_t eb, uint32_t m, WarpStats& ws) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  const uint32_t tout = cP + m;
+  const uint32_t kp = tout <= FAN ? 1u : (tout + FAN - 1) / FAN;
+  const uint32_t first = kp > 1 ? warp_alloc(&t.hdr->inner_count, kp - 1) : 0u;
+  if (kp > 1 && lane == 0) atomicAdd(&t.hdr->level_count[L], kp - 1);
+  const uint32_t bs = tout / kp, rem = tout % kp, big = rem * (bs + 1);
+  // element at merged position g -> (node, slot); slot 0 of node q >= 1 is that node's lo
+  auto place = [&](uint32_t g, uint32_t child, uint64_t lowsep) {
+    uint32_t q, start;
+    if (g < big) {
+      q = g / (bs + 1);
+      start = q * (bs + 1);
+    } else {
+      q = rem + (g - big) / bs;
+      start = big + (q - rem) * bs;
+    }
+    const uint32_t slot = g - start;
+    const uint32_t id = q == 0 ? P : first + q - 1;
+    t.ichild[(size_t)id * FAN + slot] = child;
+    if (slot > 0) {
+      t.ikeys[(size_t)id * FAN + slot - 1] = lowsep;
+    } else if (q > 0) {
+      K2[eb + q - 1] = lowsep;
+      Ch2[eb + q - 1] = id;
+    }
+  };
+  // P's children: position i + #(entries < lowsep_i)
+  const uint64_t left_sep = shfl64(pk, (lane + 31) & 31);
+  const uint64_t my_low = lane == 0 ? plo : left_sep;
+  uint32_t below = 0;
+  for (uint32_t base = 0; base < m; base += 32) {
+    const uint32_t x = base + lane;
+    const uint64_t ek = x < m ? ld_cg(K + eb + x) : KEY_MAX;
+    for (uint32_t i = 1; i < cP; ++i) {   // entries are > plo, so child 0 stays first
+      const uint64_t li = shfl64(pk, i - 1);
+      const uint32_t bm = __ballot_sync(FULL, ek < li);
+      if (lane == (int)i) below += __popc(bm);
+    }
+  }
+  // padding first (disjoint from the element slots below)
+  for (uint32_t q0 = 0; q0 < kp; q0 += 2) {
+    const uint32_t q = q0 + (lane >> 4), s = lane & 15;
+    if (q < kp) {
+      const uint32_t size = bs + (q < rem ? 1u : 0u);
+      const uint32_t id = q == 0 ? P : first + q - 1;
+      if (s >= size) t.ichild[(size_t)id * FAN + s] = NIL;
+      if (s + 1 >= size) t.ikeys[(size_t)id * FAN + s] = KEY_MAX;
+    }
+  }
+  __syncwarp();
+  if (lane < (int)cP) place(lane + below, pc, my_low);
+  // entries: position x + 1 + #(P separators < key)
+  for (uint32_t base = 0; base < m; base += 32) {
+    const uint32_t x = base + lane;
+    const bool act = x < m;
+    const uint64_t ek = act ? ld_cg(K + eb + x) : KEY_MAX;
+    const uint32_t ec = act ? ld_cg(Ch + eb + x) : NIL;
+    uint32_t lt = 0;
+#pragma unroll
+    for (int i = 0; i < FAN - 1; ++i) lt += shfl64(pk, i) < ek ? 1u : 0u;   // pk[>= cP-1] == KEY_MAX
+    if (act) place(x + 1 + lt, ec, ek);
+  }
+  __threadfence();
+  __syncwarp();
+  if (kp == 1) {
+    if (lane == 0) t.imeta[P].count = tout;
+    __threadfence();
+    __syncwarp();
+    return 0;
+  }
+  for (uint32_t q = 1 + lane; q < kp; q += 32) {
+    const uint32_t id = first + q - 1;
+    NodeMeta mt;
+    mt.version = 0;
+    mt.lo = ld_cg(K2 + eb + q - 1);
+    mt.hi = (q + 1 < kp) ? ld_cg(K2 + eb + q) : phi;
+    mt.next = (q + 1 < kp) ? id + 1 : pnext;
+    mt.count = bs + (q < rem ? 1u : 0u);
+    mt.level = L;
+    t.imeta[id] = mt;
+  }
+  __threadfence();
+  __syncwarp();
+  if (lane == 0) {
+    t.imeta[P].count = bs + (rem > 0 ? 1u : 0u);
+    t.imeta[P].hi = ld_cg(K2 + eb);
+    t.imeta[P].next = first;
+  }
+  __threadfence();
+  __syncwarp();
+  ws.inner_splits += 1;
+  ws.new_inner += kp - 1;
+  return kp - 1;
+}
+
+// Insert m entries (separator, new node) produced by splits at level L into
+// level L+1, repeating upward while parents split.  Entries are merged into a
+// parent BY KEY, so two splits of the same node whose parent insertions arrive
+// in either order still leave the separators sorted.  Pending lists form a
+// depth-first stack; a list produced from a consumed chunk [eb, eb+c) is at
+// most c long and lives at [eb, ..) of the other ping-pong buffer, so the
+// stacked lists never overlap.
+__device__ void insert_up(const Ctx& C, uint32_t L0, uint32_t eb0, uint32_t m0, WarpStats& ws) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  uint32_t st_L[MAX_LEVELS], st_eb[MAX_LEVELS], st_m[MAX_LEVELS];
+  int sp = 0;
+  st_L[0] = L0;
+  st_eb[0] = eb0;
+  st_m[0] = m0;
+  while (sp >= 0) {
+    if (st_m[sp] == 0) {
+      --sp;
+      continue;
+    }
+    const uint32_t L = st_L[sp], eb = st_eb[sp], m = st_m[sp];
+    if (sp + 1 >= MAX_LEVELS) {
+      watchdog(C, ws, 3, L, eb, m, 0);
+      return;
+    }
+    uint64_t* K = C.eK[L & 1];
+    uint32_t* Ch = C.eC[L & 1];
+    uint64_t* K2 = C.eK[(L + 1) & 1];
+    uint32_t* Ch2 = C.eC[(L + 1) & 1];
+    const uint64_t s = ld_cg(K + eb);
+    uint32_t retry = 0, next_m = 0, P = NIL, consumed = 0;
+    for (;;) {
+      const bool stm = C.force_stm || retry >= C.threshold;
+      if (stm) ws.stm += 1;
+      P = descend(C, s, L + 1, stm);
+      if (P != NIL) {
+        uint32_t* vp = &t.imeta[P].version;
+        uint32_t v;
+        if (try_lock(vp, &v)) {
+          const size_t pb = (size_t)P * FAN;
+          const uint64_t pk = lane < FAN ? ld_cg(t.ikeys + pb + lane) : KEY_MAX;
+          const uint32_t pc = lane < FAN ? ld_cg(t.ichild + pb + lane) : NIL;
+          const uint32_t cP = ld_cg(&t.imeta[P].count);
+          const uint64_t plo = ld_cg(&t.imeta[P].lo), phi = ld_cg(&t.imeta[P].hi);
+          const uint32_t pnext = ld_cg(&t.imeta[P].next);
+          if (s >= plo && s < phi) {   // P covers s: "key in range(node)" (Alg.1:38)
+            // the prefix of the entries that P covers; the rest belongs to P's right siblings
+            uint32_t m1 = m;
+            for (uint32_t base = 0; base < m; base += 32) {
+              const uint32_t x = base + lane;
+              const uint32_t mk = __ballot_sync(FULL, x < m && ld_cg(K + eb + x) >= phi);
+              if (mk) {
+                m1 = base + __ffs(mk) - 1;
+                break;
+              }
+            }
+            next_m = inner_apply(C, P, L + 1, pk, pc, cP, plo, phi, pnext, K, Ch, K2, Ch2, eb, m1, ws);
+            if (next_m > 0 && is_root(t, P, L + 1)) {   // root: phi is the top fence, so m1 == m
+              build_root(C, L + 1, P, plo, phi, K2, Ch2, K, Ch, eb, next_m, ws);
+              next_m = 0;
+            }
+            unlock(vp, v + 2u);
+            consumed = m1;
+            break;
+          }
+          unlock(vp, v);   // validation failed: P does not cover s (any more)
+        }
+      }
+      ++retry;
+      ws.retries += 1;
+      if (watchdog(C, ws, 2, L, eb, P, retry)) return;
+      backoff(retry);
+    }
+    // depth first: the entries P's split produced (level L+2 list, at the same
+    // offset eb) go before the rest of this level's list
+    st_eb[sp] = eb + consumed;
+    st_m[sp] = m - consumed;
+    if (next_m > 0) {
+      ++sp;
+      st_L[sp] = L + 1;
+      st_eb[sp] = eb;
+      st_m[sp] = next_m;
+    }
+  }
+}
+
+// One run of writes [b, e) whose first key was located in leaf `hint`.
+__device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint, WarpStats& ws) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  uint32_t retry = 0;
+  while (b < e && !ws.dead) {
+    const uint64_t k0 = C.wkey[b];
+    const bool stm = C.force_stm || retry >= C.threshold;
+    uint32_t X;
+    if (retry == 0 && !stm) {
+      X = hint;   // the unprotected traversal already done by the locate pass (Alg.1:29)
+    } else {
+      if (stm) ws.stm += 1;
+      X = descend(C, k0, 0, stm);
+    }
+    if (X != NIL && X < t.leaf_cap) {
+      uint32_t* vp = &t.lmeta[X].version;
+      uint32_t v;
+      if (try_lock(vp, &v)) {   // leafvers == leaf.version: the CAS expects v (Alg.1:35-38)
+        const uint64_t lo = ld_cg(&t.lmeta[X].lo), hi = ld_cg(&t.lmeta[X].hi);
+        if (k0 >= lo && k0 < hi) {
+          uint32_t e2 = e;
+          for (uint32_t base = b; base < e; base += 32) {
+            const uint32_t j = base + lane;
+            const uint32_t mk = __ballot_sync(FULL, j < e && C.wkey[j] >= hi);
+            if (mk) {
+              e2 = base + __ffs(mk) - 1;
+              break;
+            }
+          }
+          const uint32_t nxt = ld_cg(&t.lmeta[X].next);
+          const uint32_t k = leaf_apply(C, X, b, e2, hi, nxt, C.eK[0], C.eC[0], ws);
+          ws.runs += 1;
+          if (k > 1) {
+            bool rooted = false;
+            if (is_root(t, X, 0)) {
+              build_root(C, 0, X, lo, hi, C.eK[0], C.eC[0], C.eK[1], C.eC[1], b, k - 1, ws);
+              rooted = true;
+            }
+            unlock(vp, v + 2u);   // split: version + 1 step
+            if (!rooted) insert_up(C, 0, b, k - 1, ws);
+          } else {
+            unlock(vp, v);
+          }
+          b = e2;
+          hint = nxt;
+          retry = 0;
+          continue;
+        }
+        unlock(vp, v);   // key not in range(leaf): abort (Alg.1:40-43)
+      }
+    }
+    ++retry;
+    ws.retries += 1;
+    if (watchdog(C, ws, 1, b, e, X, retry)) return;
+    backoff(retry);
+  }
+}
+
+__global__ void __launch_bounds__(128) update_kernel(Ctx C) {
+  const BatchCtl* ctl = C.ctl;
+  if (ctl->invalid || ctl->status != 0) return;
+  const uint32_t nw = ctl->nw;
+  const int lane = lane_id();
+  const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  WarpStats ws;
+  ws.t0 = gtime_ns();
+  if (C.regroup) {
+    for (uint32_t chunk = gw; chunk * 32 < nw; chunk += nwarps) {
+      const uint32_t base = chunk * 32;
+      const uint32_t j = base + lane;
+      const bool act = j < nw;
+      const uint32_t lf = act ? C.wleaf[j] : NIL;
+      const uint32_t pv = (act && j > 0) ? C.wleaf[j - 1] : NIL;
+      uint32_t heads = __ballot_sync(FULL, act && (j == 0 || lf != pv));
+      while (heads) {
+        const int h = __ffs(heads) - 1;
+        heads &= heads - 1;
+        const uint32_t b = base + h;
+        const uint32_t leaf = shfl32(lf, h);
+        uint32_t e;
+        if (heads) {
+          e = base + __ffs(heads) - 1;
+        } else {
+          e = nw;
+          for (uint32_t s = base + 32; s < nw; s += 32) {
+            const uint32_t jj = s + lane;
+            const uint32_t mk = __ballot_sync(FULL, jj < nw && C.wleaf[jj] != leaf);
+            if (mk) {
+              e = s + __ffs(mk) - 1;
+              break;
+            }
+            if (s + 32 >= nw) e = nw;
+          }
+        }
+        process_run(C, b, e, leaf, ws);
+        if (ws.dead) break;
+      }
+    }
+  } else {
+    for (uint32_t j = gw; j < nw && !ws.dead; j += nwarps) process_run(C, j, j + 1, C.wleaf[j], ws);
+  }
+  if (C.stats && lane == 0) {
+    BatchCtl* c = C.ctl;
+    if (ws.runs) atomicAdd(&c->leaf_runs, ws.runs);
+    if (ws.retries) atomicAdd(&c->retries, ws.retries);
+    if (ws.stm) atomicAdd(&c->stm_fallbacks, ws.stm);
+    if (ws.leaf_splits) atomicAdd(&c->leaf_splits, ws.leaf_splits);
+    if (ws.inner_splits) atomicAdd(&c->inner_splits, ws.inner_splits);
+    if (ws.new_leaves) atomicAdd(&c->new_leaves, ws.new_leaves);
+    if (ws.new_inner) atomicAdd(&c->new_inner, ws.new_inner);
+  }
+}
+
+}  // namespace
+
+void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms, cudaStream_t st,
+                   int* launches) {
+  Ctx C;
+  C.t = t;
+  C.wkey = c.wkey;
+  C.wop = c.wop;
+  C.wval = c.wval;
+  C.wseg = c.wseg;
+  C.wleaf = c.wleaf;
+  C.old = c.old;
+  C.eK[0] = p.entA_key;
+  C.eC[0] = p.entA_child;
+  C.eK[1] = p.entB_key;
+  C.eC[1] = p.entB_child;
+  C.threshold = (p.flags & EIRENE_F_FORCE_STM) ? 0u : p.threshold;
+  C.force_stm = (p.flags & EIRENE_F_FORCE_STM) != 0 || p.threshold == 0;
+  C.regroup = (p.flags & EIRENE_F_REGROUP) != 0;
+  C.stats = (p.flags & EIRENE_F_STATS) != 0;
+  C.ctl = ctl;
+  const uint32_t warps_needed = C.regroup ? (n + 31) / 32 : n;
+  uint32_t blocks = (warps_needed + 3) / 4;
+  blocks = std::min<uint32_t>(blocks, (uint32_t)num_sms * 8u);
+  if (blocks < 1) blocks = 1;
+  static const char* serial = std::getenv("EIRENE_UPDATE_SERIAL");   // debug: one warp, no concurrency
+  if (serial) {
+    update_kernel<<<1, 32, 0, st>>>(C);
+  } else {
+    update_kernel<<<blocks, 128, 0, st>>>(C);
+  }
+  ++*launches;
+}
+
+}  // namespace eirene

@@ -1,0 +1,181 @@
+"""Python face of the C ABI: an Eirene tree on one GPU, fed with torch tensors.
+
+PyTorch only provides device memory and streams here; every step of the batch
+pipeline runs in the sm_100a kernels behind libeirene.so (include/eirene.h).
+
+    t = EireneTree(max_keys=1 << 24, max_batch=1 << 20)
+    t.bulk_load(keys_u64, vals_u64)                   # torch.uint64 on cuda
+    ticket = t.submit(ops_u8, keys_u64, vals_u64, results_u64)
+    stats = t.results(ticket)                         # waits, returns a dict
+    k, v = t.scan()                                   # in-order contents
+"""
+from __future__ import annotations
+
+import ctypes
+
+import torch
+
+from . import _ffi
+from ._ffi import check
+
+U64_MAX = (1 << 64) - 1
+
+
+def _ptr(t: torch.Tensor | None) -> int | None:
+    return None if t is None else t.data_ptr()
+
+
+def _need(t: torch.Tensor, dtype: torch.dtype, dev: torch.device, name: str, n: int | None = None):
+    if t.dtype != dtype:
+        raise TypeError(f"{name}: expected {dtype}, got {t.dtype}")
+    if t.device != dev:
+        raise ValueError(f"{name}: expected device {dev}, got {t.device}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name}: must be contiguous")
+    if n is not None and t.numel() < n:
+        raise ValueError(f"{name}: needs {n} elements")
+
+
+class EireneTree:
+    """One B+tree (or one key-range shard of it) resident on one GPU."""
+
+    def __init__(self, max_keys: int = 1 << 24, max_batch: int = 1 << 20, device: int | None = None,
+                 retry_threshold: int = 4, regroup: bool = True, stats: bool = True, force_stm: bool = False,
+                 timing: bool = False, key_lo: int = 0, key_hi: int = U64_MAX):
+        L = _ffi.lib()
+        if device is None:
+            device = torch.cuda.current_device()
+        self.device = torch.device("cuda", device)
+        cfg = _ffi.eirene_config()
+        L.eirene_default_config(ctypes.byref(cfg))
+        cfg.device = device
+        cfg.max_keys = max_keys
+        cfg.max_batch = max_batch
+        cfg.retry_threshold = retry_threshold
+        cfg.flags = ((_ffi.EIRENE_F_REGROUP if regroup else 0) | (_ffi.EIRENE_F_STATS if stats else 0) |
+                     (_ffi.EIRENE_F_FORCE_STM if force_stm else 0) | (_ffi.EIRENE_F_TIMING if timing else 0))
+        cfg.key_lo = key_lo
+        cfg.key_hi = key_hi
+        self.cfg = cfg
+        h = ctypes.c_void_p()
+        check(L.eirene_create(ctypes.byref(cfg), ctypes.byref(h)), "eirene_create")
+        self._h = h
+        self._L = L
+        self.max_batch = max_batch
+
+    # ---------------------------------------------------------------- lifecycle
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            self._L.eirene_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def _stream(self, stream):
+        s = stream if stream is not None else torch.cuda.current_stream(self.device)
+        return s.cuda_stream
+
+    # ---------------------------------------------------------------- ABI calls
+    def bulk_load(self, keys: torch.Tensor, vals: torch.Tensor, leaf_fill: float = 1.0, stream=None):
+        _need(keys, torch.uint64, self.device, "keys")
+        _need(vals, torch.uint64, self.device, "vals", keys.numel())
+        check(self._L.eirene_bulk_load(self._h, _ptr(keys), _ptr(vals), keys.numel(), leaf_fill,
+                                       self._stream(stream)), "eirene_bulk_load")
+
+    def submit(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor,
+               stream=None) -> int:
+        n = ops.numel()
+        _need(ops, torch.uint8, self.device, "ops")
+        _need(keys, torch.uint64, self.device, "keys", n)
+        _need(vals, torch.uint64, self.device, "vals", n)
+        _need(results, torch.uint64, self.device, "results", n)
+        tk = ctypes.c_uint64()
+        check(self._L.eirene_submit_batch(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n, _ptr(results),
+                                          self._stream(stream), ctypes.byref(tk)), "eirene_submit_batch")
+        return tk.value
+
+    def submit_host(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor,
+                    stream=None) -> int:
+        """Host (ideally pinned) buffers; H2D and D2H copies run inside the call's stream."""
+        n = ops.numel()
+        cpu = torch.device("cpu")
+        _need(ops, torch.uint8, cpu, "ops")
+        _need(keys, torch.uint64, cpu, "keys", n)
+        _need(vals, torch.uint64, cpu, "vals", n)
+        _need(results, torch.uint64, cpu, "results", n)
+        tk = ctypes.c_uint64()
+        check(self._L.eirene_submit_batch_host(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n, _ptr(results),
+                                               self._stream(stream), ctypes.byref(tk)), "eirene_submit_batch_host")
+        return tk.value
+
+    def results(self, ticket: int, raise_on_error: bool = True) -> dict:
+        st = _ffi.eirene_batch_stats()
+        rc = self._L.eirene_results(self._h, ticket, ctypes.byref(st))
+        if rc != _ffi.EIRENE_OK and raise_on_error:
+            raise _ffi.EireneError(rc, "eirene_results")
+        d = st.to_dict()
+        d["rc"] = rc
+        return d
+
+    def apply(self, ops, keys, vals, results=None, stream=None):
+        """submit + results: returns (results tensor, stats dict)."""
+        if results is None:
+            results = torch.empty(ops.numel(), dtype=torch.uint64, device=self.device)
+        tk = self.submit(ops, keys, vals, results, stream)
+        return results, self.results(tk)
+
+    def scan(self, lo: int = 0, hi: int = U64_MAX - 1, stream=None):
+        cnt = ctypes.c_uint64()
+        s = self._stream(stream)
+        check(self._L.eirene_scan(self._h, lo, hi, None, None, 0, ctypes.byref(cnt), s), "eirene_scan")
+        n = cnt.value
+        k = torch.empty(max(n, 1), dtype=torch.uint64, device=self.device)
+        v = torch.empty(max(n, 1), dtype=torch.uint64, device=self.device)
+        check(self._L.eirene_scan(self._h, lo, hi, _ptr(k), _ptr(v), n, ctypes.byref(cnt), s), "eirene_scan")
+        return k[:n], v[:n]
+
+    def check_invariants(self) -> tuple[int, int]:
+        nk = ctypes.c_uint64()
+        rc = self._L.eirene_check_invariants(self._h, ctypes.byref(nk))
+        if rc < 0:
+            raise _ffi.EireneError(rc, "eirene_check_invariants")
+        return rc, nk.value
+
+    def info(self) -> dict:
+        i = _ffi.eirene_tree_info()
+        check(self._L.eirene_get_info(self._h, ctypes.byref(i)), "eirene_get_info")
+        return {f: getattr(i, f) for f, _ in i._fields_}
+
+    # ---------------------------------------------------------------- routing
+    def route_partition(self, ops, keys, vals, splitters: torch.Tensor | None, P: int, stream=None):
+        """Stable partition by destination shard; returns (send_ops, send_keys, send_vals, perm, counts)."""
+        n = ops.numel()
+        dev = self.device
+        sops = torch.empty(n, dtype=torch.uint8, device=dev)
+        skeys = torch.empty(n, dtype=torch.uint64, device=dev)
+        svals = torch.empty(n, dtype=torch.uint64, device=dev)
+        perm = torch.empty(n, dtype=torch.int32, device=dev)
+        counts = torch.empty(P, dtype=torch.int32, device=dev)
+        check(self._L.eirene_route_partition(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n,
+                                             _ptr(splitters) if splitters is not None else None, P, _ptr(sops),
+                                             _ptr(skeys), _ptr(svals), _ptr(perm), _ptr(counts),
+                                             self._stream(stream)), "eirene_route_partition")
+        return sops, skeys, svals, perm, counts
+
+    def route_unpermute(self, recv: torch.Tensor, perm: torch.Tensor, out: torch.Tensor | None = None, stream=None):
+        n = recv.numel()
+        if out is None:
+            out = torch.empty(n, dtype=torch.uint64, device=self.device)
+        check(self._L.eirene_route_unpermute(self._h, _ptr(recv), _ptr(perm), n, _ptr(out), self._stream(stream)),
+              "eirene_route_unpermute")
+        return out

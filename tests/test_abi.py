@@ -1,0 +1,74 @@
+"""CPU-side checks of the boundary: the C-ABI library builds/loads and exports
+every function include/eirene.h declares (no compute calls without a GPU)."""
+import ctypes
+import os
+import subprocess
+
+import pytest
+
+from paper_conf_ppopp_zhangz0lzl23_b200 import _ffi
+from paper_conf_ppopp_zhangz0lzl23_b200.build import LIB, build
+
+
+@pytest.fixture(scope="module")
+def libpath():
+    return build()
+
+
+def test_library_exports_every_header_symbol(libpath):
+    names = _ffi.header_functions()
+    assert len(names) >= 14
+    L = ctypes.CDLL(libpath)
+    missing = [n for n in names if not hasattr(L, n)]
+    assert not missing, f"missing exports: {missing}"
+    # the binding declares a signature for every header function, and nothing else
+    assert sorted(_ffi._SIGS) == names
+
+
+def test_exports_are_c_linkage(libpath):
+    out = subprocess.run(["nm", "-D", "--defined-only", libpath], capture_output=True, text=True).stdout
+    exported = {line.split()[-1] for line in out.splitlines() if " T " in line}
+    for n in _ffi.header_functions():
+        assert n in exported, n
+
+
+def test_sm100a_code_only(libpath):
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", libpath], capture_output=True,
+                         text=True).stdout
+    assert "sm_100a" in out
+    for other in ("sm_80", "sm_90"):
+        assert other + "." not in out
+
+
+def test_host_only_calls_without_gpu(libpath):
+    L = _ffi.lib()
+    cfg = _ffi.eirene_config()
+    L.eirene_default_config(ctypes.byref(cfg))
+    assert cfg.fanout == 16 and cfg.max_batch == 1 << 20 and cfg.retry_threshold == 4
+    assert cfg.key_hi == (1 << 64) - 1
+    assert L.eirene_strerror(_ffi.EIRENE_EFULL).decode().startswith("node pools")
+    # argument validation happens before any device call
+    h = ctypes.c_void_p()
+    bad = _ffi.eirene_config()
+    L.eirene_default_config(ctypes.byref(bad))
+    bad.fanout = 8
+    assert L.eirene_create(ctypes.byref(bad), ctypes.byref(h)) == _ffi.EIRENE_EINVAL
+    assert L.eirene_create(None, ctypes.byref(h)) == _ffi.EIRENE_EINVAL
+    assert L.eirene_results(None, 1, None) == _ffi.EIRENE_EINVAL
+    assert L.eirene_destroy(None) == _ffi.EIRENE_EINVAL
+
+
+def test_product_package_never_imports_oracle():
+    root = os.path.dirname(_ffi.PKG)
+    pkg = _ffi.PKG
+    for dirpath, _, files in os.walk(pkg):
+        for f in files:
+            if f.endswith((".py", ".cu", ".cuh", ".h")):
+                text = open(os.path.join(dirpath, f)).read()
+                assert "import oracle" not in text and "from oracle" not in text, f
+                assert "eirene_oracle" not in text, f
+    # the oracle includes nothing from the product
+    for f in os.listdir(os.path.join(root, "oracle")):
+        if f.endswith((".cpp", ".h")):
+            text = open(os.path.join(root, "oracle", f)).read()
+            assert "eirene.h\"" not in text.replace("eirene_oracle.h\"", "") and "csrc" not in text.split("*/")[-1]
