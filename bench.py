@@ -1,0 +1,392 @@
+#!/usr/bin/env python
+"""Benchmark of the Eirene batched B+tree hot path on B200 (BASELINE.json metric).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 2] [--impl ours|reference]
+
+One step = one batch through the whole hot path (sort -> combine -> partition ->
+query -> update -> RESULT_CAL) on synthetic YCSB-style input
+(workload.py, BASELINE.json configs).  N=1 workload = configs[1] (cfg2): 2^24
+u64 keys, 2^20-request batches, 95% query / 5% update, uniform keys.  With
+N > 1 (torchrun, one rank per GPU, NCCL) the tree is range-partitioned and
+every rank routes its timestamp slice of each global batch with all-to-all
+(weak scaling: 2^24 keys and 2^20 requests per GPU).
+
+Prints ONE JSON line on rank 0 (see DESIGN.md §6 for every field).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_ppopp_zhangz0lzl23_b200 import workload as W  # noqa: E402
+
+PEAKS_FALLBACK = {"hbm_gbs": 6650.0, "source": "fallback (B200_PROFILING.md)"}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return {"hbm_gbs": float(d["hbm_gbs"]), "source": "measured (MEASURED_PEAKS.json)"}
+    except Exception:
+        return dict(PEAKS_FALLBACK)
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[1]) for r in self.rows if len(r) > 2 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) > 2 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            for i, nm in enumerate(names):
+                if len(r) > 5 + i and r[5 + i].lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(self.rows)}
+
+
+# --------------------------------------------------------------------------- stats
+def algorithmic_bytes_query(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, per_leaf: int) -> dict:
+    """Algorithmic HBM bytes of the QUERY kernel for one cfg2 batch:
+    per issued query 8 B key + 4 B seg read + 8 B result write, one 128 B leaf key
+    line per distinct leaf touched, one 32 B value sector per distinct (leaf, sector)
+    hit.  Valid for batches on the bulk-loaded shape (cfg2 never splits)."""
+    uk, first = np.unique(keys, return_index=True)
+    issued_w = np.zeros(uk.size, bool)
+    w = ops != W.QUERY
+    # a key issues a write iff any write on it
+    wk = np.unique(keys[w])
+    issued_w[np.searchsorted(uk, wk)] = True
+    qk = uk[~issued_w]
+    pos = np.searchsorted(loaded, qk)
+    hit = (pos < loaded.size) & (loaded[np.minimum(pos, loaded.size - 1)] == qk)
+    leaf = pos // per_leaf
+    slot = pos % per_leaf
+    lines = np.unique(leaf).size
+    sectors = np.unique(leaf[hit] * 4 + slot[hit] // 4).size
+    nq = qk.size
+    return {"issued_q": int(nq), "leaf_lines": int(lines), "value_sectors": int(sectors),
+            "bytes": int(nq * (8 + 4 + 8) + lines * 128 + sectors * 32)}
+
+
+def run_reference(args):
+    """--impl reference: the CPU oracle (sequential B+tree, 1 thread) as it stands,
+    each step a bounded sample of the same workload."""
+    import oracle
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    cfg = args.config
+    wl = W.Workload(cfg)
+    t = oracle.BTreeOracle(16)
+    t0 = time.time()
+    t.load(wl.keys, wl.vals)
+    load_s = time.time() - t0
+    sample = args.ref_sample
+    times = []
+    total = 0
+    for s in range(args.warmup + args.steps):
+        ops, keys, vals = wl.batch_arrays(s)
+        ops, keys, vals = ops[:sample], keys[:sample], vals[:sample]
+        a = time.perf_counter()
+        t.apply(ops, keys, vals)
+        dt = time.perf_counter() - a
+        if s >= args.warmup:
+            times.append(dt)
+            total += sample
+    tt = sum(times)
+    v = total / tt / 1e9
+    line = {
+        "impl": "reference", "metric": "requests/sec per batch", "value": v, "unit": "Greq/s",
+        "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tt / len(times),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": f"cfg{cfg}: {W.CONFIGS[cfg]['tree']} keys, batch sample {sample} of "
+                               f"{W.CONFIGS[cfg]['batch']} requests", "cfg": cfg},
+        "cpu_baseline": {"value": v, "unit": "Greq/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{args.steps} batches x first {sample} requests; oracle B+tree bulk load "
+                                   f"{load_s:.1f}s untimed"},
+        "e2e": {"value": v, "unit": "Greq/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(args):
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_ppopp_zhangz0lzl23_b200.tree import EireneTree
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.gpus != world and world > 1:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE {world}")
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        from paper_conf_ppopp_zhangz0lzl23_b200.parallel import ShardedEirene
+    cfg = args.config
+    C = W.CONFIGS[cfg]
+    tree_n, batch_n = C["tree"], C["batch"]
+    if args.tree:
+        tree_n = args.tree
+    if args.batch:
+        batch_n = args.batch
+    nb = args.warmup + args.steps
+    stream = torch.cuda.current_stream(dev)
+
+    # ------------------------------------------------------------ inputs
+    t_gen = time.time()
+    if world == 1:
+        wl = W.Workload(cfg, tree=tree_n, batch=batch_n)
+        keys_d = torch.from_numpy(wl.keys).to(dev)
+        vals_d = torch.from_numpy(wl.vals).to(dev)
+        tree = EireneTree(max_keys=max(tree_n * 2, 1 << 20), max_batch=batch_n, timing=True)
+        tree.bulk_load(keys_d, vals_d)
+        del keys_d, vals_d
+        host_batches = [wl.batch_arrays(b) for b in range(nb)]
+        batches = [tuple(torch.from_numpy(a).to(dev) for a in hb) for hb in host_batches]
+        results = [torch.empty(batch_n, dtype=torch.uint64, device=dev) for _ in range(nb)]
+    else:
+        # weak scaling: the global tree holds world * tree_n keys, the global batch
+        # world * batch_n requests; rank r owns key range r and ts-slice r
+        wl = W.Workload(cfg, tree=tree_n * world, batch=batch_n * world)
+        sh = ShardedEirene(wl.keys, wl.vals, max_batch=batch_n, device=dev, timing=True)
+        host_batches = []
+        batches = []
+        for b in range(nb):
+            o, k, v = wl.batch_arrays(b)
+            sl = slice(rank * batch_n, (rank + 1) * batch_n)
+            host_batches.append((o[sl], k[sl], v[sl]))
+            batches.append(tuple(torch.from_numpy(np.ascontiguousarray(a[sl])).to(dev) for a in (o, k, v)))
+        results = [torch.empty(batch_n, dtype=torch.uint64, device=dev) for _ in range(nb)]
+    torch.cuda.synchronize()
+    gen_s = time.time() - t_gen
+
+    # ------------------------------------------------------------ device-timed run
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(nb)]
+    stats = []
+    launches = 0
+
+    def step(b):
+        nonlocal launches
+        o, k, v = batches[b]
+        ev[b][0].record(stream)
+        if world == 1:
+            tk = tree.submit(o, k, v, results[b])
+            ev[b][1].record(stream)
+            return tk
+        st = sh.apply(o, k, v, results[b])
+        ev[b][1].record(stream)
+        return st
+
+    for b in range(args.warmup):
+        r = step(b)
+        stats.append(tree.results(r) if world == 1 else r)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks = ClockSampler(local)
+    with clocks:
+        t_start = torch.cuda.Event(enable_timing=True)
+        t_end = torch.cuda.Event(enable_timing=True)
+        t_start.record(stream)
+        tickets = []
+        for b in range(args.warmup, nb):
+            tickets.append(step(b))
+        t_end.record(stream)
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+    for r in tickets:
+        stats.append(tree.results(r) if world == 1 else r)
+    elapsed_ms = t_start.elapsed_time(t_end)
+    per_batch_ms = np.array([ev[b][0].elapsed_time(ev[b][1]) for b in range(args.warmup, nb)])
+    launches = int(sum(s["launches"] for s in stats[args.warmup:]))
+    if world > 1:
+        tmax = torch.tensor([elapsed_ms], device=dev)
+        dist.all_reduce(tmax, op=dist.ReduceOp.MAX)
+        elapsed_ms = float(tmax.item())
+    total_req = batch_n * world * args.steps
+    value = total_req / (elapsed_ms * 1e-3) / 1e9
+
+    # stage breakdown (CUDA events recorded by the library on the same stream)
+    stage_names = ["sort", "combine", "partition", "query", "update", "result"]
+    stage_ms = np.array([s["stage_ms"][:6] for s in stats[args.warmup:]]).mean(axis=0)
+
+    # ------------------------------------------------------------ e2e through the public API (host buffers)
+    e2e = None
+    if world == 1 and args.e2e_steps > 0:
+        hb = [wl.batch_arrays(nb + i) for i in range(args.e2e_steps)]
+        pin = [tuple(torch.from_numpy(a).pin_memory() for a in x) for x in hb]
+        hres = [torch.empty(batch_n, dtype=torch.uint64).pin_memory() for _ in hb]
+        tk = tree.submit_host(*pin[0], hres[0])   # warm the path
+        tree.results(tk)
+        torch.cuda.synchronize()
+        a = torch.cuda.Event(enable_timing=True)
+        z = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        tks = [tree.submit_host(*pin[i], hres[i]) for i in range(1, len(pin))]
+        z.record(stream)
+        for t_ in tks:
+            tree.results(t_)
+        torch.cuda.synchronize()
+        e_ms = a.elapsed_time(z)
+        n_e = len(pin) - 1
+        e2e = {"value": batch_n * n_e / (e_ms * 1e-3) / 1e9, "unit": "Greq/s",
+               "h2d_bytes_per_step": int(batch_n * 17), "d2h_bytes_per_step": int(batch_n * 8),
+               "steps": n_e, "path": "eirene_submit_batch_host (pinned host buffers, H2D+kernels+D2H on one stream)"}
+    elif world > 1:
+        e2e = {"value": None, "unit": "Greq/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
+               "note": "multi-GPU e2e not measured this round"}
+
+    # ------------------------------------------------------------ parity + CPU baseline (rank 0, N=1)
+    parity = None
+    cpu = None
+    roof = None
+    if rank == 0 and world == 1 and args.cpu_batches > 0:
+        import oracle
+        ref = oracle.BTreeOracle(16)
+        t0 = time.time()
+        ref.load(wl.keys, wl.vals)
+        load_s = time.time() - t0
+        n_check = min(args.cpu_batches, nb)
+        cpu_t = 0.0
+        bad = 0
+        for b in range(n_check):
+            o, k, v = host_batches[b]
+            a = time.perf_counter()
+            want = ref.apply(o, k, v)
+            cpu_t += time.perf_counter() - a
+            bad += int(np.sum(results[b].cpu().numpy() != want))
+        parity = {"batches_checked": n_check, "mismatches": bad, "vs": "oracle B+tree, every request, bit-exact"}
+        cpu = {"value": n_check * batch_n / cpu_t / 1e9, "unit": "Greq/s", "cores": 1, "kind": "oracle",
+               "sample": f"first {n_check} batches of the same workload ({n_check * batch_n} requests), "
+                         f"sequential B+tree, 1 thread; bulk load {load_s:.1f}s untimed"}
+        # roofline of the dominant kernel
+        peaks = load_peaks()
+        dom = int(np.argmax(stage_ms))
+        if stage_names[dom] == "query" or args.roofline_kernel == "query":
+            ab = [algorithmic_bytes_query(wl.keys, *host_batches[b][:2], 16)["bytes"] for b in range(args.warmup, min(nb, args.warmup + 4))]
+            bytes_per = float(np.mean(ab))
+            ms = stage_ms[3]
+            kern = "query_kernel"
+        else:
+            # sort stage: 1 upsweep (8+1+8 B/req read) + 8 passes x (12 B read + 12 B write) per request
+            bytes_per = batch_n * (17 + 8 * 24)
+            ms = stage_ms[0]
+            kern = "sort (upsweep + 8 x sort_pass_kernel)"
+        ach = bytes_per / (ms * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
+                "frac": ach / peaks["hbm_gbs"], "traffic": None, "kernel": kern,
+                "stage_ms": ms, "algorithmic_bytes_per_launch": bytes_per, "peak_source": peaks["source"]}
+
+    if rank == 0:
+        line = {
+            "metric": "requests/sec per batch", "value": value, "unit": "Greq/s", "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic",
+            "config": {"workload": f"cfg{cfg}: {tree_n * world} u64 keys (fanout 16, fill 1.0), "
+                                   f"{batch_n * world}-request batches, "
+                                   + ", ".join(f"{int(p * 100)}% {['query', 'update', 'insert', 'delete'][o]}"
+                                               for o, p in sorted(C['fracs'].items())) + f", {C['dist']} keys",
+                       "cfg": cfg, "global_batch": batch_n * world,
+                       "parallelism": f"key-range shards x{world}" if world > 1 else "single GPU",
+                       "l2": "distinct input/result buffers per step (steps x 25 MiB >> 126 MB L2); "
+                             "inner levels stay L2-resident across batches (steady state)"},
+            "batch_ms": {"mean": float(per_batch_ms.mean()), "min": float(per_batch_ms.min()),
+                         "max": float(per_batch_ms.max()),
+                         "variance_maxmin_over_mean": float((per_batch_ms.max() - per_batch_ms.min()) /
+                                                            per_batch_ms.mean()),
+                         "cv": float(per_batch_ms.std() / per_batch_ms.mean())},
+            "stage_ms": {n: float(x) for n, x in zip(stage_names, stage_ms)},
+            "gpu_launches": launches,
+            "clocks": clocks.summary(),
+            "e2e": e2e,
+            "roofline": roof,
+            "cpu_baseline": cpu,
+            "parity": parity,
+            "setup_s": gen_s,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", type=int, default=2)
+    ap.add_argument("--tree", type=int, default=0, help="override tree size (keys per GPU)")
+    ap.add_argument("--batch", type=int, default=0, help="override batch size (requests per GPU)")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--e2e-steps", type=int, default=11)
+    ap.add_argument("--cpu-batches", type=int, default=2)
+    ap.add_argument("--ref-sample", type=int, default=1 << 18)
+    ap.add_argument("--roofline-kernel", default="auto")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        raise SystemExit("--warmup must be >= 3")
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

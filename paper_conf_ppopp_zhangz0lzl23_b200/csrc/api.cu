@@ -39,10 +39,13 @@ int cuda_fail(cudaError_t e, const char* where) {
     if (_e != cudaSuccess) return cuda_fail(_e, #expr); \
   } while (0)
 
-__global__ void finalize_kernel(BatchCtl* ctl, const TreeHdr* hdr) {
+__global__ void finalize_kernel(BatchCtl* ctl, const TreeHdr* hdr, int dbgprint) {
   if (threadIdx.x == 0) {
     if (ctl->invalid) ctl->status = EIRENE_EINVAL;
     ctl->height = (uint32_t)(hdr->root_word >> 32);
+    if (dbgprint)
+      printf("[eirene dbg] %u %u %u %u %u %u %u %u\n", ctl->dbg[0], ctl->dbg[1], ctl->dbg[2], ctl->dbg[3],
+             ctl->dbg[4], ctl->dbg[5], ctl->dbg[6], ctl->dbg[7]);
   }
 }
 
@@ -209,6 +212,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->cb.wval, nb);
   AL(h->cb.wseg, nb);
   AL(h->cb.wleaf, nb);
+  AL(h->cb.wslot, nb);
   AL(h->cb.old, nb);
   AL(h->up.entA_key, nb + 64);
   AL(h->up.entA_child, nb + 64);
@@ -348,7 +352,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   if (r.timing) cudaEventRecord(r.st[5], st);
   launch_result(spay, n, h->cb, results, ctl, st, &launches);
   stage("result");
-  finalize_kernel<<<1, 32, 0, st>>>(ctl, h->t.hdr);
+  finalize_kernel<<<1, 32, 0, st>>>(ctl, h->t.hdr, dbg ? 1 : 0);
   ++launches;
   if (r.timing) cudaEventRecord(r.st[6], st);
   CK(cudaGetLastError());

@@ -122,6 +122,17 @@ __device__ __forceinline__ unsigned long long ld_acquire64(const unsigned long l
   asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
   return v;
 }
+__device__ __forceinline__ uint32_t ld_relaxed(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+// CAS with acquire semantics: the lock acquisition of the STM's eager write ownership.
+__device__ __forceinline__ uint32_t atom_cas_acquire(uint32_t* p, uint32_t cmp, uint32_t val) {
+  uint32_t old;
+  asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "l"(p), "r"(cmp), "r"(val) : "memory");
+  return old;
+}
 __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
@@ -179,6 +190,7 @@ struct CombBufs {
   uint64_t* wval;
   uint32_t* wseg;
   uint32_t* wleaf;
+  uint8_t* wslot;             // [n] slot of the write's key in its leaf at locate time, 255 = absent
   uint64_t* old;              // [n] old value per segment
 };
 constexpr int COMB_THREADS = 256;

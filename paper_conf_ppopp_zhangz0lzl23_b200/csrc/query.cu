@@ -47,7 +47,8 @@ __device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_
 
 __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__ qkey,
                                                      const uint32_t* __restrict__ qseg,
-                                                     const uint64_t* __restrict__ wkey, uint32_t* __restrict__ wleaf,
+                                                     const uint64_t* __restrict__ wkey, const uint32_t* __restrict__ wseg,
+                                                     uint32_t* __restrict__ wleaf, uint8_t* __restrict__ wslot,
                                                      uint64_t* __restrict__ old, Tree t,
                                                      const BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0) return;
@@ -63,11 +64,19 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
       const uint32_t c = route16(t.ikeys + (size_t)node * FAN, k);
       node = __ldg(t.ichild + (size_t)node * FAN + c);
     }
+    // every issued request retrieves the value its key holds before the batch
+    // (queries: Alg.1:20; writes: "the old value ... retrieved by the issued
+    // request").  Issued keys are distinct, so no other request of
+    // the batch can change that value.
+    const int s = slot16(t.lkeys + (size_t)node * FAN, k);
+    const uint64_t v = s >= 0 ? __ldg(t.lvals + (size_t)node * FAN + s) : KEY_MAX;
     if (isq) {
-      const int s = slot16(t.lkeys + (size_t)node * FAN, k);
-      old[qseg[i]] = s >= 0 ? __ldg(t.lvals + (size_t)node * FAN + s) : KEY_MAX;
+      old[qseg[i]] = v;
     } else {
-      wleaf[i - nq] = node;
+      const uint32_t w = i - nq;
+      old[wseg[w]] = v;
+      wleaf[w] = node;
+      wslot[w] = s >= 0 ? (uint8_t)s : (uint8_t)255;
     }
   }
 }
@@ -77,7 +86,7 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
 void launch_query(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
-  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wleaf, c.old, t, ctl);
+  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wleaf, c.wslot, c.old, t, ctl);
   ++*launches;
 }
 

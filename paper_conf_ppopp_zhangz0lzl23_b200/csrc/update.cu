@@ -40,6 +40,7 @@ struct Ctx {
   const uint64_t* wval;
   const uint32_t* wseg;
   const uint32_t* wleaf;
+  const uint8_t* wslot;
   uint64_t* old;
   uint64_t* eK[2];    // entry ping-pong buffers: separators to insert at the next level
   uint32_t* eC[2];
@@ -92,21 +93,24 @@ __device__ __forceinline__ NodeMeta* meta_of(const Tree& t, uint32_t node, bool 
 
 // Warp-collective lock acquisition: TX_BEGIN with eager conflict detection.
 // Returns true and the pre-lock version in *v if the node was free.
+// Acquire: lane 0's CAS has acquire semantics and __syncwarp orders the other
+// lanes' subsequent (L2-coherent) reads after it.
 __device__ __forceinline__ bool try_lock(uint32_t* vp, uint32_t* v_out) {
   uint32_t v = 0, ok = 0;
   if (lane_id() == 0) {
-    v = ld_acquire(vp);
-    ok = (!(v & 1u) && atomicCAS(vp, v, v | 1u) == v) ? 1u : 0u;
+    v = ld_relaxed(vp);
+    ok = (!(v & 1u) && atom_cas_acquire(vp, v, v | 1u) == v) ? 1u : 0u;
   }
   ok = shfl32(ok, 0);
   v = shfl32(v, 0);
-  __threadfence();
+  __syncwarp();
   *v_out = v;
   return ok != 0;
 }
 
+// Release: __syncwarp makes every lane's writes happen-before lane 0's
+// release store (release is cumulative in the PTX memory model).
 __device__ __forceinline__ void unlock(uint32_t* vp, uint32_t newv) {
-  __threadfence();
   __syncwarp();
   if (lane_id() == 0) st_release(vp, newv);
   __syncwarp();
@@ -277,7 +281,6 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
     const uint64_t at = shfl64(okey, lo);
     const uint64_t ov = shfl64(oval, lo);
     const bool match = act && lo < c && at == wk;
-    if (act) C.old[C.wseg[j]] = match ? ov : KEY_MAX;   // the issued write retrieves the old value
     const bool ups = act && wo != OP_DELETE;
     mmask |= __reduce_or_sync(FULL, match ? (1u << lo) : 0u);
     const uint32_t um = __ballot_sync(FULL, ups);
@@ -301,9 +304,7 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
       for (int i = 0; i < FAN; ++i) lo += shfl64(okey, i) < wk ? 1u : 0u;
       if (act) t.lvals[xb + lo] = C.wval[j];
     }
-    __threadfence();
-    __syncwarp();
-    return 1;
+    return 1;   // ordered before the release by unlock()
   }
   const uint32_t tout = c - __popc(mmask) + U;
   const uint32_t k = tout <= FAN ? 1u : (tout + FAN - 1) / FAN;
@@ -624,6 +625,9 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
           continue;
         }
         unlock(vp, v);   // key not in range(leaf): abort (Alg.1:40-43)
+        if (lane == 0 && retry == 0) atomicAdd(&C.ctl->dbg[4], 1u);
+      } else if (lane == 0 && retry == 0) {
+        atomicAdd(&C.ctl->dbg[3], 1u);
       }
     }
     ++retry;
@@ -640,6 +644,7 @@ __global__ void __launch_bounds__(128) update_kernel(Ctx C) {
   const int lane = lane_id();
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
   const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  const Tree& t = C.t;
   WarpStats ws;
   ws.t0 = gtime_ns();
   if (C.regroup) {
@@ -649,15 +654,45 @@ __global__ void __launch_bounds__(128) update_kernel(Ctx C) {
       const bool act = j < nw;
       const uint32_t lf = act ? C.wleaf[j] : NIL;
       const uint32_t pv = (act && j > 0) ? C.wleaf[j - 1] : NIL;
-      uint32_t heads = __ballot_sync(FULL, act && (j == 0 || lf != pv));
+      const bool head = act && (j == 0 || lf != pv);
+      // Lane-parallel path for the common case of a run of ONE write that
+      // overwrites a key present in its leaf: the lane is the warp of Alg.1:24.
+      // TX: leafvers = version (Alg.1:35); CAS(v -> v|1) (TX_BEGIN, eager
+      // ownership); validate that the key still sits in the located slot (the
+      // range check of Alg.1:38 specialised to an in-place write); write; release.
+      const uint32_t nx = (act && j + 1 < nw) ? C.wleaf[j + 1] : NIL;
+      const uint8_t sl = act ? C.wslot[j] : 255;
+      bool fast = head && nx != lf && sl != 255 && C.wop[j] != OP_DELETE;
+      if (fast) {
+        uint32_t* vp = &t.lmeta[lf].version;
+        const uint32_t v = ld_relaxed(vp);
+        if (!(v & 1u) && atom_cas_acquire(vp, v, v | 1u) == v) {
+          const size_t at = (size_t)lf * FAN + sl;
+          if (ld_cg(t.lkeys + at) == C.wkey[j]) {
+            t.lvals[at] = C.wval[j];
+          } else {
+            fast = false;
+            atomicAdd(&C.ctl->dbg[2], 1u);
+          }
+          st_release(vp, v);
+        } else {
+          fast = false;
+          atomicAdd(&C.ctl->dbg[1], 1u);
+        }
+      }
+      const uint32_t fastm = __ballot_sync(FULL, fast);
+      ws.runs += __popc(fastm);
+      const uint32_t allheads = __ballot_sync(FULL, head);
+      uint32_t heads = allheads & ~fastm;
       while (heads) {
         const int h = __ffs(heads) - 1;
         heads &= heads - 1;
         const uint32_t b = base + h;
         const uint32_t leaf = shfl32(lf, h);
+        const uint32_t later = allheads & ~((2u << h) - 1u);   // heads after h (fast ones included)
         uint32_t e;
-        if (heads) {
-          e = base + __ffs(heads) - 1;
+        if (later) {
+          e = base + __ffs(later) - 1;
         } else {
           e = nw;
           for (uint32_t s = base + 32; s < nw; s += 32) {
@@ -700,6 +735,7 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
   C.wval = c.wval;
   C.wseg = c.wseg;
   C.wleaf = c.wleaf;
+  C.wslot = c.wslot;
   C.old = c.old;
   C.eK[0] = p.entA_key;
   C.eC[0] = p.entA_child;
