@@ -90,6 +90,8 @@ struct eirene_tree {
   int num_sms = 148;
   Tree t{};
   SortBufs sb{};
+  BSortBufs bs{};
+  bool legacy_sort = std::getenv("EIRENE_LEGACY_SORT") != nullptr;
   CombBufs cb{};
   UpdParams up{};
   unsigned char* zero_region = nullptr;
@@ -224,6 +226,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->st_res, nb);
   AL(h->route_lb, ((nb + 2047) / 2048) * 64);
   AL(h->route_ctr, 1);
+  AL(h->bs.bstart, 4097);
+  AL(h->bs.cursor, 4096);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
   {
     size_t off = 0;
@@ -234,6 +238,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     };
     const size_t o_ctl = bump(sizeof(BatchCtl));
     const size_t o_gh = bump(sizeof(uint32_t) * 8 * 256);
+    const size_t o_bc = bump(sizeof(uint32_t) * 4096);
     const size_t o_cs = bump(sizeof(unsigned long long) * comb_tiles);
     const size_t o_ps = bump(sizeof(unsigned long long) * comb_tiles);
     h->zero_bytes = off;
@@ -241,6 +246,11 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     if (e == cudaSuccess) {
       h->ctl = reinterpret_cast<BatchCtl*>(h->zero_region + o_ctl);
       h->sb.ghist = reinterpret_cast<uint32_t*>(h->zero_region + o_gh);
+      h->bs.bcount = reinterpret_cast<uint32_t*>(h->zero_region + o_bc);
+      h->bs.kA = h->sb.kA;
+      h->bs.pA = h->sb.pA;
+      h->bs.kB = h->sb.kB;
+      h->bs.pB = h->sb.pB;
       h->cb.comb_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_cs);
       h->cb.part_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_ps);
     }
@@ -334,8 +344,14 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   CK(cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, st));
   uint64_t* skey;
   uint32_t* spay;
-  launch_sort(keys, ops, nullptr, vals, n, h->cfg.key_lo, h->cfg.key_hi, h->sb, ctl, seq * 8u, st, &launches, &skey,
-              &spay);
+  if (h->legacy_sort) {   // 8-pass onesweep LSD (kept for A/B measurement)
+    launch_sort(keys, ops, nullptr, vals, n, h->cfg.key_lo, h->cfg.key_hi, h->sb, ctl, seq * 8u, st, &launches,
+                &skey, &spay);
+  } else {
+    launch_bucket_sort(keys, ops, vals, n, h->cfg.key_lo, h->cfg.key_hi, h->bs, ctl, h->num_sms, st, &launches);
+    skey = h->bs.kB;
+    spay = h->bs.pB;
+  }
   stage("sort");
   if (r.timing) cudaEventRecord(r.st[1], st);
   launch_combine(skey, spay, vals, results, n, h->cb, ctl, st, &launches);

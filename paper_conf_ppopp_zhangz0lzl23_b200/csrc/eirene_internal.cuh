@@ -176,6 +176,21 @@ void launch_sort(const uint64_t* keys, const uint8_t* ops, const uint32_t* pay_i
 
 size_t sort_lookback_words(uint32_t max_n);
 
+// Batch request sort (bsort.cu): bucket by the top bits, sort buckets in smem.
+struct BSortBufs {
+  uint64_t* kA;      // [n] bucketed (unordered within a bucket)
+  uint32_t* pA;
+  uint64_t* kB;      // [n] sorted output
+  uint32_t* pB;
+  uint32_t* bcount;  // [4096] zeroed per batch
+  uint32_t* bstart;  // [4097]
+  uint32_t* cursor;  // [4096]
+};
+int bsort_bits(uint32_t n);
+void launch_bucket_sort(const uint64_t* keys, const uint8_t* ops, const uint64_t* vals, uint32_t n, uint64_t key_lo,
+                        uint64_t key_hi, const BSortBufs& b, BatchCtl* ctl, int num_sms, cudaStream_t st,
+                        int* launches);
+
 struct CombBufs {
   uint32_t* pinfo;            // [n] seg | DONE
   uint64_t* ikey;             // [n] issued key per segment
