@@ -216,6 +216,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->cb.wleaf, nb);
   AL(h->cb.wslot, nb);
   AL(h->cb.old, nb);
+  AL(h->cb.istart, nb + 1);
+  AL(h->cb.longseg, nb);
   AL(h->up.entA_key, nb + 64);
   AL(h->up.entA_child, nb + 64);
   AL(h->up.entB_key, nb + 64);
@@ -360,7 +362,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   launch_partition(n, h->cb, h->t, ctl, st, &launches);
   stage("partition");
   if (r.timing) cudaEventRecord(r.st[3], st);
-  launch_query(n, h->cb, h->t, ctl, h->num_sms, st, &launches);
+  launch_query(n, h->cb, spay, results, h->t, ctl, h->num_sms, st, &launches);
   stage("query");
   if (r.timing) cudaEventRecord(r.st[4], st);
   launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, st, &launches);

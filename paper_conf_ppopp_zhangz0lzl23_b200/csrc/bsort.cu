@@ -47,14 +47,26 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const uint64_t* _
   __syncthreads();
   uint32_t* hw = h + ((tid >> 5) & 1) * nb;
   bool bad = false;
-  const uint32_t stride = gridDim.x * H_THREADS;
-  for (uint32_t i = blockIdx.x * H_THREADS + tid; i < n; i += stride) {
-    const uint64_t k = keys[i];
-    atomicAdd(&hw[(uint32_t)(k >> (64 - bb))], 1u);
-    if (ops) {
-      const uint32_t o = ops[i];
-      const bool up = (o == OP_UPDATE || o == OP_INSERT);
-      bad |= o > OP_DELETE || k == KEY_MAX || k < key_lo || k >= key_hi || (up && vals[i] == KEY_MAX);
+  // one tile of 16 x 256 requests per CTA, all loads issued before any atomic
+  constexpr int HI = 16;
+  const uint32_t t0 = blockIdx.x * (H_THREADS * HI);
+  uint64_t k[HI];
+  uint32_t o[HI];
+#pragma unroll
+  for (int j = 0; j < HI; ++j) {
+    const uint32_t i = t0 + j * H_THREADS + tid;
+    k[j] = i < n ? keys[i] : 0;
+    o[j] = (ops && i < n) ? (uint32_t)ops[i] : 0u;
+  }
+#pragma unroll
+  for (int j = 0; j < HI; ++j) {
+    const uint32_t i = t0 + j * H_THREADS + tid;
+    if (i < n) {
+      atomicAdd(&hw[(uint32_t)(k[j] >> (64 - bb))], 1u);
+      if (ops) {
+        const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
+        bad |= o[j] > OP_DELETE || k[j] == KEY_MAX || k[j] < key_lo || k[j] >= key_hi || (up && vals[i] == KEY_MAX);
+      }
     }
   }
   if (__any_sync(FULL, bad) && lane == 0) atomicOr(&ctl->invalid, 1u);
@@ -347,8 +359,7 @@ void launch_bucket_sort(const uint64_t* keys, const uint8_t* ops, const uint64_t
   }
   const int bb = bsort_bits(n);
   const uint32_t nb = 1u << bb;
-  int hb = (int)std::min<uint32_t>((n + H_THREADS * 16 - 1) / (H_THREADS * 16), (uint32_t)num_sms * 2u);
-  if (hb < 1) hb = 1;
+  const uint32_t hb = (n + H_THREADS * 16 - 1) / (H_THREADS * 16);
   bsort_hist_kernel<<<hb, H_THREADS, 2 * nb * sizeof(uint32_t), st>>>(keys, ops, vals, n, bb, key_lo, key_hi, b.bcount,
                                                                   ctl);
   bsort_plan_kernel<<<1, 1024, 0, st>>>(b.bcount, bb, b.bstart, b.cursor);

@@ -64,7 +64,8 @@ __device__ __forceinline__ Agg block_excl_scan_agg(Agg v, Agg* tmp, Agg* total) 
 __global__ void __launch_bounds__(COMB_THREADS) combine_kernel(
     const uint64_t* __restrict__ skey, const uint32_t* __restrict__ spay, const uint64_t* __restrict__ vals,
     uint64_t* __restrict__ results, uint32_t n, uint32_t* __restrict__ pinfo, uint64_t* __restrict__ ikey,
-    uint8_t* __restrict__ iop, uint64_t* __restrict__ ival, unsigned long long* __restrict__ status,
+    uint8_t* __restrict__ iop, uint64_t* __restrict__ ival, uint32_t* __restrict__ istart,
+    unsigned long long* __restrict__ status,
     BatchCtl* __restrict__ ctl) {
   __shared__ uint32_t s_tile;
   __shared__ Agg s_tmp[COMB_THREADS / 32];
@@ -100,29 +101,40 @@ __global__ void __launch_bounds__(COMB_THREADS) combine_kernel(
   Agg tile_tot;
   Agg bex = block_excl_scan_agg<COMB_THREADS>(mine, s_tmp, &tile_tot);
 
-  // decoupled look-back (one chain per tile), thread 0
-  if (tid == 0) {
+  // decoupled look-back, warp 0: 32 predecessors per step (the operator --
+  // sum of heads, max of write positions -- is commutative, so a window is
+  // reduced with warp shuffles once every tile up to the nearest inclusive
+  // prefix has published)
+  if (tid < 32) {
+    const int lane = tid;
     unsigned long long* my = status + tile;
     Agg excl = {0, 0};
     if (tile == 0) {
-      st_relaxed64(my, agg_pack(tile_tot, F_INC));
+      if (lane == 0) st_relaxed64(my, agg_pack(tile_tot, F_INC));
     } else {
-      st_relaxed64(my, agg_pack(tile_tot, F_AGG));
+      if (lane == 0) st_relaxed64(my, agg_pack(tile_tot, F_AGG));
       SpinGuard sg;
       int32_t pt = (int32_t)tile - 1;
-      while (pt >= 0) {
-        unsigned long long w = ld_relaxed64(status + pt);
-        if ((w >> 62) == 0) {
+      for (;;) {
+        const int32_t idx = pt - lane;
+        const unsigned long long w = idx >= 0 ? ld_relaxed64(status + idx) : F_INC;
+        const uint32_t fl = (uint32_t)(w >> 62);
+        const uint32_t inc = __ballot_sync(FULL, fl == 2);
+        const uint32_t need = inc ? ((2u << (__ffs(inc) - 1)) - 1u) : FULL;
+        if (__ballot_sync(FULL, fl == 0) & need) {
           if (sg.stuck(ctl)) break;
           continue;
         }
-        excl = agg_op(agg_unpack(w), excl);
-        if (w & F_INC) break;
-        --pt;
+        Agg a = ((need >> lane) & 1u) ? agg_unpack(w) : Agg{0, 0};
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) a = agg_op(a, Agg{__shfl_xor_sync(FULL, a.nh, o), __shfl_xor_sync(FULL, a.lw, o)});
+        excl = agg_op(a, excl);
+        if (inc) break;
+        pt -= 32;
       }
-      st_relaxed64(my, agg_pack(agg_op(excl, tile_tot), F_INC));
+      if (lane == 0) st_relaxed64(my, agg_pack(agg_op(excl, tile_tot), F_INC));
     }
-    s_prefix = excl;
+    if (lane == 0) s_prefix = excl;
   }
   __syncthreads();
   Agg run = agg_op(s_prefix, bex);   // state before my first item
@@ -158,6 +170,7 @@ __global__ void __launch_bounds__(COMB_THREADS) combine_kernel(
       }
     }
     pinfo[p] = seg | (done ? DONE_BIT : 0u);
+    if (head) istart[seg] = p;
     if (is_write(op)) run.lw = p + 1;
     const uint64_t kn = (j + 1 < COMB_ITEMS) ? k[j + 1] : knext;
     const bool tail = (p == n - 1) || kn != key;
@@ -185,7 +198,10 @@ __global__ void __launch_bounds__(COMB_THREADS) combine_kernel(
       } else {
         iop[seg] = OP_QUERY;
       }
-      if (p == n - 1) ctl->nseg = seg + 1;
+      if (p == n - 1) {
+        ctl->nseg = seg + 1;
+        istart[seg + 1] = n;
+      }
     }
   }
 }
@@ -260,29 +276,37 @@ __global__ void __launch_bounds__(COMB_THREADS) partition_kernel(
   }
   uint32_t tot;
   uint32_t bex = block_excl_scan_u32(mine, s_tmp, &tot);
-  if (tid == 0) {
+  if (tid < 32) {   // warp-parallel decoupled look-back (see combine_kernel)
+    const int lane = tid;
     unsigned long long* my = status + tile;
     uint32_t excl = 0;
     if (tile == 0) {
-      st_relaxed64(my, P_INC | tot);
+      if (lane == 0) st_relaxed64(my, P_INC | tot);
     } else {
-      st_relaxed64(my, P_AGG | tot);
+      if (lane == 0) st_relaxed64(my, P_AGG | tot);
       SpinGuard sg;
       int32_t pt = (int32_t)tile - 1;
-      while (pt >= 0) {
-        unsigned long long w = ld_relaxed64(status + pt);
-        if ((w >> 62) == 0) {
+      for (;;) {
+        const int32_t idx = pt - lane;
+        const unsigned long long w = idx >= 0 ? ld_relaxed64(status + idx) : P_INC;
+        const uint32_t fl = (uint32_t)(w >> 62);
+        const uint32_t inc = __ballot_sync(FULL, fl == 2);
+        const uint32_t need = inc ? ((2u << (__ffs(inc) - 1)) - 1u) : FULL;
+        if (__ballot_sync(FULL, fl == 0) & need) {
           if (sg.stuck(ctl)) break;
           continue;
         }
-        excl += (uint32_t)(w & P_VAL);
-        if (w & P_INC) break;
-        --pt;
+        uint32_t a = ((need >> lane) & 1u) ? (uint32_t)(w & P_VAL) : 0u;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(FULL, a, o);
+        excl += a;
+        if (inc) break;
+        pt -= 32;
       }
-      st_relaxed64(my, P_INC | (excl + tot));
+      if (lane == 0) st_relaxed64(my, P_INC | (excl + tot));
     }
-    s_prefix = excl;
-    if ((tile + 1) * COMB_TILE >= nseg) {   // last tile: totals + headroom check
+    if (lane == 0) s_prefix = excl;
+    if (lane == 0 && (tile + 1) * COMB_TILE >= nseg) {   // last tile: totals + headroom check
       const uint32_t nw = excl + tot;
       ctl->nw = nw;
       ctl->nq = nseg - nw;
@@ -313,15 +337,26 @@ __global__ void __launch_bounds__(COMB_THREADS) partition_kernel(
 // Alg.1:6: positions without an earlier write in their segment take the value
 // their segment's issued request retrieved (old[seg]); results are scattered
 // back to submission (timestamp) order.
-__global__ void __launch_bounds__(256) result_kernel(const uint32_t* __restrict__ spay,
-                                                      const uint32_t* __restrict__ pinfo,
-                                                      const uint64_t* __restrict__ old, uint64_t* __restrict__ results,
-                                                      uint32_t n, const BatchCtl* __restrict__ ctl) {
+// RESULT_CAL is fused into the query kernel: every issued request scatters
+// the value it retrieved to the pending positions of its own segment.  The
+// segments longer than SHORT_SEG (hot keys) are queued instead and finished
+// here with one CTA per segment, so a 56K-request Zipf key does not serialise
+// one thread.
+__global__ void __launch_bounds__(256) result_long_kernel(const uint32_t* __restrict__ spay,
+                                                           const uint32_t* __restrict__ pinfo,
+                                                           const uint32_t* __restrict__ istart,
+                                                           const uint32_t* __restrict__ longseg,
+                                                           const uint64_t* __restrict__ old,
+                                                           uint64_t* __restrict__ results,
+                                                           const BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0) return;
-  const uint32_t stride = gridDim.x * blockDim.x;
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-    const uint32_t info = pinfo[i];
-    if (!(info & DONE_BIT)) results[spay[i] >> 2] = old[info];
+  const uint32_t nl = ctl->nlong;
+  for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
+    const uint32_t s = longseg[x];
+    const uint64_t v = old[s];
+    const uint32_t e = istart[s + 1];
+    for (uint32_t p = istart[s] + threadIdx.x; p < e; p += blockDim.x)
+      if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
   }
 }
 
@@ -331,7 +366,7 @@ void launch_combine(const uint64_t* skey, const uint32_t* spay, const uint64_t* 
                     const CombBufs& c, BatchCtl* ctl, cudaStream_t st, int* launches) {
   const uint32_t tiles = (n + COMB_TILE - 1) / COMB_TILE;
   combine_kernel<<<tiles, COMB_THREADS, 0, st>>>(skey, spay, vals, results, n, c.pinfo, c.ikey, c.iop, c.ival,
-                                                 c.comb_status, ctl);
+                                                 c.istart, c.comb_status, ctl);
   ++*launches;
 }
 
@@ -344,8 +379,8 @@ void launch_partition(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, cuda
 
 void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, uint64_t* results, BatchCtl* ctl,
                    cudaStream_t st, int* launches) {
-  int blocks = (int)std::min<uint32_t>((n + 255) / 256, 148u * 8u);
-  result_kernel<<<blocks, 256, 0, st>>>(spay, c.pinfo, c.old, results, n, ctl);
+  (void)n;
+  result_long_kernel<<<148, 256, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, results, ctl);
   ++*launches;
 }
 

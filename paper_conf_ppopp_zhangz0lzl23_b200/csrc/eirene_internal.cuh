@@ -54,6 +54,7 @@ struct BatchCtl {
   uint32_t invalid;
   uint32_t tile_ctr[16];
   uint32_t nseg, nq, nw, height;
+  uint32_t nlong, pad_;
   unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
   uint32_t dbg[8];   // watchdog diagnostics
 };
@@ -207,7 +208,10 @@ struct CombBufs {
   uint32_t* wleaf;
   uint8_t* wslot;             // [n] slot of the write's key in its leaf at locate time, 255 = absent
   uint64_t* old;              // [n] old value per segment
+  uint32_t* istart;           // [n+1] sorted position of each segment's first request (+ n at nseg)
+  uint32_t* longseg;          // [n] segments longer than SHORT_SEG, finished by result_long_kernel
 };
+constexpr uint32_t SHORT_SEG = 32;
 constexpr int COMB_THREADS = 256;
 constexpr int COMB_ITEMS = 8;
 constexpr int COMB_TILE = COMB_THREADS * COMB_ITEMS;
@@ -215,8 +219,8 @@ constexpr int COMB_TILE = COMB_THREADS * COMB_ITEMS;
 void launch_combine(const uint64_t* skey, const uint32_t* spay, const uint64_t* vals, uint64_t* results,
                     uint32_t n, const CombBufs& c, BatchCtl* ctl, cudaStream_t st, int* launches);
 void launch_partition(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, cudaStream_t st, int* launches);
-void launch_query(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, int num_sms, cudaStream_t st,
-                  int* launches);
+void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, uint64_t* results, Tree t, BatchCtl* ctl,
+                  int num_sms, cudaStream_t st, int* launches);
 
 struct UpdParams {
   uint32_t threshold;

@@ -1,4 +1,5 @@
-// query.cu -- QUERY_KERNEL (Alg.1:15-21) and leaf locate for the issued writes.
+// query.cu -- QUERY_KERNEL (Alg.1:15-21), leaf locate for the issued writes,
+// and the fused RESULT_CAL (Alg.1:6) for short segments.
 //
 // Issued queries run with no concurrency control: the tree is
 // quiescent (the update kernel of the previous batch has finished, and this
@@ -10,8 +11,16 @@
 // 2^24 keys) stay L2-resident across batches; leaves (256 MiB) come from HBM:
 // one 128 B key line plus one 32 B value sector per issued query.
 //
-// The same traversal gives each issued write its target leaf (a4, the input
-// of the leaf-run regrouping in the update kernel).
+// The same traversal gives each issued write its target leaf and slot (a4,
+// the input of the leaf-run regrouping in the update kernel) and the value
+// its key holds before the batch ("the old (original) value ... retrieved by
+// the issued request").  Issued keys are distinct, so no other
+// request of the batch can change that value before the update kernel runs.
+//
+// RESULT_CAL: the un-issued requests of a segment that have no
+// earlier write take the retrieved value.  The thread that retrieved it
+// scatters it to its segment's pending positions (results in timestamp
+// order); segments longer than SHORT_SEG are queued for result_long_kernel.
 #include "eirene_internal.cuh"
 
 namespace eirene {
@@ -49,8 +58,10 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
                                                      const uint32_t* __restrict__ qseg,
                                                      const uint64_t* __restrict__ wkey, const uint32_t* __restrict__ wseg,
                                                      uint32_t* __restrict__ wleaf, uint8_t* __restrict__ wslot,
-                                                     uint64_t* __restrict__ old, Tree t,
-                                                     const BatchCtl* __restrict__ ctl) {
+                                                     uint64_t* __restrict__ old, const uint32_t* __restrict__ spay,
+                                                     const uint32_t* __restrict__ pinfo,
+                                                     const uint32_t* __restrict__ istart, uint32_t* __restrict__ longseg,
+                                                     uint64_t* __restrict__ results, Tree t, BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0) return;
   const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
   const unsigned long long rw = t.hdr->root_word;
@@ -64,29 +75,40 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
       const uint32_t c = route16(t.ikeys + (size_t)node * FAN, k);
       node = __ldg(t.ichild + (size_t)node * FAN + c);
     }
-    // every issued request retrieves the value its key holds before the batch
-    // (queries: Alg.1:20; writes: "the old value ... retrieved by the issued
-    // request").  Issued keys are distinct, so no other request of
-    // the batch can change that value.
     const int s = slot16(t.lkeys + (size_t)node * FAN, k);
     const uint64_t v = s >= 0 ? __ldg(t.lvals + (size_t)node * FAN + s) : KEY_MAX;
+    uint32_t seg;
     if (isq) {
-      old[qseg[i]] = v;
+      seg = qseg[i];
     } else {
       const uint32_t w = i - nq;
-      old[wseg[w]] = v;
+      seg = wseg[w];
       wleaf[w] = node;
       wslot[w] = s >= 0 ? (uint8_t)s : (uint8_t)255;
+    }
+    old[seg] = v;
+    const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
+    if (p1 - p0 <= SHORT_SEG) {
+      if (isq) {   // an all-query segment: every position is pending
+        for (uint32_t p = p0; p < p1; ++p) results[spay[p] >> 2] = v;
+      } else {     // positions up to (and including) the first write are pending
+        for (uint32_t p = p0; p < p1; ++p)
+          if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
+      }
+    } else {
+      longseg[atomicAdd(&ctl->nlong, 1u)] = seg;
     }
   }
 }
 
 }  // namespace
 
-void launch_query(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
+void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, uint64_t* results, Tree t, BatchCtl* ctl,
+                  int num_sms, cudaStream_t st, int* launches) {
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
-  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wleaf, c.wslot, c.old, t, ctl);
+  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wleaf, c.wslot, c.old, spay, c.pinfo,
+                                       c.istart, c.longseg, results, t, ctl);
   ++*launches;
 }
 

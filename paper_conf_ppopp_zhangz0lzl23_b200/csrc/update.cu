@@ -655,34 +655,51 @@ __global__ void __launch_bounds__(128) update_kernel(Ctx C) {
       const uint32_t lf = act ? C.wleaf[j] : NIL;
       const uint32_t pv = (act && j > 0) ? C.wleaf[j - 1] : NIL;
       const bool head = act && (j == 0 || lf != pv);
-      // Lane-parallel path for the common case of a run of ONE write that
-      // overwrites a key present in its leaf: the lane is the warp of Alg.1:24.
-      // TX: leafvers = version (Alg.1:35); CAS(v -> v|1) (TX_BEGIN, eager
-      // ownership); validate that the key still sits in the located slot (the
-      // range check of Alg.1:38 specialised to an in-place write); write; release.
+      // Lane-parallel path for the common case: a run that lies inside this
+      // chunk and whose writes all overwrite keys present in the leaf.  The run's
+      // head lane is the run's "thread" of Alg.1:24: leafvers = version
+      // (Alg.1:35); CAS(v -> v|1) (TX_BEGIN, eager ownership); every member
+      // validates that its key still sits in the located slot (the range check
+      // of Alg.1:38 specialised to an in-place write) and writes its value; the
+      // head releases.  Any failure sends the run to the general path below
+      // (value overwrites are idempotent, so redoing them there is harmless).
       const uint32_t nx = (act && j + 1 < nw) ? C.wleaf[j + 1] : NIL;
       const uint8_t sl = act ? C.wslot[j] : 255;
-      bool fast = head && nx != lf && sl != 255 && C.wop[j] != OP_DELETE;
+      const bool member = act && sl != 255 && C.wop[j] != OP_DELETE;
+      const uint32_t allheads = __ballot_sync(FULL, head);
+      const uint32_t tails = __ballot_sync(FULL, act && nx != lf);   // last write of its run
+      const uint32_t nonmember = __ballot_sync(FULL, act && !member);
+      // run of lane x: [head_x, tail_x]; fast iff it ends in this chunk and has no non-member
+      const int hl = 31 - __clz(allheads & (lanemask_lt() | (1u << lane)));   // my run's head lane
+      const uint32_t from_h = ~((1u << hl) - 1u);
+      const uint32_t tail_after = tails & from_h;
+      const int tl = tail_after ? __ffs(tail_after) - 1 : 32;
+      const uint32_t span = tl < 32 ? (from_h & ((2u << tl) - 1u)) : 0u;
+      bool fast = act && tl < 32 && (nonmember & span) == 0;
+      uint32_t lk = 0;   // head: acquired?
+      uint32_t v = 0;
+      uint32_t* vp = &t.lmeta[act ? lf : 0].version;
+      if (fast && lane == hl) {
+        v = ld_relaxed(vp);
+        lk = (!(v & 1u) && atom_cas_acquire(vp, v, v | 1u) == v) ? 1u : 0u;
+      }
+      const uint32_t got = __shfl_sync(FULL, lk, hl & 31);
+      fast = fast && got;
+      bool ok = true;
       if (fast) {
-        uint32_t* vp = &t.lmeta[lf].version;
-        const uint32_t v = ld_relaxed(vp);
-        if (!(v & 1u) && atom_cas_acquire(vp, v, v | 1u) == v) {
-          const size_t at = (size_t)lf * FAN + sl;
-          if (ld_cg(t.lkeys + at) == C.wkey[j]) {
-            t.lvals[at] = C.wval[j];
-          } else {
-            fast = false;
-            atomicAdd(&C.ctl->dbg[2], 1u);
-          }
-          st_release(vp, v);
+        const size_t at = (size_t)lf * FAN + sl;
+        if (ld_cg(t.lkeys + at) == C.wkey[j]) {
+          t.lvals[at] = C.wval[j];
         } else {
-          fast = false;
-          atomicAdd(&C.ctl->dbg[1], 1u);
+          ok = false;
         }
       }
+      const uint32_t bad = __ballot_sync(FULL, fast && !ok);
+      __syncwarp();
+      if (lk) st_release(vp, v);
+      fast = fast && (bad & span) == 0;
       const uint32_t fastm = __ballot_sync(FULL, fast);
-      ws.runs += __popc(fastm);
-      const uint32_t allheads = __ballot_sync(FULL, head);
+      ws.runs += __popc(fastm & allheads);
       uint32_t heads = allheads & ~fastm;
       while (heads) {
         const int h = __ffs(heads) - 1;
@@ -712,15 +729,25 @@ __global__ void __launch_bounds__(128) update_kernel(Ctx C) {
   } else {
     for (uint32_t j = gw; j < nw && !ws.dead; j += nwarps) process_run(C, j, j + 1, C.wleaf[j], ws);
   }
-  if (C.stats && lane == 0) {
-    BatchCtl* c = C.ctl;
-    if (ws.runs) atomicAdd(&c->leaf_runs, ws.runs);
-    if (ws.retries) atomicAdd(&c->retries, ws.retries);
-    if (ws.stm) atomicAdd(&c->stm_fallbacks, ws.stm);
-    if (ws.leaf_splits) atomicAdd(&c->leaf_splits, ws.leaf_splits);
-    if (ws.inner_splits) atomicAdd(&c->inner_splits, ws.inner_splits);
-    if (ws.new_leaves) atomicAdd(&c->new_leaves, ws.new_leaves);
-    if (ws.new_inner) atomicAdd(&c->new_inner, ws.new_inner);
+  if (C.stats) {
+    // reduce the counters per CTA first: one global atomic per CTA and counter
+    // (same-address atomics serialise in L2)
+    __shared__ unsigned long long red[7];
+    if (threadIdx.x < 7) red[threadIdx.x] = 0;
+    __syncthreads();
+    if (lane == 0) {
+      const unsigned long long v[7] = {ws.runs, ws.retries, ws.stm, ws.leaf_splits, ws.inner_splits,
+                                       ws.new_leaves, ws.new_inner};
+      for (int i = 0; i < 7; ++i)
+        if (v[i]) atomicAdd(&red[i], v[i]);
+    }
+    __syncthreads();
+    if (threadIdx.x < 7 && red[threadIdx.x]) {
+      BatchCtl* c = C.ctl;
+      unsigned long long* dst[7] = {&c->leaf_runs, &c->retries, &c->stm_fallbacks, &c->leaf_splits,
+                                    &c->inner_splits, &c->new_leaves, &c->new_inner};
+      atomicAdd(dst[threadIdx.x], red[threadIdx.x]);
+    }
   }
 }
 
