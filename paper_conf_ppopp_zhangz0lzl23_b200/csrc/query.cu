@@ -40,16 +40,35 @@ __device__ __forceinline__ uint32_t route16(const uint64_t* __restrict__ line, u
   return c;
 }
 
+struct uint4x2 {
+  uint4 a, b;
+};
+__device__ __forceinline__ ulonglong4 ldg256(const uint64_t* p) {
+  ulonglong4 v;
+  asm volatile("ld.global.nc.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint4x2 ldg256u32(const uint32_t* p) {
+  uint4x2 v;
+  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(v.a.x), "=r"(v.a.y), "=r"(v.a.z), "=r"(v.a.w), "=r"(v.b.x), "=r"(v.b.y), "=r"(v.b.z),
+                 "=r"(v.b.w)
+               : "l"(p));
+  return v;
+}
+
+// Slot of key k in a 16-key leaf line (4 x 256-bit loads), -1 if absent.
 __device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_t k) {
-  const ulonglong2* l2 = reinterpret_cast<const ulonglong2*>(line);
-  ulonglong2 v[8];
+  ulonglong4 v[4];
 #pragma unroll
-  for (int i = 0; i < 8; ++i) v[i] = __ldg(l2 + i);
+  for (int i = 0; i < 4; ++i) v[i] = ldg256(line + 4 * i);
   int s = -1;
 #pragma unroll
-  for (int i = 0; i < 8; ++i) {
-    if (v[i].x == k) s = 2 * i;
-    if (v[i].y == k) s = 2 * i + 1;
+  for (int i = 0; i < 4; ++i) {
+    if (v[i].x == k) s = 4 * i;
+    if (v[i].y == k) s = 4 * i + 1;
+    if (v[i].z == k) s = 4 * i + 2;
+    if (v[i].w == k) s = 4 * i + 3;
   }
   return s;
 }
@@ -72,7 +91,18 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
     const uint64_t k = isq ? qkey[i] : wkey[i - nq];
     uint32_t node = root;
     for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
-      const uint32_t c = route16(t.ikeys + (size_t)node * FAN, k);
+      // key line and child line are loaded together (12 independent 16-byte
+      // loads), so a level costs one memory round trip instead of two
+      // sm_100 256-bit loads (LDG.E.ENL2.256): a 128 B key line is 4 loads;
+      // then the one child pointer (loading the whole child line speculatively
+      // measured slower: it doubles L1 traffic per level)
+      const uint64_t* kl = t.ikeys + (size_t)node * FAN;
+      ulonglong4 kv[4];
+#pragma unroll
+      for (int x = 0; x < 4; ++x) kv[x] = ldg256(kl + 4 * x);
+      uint32_t c = 0;
+#pragma unroll
+      for (int x = 0; x < 4; ++x) c += (kv[x].x <= k) + (kv[x].y <= k) + (kv[x].z <= k) + (kv[x].w <= k);
       node = __ldg(t.ichild + (size_t)node * FAN + c);
     }
     const int s = slot16(t.lkeys + (size_t)node * FAN, k);
