@@ -187,13 +187,16 @@ const char* eirene_last_cuda_error(void);
  * owns [splitters[r-1], splitters[r]).  splitters_dev holds P-1 increasing
  * keys (device), 1 <= P <= 64.  Writes send_ops/keys/vals_dev[n] grouped by
  * destination in input (timestamp) order, perm_dev[n] (perm[j] = input index
- * of send slot j) and counts_dev[P] (u32).  `h` provides scratch only.
- * Asynchronous on `stream`. */
+ * of send slot j) and counts_dev[P] (u32).  If invalid_dev != NULL, the
+ * request validation of eirene_submit_batch runs here too and sets
+ * *invalid_dev = 1 (never clears it) when any request is invalid, so all
+ * ranks can agree to reject the whole global batch before any shard applies
+ * its part.  `h` provides scratch only.  Asynchronous on `stream`. */
 int eirene_route_partition(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev,
                            const uint64_t* vals_dev, uint32_t n, const uint64_t* splitters_dev,
                            int P, uint8_t* send_ops_dev, uint64_t* send_keys_dev,
                            uint64_t* send_vals_dev, uint32_t* perm_dev, uint32_t* counts_dev,
-                           eirene_stream_t stream);
+                           uint32_t* invalid_dev, eirene_stream_t stream);
 
 /* Inverse of the partition for the returned results:
  * results_dev[perm_dev[j]] = recv_results_dev[j] for j < n.  Asynchronous. */

@@ -62,7 +62,7 @@ _SIGS = {
     "eirene_destroy": (_int, [_vp]),
     "eirene_strerror": (ctypes.c_char_p, [_int]),
     "eirene_last_cuda_error": (ctypes.c_char_p, []),
-    "eirene_route_partition": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _int, _vp, _vp, _vp, _vp, _vp, _vp]),
+    "eirene_route_partition": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _int, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
     "eirene_route_unpermute": (_int, [_vp, _vp, _vp, _u32, _vp, _vp]),
 }
 

@@ -552,14 +552,14 @@ int eirene_check_invariants(eirene_handle h, uint64_t* n_keys) {
 // ---------------------------------------------------------------- routing
 int eirene_route_partition(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                            const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
-                           uint32_t* perm, uint32_t* counts, eirene_stream_t stream) {
+                           uint32_t* perm, uint32_t* counts, uint32_t* invalid, eirene_stream_t stream) {
   if (!h || P < 1 || P > 64 || !counts) return EIRENE_EINVAL;
   if (n > h->cfg.max_batch) return EIRENE_EINVAL;
   if (n > 0 && (!ops || !keys || !vals || !sops || !skeys || !svals || !perm)) return EIRENE_EINVAL;
   if (P > 1 && !splitters) return EIRENE_EINVAL;
   CK(cudaSetDevice(h->cfg.device));
   int launches = 0;
-  launch_route_partition(ops, keys, vals, n, splitters, P, sops, skeys, svals, perm, counts, h->route_lb,
+  launch_route_partition(ops, keys, vals, n, splitters, P, sops, skeys, svals, perm, counts, invalid, h->route_lb,
                          h->route_ctr, ++h->route_epoch, reinterpret_cast<cudaStream_t>(stream), &launches);
   h->launches += launches;
   CK(cudaGetLastError());

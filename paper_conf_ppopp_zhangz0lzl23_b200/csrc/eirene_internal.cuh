@@ -246,8 +246,8 @@ int scan_tree(Tree t, uint32_t leaf_count, uint64_t lo, uint64_t hi, uint64_t* k
 // routing
 void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                             const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
-                            uint32_t* perm, uint32_t* counts, unsigned long long* lookback, uint32_t* tile_ctr,
-                            uint32_t epoch, cudaStream_t st, int* launches);
+                            uint32_t* perm, uint32_t* counts, uint32_t* invalid, unsigned long long* lookback,
+                            uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st, int* launches);
 void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,
                             cudaStream_t st, int* launches);
 

@@ -28,9 +28,12 @@ __device__ __forceinline__ uint32_t dest_of(uint64_t k, const uint64_t* sp, int 
   return d;
 }
 
-__global__ void __launch_bounds__(RT_THREADS) route_count_kernel(const uint64_t* __restrict__ keys, uint32_t n,
+__global__ void __launch_bounds__(RT_THREADS) route_count_kernel(const uint64_t* __restrict__ keys,
+                                                                 const uint8_t* __restrict__ ops,
+                                                                 const uint64_t* __restrict__ vals, uint32_t n,
                                                                  const uint64_t* __restrict__ splitters, int P,
-                                                                 uint32_t* __restrict__ counts) {
+                                                                 uint32_t* __restrict__ counts,
+                                                                 uint32_t* __restrict__ invalid) {
   __shared__ uint64_t sp[RT_MAXP];
   __shared__ uint32_t h[RT_MAXP];
   const int tid = threadIdx.x;
@@ -39,9 +42,17 @@ __global__ void __launch_bounds__(RT_THREADS) route_count_kernel(const uint64_t*
     h[tid] = 0;
   }
   __syncthreads();
+  bool bad = false;
   for (uint32_t i = blockIdx.x * RT_THREADS + tid; i < n; i += gridDim.x * RT_THREADS) {
-    atomicAdd(&h[dest_of(keys[i], sp, P)], 1u);
+    const uint64_t k = keys[i];
+    atomicAdd(&h[dest_of(k, sp, P)], 1u);
+    if (invalid) {
+      const uint32_t o = ops[i];
+      const bool up = (o == OP_UPDATE || o == OP_INSERT);
+      bad |= o > OP_DELETE || k == KEY_MAX || (up && vals[i] == KEY_MAX);
+    }
   }
+  if (__any_sync(FULL, bad) && (tid & 31) == 0) atomicOr(invalid, 1u);
   __syncthreads();
   if (tid < P && h[tid]) atomicAdd(&counts[tid], h[tid]);
 }
@@ -173,8 +184,8 @@ __global__ void unpermute_kernel(const uint64_t* __restrict__ recv, const uint32
 
 void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                             const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
-                            uint32_t* perm, uint32_t* counts, unsigned long long* lookback, uint32_t* tile_ctr,
-                            uint32_t epoch, cudaStream_t st, int* launches) {
+                            uint32_t* perm, uint32_t* counts, uint32_t* invalid, unsigned long long* lookback,
+                            uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st, int* launches) {
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(route_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(RtSmem));
@@ -184,7 +195,7 @@ void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint
   cudaMemsetAsync(tile_ctr, 0, sizeof(uint32_t), st);
   if (n == 0) return;
   int blocks = (int)std::min<uint32_t>((n + RT_THREADS * 8 - 1) / (RT_THREADS * 8), 148u * 4u);
-  route_count_kernel<<<blocks, RT_THREADS, 0, st>>>(keys, n, splitters, P, counts);
+  route_count_kernel<<<blocks, RT_THREADS, 0, st>>>(keys, ops, vals, n, splitters, P, counts, invalid);
   const uint32_t tiles = (n + RT_TILE - 1) / RT_TILE;
   route_scatter_kernel<<<tiles, RT_THREADS, sizeof(RtSmem), st>>>(ops, keys, vals, n, splitters, P, counts, sops,
                                                                   skeys, svals, perm, lookback, epoch, tile_ctr);

@@ -157,8 +157,10 @@ class EireneTree:
         return {f: getattr(i, f) for f, _ in i._fields_}
 
     # ---------------------------------------------------------------- routing
-    def route_partition(self, ops, keys, vals, splitters: torch.Tensor | None, P: int, stream=None):
-        """Stable partition by destination shard; returns (send_ops, send_keys, send_vals, perm, counts)."""
+    def route_partition(self, ops, keys, vals, splitters: torch.Tensor | None, P: int, stream=None,
+                        invalid: torch.Tensor | None = None):
+        """Stable partition by destination shard; returns (send_ops, send_keys, send_vals, perm, counts).
+        `invalid` (int32[1] on the device) is set to 1 if any request is invalid."""
         n = ops.numel()
         dev = self.device
         sops = torch.empty(n, dtype=torch.uint8, device=dev)
@@ -168,7 +170,7 @@ class EireneTree:
         counts = torch.empty(P, dtype=torch.int32, device=dev)
         check(self._L.eirene_route_partition(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n,
                                              _ptr(splitters) if splitters is not None else None, P, _ptr(sops),
-                                             _ptr(skeys), _ptr(svals), _ptr(perm), _ptr(counts),
+                                             _ptr(skeys), _ptr(svals), _ptr(perm), _ptr(counts), _ptr(invalid),
                                              self._stream(stream)), "eirene_route_partition")
         return sops, skeys, svals, perm, counts
 
