@@ -170,10 +170,18 @@ def run_ours(args):
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if args.gpus != world and world > 1:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE {world}")
+    # --backend gloo / EIRENE_BENCH_ONE_GPU=1: functional check of the N>1 code
+    # path with every rank on cuda:0 (NCCL needs one GPU per rank); never a
+    # number to report
+    if os.environ.get("EIRENE_BENCH_ONE_GPU"):
+        local = 0
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        if args.backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group(args.backend)
         from paper_conf_ppopp_zhangz0lzl23_b200.parallel import ShardedEirene
     cfg = args.config
     C = W.CONFIGS[cfg]
@@ -379,6 +387,7 @@ def main():
     ap.add_argument("--cpu-batches", type=int, default=2)
     ap.add_argument("--ref-sample", type=int, default=1 << 18)
     ap.add_argument("--roofline-kernel", default="auto")
+    ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"])
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
