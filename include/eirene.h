@@ -172,6 +172,12 @@ typedef struct {
 /* Synchronous snapshot of the tree's size counters. */
 int eirene_get_info(eirene_handle h, eirene_tree_info* info);
 
+/* Replaces cfg.flags (EIRENE_F_*) for the batches submitted from now on, e.g.
+ * to turn per-stage timing on for a diagnostic run.  Batches are normally
+ * replayed from a captured CUDA graph; with EIRENE_F_TIMING the kernels are
+ * launched directly so that stage events can be recorded between them. */
+int eirene_set_flags(eirene_handle h, uint32_t flags);
+
 /* Frees every device and host resource of the handle (waits for pending work). */
 int eirene_destroy(eirene_handle h);
 

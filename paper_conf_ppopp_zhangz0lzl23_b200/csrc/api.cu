@@ -73,6 +73,27 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
   }
 }
 
+__global__ void set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
+                                uint64_t* results) {
+  if (threadIdx.x == 0) {
+    dst->ops = ops;
+    dst->keys = keys;
+    dst->vals = vals;
+    dst->results = results;
+  }
+}
+
+// kernels in one batch graph: set_args, 4 sort, combine, partition, query, update, result_long, finalize
+constexpr int GRAPH_KERNELS = 11;
+constexpr int MAX_GRAPHS = 8;
+
+struct GraphEntry {
+  uint32_t n = 0;
+  cudaGraph_t graph = nullptr;      // kept alive: args_node belongs to it
+  cudaGraphExec_t exec = nullptr;
+  cudaGraphNode_t args_node = nullptr;
+};
+
 struct Rec {
   uint64_t ticket = 0;
   bool used = false;
@@ -91,7 +112,11 @@ struct eirene_tree {
   Tree t{};
   SortBufs sb{};
   BSortBufs bs{};
-  bool legacy_sort = std::getenv("EIRENE_LEGACY_SORT") != nullptr;
+  BatchArgs* dargs = nullptr;
+  cudaStream_t cap_stream = nullptr;
+  GraphEntry graphs[MAX_GRAPHS];
+  uint32_t next_graph = 0;
+  bool use_graphs = std::getenv("EIRENE_NO_GRAPHS") == nullptr;
   CombBufs cb{};
   UpdParams up{};
   unsigned char* zero_region = nullptr;
@@ -230,6 +255,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->route_ctr, 1);
   AL(h->bs.bstart, 4097);
   AL(h->bs.cursor, 4096);
+  AL(h->dargs, 1);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
   {
     size_t off = 0;
@@ -290,6 +317,11 @@ int eirene_destroy(eirene_handle h) {
     for (int s = 0; s < NSTAGE; ++s)
       if (h->ring[i].st[s]) cudaEventDestroy(h->ring[i].st[s]);
   }
+  for (auto& g : h->graphs) {
+    if (g.exec) cudaGraphExecDestroy(g.exec);
+    if (g.graph) cudaGraphDestroy(g.graph);
+  }
+  if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
   for (void* p : h->allocs) cudaFree(p);
   if (h->host_ctl) cudaFreeHost(h->host_ctl);
   delete h;
@@ -342,38 +374,87 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     cudaError_t e = cudaStreamSynchronize(st);
     std::fprintf(stderr, "[eirene] batch %u stage %s done: %s\n", seq, name, cudaGetErrorString(e));
   };
-  if (r.timing) cudaEventRecord(r.st[0], st);
-  CK(cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, st));
-  uint64_t* skey;
-  uint32_t* spay;
-  if (h->legacy_sort) {   // 8-pass onesweep LSD (kept for A/B measurement)
-    launch_sort(keys, ops, nullptr, vals, n, h->cfg.key_lo, h->cfg.key_hi, h->sb, ctl, seq * 8u, st, &launches,
-                &skey, &spay);
+  // The pipeline: a tiny node that publishes this batch's pointers to the
+  // device-side BatchArgs, then every kernel of Alg.1 reading them from there.
+  auto last_node = [](cudaStream_t s, cudaGraphNode_t* out) -> cudaError_t {
+    cudaStreamCaptureStatus cs;
+    const cudaGraphNode_t* deps = nullptr;
+    size_t nd = 0;
+    cudaError_t e = cudaStreamGetCaptureInfo(s, &cs, nullptr, nullptr, &deps, &nd);
+    if (e != cudaSuccess) return e;
+    if (nd != 1) return cudaErrorStreamCaptureInvalidated;
+    *out = deps[0];
+    return cudaSuccess;
+  };
+  auto rec = [&](int i, cudaStream_t s) { cudaEventRecord(r.st[i], s); };
+  auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
+    set_args_kernel<<<1, 32, 0, s>>>(h->dargs, ops, keys, vals, results);
+    ++launches;
+    if (args_node) {
+      cudaError_t e = last_node(s, args_node);
+      if (e != cudaSuccess) return e;
+    }
+    if (timing) rec(0, s);
+    cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, s);
+    launch_bucket_sort(h->dargs, n, h->cfg.key_lo, h->cfg.key_hi, h->bs, ctl, h->num_sms, s, &launches);
+    const uint64_t* skey = h->bs.kB;
+    const uint32_t* spay = h->bs.pB;
+    stage("sort");
+    if (timing) rec(1, s);
+    launch_combine(skey, spay, h->dargs, n, h->cb, ctl, s, &launches);
+    stage("combine");
+    if (timing) rec(2, s);
+    launch_partition(n, h->cb, h->t, ctl, s, &launches);
+    stage("partition");
+    if (timing) rec(3, s);
+    launch_query(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, s, &launches);
+    stage("query");
+    if (timing) rec(4, s);
+    launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
+    stage("update");
+    if (timing) rec(5, s);
+    launch_result(spay, n, h->cb, h->dargs, ctl, s, &launches);
+    stage("result");
+    finalize_kernel<<<1, 32, 0, s>>>(ctl, h->t.hdr, dbg ? 1 : 0);
+    ++launches;
+    if (timing) rec(6, s);
+    return cudaGetLastError();
+  };
+  if (dbg || r.timing || !h->use_graphs) {   // per-stage events: direct launches
+    CK(enqueue(st, r.timing, nullptr));
   } else {
-    launch_bucket_sort(keys, ops, vals, n, h->cfg.key_lo, h->cfg.key_hi, h->bs, ctl, h->num_sms, st, &launches);
-    skey = h->bs.kB;
-    spay = h->bs.pB;
+    // one captured graph per batch size; a replay updates only the args node
+    GraphEntry* g = nullptr;
+    for (auto& e : h->graphs)
+      if (e.exec && e.n == n) g = &e;
+    if (!g) {
+      GraphEntry& e = h->graphs[h->next_graph++ % MAX_GRAPHS];
+      if (e.exec) cudaGraphExecDestroy(e.exec);
+      if (e.graph) cudaGraphDestroy(e.graph);
+      e = GraphEntry{};
+      CK(cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeRelaxed));
+      cudaError_t ce = enqueue(h->cap_stream, false, &e.args_node);
+      cudaError_t ee = cudaStreamEndCapture(h->cap_stream, &e.graph);
+      if (ce != cudaSuccess) return cuda_fail(ce, "capture");
+      CK(ee);
+      CK(cudaGraphInstantiate(&e.exec, e.graph, 0));
+      e.n = n;
+      g = &e;
+      launches = 0;
+    }
+    void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
+                      const_cast<uint64_t**>(&vals), &results};
+    cudaKernelNodeParams p{};
+    p.func = reinterpret_cast<void*>(set_args_kernel);
+    p.gridDim = dim3(1);
+    p.blockDim = dim3(32);
+    p.sharedMemBytes = 0;
+    p.kernelParams = params;
+    p.extra = nullptr;
+    CK(cudaGraphExecKernelNodeSetParams(g->exec, g->args_node, &p));
+    CK(cudaGraphLaunch(g->exec, st));
+    launches = GRAPH_KERNELS;
   }
-  stage("sort");
-  if (r.timing) cudaEventRecord(r.st[1], st);
-  launch_combine(skey, spay, vals, results, n, h->cb, ctl, st, &launches);
-  stage("combine");
-  if (r.timing) cudaEventRecord(r.st[2], st);
-  launch_partition(n, h->cb, h->t, ctl, st, &launches);
-  stage("partition");
-  if (r.timing) cudaEventRecord(r.st[3], st);
-  launch_query(n, h->cb, spay, results, h->t, ctl, h->num_sms, st, &launches);
-  stage("query");
-  if (r.timing) cudaEventRecord(r.st[4], st);
-  launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, st, &launches);
-  stage("update");
-  if (r.timing) cudaEventRecord(r.st[5], st);
-  launch_result(spay, n, h->cb, results, ctl, st, &launches);
-  stage("result");
-  finalize_kernel<<<1, 32, 0, st>>>(ctl, h->t.hdr, dbg ? 1 : 0);
-  ++launches;
-  if (r.timing) cudaEventRecord(r.st[6], st);
-  CK(cudaGetLastError());
   if (results_host) CK(cudaMemcpyAsync(results_host, results, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, st));
   CK(cudaMemcpyAsync(&h->host_ctl[tk % RING], ctl, sizeof(BatchCtl), cudaMemcpyDeviceToHost, st));
   CK(cudaEventRecord(r.done, st));
@@ -447,6 +528,19 @@ int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out, u
   h->launches += launches;
   if (rc == EIRENE_ECUDA) return cuda_fail(cudaGetLastError(), "eirene_scan");
   return rc;
+}
+
+int eirene_set_flags(eirene_handle h, uint32_t flags) {
+  if (!h) return EIRENE_EINVAL;
+  h->cfg.flags = flags;
+  h->up.flags = flags;
+  // captured graphs bake the update kernel's flags in: drop them
+  for (auto& g : h->graphs) {
+    if (g.exec) cudaGraphExecDestroy(g.exec);
+    if (g.graph) cudaGraphDestroy(g.graph);
+    g = GraphEntry{};
+  }
+  return EIRENE_OK;
 }
 
 int eirene_get_info(eirene_handle h, eirene_tree_info* info) {

@@ -35,12 +35,13 @@ __device__ __forceinline__ bool kp_less(uint64_t ka, uint32_t pa, uint64_t kb, u
   return ka < kb || (ka == kb && pa < pb);
 }
 
-__global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const uint64_t* __restrict__ keys,
-                                                               const uint8_t* __restrict__ ops,
-                                                               const uint64_t* __restrict__ vals, uint32_t n,
+__global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* __restrict__ A, uint32_t n,
                                                                int bb, uint64_t key_lo, uint64_t key_hi,
                                                                uint32_t* __restrict__ bcount, BatchCtl* ctl) {
   extern __shared__ uint32_t h[];   // [2][1 << bb]: two copies (even / odd warps) halve contention
+  const uint64_t* __restrict__ keys = A->keys;
+  const uint8_t* __restrict__ ops = A->ops;
+  const uint64_t* __restrict__ vals = A->vals;
   const int tid = threadIdx.x, lane = tid & 31;
   const uint32_t nb = 1u << bb;
   for (uint32_t i = tid; i < 2 * nb; i += H_THREADS) h[i] = 0;
@@ -119,11 +120,12 @@ __global__ void __launch_bounds__(1024) bsort_plan_kernel(const uint32_t* __rest
 // the scatter.  Global atomics per bucket address = number of tiles (256 at
 // n = 2^20) instead of one per request.
 constexpr int SC_ITEMS = 16;
-__global__ void __launch_bounds__(256) bsort_scatter_kernel(const uint64_t* __restrict__ keys,
-                                                            const uint8_t* __restrict__ ops, uint32_t n, int bb,
+__global__ void __launch_bounds__(256) bsort_scatter_kernel(const BatchArgs* __restrict__ A, uint32_t n, int bb,
                                                             uint32_t* __restrict__ cursor, uint64_t* __restrict__ kout,
                                                             uint32_t* __restrict__ pout, const BatchCtl* ctl) {
   extern __shared__ uint32_t sh[];   // [2 << bb]: tile histogram, then global base per bucket
+  const uint64_t* __restrict__ keys = A->keys;
+  const uint8_t* __restrict__ ops = A->ops;
   if (ctl->invalid) return;
   const int tid = threadIdx.x;
   const uint32_t nb = 1u << bb;
@@ -349,9 +351,9 @@ int bsort_bits(uint32_t n) {
   return bb;
 }
 
-void launch_bucket_sort(const uint64_t* keys, const uint8_t* ops, const uint64_t* vals, uint32_t n, uint64_t key_lo,
-                        uint64_t key_hi, const BSortBufs& b, BatchCtl* ctl, int num_sms, cudaStream_t st,
-                        int* launches) {
+void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
+                        BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
+  (void)num_sms;
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(bsort_local_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(LocSmem));
@@ -360,11 +362,10 @@ void launch_bucket_sort(const uint64_t* keys, const uint8_t* ops, const uint64_t
   const int bb = bsort_bits(n);
   const uint32_t nb = 1u << bb;
   const uint32_t hb = (n + H_THREADS * 16 - 1) / (H_THREADS * 16);
-  bsort_hist_kernel<<<hb, H_THREADS, 2 * nb * sizeof(uint32_t), st>>>(keys, ops, vals, n, bb, key_lo, key_hi, b.bcount,
-                                                                  ctl);
+  bsort_hist_kernel<<<hb, H_THREADS, 2 * nb * sizeof(uint32_t), st>>>(A, n, bb, key_lo, key_hi, b.bcount, ctl);
   bsort_plan_kernel<<<1, 1024, 0, st>>>(b.bcount, bb, b.bstart, b.cursor);
   const uint32_t sbk = (n + 256 * SC_ITEMS - 1) / (256 * SC_ITEMS);
-  bsort_scatter_kernel<<<sbk, 256, 2 * nb * sizeof(uint32_t), st>>>(keys, ops, n, bb, b.cursor, b.kA, b.pA, ctl);
+  bsort_scatter_kernel<<<sbk, 256, 2 * nb * sizeof(uint32_t), st>>>(A, n, bb, b.cursor, b.kA, b.pA, ctl);
   bsort_local_kernel<<<nb, LOC_THREADS, sizeof(LocSmem), st>>>(b.kA, b.pA, b.kB, b.pB, b.bcount, b.bstart, bb, ctl);
   *launches += 4;
 }

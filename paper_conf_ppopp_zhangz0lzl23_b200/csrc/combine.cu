@@ -47,10 +47,12 @@ __device__ __forceinline__ Agg agg_unpack(unsigned long long w) {
 __device__ __forceinline__ uint32_t lanemask_le() { return lanemask_lt() | (1u << lane_id()); }
 
 __global__ void __launch_bounds__(COMB_THREADS) combine_kernel(
-    const uint64_t* __restrict__ skey, const uint32_t* __restrict__ spay, const uint64_t* __restrict__ vals,
-    uint64_t* __restrict__ results, uint32_t n, uint32_t* __restrict__ pinfo, uint64_t* __restrict__ ikey,
+    const uint64_t* __restrict__ skey, const uint32_t* __restrict__ spay, const BatchArgs* __restrict__ A,
+    uint32_t n, uint32_t* __restrict__ pinfo, uint64_t* __restrict__ ikey,
     uint8_t* __restrict__ iop, uint64_t* __restrict__ ival, uint32_t* __restrict__ istart,
     unsigned long long* __restrict__ status, BatchCtl* __restrict__ ctl) {
+  const uint64_t* __restrict__ vals = A->vals;
+  uint64_t* __restrict__ results = A->results;
   __shared__ uint32_t s_tile;
   __shared__ Agg s_w[CW];
   __shared__ Agg s_prefix;
@@ -323,9 +325,10 @@ __global__ void __launch_bounds__(256) result_long_kernel(const uint32_t* __rest
                                                            const uint32_t* __restrict__ istart,
                                                            const uint32_t* __restrict__ longseg,
                                                            const uint64_t* __restrict__ old,
-                                                           uint64_t* __restrict__ results,
+                                                           const BatchArgs* __restrict__ A,
                                                            const BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0) return;
+  uint64_t* __restrict__ results = A->results;
   const uint32_t nl = ctl->nlong;
   for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
     const uint32_t s = longseg[x];
@@ -338,10 +341,10 @@ __global__ void __launch_bounds__(256) result_long_kernel(const uint32_t* __rest
 
 }  // namespace
 
-void launch_combine(const uint64_t* skey, const uint32_t* spay, const uint64_t* vals, uint64_t* results, uint32_t n,
+void launch_combine(const uint64_t* skey, const uint32_t* spay, const BatchArgs* A, uint32_t n,
                     const CombBufs& c, BatchCtl* ctl, cudaStream_t st, int* launches) {
   const uint32_t tiles = (n + COMB_TILE - 1) / COMB_TILE;
-  combine_kernel<<<tiles, COMB_THREADS, 0, st>>>(skey, spay, vals, results, n, c.pinfo, c.ikey, c.iop, c.ival,
+  combine_kernel<<<tiles, COMB_THREADS, 0, st>>>(skey, spay, A, n, c.pinfo, c.ikey, c.iop, c.ival,
                                                  c.istart, c.comb_status, ctl);
   ++*launches;
 }
@@ -353,10 +356,10 @@ void launch_partition(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, cuda
   ++*launches;
 }
 
-void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, uint64_t* results, BatchCtl* ctl,
+void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
                    cudaStream_t st, int* launches) {
   (void)n;
-  result_long_kernel<<<148, 256, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, results, ctl);
+  result_long_kernel<<<148, 256, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, A, ctl);
   ++*launches;
 }
 

@@ -86,6 +86,16 @@ struct SpinGuard {
   }
 };
 
+// Per-batch caller pointers, written on the device by the first node of the
+// batch graph so the captured pipeline can be replayed on new buffers by
+// updating that single node (api.cu).
+struct BatchArgs {
+  const uint8_t* ops;
+  const uint64_t* keys;
+  const uint64_t* vals;
+  uint64_t* results;
+};
+
 // tile counters
 enum { TC_SORT0 = 0, TC_COMB = 8, TC_PART = 9, TC_ROUTE = 10, TC_SCAN = 11 };
 
@@ -188,9 +198,8 @@ struct BSortBufs {
   uint32_t* cursor;  // [4096]
 };
 int bsort_bits(uint32_t n);
-void launch_bucket_sort(const uint64_t* keys, const uint8_t* ops, const uint64_t* vals, uint32_t n, uint64_t key_lo,
-                        uint64_t key_hi, const BSortBufs& b, BatchCtl* ctl, int num_sms, cudaStream_t st,
-                        int* launches);
+void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
+                        BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches);
 
 struct CombBufs {
   uint32_t* pinfo;            // [n] seg | DONE
@@ -216,10 +225,10 @@ constexpr int COMB_THREADS = 256;
 constexpr int COMB_ITEMS = 8;
 constexpr int COMB_TILE = COMB_THREADS * COMB_ITEMS;
 
-void launch_combine(const uint64_t* skey, const uint32_t* spay, const uint64_t* vals, uint64_t* results,
+void launch_combine(const uint64_t* skey, const uint32_t* spay, const BatchArgs* A,
                     uint32_t n, const CombBufs& c, BatchCtl* ctl, cudaStream_t st, int* launches);
 void launch_partition(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, cudaStream_t st, int* launches);
-void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, uint64_t* results, Tree t, BatchCtl* ctl,
+void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches);
 
 struct UpdParams {
@@ -232,7 +241,7 @@ struct UpdParams {
 };
 void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms,
                    cudaStream_t st, int* launches);
-void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, uint64_t* results, BatchCtl* ctl,
+void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
                    cudaStream_t st, int* launches);
 
 // bulk build / scan

@@ -80,8 +80,10 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
                                                      uint64_t* __restrict__ old, const uint32_t* __restrict__ spay,
                                                      const uint32_t* __restrict__ pinfo,
                                                      const uint32_t* __restrict__ istart, uint32_t* __restrict__ longseg,
-                                                     uint64_t* __restrict__ results, Tree t, BatchCtl* __restrict__ ctl) {
+                                                     const BatchArgs* __restrict__ A, Tree t,
+                                                     BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0) return;
+  uint64_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
@@ -133,12 +135,12 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
 
 }  // namespace
 
-void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, uint64_t* results, Tree t, BatchCtl* ctl,
+void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches) {
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
   query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wleaf, c.wslot, c.old, spay, c.pinfo,
-                                       c.istart, c.longseg, results, t, ctl);
+                                       c.istart, c.longseg, A, t, ctl);
   ++*launches;
 }
 

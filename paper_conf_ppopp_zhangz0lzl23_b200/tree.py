@@ -151,6 +151,16 @@ class EireneTree:
             raise _ffi.EireneError(rc, "eirene_check_invariants")
         return rc, nk.value
 
+    def set_flags(self, regroup: bool | None = None, stats: bool | None = None, force_stm: bool | None = None,
+                  timing: bool | None = None):
+        f = self.cfg.flags
+        for on, bit in ((regroup, _ffi.EIRENE_F_REGROUP), (stats, _ffi.EIRENE_F_STATS),
+                        (force_stm, _ffi.EIRENE_F_FORCE_STM), (timing, _ffi.EIRENE_F_TIMING)):
+            if on is not None:
+                f = (f | bit) if on else (f & ~bit)
+        self.cfg.flags = f
+        check(self._L.eirene_set_flags(self._h, f), "eirene_set_flags")
+
     def info(self) -> dict:
         i = _ffi.eirene_tree_info()
         check(self._L.eirene_get_info(self._h, ctypes.byref(i)), "eirene_get_info")
