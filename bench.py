@@ -322,7 +322,8 @@ def run_ours(args):
         n_e = len(pin) - 1
         e2e = {"value": batch_n * n_e / (e_ms * 1e-3) / 1e9, "unit": "Greq/s",
                "h2d_bytes_per_step": int(batch_n * 17), "d2h_bytes_per_step": int(batch_n * 8),
-               "steps": n_e, "path": "eirene_submit_batch_host (pinned host buffers, H2D+kernels+D2H on one stream)"}
+               "steps": n_e, "path": "eirene_submit_batch_host (pinned host buffers; H2D of batch b+1 on the "
+                                     "library's copy stream overlaps batch b's kernels + D2H)"}
     elif world > 1:
         e2e = {"value": None, "unit": "Greq/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
                "note": "multi-GPU e2e not measured this round"}
@@ -411,7 +412,7 @@ def main():
     ap.add_argument("--tree", type=int, default=0, help="override tree size (keys per GPU)")
     ap.add_argument("--batch", type=int, default=0, help="override batch size (requests per GPU)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--e2e-steps", type=int, default=11)
+    ap.add_argument("--e2e-steps", type=int, default=21)
     ap.add_argument("--cpu-batches", type=int, default=2)
     ap.add_argument("--ref-sample", type=int, default=1 << 18)
     ap.add_argument("--roofline-kernel", default="auto")

@@ -123,6 +123,10 @@ struct eirene_tree {
   size_t zero_bytes = 0;
   BatchCtl* ctl = nullptr;
   BatchCtl* host_ctl = nullptr;   // pinned [RING]
+  cudaStream_t h2d_stream = nullptr;
+  cudaEvent_t h2d_done[2] = {}, comp_done[2] = {};
+  bool slot_used[2] = {false, false};
+  uint32_t host_slot = 0;
   uint8_t* st_ops = nullptr;
   uint64_t* st_keys = nullptr;
   uint64_t* st_vals = nullptr;
@@ -247,10 +251,15 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->up.entA_child, nb + 64);
   AL(h->up.entB_key, nb + 64);
   AL(h->up.entB_child, nb + 64);
-  AL(h->st_ops, nb);
-  AL(h->st_keys, nb);
-  AL(h->st_vals, nb);
-  AL(h->st_res, nb);
+  AL(h->st_ops, 2 * nb);
+  AL(h->st_keys, 2 * nb);
+  AL(h->st_vals, 2 * nb);
+  AL(h->st_res, 2 * nb);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->h2d_stream, cudaStreamNonBlocking);
+  for (int s = 0; s < 2 && e == cudaSuccess; ++s) {
+    e = cudaEventCreateWithFlags(&h->h2d_done[s], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->comp_done[s], cudaEventDisableTiming);
+  }
   AL(h->route_lb, ((nb + 2047) / 2048) * 64);
   AL(h->route_ctr, 1);
   AL(h->bs.bstart, 4097);
@@ -322,6 +331,11 @@ int eirene_destroy(eirene_handle h) {
     if (g.graph) cudaGraphDestroy(g.graph);
   }
   if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
+  if (h->h2d_stream) cudaStreamDestroy(h->h2d_stream);
+  for (int s = 0; s < 2; ++s) {
+    if (h->h2d_done[s]) cudaEventDestroy(h->h2d_done[s]);
+    if (h->comp_done[s]) cudaEventDestroy(h->comp_done[s]);
+  }
   for (void* p : h->allocs) cudaFree(p);
   if (h->host_ctl) cudaFreeHost(h->host_ctl);
   delete h;
@@ -478,10 +492,26 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   CK(cudaSetDevice(h->cfg.device));
-  CK(cudaMemcpyAsync(h->st_ops, ops, n, cudaMemcpyHostToDevice, st));
-  CK(cudaMemcpyAsync(h->st_keys, keys, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, st));
-  CK(cudaMemcpyAsync(h->st_vals, vals, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, st));
-  return submit_impl(h, h->st_ops, h->st_keys, h->st_vals, n, h->st_res, st, results, ticket);
+  // Double-buffered staging: the H2D copy of this batch runs on the handle's
+  // copy stream into slot s while the previous batch computes on `st`; the
+  // slot is reused only after the batch that last used it has finished (its
+  // D2H of results is ordered on `st` behind its kernels).
+  const int s = (int)(h->host_slot++ & 1u);
+  if (h->slot_used[s]) CK(cudaStreamWaitEvent(h->h2d_stream, h->comp_done[s], 0));
+  CK(cudaMemcpyAsync(h->st_ops + (size_t)s * h->cfg.max_batch, ops, n, cudaMemcpyHostToDevice, h->h2d_stream));
+  CK(cudaMemcpyAsync(h->st_keys + (size_t)s * h->cfg.max_batch, keys, sizeof(uint64_t) * n, cudaMemcpyHostToDevice,
+                     h->h2d_stream));
+  CK(cudaMemcpyAsync(h->st_vals + (size_t)s * h->cfg.max_batch, vals, sizeof(uint64_t) * n, cudaMemcpyHostToDevice,
+                     h->h2d_stream));
+  CK(cudaEventRecord(h->h2d_done[s], h->h2d_stream));
+  CK(cudaStreamWaitEvent(st, h->h2d_done[s], 0));
+  int rc = submit_impl(h, h->st_ops + (size_t)s * h->cfg.max_batch, h->st_keys + (size_t)s * h->cfg.max_batch,
+                       h->st_vals + (size_t)s * h->cfg.max_batch, n, h->st_res + (size_t)s * h->cfg.max_batch, st,
+                       results, ticket);
+  if (rc != EIRENE_OK) return rc;
+  CK(cudaEventRecord(h->comp_done[s], st));
+  h->slot_used[s] = true;
+  return EIRENE_OK;
 }
 
 int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) {
