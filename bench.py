@@ -268,7 +268,7 @@ def run_ours(args):
     per_batch_ms = np.array([ev[b][0].elapsed_time(ev[b][1]) for b in range(args.warmup, nb)])
     if os.environ.get("EIRENE_BENCH_VERBOSE"):
         print("per-batch ms:", " ".join(f"{x:.3f}" for x in per_batch_ms), file=sys.stderr)
-        print("stage ms per batch:", [[round(x, 3) for x in s["stage_ms"][:6]] for s in stats[args.warmup:]][:8],
+        print("stage ms per batch:", [[round(x, 3) for x in s["stage_ms"][:5]] for s in stats[args.warmup:]][:8],
               file=sys.stderr)
     launches = int(sum(s["launches"] for s in stats[args.warmup:]))
     if world > 1:
@@ -283,7 +283,7 @@ def run_ours(args):
     # (graph replay is off while stage events are on, so this region also
     # shows the cost of direct launches).  Its batches reuse the pre-staged
     # input buffers of the first timed batches.
-    stage_names = ["sort", "combine", "partition", "query", "update", "result"]
+    stage_names = ["sort", "group", "query", "update", "result"]
     engine = tree if world == 1 else sh.engine
     engine.set_flags(timing=True)
     n_stage = min(args.steps, 10)
@@ -298,7 +298,7 @@ def run_ours(args):
     sstats = [tree.results(r) for r in srs] if world == 1 else srs
     torch.cuda.synchronize()
     direct_ms = sa.elapsed_time(sz) / n_stage
-    stage_ms = np.array([s["stage_ms"][:6] for s in sstats]).mean(axis=0)
+    stage_ms = np.array([s["stage_ms"][:5] for s in sstats]).mean(axis=0)
     engine.set_flags(timing=False)
 
     # ------------------------------------------------------------ e2e through the public API (host buffers)
@@ -357,13 +357,20 @@ def run_ours(args):
         if stage_names[dom] == "query" or args.roofline_kernel == "query":
             ab = [algorithmic_bytes_query(wl.keys, *host_batches[b][:2], 16)["bytes"] for b in range(args.warmup, min(nb, args.warmup + 4))]
             bytes_per = float(np.mean(ab))
-            ms = stage_ms[3]
+            ms = stage_ms[2]
             kern = "query_kernel"
+        elif stage_names[dom] == "group":
+            # bucket read 12 B + sorted payload 4 B + pinfo 4 B per request; one issued entry per key
+            o0, k0 = host_batches[args.warmup][:2]
+            d = len(np.unique(k0))
+            bytes_per = batch_n * 20 + d * 17
+            ms = stage_ms[1]
+            kern = "group_kernel"
         else:
-            # sort stage: 1 upsweep (8+1+8 B/req read) + 8 passes x (12 B read + 12 B write) per request
-            bytes_per = batch_n * (17 + 8 * 24)
+            # bucket scatter: key 8 B + op 1 B read, 12 B written per request (+ hist pass 8 B)
+            bytes_per = batch_n * (8 + 9 + 12)
             ms = stage_ms[0]
-            kern = "sort (upsweep + 8 x sort_pass_kernel)"
+            kern = "bsort_hist_kernel + bsort_scatter_kernel"
         ach = bytes_per / (ms * 1e-3) / 1e9
         roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": ach / peaks["hbm_gbs"], "traffic": None, "kernel": kern,

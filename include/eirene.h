@@ -98,8 +98,9 @@ typedef struct {
   uint64_t new_leaves, new_inner;
   uint32_t height;            /* tree height after the batch (1 = root is a leaf)              */
   uint32_t launches;          /* kernels launched for this batch                               */
-  float stage_ms[8];          /* EIRENE_F_TIMING: sort, combine, partition, query, update,
-                                 result, (unused), total                                       */
+  float stage_ms[8];          /* EIRENE_F_TIMING: [0] sort (bucket scatter), [1] group (bucket
+                                 sort + combine + partition), [2] query, [3] update, [4] result,
+                                 [5], [6] unused, [7] total                                    */
 } eirene_batch_stats;
 
 /* Creates a tree (one empty leaf) on cfg->device and allocates every pool and

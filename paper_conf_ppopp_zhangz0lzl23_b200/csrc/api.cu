@@ -22,7 +22,7 @@ using namespace eirene;
 namespace {
 
 constexpr int RING = 64;
-constexpr int NSTAGE = 7;
+constexpr int NSTAGE = 6;   // events: before sort, after sort / group / query / update / result
 
 std::mutex g_err_mu;
 std::string g_last_cuda_error = "no error";
@@ -83,8 +83,8 @@ __global__ void set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64
   }
 }
 
-// kernels in one batch graph: set_args, 4 sort, combine, partition, query, update, result_long, finalize
-constexpr int GRAPH_KERNELS = 11;
+// kernels in one batch graph: set_args, 2 sort, group, query, update, result_long, finalize
+constexpr int GRAPH_KERNELS = 8;
 constexpr int MAX_GRAPHS = 8;
 
 struct GraphEntry {
@@ -217,7 +217,6 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   t.leaf_cap = (uint32_t)leaf_cap;
   t.inner_cap = (uint32_t)inner_cap;
   const size_t sort_tiles = (nb + SORT_TILE - 1) / SORT_TILE;
-  const size_t comb_tiles = (nb + COMB_TILE - 1) / COMB_TILE;
 #define AL(p, n)                                 \
   if (e == cudaSuccess) e = h->dalloc(&(p), (n));
   AL(t.lkeys, leaf_cap * FAN);
@@ -233,9 +232,6 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->sb.pB, nb);
   AL(h->sb.lookback, sort_tiles * 256);
   AL(h->cb.pinfo, nb);
-  AL(h->cb.ikey, nb);
-  AL(h->cb.iop, nb);
-  AL(h->cb.ival, nb);
   AL(h->cb.qkey, nb);
   AL(h->cb.qseg, nb);
   AL(h->cb.wkey, nb);
@@ -263,7 +259,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->route_lb, ((nb + 2047) / 2048) * 64);
   AL(h->route_ctr, 1);
   AL(h->bs.bstart, 4097);
-  AL(h->bs.cursor, 4096);
+  AL(h->bs.cursor, BSORT_CTR_WORDS);
   AL(h->dargs, 1);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
@@ -276,9 +272,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     };
     const size_t o_ctl = bump(sizeof(BatchCtl));
     const size_t o_gh = bump(sizeof(uint32_t) * 8 * 256);
-    const size_t o_bc = bump(sizeof(uint32_t) * 4096);
-    const size_t o_cs = bump(sizeof(unsigned long long) * comb_tiles);
-    const size_t o_ps = bump(sizeof(unsigned long long) * comb_tiles);
+    const size_t o_bc = bump(sizeof(uint32_t) * BSORT_CTR_WORDS);
+    const size_t o_gs = bump(sizeof(unsigned long long) * GROUP_STATUS_WORDS);
     h->zero_bytes = off;
     AL(h->zero_region, off);
     if (e == cudaSuccess) {
@@ -289,8 +284,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
       h->bs.pA = h->sb.pA;
       h->bs.kB = h->sb.kB;
       h->bs.pB = h->sb.pB;
-      h->cb.comb_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_cs);
-      h->cb.part_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_ps);
+      h->cb.group_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_gs);
     }
   }
 #undef AL
@@ -411,27 +405,23 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     if (timing) rec(0, s);
     cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, s);
     launch_bucket_sort(h->dargs, n, h->cfg.key_lo, h->cfg.key_hi, h->bs, ctl, h->num_sms, s, &launches);
-    const uint64_t* skey = h->bs.kB;
-    const uint32_t* spay = h->bs.pB;
     stage("sort");
     if (timing) rec(1, s);
-    launch_combine(skey, spay, h->dargs, n, h->cb, ctl, s, &launches);
-    stage("combine");
+    launch_group(h->dargs, n, h->bs, h->cb, h->t, ctl, s, &launches);
+    const uint32_t* spay = h->bs.pB;
+    stage("group");
     if (timing) rec(2, s);
-    launch_partition(n, h->cb, h->t, ctl, s, &launches);
-    stage("partition");
-    if (timing) rec(3, s);
     launch_query(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, s, &launches);
     stage("query");
-    if (timing) rec(4, s);
+    if (timing) rec(3, s);
     launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
     stage("update");
-    if (timing) rec(5, s);
+    if (timing) rec(4, s);
     launch_result(spay, n, h->cb, h->dargs, ctl, s, &launches);
     stage("result");
     finalize_kernel<<<1, 32, 0, s>>>(ctl, h->t.hdr, dbg ? 1 : 0);
     ++launches;
-    if (timing) rec(6, s);
+    if (timing) rec(5, s);
     return cudaGetLastError();
   };
   if (dbg || r.timing || !h->use_graphs) {   // per-stage events: direct launches

@@ -97,7 +97,7 @@ struct BatchArgs {
 };
 
 // tile counters
-enum { TC_SORT0 = 0, TC_COMB = 8, TC_PART = 9, TC_ROUTE = 10, TC_SCAN = 11 };
+enum { TC_SORT0 = 0, TC_GROUP = 8, TC_ROUTE = 10, TC_SCAN = 11, TC_HIST = 12 };
 
 struct Tree {
   uint64_t* lkeys;
@@ -188,26 +188,24 @@ void launch_sort(const uint64_t* keys, const uint8_t* ops, const uint32_t* pay_i
 size_t sort_lookback_words(uint32_t max_n);
 
 // Batch request sort (bsort.cu): bucket by the top bits, sort buckets in smem.
+constexpr int BSORT_CTR_WORDS = 8192;
 struct BSortBufs {
   uint64_t* kA;      // [n] bucketed (unordered within a bucket)
   uint32_t* pA;
   uint64_t* kB;      // [n] sorted output
   uint32_t* pB;
-  uint32_t* bcount;  // [4096] zeroed per batch
+  uint32_t* bcount;  // [BSORT_CTR_WORDS] zeroed per batch (bucket b at b << bsh)
   uint32_t* bstart;  // [4097]
-  uint32_t* cursor;  // [4096]
+  uint32_t* cursor;  // [BSORT_CTR_WORDS] (bucket b at b << bsh)
 };
 int bsort_bits(uint32_t n);
+int bsort_ctr_shift(int bb);
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
                         BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches);
 
 struct CombBufs {
   uint32_t* pinfo;            // [n] seg | DONE
-  uint64_t* ikey;             // [n] issued key per segment
-  uint8_t* iop;               // [n]
-  uint64_t* ival;             // [n]
-  unsigned long long* comb_status;  // [tiles]  (zeroed per batch)
-  unsigned long long* part_status;  // [tiles]  (zeroed per batch)
+  unsigned long long* group_status;  // [GROUP_STATUS_WORDS] bucket look-back words (zeroed per batch)
   uint64_t* qkey;
   uint32_t* qseg;
   uint64_t* wkey;
@@ -221,13 +219,11 @@ struct CombBufs {
   uint32_t* longseg;          // [n] segments longer than SHORT_SEG, finished by result_long_kernel
 };
 constexpr uint32_t SHORT_SEG = 32;
-constexpr int COMB_THREADS = 256;
-constexpr int COMB_ITEMS = 8;
-constexpr int COMB_TILE = COMB_THREADS * COMB_ITEMS;
+constexpr int GROUP_STATUS_WORDS = 4096;   // >= 2^bsort_bits(n) for every n
 
-void launch_combine(const uint64_t* skey, const uint32_t* spay, const BatchArgs* A,
-                    uint32_t n, const CombBufs& c, BatchCtl* ctl, cudaStream_t st, int* launches);
-void launch_partition(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, cudaStream_t st, int* launches);
+// bucket finish (sort in smem) + combine + partition, one CTA per bucket (group.cu)
+void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
+                  cudaStream_t st, int* launches);
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches);
 

@@ -5,7 +5,7 @@
 // quiescent (the update kernel of the previous batch has finished, and this
 // batch's update kernel runs after this one).  Each thread owns
 // one issued request; the issued list is key-sorted, so the 32 lanes of a warp
-// walk overlapping root-to-leaf paths and their 128-bit loads of shared upper
+// walk overlapping root-to-leaf paths and their 256-bit loads of shared upper
 // nodes coalesce into one L1/L2 request per distinct node (the B200 analogue
 // of Harmonia's path sharing / NTG).  Inner levels (<= 18 MB at
 // 2^24 keys) stay L2-resident across batches; leaves (256 MiB) come from HBM:
@@ -27,36 +27,11 @@ namespace eirene {
 
 namespace {
 
-// Count of separators <= k in a 16-key node line (key[c-1..15] == KEY_MAX,
-// and k < KEY_MAX, so the count is the child index).
-__device__ __forceinline__ uint32_t route16(const uint64_t* __restrict__ line, uint64_t k) {
-  const ulonglong2* l2 = reinterpret_cast<const ulonglong2*>(line);
-  ulonglong2 v[8];
-#pragma unroll
-  for (int i = 0; i < 8; ++i) v[i] = __ldg(l2 + i);
-  uint32_t c = 0;
-#pragma unroll
-  for (int i = 0; i < 8; ++i) c += (v[i].x <= k) + (v[i].y <= k);
-  return c;
-}
-
-struct uint4x2 {
-  uint4 a, b;
-};
 __device__ __forceinline__ ulonglong4 ldg256(const uint64_t* p) {
   ulonglong4 v;
   asm volatile("ld.global.nc.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p));
   return v;
 }
-__device__ __forceinline__ uint4x2 ldg256u32(const uint32_t* p) {
-  uint4x2 v;
-  asm volatile("ld.global.nc.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
-               : "=r"(v.a.x), "=r"(v.a.y), "=r"(v.a.z), "=r"(v.a.w), "=r"(v.b.x), "=r"(v.b.y), "=r"(v.b.z),
-                 "=r"(v.b.w)
-               : "l"(p));
-  return v;
-}
-
 // Slot of key k in a 16-key leaf line (4 x 256-bit loads), -1 if absent.
 __device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_t k) {
   ulonglong4 v[4];
@@ -73,15 +48,16 @@ __device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_
   return s;
 }
 
-__global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__ qkey,
-                                                     const uint32_t* __restrict__ qseg,
-                                                     const uint64_t* __restrict__ wkey, const uint32_t* __restrict__ wseg,
-                                                     uint32_t* __restrict__ wleaf, uint8_t* __restrict__ wslot,
-                                                     uint64_t* __restrict__ old, const uint32_t* __restrict__ spay,
-                                                     const uint32_t* __restrict__ pinfo,
-                                                     const uint32_t* __restrict__ istart, uint32_t* __restrict__ longseg,
-                                                     const BatchArgs* __restrict__ A, Tree t,
-                                                     BatchCtl* __restrict__ ctl) {
+__global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restrict__ qkey,
+                                                        const uint32_t* __restrict__ qseg,
+                                                        const uint64_t* __restrict__ wkey,
+                                                        const uint32_t* __restrict__ wseg, uint32_t* __restrict__ wleaf,
+                                                        uint8_t* __restrict__ wslot, uint64_t* __restrict__ old,
+                                                        const uint32_t* __restrict__ spay,
+                                                        const uint32_t* __restrict__ pinfo,
+                                                        const uint32_t* __restrict__ istart,
+                                                        uint32_t* __restrict__ longseg, const BatchArgs* __restrict__ A,
+                                                        Tree t, BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
@@ -93,11 +69,10 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
     const uint64_t k = isq ? qkey[i] : wkey[i - nq];
     uint32_t node = root;
     for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
-      // key line and child line are loaded together (12 independent 16-byte
-      // loads), so a level costs one memory round trip instead of two
-      // sm_100 256-bit loads (LDG.E.ENL2.256): a 128 B key line is 4 loads;
-      // then the one child pointer (loading the whole child line speculatively
-      // measured slower: it doubles L1 traffic per level)
+      // a 128 B separator line is four 256-bit loads (LDG.E.ENL2.256), then
+      // the one child pointer: loading the whole child line alongside the keys
+      // (one round trip per level instead of two) measured slower, as did two
+      // or four interleaved traversals per thread (tools/ab.py)
       const uint64_t* kl = t.ikeys + (size_t)node * FAN;
       ulonglong4 kv[4];
 #pragma unroll
@@ -133,14 +108,46 @@ __global__ void __launch_bounds__(256) query_kernel(const uint64_t* __restrict__
   }
 }
 
+// RESULT_CAL is fused into the query kernel: every issued request scatters
+// the value it retrieved to the pending positions of its own segment.  The
+// segments longer than SHORT_SEG (hot keys) are queued instead and finished
+// here with one CTA per segment, so a 56K-request Zipf key does not serialise
+// one thread.
+__global__ void __launch_bounds__(256) result_long_kernel(const uint32_t* __restrict__ spay,
+                                                           const uint32_t* __restrict__ pinfo,
+                                                           const uint32_t* __restrict__ istart,
+                                                           const uint32_t* __restrict__ longseg,
+                                                           const uint64_t* __restrict__ old,
+                                                           const BatchArgs* __restrict__ A,
+                                                           const BatchCtl* __restrict__ ctl) {
+  if (ctl->invalid || ctl->status != 0) return;
+  uint64_t* __restrict__ results = A->results;
+  const uint32_t nl = ctl->nlong;
+  for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
+    const uint32_t s = longseg[x];
+    const uint64_t v = old[s];
+    const uint32_t e = istart[s + 1];
+    for (uint32_t p = istart[s] + threadIdx.x; p < e; p += blockDim.x)
+      if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
+  }
+}
+
 }  // namespace
 
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches) {
+  // one resident wave: 8 CTAs of 256 threads per SM at <= 32 registers
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
   query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wleaf, c.wslot, c.old, spay, c.pinfo,
                                        c.istart, c.longseg, A, t, ctl);
+  ++*launches;
+}
+
+void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
+                   cudaStream_t st, int* launches) {
+  (void)n;
+  result_long_kernel<<<148, 256, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, A, ctl);
   ++*launches;
 }
 
