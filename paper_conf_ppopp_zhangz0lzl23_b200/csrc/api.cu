@@ -258,8 +258,9 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   }
   AL(h->route_lb, ((nb + 2047) / 2048) * 64);
   AL(h->route_ctr, 1);
-  AL(h->bs.bstart, 4097);
-  AL(h->bs.cursor, BSORT_CTR_WORDS);
+  AL(h->bs.gstart, NBINS + 1);
+  AL(h->bs.bin2grp, NBINS);
+  AL(h->bs.cursor, NBINS);
   AL(h->dargs, 1);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
@@ -272,7 +273,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     };
     const size_t o_ctl = bump(sizeof(BatchCtl));
     const size_t o_gh = bump(sizeof(uint32_t) * 8 * 256);
-    const size_t o_bc = bump(sizeof(uint32_t) * BSORT_CTR_WORDS);
+    const size_t o_bc = bump(sizeof(uint32_t) * NBINS);
     const size_t o_gs = bump(sizeof(unsigned long long) * GROUP_STATUS_WORDS);
     h->zero_bytes = off;
     AL(h->zero_region, off);
@@ -407,7 +408,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     launch_bucket_sort(h->dargs, n, h->cfg.key_lo, h->cfg.key_hi, h->bs, ctl, h->num_sms, s, &launches);
     stage("sort");
     if (timing) rec(1, s);
-    launch_group(h->dargs, n, h->bs, h->cb, h->t, ctl, s, &launches);
+    launch_group(h->dargs, n, h->bs, h->cb, h->t, ctl, h->num_sms, s, &launches);
     const uint32_t* spay = h->bs.pB;
     stage("group");
     if (timing) rec(2, s);

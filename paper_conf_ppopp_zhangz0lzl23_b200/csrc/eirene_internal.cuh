@@ -188,18 +188,19 @@ void launch_sort(const uint64_t* keys, const uint8_t* ops, const uint32_t* pay_i
 size_t sort_lookback_words(uint32_t max_n);
 
 // Batch request sort (bsort.cu): bucket by the top bits, sort buckets in smem.
-constexpr int BSORT_CTR_WORDS = 8192;
+constexpr int BIN_BITS = 12;                  // bucket-sort bins = top key bits
+constexpr int NBINS = 1 << BIN_BITS;
 struct BSortBufs {
-  uint64_t* kA;      // [n] bucketed (unordered within a bucket)
+  uint64_t* kA;      // [n] grouped (unordered inside a group)
   uint32_t* pA;
-  uint64_t* kB;      // [n] sorted output
-  uint32_t* pB;
-  uint32_t* bcount;  // [BSORT_CTR_WORDS] zeroed per batch (bucket b at b << bsh)
-  uint32_t* bstart;  // [4097]
-  uint32_t* cursor;  // [BSORT_CTR_WORDS] (bucket b at b << bsh)
+  uint64_t* kB;      // [n] scratch for oversized groups
+  uint32_t* pB;      // [n] sorted payloads (output)
+  uint32_t* bcount;  // [NBINS] zeroed per batch
+  uint16_t* bin2grp; // [NBINS]
+  uint32_t* gstart;  // [NBINS + 1] group starts
+  uint32_t* cursor;  // [NBINS] group fill cursors
 };
-int bsort_bits(uint32_t n);
-int bsort_ctr_shift(int bb);
+uint32_t bsort_groups(uint32_t n, int num_sms);
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
                         BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches);
 
@@ -219,11 +220,11 @@ struct CombBufs {
   uint32_t* longseg;          // [n] segments longer than SHORT_SEG, finished by result_long_kernel
 };
 constexpr uint32_t SHORT_SEG = 32;
-constexpr int GROUP_STATUS_WORDS = 4096;   // >= 2^bsort_bits(n) for every n
+constexpr int GROUP_STATUS_WORDS = NBINS;   // >= bsort_groups(n) for every n
 
 // bucket finish (sort in smem) + combine + partition, one CTA per bucket (group.cu)
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
-                  cudaStream_t st, int* launches);
+                  int num_sms, cudaStream_t st, int* launches);
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches);
 

@@ -32,14 +32,15 @@
 // rounds with a carry; a round-walk is repeated after the look-back to emit.
 #include "eirene_internal.cuh"
 
+
 namespace eirene {
 
 namespace {
 
 constexpr int G_THREADS = 512;
 constexpr int G_WARPS = G_THREADS / 32;
-constexpr int G_ITEMS = 12;
-constexpr int G_CAP = G_THREADS * G_ITEMS;    // 6144 positions sorted in smem
+constexpr int G_ITEMS = 8;
+constexpr int G_CAP = G_THREADS * G_ITEMS;    // 4096 positions sorted in smem
 constexpr int SB_BITS = 12;                   // sub-bucket bits inside a bucket
 constexpr int SB_N = 1 << SB_BITS;
 
@@ -50,10 +51,14 @@ constexpr unsigned long long F_VAL = (1ull << 62) - 1;
 struct GSmem {
   uint64_t k[G_CAP];
   uint32_t p[G_CAP];
-  uint32_t sb[SB_N + 1];
+  uint32_t sb[SB_N + 1];       // sub-bucket starts; per-warp digit counters of the L2 passes
+  uint32_t whist[64 * G_WARPS];  // [digit][warp] counters of the stable smem passes
   uint32_t wsum[G_WARPS];
-  uint32_t hist[256];
-  uint32_t off[256];
+  unsigned long long wmin[G_WARPS], wmax[G_WARPS];
+  uint32_t wcmax[G_WARPS];
+  uint64_t kmin, kmax;
+  uint32_t cmax;
+  uint32_t dhist[256];         // digit counts / running offsets of the L2 passes
   // per-warp aggregates and exclusive carries of the current round
   uint32_t w_nh[G_WARPS], w_lw[G_WARPS], w_nw[G_WARPS];
   uint32_t c_nh[G_WARPS], c_lw[G_WARPS], c_nw[G_WARPS];
@@ -66,108 +71,106 @@ __device__ __forceinline__ bool kp_less(uint64_t ka, uint32_t pa, uint64_t kb, u
 }
 __device__ __forceinline__ uint32_t lanemask_le() { return lanemask_lt() | (1u << lane_id()); }
 
-// Stable LSD pass over [0, cnt) of (ks, ps) -> (kd, pd) by an 8-bit digit, by
-// one CTA walking the bucket in G_THREADS-sized tiles; warps of a tile take
-// their offsets in warp order, lanes in lane order, so the pass is stable.
-template <class DigitFn>
-__device__ void cta_lsd_pass(const uint64_t* ks, const uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt,
-                             DigitFn dig, GSmem& S) {
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  if (tid < 256) S.hist[tid] = 0;
-  __syncthreads();
-  for (uint32_t i = tid; i < cnt; i += G_THREADS) atomicAdd(&S.hist[dig(ks[i], ps[i])], 1u);
-  __syncthreads();
-  if (tid == 0) {
-    uint32_t r = 0;
-    for (int d = 0; d < 256; ++d) {
-      S.off[d] = r;
-      r += S.hist[d];
-    }
+// Block-wide min / max of the group's keys -> S.kmin, S.kmax.
+__device__ void key_range(uint64_t mn, uint64_t mx, GSmem& S) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    mn = min(mn, (uint64_t)__shfl_xor_sync(FULL, mn, o));
+    mx = max(mx, (uint64_t)__shfl_xor_sync(FULL, mx, o));
+  }
+  if (lane == 0) {
+    S.wmin[warp] = mn;
+    S.wmax[warp] = mx;
   }
   __syncthreads();
-  for (uint32_t base = 0; base < cnt; base += G_THREADS) {
-    const uint32_t i = base + tid;
-    const bool act = i < cnt;
-    const uint64_t k = act ? ks[i] : 0;
-    const uint32_t p = act ? ps[i] : 0;
-    const uint32_t d = act ? dig(k, p) : 256u;
-    const uint32_t peers = __match_any_sync(FULL, d);
-    uint32_t before = 0;
-    for (int w = 0; w < G_WARPS; ++w) {
-      if (warp == w && act) before = S.off[d];
-      __syncthreads();
-      if (warp == w && act && lane == 31 - __clz(peers)) S.off[d] += __popc(peers);
-      __syncthreads();
+  if (threadIdx.x == 0) {
+    uint64_t a = S.wmin[0], z = S.wmax[0];
+    for (int w = 1; w < G_WARPS; ++w) {
+      a = min(a, (uint64_t)S.wmin[w]);
+      z = max(z, (uint64_t)S.wmax[w]);
     }
-    if (act) {
-      const uint32_t pos = before + __popc(peers & lanemask_lt());
-      kd[pos] = k;
-      pd[pos] = p;
-    }
+    S.kmin = a;
+    S.kmax = z;
   }
   __syncthreads();
 }
 
-// Sort a bucket of cnt <= G_CAP requests into S.k / S.p: sub-bucket by the
-// next SB_BITS key bits (smem atomics + block scan + scatter), then finish
-// each sub-bucket (~1 request on average) by insertion sort on (key, payload).
-__device__ void smem_sort(const uint64_t* __restrict__ ks, const uint32_t* __restrict__ ps, uint32_t cnt, int sb_shift,
-                          GSmem& S) {
-  const int tid = threadIdx.x;
-  for (int i = tid; i <= SB_N; i += G_THREADS) S.sb[i] = 0;
+// Exclusive scan, in place, of the 1024 [digit][warp] counters (2 per thread).
+__device__ void scan_whist(GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t a = S.whist[2 * tid], b = S.whist[2 * tid + 1];
+  uint32_t x = a + b;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) S.wsum[warp] = x;
   __syncthreads();
+  uint32_t run = x - a - b;
+  for (int w = 0; w < warp; ++w) run += S.wsum[w];
+  S.whist[2 * tid] = run;
+  S.whist[2 * tid + 1] = run + a;
+  __syncthreads();
+}
+
+// Slow path of smem_sort, items parked in S.k / S.p: stable LSD passes,
+// ceil(tsbits / 6) on the timestamp, then (unless the group is one key) 2 on
+// the sub-bucket index, then insertion sort of each sub-bucket (S.sb holds
+// the sub-bucket starts).  Kept out of line so the fast path keeps its
+// registers.
+__device__ __noinline__ void slow_sort(uint32_t cnt, int tsbits, uint64_t kmin, int shift, bool multi, GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t C = 32u * ((cnt + G_THREADS - 1) / G_THREADS);
+  const uint32_t wb = warp * C;
   uint64_t kr[G_ITEMS];
-  uint32_t r[G_ITEMS];
+  uint32_t pr[G_ITEMS], r[G_ITEMS];
+  const int tpass = (tsbits + 5) / 6;
+  const int npass = tpass + (multi ? 2 : 0);
+  for (int pass = 0; pass < npass; ++pass) {
+    const bool ts = pass < tpass;
+    const int dsh = 6 * (ts ? pass : pass - tpass);
 #pragma unroll
-  for (int j = 0; j < G_ITEMS; ++j) {
-    const uint32_t i = tid + j * G_THREADS;
-    kr[j] = i < cnt ? ks[i] : 0;
-  }
-#pragma unroll
-  for (int j = 0; j < G_ITEMS; ++j) {
-    const uint32_t i = tid + j * G_THREADS;
-    r[j] = i < cnt ? atomicAdd(&S.sb[(uint32_t)(kr[j] >> sb_shift) & (SB_N - 1)], 1u) : 0u;
-  }
-  __syncthreads();
-  {   // exclusive scan of S.sb[0..SB_N) (8 per thread)
-    constexpr int PER = SB_N / G_THREADS;
-    uint32_t loc[PER], s = 0;
-#pragma unroll
-    for (int j = 0; j < PER; ++j) {
-      loc[j] = S.sb[tid * PER + j];
-      s += loc[j];
+    for (int j = 0; j < G_ITEMS; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      if (32u * j < C && i < cnt) {
+        kr[j] = S.k[i];
+        pr[j] = S.p[i];
+      }
     }
-    const int lane = tid & 31, warp = tid >> 5;
-    uint32_t x = s;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL, x, o);
-      if (lane >= o) x += y;
-    }
-    if (lane == 31) S.wsum[warp] = x;
+    for (int i = tid; i < 64 * G_WARPS; i += G_THREADS) S.whist[i] = 0;
     __syncthreads();
-    uint32_t run = x - s;
-    for (int w = 0; w < warp; ++w) run += S.wsum[w];
 #pragma unroll
-    for (int j = 0; j < PER; ++j) {
-      S.sb[tid * PER + j] = run;
-      run += loc[j];
+    for (int j = 0; j < G_ITEMS; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      const bool v = 32u * j < C && i < cnt;
+      const uint32_t src = ts ? (pr[j] >> 2) : (uint32_t)((kr[j] - kmin) >> shift);
+      const uint32_t d = v ? (src >> dsh) & 63u : 64u;
+      const uint32_t peers = __match_any_sync(FULL, d);
+      const uint32_t base = v ? S.whist[d * G_WARPS + warp] : 0u;
+      r[j] = base + __popc(peers & lanemask_lt());
+      __syncwarp();
+      if (v && lane == 31 - __clz(peers)) S.whist[d * G_WARPS + warp] = base + __popc(peers);
+      __syncwarp();
     }
-    if (tid == 0) S.sb[SB_N] = cnt;
-  }
-  __syncthreads();
+    __syncthreads();
+    scan_whist(S);
 #pragma unroll
-  for (int j = 0; j < G_ITEMS; ++j) {
-    const uint32_t i = tid + j * G_THREADS;
-    if (i < cnt) {
-      const uint32_t pos = S.sb[(uint32_t)(kr[j] >> sb_shift) & (SB_N - 1)] + r[j];
-      S.k[pos] = kr[j];
-      S.p[pos] = ps[i];
+    for (int j = 0; j < G_ITEMS; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      if (32u * j < C && i < cnt) {
+        const uint32_t src = ts ? (pr[j] >> 2) : (uint32_t)((kr[j] - kmin) >> shift);
+        const uint32_t pos = S.whist[((src >> dsh) & 63u) * G_WARPS + warp] + r[j];
+        S.k[pos] = kr[j];
+        S.p[pos] = pr[j];
+      }
     }
+    __syncthreads();
   }
-  __syncthreads();
-  for (int s = tid; s < SB_N; s += G_THREADS) {
-    const uint32_t lo = S.sb[s], hi = S.sb[s + 1];
+  if (!multi) return;   // one key: timestamp order is final
+  for (int sb = tid; sb < SB_N; sb += G_THREADS) {
+    const uint32_t lo = S.sb[sb], hi = S.sb[sb + 1];
     for (uint32_t a = lo + 1; a < hi; ++a) {
       const uint64_t k = S.k[a];
       const uint32_t p = S.p[a];
@@ -184,35 +187,233 @@ __device__ void smem_sort(const uint64_t* __restrict__ ks, const uint32_t* __res
   __syncthreads();
 }
 
-// Oversized bucket: stable LSD in L2 on the payload (4 x 8 bits) and then the
-// key bits below the bucket prefix; an odd number of passes ends in (kd, pd).
-__device__ void l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int bb, GSmem& S) {
-  const int tid = threadIdx.x;
-  const int key_passes = (64 - bb + 7) / 8;
-  const int total = 4 + key_passes;
-  uint64_t* k0 = ks;
-  uint32_t* p0 = ps;
-  uint64_t* k1 = kd;
-  uint32_t* p1 = pd;
-  if ((total & 1) == 0) {   // make the count odd with a copy pass into (kd, pd) first
-    for (uint32_t i = tid; i < cnt; i += G_THREADS) {
-      kd[i] = ks[i];
-      pd[i] = ps[i];
+// Sort a group of 2 <= cnt <= G_CAP requests (in no particular order) into
+// S.k / S.p by (key, payload).  Items live in registers in warp-contiguous
+// order (position = warp * C + 32 j + lane).  Sub-bucket index =
+// (key - kmin) >> shift, SB_BITS wide, so sub-buckets adapt to the group's key
+// range.  Uniform keys (every sub-bucket <= FAST_SB): scatter by smem-atomic
+// rank.  Otherwise (hot / clustered keys): stable 6-bit counting passes, first
+// on the timestamp bits, then on the sub-bucket index, leave every sub-bucket
+// in timestamp order.  Either way each sub-bucket is finished by insertion
+// sort on (key, payload), whose cost is its number of inversions -- for a hot
+// key in timestamp order, only those against the few other keys beside it.
+// One key in the whole group: the timestamp passes alone finish it.
+constexpr uint32_t FAST_SB = 32;
+__device__ void smem_sort(const uint64_t* __restrict__ ks, const uint32_t* __restrict__ ps, uint32_t cnt, int tsbits,
+                          GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t C = 32u * ((cnt + G_THREADS - 1) / G_THREADS);
+  const uint32_t wb = warp * C;
+  uint64_t kr[G_ITEMS];
+  uint32_t pr[G_ITEMS], r[G_ITEMS];
+  uint64_t mn = KEY_MAX, mx = 0;
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = wb + 32 * j + lane;
+    const bool v = 32u * j < C && i < cnt;
+    kr[j] = v ? ks[i] : 0;
+    pr[j] = v ? ps[i] : 0;
+    if (v) {
+      mn = min(mn, kr[j]);
+      mx = max(mx, kr[j]);
+    }
+  }
+  for (int i = tid; i <= SB_N; i += G_THREADS) S.sb[i] = 0;
+  key_range(mn, mx, S);   // (its barriers also order the sb zeroing)
+  const uint64_t kmin = S.kmin, range = S.kmax - S.kmin;
+  const int bits = 64 - __clzll((long long)range);
+  const int shift = bits > SB_BITS ? bits - SB_BITS : 0;
+  uint32_t cm = 0;
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = wb + 32 * j + lane;
+    r[j] = 0;
+    if (range != 0 && 32u * j < C && i < cnt) {   // (one key: no sub-buckets, no hot-spot atomics)
+      r[j] = atomicAdd(&S.sb[(uint32_t)((kr[j] - kmin) >> shift)], 1u);
+      cm = max(cm, r[j] + 1);
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) cm = max(cm, __shfl_xor_sync(FULL, cm, o));
+  if (lane == 0) S.wcmax[warp] = cm;
+  __syncthreads();
+  if (tid == 0) {
+    uint32_t c = 0;
+    for (int w = 0; w < G_WARPS; ++w) c = max(c, S.wcmax[w]);
+    S.cmax = c;
+  }
+  {   // exclusive scan of S.sb[0..SB_N) (8 per thread)
+    constexpr int PER = SB_N / G_THREADS;
+    uint32_t loc[PER], sum = 0;
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+      loc[j] = S.sb[tid * PER + j];
+      sum += loc[j];
+    }
+    uint32_t x = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, x, o);
+      if (lane >= o) x += y;
+    }
+    if (lane == 31) S.wsum[warp] = x;
+    __syncthreads();
+    uint32_t run = x - sum;
+    for (int w = 0; w < warp; ++w) run += S.wsum[w];
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+      S.sb[tid * PER + j] = run;
+      run += loc[j];
+    }
+    if (tid == 0) S.sb[SB_N] = cnt;
+  }
+  __syncthreads();
+  if (range != 0 && S.cmax <= FAST_SB) {
+    // scatter by atomic rank, then every request takes its final position:
+    // sub-bucket start + number of (key, payload) smaller in its sub-bucket
+#pragma unroll
+    for (int j = 0; j < G_ITEMS; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      if (32u * j < C && i < cnt) {
+        const uint32_t pos = S.sb[(uint32_t)((kr[j] - kmin) >> shift)] + r[j];
+        S.k[pos] = kr[j];
+        S.p[pos] = pr[j];
+      }
     }
     __syncthreads();
-    k0 = kd; p0 = pd; k1 = ks; p1 = ps;
-  }
-  for (int pass = 0; pass < total; ++pass) {
-    if (pass < 4) {
-      const int sh = pass * 8;
-      cta_lsd_pass(k0, p0, k1, p1, cnt, [sh](uint64_t, uint32_t p) { return (p >> sh) & 0xFFu; }, S);
-    } else {
-      const int sh = (pass - 4) * 8;
-      cta_lsd_pass(k0, p0, k1, p1, cnt, [sh](uint64_t k, uint32_t) { return (uint32_t)(k >> sh) & 0xFFu; }, S);
+#pragma unroll
+    for (int j = 0; j < G_ITEMS; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      if (32u * j < C && i < cnt) {
+        const uint32_t x = (uint32_t)((kr[j] - kmin) >> shift);
+        const uint32_t lo = S.sb[x], hi = S.sb[x + 1];
+        uint32_t less = 0;
+        for (uint32_t m = lo; m < hi; ++m) less += kp_less(S.k[m], S.p[m], kr[j], pr[j]);
+        r[j] = lo + less;
+      }
     }
-    uint64_t* tk = k0; k0 = k1; k1 = tk;
-    uint32_t* tp = p0; p0 = p1; p1 = tp;
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < G_ITEMS; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      if (32u * j < C && i < cnt) {
+        S.k[r[j]] = kr[j];
+        S.p[r[j]] = pr[j];
+      }
+    }
+    __syncthreads();
+    return;
   }
+  // slow path (hot / clustered keys): park the items in position order
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = wb + 32 * j + lane;
+    if (32u * j < C && i < cnt) {
+      S.k[i] = kr[j];
+      S.p[i] = pr[j];
+    }
+  }
+  __syncthreads();
+  slow_sort(cnt, tsbits, kmin, shift, range != 0, S);
+}
+
+// One stable LSD pass in L2 over [0, cnt) of (ks, ps) -> (kd, pd) by an 8-bit
+// digit -- of the timestamp (ts) or of key - kmin: digit counts, then tiles of
+// G_THREADS * 8 requests ranked by match_any and per-warp counters
+// (S.sb as [digit][warp]) with running per-digit offsets in S.dhist.
+__device__ __forceinline__ uint32_t l2_digit(uint64_t k, uint32_t p, bool ts, uint64_t kmin, int sh) {
+  return (ts ? (uint32_t)((p >> 2) >> sh) : (uint32_t)((k - kmin) >> sh)) & 255u;
+}
+__device__ void l2_pass(const uint64_t* ks, const uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, bool ts,
+                        uint64_t kmin, int sh, GSmem& S) {
+  constexpr int IT = 8;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid < 256) S.dhist[tid] = 0;
+  __syncthreads();
+  for (uint32_t i = tid; i < cnt; i += G_THREADS) atomicAdd(&S.dhist[l2_digit(ks[i], ps[i], ts, kmin, sh)], 1u);
+  __syncthreads();
+  if (tid == 0) {
+    uint32_t run = 0;
+    for (int d = 0; d < 256; ++d) {
+      const uint32_t c = S.dhist[d];
+      S.dhist[d] = run;
+      run += c;
+    }
+  }
+  __syncthreads();
+  uint32_t* wh = S.sb;   // [256][G_WARPS]
+  for (uint32_t t0 = 0; t0 < cnt; t0 += G_THREADS * IT) {
+    for (int i = tid; i < 256 * G_WARPS; i += G_THREADS) wh[i] = 0;
+    __syncthreads();
+    uint64_t k[IT];
+    uint32_t p[IT], d[IT], r[IT];
+    const uint32_t wb = t0 + warp * 32 * IT;
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      const bool v = i < cnt;
+      k[j] = v ? ks[i] : 0;
+      p[j] = v ? ps[i] : 0;
+      d[j] = v ? l2_digit(k[j], p[j], ts, kmin, sh) : 256u;
+    }
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+      const bool v = d[j] < 256u;
+      const uint32_t peers = __match_any_sync(FULL, d[j]);
+      const uint32_t base = v ? wh[d[j] * G_WARPS + warp] : 0u;
+      r[j] = base + __popc(peers & lanemask_lt());
+      __syncwarp();
+      if (v && lane == 31 - __clz(peers)) wh[d[j] * G_WARPS + warp] = base + __popc(peers);
+      __syncwarp();
+    }
+    __syncthreads();
+    if (tid < 256) {   // per digit: exclusive over warps, tile total
+      uint32_t c = 0;
+#pragma unroll
+      for (int w = 0; w < G_WARPS; ++w) {
+        const uint32_t x = wh[tid * G_WARPS + w];
+        wh[tid * G_WARPS + w] = c + S.dhist[tid];
+        c += x;
+      }
+      S.dhist[tid] += c;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+      if (d[j] < 256u) {
+        const uint32_t pos = wh[d[j] * G_WARPS + warp] + r[j];
+        kd[pos] = k[j];
+        pd[pos] = p[j];
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// Oversized group (cnt > G_CAP, hot keys): stable LSD in L2, first on the
+// timestamp bits, then on the bits of key - kmin (none for a one-key group),
+// ping-pong between the group's two L2 ranges.  Returns the range that holds
+// the result (0: ks/ps, 1: kd/pd).
+__device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int tsbits, GSmem& S) {
+  uint64_t mn = KEY_MAX, mx = 0;
+  for (uint32_t i = threadIdx.x; i < cnt; i += G_THREADS) {
+    const uint64_t k = ks[i];
+    mn = min(mn, k);
+    mx = max(mx, k);
+  }
+  key_range(mn, mx, S);
+  const uint64_t kmin = S.kmin, range = S.kmax - S.kmin;
+  const int tpass = (tsbits + 7) / 8;
+  const int passes = tpass + (range ? (64 - __clzll((long long)range) + 7) / 8 : 0);
+  for (int pass = 0; pass < passes; ++pass) {
+    const bool ts = pass < tpass;
+    const int sh = 8 * (ts ? pass : pass - tpass);
+    if (pass & 1)
+      l2_pass(kd, pd, ks, ps, cnt, ts, kmin, sh, S);
+    else
+      l2_pass(ks, ps, kd, pd, cnt, ts, kmin, sh, S);
+  }
+  return passes & 1;
 }
 
 // Worst-case node demand of the update kernel (EFULL pre-check, SURVEY
@@ -241,10 +442,9 @@ struct GroupArgs {
   uint32_t* pA;
   uint64_t* kB;                 // L2 scratch for oversized buckets
   uint32_t* pB;                 // sorted payloads (output, read by RESULT_CAL)
-  const uint32_t* bcount;
-  const uint32_t* bstart;
-  int bb, bsh;
-  uint32_t n, nb;
+  const uint32_t* gstart;       // [G + 1]
+  uint32_t n, nb;               // requests, groups
+  int tsbits;                   // bits of the largest timestamp (n - 1)
   uint32_t* pinfo;
   uint32_t* istart;
   uint64_t* qkey;
@@ -381,7 +581,7 @@ __device__ void round_emit(const GroupArgs& g, const uint64_t* K, const uint32_t
   }
 }
 
-__global__ void __launch_bounds__(G_THREADS) group_kernel(GroupArgs g) {
+__global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GSmem& S = *reinterpret_cast<GSmem*>(smem_raw);
   BatchCtl* ctl = g.ctl;
@@ -390,19 +590,25 @@ __global__ void __launch_bounds__(G_THREADS) group_kernel(GroupArgs g) {
   if (tid == 0) S.ticket = atomicAdd(&ctl->tile_ctr[TC_GROUP], 1u);
   __syncthreads();
   const uint32_t b = S.ticket;
-  const uint32_t cnt = g.bcount[b << g.bsh];
-  const uint32_t base = g.bstart[b];
+  const uint32_t base = g.gstart[b];
+  const uint32_t cnt = g.gstart[b + 1] - base;
   const bool small = cnt <= (uint32_t)G_CAP;
   const uint64_t* K;
   const uint32_t* P;
   if (small) {
-    if (cnt) smem_sort(g.kA + base, g.pA + base, cnt, 64 - g.bb - SB_BITS, S);
+    if (cnt == 1 && tid == 0) {
+      S.k[0] = g.kA[base];
+      S.p[0] = g.pA[base];
+    } else if (cnt > 1) {
+      smem_sort(g.kA + base, g.pA + base, cnt, g.tsbits, S);
+    }
+    __syncthreads();
     K = S.k;
     P = S.p;
   } else {
-    l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.bb, S);
-    K = g.kB + base;
-    P = g.pB + base;
+    const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S);
+    K = (where ? g.kB : g.kA) + base;
+    P = (where ? g.pB : g.pA) + base;
   }
   // sweep 1: bucket totals (heads, write segments)
   uint32_t c_nh = 0, c_lw = 0, c_nw = 0;
@@ -462,11 +668,12 @@ __global__ void __launch_bounds__(G_THREADS) group_kernel(GroupArgs g) {
   if (small) {
     if (cnt) round_emit(g, K, P, cnt, base, 0, cnt, true, S);
   } else {
+    const bool write_spay = P != g.pB + base;
     c_nh = c_lw = c_nw = 0;
     for (uint32_t r0 = 0; r0 < cnt; r0 += G_CAP) {
       const uint32_t r1 = min(cnt, r0 + (uint32_t)G_CAP);
       round_scan(K, P, cnt, r0, r1, c_nh, c_lw, c_nw, S);
-      round_emit(g, K, P, cnt, base, r0, r1, false, S);
+      round_emit(g, K, P, cnt, base, r0, r1, write_spay, S);
       c_nh = S.r_nh;
       c_lw = S.r_lw;
       c_nw = S.r_nw;
@@ -478,25 +685,22 @@ __global__ void __launch_bounds__(G_THREADS) group_kernel(GroupArgs g) {
 }  // namespace
 
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
-                  cudaStream_t st, int* launches) {
+                  int num_sms, cudaStream_t st, int* launches) {
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(group_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(GSmem));
     attr = true;
   }
-  const int bb = bsort_bits(n);
   GroupArgs g;
   g.A = A;
   g.kA = b.kA;
   g.pA = b.pA;
   g.kB = b.kB;
   g.pB = b.pB;
-  g.bcount = b.bcount;
-  g.bstart = b.bstart;
-  g.bb = bb;
-  g.bsh = bsort_ctr_shift(bb);
+  g.gstart = b.gstart;
   g.n = n;
-  g.nb = 1u << bb;
+  g.nb = bsort_groups(n, num_sms);
+  g.tsbits = n > 1 ? 32 - __builtin_clz(n - 1) : 0;
   g.pinfo = c.pinfo;
   g.istart = c.istart;
   g.qkey = c.qkey;

@@ -60,7 +60,7 @@ def main():
             out[v].append(s0.elapsed_time(s1) / a.steps)
             if a.timing:
                 tree.set_flags(timing=True)
-                tks = [tree.submit(*batches[3 + b], res) for b in range(8)]
+                tks = [tree.submit(*batches[3 + b % a.steps], res) for b in range(8)]
                 st = np.array([tree.results(t)["stage_ms"][:5] for t in tks]).mean(axis=0)
                 stages[v].append(st)
             for kv in v.split(","):
