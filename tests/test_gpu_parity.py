@@ -180,6 +180,53 @@ def test_single_key_storm(dev):
     assert st["distinct"] == 1
 
 
+@pytest.mark.parametrize("seed", [0, 1])
+def test_hot_key_groups(dev, seed):
+    """Skewed batch over the full 64-bit key space: keys with 9000 (more than one
+    group's shared-memory capacity), 5000 + 4000 (two hot keys, one oversized
+    group if they share a bin), 300 and 40 copies, among uniform keys.  Covers
+    the oversized-group L2 sort, the timestamp-stable slow path and the
+    rank-placement fast path of the group sort (group.cu)."""
+    rng = np.random.default_rng(40 + seed)
+    keys, vals = _rand_keys(rng, 20000, hi=1 << 63)
+    t = make_tree(dev, keys, vals, max_batch=1 << 16)
+    ref = oracle.MapOracle(); ref.load(keys, vals)
+    n = 1 << 16
+    hot = [(keys[3], 9000), (keys[11], 5000), (keys[11] + np.uint64(1), 4000), (keys[20], 300),
+           (keys[21], 40), (rng.integers(1, 1 << 63, dtype=np.uint64), 500)]
+    parts = [np.full(c, k, np.uint64) for k, c in hot]
+    rest = n - sum(c for _, c in hot)
+    parts.append(np.where(rng.random(rest) < 0.5, rng.choice(keys, rest),
+                          rng.integers(1, 1 << 63, rest, dtype=np.uint64)).astype(np.uint64))
+    ks = np.concatenate(parts)
+    rng.shuffle(ks)
+    ops = rng.integers(0, 4, n).astype(np.uint8)
+    vs = rng.integers(0, 1 << 62, n, dtype=np.uint64)
+    run_and_compare(t, ref, ops, ks, vs, dev)
+    # and a second batch on the grown tree
+    ops2 = rng.integers(0, 4, n).astype(np.uint8)
+    rng.shuffle(ks)
+    run_and_compare(t, ref, ops2, ks, vs, dev)
+    assert t.check_invariants()[0] == 0
+
+
+def test_dense_key_range(dev):
+    """Dense small integer keys: every request falls in the first bin, so one
+    group holds the whole batch (oversized, many distinct keys: the generic
+    L2 radix path)."""
+    rng = np.random.default_rng(9)
+    keys = np.arange(1, 20001, dtype=np.uint64)
+    vals = rng.integers(0, 1 << 62, keys.size, dtype=np.uint64)
+    t = make_tree(dev, keys, vals, max_batch=1 << 15)
+    ref = oracle.MapOracle(); ref.load(keys, vals)
+    n = 1 << 15
+    ops = rng.integers(0, 4, n).astype(np.uint8)
+    ks = rng.integers(1, 30000, n, dtype=np.uint64)
+    vs = rng.integers(0, 1 << 62, n, dtype=np.uint64)
+    run_and_compare(t, ref, ops, ks, vs, dev)
+    assert t.check_invariants()[0] == 0
+
+
 def test_tiny_tree_root_splits(dev):
     """Start from an empty tree (root is a leaf) and grow it by inserts: root splits."""
     rng = np.random.default_rng(8)
