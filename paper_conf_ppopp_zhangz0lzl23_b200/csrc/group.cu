@@ -52,7 +52,7 @@ struct GSmem {
   uint64_t k[G_CAP];
   uint32_t p[G_CAP];
   uint32_t sb[SB_N + 1];       // sub-bucket starts; per-warp digit counters of the L2 passes
-  uint32_t whist[64 * G_WARPS];  // [digit][warp] counters of the stable smem passes
+  uint32_t whist[G_CAP / 32];  // list of the sub-buckets larger than FAST_SB
   uint32_t wsum[G_WARPS];
   unsigned long long wmin[G_WARPS], wmax[G_WARPS];
   uint32_t wcmax[G_WARPS];
@@ -96,111 +96,53 @@ __device__ void key_range(uint64_t mn, uint64_t mx, GSmem& S) {
   __syncthreads();
 }
 
-// Exclusive scan, in place, of the 1024 [digit][warp] counters (2 per thread).
-__device__ void scan_whist(GSmem& S) {
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t a = S.whist[2 * tid], b = S.whist[2 * tid + 1];
-  uint32_t x = a + b;
-#pragma unroll
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t y = __shfl_up_sync(FULL, x, o);
-    if (lane >= o) x += y;
-  }
-  if (lane == 31) S.wsum[warp] = x;
-  __syncthreads();
-  uint32_t run = x - a - b;
-  for (int w = 0; w < warp; ++w) run += S.wsum[w];
-  S.whist[2 * tid] = run;
-  S.whist[2 * tid + 1] = run + a;
-  __syncthreads();
-}
-
-// Slow path of smem_sort, items parked in S.k / S.p: stable LSD passes,
-// ceil(tsbits / 6) on the timestamp, then (unless the group is one key) 2 on
-// the sub-bucket index, then insertion sort of each sub-bucket (S.sb holds
-// the sub-bucket starts).  Kept out of line so the fast path keeps its
-// registers.
-__device__ __noinline__ void slow_sort(uint32_t cnt, int tsbits, uint64_t kmin, int shift, bool multi, GSmem& S) {
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const uint32_t C = 32u * ((cnt + G_THREADS - 1) / G_THREADS);
-  const uint32_t wb = warp * C;
-  uint64_t kr[G_ITEMS];
-  uint32_t pr[G_ITEMS], r[G_ITEMS];
-  const int tpass = (tsbits + 5) / 6;
-  const int npass = tpass + (multi ? 2 : 0);
-  for (int pass = 0; pass < npass; ++pass) {
-    const bool ts = pass < tpass;
-    const int dsh = 6 * (ts ? pass : pass - tpass);
-#pragma unroll
-    for (int j = 0; j < G_ITEMS; ++j) {
-      const uint32_t i = wb + 32 * j + lane;
-      if (32u * j < C && i < cnt) {
-        kr[j] = S.k[i];
-        pr[j] = S.p[i];
+// Bitonic sort of S.k / S.p [lo, lo + m) by (key, payload), in place, by the
+// threads [t0, t0 + nt) of a warp (nt = 32, warp sync) or of the CTA (nt =
+// G_THREADS, block sync).  The network is the "flip" variant whose merges all
+// run ascending, so positions >= m act as +infinity and are simply skipped.
+template <bool CTA>
+__device__ void bitonic_run(uint32_t lo, uint32_t m, int t, int nt, GSmem& S) {
+  uint32_t N = 2;
+  while (N < m) N <<= 1;
+  for (uint32_t k = 2; k <= N; k <<= 1) {
+    for (uint32_t sdist = k >> 1; sdist > 0; sdist >>= 1) {
+      const bool flip = sdist == (k >> 1);
+      for (uint32_t q = t; q < N / 2; q += nt) {
+        // q-th pair of this step: i has bit log2(sdist) clear
+        const uint32_t i = ((q & ~(sdist - 1)) << 1) | (q & (sdist - 1));
+        const uint32_t j = flip ? (i ^ (k - 1)) : (i | sdist);
+        if (j < m) {
+          const uint64_t ki = S.k[lo + i], kj = S.k[lo + j];
+          const uint32_t pi = S.p[lo + i], pj = S.p[lo + j];
+          if (kp_less(kj, pj, ki, pi)) {
+            S.k[lo + i] = kj;
+            S.k[lo + j] = ki;
+            S.p[lo + i] = pj;
+            S.p[lo + j] = pi;
+          }
+        }
       }
-    }
-    for (int i = tid; i < 64 * G_WARPS; i += G_THREADS) S.whist[i] = 0;
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < G_ITEMS; ++j) {
-      const uint32_t i = wb + 32 * j + lane;
-      const bool v = 32u * j < C && i < cnt;
-      const uint32_t src = ts ? (pr[j] >> 2) : (uint32_t)((kr[j] - kmin) >> shift);
-      const uint32_t d = v ? (src >> dsh) & 63u : 64u;
-      const uint32_t peers = __match_any_sync(FULL, d);
-      const uint32_t base = v ? S.whist[d * G_WARPS + warp] : 0u;
-      r[j] = base + __popc(peers & lanemask_lt());
-      __syncwarp();
-      if (v && lane == 31 - __clz(peers)) S.whist[d * G_WARPS + warp] = base + __popc(peers);
-      __syncwarp();
-    }
-    __syncthreads();
-    scan_whist(S);
-#pragma unroll
-    for (int j = 0; j < G_ITEMS; ++j) {
-      const uint32_t i = wb + 32 * j + lane;
-      if (32u * j < C && i < cnt) {
-        const uint32_t src = ts ? (pr[j] >> 2) : (uint32_t)((kr[j] - kmin) >> shift);
-        const uint32_t pos = S.whist[((src >> dsh) & 63u) * G_WARPS + warp] + r[j];
-        S.k[pos] = kr[j];
-        S.p[pos] = pr[j];
-      }
-    }
-    __syncthreads();
-  }
-  if (!multi) return;   // one key: timestamp order is final
-  for (int sb = tid; sb < SB_N; sb += G_THREADS) {
-    const uint32_t lo = S.sb[sb], hi = S.sb[sb + 1];
-    for (uint32_t a = lo + 1; a < hi; ++a) {
-      const uint64_t k = S.k[a];
-      const uint32_t p = S.p[a];
-      uint32_t c = a;
-      while (c > lo && kp_less(k, p, S.k[c - 1], S.p[c - 1])) {
-        S.k[c] = S.k[c - 1];
-        S.p[c] = S.p[c - 1];
-        --c;
-      }
-      S.k[c] = k;
-      S.p[c] = p;
+      if (CTA)
+        __syncthreads();
+      else
+        __syncwarp();
     }
   }
-  __syncthreads();
 }
 
 // Sort a group of 2 <= cnt <= G_CAP requests (in no particular order) into
 // S.k / S.p by (key, payload).  Items live in registers in warp-contiguous
 // order (position = warp * C + 32 j + lane).  Sub-bucket index =
 // (key - kmin) >> shift, SB_BITS wide, so sub-buckets adapt to the group's key
-// range.  Uniform keys (every sub-bucket <= FAST_SB): scatter by smem-atomic
-// rank.  Otherwise (hot / clustered keys): stable 6-bit counting passes, first
-// on the timestamp bits, then on the sub-bucket index, leave every sub-bucket
-// in timestamp order.  Either way each sub-bucket is finished by insertion
-// sort on (key, payload), whose cost is its number of inversions -- for a hot
-// key in timestamp order, only those against the few other keys beside it.
-// One key in the whole group: the timestamp passes alone finish it.
+// range.  Requests are scattered to their sub-bucket by smem-atomic rank;
+// a request of a sub-bucket of <= FAST_SB requests then moves to sub-bucket
+// start + number of smaller (key, payload) in it (uniform keys: all of them).
+// Larger sub-buckets (hot keys: a key's requests always share one) are
+// sorted by a bitonic network, one warp per sub-bucket up to WARP_SB
+// requests, the whole CTA above, so no distribution costs O(m^2).
 constexpr uint32_t FAST_SB = 32;
-__device__ void smem_sort(const uint64_t* __restrict__ ks, const uint32_t* __restrict__ ps, uint32_t cnt, int tsbits,
-                          GSmem& S) {
+constexpr uint32_t WARP_SB = 1024;
+__device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, GSmem& S) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t C = 32u * ((cnt + G_THREADS - 1) / G_THREADS);
   const uint32_t wb = warp * C;
@@ -228,7 +170,7 @@ __device__ void smem_sort(const uint64_t* __restrict__ ks, const uint32_t* __res
   for (int j = 0; j < G_ITEMS; ++j) {
     const uint32_t i = wb + 32 * j + lane;
     r[j] = 0;
-    if (range != 0 && 32u * j < C && i < cnt) {   // (one key: no sub-buckets, no hot-spot atomics)
+    if (32u * j < C && i < cnt) {
       r[j] = atomicAdd(&S.sb[(uint32_t)((kr[j] - kmin) >> shift)], 1u);
       cm = max(cm, r[j] + 1);
     }
@@ -268,53 +210,59 @@ __device__ void smem_sort(const uint64_t* __restrict__ ks, const uint32_t* __res
     if (tid == 0) S.sb[SB_N] = cnt;
   }
   __syncthreads();
-  if (range != 0 && S.cmax <= FAST_SB) {
-    // scatter by atomic rank, then every request takes its final position:
-    // sub-bucket start + number of (key, payload) smaller in its sub-bucket
 #pragma unroll
-    for (int j = 0; j < G_ITEMS; ++j) {
-      const uint32_t i = wb + 32 * j + lane;
-      if (32u * j < C && i < cnt) {
-        const uint32_t pos = S.sb[(uint32_t)((kr[j] - kmin) >> shift)] + r[j];
-        S.k[pos] = kr[j];
-        S.p[pos] = pr[j];
-      }
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = wb + 32 * j + lane;
+    if (32u * j < C && i < cnt) {
+      const uint32_t pos = S.sb[(uint32_t)((kr[j] - kmin) >> shift)] + r[j];
+      S.k[pos] = kr[j];
+      S.p[pos] = pr[j];
     }
-    __syncthreads();
+  }
+  __syncthreads();
 #pragma unroll
-    for (int j = 0; j < G_ITEMS; ++j) {
-      const uint32_t i = wb + 32 * j + lane;
-      if (32u * j < C && i < cnt) {
-        const uint32_t x = (uint32_t)((kr[j] - kmin) >> shift);
-        const uint32_t lo = S.sb[x], hi = S.sb[x + 1];
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = wb + 32 * j + lane;
+    r[j] = 0xFFFFFFFFu;
+    if (32u * j < C && i < cnt) {
+      const uint32_t x = (uint32_t)((kr[j] - kmin) >> shift);
+      const uint32_t lo = S.sb[x], hi = S.sb[x + 1];
+      if (hi - lo <= FAST_SB) {
         uint32_t less = 0;
         for (uint32_t m = lo; m < hi; ++m) less += kp_less(S.k[m], S.p[m], kr[j], pr[j]);
         r[j] = lo + less;
       }
     }
-    __syncthreads();
-#pragma unroll
-    for (int j = 0; j < G_ITEMS; ++j) {
-      const uint32_t i = wb + 32 * j + lane;
-      if (32u * j < C && i < cnt) {
-        S.k[r[j]] = kr[j];
-        S.p[r[j]] = pr[j];
-      }
-    }
-    __syncthreads();
-    return;
   }
-  // slow path (hot / clustered keys): park the items in position order
+  __syncthreads();
 #pragma unroll
   for (int j = 0; j < G_ITEMS; ++j) {
-    const uint32_t i = wb + 32 * j + lane;
-    if (32u * j < C && i < cnt) {
-      S.k[i] = kr[j];
-      S.p[i] = pr[j];
+    if (r[j] != 0xFFFFFFFFu) {
+      S.k[r[j]] = kr[j];
+      S.p[r[j]] = pr[j];
     }
   }
   __syncthreads();
-  slow_sort(cnt, tsbits, kmin, shift, range != 0, S);
+  if (S.cmax <= FAST_SB) return;
+  // big sub-buckets: list them, then bitonic-sort each in place
+  if (tid == 0) S.r_nh = 0;
+  __syncthreads();
+  for (uint32_t x = tid; x < (uint32_t)SB_N; x += G_THREADS) {
+    const uint32_t m = S.sb[x + 1] - S.sb[x];
+    if (m > FAST_SB) S.whist[atomicAdd(&S.r_nh, 1u)] = x;   // <= G_CAP / FAST_SB entries
+  }
+  __syncthreads();
+  const uint32_t nbig = S.r_nh;
+  for (uint32_t e = warp; e < nbig; e += G_WARPS) {
+    const uint32_t x = S.whist[e], lo = S.sb[x], m = S.sb[x + 1] - lo;
+    if (m <= WARP_SB) bitonic_run<false>(lo, m, lane, 32, S);
+  }
+  __syncthreads();
+  for (uint32_t e = 0; e < nbig; ++e) {
+    const uint32_t x = S.whist[e], lo = S.sb[x], m = S.sb[x + 1] - lo;
+    if (m > WARP_SB) bitonic_run<true>(lo, m, tid, G_THREADS, S);
+  }
+  __syncthreads();
 }
 
 // One stable LSD pass in L2 over [0, cnt) of (ks, ps) -> (kd, pd) by an 8-bit
@@ -330,7 +278,17 @@ __device__ void l2_pass(const uint64_t* ks, const uint32_t* ps, uint64_t* kd, ui
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   if (tid < 256) S.dhist[tid] = 0;
   __syncthreads();
-  for (uint32_t i = tid; i < cnt; i += G_THREADS) atomicAdd(&S.dhist[l2_digit(ks[i], ps[i], ts, kmin, sh)], 1u);
+  for (uint32_t i0 = tid; i0 < cnt; i0 += 8 * G_THREADS) {   // 8 loads in flight per thread
+    uint32_t d[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const uint32_t i = i0 + u * G_THREADS;
+      d[u] = i < cnt ? l2_digit(ks[i], ps[i], ts, kmin, sh) : 256u;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      if (d[u] < 256u) atomicAdd(&S.dhist[d[u]], 1u);
+  }
   __syncthreads();
   if (tid == 0) {
     uint32_t run = 0;
@@ -390,19 +348,189 @@ __device__ void l2_pass(const uint64_t* ks, const uint32_t* ps, uint64_t* kd, ui
   }
 }
 
-// Oversized group (cnt > G_CAP, hot keys): stable LSD in L2, first on the
-// timestamp bits, then on the bits of key - kmin (none for a one-key group),
-// ping-pong between the group's two L2 ranges.  Returns the range that holds
-// the result (0: ks/ps, 1: kd/pd).
-__device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int tsbits, GSmem& S) {
-  uint64_t mn = KEY_MAX, mx = 0;
-  for (uint32_t i = threadIdx.x; i < cnt; i += G_THREADS) {
-    const uint64_t k = ks[i];
-    mn = min(mn, k);
-    mx = max(mx, k);
+// One stable LSD pass in L2 over a payload-only array (one key's requests):
+// digit = 8 bits of the timestamp at sh.
+__device__ void l2_pass_pay(const uint32_t* ps, uint32_t* pd, uint32_t cnt, int sh, GSmem& S) {
+  constexpr int IT = 8;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tid < 256) S.dhist[tid] = 0;
+  __syncthreads();
+  for (uint32_t i0 = tid; i0 < cnt; i0 += 8 * G_THREADS) {   // 8 loads in flight per thread
+    uint32_t d[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const uint32_t i = i0 + u * G_THREADS;
+      d[u] = i < cnt ? ((ps[i] >> 2) >> sh) & 255u : 256u;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      if (d[u] < 256u) atomicAdd(&S.dhist[d[u]], 1u);
   }
-  key_range(mn, mx, S);
+  __syncthreads();
+  if (tid == 0) {
+    uint32_t run = 0;
+    for (int d = 0; d < 256; ++d) {
+      const uint32_t c = S.dhist[d];
+      S.dhist[d] = run;
+      run += c;
+    }
+  }
+  __syncthreads();
+  uint32_t* wh = S.sb;   // [256][G_WARPS]
+  for (uint32_t t0 = 0; t0 < cnt; t0 += G_THREADS * IT) {
+    for (int i = tid; i < 256 * G_WARPS; i += G_THREADS) wh[i] = 0;
+    __syncthreads();
+    uint32_t p[IT], d[IT], r[IT];
+    const uint32_t wb = t0 + warp * 32 * IT;
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+      const uint32_t i = wb + 32 * j + lane;
+      p[j] = i < cnt ? ps[i] : 0u;
+      d[j] = i < cnt ? ((p[j] >> 2) >> sh) & 255u : 256u;
+    }
+#pragma unroll
+    for (int j = 0; j < IT; ++j) {
+      const bool v = d[j] < 256u;
+      const uint32_t peers = __match_any_sync(FULL, d[j]);
+      const uint32_t base = v ? wh[d[j] * G_WARPS + warp] : 0u;
+      r[j] = base + __popc(peers & lanemask_lt());
+      __syncwarp();
+      if (v && lane == 31 - __clz(peers)) wh[d[j] * G_WARPS + warp] = base + __popc(peers);
+      __syncwarp();
+    }
+    __syncthreads();
+    if (tid < 256) {
+      uint32_t c = 0;
+#pragma unroll
+      for (int w = 0; w < G_WARPS; ++w) {
+        const uint32_t x = wh[tid * G_WARPS + w];
+        wh[tid * G_WARPS + w] = c + S.dhist[tid];
+        c += x;
+      }
+      S.dhist[tid] += c;
+    }
+    __syncthreads();
+#pragma unroll
+    for (int j = 0; j < IT; ++j)
+      if (d[j] < 256u) pd[wh[d[j] * G_WARPS + warp] + r[j]] = p[j];
+    __syncthreads();
+  }
+}
+
+// Oversized group (cnt > G_CAP): hot keys.  One pass finds the key range and
+// counts three sampled candidates; the most frequent one, hk, is split off
+// when the rest fits in shared memory: the rest is sorted there (smem_sort),
+// hk's payloads are sorted by timestamp with payload-only LSD passes in L2,
+// and the group is laid out as [rest < hk][hk in timestamp order][rest > hk]
+// in (kd, pd).  Otherwise: stable LSD on the timestamp bits, then on the bits
+// of key - kmin, ping-pong between the group's two L2 ranges.  Returns the
+// range that holds the result (0: ks/ps, 1: kd/pd).
+__device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int tsbits, GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint64_t c0 = ks[0], c1 = ks[cnt / 3], c2 = ks[(2 * (uint64_t)cnt) / 3];
+  uint64_t mn = KEY_MAX, mx = 0;
+  uint32_t n0 = 0, n1 = 0, n2 = 0;
+  for (uint32_t i0 = tid; i0 < cnt; i0 += 8 * G_THREADS) {   // 8 loads in flight per thread
+    uint64_t kk[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const uint32_t i = i0 + u * G_THREADS;
+      kk[u] = i < cnt ? ks[i] : ks[0];
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      if (i0 + u * G_THREADS < cnt) {
+        mn = min(mn, kk[u]);
+        mx = max(mx, kk[u]);
+        n0 += kk[u] == c0;
+        n1 += kk[u] == c1;
+        n2 += kk[u] == c2;
+      }
+    }
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) {
+    n0 += __shfl_xor_sync(FULL, n0, o);
+    n1 += __shfl_xor_sync(FULL, n1, o);
+    n2 += __shfl_xor_sync(FULL, n2, o);
+  }
+  if (lane == 0) {
+    S.w_nh[warp] = n0;
+    S.w_lw[warp] = n1;
+    S.w_nw[warp] = n2;
+  }
+  key_range(mn, mx, S);   // (its barriers publish the per-warp counts)
+  n0 = n1 = n2 = 0;
+  for (int w = 0; w < G_WARPS; ++w) {
+    n0 += S.w_nh[w];
+    n1 += S.w_lw[w];
+    n2 += S.w_nw[w];
+  }
   const uint64_t kmin = S.kmin, range = S.kmax - S.kmin;
+  const uint64_t hk = (n0 >= n1 && n0 >= n2) ? c0 : (n1 >= n2 ? c1 : c2);
+  const uint32_t hcnt = max(n0, max(n1, n2));
+  if (cnt - hcnt <= (uint32_t)G_CAP) {
+    // split: the rest into S.k / S.p, hk's payloads into kd (as u32 scratch)
+    uint32_t* hs = reinterpret_cast<uint32_t*>(kd);
+    if (tid == 0) {
+      S.r_nh = 0;   // rest
+      S.r_lw = 0;   // hk
+      S.r_nw = 0;   // rest below hk
+    }
+    __syncthreads();
+    for (uint32_t b0 = 0; b0 < cnt; b0 += 8 * G_THREADS) {   // 8 loads in flight per thread
+      uint64_t kk[8];
+      uint32_t pp[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint32_t i = b0 + u * G_THREADS + tid;
+        kk[u] = i < cnt ? ks[i] : 0;
+        pp[u] = i < cnt ? ps[i] : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const bool v = b0 + u * G_THREADS + tid < cnt;
+        const uint64_t k = kk[u];
+        const uint32_t p = pp[u];
+        const bool hot = v && k == hk;
+        const uint32_t mh = __ballot_sync(FULL, hot), mo = __ballot_sync(FULL, v && !hot);
+        const uint32_t below = __popc(__ballot_sync(FULL, v && !hot && k < hk));
+        uint32_t bh = 0, bo = 0;
+        if (lane == 0) {
+          if (mh) bh = atomicAdd(&S.r_lw, __popc(mh));
+          if (mo) bo = atomicAdd(&S.r_nh, __popc(mo));
+          if (below) atomicAdd(&S.r_nw, below);
+        }
+        bh = __shfl_sync(FULL, bh, 0);
+        bo = __shfl_sync(FULL, bo, 0);
+        if (hot) hs[bh + __popc(mh & lanemask_lt())] = p;
+        if (v && !hot) {
+          const uint32_t x = bo + __popc(mo & lanemask_lt());
+          S.k[x] = k;
+          S.p[x] = p;
+        }
+      }
+    }
+    __syncthreads();
+    const uint32_t o = S.r_nh, h = S.r_lw, lo = S.r_nw;
+    if (o > 1) smem_sort(S.k, S.p, o, S);
+    __syncthreads();
+    // hk's payloads by timestamp: hs -> ps -> hs ... -> pd + lo (last pass)
+    const int tpass = max(1, (tsbits + 7) / 8);
+    for (int pass = 0; pass < tpass; ++pass) {
+      const uint32_t* src = (pass & 1) ? ps : hs;
+      uint32_t* dst = pass + 1 == tpass ? pd + lo : ((pass & 1) ? hs : ps);
+      l2_pass_pay(src, dst, h, 8 * pass, S);
+    }
+    for (uint32_t x = tid; x < h; x += G_THREADS) kd[lo + x] = hk;
+    for (uint32_t x = tid; x < o; x += G_THREADS) {
+      const uint32_t d = x < lo ? x : x + h;
+      kd[d] = S.k[x];
+      pd[d] = S.p[x];
+    }
+    __syncthreads();
+    return 1;
+  }
   const int tpass = (tsbits + 7) / 8;
   const int passes = tpass + (range ? (64 - __clzll((long long)range) + 7) / 8 : 0);
   for (int pass = 0; pass < passes; ++pass) {
@@ -458,10 +586,23 @@ struct GroupArgs {
   BatchCtl* ctl;
 };
 
+// The sorted group as seen by the combine passes: positions [c0, c1) from a
+// shared-memory copy (the whole group when it fits, else the current round of
+// an oversized group), the rest (a round's neighbours) from L2.
+struct GView {
+  const uint64_t* Kg;
+  const uint32_t* Pg;
+  const uint64_t* Ks;
+  const uint32_t* Ps;
+  uint32_t c0, c1;
+  __device__ __forceinline__ uint64_t k(uint32_t x) const { return x - c0 < c1 - c0 ? Ks[x - c0] : Kg[x]; }
+  __device__ __forceinline__ uint32_t p(uint32_t x) const { return x - c0 < c1 - c0 ? Ps[x - c0] : Pg[x]; }
+};
+
 // Round [r0, r1) of a bucket walked by 16 warps: pass 1 (heads, last write per
 // warp), warp scan, pass 2 (write segments ending in each warp), warp scan.
 // Leaves the exclusive per-warp carries in S.c_* and the carry-out in S.r_*.
-__device__ void round_scan(const uint64_t* K, const uint32_t* P, uint32_t cnt, uint32_t r0, uint32_t r1,
+__device__ void round_scan(const GView& V, uint32_t cnt, uint32_t r0, uint32_t r1,
                            uint32_t cin_nh, uint32_t cin_lw, uint32_t cin_nw, GSmem& S) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t len = r1 - r0;
@@ -472,9 +613,9 @@ __device__ void round_scan(const uint64_t* K, const uint32_t* P, uint32_t cnt, u
   for (uint32_t b = wb; b < we; b += 32) {
     const uint32_t x = b + lane;
     const bool valid = x < we;
-    const uint64_t k = valid ? K[x] : 0;
-    const bool head = valid && (x == 0 || K[x - 1] != k);
-    const uint32_t W = __ballot_sync(FULL, valid && is_write(P[valid ? x : 0] & 3));
+    const uint64_t k = valid ? V.k(x) : 0;
+    const bool head = valid && (x == 0 || V.k(x - 1) != k);
+    const uint32_t W = __ballot_sync(FULL, valid && is_write(V.p(valid ? x : 0) & 3));
     nh += __popc(__ballot_sync(FULL, head));
     if (W) lw = b + (31 - __clz(W)) + 1;
   }
@@ -499,12 +640,12 @@ __device__ void round_scan(const uint64_t* K, const uint32_t* P, uint32_t cnt, u
   for (uint32_t b = wb; b < we; b += 32) {
     const uint32_t x = b + lane;
     const bool valid = x < we;
-    const uint64_t k = valid ? K[x] : 0;
-    const uint32_t W = __ballot_sync(FULL, valid && is_write(P[valid ? x : 0] & 3));
+    const uint64_t k = valid ? V.k(x) : 0;
+    const uint32_t W = __ballot_sync(FULL, valid && is_write(V.p(valid ? x : 0) & 3));
     const uint32_t wle = W & lanemask_le();
     const uint32_t lwi = wle ? b + (31 - __clz(wle)) + 1 : lwc;
-    const bool tail = valid && (x + 1 == cnt || K[x + 1] != k);
-    const bool hasw = tail && lwi && K[lwi - 1] == k;
+    const bool tail = valid && (x + 1 == cnt || V.k(x + 1) != k);
+    const bool hasw = tail && lwi && V.k(lwi - 1) == k;
     nwt += __popc(__ballot_sync(FULL, hasw));
     if (W) lwc = b + (31 - __clz(W)) + 1;
   }
@@ -522,7 +663,7 @@ __device__ void round_scan(const uint64_t* K, const uint32_t* P, uint32_t cnt, u
 }
 
 // Pass 3 of round [r0, r1): every output of the combine and the partition.
-__device__ void round_emit(const GroupArgs& g, const uint64_t* K, const uint32_t* P, uint32_t cnt, uint32_t gbase,
+__device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uint32_t gbase,
                            uint32_t r0, uint32_t r1, bool write_spay, GSmem& S) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t* __restrict__ vals = g.A->vals;
@@ -536,9 +677,9 @@ __device__ void round_emit(const GroupArgs& g, const uint64_t* K, const uint32_t
   for (uint32_t b = wb; b < we; b += 32) {
     const uint32_t x = b + lane;
     const bool valid = x < we;
-    const uint64_t k = valid ? K[x] : 0;
-    const uint32_t p = valid ? P[x] : 0;
-    const bool head = valid && (x == 0 || K[x - 1] != k);
+    const uint64_t k = valid ? V.k(x) : 0;
+    const uint32_t p = valid ? V.p(x) : 0;
+    const bool head = valid && (x == 0 || V.k(x - 1) != k);
     const uint32_t H = __ballot_sync(FULL, head);
     const uint32_t W = __ballot_sync(FULL, valid && is_write(p & 3));
     const uint32_t seg = seg0 + nh + __popc(H & lanemask_le()) - 1u;
@@ -547,9 +688,9 @@ __device__ void round_emit(const GroupArgs& g, const uint64_t* K, const uint32_t
     const uint32_t lwb = wl ? b + (31 - __clz(wl)) + 1 : lwc;
     const uint32_t wle = W & lanemask_le();
     const uint32_t lwi = wle ? b + (31 - __clz(wle)) + 1 : lwc;
-    const bool done = valid && !head && lwb && K[lwb - 1] == k;
+    const bool done = valid && !head && lwb && V.k(lwb - 1) == k;
     if (done) {
-      const uint32_t pw = P[lwb - 1];
+      const uint32_t pw = V.p(lwb - 1);
       results[p >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
     }
     if (valid) {
@@ -557,13 +698,13 @@ __device__ void round_emit(const GroupArgs& g, const uint64_t* K, const uint32_t
       if (write_spay) g.pB[gbase + x] = p;
     }
     if (head) g.istart[seg] = gbase + x;
-    const bool tail = valid && (x + 1 == cnt || K[x + 1] != k);
-    const bool hasw = tail && lwi && K[lwi - 1] == k;
+    const bool tail = valid && (x + 1 == cnt || V.k(x + 1) != k);
+    const bool hasw = tail && lwi && V.k(lwi - 1) == k;
     const uint32_t WT = __ballot_sync(FULL, hasw);
     if (tail) {
       const uint32_t wi = w0 + nwc + __popc(WT & lanemask_lt());
       if (hasw) {   // issue rule: the segment's last write
-        const uint32_t pw = P[lwi - 1];
+        const uint32_t pw = V.p(lwi - 1);
         const uint32_t opw = pw & 3;
         g.wkey[wi] = k;
         g.wop[wi] = (uint8_t)opw;
@@ -600,7 +741,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       S.k[0] = g.kA[base];
       S.p[0] = g.pA[base];
     } else if (cnt > 1) {
-      smem_sort(g.kA + base, g.pA + base, cnt, g.tsbits, S);
+      smem_sort(g.kA + base, g.pA + base, cnt, S);
     }
     __syncthreads();
     K = S.k;
@@ -610,11 +751,36 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     K = (where ? g.kB : g.kA) + base;
     P = (where ? g.pB : g.pA) + base;
   }
+  // an oversized group is walked in rounds of G_CAP positions copied to smem
+  auto load_round = [&](uint32_t r0, uint32_t r1) {
+    __syncthreads();
+    for (uint32_t i0 = r0 + tid; i0 < r1; i0 += 8 * G_THREADS) {   // 8 loads in flight per thread
+      uint64_t kk[8];
+      uint32_t pp[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint32_t i = i0 + u * G_THREADS;
+        kk[u] = i < r1 ? K[i] : 0;
+        pp[u] = i < r1 ? P[i] : 0;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint32_t i = i0 + u * G_THREADS;
+        if (i < r1) {
+          S.k[i - r0] = kk[u];
+          S.p[i - r0] = pp[u];
+        }
+      }
+    }
+    __syncthreads();
+    return GView{K, P, S.k, S.p, r0, r1};
+  };
   // sweep 1: bucket totals (heads, write segments)
   uint32_t c_nh = 0, c_lw = 0, c_nw = 0;
   for (uint32_t r0 = 0; r0 < cnt; r0 += G_CAP) {
     const uint32_t r1 = min(cnt, r0 + (uint32_t)G_CAP);
-    round_scan(K, P, cnt, r0, r1, c_nh, c_lw, c_nw, S);
+    const GView V = small ? GView{K, P, K, P, 0, cnt} : load_round(r0, r1);
+    round_scan(V, cnt, r0, r1, c_nh, c_lw, c_nw, S);
     c_nh = S.r_nh;
     c_lw = S.r_lw;
     c_nw = S.r_nw;
@@ -666,14 +832,15 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   __syncthreads();
   // sweep 2: emit (a small bucket reuses the carries of its single round)
   if (small) {
-    if (cnt) round_emit(g, K, P, cnt, base, 0, cnt, true, S);
+    if (cnt) round_emit(g, GView{K, P, K, P, 0, cnt}, cnt, base, 0, cnt, true, S);
   } else {
     const bool write_spay = P != g.pB + base;
     c_nh = c_lw = c_nw = 0;
     for (uint32_t r0 = 0; r0 < cnt; r0 += G_CAP) {
       const uint32_t r1 = min(cnt, r0 + (uint32_t)G_CAP);
-      round_scan(K, P, cnt, r0, r1, c_nh, c_lw, c_nw, S);
-      round_emit(g, K, P, cnt, base, r0, r1, write_spay, S);
+      const GView V = load_round(r0, r1);
+      round_scan(V, cnt, r0, r1, c_nh, c_lw, c_nw, S);
+      round_emit(g, V, cnt, base, r0, r1, write_spay, S);
       c_nh = S.r_nh;
       c_lw = S.r_lw;
       c_nw = S.r_nw;

@@ -113,13 +113,13 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
 // segments longer than SHORT_SEG (hot keys) are queued instead and finished
 // here with one CTA per segment, so a 56K-request Zipf key does not serialise
 // one thread.
-__global__ void __launch_bounds__(256) result_long_kernel(const uint32_t* __restrict__ spay,
-                                                           const uint32_t* __restrict__ pinfo,
-                                                           const uint32_t* __restrict__ istart,
-                                                           const uint32_t* __restrict__ longseg,
-                                                           const uint64_t* __restrict__ old,
-                                                           const BatchArgs* __restrict__ A,
-                                                           const BatchCtl* __restrict__ ctl) {
+__global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __restrict__ spay,
+                                                            const uint32_t* __restrict__ pinfo,
+                                                            const uint32_t* __restrict__ istart,
+                                                            const uint32_t* __restrict__ longseg,
+                                                            const uint64_t* __restrict__ old,
+                                                            const BatchArgs* __restrict__ A,
+                                                            const BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
   const uint32_t nl = ctl->nlong;
@@ -127,8 +127,18 @@ __global__ void __launch_bounds__(256) result_long_kernel(const uint32_t* __rest
     const uint32_t s = longseg[x];
     const uint64_t v = old[s];
     const uint32_t e = istart[s + 1];
-    for (uint32_t p = istart[s] + threadIdx.x; p < e; p += blockDim.x)
-      if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
+    for (uint32_t p0 = istart[s] + threadIdx.x; p0 < e; p0 += 8 * blockDim.x) {   // 8 loads in flight
+      uint32_t pi[8], py[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const uint32_t p = p0 + u * blockDim.x;
+        pi[u] = p < e ? pinfo[p] : DONE_BIT;
+        py[u] = p < e ? spay[p] : 0u;
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u)
+        if (!(pi[u] & DONE_BIT)) results[py[u] >> 2] = v;
+    }
   }
 }
 
@@ -147,7 +157,7 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
 void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
                    cudaStream_t st, int* launches) {
   (void)n;
-  result_long_kernel<<<148, 256, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, A, ctl);
+  result_long_kernel<<<148, 1024, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, A, ctl);
   ++*launches;
 }
 
