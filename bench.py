@@ -372,8 +372,16 @@ def run_ours(args):
             ms = stage_ms[0]
             kern = "bsort_hist_kernel + bsort_scatter_kernel"
         ach = bytes_per / (ms * 1e-3) / 1e9
+        # measured DRAM traffic of the same kernel per launch, from the committed
+        # ncu capture (tools/ncu_traffic.sh -> profiles/traffic.json); null if absent
+        traffic, traffic_src = None, None
+        tpath = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "traffic.json")
+        if os.path.exists(tpath):
+            tj = json.load(open(tpath)).get(kern)
+            if tj:
+                traffic, traffic_src = tj["dram_bytes_per_launch"], tj["source"]
         roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
-                "frac": ach / peaks["hbm_gbs"], "traffic": None, "kernel": kern,
+                "frac": ach / peaks["hbm_gbs"], "traffic": traffic, "traffic_source": traffic_src, "kernel": kern,
                 "stage_ms": ms, "algorithmic_bytes_per_launch": bytes_per, "peak_source": peaks["source"]}
 
     if rank == 0:

@@ -2,7 +2,7 @@
 # Profiling recipe (B200_PROFILING.md): launch list + one full capture per hot kernel.
 # usage: bash tools_profile.sh <tag> [kernel-regex]
 TAG=${1:-r1}
-KRE=${2:-"combine_kernel|partition_kernel|query_kernel|update_kernel|bsort_|result_long|finalize"}
+KRE=${2:-"group_kernel|query_kernel|update_kernel|bsort_|result_long|finalize"}
 OUT=gpurun_out/prof_$TAG
 mkdir -p $OUT
 BENCH="python bench.py --steps 3 --warmup 3 --e2e-steps 0 --cpu-batches 0"
