@@ -39,16 +39,6 @@ int cuda_fail(cudaError_t e, const char* where) {
     if (_e != cudaSuccess) return cuda_fail(_e, #expr); \
   } while (0)
 
-__global__ void finalize_kernel(BatchCtl* ctl, const TreeHdr* hdr, int dbgprint) {
-  if (threadIdx.x == 0) {
-    if (ctl->invalid) ctl->status = EIRENE_EINVAL;
-    ctl->height = (uint32_t)(hdr->root_word >> 32);
-    if (dbgprint)
-      printf("[eirene dbg] %u %u %u %u %u %u %u %u\n", ctl->dbg[0], ctl->dbg[1], ctl->dbg[2], ctl->dbg[3],
-             ctl->dbg[4], ctl->dbg[5], ctl->dbg[6], ctl->dbg[7]);
-  }
-}
-
 __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
   const int i = threadIdx.x;
   if (i < FAN) {
@@ -73,18 +63,23 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
   }
 }
 
-__global__ void set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
-                                uint64_t* results) {
+// First node of the batch graph: zero the per-batch control region (BatchCtl,
+// bin counts, group look-back words) and publish the batch's pointers.
+__global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys,
+                                                        const uint64_t* vals, uint64_t* results, BatchCtl* host_ctl,
+                                                        uint4* zero, uint32_t zero_n16) {
+  for (uint32_t i = threadIdx.x; i < zero_n16; i += blockDim.x) zero[i] = make_uint4(0, 0, 0, 0);
   if (threadIdx.x == 0) {
     dst->ops = ops;
     dst->keys = keys;
     dst->vals = vals;
     dst->results = results;
+    dst->host_ctl = host_ctl;
   }
 }
 
-// kernels in one batch graph: set_args, 2 sort, group, query, update, result_long, finalize
-constexpr int GRAPH_KERNELS = 8;
+// kernels in one batch graph: set_args, 2 sort, group, query, update, result_long
+constexpr int GRAPH_KERNELS = 7;
 constexpr int MAX_GRAPHS = 8;
 
 struct GraphEntry {
@@ -122,7 +117,8 @@ struct eirene_tree {
   unsigned char* zero_region = nullptr;
   size_t zero_bytes = 0;
   BatchCtl* ctl = nullptr;
-  BatchCtl* host_ctl = nullptr;   // pinned [RING]
+  BatchCtl* host_ctl = nullptr;   // pinned, mapped [RING]
+  BatchCtl* host_ctl_dev = nullptr;   // its device address
   cudaStream_t h2d_stream = nullptr;
   cudaEvent_t h2d_done[2] = {}, comp_done[2] = {};
   bool slot_used[2] = {false, false};
@@ -289,7 +285,9 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     }
   }
 #undef AL
-  if (e == cudaSuccess) e = cudaMallocHost(reinterpret_cast<void**>(&h->host_ctl), sizeof(BatchCtl) * RING);
+  if (e == cudaSuccess)
+    e = cudaHostAlloc(reinterpret_cast<void**>(&h->host_ctl), sizeof(BatchCtl) * RING, cudaHostAllocMapped);
+  if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->host_ctl_dev), h->host_ctl, 0);
   for (int i = 0; i < RING && e == cudaSuccess; ++i) {
     e = cudaEventCreateWithFlags(&h->ring[i].done, cudaEventDisableTiming);
     for (int s = 0; s < NSTAGE && e == cudaSuccess; ++s) e = cudaEventCreate(&h->ring[i].st[s]);
@@ -396,15 +394,17 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     return cudaSuccess;
   };
   auto rec = [&](int i, cudaStream_t s) { cudaEventRecord(r.st[i], s); };
+  BatchCtl* host_ctl_slot = h->host_ctl_dev + tk % RING;
+  uint4* zero16 = reinterpret_cast<uint4*>(h->zero_region);
+  uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
   auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
-    set_args_kernel<<<1, 32, 0, s>>>(h->dargs, ops, keys, vals, results);
+    set_args_kernel<<<1, 1024, 0, s>>>(h->dargs, ops, keys, vals, results, host_ctl_slot, zero16, zero_n16);
     ++launches;
     if (args_node) {
       cudaError_t e = last_node(s, args_node);
       if (e != cudaSuccess) return e;
     }
     if (timing) rec(0, s);
-    cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, s);
     launch_bucket_sort(h->dargs, n, h->cfg.key_lo, h->cfg.key_hi, h->bs, ctl, h->num_sms, s, &launches);
     stage("sort");
     if (timing) rec(1, s);
@@ -418,10 +418,8 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
     stage("update");
     if (timing) rec(4, s);
-    launch_result(spay, n, h->cb, h->dargs, ctl, s, &launches);
+    launch_result(spay, n, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, s, &launches);
     stage("result");
-    finalize_kernel<<<1, 32, 0, s>>>(ctl, h->t.hdr, dbg ? 1 : 0);
-    ++launches;
     if (timing) rec(5, s);
     return cudaGetLastError();
   };
@@ -448,11 +446,11 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       launches = 0;
     }
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
-                      const_cast<uint64_t**>(&vals), &results};
+                      const_cast<uint64_t**>(&vals), &results, &host_ctl_slot, &zero16, &zero_n16};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
     p.gridDim = dim3(1);
-    p.blockDim = dim3(32);
+    p.blockDim = dim3(1024);
     p.sharedMemBytes = 0;
     p.kernelParams = params;
     p.extra = nullptr;
@@ -461,7 +459,6 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     launches = GRAPH_KERNELS;
   }
   if (results_host) CK(cudaMemcpyAsync(results_host, results, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, st));
-  CK(cudaMemcpyAsync(&h->host_ctl[tk % RING], ctl, sizeof(BatchCtl), cudaMemcpyDeviceToHost, st));
   CK(cudaEventRecord(r.done, st));
   r.launches = launches;
   h->launches += launches;

@@ -94,6 +94,7 @@ struct BatchArgs {
   const uint64_t* keys;
   const uint64_t* vals;
   uint64_t* results;
+  BatchCtl* host_ctl;   // mapped pinned ring slot: the batch's BatchCtl is written here at the end
 };
 
 // tile counters
@@ -239,6 +240,7 @@ struct UpdParams {
 void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms,
                    cudaStream_t st, int* launches);
 void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
+                   const TreeHdr* hdr, int dbgprint,
                    cudaStream_t st, int* launches);
 
 // bulk build / scan
