@@ -78,8 +78,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
   }
 }
 
-// kernels in one batch graph: set_args, 2 sort, group, query, update, result_long
-constexpr int GRAPH_KERNELS = 7;
+// kernels in one batch graph: set_args, 1-2 sort, group, query, update, result_long
 constexpr int MAX_GRAPHS = 8;
 
 struct GraphEntry {
@@ -87,6 +86,7 @@ struct GraphEntry {
   cudaGraph_t graph = nullptr;      // kept alive: args_node belongs to it
   cudaGraphExec_t exec = nullptr;
   cudaGraphNode_t args_node = nullptr;
+  int launches = 0;                 // kernels in the graph
 };
 
 struct Rec {
@@ -256,7 +256,6 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->route_ctr, 1);
   AL(h->bs.gstart, NBINS + 1);
   AL(h->bs.bin2grp, NBINS);
-  AL(h->bs.cursor, NBINS);
   AL(h->dargs, 1);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
@@ -270,6 +269,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     const size_t o_ctl = bump(sizeof(BatchCtl));
     const size_t o_gh = bump(sizeof(uint32_t) * 8 * 256);
     const size_t o_bc = bump(sizeof(uint32_t) * NBINS);
+    const size_t o_cu = bump(sizeof(uint32_t) * NBINS);
     const size_t o_gs = bump(sizeof(unsigned long long) * GROUP_STATUS_WORDS);
     h->zero_bytes = off;
     AL(h->zero_region, off);
@@ -277,6 +277,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
       h->ctl = reinterpret_cast<BatchCtl*>(h->zero_region + o_ctl);
       h->sb.ghist = reinterpret_cast<uint32_t*>(h->zero_region + o_gh);
       h->bs.bcount = reinterpret_cast<uint32_t*>(h->zero_region + o_bc);
+      h->bs.cursor = reinterpret_cast<uint32_t*>(h->zero_region + o_cu);
       h->bs.kA = h->sb.kA;
       h->bs.pA = h->sb.pA;
       h->bs.kB = h->sb.kB;
@@ -442,8 +443,8 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       CK(ee);
       CK(cudaGraphInstantiate(&e.exec, e.graph, 0));
       e.n = n;
+      e.launches = launches;
       g = &e;
-      launches = 0;
     }
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
                       const_cast<uint64_t**>(&vals), &results, &host_ctl_slot, &zero16, &zero_n16};
@@ -456,7 +457,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     p.extra = nullptr;
     CK(cudaGraphExecKernelNodeSetParams(g->exec, g->args_node, &p));
     CK(cudaGraphLaunch(g->exec, st));
-    launches = GRAPH_KERNELS;
+    launches = g->launches;
   }
   if (results_host) CK(cudaMemcpyAsync(results_host, results, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, st));
   CK(cudaEventRecord(r.done, st));

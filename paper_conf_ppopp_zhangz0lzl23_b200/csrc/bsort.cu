@@ -170,6 +170,147 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
   }
 }
 
+// Fused K0 + K1 for batches that fit in registers (n <= grid * D_THREADS *
+// D_ITEMS): one persistent wave (every CTA resident), each CTA owns a
+// contiguous slice of the batch and keeps its keys and ops in registers.
+// Phase 1: validation + 4096-bin smem histogram -> global bin counts.  Grid
+// barrier.  Phase 2: every CTA recomputes the group cut from the global counts
+// (CTA 0 also publishes the group starts).  Phase 3: tile histogram over the
+// groups, one atomic per (CTA, group) on the group cursor (zeroed per batch,
+// relative to the group start), scatter from registers.  One launch and one
+// read of the keys instead of two of each.
+constexpr int D_THREADS = 512;
+constexpr int D_ITEMS = 8;
+__global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
+    const BatchArgs* __restrict__ A, uint32_t n, uint32_t G, uint32_t per_cta, uint64_t key_lo, uint64_t key_hi,
+    uint32_t* __restrict__ bcount, uint32_t* __restrict__ gstart, uint32_t* __restrict__ cursor,
+    uint64_t* __restrict__ kout, uint32_t* __restrict__ pout, BatchCtl* ctl) {
+  __shared__ uint32_t h[NBINS];        // bin counts; then bin -> group
+  __shared__ uint32_t gs[NBINS + 1];   // exclusive bin prefix; then group starts / bases
+  __shared__ uint32_t wsum[D_THREADS / 32];
+  const uint64_t* __restrict__ keys = A->keys;
+  const uint8_t* __restrict__ ops = A->ops;
+  const uint64_t* __restrict__ vals = A->vals;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  for (uint32_t i = tid; i < NBINS; i += D_THREADS) h[i] = 0;
+  __syncthreads();
+  const uint32_t t0 = blockIdx.x * per_cta;
+  const uint32_t t1 = min(n, t0 + per_cta);
+  uint64_t k[D_ITEMS];
+  uint32_t o[D_ITEMS];
+#pragma unroll
+  for (int j = 0; j < D_ITEMS; ++j) {
+    const uint32_t i = t0 + j * D_THREADS + tid;
+    k[j] = i < t1 ? keys[i] : 0;
+    o[j] = i < t1 ? (uint32_t)ops[i] : 0u;
+  }
+  bool bad = false;
+#pragma unroll
+  for (int j = 0; j < D_ITEMS; ++j) {
+    const uint32_t i = t0 + j * D_THREADS + tid;
+    const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
+    const uint64_t v = (i < t1 && up) ? vals[i] : 0;
+    bad |= i < t1 && (o[j] > OP_DELETE || k[j] == KEY_MAX || k[j] < key_lo || k[j] >= key_hi || (up && v == KEY_MAX));
+    if (i < t1) atomicAdd(&h[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
+  }
+  if (__any_sync(FULL, bad) && lane == 0) atomicOr(&ctl->invalid, 1u);
+  __syncthreads();
+  for (uint32_t i = tid; i < NBINS; i += D_THREADS)
+    if (h[i]) atomicAdd(&bcount[i], h[i]);
+  // grid barrier (all CTAs are resident: the grid is one occupancy wave)
+  __syncthreads();
+  if (tid == 0) {
+    __threadfence();
+    atomicAdd(&ctl->gbar, 1u);
+    SpinGuard sg;
+    while (ld_acquire(&ctl->gbar) < gridDim.x)
+      if (sg.stuck(ctl)) break;
+  }
+  __syncthreads();
+  // phase 2: the group cut, as in bsort_hist_kernel's last CTA
+  constexpr int PER = NBINS / D_THREADS;
+  uint32_t cnt[PER];
+  uint32_t sum = 0;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    cnt[j] = ld_cg(bcount + tid * PER + j);
+    sum += cnt[j];
+  }
+  uint32_t x = sum;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, x, d);
+    if (lane >= d) x += y;
+  }
+  if (lane == 31) wsum[warp] = x;
+  __syncthreads();
+  uint32_t run = x - sum;
+  for (int w = 0; w < warp; ++w) run += wsum[w];
+  const bool identity = G == (uint32_t)NBINS;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    const uint32_t bin = tid * PER + j;
+    const uint32_t g = identity ? bin
+                                : (uint32_t)min((unsigned long long)(G - 1),
+                                                ((unsigned long long)run + cnt[j] / 2) * G / max(n, 1u));
+    h[bin] = g;
+    gs[bin] = run;
+    run += cnt[j];
+  }
+  __syncthreads();
+  // group starts into registers of the bins' threads, then gs[] = group starts
+  uint32_t gq[PER], ge[PER];
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    const uint32_t bin = tid * PER + j;
+    gq[j] = h[bin];
+    ge[j] = gs[bin];
+  }
+  const uint32_t gprev = tid ? h[tid * PER - 1] : 0xFFFFFFFFu;
+  __syncthreads();
+  {
+    uint32_t gp = gprev;
+#pragma unroll
+    for (int j = 0; j < PER; ++j) {
+      for (uint32_t q = gp + 1; q <= gq[j]; ++q) gs[q] = ge[j];
+      gp = gq[j];
+    }
+    if (tid == D_THREADS - 1)
+      for (uint32_t q = gp + 1; q <= G; ++q) gs[q] = n;
+  }
+  __syncthreads();
+  if (blockIdx.x == 0)
+    for (uint32_t q = tid; q <= G; q += D_THREADS) gstart[q] = gs[q];
+  // phase 3: tile histogram over the groups (reuses the tail of h as counters)
+  uint32_t* th = h + NBINS - G;   // bins are no longer needed once g is known per item
+  uint32_t g[D_ITEMS], r[D_ITEMS];
+#pragma unroll
+  for (int j = 0; j < D_ITEMS; ++j) g[j] = h[(uint32_t)(k[j] >> (64 - BIN_BITS))];
+  __syncthreads();
+  for (uint32_t q = tid; q < G; q += D_THREADS) th[q] = 0;
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < D_ITEMS; ++j) {
+    const uint32_t i = t0 + j * D_THREADS + tid;
+    r[j] = i < t1 ? atomicAdd(&th[g[j]], 1u) : 0u;
+  }
+  __syncthreads();
+  for (uint32_t q = tid; q < G; q += D_THREADS) {
+    const uint32_t c = th[q];
+    th[q] = c ? gs[q] + atomicAdd(&cursor[q], c) : 0u;
+  }
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < D_ITEMS; ++j) {
+    const uint32_t i = t0 + j * D_THREADS + tid;
+    if (i < t1) {
+      const uint32_t pos = th[g[j]] + r[j];
+      kout[pos] = k[j];
+      pout[pos] = (i << 2) | o[j];
+    }
+  }
+}
+
 }  // namespace
 
 uint32_t bsort_groups(uint32_t n, int num_sms) {
@@ -185,8 +326,23 @@ uint32_t bsort_groups(uint32_t n, int num_sms) {
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
                         BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
   const uint32_t G = bsort_groups(n, num_sms);
-  const uint32_t hb = (n + H_THREADS * H_ITEMS - 1) / (H_THREADS * H_ITEMS);
-  bsort_hist_kernel<<<hb, H_THREADS, 0, st>>>(A, n, G, b.bcount, b.bin2grp, b.gstart, b.cursor, ctl);
+  static int dist_per_sm = -1;
+  if (dist_per_sm < 0) {
+    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&dist_per_sm, bsort_dist_kernel, D_THREADS, 0) != cudaSuccess)
+      dist_per_sm = 0;
+  }
+  const uint32_t grid = (uint32_t)num_sms * (uint32_t)dist_per_sm;
+  if (G < NBINS && grid > 0 && (uint64_t)grid * D_THREADS * D_ITEMS >= n) {
+    // fused single launch; slices of whole 512-request rows per CTA
+    const uint32_t rows = (n + D_THREADS - 1) / D_THREADS;
+    const uint32_t per_cta = ((rows + grid - 1) / grid) * D_THREADS;
+    bsort_dist_kernel<<<grid, D_THREADS, 0, st>>>(A, n, G, per_cta, key_lo, key_hi, b.bcount, b.gstart, b.cursor,
+                                                  b.kA, b.pA, ctl);
+    *launches += 1;
+    return;
+  }
+  bsort_hist_kernel<<<(n + H_THREADS * H_ITEMS - 1) / (H_THREADS * H_ITEMS), H_THREADS, 0, st>>>(
+      A, n, G, b.bcount, b.bin2grp, b.gstart, b.cursor, ctl);
   const size_t sm = NBINS * sizeof(uint16_t) + (size_t)G * sizeof(uint32_t);
   bsort_scatter_kernel<<<(n + S_TILE - 1) / S_TILE, S_THREADS, sm, st>>>(A, n, G, key_lo, key_hi, b.bin2grp,
                                                                          b.cursor, b.kA, b.pA, ctl);

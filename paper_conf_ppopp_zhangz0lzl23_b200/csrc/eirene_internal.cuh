@@ -54,7 +54,7 @@ struct BatchCtl {
   uint32_t invalid;
   uint32_t tile_ctr[16];
   uint32_t nseg, nq, nw, height;
-  uint32_t nlong, pad_;
+  uint32_t nlong, gbar;   // gbar: grid barrier of bsort_dist_kernel
   unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
   uint32_t dbg[8];   // watchdog diagnostics
 };
@@ -199,7 +199,7 @@ struct BSortBufs {
   uint32_t* bcount;  // [NBINS] zeroed per batch
   uint16_t* bin2grp; // [NBINS]
   uint32_t* gstart;  // [NBINS + 1] group starts
-  uint32_t* cursor;  // [NBINS] group fill cursors
+  uint32_t* cursor;  // [NBINS] group fill cursors (zeroed per batch)
 };
 uint32_t bsort_groups(uint32_t n, int num_sms);
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
