@@ -66,19 +66,21 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
 // First node of the batch graph: zero the per-batch control region (BatchCtl,
 // bin counts, group look-back words) and publish the batch's pointers.
 __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys,
-                                                        const uint64_t* vals, uint64_t* results, BatchCtl* host_ctl,
+                                                        const uint64_t* vals, uint64_t* results, BatchCtl* ctl_out,
                                                         uint4* zero, uint32_t zero_n16) {
-  for (uint32_t i = threadIdx.x; i < zero_n16; i += blockDim.x) zero[i] = make_uint4(0, 0, 0, 0);
-  if (threadIdx.x == 0) {
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
+    zero[i] = make_uint4(0, 0, 0, 0);
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
     dst->ops = ops;
     dst->keys = keys;
     dst->vals = vals;
     dst->results = results;
-    dst->host_ctl = host_ctl;
+    dst->ctl_out = ctl_out;
   }
 }
 
 // kernels in one batch graph: set_args, 1-2 sort, group, query, update, result_long
+constexpr int SET_ARGS_CTAS = 4;
 constexpr int MAX_GRAPHS = 8;
 
 struct GraphEntry {
@@ -117,8 +119,9 @@ struct eirene_tree {
   unsigned char* zero_region = nullptr;
   size_t zero_bytes = 0;
   BatchCtl* ctl = nullptr;
-  BatchCtl* host_ctl = nullptr;   // pinned, mapped [RING]
-  BatchCtl* host_ctl_dev = nullptr;   // its device address
+  BatchCtl* host_ctl = nullptr;   // pinned [RING]: landing buffer of eirene_results
+  BatchCtl* ctl_ring = nullptr;   // device [RING]: each batch's final BatchCtl (written by result_long)
+  cudaStream_t res_stream = nullptr;
   cudaStream_t h2d_stream = nullptr;
   cudaEvent_t h2d_done[2] = {}, comp_done[2] = {};
   bool slot_used[2] = {false, false};
@@ -257,6 +260,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->bs.gstart, NBINS + 1);
   AL(h->bs.bin2grp, NBINS);
   AL(h->dargs, 1);
+  AL(h->ctl_ring, RING);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
   {
@@ -286,9 +290,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     }
   }
 #undef AL
-  if (e == cudaSuccess)
-    e = cudaHostAlloc(reinterpret_cast<void**>(&h->host_ctl), sizeof(BatchCtl) * RING, cudaHostAllocMapped);
-  if (e == cudaSuccess) e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&h->host_ctl_dev), h->host_ctl, 0);
+  if (e == cudaSuccess) e = cudaMallocHost(reinterpret_cast<void**>(&h->host_ctl), sizeof(BatchCtl) * RING);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->res_stream, cudaStreamNonBlocking);
   for (int i = 0; i < RING && e == cudaSuccess; ++i) {
     e = cudaEventCreateWithFlags(&h->ring[i].done, cudaEventDisableTiming);
     for (int s = 0; s < NSTAGE && e == cudaSuccess; ++s) e = cudaEventCreate(&h->ring[i].st[s]);
@@ -332,6 +335,7 @@ int eirene_destroy(eirene_handle h) {
   }
   for (void* p : h->allocs) cudaFree(p);
   if (h->host_ctl) cudaFreeHost(h->host_ctl);
+  if (h->res_stream) cudaStreamDestroy(h->res_stream);
   delete h;
   return EIRENE_OK;
 }
@@ -395,11 +399,11 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     return cudaSuccess;
   };
   auto rec = [&](int i, cudaStream_t s) { cudaEventRecord(r.st[i], s); };
-  BatchCtl* host_ctl_slot = h->host_ctl_dev + tk % RING;
+  BatchCtl* ctl_slot = h->ctl_ring + tk % RING;
   uint4* zero16 = reinterpret_cast<uint4*>(h->zero_region);
   uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
   auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
-    set_args_kernel<<<1, 1024, 0, s>>>(h->dargs, ops, keys, vals, results, host_ctl_slot, zero16, zero_n16);
+    set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, results, ctl_slot, zero16, zero_n16);
     ++launches;
     if (args_node) {
       cudaError_t e = last_node(s, args_node);
@@ -447,10 +451,10 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       g = &e;
     }
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
-                      const_cast<uint64_t**>(&vals), &results, &host_ctl_slot, &zero16, &zero_n16};
+                      const_cast<uint64_t**>(&vals), &results, &ctl_slot, &zero16, &zero_n16};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
-    p.gridDim = dim3(1);
+    p.gridDim = dim3(SET_ARGS_CTAS);
     p.blockDim = dim3(1024);
     p.sharedMemBytes = 0;
     p.kernelParams = params;
@@ -508,6 +512,11 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) 
   Rec& r = h->ring[ticket % RING];
   if (!r.used || r.ticket != ticket) return EIRENE_ESTATE;
   CK(cudaEventSynchronize(r.done));
+  // the batch's BatchCtl stays on the device (no copy on the batch's stream);
+  // fetched here, off the GPU pipeline
+  CK(cudaMemcpyAsync(&h->host_ctl[ticket % RING], h->ctl_ring + ticket % RING, sizeof(BatchCtl),
+                     cudaMemcpyDeviceToHost, h->res_stream));
+  CK(cudaStreamSynchronize(h->res_stream));
   const BatchCtl& c = h->host_ctl[ticket % RING];
   if (stats) {
     std::memset(stats, 0, sizeof(*stats));

@@ -94,7 +94,7 @@ struct BatchArgs {
   const uint64_t* keys;
   const uint64_t* vals;
   uint64_t* results;
-  BatchCtl* host_ctl;   // mapped pinned ring slot: the batch's BatchCtl is written here at the end
+  BatchCtl* ctl_out;    // device ring slot: the batch's final BatchCtl is copied here at the end
 };
 
 // tile counters

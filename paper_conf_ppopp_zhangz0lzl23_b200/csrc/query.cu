@@ -124,10 +124,10 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
                                                             int dbgprint) {
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     // end of the batch (the last kernel; nothing below changes ctl): final
-    // status and height, then the whole BatchCtl to the mapped host ring slot
+    // status and height, then the whole BatchCtl to the batch's ring slot
     if (ctl->invalid) ctl->status = EIRENE_EINVAL;
     ctl->height = (uint32_t)(hdr->root_word >> 32);
-    *A->host_ctl = *ctl;
+    *A->ctl_out = *ctl;
     if (dbgprint)
       printf("[eirene dbg] %u %u %u %u %u %u %u %u\n", ctl->dbg[0], ctl->dbg[1], ctl->dbg[2], ctl->dbg[3],
              ctl->dbg[4], ctl->dbg[5], ctl->dbg[6], ctl->dbg[7]);
@@ -169,7 +169,7 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
 void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
                    const TreeHdr* hdr, int dbgprint, cudaStream_t st, int* launches) {
   (void)n;
-  result_long_kernel<<<148, 1024, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr, dbgprint);
+  result_long_kernel<<<64, 1024, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr, dbgprint);
   ++*launches;
 }
 
