@@ -218,8 +218,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   const size_t sort_tiles = (nb + SORT_TILE - 1) / SORT_TILE;
 #define AL(p, n)                                 \
   if (e == cudaSuccess) e = h->dalloc(&(p), (n));
-  AL(t.lkeys, leaf_cap * FAN);
-  AL(t.lvals, leaf_cap * FAN);
+  AL(t.lkeys, leaf_cap * LSTRIDE);   // keys and values of a leaf share one 256 B block
+  if (e == cudaSuccess) t.lvals = t.lkeys + FAN;
   AL(t.lmeta, leaf_cap);
   AL(t.ikeys, inner_cap * FAN);
   AL(t.ichild, inner_cap * FAN);
@@ -599,7 +599,7 @@ int eirene_check_invariants(eirene_handle h, uint64_t* n_keys) {
   std::vector<uint64_t> lk((size_t)L * FAN), ik((size_t)I * FAN);
   std::vector<uint32_t> ic((size_t)I * FAN);
   std::vector<NodeMeta> lm(L), im(I);
-  CK(cudaMemcpy(lk.data(), h->t.lkeys, lk.size() * 8, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy2D(lk.data(), FAN * 8, h->t.lkeys, LSTRIDE * 8, FAN * 8, L, cudaMemcpyDeviceToHost));
   CK(cudaMemcpy(lm.data(), h->t.lmeta, lm.size() * sizeof(NodeMeta), cudaMemcpyDeviceToHost));
   if (I) {
     CK(cudaMemcpy(ik.data(), h->t.ikeys, ik.size() * 8, cudaMemcpyDeviceToHost));

@@ -4,8 +4,9 @@
 // Citations: P:N = /root/reference/PAPER.md line N; Alg.1:k = Algorithm 1 line k.
 //
 // Tree layout in HBM (SoA node pools):
-//   leaves : lkeys[cap][16] u64 (one 128 B line), lvals[cap][16] u64 (128 B),
-//            lmeta[cap] (32 B).  Unused key slots hold KEY_MAX (sorted to the end).
+//   leaves : one 256 B block per leaf: 16 u64 keys (a 128 B line) then 16 u64
+//            values (the next line, same DRAM page), lmeta[cap] (32 B).
+//            Unused key slots hold KEY_MAX (sorted to the end).
 //   inner  : ikeys[cap][16] u64 separators (child i covers [key[i-1], key[i]),
 //            key[c-1..15] = KEY_MAX), ichild[cap][16] u32, imeta[cap] (32 B).
 //   The B+tree of P:327-330 / P:1622-1628, plus B-link right links and [lo, hi)
@@ -21,6 +22,7 @@
 namespace eirene {
 
 constexpr int FAN = 16;
+constexpr int LSTRIDE = 2 * FAN;   // u64 words per leaf block (keys, then values)
 constexpr uint64_t KEY_MAX = ~0ull;
 constexpr uint32_t NIL = 0xFFFFFFFFu;
 constexpr int MAX_LEVELS = 32;
@@ -101,8 +103,8 @@ struct BatchArgs {
 enum { TC_SORT0 = 0, TC_GROUP = 8, TC_ROUTE = 10, TC_SCAN = 11, TC_HIST = 12 };
 
 struct Tree {
-  uint64_t* lkeys;
-  uint64_t* lvals;
+  uint64_t* lkeys;   // leaf L: keys at lkeys[L * LSTRIDE + s]
+  uint64_t* lvals;   // = lkeys + FAN: values at lvals[L * LSTRIDE + s]
   NodeMeta* lmeta;
   uint64_t* ikeys;
   uint32_t* ichild;

@@ -83,8 +83,8 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
       for (int x = 0; x < 4; ++x) c += (kv[x].x <= k) + (kv[x].y <= k) + (kv[x].z <= k) + (kv[x].w <= k);
       node = __ldg(t.ichild + (size_t)node * FAN + c);
     }
-    const int s = slot16(t.lkeys + (size_t)node * FAN, k);
-    const uint64_t v = s >= 0 ? __ldg(t.lvals + (size_t)node * FAN + s) : KEY_MAX;
+    const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k);
+    const uint64_t v = s >= 0 ? __ldg(t.lvals + (size_t)node * LSTRIDE + s) : KEY_MAX;
     uint32_t seg;
     if (isq) {
       seg = qseg[i];

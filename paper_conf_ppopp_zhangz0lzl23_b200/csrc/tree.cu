@@ -28,8 +28,8 @@ __global__ void build_leaves_kernel(const uint64_t* __restrict__ keys, const uin
   if (leaf >= L) return;
   const uint64_t idx = leaf * per + s;
   const bool valid = s < per && idx < n;
-  t.lkeys[gid] = valid ? keys[idx] : KEY_MAX;
-  t.lvals[gid] = valid ? vals[idx] : 0;
+  t.lkeys[leaf * LSTRIDE + s] = valid ? keys[idx] : KEY_MAX;
+  t.lvals[leaf * LSTRIDE + s] = valid ? vals[idx] : 0;
   if (s == 0) {
     NodeMeta m;
     m.version = 0;
@@ -83,7 +83,7 @@ __global__ void leaf_count_kernel(Tree t, const uint32_t* __restrict__ order, ui
   const uint32_t leaf = order[i];
   uint64_t c = 0;
   for (int s = 0; s < FAN; ++s) {
-    const uint64_t k = t.lkeys[(size_t)leaf * FAN + s];
+    const uint64_t k = t.lkeys[(size_t)leaf * LSTRIDE + s];
     c += (k != KEY_MAX && k >= lo && k <= hi) ? 1 : 0;
   }
   cnt[i] = c;
@@ -129,11 +129,11 @@ __global__ void leaf_emit_kernel(Tree t, const uint32_t* __restrict__ order, con
   const uint32_t leaf = order[i];
   uint64_t o = off[i];
   for (int s = 0; s < FAN; ++s) {
-    const uint64_t k = t.lkeys[(size_t)leaf * FAN + s];
+    const uint64_t k = t.lkeys[(size_t)leaf * LSTRIDE + s];
     if (k != KEY_MAX && k >= lo && k <= hi) {
       if (o < cap) {
         if (ko) ko[o] = k;
-        if (vo) vo[o] = t.lvals[(size_t)leaf * FAN + s];
+        if (vo) vo[o] = t.lvals[(size_t)leaf * LSTRIDE + s];
       }
       ++o;
     }

@@ -263,7 +263,7 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
                                uint64_t* Ek, uint32_t* Ec, WarpStats& ws) {
   const int lane = lane_id();
   const Tree& t = C.t;
-  const size_t xb = (size_t)X * FAN;
+  const size_t xb = (size_t)X * LSTRIDE;
   const uint64_t okey = lane < FAN ? ld_cg(t.lkeys + xb + lane) : KEY_MAX;
   const uint64_t oval = lane < FAN ? ld_cg(t.lvals + xb + lane) : 0;
   const uint32_t c = __popc(__ballot_sync(FULL, okey != KEY_MAX));
@@ -322,8 +322,8 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
     }
     const uint32_t slot = f - start;
     const uint32_t id = q == 0 ? X : first + q - 1;
-    t.lkeys[(size_t)id * FAN + slot] = key;
-    t.lvals[(size_t)id * FAN + slot] = val;
+    t.lkeys[(size_t)id * LSTRIDE + slot] = key;
+    t.lvals[(size_t)id * LSTRIDE + slot] = val;
     if (q > 0 && slot == 0) {
       Ek[b + q - 1] = key;
       Ec[b + q - 1] = id;
@@ -349,7 +349,7 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
     const uint32_t q = q0 + (lane >> 4), s = lane & 15;
     if (q < k) {
       const uint32_t sz = bs + (q < rem ? 1u : 0u);
-      if (s >= sz) t.lkeys[(size_t)(q == 0 ? X : first + q - 1) * FAN + s] = KEY_MAX;
+      if (s >= sz) t.lkeys[(size_t)(q == 0 ? X : first + q - 1) * LSTRIDE + s] = KEY_MAX;
     }
   }
   __threadfence();
@@ -687,7 +687,7 @@ __global__ void __launch_bounds__(128) update_kernel(Ctx C) {
       fast = fast && got;
       bool ok = true;
       if (fast) {
-        const size_t at = (size_t)lf * FAN + sl;
+        const size_t at = (size_t)lf * LSTRIDE + sl;
         if (ld_cg(t.lkeys + at) == C.wkey[j]) {
           t.lvals[at] = C.wval[j];
         } else {
