@@ -309,21 +309,32 @@ def run_ours(args):
         hres = [torch.empty(batch_n, dtype=torch.uint64).pin_memory() for _ in hb]
         tk = tree.submit_host(*pin[0], hres[0])   # warm the path
         tree.results(tk)
+        # first DMA touch of each freshly pinned buffer (IOMMU / page mapping) is a
+        # one-time cost a serving process with long-lived staging buffers never
+        # pays: touch every buffer once, untimed (no batch is run)
+        for x, r_ in zip(pin, hres):
+            for t_ in x:
+                torch.empty(t_.shape, dtype=t_.dtype, device=dev).copy_(t_, non_blocking=True)
+            r_.copy_(torch.empty(r_.shape, dtype=r_.dtype, device=dev), non_blocking=True)
         torch.cuda.synchronize()
         a = torch.cuda.Event(enable_timing=True)
         z = torch.cuda.Event(enable_timing=True)
         a.record(stream)
         tks = [tree.submit_host(*pin[i], hres[i]) for i in range(1, len(pin))]
-        z.record(stream)
         for t_ in tks:
-            tree.results(t_)
+            tree.results(t_)   # waits for the batch's D2H (library's d2h stream)
+        z.record(stream)       # after the last results() returned: covers every H2D, kernel and D2H
         torch.cuda.synchronize()
         e_ms = a.elapsed_time(z)
         n_e = len(pin) - 1
+        # bytes actually moved per step: ops + keys copied; values of upserts
+        # read zero-copy from the pinned buffer by the distribution kernel
+        ups = np.mean([int(np.count_nonzero((x[0] == W.UPDATE) | (x[0] == W.INSERT))) for x in hb[1:]])
         e2e = {"value": batch_n * n_e / (e_ms * 1e-3) / 1e9, "unit": "Greq/s",
-               "h2d_bytes_per_step": int(batch_n * 17), "d2h_bytes_per_step": int(batch_n * 8),
+               "h2d_bytes_per_step": int(batch_n * 9 + 8 * ups), "d2h_bytes_per_step": int(batch_n * 8),
                "steps": n_e, "path": "eirene_submit_batch_host (pinned host buffers; H2D of batch b+1 on the "
-                                     "library's copy stream overlaps batch b's kernels + D2H)"}
+                                     "library's copy stream and D2H of batch b-1 on its d2h stream overlap "
+                                     "batch b's kernels; upsert values read zero-copy)"}
     elif world > 1:
         e2e = {"value": None, "unit": "Greq/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
                "note": "multi-GPU e2e not measured this round"}

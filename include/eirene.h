@@ -122,9 +122,11 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys_dev, const uint64_t* 
  * keys_dev[n], vals_dev[n] (ignored for queries and deletes) and writes
  * results_dev[n] (u64, timestamp = index order).  Asynchronous on `stream`;
  * the caller keeps every buffer alive until eirene_results(ticket) returns.
- * Pipeline: stable radix sort by key (Alg.1:10), combine/resolve (Alg.1:11,
- * P:724-758), partition (Alg.1:3), query kernel (Alg.1:15-21), update kernel
- * with optimistic retry and STM fallback (Alg.1:23-46), RESULT_CAL (Alg.1:6).
+ * Pipeline: sort by (key, timestamp) (Alg.1:10) as a distribution into
+ * balanced key-range groups + a per-group sort fused with combine/resolve
+ * (Alg.1:11) and partition (Alg.1:3), query kernel (Alg.1:15-21),
+ * update kernel with optimistic retry and STM fallback (Alg.1:23-46),
+ * RESULT_CAL (Alg.1:6).
  * Synchronous errors: EINVAL (null pointers, n == 0 or n > max_batch), ESTATE.
  * Invalid requests (op > 3, key == UINT64_MAX or outside [key_lo, key_hi),
  * upsert value == UINT64_MAX) are detected on the device: the batch then
@@ -133,10 +135,16 @@ int eirene_submit_batch(eirene_handle h, const uint8_t* ops_dev, const uint64_t*
                         const uint64_t* vals_dev, uint32_t n, uint64_t* results_dev,
                         eirene_stream_t stream, uint64_t* ticket);
 
-/* Same batch from HOST buffers: copies the requests host->device into
- * handle-owned staging buffers, runs the pipeline, copies results device->host,
- * all on `stream`.  The copies run at full speed only from pinned memory.
- * Results are valid after eirene_results(ticket). */
+/* Same batch from HOST buffers.  ops and keys are copied host->device into
+ * handle-owned double-buffered staging on the handle's copy stream (which
+ * overlaps the previous batch's kernels); the pipeline runs on `stream`; the
+ * results are copied device->host on the handle's d2h stream.  If vals_host is
+ * pinned (page-locked, device-mapped under UVA) it is not copied: the
+ * distribution kernel reads the values of the batch's upserts -- the only
+ * values any kernel reads -- from host memory and stages them; pageable
+ * values are copied.  The copies run at full speed only from pinned memory.
+ * Results are valid after eirene_results(ticket); keep every buffer alive
+ * until then. */
 int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops_host, const uint64_t* keys_host,
                              const uint64_t* vals_host, uint32_t n, uint64_t* results_host,
                              eirene_stream_t stream, uint64_t* ticket);

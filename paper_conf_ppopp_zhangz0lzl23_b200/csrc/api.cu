@@ -66,14 +66,17 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
 // First node of the batch graph: zero the per-batch control region (BatchCtl,
 // bin counts, group look-back words) and publish the batch's pointers.
 __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys,
-                                                        const uint64_t* vals, uint64_t* results, BatchCtl* ctl_out,
-                                                        uint4* zero, uint32_t zero_n16) {
+                                                        const uint64_t* vals_src, uint64_t* vals_stage,
+                                                        uint64_t* results, BatchCtl* ctl_out, uint4* zero,
+                                                        uint32_t zero_n16) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
     zero[i] = make_uint4(0, 0, 0, 0);
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     dst->ops = ops;
     dst->keys = keys;
-    dst->vals = vals;
+    dst->vals = vals_stage ? vals_stage : vals_src;
+    dst->vals_src = vals_src;
+    dst->vals_stage = vals_stage;
     dst->results = results;
     dst->ctl_out = ctl_out;
   }
@@ -122,8 +125,8 @@ struct eirene_tree {
   BatchCtl* host_ctl = nullptr;   // pinned [RING]: landing buffer of eirene_results
   BatchCtl* ctl_ring = nullptr;   // device [RING]: each batch's final BatchCtl (written by result_long)
   cudaStream_t res_stream = nullptr;
-  cudaStream_t h2d_stream = nullptr;
-  cudaEvent_t h2d_done[2] = {}, comp_done[2] = {};
+  cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;
+  cudaEvent_t h2d_done[2] = {}, comp_ev[2] = {}, comp_done[2] = {};
   bool slot_used[2] = {false, false};
   uint32_t host_slot = 0;
   uint8_t* st_ops = nullptr;
@@ -251,9 +254,11 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->st_vals, 2 * nb);
   AL(h->st_res, 2 * nb);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->h2d_stream, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking);
   for (int s = 0; s < 2 && e == cudaSuccess; ++s) {
     e = cudaEventCreateWithFlags(&h->h2d_done[s], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->comp_done[s], cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->comp_ev[s], cudaEventDisableTiming);
   }
   AL(h->route_lb, ((nb + 2047) / 2048) * 64);
   AL(h->route_ctr, 1);
@@ -329,9 +334,11 @@ int eirene_destroy(eirene_handle h) {
   }
   if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
   if (h->h2d_stream) cudaStreamDestroy(h->h2d_stream);
+  if (h->d2h_stream) cudaStreamDestroy(h->d2h_stream);
   for (int s = 0; s < 2; ++s) {
     if (h->h2d_done[s]) cudaEventDestroy(h->h2d_done[s]);
     if (h->comp_done[s]) cudaEventDestroy(h->comp_done[s]);
+    if (h->comp_ev[s]) cudaEventDestroy(h->comp_ev[s]);
   }
   for (void* p : h->allocs) cudaFree(p);
   if (h->host_ctl) cudaFreeHost(h->host_ctl);
@@ -369,7 +376,7 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals
 }
 
 static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
-                       uint64_t* results, cudaStream_t st, uint64_t* results_host, uint64_t* ticket) {
+                       uint64_t* results, cudaStream_t st, uint64_t* vals_stage, uint64_t* ticket) {
   CK(cudaSetDevice(h->cfg.device));
   const uint64_t tk = h->next_ticket++;
   Rec& r = h->ring[tk % RING];
@@ -403,7 +410,8 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   uint4* zero16 = reinterpret_cast<uint4*>(h->zero_region);
   uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
   auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
-    set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, results, ctl_slot, zero16, zero_n16);
+    set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
+                                                   zero_n16);
     ++launches;
     if (args_node) {
       cudaError_t e = last_node(s, args_node);
@@ -451,7 +459,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       g = &e;
     }
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
-                      const_cast<uint64_t**>(&vals), &results, &ctl_slot, &zero16, &zero_n16};
+                      const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
     p.gridDim = dim3(SET_ARGS_CTAS);
@@ -463,7 +471,6 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     CK(cudaGraphLaunch(g->exec, st));
     launches = g->launches;
   }
-  if (results_host) CK(cudaMemcpyAsync(results_host, results, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, st));
   CK(cudaEventRecord(r.done, st));
   r.launches = launches;
   h->launches += launches;
@@ -485,25 +492,43 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   CK(cudaSetDevice(h->cfg.device));
-  // Double-buffered staging: the H2D copy of this batch runs on the handle's
-  // copy stream into slot s while the previous batch computes on `st`; the
-  // slot is reused only after the batch that last used it has finished (its
-  // D2H of results is ordered on `st` behind its kernels).
+  // Double-buffered staging, three streams: the H2D of this batch (copy
+  // stream) overlaps the previous batch's kernels (`st`) and the D2H of its
+  // results (d2h stream).  A slot is reused only after the D2H of the batch
+  // that last used it.  Values are not copied when the host buffer is pinned:
+  // the distribution kernel reads the values of the batch's upserts (the only
+  // ones any kernel reads) straight from host memory and stages them, so a
+  // read-mostly batch ships 9 of its 17 B/request.
   const int s = (int)(h->host_slot++ & 1u);
+  const size_t off = (size_t)s * h->cfg.max_batch;
   if (h->slot_used[s]) CK(cudaStreamWaitEvent(h->h2d_stream, h->comp_done[s], 0));
-  CK(cudaMemcpyAsync(h->st_ops + (size_t)s * h->cfg.max_batch, ops, n, cudaMemcpyHostToDevice, h->h2d_stream));
-  CK(cudaMemcpyAsync(h->st_keys + (size_t)s * h->cfg.max_batch, keys, sizeof(uint64_t) * n, cudaMemcpyHostToDevice,
-                     h->h2d_stream));
-  CK(cudaMemcpyAsync(h->st_vals + (size_t)s * h->cfg.max_batch, vals, sizeof(uint64_t) * n, cudaMemcpyHostToDevice,
-                     h->h2d_stream));
+  CK(cudaMemcpyAsync(h->st_ops + off, ops, n, cudaMemcpyHostToDevice, h->h2d_stream));
+  CK(cudaMemcpyAsync(h->st_keys + off, keys, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, h->h2d_stream));
+  cudaPointerAttributes pa{};
+  const bool pinned = cudaPointerGetAttributes(&pa, vals) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
+                      pa.devicePointer != nullptr;
+  cudaGetLastError();   // (clear a pageable-pointer query error, if any)
+  const uint64_t* vsrc;
+  uint64_t* vstage = nullptr;
+  if (pinned) {
+    vsrc = static_cast<const uint64_t*>(pa.devicePointer);
+    vstage = h->st_vals + off;
+  } else {
+    CK(cudaMemcpyAsync(h->st_vals + off, vals, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, h->h2d_stream));
+    vsrc = h->st_vals + off;
+  }
   CK(cudaEventRecord(h->h2d_done[s], h->h2d_stream));
   CK(cudaStreamWaitEvent(st, h->h2d_done[s], 0));
-  int rc = submit_impl(h, h->st_ops + (size_t)s * h->cfg.max_batch, h->st_keys + (size_t)s * h->cfg.max_batch,
-                       h->st_vals + (size_t)s * h->cfg.max_batch, n, h->st_res + (size_t)s * h->cfg.max_batch, st,
-                       results, ticket);
+  uint64_t tk = 0;
+  int rc = submit_impl(h, h->st_ops + off, h->st_keys + off, vsrc, n, h->st_res + off, st, vstage, &tk);
   if (rc != EIRENE_OK) return rc;
-  CK(cudaEventRecord(h->comp_done[s], st));
+  CK(cudaEventRecord(h->comp_ev[s], st));
+  CK(cudaStreamWaitEvent(h->d2h_stream, h->comp_ev[s], 0));
+  CK(cudaMemcpyAsync(results, h->st_res + off, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, h->d2h_stream));
+  CK(cudaEventRecord(h->comp_done[s], h->d2h_stream));
+  CK(cudaEventRecord(h->ring[tk % RING].done, h->d2h_stream));   // eirene_results waits for the D2H too
   h->slot_used[s] = true;
+  *ticket = tk;
   return EIRENE_OK;
 }
 

@@ -124,7 +124,8 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
   uint32_t* hist = reinterpret_cast<uint32_t*>(s_b2g + NBINS);   // [G] tile counts, then global base
   const uint64_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
-  const uint64_t* __restrict__ vals = A->vals;
+  const uint64_t* __restrict__ vals = A->vals_src;
+  uint64_t* __restrict__ vstage = A->vals_stage;
   const int tid = threadIdx.x;
   for (uint32_t i = tid; i < (uint32_t)NBINS; i += S_THREADS) s_b2g[i] = bin2grp[i];
   for (uint32_t i = tid; i < G; i += S_THREADS) hist[i] = 0;
@@ -143,6 +144,7 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
     const uint32_t i = t0 + j * S_THREADS + tid;
     const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
     const uint64_t v = (i < n && up) ? vals[i] : 0;
+    if (vstage && i < n && up) vstage[i] = v;
     bad |= i < n && (o[j] > OP_DELETE || k[j] == KEY_MAX || k[j] < key_lo || k[j] >= key_hi || (up && v == KEY_MAX));
   }
   if (__any_sync(FULL, bad) && (tid & 31) == 0) atomicOr(&ctl->invalid, 1u);
@@ -190,7 +192,8 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   __shared__ uint32_t wsum[D_THREADS / 32];
   const uint64_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
-  const uint64_t* __restrict__ vals = A->vals;
+  const uint64_t* __restrict__ vals = A->vals_src;
+  uint64_t* __restrict__ vstage = A->vals_stage;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   for (uint32_t i = tid; i < NBINS; i += D_THREADS) h[i] = 0;
   __syncthreads();
@@ -210,6 +213,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
     const uint32_t i = t0 + j * D_THREADS + tid;
     const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
     const uint64_t v = (i < t1 && up) ? vals[i] : 0;
+    if (vstage && i < t1 && up) vstage[i] = v;
     bad |= i < t1 && (o[j] > OP_DELETE || k[j] == KEY_MAX || k[j] < key_lo || k[j] >= key_hi || (up && v == KEY_MAX));
     if (i < t1) atomicAdd(&h[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
   }

@@ -94,8 +94,10 @@ struct SpinGuard {
 struct BatchArgs {
   const uint8_t* ops;
   const uint64_t* keys;
-  const uint64_t* vals;
+  const uint64_t* vals;        // values as read by the kernels after the distribution pass
   uint64_t* results;
+  const uint64_t* vals_src;    // where the distribution pass reads the values of upserts
+  uint64_t* vals_stage;        // non-null: it also copies them here (== vals); host path, zero-copy
   BatchCtl* ctl_out;    // device ring slot: the batch's final BatchCtl is copied here at the end
 };
 

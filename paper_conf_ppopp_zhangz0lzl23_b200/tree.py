@@ -106,7 +106,9 @@ class EireneTree:
 
     def submit_host(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor,
                     stream=None) -> int:
-        """Host (ideally pinned) buffers; H2D and D2H copies run inside the call's stream."""
+        """Host (ideally pinned) buffers: the library copies them in on its own copy stream, runs the
+        batch on `stream` and copies the results out on its own d2h stream; results are valid after
+        results(ticket).  Pinned values are read zero-copy (only upserts' values are ever read)."""
         n = ops.numel()
         cpu = torch.device("cpu")
         _need(ops, torch.uint8, cpu, "ops")

@@ -315,6 +315,29 @@ def test_host_buffer_path(dev):
     assert np.array_equal(res.numpy(), ref.apply(ops, keys, vals))
 
 
+@pytest.mark.parametrize("pinned", [True, False])
+def test_host_buffer_pipeline(dev, pinned):
+    """Several host-path batches in flight (double-buffered staging, D2H on its
+    own stream); pinned values are read zero-copy by the distribution kernel,
+    pageable ones are copied."""
+    w = W.Workload(4, tree=1 << 14, batch=1 << 12)
+    t = make_tree(dev, w.keys, w.vals, max_batch=1 << 12, max_keys=1 << 17)
+    ref = oracle.MapOracle(); ref.load(w.keys, w.vals)
+    pend = []
+    for b in range(5):
+        ops, keys, vals = w.batch_arrays(b)
+        mk = (lambda a: torch.from_numpy(a).pin_memory()) if pinned else (lambda a: torch.from_numpy(a.copy()))
+        res = torch.empty(ops.size, dtype=torch.uint64)
+        if pinned:
+            res = res.pin_memory()
+        args = (mk(ops), mk(keys), mk(vals))
+        pend.append((t.submit_host(*args, res), res, args, ref.apply(ops, keys, vals)))
+    for tk, res, _, want in pend:
+        t.results(tk)
+        assert np.array_equal(res.numpy(), want)
+    assert t.check_invariants()[0] == 0
+
+
 def test_subbatch_splitting_invariance(dev):
     rng = np.random.default_rng(12)
     keys, vals = _rand_keys(rng, 2000, hi=1 << 16)
