@@ -22,6 +22,7 @@ using namespace eirene;
 namespace {
 
 constexpr int RING = 64;
+constexpr int HOST_SLOTS = 3;   // host-path staging depth: H2D(b+1), kernels(b), D2H(b-1) in flight
 constexpr int NSTAGE = 6;   // events: before sort, after sort / group / query / update / result
 
 std::mutex g_err_mu;
@@ -126,8 +127,8 @@ struct eirene_tree {
   BatchCtl* ctl_ring = nullptr;   // device [RING]: each batch's final BatchCtl (written by result_long)
   cudaStream_t res_stream = nullptr;
   cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;
-  cudaEvent_t h2d_done[2] = {}, comp_ev[2] = {}, comp_done[2] = {};
-  bool slot_used[2] = {false, false};
+  cudaEvent_t h2d_done[HOST_SLOTS] = {}, comp_ev[HOST_SLOTS] = {}, comp_done[HOST_SLOTS] = {};
+  bool slot_used[HOST_SLOTS] = {};
   uint32_t host_slot = 0;
   uint8_t* st_ops = nullptr;
   uint64_t* st_keys = nullptr;
@@ -249,13 +250,13 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->up.entA_child, nb + 64);
   AL(h->up.entB_key, nb + 64);
   AL(h->up.entB_child, nb + 64);
-  AL(h->st_ops, 2 * nb);
-  AL(h->st_keys, 2 * nb);
-  AL(h->st_vals, 2 * nb);
-  AL(h->st_res, 2 * nb);
+  AL(h->st_ops, HOST_SLOTS * nb);
+  AL(h->st_keys, HOST_SLOTS * nb);
+  AL(h->st_vals, HOST_SLOTS * nb);
+  AL(h->st_res, HOST_SLOTS * nb);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->h2d_stream, cudaStreamNonBlocking);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->d2h_stream, cudaStreamNonBlocking);
-  for (int s = 0; s < 2 && e == cudaSuccess; ++s) {
+  for (int s = 0; s < HOST_SLOTS && e == cudaSuccess; ++s) {
     e = cudaEventCreateWithFlags(&h->h2d_done[s], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->comp_done[s], cudaEventDisableTiming);
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->comp_ev[s], cudaEventDisableTiming);
@@ -335,7 +336,7 @@ int eirene_destroy(eirene_handle h) {
   if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
   if (h->h2d_stream) cudaStreamDestroy(h->h2d_stream);
   if (h->d2h_stream) cudaStreamDestroy(h->d2h_stream);
-  for (int s = 0; s < 2; ++s) {
+  for (int s = 0; s < HOST_SLOTS; ++s) {
     if (h->h2d_done[s]) cudaEventDestroy(h->h2d_done[s]);
     if (h->comp_done[s]) cudaEventDestroy(h->comp_done[s]);
     if (h->comp_ev[s]) cudaEventDestroy(h->comp_ev[s]);
@@ -492,14 +493,14 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   CK(cudaSetDevice(h->cfg.device));
-  // Double-buffered staging, three streams: the H2D of this batch (copy
+  // Triple-buffered staging (HOST_SLOTS), three streams: the H2D of this batch (copy
   // stream) overlaps the previous batch's kernels (`st`) and the D2H of its
   // results (d2h stream).  A slot is reused only after the D2H of the batch
   // that last used it.  Values are not copied when the host buffer is pinned:
   // the distribution kernel reads the values of the batch's upserts (the only
   // ones any kernel reads) straight from host memory and stages them, so a
   // read-mostly batch ships 9 of its 17 B/request.
-  const int s = (int)(h->host_slot++ & 1u);
+  const int s = (int)(h->host_slot++ % HOST_SLOTS);
   const size_t off = (size_t)s * h->cfg.max_batch;
   if (h->slot_used[s]) CK(cudaStreamWaitEvent(h->h2d_stream, h->comp_done[s], 0));
   CK(cudaMemcpyAsync(h->st_ops + off, ops, n, cudaMemcpyHostToDevice, h->h2d_stream));
