@@ -64,6 +64,12 @@ def lib():
             "orc_bt_corrupt": (ctypes.c_int, [_vp, ctypes.c_int]),
             "orc_comb_apply": (ctypes.c_int, [_vp, _u8p, _u64p, _u64p, ctypes.c_uint64, _u64p, _u32p, _u32p,
                                               _u64p, _u8p, _u64p, _u64p, _u64p]),
+            "orc_map_apply_range": (ctypes.c_int, [_vp, _u8p, _u64p, _u64p, ctypes.c_uint64, _u64p, ctypes.c_uint32,
+                                                   _u64p, _u64p]),
+            "orc_bt_apply_range": (ctypes.c_int, [_vp, _u8p, _u64p, _u64p, ctypes.c_uint64, _u64p, ctypes.c_uint32,
+                                                  _u64p, _u64p]),
+            "orc_comb_apply_range": (ctypes.c_int, [_vp, _u8p, _u64p, _u64p, ctypes.c_uint64, _u64p, ctypes.c_uint32,
+                                                    _u64p, _u64p, _u64p]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -115,6 +121,22 @@ class _Engine:
         if rc != 0:
             raise ValueError("oracle apply: invalid request (op > 3, key == UINT64_MAX, or upsert of UINT64_MAX)")
         return res
+
+    def apply_range(self, ops, keys, vals, cap: int):
+        """Batch with range queries (op RANGE = 4: key = l, val = u, inclusive).
+        Returns (results[n], rkeys[n, cap], rvals[n, cap]); for a range request
+        results[i] = pairs written (first `cap` of [l, u] in key order), rows of
+        non-range requests and unused slots are left zero."""
+        ops, keys, vals = _req(ops, keys, vals)
+        n = ops.size
+        res = np.empty(n, dtype=np.uint64)
+        rk = np.zeros((n, max(cap, 1)), dtype=np.uint64)
+        rv = np.zeros((n, max(cap, 1)), dtype=np.uint64)
+        rc = getattr(self.L, f"orc_{self._pre}_apply_range")(self.h, _p(ops, _u8p), _p(keys, _u64p), _p(vals, _u64p),
+                                                             n, _p(res, _u64p), cap, _p(rk, _u64p), _p(rv, _u64p))
+        if rc != 0:
+            raise ValueError("oracle apply_range: invalid request")
+        return res, rk[:, :cap], rv[:, :cap]
 
     def size(self) -> int:
         return int(getattr(self.L, f"orc_{self._pre}_size")(self.h))
@@ -178,3 +200,23 @@ def combine_apply(m: MapOracle, ops, keys, vals):
     mi = ni.value
     return dict(results=res, sorted_ts=sts, seg=seg, issued_key=ik[:mi], issued_op=io[:mi],
                 issued_val=iv[:mi], n_issued=mi, n_issued_w=nw.value)
+
+
+RANGE = 4
+
+
+def combine_apply_range(m: MapOracle, ops, keys, vals, cap: int):
+    """Engine (iii) with range queries: the artificial-query mechanism of
+    P:920-938 around Algorithm 1, on MapOracle `m` (mutated).  Returns
+    (results[n], rkeys[n, cap], rvals[n, cap], n_artificial)."""
+    ops, keys, vals = _req(ops, keys, vals)
+    n = ops.size
+    res = np.empty(n, dtype=np.uint64)
+    rk = np.zeros((n, max(cap, 1)), dtype=np.uint64)
+    rv = np.zeros((n, max(cap, 1)), dtype=np.uint64)
+    na = ctypes.c_uint64(0)
+    rc = lib().orc_comb_apply_range(m.h, _p(ops, _u8p), _p(keys, _u64p), _p(vals, _u64p), n, _p(res, _u64p), cap,
+                                    _p(rk, _u64p), _p(rv, _u64p), ctypes.byref(na))
+    if rc != 0:
+        raise ValueError("oracle combine_apply_range: invalid request")
+    return res, rk[:, :cap], rv[:, :cap], na.value

@@ -45,7 +45,7 @@ extern "C" {
 #endif
 
 #define ORC_NOT_FOUND UINT64_MAX
-enum { ORC_QUERY = 0, ORC_UPDATE = 1, ORC_INSERT = 2, ORC_DELETE = 3 };
+enum { ORC_QUERY = 0, ORC_UPDATE = 1, ORC_INSERT = 2, ORC_DELETE = 3, ORC_RANGE = 4 };
 
 /* ---- engine (i): std::map definition ---- */
 void*    orc_map_new(void);
@@ -90,6 +90,36 @@ int      orc_comb_apply(void* map_h, const uint8_t* ops, const uint64_t* keys,
                         uint32_t* sorted_ts, uint32_t* seg_of_sorted,
                         uint64_t* issued_key, uint8_t* issued_op, uint64_t* issued_val,
                         uint64_t* n_issued, uint64_t* n_issued_w);
+
+/* ---- range queries R(l, u) ----
+ * A batch may hold ORC_RANGE requests: key = lower bound l, val = upper
+ * bound u, both inclusive (§8(c) reading 23).  The result of range request i
+ * is the set of pairs (k, v) of the state visible immediately before i
+ * (linearizability) with l <= k <= u, in ascending key order,
+ * limited to its first `cap` pairs (reading R1): results[i] = the
+ * number of pairs written, the pairs go to rkeys[i*cap + j], rvals[i*cap + j].
+ * l > u is an empty range.  Point requests are as in *_apply.
+ *   orc_map_apply_range  : engine (i), the plain definition.
+ *   orc_bt_apply_range   : engine (ii), leaf-chain walk of the B+tree.
+ *   orc_comb_apply_range : engine (iii), the paper's mechanism step by step:
+ *     sort with range queries placed by their lower bound; scan;
+ *     an artificial query Qr(k)@t for every key k in [l, u] that has update
+ *     requests in the batch, inserted into k's sequence by timestamp
+ *     (P:925-935); combine / partition / query / update / RESULT_CAL as
+ *     Alg.1 with the range query in the query kernel reading the tree "in
+ *     the original manner"; then every key with an artificial query
+ *     takes that query's result (NOT_FOUND removes it, a value
+ *     adds or replaces it).  *n_artificial = artificial queries generated. */
+int      orc_map_apply_range(void* h, const uint8_t* ops, const uint64_t* keys,
+                             const uint64_t* vals, uint64_t n, uint64_t* results,
+                             uint32_t cap, uint64_t* rkeys, uint64_t* rvals);
+int      orc_bt_apply_range(void* h, const uint8_t* ops, const uint64_t* keys,
+                            const uint64_t* vals, uint64_t n, uint64_t* results,
+                            uint32_t cap, uint64_t* rkeys, uint64_t* rvals);
+int      orc_comb_apply_range(void* map_h, const uint8_t* ops, const uint64_t* keys,
+                              const uint64_t* vals, uint64_t n, uint64_t* results,
+                              uint32_t cap, uint64_t* rkeys, uint64_t* rvals,
+                              uint64_t* n_artificial);
 
 #ifdef __cplusplus
 }
