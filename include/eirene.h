@@ -53,8 +53,9 @@ enum {
                            tree must be discarded                              */
 };
 
-/* Request types. */
-enum { EIRENE_QUERY = 0, EIRENE_UPDATE = 1, EIRENE_INSERT = 2, EIRENE_DELETE = 3 };
+/* Request types; EIRENE_RANGE = range query R(l, u),
+ * accepted only by eirene_submit_batch_range. */
+enum { EIRENE_QUERY = 0, EIRENE_UPDATE = 1, EIRENE_INSERT = 2, EIRENE_DELETE = 3, EIRENE_RANGE = 4 };
 
 /* eirene_config.flags */
 enum {
@@ -101,6 +102,8 @@ typedef struct {
   float stage_ms[8];          /* EIRENE_F_TIMING: [0] sort (bucket scatter), [1] group (bucket
                                  sort + combine + partition), [2] query, [3] update, [4] result,
                                  [5], [6] unused, [7] total                                    */
+  uint64_t ranges;            /* range queries in the batch (eirene_submit_batch_range)         */
+  uint64_t artificial;        /* artificial queries resolved for them               */
 } eirene_batch_stats;
 
 /* Creates a tree (one empty leaf) on cfg->device and allocates every pool and
@@ -148,6 +151,29 @@ int eirene_submit_batch(eirene_handle h, const uint8_t* ops_dev, const uint64_t*
 int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops_host, const uint64_t* keys_host,
                              const uint64_t* vals_host, uint32_t n, uint64_t* results_host,
                              eirene_stream_t stream, uint64_t* ticket);
+
+/* Same as eirene_submit_batch, and the batch may also hold range queries
+ * (§4.1.2): ops_dev[i] == EIRENE_RANGE with
+ * keys_dev[i] = l and vals_dev[i] = u asks for the pairs with l <= key <= u
+ * (inclusive, any u64 bounds; l > u is empty) of the state visible
+ * immediately before request i (linearizable), in ascending key
+ * order, limited to the first `cap` pairs (reading R1).  They go to
+ * range_keys_dev[i*cap + j] / range_vals_dev[i*cap + j] (caller-owned device
+ * buffers of n*cap u64 each; rows of other requests are not touched) and
+ * results_dev[i] = the number of pairs written (<= cap).  1 <= cap <= 4096.
+ * Point requests behave exactly as in eirene_submit_batch.
+ * Mechanism: range queries do not enter the sort; they read the pre-batch
+ * tree in a range kernel between the query and update kernels (P:1066-1074:
+ * range queries run in the query kernel's phase), and every key in [l, u]
+ * that has update requests in the batch takes the result of an "artificial
+ * query" at the range's timestamp, resolved by a binary search of
+ * that key's timestamp-sorted segment.  Not accepted by the multi-GPU
+ * routing (EINVAL there).  Errors as eirene_submit_batch, plus EINVAL for
+ * cap == 0, cap > 4096 or null range buffers. */
+int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev,
+                              const uint64_t* vals_dev, uint32_t n, uint64_t* results_dev,
+                              uint32_t cap, uint64_t* range_keys_dev, uint64_t* range_vals_dev,
+                              eirene_stream_t stream, uint64_t* ticket);
 
 /* Waits for batch `ticket` and returns its status (EIRENE_OK, EINVAL, EFULL);
  * fills *stats if non-NULL.  ESTATE if the ticket is unknown or too old (the

@@ -17,7 +17,7 @@ LIB_PATH = os.path.join(PKG, "libeirene.so")
 HEADER = os.path.join(ROOT, "include", "eirene.h")
 
 EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECUDA = 0, -1, -2, -3, -4, -5
-EIRENE_QUERY, EIRENE_UPDATE, EIRENE_INSERT, EIRENE_DELETE = 0, 1, 2, 3
+EIRENE_QUERY, EIRENE_UPDATE, EIRENE_INSERT, EIRENE_DELETE, EIRENE_RANGE = 0, 1, 2, 3, 4
 EIRENE_F_REGROUP, EIRENE_F_STATS, EIRENE_F_FORCE_STM, EIRENE_F_TIMING = 1, 2, 4, 8
 NOT_FOUND = 0xFFFFFFFFFFFFFFFF
 
@@ -36,7 +36,8 @@ class eirene_batch_stats(ctypes.Structure):
     _fields_ = [("status", ctypes.c_int32), ("n", _u32), ("distinct", _u64), ("issued_q", _u64),
                 ("issued_w", _u64), ("leaf_runs", _u64), ("retries", _u64), ("stm_fallbacks", _u64),
                 ("leaf_splits", _u64), ("inner_splits", _u64), ("new_leaves", _u64), ("new_inner", _u64),
-                ("height", _u32), ("launches", _u32), ("stage_ms", ctypes.c_float * 8)]
+                ("height", _u32), ("launches", _u32), ("stage_ms", ctypes.c_float * 8),
+                ("ranges", _u64), ("artificial", _u64)]
 
     def to_dict(self) -> dict:
         d = {f: getattr(self, f) for f, _ in self._fields_ if f != "stage_ms"}
@@ -55,6 +56,7 @@ _SIGS = {
     "eirene_bulk_load": (_int, [_vp, _vp, _vp, _u64, ctypes.c_float, _vp]),
     "eirene_submit_batch": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _vp, ctypes.POINTER(_u64)]),
     "eirene_submit_batch_host": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _vp, ctypes.POINTER(_u64)]),
+    "eirene_submit_batch_range": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _u32, _vp, _vp, _vp, ctypes.POINTER(_u64)]),
     "eirene_results": (_int, [_vp, _u64, ctypes.POINTER(eirene_batch_stats)]),
     "eirene_scan": (_int, [_vp, _u64, _u64, _vp, _vp, _u64, ctypes.POINTER(_u64), _vp]),
     "eirene_check_invariants": (_int, [_vp, ctypes.POINTER(_u64)]),

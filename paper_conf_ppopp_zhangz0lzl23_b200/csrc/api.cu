@@ -69,7 +69,8 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
 __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys,
                                                         const uint64_t* vals_src, uint64_t* vals_stage,
                                                         uint64_t* results, BatchCtl* ctl_out, uint4* zero,
-                                                        uint32_t zero_n16) {
+                                                        uint32_t zero_n16, uint64_t* rkeys, uint64_t* rvals,
+                                                        uint32_t rcap) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
     zero[i] = make_uint4(0, 0, 0, 0);
   if (blockIdx.x == 0 && threadIdx.x == 0) {
@@ -80,6 +81,9 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
     dst->vals_stage = vals_stage;
     dst->results = results;
     dst->ctl_out = ctl_out;
+    dst->rkeys = rkeys;
+    dst->rvals = rvals;
+    dst->rcap = rcap;
   }
 }
 
@@ -89,6 +93,7 @@ constexpr int MAX_GRAPHS = 8;
 
 struct GraphEntry {
   uint32_t n = 0;
+  bool range = false;               // batch graph with the range kernel
   cudaGraph_t graph = nullptr;      // kept alive: args_node belongs to it
   cudaGraphExec_t exec = nullptr;
   cudaGraphNode_t args_node = nullptr;
@@ -377,7 +382,9 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals
 }
 
 static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
-                       uint64_t* results, cudaStream_t st, uint64_t* vals_stage, uint64_t* ticket) {
+                       uint64_t* results, cudaStream_t st, uint64_t* vals_stage, uint64_t* ticket,
+                       uint64_t* rkeys = nullptr, uint64_t* rvals = nullptr, uint32_t rcap = 0) {
+  const bool range = rkeys != nullptr;
   CK(cudaSetDevice(h->cfg.device));
   const uint64_t tk = h->next_ticket++;
   Rec& r = h->ring[tk % RING];
@@ -412,7 +419,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
   auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
     set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
-                                                   zero_n16);
+                                                   zero_n16, rkeys, rvals, rcap);
     ++launches;
     if (args_node) {
       cudaError_t e = last_node(s, args_node);
@@ -427,6 +434,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     stage("group");
     if (timing) rec(2, s);
     launch_query(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, s, &launches);
+    if (range) launch_range(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, s, &launches);
     stage("query");
     if (timing) rec(3, s);
     launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
@@ -443,7 +451,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     // one captured graph per batch size; a replay updates only the args node
     GraphEntry* g = nullptr;
     for (auto& e : h->graphs)
-      if (e.exec && e.n == n) g = &e;
+      if (e.exec && e.n == n && e.range == range) g = &e;
     if (!g) {
       GraphEntry& e = h->graphs[h->next_graph++ % MAX_GRAPHS];
       if (e.exec) cudaGraphExecDestroy(e.exec);
@@ -456,11 +464,13 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       CK(ee);
       CK(cudaGraphInstantiate(&e.exec, e.graph, 0));
       e.n = n;
+      e.range = range;
       e.launches = launches;
       g = &e;
     }
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
-                      const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16};
+                      const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
+                      &rkeys, &rvals, &rcap};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
     p.gridDim = dim3(SET_ARGS_CTAS);
@@ -485,6 +495,15 @@ int eirene_submit_batch(eirene_handle h, const uint8_t* ops, const uint64_t* key
   if (!h || !ops || !keys || !vals || !results || !ticket) return EIRENE_EINVAL;
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   return submit_impl(h, ops, keys, vals, n, results, reinterpret_cast<cudaStream_t>(stream), nullptr, ticket);
+}
+
+int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
+                              uint32_t n, uint64_t* results, uint32_t cap, uint64_t* range_keys,
+                              uint64_t* range_vals, eirene_stream_t stream, uint64_t* ticket) {
+  if (!h || !ops || !keys || !vals || !results || !ticket || !range_keys || !range_vals) return EIRENE_EINVAL;
+  if (n == 0 || n > h->cfg.max_batch || cap == 0 || cap > 4096) return EIRENE_EINVAL;
+  return submit_impl(h, ops, keys, vals, n, results, reinterpret_cast<cudaStream_t>(stream), nullptr, ticket,
+                     range_keys, range_vals, cap);
 }
 
 int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
@@ -560,6 +579,8 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) 
     stats->new_inner = c.new_inner;
     stats->height = c.height;
     stats->launches = (uint32_t)r.launches;
+    stats->ranges = c.nrange;
+    stats->artificial = c.nart;
     if (r.timing) {
       for (int s = 0; s + 1 < NSTAGE; ++s) cudaEventElapsedTime(&stats->stage_ms[s], r.st[s], r.st[s + 1]);
       cudaEventElapsedTime(&stats->stage_ms[7], r.st[0], r.st[NSTAGE - 1]);

@@ -21,6 +21,20 @@ namespace eirene {
 
 namespace {
 
+// Request validation: op in range, key != UINT64_MAX and
+// inside the shard, upsert value != UINT64_MAX.  A range query R(l, u)
+// (op RANGE, key = l, val = u) is valid with any bounds, but only in a batch
+// submitted with range outputs (rok).
+__device__ __forceinline__ bool request_invalid(uint32_t o, uint64_t k, uint64_t v, bool up, bool rok,
+                                                  uint64_t key_lo, uint64_t key_hi) {
+  if (o == OP_RANGE) return !rok;
+  return o > OP_DELETE || k == KEY_MAX || k < key_lo || k >= key_hi || (up && v == KEY_MAX);
+}
+__device__ __forceinline__ void count_ranges(uint32_t nr, BatchCtl* ctl) {
+  nr = __reduce_add_sync(FULL, nr);
+  if (nr && (threadIdx.x & 31) == 0) atomicAdd(&ctl->nrange, nr);
+}
+
 constexpr int H_THREADS = 512;
 constexpr int H_ITEMS = 16;                      // 8192 requests per CTA
 constexpr int S_THREADS = 256;
@@ -35,21 +49,25 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
   __shared__ uint32_t h[2 * NBINS];   // two copies (even / odd warps); reused by the last CTA
   __shared__ uint32_t s_last;
   __shared__ uint32_t wsum[H_THREADS / 32];
+  __shared__ uint32_t s_total;
   const uint64_t* __restrict__ keys = A->keys;
+  const uint8_t* __restrict__ ops = A->ops;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   for (uint32_t i = tid; i < 2 * NBINS; i += H_THREADS) h[i] = 0;
   __syncthreads();
   uint32_t* hw = h + (warp & 1) * NBINS;
   const uint32_t t0 = blockIdx.x * (H_THREADS * H_ITEMS);
   uint64_t k[H_ITEMS];
+  bool pt[H_ITEMS];   // point request (range queries do not enter the sort)
 #pragma unroll
   for (int j = 0; j < H_ITEMS; ++j) {
     const uint32_t i = t0 + j * H_THREADS + tid;
     k[j] = i < n ? keys[i] : 0;
+    pt[j] = i < n && ops[i] != OP_RANGE;
   }
 #pragma unroll
   for (int j = 0; j < H_ITEMS; ++j)
-    if (t0 + j * H_THREADS + tid < n) atomicAdd(&hw[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
+    if (pt[j]) atomicAdd(&hw[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
   __syncthreads();
   for (uint32_t i = tid; i < NBINS; i += H_THREADS) {
     const uint32_t c = h[i] + h[NBINS + i];
@@ -82,6 +100,9 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
   __syncthreads();
   uint32_t run = x - s;
   for (int w = 0; w < warp; ++w) run += wsum[w];
+  if (tid == H_THREADS - 1) s_total = run + s;   // point requests in the batch
+  __syncthreads();
+  const uint32_t total = s_total;
   uint32_t* sg = h;            // group of every bin
   uint32_t* se = h + NBINS;    // exclusive prefix of every bin
   const bool identity = G == (uint32_t)NBINS;
@@ -90,7 +111,7 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
     const uint32_t bin = tid * PER + j;
     const uint32_t g = identity ? bin
                                 : (uint32_t)min((unsigned long long)(G - 1),
-                                                ((unsigned long long)run + cnt[j] / 2) * G / max(n, 1u));
+                                                ((unsigned long long)run + cnt[j] / 2) * G / max(total, 1u));
     sg[bin] = g;
     se[bin] = run;
     bin2grp[bin] = (uint16_t)g;
@@ -106,7 +127,7 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
       cursor[q] = se[bin];
     }
     if (bin == NBINS - 1)
-      for (uint32_t q = g + 1; q <= G; ++q) gstart[q] = n;
+      for (uint32_t q = g + 1; q <= G; ++q) gstart[q] = total;
   }
 }
 
@@ -139,21 +160,25 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
     o[j] = i < n ? (uint32_t)ops[i] : 0u;
   }
   bool bad = false;
+  const bool rok = A->rkeys != nullptr;
+  uint32_t nr = 0;
 #pragma unroll
   for (int j = 0; j < S_ITEMS; ++j) {
     const uint32_t i = t0 + j * S_THREADS + tid;
     const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
     const uint64_t v = (i < n && up) ? vals[i] : 0;
     if (vstage && i < n && up) vstage[i] = v;
-    bad |= i < n && (o[j] > OP_DELETE || k[j] == KEY_MAX || k[j] < key_lo || k[j] >= key_hi || (up && v == KEY_MAX));
+    bad |= i < n && request_invalid(o[j], k[j], v, up, rok, key_lo, key_hi);
+    nr += i < n && o[j] == OP_RANGE;
   }
   if (__any_sync(FULL, bad) && (tid & 31) == 0) atomicOr(&ctl->invalid, 1u);
+  if (rok) count_ranges(nr, ctl);
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < S_ITEMS; ++j) {
     const uint32_t i = t0 + j * S_THREADS + tid;
     g[j] = s_b2g[(uint32_t)(k[j] >> (64 - BIN_BITS))];
-    r[j] = i < n ? atomicAdd(&hist[g[j]], 1u) : 0u;
+    r[j] = (i < n && o[j] != OP_RANGE) ? atomicAdd(&hist[g[j]], 1u) : 0u;
   }
   __syncthreads();
   for (uint32_t q = tid; q < G; q += S_THREADS) {
@@ -164,7 +189,7 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
 #pragma unroll
   for (int j = 0; j < S_ITEMS; ++j) {
     const uint32_t i = t0 + j * S_THREADS + tid;
-    if (i < n) {
+    if (i < n && o[j] != OP_RANGE) {
       const uint32_t pos = hist[g[j]] + r[j];
       kout[pos] = k[j];
       pout[pos] = (i << 2) | o[j];
@@ -208,16 +233,20 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
     o[j] = i < t1 ? (uint32_t)ops[i] : 0u;
   }
   bool bad = false;
+  const bool rok = A->rkeys != nullptr;
+  uint32_t nr = 0;
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
     const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
     const uint64_t v = (i < t1 && up) ? vals[i] : 0;
     if (vstage && i < t1 && up) vstage[i] = v;
-    bad |= i < t1 && (o[j] > OP_DELETE || k[j] == KEY_MAX || k[j] < key_lo || k[j] >= key_hi || (up && v == KEY_MAX));
-    if (i < t1) atomicAdd(&h[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
+    bad |= i < t1 && request_invalid(o[j], k[j], v, up, rok, key_lo, key_hi);
+    nr += i < t1 && o[j] == OP_RANGE;
+    if (i < t1 && o[j] != OP_RANGE) atomicAdd(&h[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
   }
   if (__any_sync(FULL, bad) && lane == 0) atomicOr(&ctl->invalid, 1u);
+  if (rok) count_ranges(nr, ctl);
   __syncthreads();
   for (uint32_t i = tid; i < NBINS; i += D_THREADS)
     if (h[i]) atomicAdd(&bcount[i], h[i]);
@@ -250,13 +279,17 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   __syncthreads();
   uint32_t run = x - sum;
   for (int w = 0; w < warp; ++w) run += wsum[w];
+  __shared__ uint32_t s_total;
+  if (tid == D_THREADS - 1) s_total = run + sum;   // point requests in the batch
+  __syncthreads();
+  const uint32_t total = s_total;
   const bool identity = G == (uint32_t)NBINS;
 #pragma unroll
   for (int j = 0; j < PER; ++j) {
     const uint32_t bin = tid * PER + j;
     const uint32_t g = identity ? bin
                                 : (uint32_t)min((unsigned long long)(G - 1),
-                                                ((unsigned long long)run + cnt[j] / 2) * G / max(n, 1u));
+                                                ((unsigned long long)run + cnt[j] / 2) * G / max(total, 1u));
     h[bin] = g;
     gs[bin] = run;
     run += cnt[j];
@@ -280,7 +313,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
       gp = gq[j];
     }
     if (tid == D_THREADS - 1)
-      for (uint32_t q = gp + 1; q <= G; ++q) gs[q] = n;
+      for (uint32_t q = gp + 1; q <= G; ++q) gs[q] = total;
   }
   __syncthreads();
   if (blockIdx.x == 0)
@@ -296,7 +329,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
-    r[j] = i < t1 ? atomicAdd(&th[g[j]], 1u) : 0u;
+    r[j] = (i < t1 && o[j] != OP_RANGE) ? atomicAdd(&th[g[j]], 1u) : 0u;
   }
   __syncthreads();
   for (uint32_t q = tid; q < G; q += D_THREADS) {
@@ -307,7 +340,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
-    if (i < t1) {
+    if (i < t1 && o[j] != OP_RANGE) {
       const uint32_t pos = th[g[j]] + r[j];
       kout[pos] = k[j];
       pout[pos] = (i << 2) | o[j];

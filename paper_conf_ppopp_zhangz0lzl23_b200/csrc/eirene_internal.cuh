@@ -29,7 +29,7 @@ constexpr int MAX_LEVELS = 32;
 constexpr uint32_t DONE_BIT = 0x80000000u;
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 
-enum { OP_QUERY = 0, OP_UPDATE = 1, OP_INSERT = 2, OP_DELETE = 3 };
+enum { OP_QUERY = 0, OP_UPDATE = 1, OP_INSERT = 2, OP_DELETE = 3, OP_RANGE = 4 };
 
 // Version word (D2, SURVEY §8(c) reading 18): bit 0 = lock (eager write
 // ownership of the STM), bits 1.. = modification counter.
@@ -57,6 +57,7 @@ struct BatchCtl {
   uint32_t tile_ctr[16];
   uint32_t nseg, nq, nw, height;
   uint32_t nlong, gbar;   // gbar: grid barrier of bsort_dist_kernel
+  uint32_t nrange, nart;  // range queries in the batch; artificial queries resolved
   unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
   uint32_t dbg[8];   // watchdog diagnostics
 };
@@ -99,6 +100,9 @@ struct BatchArgs {
   const uint64_t* vals_src;    // where the distribution pass reads the values of upserts
   uint64_t* vals_stage;        // non-null: it also copies them here (== vals); host path, zero-copy
   BatchCtl* ctl_out;    // device ring slot: the batch's final BatchCtl is copied here at the end
+  uint64_t* rkeys;      // range-query output (eirene_submit_batch_range), else null: RANGE ops invalid
+  uint64_t* rvals;
+  uint32_t rcap;
 };
 
 // tile counters
@@ -243,6 +247,9 @@ struct UpdParams {
 };
 void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms,
                    cudaStream_t st, int* launches);
+// range queries R(l, u): between the query and the update kernel
+void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
+                  int num_sms, cudaStream_t st, int* launches);
 void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
                    const TreeHdr* hdr, int dbgprint,
                    cudaStream_t st, int* launches);

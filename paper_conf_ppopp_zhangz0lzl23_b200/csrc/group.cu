@@ -824,7 +824,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
         ctl->nseg = nseg;
         ctl->nw = nw;
         ctl->nq = nseg - nw;
-        g.istart[nseg] = g.n;
+        g.istart[nseg] = g.gstart[g.nb];   // point requests (range queries are not sorted)
         if (!headroom_ok(g.t, nw)) ctl->status = EIRENE_EFULL;
       }
     }

@@ -154,6 +154,164 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
   }
 }
 
+// ---------------------------------------------------------------- range queries
+// R(l, u) at timestamp t (§4.1.2).  Range queries are
+// not sorted or combined; each one reads the pre-batch tree (this kernel runs
+// after the query kernel and before the update kernel, the query-kernel phase
+// of P:1066-1074) and merges two key-ordered streams:
+//   * the tree's pairs in [l, u]: leaf of l by the same descent as the query
+//     kernel, then the leaf chain until a leaf's hi fence
+//     passes u -- the range's result "in the original manner";
+//   * the batch's written keys in [l, u]: the issued-write list is
+//     key-sorted (one entry per key with update requests), found by binary
+//     search.  Each such key k takes the result of the "artificial query"
+//     Qr(k)@t: k's segment is timestamp-ordered, so a binary
+//     search finds where t would be inserted; the request just before that
+//     point decides -- a write gives its value (NOT_FOUND for a delete), a
+//     query gives its own result (its early result when a write precedes it
+//     in the segment, else the pre-batch value), no request gives the
+//     pre-batch value.  NOT_FOUND drops k from the range, a value adds or
+//     replaces it (reading R2).
+// The first `cap` merged pairs are written to the request's row of the range
+// output; results[t] = pairs written.  One thread per range query.
+__device__ __forceinline__ uint64_t artificial_query(uint32_t w, uint32_t t, uint64_t pre,
+                                                     const uint32_t* __restrict__ wseg,
+                                                     const uint32_t* __restrict__ istart,
+                                                     const uint32_t* __restrict__ spay,
+                                                     const uint32_t* __restrict__ pinfo,
+                                                     const uint64_t* __restrict__ vals,
+                                                     const uint64_t* __restrict__ results) {
+  const uint32_t seg = wseg[w];
+  uint32_t lo = istart[seg], hi = istart[seg + 1];
+  const uint32_t p0 = lo;
+  while (lo < hi) {   // first position with timestamp > t
+    const uint32_t mid = (lo + hi) >> 1;
+    if ((spay[mid] >> 2) < t) lo = mid + 1;
+    else hi = mid;
+  }
+  if (lo == p0) return pre;
+  const uint32_t pj = spay[lo - 1];
+  const uint32_t op = pj & 3;
+  if (op == OP_DELETE) return KEY_MAX;
+  if (op != OP_QUERY) return vals[pj >> 2];
+  return (pinfo[lo - 1] & DONE_BIT) ? ld_cg(results + (pj >> 2)) : pre;
+}
+
+__global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* __restrict__ wkey,
+                                                    const uint32_t* __restrict__ wseg,
+                                                    const uint32_t* __restrict__ spay,
+                                                    const uint32_t* __restrict__ pinfo,
+                                                    const uint32_t* __restrict__ istart,
+                                                    const BatchArgs* __restrict__ A, Tree t, BatchCtl* __restrict__ ctl) {
+  if (ctl->invalid || ctl->status != 0 || ctl->nrange == 0) return;
+  const uint8_t* __restrict__ ops = A->ops;
+  const uint64_t* __restrict__ keys = A->keys;
+  const uint64_t* __restrict__ vals = A->vals;
+  uint64_t* __restrict__ results = A->results;
+  uint64_t* __restrict__ rkeys = A->rkeys;
+  uint64_t* __restrict__ rvals = A->rvals;
+  const uint32_t cap = A->rcap;
+  const uint32_t nw = ctl->nw;
+  const unsigned long long rw = t.hdr->root_word;
+  const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
+  uint32_t nart = 0;
+  const uint32_t stride = gridDim.x * blockDim.x;
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
+    if (ops[i] != OP_RANGE) continue;
+    const uint64_t l = keys[i], u = vals[i];
+    uint64_t* __restrict__ ok = rkeys + (size_t)i * cap;
+    uint64_t* __restrict__ ov = rvals + (size_t)i * cap;
+    uint32_t c = 0;
+    if (l <= u && l != KEY_MAX) {   // (no key is UINT64_MAX; the descent needs l < the separator padding)
+      // written keys >= l: lower_bound over the key-sorted issued writes
+      uint32_t w = 0, whi = nw;
+      while (w < whi) {
+        const uint32_t mid = (w + whi) >> 1;
+        if (wkey[mid] < l) w = mid + 1;
+        else whi = mid;
+      }
+      uint64_t wk = w < nw ? wkey[w] : KEY_MAX;
+      // leaf of l
+      uint32_t node = root;
+      for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
+        const uint64_t* kl = t.ikeys + (size_t)node * FAN;
+        ulonglong4 kv[4];
+#pragma unroll
+        for (int x = 0; x < 4; ++x) kv[x] = ldg256(kl + 4 * x);
+        uint32_t cc = 0;
+#pragma unroll
+        for (int x = 0; x < 4; ++x) cc += (kv[x].x <= l) + (kv[x].y <= l) + (kv[x].z <= l) + (kv[x].w <= l);
+        node = __ldg(t.ichild + (size_t)node * FAN + cc);
+      }
+      // merge the leaf chain with the written keys
+      bool more = true;
+      while (more && c < cap) {
+        const uint64_t* lk = t.lkeys + (size_t)node * LSTRIDE;
+        ulonglong4 kv[4];
+#pragma unroll
+        for (int x = 0; x < 4; ++x) kv[x] = ldg256(lk + 4 * x);
+        uint32_t s = 0;   // first slot with key >= l (keys ascending, KEY_MAX padded)
+#pragma unroll
+        for (int x = 0; x < 4; ++x) s += (kv[x].x < l) + (kv[x].y < l) + (kv[x].z < l) + (kv[x].w < l);
+        for (; s < FAN && c < cap; ++s) {
+          const uint64_t k = __ldg(lk + s);
+          if (k == KEY_MAX) break;   // end of this leaf's keys: go on to the next leaf
+          if (k > u) {
+            more = false;
+            break;
+          }
+          // written keys before k are absent from the pre-batch tree
+          while (wk < k && c < cap) {
+            const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, vals, results);
+            ++nart;
+            if (v != KEY_MAX) {
+              ok[c] = wk;
+              ov[c] = v;
+              ++c;
+            }
+            ++w;
+            wk = w < nw ? wkey[w] : KEY_MAX;
+          }
+          if (c >= cap) break;
+          uint64_t v = __ldg(t.lvals + (size_t)node * LSTRIDE + s);
+          if (wk == k) {
+            v = artificial_query(w, i, v, wseg, istart, spay, pinfo, vals, results);
+            ++nart;
+            ++w;
+            wk = w < nw ? wkey[w] : KEY_MAX;
+          }
+          if (v != KEY_MAX) {
+            ok[c] = k;
+            ov[c] = v;
+            ++c;
+          }
+        }
+        if (!more || c >= cap) break;
+        const NodeMeta* m = t.lmeta + node;
+        const uint64_t hi = __ldg(&m->hi);
+        const uint32_t nx = __ldg(&m->next);
+        if (hi > u || hi == KEY_MAX || nx == NIL) break;   // every later key is > u
+        node = nx;
+      }
+      // written keys after the last tree key in range
+      while (w < nw && wk <= u && c < cap) {   // (u may be UINT64_MAX, the no-more-writes sentinel)
+        const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, vals, results);
+        ++nart;
+        if (v != KEY_MAX) {
+          ok[c] = wk;
+          ov[c] = v;
+          ++c;
+        }
+        ++w;
+        wk = w < nw ? wkey[w] : KEY_MAX;
+      }
+    }
+    results[i] = c;
+  }
+  nart = __reduce_add_sync(FULL, nart);
+  if (nart && (threadIdx.x & 31) == 0) atomicAdd(&ctl->nart, nart);
+}
+
 }  // namespace
 
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
@@ -163,6 +321,14 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
   if (blocks < 1) blocks = 1;
   query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wleaf, c.wslot, c.old, spay, c.pinfo,
                                        c.istart, c.longseg, A, t, ctl);
+  ++*launches;
+}
+
+void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
+                  int num_sms, cudaStream_t st, int* launches) {
+  int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
+  if (blocks < 1) blocks = 1;
+  range_kernel<<<blocks, 256, 0, st>>>(n, c.wkey, c.wseg, spay, c.pinfo, c.istart, A, t, ctl);
   ++*launches;
 }
 

@@ -104,6 +104,32 @@ class EireneTree:
                                           self._stream(stream), ctypes.byref(tk)), "eirene_submit_batch")
         return tk.value
 
+    def submit_range(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor,
+                     cap: int, range_keys: torch.Tensor, range_vals: torch.Tensor, stream=None) -> int:
+        """Batch that may hold range queries (op RANGE = 4, key = l, val = u, inclusive):
+        range_keys / range_vals are [n, cap] u64; row i receives the first results[i] pairs of R(l, u)."""
+        n = ops.numel()
+        _need(ops, torch.uint8, self.device, "ops")
+        _need(keys, torch.uint64, self.device, "keys", n)
+        _need(vals, torch.uint64, self.device, "vals", n)
+        _need(results, torch.uint64, self.device, "results", n)
+        _need(range_keys, torch.uint64, self.device, "range_keys", n * cap)
+        _need(range_vals, torch.uint64, self.device, "range_vals", n * cap)
+        tk = ctypes.c_uint64()
+        check(self._L.eirene_submit_batch_range(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n, _ptr(results), cap,
+                                                _ptr(range_keys), _ptr(range_vals), self._stream(stream),
+                                                ctypes.byref(tk)), "eirene_submit_batch_range")
+        return tk.value
+
+    def apply_range(self, ops, keys, vals, cap: int, stream=None):
+        """submit_range + results: returns (results, range_keys [n, cap], range_vals [n, cap], stats)."""
+        n = ops.numel()
+        res = torch.empty(n, dtype=torch.uint64, device=self.device)
+        rk = torch.zeros((n, cap), dtype=torch.uint64, device=self.device)
+        rv = torch.zeros((n, cap), dtype=torch.uint64, device=self.device)
+        tk = self.submit_range(ops, keys, vals, res, cap, rk, rv, stream)
+        return res, rk, rv, self.results(tk)
+
     def submit_host(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor,
                     stream=None) -> int:
         """Host (ideally pinned) buffers: the library copies them in on its own copy stream, runs the

@@ -12,18 +12,21 @@ configs[0]) instead of the paper's 32-bit records.
 PRNG: counter-based splitmix64, x(seed, stream, i) = splitmix64(seed ^ (stream<<56) ^ i),
 so any batch can be regenerated independently of the others.
 
-Op codes (include/eirene.h): QUERY=0, UPDATE=1, INSERT=2, DELETE=3.
+Op codes (include/eirene.h): QUERY=0, UPDATE=1, INSERT=2, DELETE=3, RANGE=4.
+A range request R(l, u) has key = l and val = u; the generator
+picks l = loaded[j] and u = loaded[j + L - 1] so the range covers L loaded keys
+("range query length" L of the paper's Fig.13).
 Reserved sentinel: UINT64_MAX is never produced as a key or a write value.
 """
 from __future__ import annotations
 
 import numpy as np
 
-QUERY, UPDATE, INSERT, DELETE = 0, 1, 2, 3
+QUERY, UPDATE, INSERT, DELETE, RANGE = 0, 1, 2, 3, 4
 U64_MAX = np.uint64(0xFFFFFFFFFFFFFFFF)
 
 # stream ids (top byte of the counter)
-S_LOAD_KEY, S_LOAD_VAL, S_MIX, S_PICK, S_WVAL, S_FRESH, S_ZIPF, S_DEL = 1, 2, 3, 4, 5, 6, 7, 8
+S_LOAD_KEY, S_LOAD_VAL, S_MIX, S_PICK, S_WVAL, S_FRESH, S_ZIPF, S_DEL, S_RANGE = 1, 2, 3, 4, 5, 6, 7, 8, 9
 
 _M1 = np.uint64(0xBF58476D1CE4E5B9)
 _M2 = np.uint64(0x94D049BB133111EB)
@@ -146,7 +149,7 @@ def shuffled_ops(n: int, fracs: dict[int, float], seed: int, batch: int) -> np.n
 
 
 def make_batch(loaded: np.ndarray, n: int, fracs: dict[int, float], dist: str, seed: int,
-               batch: int, zipf: Zipf | None = None, live: np.ndarray | None = None):
+               batch: int, zipf: Zipf | None = None, live: np.ndarray | None = None, range_len: int = 8):
     """One request batch: (ops u8[n], keys u64[n], vals u64[n]).
 
     QUERY/UPDATE keys are drawn from `loaded` (uniform or scrambled Zipf);
@@ -173,6 +176,12 @@ def make_batch(loaded: np.ndarray, n: int, fracs: dict[int, float], dist: str, s
         keys[dele] = pool[uniform_index(rand_u64(seed, S_DEL, batch << 32, int(dele.sum())), len(pool))]
     vals = rand_u64(seed, S_WVAL, batch << 32, n) >> np.uint64(1)
     vals[ops == QUERY] = 0
+    rng_ = ops == RANGE
+    if rng_.any():
+        L = max(1, min(range_len, m))
+        j = uniform_index(rand_u64(seed, S_RANGE, batch << 32, int(rng_.sum())), m - L + 1)
+        keys[rng_] = loaded[j]
+        vals[rng_] = loaded[j + L - 1]
     return ops, keys, vals
 
 
@@ -184,6 +193,8 @@ CONFIGS = {
     3: dict(tree=1 << 24, batch=1 << 20, fracs={QUERY: 0.5, UPDATE: 0.5}, dist="zipf"),
     4: dict(tree=1 << 20, batch=1 << 20, fracs={INSERT: 0.9, DELETE: 0.1}, dist="uniform"),
     5: dict(tree=1 << 28, batch=1 << 24, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="zipf"),
+    # the paper's pure range-query workload (Fig.13), length 8
+    6: dict(tree=1 << 24, batch=1 << 20, fracs={RANGE: 1.0}, dist="uniform", range_len=8),
 }
 
 
@@ -196,8 +207,10 @@ class Workload:
     optionally scaled down (tree/batch sizes overridden) for parity tests."""
 
     def __init__(self, cfg: int, tree: int | None = None, batch: int | None = None,
-                 fracs: dict | None = None, dist: str | None = None, seed: int | None = None):
+                 fracs: dict | None = None, dist: str | None = None, seed: int | None = None,
+                 range_len: int | None = None):
         c = dict(CONFIGS[cfg])
+        self.range_len = range_len or c.get("range_len", 8)
         self.cfg = cfg
         self.tree = tree or c["tree"]
         self.batch = batch or c["batch"]
@@ -210,7 +223,7 @@ class Workload:
 
     def batch_arrays(self, b: int):
         ops, keys, vals = make_batch(self.keys, self.batch, self.fracs, self.dist, self.seed, b,
-                                     zipf=self.zipf, live=self.live)
+                                     zipf=self.zipf, live=self.live, range_len=self.range_len)
         if self.live is not None:
             # live-key snapshot for the next batch (generator bookkeeping only)
             ins = keys[ops == INSERT]
