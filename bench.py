@@ -118,6 +118,27 @@ def algorithmic_bytes_query(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarra
             "bytes": int(nq * (8 + 4 + 8) + lines * 128 + sectors * 32)}
 
 
+def algorithmic_bytes_range(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, vals: np.ndarray,
+                            per_leaf: int, cap: int) -> dict:
+    """Algorithmic HBM bytes of the RANGE kernel for one range-only batch on the
+    bulk-loaded shape (no writes): per range 1 B op + 8 B l + 8 B u read, 8 B
+    count + 16 B per returned pair written; one 128 B leaf key line per distinct
+    leaf the walks touch and one 32 B value sector per distinct (leaf, sector)
+    returned.  Inner levels are L2-resident (not counted)."""
+    r = ops == W.RANGE
+    lo = np.searchsorted(loaded, keys[r], "left")
+    hi = np.searchsorted(loaded, vals[r], "right")
+    cnt = np.minimum(np.maximum(hi - lo, 0), cap)
+    idx = np.concatenate([np.arange(a, a + c) for a, c in zip(lo, cnt)]) if cnt.size else np.empty(0, np.int64)
+    leaf = idx // per_leaf
+    # the walk reads the leaf of l even when it holds no key of the range
+    lines = np.unique(np.concatenate([leaf, np.minimum(lo, loaded.size - 1) // per_leaf])).size
+    sectors = np.unique(leaf * 4 + (idx % per_leaf) // 4).size
+    nr = int(r.sum())
+    return {"ranges": nr, "pairs": int(cnt.sum()), "leaf_lines": int(lines), "value_sectors": int(sectors),
+            "bytes": int(nr * (1 + 8 + 8 + 8) + int(cnt.sum()) * 16 + lines * 128 + sectors * 32)}
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle (sequential B+tree, 1 thread) as it stands,
     each step a bounded sample of the same workload."""
@@ -134,11 +155,15 @@ def run_reference(args):
     sample = args.ref_sample
     times = []
     total = 0
+    cap = W.CONFIGS[cfg].get("range_len", 0)
     for s in range(args.warmup + args.steps):
         ops, keys, vals = wl.batch_arrays(s)
         ops, keys, vals = ops[:sample], keys[:sample], vals[:sample]
         a = time.perf_counter()
-        t.apply(ops, keys, vals)
+        if cap:
+            t.apply_range(ops, keys, vals, cap)
+        else:
+            t.apply(ops, keys, vals)
         dt = time.perf_counter() - a
         if s >= args.warmup:
             times.append(dt)
@@ -192,6 +217,11 @@ def run_ours(args):
         batch_n = args.batch
     nb = args.warmup + args.steps
     stream = torch.cuda.current_stream(dev)
+    # range-query workload: eirene_submit_batch_range with
+    # per-step output rows of `cap` pairs
+    cap = C.get("range_len", 0) if W.RANGE in C["fracs"] else 0
+    if cap and world > 1:
+        raise SystemExit("range-query configs run on one GPU (DESIGN.md §7)")
 
     # ------------------------------------------------------------ inputs
     t_gen = time.time()
@@ -205,6 +235,9 @@ def run_ours(args):
         host_batches = [wl.batch_arrays(b) for b in range(nb)]
         batches = [tuple(torch.from_numpy(a).to(dev) for a in hb) for hb in host_batches]
         results = [torch.empty(batch_n, dtype=torch.uint64, device=dev) for _ in range(nb)]
+        if cap:
+            rrows = [(torch.empty(batch_n * cap, dtype=torch.uint64, device=dev),
+                      torch.empty(batch_n * cap, dtype=torch.uint64, device=dev)) for _ in range(nb)]
     else:
         # weak scaling: the global tree holds world * tree_n keys, the global batch
         # world * batch_n requests; rank r owns key range r and ts-slice r
@@ -231,7 +264,10 @@ def run_ours(args):
         o, k, v = batches[b]
         ev[b][0].record(stream)
         if world == 1:
-            tk = tree.submit(o, k, v, results[b])
+            if cap:
+                tk = tree.submit_range(o, k, v, results[b], cap, *rrows[b])
+            else:
+                tk = tree.submit(o, k, v, results[b])
             ev[b][1].record(stream)
             return tk
         st = sh.apply(o, k, v, results[b])
@@ -283,7 +319,7 @@ def run_ours(args):
     # (graph replay is off while stage events are on, so this region also
     # shows the cost of direct launches).  Its batches reuse the pre-staged
     # input buffers of the first timed batches.
-    stage_names = ["sort", "group", "query", "update", "result"]
+    stage_names = ["sort", "group", "query+range" if cap else "query", "update", "result"]
     engine = tree if world == 1 else sh.engine
     engine.set_flags(timing=True)
     n_stage = min(args.steps, 10)
@@ -303,7 +339,47 @@ def run_ours(args):
 
     # ------------------------------------------------------------ e2e through the public API (host buffers)
     e2e = None
-    if world == 1 and args.e2e_steps > 0:
+    if world == 1 and args.e2e_steps > 0 and cap:
+        # range batches through the public API with host buffers: pinned H2D of
+        # the inputs, submit_range, D2H of the counts and the range rows, all on
+        # the submit stream inside the timed region (no overlap across steps)
+        hb = [wl.batch_arrays(nb + i) for i in range(args.e2e_steps)]
+        pin = [tuple(torch.from_numpy(a).pin_memory() for a in x) for x in hb]
+        hout = [(torch.empty(batch_n, dtype=torch.uint64).pin_memory(),
+                 torch.empty(batch_n * cap, dtype=torch.uint64).pin_memory(),
+                 torch.empty(batch_n * cap, dtype=torch.uint64).pin_memory()) for _ in hb]
+        dbuf = [torch.empty(batch_n, dtype=torch.uint8, device=dev), torch.empty(batch_n, dtype=torch.uint64, device=dev),
+                torch.empty(batch_n, dtype=torch.uint64, device=dev)]
+        dres = torch.empty(batch_n, dtype=torch.uint64, device=dev)
+        drk = torch.empty(batch_n * cap, dtype=torch.uint64, device=dev)
+        drv = torch.empty(batch_n * cap, dtype=torch.uint64, device=dev)
+
+        def e2e_step(i):
+            for d_, h_ in zip(dbuf, pin[i]):
+                d_.copy_(h_, non_blocking=True)
+            tk_ = tree.submit_range(*dbuf, dres, cap, drk, drv)
+            hout[i][0].copy_(dres, non_blocking=True)
+            hout[i][1].copy_(drk, non_blocking=True)
+            hout[i][2].copy_(drv, non_blocking=True)
+            return tk_
+
+        tree.results(e2e_step(0))
+        torch.cuda.synchronize()
+        a = torch.cuda.Event(enable_timing=True)
+        z = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        tks = [e2e_step(i) for i in range(1, len(pin))]
+        z.record(stream)
+        torch.cuda.synchronize()
+        for t_ in tks:
+            tree.results(t_)
+        e_ms = a.elapsed_time(z)
+        n_e = len(pin) - 1
+        e2e = {"value": batch_n * n_e / (e_ms * 1e-3) / 1e9, "unit": "Greq/s",
+               "h2d_bytes_per_step": int(batch_n * 17), "d2h_bytes_per_step": int(batch_n * (8 + 16 * cap)),
+               "steps": n_e, "path": "torch pinned H2D copies + EireneTree.submit_range + D2H of counts and "
+                                     "range rows, one stream"}
+    elif world == 1 and args.e2e_steps > 0:
         hb = [wl.batch_arrays(nb + i) for i in range(args.e2e_steps)]
         pin = [tuple(torch.from_numpy(a).pin_memory() for a in x) for x in hb]
         hres = [torch.empty(batch_n, dtype=torch.uint64).pin_memory() for _ in hb]
@@ -355,9 +431,18 @@ def run_ours(args):
         for b in range(n_check):
             o, k, v = host_batches[b]
             a = time.perf_counter()
-            want = ref.apply(o, k, v)
+            if cap:
+                want, wk, wv = ref.apply_range(o, k, v, cap)
+            else:
+                want = ref.apply(o, k, v)
             cpu_t += time.perf_counter() - a
-            bad += int(np.sum(results[b].cpu().numpy() != want))
+            got = results[b].cpu().numpy()
+            bad += int(np.sum(got != want))
+            if cap:
+                gk = rrows[b][0].view(batch_n, cap).cpu().numpy()
+                gv = rrows[b][1].view(batch_n, cap).cpu().numpy()
+                col = np.arange(cap)[None, :] < want.astype(np.int64)[:, None]
+                bad += int(np.sum((gk != wk) & col)) + int(np.sum((gv != wv) & col))
         parity = {"batches_checked": n_check, "mismatches": bad, "vs": "oracle B+tree, every request, bit-exact"}
         cpu = {"value": n_check * batch_n / cpu_t / 1e9, "unit": "Greq/s", "cores": 1, "kind": "oracle",
                "sample": f"first {n_check} batches of the same workload ({n_check * batch_n} requests), "
@@ -365,7 +450,13 @@ def run_ours(args):
         # roofline of the dominant kernel
         peaks = load_peaks()
         dom = int(np.argmax(stage_ms))
-        if stage_names[dom] == "query" or args.roofline_kernel == "query":
+        if cap:
+            ab = [algorithmic_bytes_range(wl.keys, *host_batches[b], 16, cap)["bytes"]
+                  for b in range(args.warmup, min(nb, args.warmup + 4))]
+            bytes_per = float(np.mean(ab))
+            ms = stage_ms[2]
+            kern = "range_kernel"
+        elif stage_names[dom] == "query" or args.roofline_kernel == "query":
             ab = [algorithmic_bytes_query(wl.keys, *host_batches[b][:2], 16)["bytes"] for b in range(args.warmup, min(nb, args.warmup + 4))]
             bytes_per = float(np.mean(ab))
             ms = stage_ms[2]
@@ -403,8 +494,9 @@ def run_ours(args):
             "data": "synthetic",
             "config": {"workload": f"cfg{cfg}: {tree_n * world} u64 keys (fanout 16, fill 1.0), "
                                    f"{batch_n * world}-request batches, "
-                                   + ", ".join(f"{int(p * 100)}% {['query', 'update', 'insert', 'delete'][o]}"
-                                               for o, p in sorted(C['fracs'].items())) + f", {C['dist']} keys",
+                                   + ", ".join(f"{int(p * 100)}% {['query', 'update', 'insert', 'delete', 'range'][o]}"
+                                               for o, p in sorted(C['fracs'].items())) + f", {C['dist']} keys"
+                                   + (f", range length {cap} (first {cap} pairs returned)" if cap else ""),
                        "cfg": cfg, "global_batch": batch_n * world,
                        "parallelism": f"key-range shards x{world}" if world > 1 else "single GPU",
                        "l2": "distinct input/result buffers per step (steps x 25 MiB >> 126 MB L2); "

@@ -165,6 +165,42 @@ __device__ __forceinline__ void st_relaxed64(unsigned long long* p, unsigned lon
   asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
 }
 
+// L2 eviction-priority policies (createpolicy) for per-load cache hints: the
+// inner levels (<= 18 MB at 2^24 keys) are re-read by every batch and are
+// loaded evict_last; leaf lines, values and streaming outputs are touched
+// once per batch and are loaded / stored evict_first, so a batch's own
+// streams do not push the inner levels out of L2.
+__device__ __forceinline__ uint64_t pol_evict_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t pol_evict_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+// read-only (nc) loads with an L2 policy; 256-bit loads skip L1 allocation
+__device__ __forceinline__ ulonglong4 ldg256_pol(const uint64_t* p, uint64_t pol) {
+  ulonglong4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+               : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ uint64_t ldg64_pol(const uint64_t* p, uint64_t pol) {
+  uint64_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ uint32_t ldg32_pol(const uint32_t* p, uint64_t pol) {
+  uint32_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ void st64_pol(uint64_t* p, uint64_t v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol) : "memory");
+}
+
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
   return __shfl_sync(FULL, (unsigned long long)v, src);
 }

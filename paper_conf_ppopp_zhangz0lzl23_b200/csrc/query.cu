@@ -28,16 +28,26 @@ namespace eirene {
 
 namespace {
 
-__device__ __forceinline__ ulonglong4 ldg256(const uint64_t* p) {
+// inner-node separator line: L1-allocating (lanes of neighbouring warps walk
+// shared upper nodes) with an L2 policy (evict_last: re-read every batch)
+__device__ __forceinline__ ulonglong4 ldg256_l1(const uint64_t* p, uint64_t pol) {
   ulonglong4 v;
-  asm volatile("ld.global.nc.v4.u64 {%0,%1,%2,%3}, [%4];" : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p));
+  asm volatile("ld.global.nc.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+               : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p), "l"(pol));
   return v;
 }
-// Slot of key k in a 16-key leaf line (4 x 256-bit loads), -1 if absent.
-__device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_t k) {
+// key s of a 16-key line held in registers (selects, no local memory)
+__device__ __forceinline__ uint64_t pick16(const ulonglong4 (&kv)[4], uint32_t s) {
+  const ulonglong4 q = (s < 8) ? ((s < 4) ? kv[0] : kv[1]) : ((s < 12) ? kv[2] : kv[3]);
+  const uint32_t r = s & 3;
+  return r == 0 ? q.x : r == 1 ? q.y : r == 2 ? q.z : q.w;
+}
+// Slot of key k in a 16-key leaf line (4 x 256-bit loads, L2 evict_first:
+// leaves are touched once per batch), -1 if absent.
+__device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_t k, uint64_t pol) {
   ulonglong4 v[4];
 #pragma unroll
-  for (int i = 0; i < 4; ++i) v[i] = ldg256(line + 4 * i);
+  for (int i = 0; i < 4; ++i) v[i] = ldg256_pol(line + 4 * i, pol);
   int s = -1;
 #pragma unroll
   for (int i = 0; i < 4; ++i) {
@@ -65,6 +75,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
   const uint32_t stride = gridDim.x * blockDim.x;
+  const uint64_t pl = pol_evict_last(), pf = pol_evict_first();
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += stride) {
     const bool isq = i < nq;
     const uint64_t k = isq ? qkey[i] : wkey[i - nq];
@@ -77,14 +88,14 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
       const uint64_t* kl = t.ikeys + (size_t)node * FAN;
       ulonglong4 kv[4];
 #pragma unroll
-      for (int x = 0; x < 4; ++x) kv[x] = ldg256(kl + 4 * x);
+      for (int x = 0; x < 4; ++x) kv[x] = ldg256_l1(kl + 4 * x, pl);
       uint32_t c = 0;
 #pragma unroll
       for (int x = 0; x < 4; ++x) c += (kv[x].x <= k) + (kv[x].y <= k) + (kv[x].z <= k) + (kv[x].w <= k);
-      node = __ldg(t.ichild + (size_t)node * FAN + c);
+      node = ldg32_pol(t.ichild + (size_t)node * FAN + c, pl);
     }
-    const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k);
-    const uint64_t v = s >= 0 ? __ldg(t.lvals + (size_t)node * LSTRIDE + s) : KEY_MAX;
+    const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
+    const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
     uint32_t seg;
     if (isq) {
       seg = qseg[i];
@@ -215,6 +226,7 @@ __global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* 
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
   uint32_t nart = 0;
+  const uint64_t pl = pol_evict_last(), pf = pol_evict_first();
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
     if (ops[i] != OP_RANGE) continue;
@@ -237,56 +249,81 @@ __global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* 
         const uint64_t* kl = t.ikeys + (size_t)node * FAN;
         ulonglong4 kv[4];
 #pragma unroll
-        for (int x = 0; x < 4; ++x) kv[x] = ldg256(kl + 4 * x);
+        for (int x = 0; x < 4; ++x) kv[x] = ldg256_l1(kl + 4 * x, pl);
         uint32_t cc = 0;
 #pragma unroll
         for (int x = 0; x < 4; ++x) cc += (kv[x].x <= l) + (kv[x].y <= l) + (kv[x].z <= l) + (kv[x].w <= l);
-        node = __ldg(t.ichild + (size_t)node * FAN + cc);
+        node = ldg32_pol(t.ichild + (size_t)node * FAN + cc, pl);
       }
-      // merge the leaf chain with the written keys
-      bool more = true;
-      while (more && c < cap) {
+      // walk the leaf chain, merged with the written keys
+      for (;;) {
         const uint64_t* lk = t.lkeys + (size_t)node * LSTRIDE;
+        const uint64_t* lv = lk + FAN;
         ulonglong4 kv[4];
 #pragma unroll
-        for (int x = 0; x < 4; ++x) kv[x] = ldg256(lk + 4 * x);
-        uint32_t s = 0;   // first slot with key >= l (keys ascending, KEY_MAX padded)
+        for (int x = 0; x < 4; ++x) kv[x] = ldg256_pol(lk + 4 * x, pf);
+        // slots [s0, s1) hold the leaf's keys in [l, u] (keys ascending, KEY_MAX padded)
+        uint32_t s0 = 0, s1 = 0, nk = 0;
 #pragma unroll
-        for (int x = 0; x < 4; ++x) s += (kv[x].x < l) + (kv[x].y < l) + (kv[x].z < l) + (kv[x].w < l);
-        for (; s < FAN && c < cap; ++s) {
-          const uint64_t k = __ldg(lk + s);
-          if (k == KEY_MAX) break;   // end of this leaf's keys: go on to the next leaf
-          if (k > u) {
-            more = false;
-            break;
+        for (int x = 0; x < 4; ++x) {
+          const uint64_t q[4] = {kv[x].x, kv[x].y, kv[x].z, kv[x].w};
+#pragma unroll
+          for (int y = 0; y < 4; ++y) {
+            s0 += q[y] < l;
+            s1 += q[y] <= u && q[y] != KEY_MAX;
+            nk += q[y] != KEY_MAX;
           }
-          // written keys before k are absent from the pre-batch tree
-          while (wk < k && c < cap) {
-            const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, vals, results);
-            ++nart;
+        }
+        if (wk > u) {
+          // no written key left in [l, u]: the pairs come straight from the leaf;
+          // the value sectors needed are loaded together, then written out
+          const uint32_t take = s1 > s0 ? min(s1 - s0, cap - c) : 0u;
+          const uint32_t e = s0 + take;
+          ulonglong4 vv[4];
+#pragma unroll
+          for (int x = 0; x < 4; ++x) {
+            vv[x] = make_ulonglong4(0, 0, 0, 0);
+            if (4u * x < e && 4u * x + 4 > s0) vv[x] = ldg256_pol(lv + 4 * x, pf);
+          }
+#pragma unroll
+          for (uint32_t j = 0; j < (uint32_t)FAN; ++j)
+            if (j >= s0 && j < e) {
+              st64_pol(ok + c + (j - s0), pick16(kv, j), pf);
+              st64_pol(ov + c + (j - s0), pick16(vv, j), pf);
+            }
+          c += take;
+        } else {
+          for (uint32_t s = s0; s < s1 && c < cap; ++s) {
+            const uint64_t k = pick16(kv, s);
+            // written keys before k are absent from the pre-batch tree
+            while (wk < k && c < cap) {
+              const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, vals, results);
+              ++nart;
+              if (v != KEY_MAX) {
+                ok[c] = wk;
+                ov[c] = v;
+                ++c;
+              }
+              ++w;
+              wk = w < nw ? wkey[w] : KEY_MAX;
+            }
+            if (c >= cap) break;
+            uint64_t v = ldg64_pol(lv + s, pf);
+            if (wk == k) {
+              v = artificial_query(w, i, v, wseg, istart, spay, pinfo, vals, results);
+              ++nart;
+              ++w;
+              wk = w < nw ? wkey[w] : KEY_MAX;
+            }
             if (v != KEY_MAX) {
-              ok[c] = wk;
+              ok[c] = k;
               ov[c] = v;
               ++c;
             }
-            ++w;
-            wk = w < nw ? wkey[w] : KEY_MAX;
-          }
-          if (c >= cap) break;
-          uint64_t v = __ldg(t.lvals + (size_t)node * LSTRIDE + s);
-          if (wk == k) {
-            v = artificial_query(w, i, v, wseg, istart, spay, pinfo, vals, results);
-            ++nart;
-            ++w;
-            wk = w < nw ? wkey[w] : KEY_MAX;
-          }
-          if (v != KEY_MAX) {
-            ok[c] = k;
-            ov[c] = v;
-            ++c;
           }
         }
-        if (!more || c >= cap) break;
+        // a key > u in this leaf ends the walk; so does a full output row
+        if (s1 < nk || c >= cap) break;
         const NodeMeta* m = t.lmeta + node;
         const uint64_t hi = __ldg(&m->hi);
         const uint32_t nx = __ldg(&m->next);
@@ -306,7 +343,7 @@ __global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* 
         wk = w < nw ? wkey[w] : KEY_MAX;
       }
     }
-    results[i] = c;
+    st64_pol(results + i, c, pf);
   }
   nart = __reduce_add_sync(FULL, nart);
   if (nart && (threadIdx.x & 31) == 0) atomicAdd(&ctl->nart, nart);
