@@ -250,7 +250,9 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->cb.wslot, nb);
   AL(h->cb.old, nb);
   AL(h->cb.istart, nb + 1);
-  AL(h->cb.longseg, nb);
+  AL(h->cb.longseg, nb + 64);   // (segment, chunk) pairs of the long segments
+  h->cb.hot_words = (uint32_t)(((nb + 127) / 128) * 4);   // multiple of 4 (uint4 access)
+  AL(h->cb.hot_bits, (size_t)HOT_SLOTS * 3 * h->cb.hot_words);
   AL(h->up.entA_key, nb + 64);
   AL(h->up.entA_child, nb + 64);
   AL(h->up.entB_key, nb + 64);
@@ -307,6 +309,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     e = cudaEventCreateWithFlags(&h->ring[i].done, cudaEventDisableTiming);
     for (int s = 0; s < NSTAGE && e == cudaSuccess; ++s) e = cudaEventCreate(&h->ring[i].st[s]);
   }
+  if (e == cudaSuccess) e = cudaMemset(h->cb.hot_bits, 0, sizeof(uint32_t) * HOT_SLOTS * 3 * h->cb.hot_words);
   if (e == cudaSuccess) e = cudaMemset(h->sb.lookback, 0, sizeof(unsigned long long) * sort_tiles * 256);
   if (e == cudaSuccess) e = cudaMemset(h->route_lb, 0, sizeof(unsigned long long) * ((nb + 2047) / 2048) * 64);
   if (e == cudaSuccess) {
@@ -434,13 +437,13 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     stage("group");
     if (timing) rec(2, s);
     launch_query(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, s, &launches);
-    if (range) launch_range(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, s, &launches);
+    if (range) launch_range(n, h->cb, spay, h->bs.kB, h->dargs, h->t, ctl, h->num_sms, s, &launches);
     stage("query");
     if (timing) rec(3, s);
     launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
     stage("update");
     if (timing) rec(4, s);
-    launch_result(spay, n, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, s, &launches);
+    launch_result(spay, h->bs.kB, n, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, s, &launches);
     stage("result");
     if (timing) rec(5, s);
     return cudaGetLastError();

@@ -26,7 +26,11 @@ constexpr int LSTRIDE = 2 * FAN;   // u64 words per leaf block (keys, then value
 constexpr uint64_t KEY_MAX = ~0ull;
 constexpr uint32_t NIL = 0xFFFFFFFFu;
 constexpr int MAX_LEVELS = 32;
-constexpr uint32_t DONE_BIT = 0x80000000u;
+constexpr uint32_t DONE_BIT = 0x80000000u;    // pinfo: an earlier write of the segment decides the result
+constexpr uint32_t DEFER_BIT = 0x40000000u;   // pinfo (hot-key segments): that early result is written by
+                                              // result_long_kernel from the nearest write's payload in kB
+constexpr uint32_t SEG_MASK = 0x3FFFFFFFu;
+constexpr uint32_t RCHUNK = 4096;             // result_long_kernel work item: positions of one long segment
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 
 enum { OP_QUERY = 0, OP_UPDATE = 1, OP_INSERT = 2, OP_DELETE = 3, OP_RANGE = 4 };
@@ -58,6 +62,7 @@ struct BatchCtl {
   uint32_t nseg, nq, nw, height;
   uint32_t nlong, gbar;   // gbar: grid barrier of bsort_dist_kernel
   uint32_t nrange, nart;  // range queries in the batch; artificial queries resolved
+  uint32_t hot_ctr;       // hot-key timestamp bitmaps claimed by oversized groups
   unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
   uint32_t dbg[8];   // watchdog diagnostics
 };
@@ -263,7 +268,11 @@ struct CombBufs {
   uint64_t* old;              // [n] old value per segment
   uint32_t* istart;           // [n+1] sorted position of each segment's first request (+ n at nseg)
   uint32_t* longseg;          // [n] segments longer than SHORT_SEG, finished by result_long_kernel
+  uint32_t* hot_bits;         // [HOT_SLOTS][3][hot_words] timestamp bitmaps of hot keys: present, op bit 0,
+                              // op bit 1 (all zero between batches)
+  uint32_t hot_words;         // >= max_batch / 32, a multiple of 4
 };
+constexpr int HOT_SLOTS = 64;
 constexpr uint32_t SHORT_SEG = 32;
 constexpr int GROUP_STATUS_WORDS = NBINS;   // >= bsort_groups(n) for every n
 
@@ -284,9 +293,10 @@ struct UpdParams {
 void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms,
                    cudaStream_t st, int* launches);
 // range queries R(l, u): between the query and the update kernel
-void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
-                  int num_sms, cudaStream_t st, int* launches);
-void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
+void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const uint64_t* kB, const BatchArgs* A, Tree t,
+                  BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches);
+void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const CombBufs& c, const BatchArgs* A,
+                   BatchCtl* ctl,
                    const TreeHdr* hdr, int dbgprint,
                    cudaStream_t st, int* launches);
 

@@ -31,6 +31,8 @@
 // bucket larger than G_CAP (skewed keys) is sorted in L2 and walked in several
 // rounds with a carry; a round-walk is repeated after the look-back to emit.
 #include "eirene_internal.cuh"
+#include <cstdio>
+#include <cstdlib>
 
 
 namespace eirene {
@@ -64,6 +66,9 @@ struct GSmem {
   uint32_t c_nh[G_WARPS], c_lw[G_WARPS], c_nw[G_WARPS];
   uint32_t r_nh, r_lw, r_nw;   // round carry-out
   uint32_t seg0, w0, ticket;
+  uint32_t h_cnt[G_WARPS], h_lw[G_WARPS], h_lp[G_WARPS];   // hot_pass1 per-warp results
+  uint64_t hk;                 // split-off hot key of an oversized group
+  uint32_t* hot_bits;          // its timestamp bitmap slot (null: none free)
 };
 
 __device__ __forceinline__ bool kp_less(uint64_t ka, uint32_t pa, uint64_t kb, uint32_t pb) {
@@ -425,7 +430,8 @@ __device__ void l2_pass_pay(const uint32_t* ps, uint32_t* pd, uint32_t cnt, int 
 // in (kd, pd).  Otherwise: stable LSD on the timestamp bits, then on the bits
 // of key - kmin, ping-pong between the group's two L2 ranges.  Returns the
 // range that holds the result (0: ks/ps, 1: kd/pd).
-__device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int tsbits, GSmem& S) {
+__device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int tsbits, GSmem& S,
+                       uint32_t* bits, uint32_t hot_words) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint64_t c0 = ks[0], c1 = ks[cnt / 3], c2 = ks[(2 * (uint64_t)cnt) / 3];
   uint64_t mn = KEY_MAX, mx = 0;
@@ -503,7 +509,16 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
         }
         bh = __shfl_sync(FULL, bh, 0);
         bo = __shfl_sync(FULL, bo, 0);
-        if (hot) hs[bh + __popc(mh & lanemask_lt())] = p;
+        if (hot) {
+          if (bits) {   // timestamp bitmaps: the set bits ARE the hot key's requests in timestamp order
+            const uint32_t ts = p >> 2, wd = ts >> 5, bit = 1u << (ts & 31);
+            atomicOr(bits + wd, bit);
+            if (p & 1) atomicOr(bits + hot_words + wd, bit);
+            if (p & 2) atomicOr(bits + 2 * hot_words + wd, bit);
+          }
+          else
+            hs[bh + __popc(mh & lanemask_lt())] = p;
+        }
         if (v && !hot) {
           const uint32_t x = bo + __popc(mo & lanemask_lt());
           S.k[x] = k;
@@ -515,6 +530,16 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
     const uint32_t o = S.r_nh, h = S.r_lw, lo = S.r_nw;
     if (o > 1) smem_sort(S.k, S.p, o, S);
     __syncthreads();
+    if (bits) {   // SPLIT: the rest stays sorted in S.k / S.p, hk in the bitmap
+      if (tid == 0) {
+        S.r_nh = o;
+        S.r_lw = h;
+        S.r_nw = lo;
+        S.hk = hk;
+      }
+      __syncthreads();
+      return 2;
+    }
     // hk's payloads by timestamp: hs -> ps -> hs ... -> pd + lo (last pass)
     const int tpass = max(1, (tsbits + 7) / 8);
     for (int pass = 0; pass < tpass; ++pass) {
@@ -582,6 +607,9 @@ struct GroupArgs {
   uint64_t* wval;
   uint32_t* wseg;
   unsigned long long* status;   // [nb] look-back words (zeroed per batch)
+  uint32_t* hot_bits;           // [HOT_SLOTS][hot_words] timestamp bitmaps, zero between uses
+  uint32_t hot_words;
+  int prof;                     // EIRENE_GROUP_PROF: print the phases of slow groups (diagnostic)
   Tree t;
   BatchCtl* ctl;
 };
@@ -664,7 +692,8 @@ __device__ void round_scan(const GView& V, uint32_t cnt, uint32_t r0, uint32_t r
 
 // Pass 3 of round [r0, r1): every output of the combine and the partition.
 __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uint32_t gbase,
-                           uint32_t r0, uint32_t r1, bool write_spay, GSmem& S) {
+                           uint32_t r0, uint32_t r1, bool write_spay, GSmem& S,
+                           uint32_t split_lo = 0xFFFFFFFFu, uint32_t split_h = 0, uint32_t split_w = 0) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const uint64_t* __restrict__ vals = g.A->vals;
   uint64_t* __restrict__ results = g.A->results;
@@ -682,7 +711,11 @@ __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uin
     const bool head = valid && (x == 0 || V.k(x - 1) != k);
     const uint32_t H = __ballot_sync(FULL, head);
     const uint32_t W = __ballot_sync(FULL, valid && is_write(p & 3));
-    const uint32_t seg = seg0 + nh + __popc(H & lanemask_le()) - 1u;
+    // SPLIT groups: positions >= split_lo come after the hot key's segment
+    // (split_h positions, one segment, split_w issued writes)
+    const bool after = x >= split_lo;
+    const uint32_t seg = seg0 + nh + __popc(H & lanemask_le()) - 1u + (after ? 1u : 0u);
+    const uint32_t gx = gbase + x + (after ? split_h : 0u);
     // nearest write strictly before x, and at or before x (bucket positions + 1)
     const uint32_t wl = W & lanemask_lt();
     const uint32_t lwb = wl ? b + (31 - __clz(wl)) + 1 : lwc;
@@ -694,15 +727,15 @@ __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uin
       results[p >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
     }
     if (valid) {
-      g.pinfo[gbase + x] = seg | (done ? DONE_BIT : 0u);
-      if (write_spay) g.pB[gbase + x] = p;
+      g.pinfo[gx] = seg | (done ? DONE_BIT : 0u);
+      if (write_spay) g.pB[gx] = p;
     }
-    if (head) g.istart[seg] = gbase + x;
+    if (head) g.istart[seg] = gx;
     const bool tail = valid && (x + 1 == cnt || V.k(x + 1) != k);
     const bool hasw = tail && lwi && V.k(lwi - 1) == k;
     const uint32_t WT = __ballot_sync(FULL, hasw);
     if (tail) {
-      const uint32_t wi = w0 + nwc + __popc(WT & lanemask_lt());
+      const uint32_t wi = w0 + nwc + __popc(WT & lanemask_lt()) + (after ? split_w : 0u);
       if (hasw) {   // issue rule: the segment's last write
         const uint32_t pw = V.p(lwi - 1);
         const uint32_t opw = pw & 3;
@@ -722,6 +755,184 @@ __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uin
   }
 }
 
+
+// ---------------------------------------------------------------- hot key
+// The split-off hot key hk of an oversized group is one key segment.  Its
+// requests were recorded by l2_sort in the group's timestamp bitmap slot --
+// three bitmaps over [0, n): present, op bit 0, op bit 1 -- so walking the
+// bitmaps in ts order visits them in timestamp order: the (key, ts) sort of
+// that segment for O(n / 32) word reads instead of radix passes over its
+// requests, and the ops come with the bits (no gather of the batch's ops).
+// Thread t owns the contiguous words [t*PW, (t+1)*PW) (PW a multiple of 4,
+// read as uint4).
+//   pass 1: per thread, requests and last write / last request payload;
+//           CTA scan -> the thread's rank carry and nearest-write carry;
+//   pass 2: sorted payload, pinfo (seg | DONE) and, in the group's unused
+//           kB range, the payload of each position's nearest earlier write;
+//           words are cleared as they are read;
+//   results: the early results (nearest write P:834-835) of the
+//           DONE positions, all positions in parallel.
+struct HotCarry {
+  uint32_t rank, lw;       // this thread's exclusive carries
+  uint32_t total, last_w, last_p;
+};
+__device__ __forceinline__ uint32_t hot_pw(uint32_t W) { return 4u * ((W + 4u * G_THREADS - 1) / (4u * G_THREADS)); }
+
+__device__ HotCarry hot_pass1(const GroupArgs& g, const uint32_t* bits, GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const uint32_t W = g.hot_words, PW = hot_pw(W);
+  const uint32_t w0 = min(W, tid * PW), w1 = min(W, w0 + PW);
+  uint32_t cnt = 0, lw = 0, lp = 0;   // payload 0 = none (a write has op != 0)
+  for (uint32_t x = w0; x < w1; x += 4) {
+    const uint4 P = __ldcg(reinterpret_cast<const uint4*>(bits + x));
+    const uint4 B0 = __ldcg(reinterpret_cast<const uint4*>(bits + W + x));
+    const uint4 B1 = __ldcg(reinterpret_cast<const uint4*>(bits + 2 * W + x));
+    const uint32_t pw[4] = {P.x, P.y, P.z, P.w}, b0[4] = {B0.x, B0.y, B0.z, B0.w}, b1[4] = {B1.x, B1.y, B1.z, B1.w};
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      cnt += __popc(pw[j]);
+      const uint32_t base = (x + j) * 32;
+      if (pw[j]) {
+        const uint32_t t = 31 - __clz(pw[j]);
+        lp = ((base + t) << 2) | ((b0[j] >> t) & 1u) | (((b1[j] >> t) & 1u) << 1);
+      }
+      const uint32_t wm = b0[j] | b1[j];
+      if (wm) {
+        const uint32_t t = 31 - __clz(wm);
+        lw = ((base + t) << 2) | ((b0[j] >> t) & 1u) | (((b1[j] >> t) & 1u) << 1);
+      }
+    }
+  }
+  // CTA scan: exclusive sum of cnt, exclusive max of lw (ascending chunks)
+  uint32_t inc = cnt, mx = lw;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, inc, o), z = __shfl_up_sync(FULL, mx, o);
+    if (lane >= o) {
+      inc += y;
+      mx = max(mx, z);
+    }
+  }
+  if (lane == 31) {
+    S.h_cnt[warp] = inc;
+    S.h_lw[warp] = mx;
+  }
+  uint32_t lpw = lp;
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) lpw = max(lpw, __shfl_xor_sync(FULL, lpw, o));
+  if (lane == 0) S.h_lp[warp] = lpw;
+  __syncthreads();
+  HotCarry c;
+  uint32_t rb = 0, mb = 0;
+  c.total = 0;
+  c.last_w = 0;
+  c.last_p = 0;
+  for (int w = 0; w < G_WARPS; ++w) {
+    if (w < warp) {
+      rb += S.h_cnt[w];
+      mb = max(mb, S.h_lw[w]);
+    }
+    c.total += S.h_cnt[w];
+    c.last_w = max(c.last_w, S.h_lw[w]);
+    c.last_p = max(c.last_p, S.h_lp[w]);
+  }
+  const uint32_t ex_inc = __shfl_up_sync(FULL, inc, 1), ex_mx = __shfl_up_sync(FULL, mx, 1);
+  c.rank = rb + (lane ? ex_inc : 0u);
+  c.lw = max(mb, lane ? ex_mx : 0u);
+  __syncthreads();
+  return c;
+}
+
+// Pass 2 + results; sH = the hot segment's index, pos0 = its first sorted position.
+// The early results of the DONE positions are written here only for a short
+// segment; a long one's positions are marked DEFER and result_long_kernel,
+// which spreads long segments over many CTAs, writes them.
+// Pass 2 walks the bitmaps warp-contiguously (warp w owns the words of
+// threads [32w, 32w + 32) of pass 1, lanes read consecutive words), so the
+// positions written by a warp step are contiguous and the stores coalesce;
+// the lane carries come from a warp scan of the words' counts and last writes.
+__device__ void hot_pass2(const GroupArgs& g, uint32_t* bits, const HotCarry& c, uint32_t sH, uint32_t pos0) {
+  const int tid = threadIdx.x, lane = tid & 31;
+  const uint32_t W = g.hot_words, PW = hot_pw(W);
+  const uint32_t wbeg = min(W, (uint32_t)(tid & ~31) * PW), wend = min(W, wbeg + 32u * PW);
+  // the warp's carries = those of its lane 0 in pass 1
+  uint32_t rank = __shfl_sync(FULL, c.rank, 0), prev = __shfl_sync(FULL, c.lw, 0);
+  // a long hot segment's early results are left to result_long_kernel (many CTAs)
+  const bool defer = c.total > SHORT_SEG;
+  const uint32_t dbits = DONE_BIT | (defer ? DEFER_BIT : 0u);
+  constexpr int D = 4;   // steps whose loads are issued together
+  for (uint32_t xb = wbeg; xb < wend; xb += 32 * D) {
+    uint32_t P[D], B0[D], B1[D];
+#pragma unroll
+    for (int k = 0; k < D; ++k) {
+      const uint32_t x = xb + 32 * k + lane;
+      const bool v = x < wend;
+      P[k] = v ? __ldcg(bits + x) : 0u;
+      B0[k] = v ? __ldcg(bits + W + x) : 0u;
+      B1[k] = v ? __ldcg(bits + 2 * W + x) : 0u;
+    }
+#pragma unroll
+    for (int k = 0; k < D; ++k) {
+      const uint32_t x = xb + 32 * k + lane;
+      const uint32_t word = P[k];
+      if (!__any_sync(FULL, word)) continue;
+      const uint32_t wm = word & (B0[k] | B1[k]);   // write requests of this word
+      const uint32_t pc = __popc(word);
+      uint32_t mylw = 0;
+      if (wm) {
+        const uint32_t t = 31 - __clz(wm);
+        mylw = ((x * 32 + t) << 2) | ((B0[k] >> t) & 1u) | (((B1[k] >> t) & 1u) << 1);
+      }
+      uint32_t inc = pc, mx = mylw;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, inc, o), z = __shfl_up_sync(FULL, mx, o);
+        if (lane >= o) {
+          inc += y;
+          mx = max(mx, z);
+        }
+      }
+      const uint32_t tot = __shfl_sync(FULL, inc, 31), mxall = __shfl_sync(FULL, mx, 31);
+      const uint32_t ex_mx = __shfl_up_sync(FULL, mx, 1);
+      uint32_t pv = max(prev, lane ? ex_mx : 0u);
+      uint32_t pos = pos0 + rank + inc - pc;
+      for (uint32_t m = word; m; m &= m - 1) {
+        const uint32_t t = __ffs(m) - 1;
+        const uint32_t op = ((B0[k] >> t) & 1u) | (((B1[k] >> t) & 1u) << 1);
+        const uint32_t pay = ((x * 32 + t) << 2) | op;
+        g.pB[pos] = pay;
+        g.pinfo[pos] = sH | (pv ? dbits : 0u);
+        g.kB[pos] = pv;   // nearest earlier write (0: none)
+        ++pos;
+        if (op) pv = pay;
+      }
+      if (word) {   // leave the slot clean for the next batch
+        bits[x] = 0u;
+        bits[W + x] = 0u;
+        bits[2 * W + x] = 0u;
+      }
+      rank += tot;
+      prev = max(prev, mxall);
+    }
+  }
+  __syncthreads();
+  const uint64_t* __restrict__ vals = g.A->vals;
+  uint64_t* __restrict__ results = g.A->results;
+  const uint32_t e = pos0 + c.total;
+  for (uint32_t q0 = pos0 + tid; q0 < e && !defer; q0 += 8 * G_THREADS) {   // 8 in flight per thread
+    uint32_t pw[8], py[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const uint32_t q = q0 + u * G_THREADS;
+      pw[u] = q < e ? (uint32_t)__ldcg(reinterpret_cast<const unsigned long long*>(g.kB + q)) : 0u;
+      py[u] = q < e ? __ldcg(g.pB + q) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      if (pw[u]) results[py[u] >> 2] = ((pw[u] & 3) == OP_DELETE) ? KEY_MAX : vals[pw[u] >> 2];
+  }
+}
+
 __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GSmem& S = *reinterpret_cast<GSmem*>(smem_raw);
@@ -731,6 +942,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   if (tid == 0) S.ticket = atomicAdd(&ctl->tile_ctr[TC_GROUP], 1u);
   __syncthreads();
   const uint32_t b = S.ticket;
+  const unsigned long long tp0 = g.prof ? gtime_ns() : 0;
   const uint32_t base = g.gstart[b];
   const uint32_t cnt = g.gstart[b + 1] - base;
   const bool small = cnt <= (uint32_t)G_CAP;
@@ -746,11 +958,29 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     __syncthreads();
     K = S.k;
     P = S.p;
-  } else {
-    const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S);
-    K = (where ? g.kB : g.kA) + base;
-    P = (where ? g.pB : g.pA) + base;
   }
+  int mode = 0;   // 0: small / L2-sorted group, 2: SPLIT (rest in smem, hot key in a bitmap)
+  uint32_t sp_o = 0, sp_h = 0, sp_lo = 0;
+  if (!small) {
+    if (tid == 0) {
+      const uint32_t slot = atomicAdd(&ctl->hot_ctr, 1u);
+      S.hot_bits = slot < (uint32_t)HOT_SLOTS ? g.hot_bits + (size_t)slot * 3 * g.hot_words : nullptr;
+    }
+    __syncthreads();
+    const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S, S.hot_bits, g.hot_words);
+    if (where == 2) {
+      mode = 2;
+      sp_o = S.r_nh;
+      sp_h = S.r_lw;
+      sp_lo = S.r_nw;
+      K = S.k;
+      P = S.p;
+    } else {
+      K = (where ? g.kB : g.kA) + base;
+      P = (where ? g.pB : g.pA) + base;
+    }
+  }
+  const unsigned long long tp1 = g.prof ? gtime_ns() : 0;
   // an oversized group is walked in rounds of G_CAP positions copied to smem
   auto load_round = [&](uint32_t r0, uint32_t r1) {
     __syncthreads();
@@ -777,7 +1007,29 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   };
   // sweep 1: bucket totals (heads, write segments)
   uint32_t c_nh = 0, c_lw = 0, c_nw = 0;
-  for (uint32_t r0 = 0; r0 < cnt; r0 += G_CAP) {
+  uint32_t a_nh = 0, a_nw = 0, hot_w = 0, hot_last = 0;   // SPLIT: rest below hk; hk's issue
+  HotCarry hc{};
+  if (mode == 2) {
+    const GView V{K, P, K, P, 0, sp_o};
+    if (sp_lo) {   // the part of the rest below hk, alone (its tail ends at hk)
+      round_scan(V, sp_lo, 0, sp_lo, 0, 0, 0, S);
+      a_nh = S.r_nh;
+      a_nw = S.r_nw;
+    }
+    if (sp_o) {
+      round_scan(V, sp_o, 0, sp_o, 0, 0, 0, S);
+      c_nh = S.r_nh;
+      c_nw = S.r_nw;
+    }
+    __syncthreads();
+    hc = hot_pass1(g, S.hot_bits, S);
+    hot_w = hc.last_w ? 1u : 0u;
+    hot_last = hc.last_w ? hc.last_w : hc.last_p;   // issue rule: the last write, else the last query
+    c_nh += 1;
+    c_nw += hot_w;
+    __syncthreads();
+  }
+  for (uint32_t r0 = 0; mode == 0 && r0 < cnt; r0 += G_CAP) {
     const uint32_t r1 = min(cnt, r0 + (uint32_t)G_CAP);
     const GView V = small ? GView{K, P, K, P, 0, cnt} : load_round(r0, r1);
     round_scan(V, cnt, r0, r1, c_nh, c_lw, c_nw, S);
@@ -785,6 +1037,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     c_lw = S.r_lw;
     c_nw = S.r_nw;
   }
+  const unsigned long long tp2 = g.prof ? gtime_ns() : 0;
   // decoupled look-back over the buckets (ticket order) on (heads << 31 | writes)
   if (warp == 0) {
     const unsigned long long tot = ((unsigned long long)c_nh << 31) | c_nw;
@@ -830,8 +1083,36 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     }
   }
   __syncthreads();
+  const unsigned long long tp3 = g.prof ? gtime_ns() : 0;
   // sweep 2: emit (a small bucket reuses the carries of its single round)
-  if (small) {
+  if (mode == 2) {
+    const GView V{K, P, K, P, 0, sp_o};
+    if (sp_o) {
+      round_scan(V, sp_o, 0, sp_o, 0, 0, 0, S);
+      round_emit(g, V, sp_o, base, 0, sp_o, true, S, sp_lo, sp_h, hot_w);
+    }
+    __syncthreads();
+    const uint32_t sH = S.seg0 + a_nh, wH = S.w0 + a_nw, pos0 = base + sp_lo;
+    const unsigned long long th0 = g.prof ? gtime_ns() : 0;
+    hot_pass2(g, S.hot_bits, hc, sH, pos0);
+    if ((g.prof & 1) && tid == 0)
+      printf("[hot prof] ticket %u h %u pass2 %.1f us, rest emit before %.1f us\n", b, hc.total, (gtime_ns() - th0) * 1e-3,
+             (th0 - tp3) * 1e-3);
+    if (tid == 0) {
+      const uint64_t hk = S.hk;
+      g.istart[sH] = pos0;
+      if (hot_w) {   // issue rule: the segment's last write
+        const uint32_t opw = hot_last & 3;
+        g.wkey[wH] = hk;
+        g.wop[wH] = (uint8_t)opw;
+        g.wval[wH] = (opw == OP_DELETE) ? KEY_MAX : g.A->vals[hot_last >> 2];
+        g.wseg[wH] = sH;
+      } else {       // all-query segment: its last query
+        g.qkey[sH - wH] = hk;
+        g.qseg[sH - wH] = sH;
+      }
+    }
+  } else if (small) {
     if (cnt) round_emit(g, GView{K, P, K, P, 0, cnt}, cnt, base, 0, cnt, true, S);
   } else {
     const bool write_spay = P != g.pB + base;
@@ -846,6 +1127,12 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       c_nw = S.r_nw;
       __syncthreads();
     }
+  }
+  if ((g.prof & 1) && tid == 0) {
+    const unsigned long long tp4 = gtime_ns();
+    if (tp4 - tp0 > 20000)
+      printf("[group prof] ticket %u cnt %u mode %d sort %.1f sweep1 %.1f lookback %.1f emit %.1f us\n", b, cnt, mode,
+             (tp1 - tp0) * 1e-3, (tp2 - tp1) * 1e-3, (tp3 - tp2) * 1e-3, (tp4 - tp3) * 1e-3);
   }
 }
 
@@ -877,6 +1164,10 @@ void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const Comb
   g.wval = c.wval;
   g.wseg = c.wseg;
   g.status = c.group_status;
+  g.hot_bits = c.hot_bits;
+  g.hot_words = c.hot_words;
+  static const int prof = std::getenv("EIRENE_GROUP_PROF") ? std::atoi(std::getenv("EIRENE_GROUP_PROF")) : 0;
+  g.prof = prof;
   g.t = t;
   g.ctl = ctl;
   group_kernel<<<g.nb, G_THREADS, sizeof(GSmem), st>>>(g);

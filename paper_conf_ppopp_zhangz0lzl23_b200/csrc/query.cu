@@ -114,8 +114,13 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
         for (uint32_t p = p0; p < p1; ++p)
           if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
       }
-    } else {
-      longseg[atomicAdd(&ctl->nlong, 1u)] = seg;
+    } else {   // work items of RCHUNK positions: (segment, chunk) pairs
+      const uint32_t nc = (p1 - p0 + RCHUNK - 1) / RCHUNK;
+      const uint32_t at = atomicAdd(&ctl->nlong, nc);
+      for (uint32_t c = 0; c < nc; ++c) {
+        longseg[2 * (at + c)] = seg;
+        longseg[2 * (at + c) + 1] = c;
+      }
     }
   }
 }
@@ -126,6 +131,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
 // here with one CTA per segment, so a 56K-request Zipf key does not serialise
 // one thread.
 __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __restrict__ spay,
+                                                            const uint64_t* __restrict__ kB,
                                                             const uint32_t* __restrict__ pinfo,
                                                             const uint32_t* __restrict__ istart,
                                                             const uint32_t* __restrict__ longseg,
@@ -145,22 +151,30 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
   }
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
+  const uint64_t* __restrict__ vals = A->vals;
   const uint32_t nl = ctl->nlong;
   for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
-    const uint32_t s = longseg[x];
+    const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
     const uint64_t v = old[s];
-    const uint32_t e = istart[s + 1];
-    for (uint32_t p0 = istart[s] + threadIdx.x; p0 < e; p0 += 8 * blockDim.x) {   // 8 loads in flight
-      uint32_t pi[8], py[8];
+    const uint32_t b = istart[s] + ch * RCHUNK;
+    const uint32_t e = min(istart[s + 1], b + RCHUNK);
+    for (uint32_t p0 = b + threadIdx.x; p0 < e; p0 += 4 * blockDim.x) {   // 4 loads in flight
+      uint32_t pi[4], py[4];
 #pragma unroll
-      for (int u = 0; u < 8; ++u) {
+      for (int u = 0; u < 4; ++u) {
         const uint32_t p = p0 + u * blockDim.x;
         pi[u] = p < e ? pinfo[p] : DONE_BIT;
         py[u] = p < e ? spay[p] : 0u;
       }
 #pragma unroll
-      for (int u = 0; u < 8; ++u)
-        if (!(pi[u] & DONE_BIT)) results[py[u] >> 2] = v;
+      for (int u = 0; u < 4; ++u) {
+        if (!(pi[u] & DONE_BIT)) {
+          results[py[u] >> 2] = v;   // no earlier write in the segment: the issued request's value
+        } else if (pi[u] & DEFER_BIT) {   // hot key: the nearest earlier write (its payload in kB)
+          const uint32_t pw = (uint32_t)kB[p0 + u * blockDim.x];
+          results[py[u] >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
+        }
+      }
     }
   }
 }
@@ -190,6 +204,7 @@ __device__ __forceinline__ uint64_t artificial_query(uint32_t w, uint32_t t, uin
                                                      const uint32_t* __restrict__ istart,
                                                      const uint32_t* __restrict__ spay,
                                                      const uint32_t* __restrict__ pinfo,
+                                                     const uint64_t* __restrict__ kB,
                                                      const uint64_t* __restrict__ vals,
                                                      const uint64_t* __restrict__ results) {
   const uint32_t seg = wseg[w];
@@ -205,14 +220,21 @@ __device__ __forceinline__ uint64_t artificial_query(uint32_t w, uint32_t t, uin
   const uint32_t op = pj & 3;
   if (op == OP_DELETE) return KEY_MAX;
   if (op != OP_QUERY) return vals[pj >> 2];
-  return (pinfo[lo - 1] & DONE_BIT) ? ld_cg(results + (pj >> 2)) : pre;
+  const uint32_t pi = pinfo[lo - 1];
+  if (!(pi & DONE_BIT)) return pre;
+  if (pi & DEFER_BIT) {   // hot key: its early results are written later; the nearest write decides
+    const uint32_t pw = (uint32_t)kB[lo - 1];
+    return ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
+  }
+  return ld_cg(results + (pj >> 2));
 }
 
-__global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* __restrict__ wkey,
+__global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_t* __restrict__ wkey,
                                                     const uint32_t* __restrict__ wseg,
                                                     const uint32_t* __restrict__ spay,
                                                     const uint32_t* __restrict__ pinfo,
                                                     const uint32_t* __restrict__ istart,
+                                                    const uint64_t* __restrict__ kB,
                                                     const BatchArgs* __restrict__ A, Tree t, BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0 || ctl->nrange == 0) return;
   const uint8_t* __restrict__ ops = A->ops;
@@ -279,25 +301,25 @@ __global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* 
           // the value sectors needed are loaded together, then written out
           const uint32_t take = s1 > s0 ? min(s1 - s0, cap - c) : 0u;
           const uint32_t e = s0 + take;
-          ulonglong4 vv[4];
+          // keys first (their registers die), then the value chunks that hold slots [s0, e)
+#pragma unroll
+          for (uint32_t j = 0; j < (uint32_t)FAN; ++j)
+            if (j >= s0 && j < e) st64_pol(ok + c + (j - s0), pick16(kv, j), pf);
 #pragma unroll
           for (int x = 0; x < 4; ++x) {
-            vv[x] = make_ulonglong4(0, 0, 0, 0);
-            if (4u * x < e && 4u * x + 4 > s0) vv[x] = ldg256_pol(lv + 4 * x, pf);
+            kv[x] = make_ulonglong4(0, 0, 0, 0);
+            if (4u * x < e && 4u * x + 4 > s0) kv[x] = ldg256_pol(lv + 4 * x, pf);
           }
 #pragma unroll
           for (uint32_t j = 0; j < (uint32_t)FAN; ++j)
-            if (j >= s0 && j < e) {
-              st64_pol(ok + c + (j - s0), pick16(kv, j), pf);
-              st64_pol(ov + c + (j - s0), pick16(vv, j), pf);
-            }
+            if (j >= s0 && j < e) st64_pol(ov + c + (j - s0), pick16(kv, j), pf);
           c += take;
         } else {
           for (uint32_t s = s0; s < s1 && c < cap; ++s) {
             const uint64_t k = pick16(kv, s);
             // written keys before k are absent from the pre-batch tree
             while (wk < k && c < cap) {
-              const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, vals, results);
+              const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, kB, vals, results);
               ++nart;
               if (v != KEY_MAX) {
                 ok[c] = wk;
@@ -310,7 +332,7 @@ __global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* 
             if (c >= cap) break;
             uint64_t v = ldg64_pol(lv + s, pf);
             if (wk == k) {
-              v = artificial_query(w, i, v, wseg, istart, spay, pinfo, vals, results);
+              v = artificial_query(w, i, v, wseg, istart, spay, pinfo, kB, vals, results);
               ++nart;
               ++w;
               wk = w < nw ? wkey[w] : KEY_MAX;
@@ -332,7 +354,7 @@ __global__ void __launch_bounds__(256) range_kernel(uint32_t n, const uint64_t* 
       }
       // written keys after the last tree key in range
       while (w < nw && wk <= u && c < cap) {   // (u may be UINT64_MAX, the no-more-writes sentinel)
-        const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, vals, results);
+        const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, kB, vals, results);
         ++nart;
         if (v != KEY_MAX) {
           ok[c] = wk;
@@ -361,18 +383,31 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
   ++*launches;
 }
 
-void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
-                  int num_sms, cudaStream_t st, int* launches) {
+void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const uint64_t* kB, const BatchArgs* A, Tree t,
+                  BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
-  range_kernel<<<blocks, 256, 0, st>>>(n, c.wkey, c.wseg, spay, c.pinfo, c.istart, A, t, ctl);
+  range_kernel<<<blocks, 256, 0, st>>>(n, c.wkey, c.wseg, spay, c.pinfo, c.istart, kB, A, t, ctl);
   ++*launches;
 }
 
-void launch_result(const uint32_t* spay, uint32_t n, const CombBufs& c, const BatchArgs* A, BatchCtl* ctl,
+static int num_long_ctas() {
+  static int n = 0;
+  if (!n) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    n = 2 * sms;
+  }
+  return n;
+}
+
+void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const CombBufs& c, const BatchArgs* A,
+                   BatchCtl* ctl,
                    const TreeHdr* hdr, int dbgprint, cudaStream_t st, int* launches) {
   (void)n;
-  result_long_kernel<<<64, 1024, 0, st>>>(spay, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr, dbgprint);
+  result_long_kernel<<<num_long_ctas(), 1024, 0, st>>>(spay, kB, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr,
+                                                       dbgprint);
   ++*launches;
 }
 
