@@ -225,14 +225,39 @@ def run_ours(args):
 
     # ------------------------------------------------------------ inputs
     t_gen = time.time()
+    per_tree = C.get("per_tree", 0)
     if world == 1:
-        wl = W.Workload(cfg, tree=tree_n, batch=batch_n)
-        keys_d = torch.from_numpy(wl.keys).to(dev)
-        vals_d = torch.from_numpy(wl.vals).to(dev)
-        tree = EireneTree(max_keys=max(tree_n * 2, 1 << 20), max_batch=batch_n)
-        tree.bulk_load(keys_d, vals_d)
-        del keys_d, vals_d
-        host_batches = [wl.batch_arrays(b) for b in range(nb)]
+        def build_plan(tag: int, nsteps: int):
+            """Trees and pre-staged batches for nsteps steps.  Single-tree configs: one
+            bulk-loaded tree, step s = batch s.  Fresh-tree configs (cfg1, cfg4;
+            SURVEY §8(d)): step s runs batch s % per_tree on tree s // per_tree,
+            every tree bulk-loaded from its own seed (untimed)."""
+            if not per_tree:
+                return None
+            ntr = (nsteps + per_tree - 1) // per_tree
+            wls_ = [W.Workload(cfg, tree=tree_n, batch=batch_n, seed=W.seed_for(cfg) + 7919 * (1000 * tag + t + 1))
+                    for t in range(ntr)]
+            trees_ = []
+            for w_ in wls_:
+                tr = EireneTree(max_keys=tree_n + per_tree * batch_n + (1 << 12), max_batch=batch_n)
+                tr.bulk_load(torch.from_numpy(w_.keys).to(dev), torch.from_numpy(w_.vals).to(dev))
+                tr.prepare(batch_n, bool(cap))   # graph capture outside every timed region
+                trees_.append(tr)
+            hb_ = [wls_[s_ // per_tree].batch_arrays(s_ % per_tree) for s_ in range(nsteps)]
+            return wls_, trees_, [s_ // per_tree for s_ in range(nsteps)], hb_
+
+        if per_tree:
+            wls, trees, step_tree, host_batches = build_plan(0, nb)
+            wl, tree = wls[0], trees[0]
+        else:
+            wl = W.Workload(cfg, tree=tree_n, batch=batch_n)
+            keys_d = torch.from_numpy(wl.keys).to(dev)
+            vals_d = torch.from_numpy(wl.vals).to(dev)
+            tree = EireneTree(max_keys=max(tree_n * 2, 1 << 20), max_batch=batch_n)
+            tree.bulk_load(keys_d, vals_d)
+            del keys_d, vals_d
+            wls, trees, step_tree = [wl], [tree], [0] * nb
+            host_batches = [wl.batch_arrays(b) for b in range(nb)]
         batches = [tuple(torch.from_numpy(a).to(dev) for a in hb) for hb in host_batches]
         results = [torch.empty(batch_n, dtype=torch.uint64, device=dev) for _ in range(nb)]
         if cap:
@@ -259,24 +284,27 @@ def run_ours(args):
     stats = []
     launches = 0
 
-    def step(b):
+    def step(b, tr_list=None, st_tree=None, bt=None):
         nonlocal launches
-        o, k, v = batches[b]
+        o, k, v = (bt or batches)[b]
         ev[b][0].record(stream)
         if world == 1:
+            tr = (tr_list or trees)[(st_tree or step_tree)[b]]
             if cap:
-                tk = tree.submit_range(o, k, v, results[b], cap, *rrows[b])
+                tk = tr.submit_range(o, k, v, results[b], cap, *rrows[b])
             else:
-                tk = tree.submit(o, k, v, results[b])
+                tk = tr.submit(o, k, v, results[b])
             ev[b][1].record(stream)
-            return tk
+            return (tr, tk)
         st = sh.apply(o, k, v, results[b])
         ev[b][1].record(stream)
         return st
 
+    def fetch(r):
+        return r[0].results(r[1]) if world == 1 else r
+
     for b in range(args.warmup):
-        r = step(b)
-        stats.append(tree.results(r) if world == 1 else r)
+        stats.append(fetch(step(b)))
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
@@ -299,7 +327,7 @@ def run_ours(args):
             dist.barrier()
         torch.cuda.synchronize()
     for r in tickets:
-        stats.append(tree.results(r) if world == 1 else r)
+        stats.append(fetch(r))
     elapsed_ms = t_start.elapsed_time(t_end)
     per_batch_ms = np.array([ev[b][0].elapsed_time(ev[b][1]) for b in range(args.warmup, nb)])
     if os.environ.get("EIRENE_BENCH_VERBOSE"):
@@ -320,22 +348,35 @@ def run_ours(args):
     # shows the cost of direct launches).  Its batches reuse the pre-staged
     # input buffers of the first timed batches.
     stage_names = ["sort", "group", "query+range" if cap else "query", "update", "result"]
-    engine = tree if world == 1 else sh.engine
-    engine.set_flags(timing=True)
     n_stage = min(args.steps, 10)
+    if world == 1 and per_tree:
+        # fresh trees for the stage region too (a re-applied insert batch would not split)
+        _, s_trees, s_tree_of, s_hb = build_plan(1, n_stage)
+        # (indexed from args.warmup like the single-tree region: results[0..warmup) keep
+        # the parity batches)
+        s_batches = [None] * args.warmup + [tuple(torch.from_numpy(a).to(dev) for a in hb) for hb in s_hb]
+        s_tree_of = [0] * args.warmup + s_tree_of
+        engines = s_trees
+        stage_step = lambda i: step(args.warmup + i, s_trees, s_tree_of, s_batches)  # noqa: E731
+    else:
+        engines = [tree] if world == 1 else [sh.engine]
+        stage_step = lambda i: step(args.warmup + i)  # noqa: E731
+    for e_ in engines:
+        e_.set_flags(timing=True)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     sa = torch.cuda.Event(enable_timing=True)
     sz = torch.cuda.Event(enable_timing=True)
     sa.record(stream)
-    srs = [step(args.warmup + i) for i in range(n_stage)]
+    srs = [stage_step(i) for i in range(n_stage)]
     sz.record(stream)
-    sstats = [tree.results(r) for r in srs] if world == 1 else srs
+    sstats = [fetch(r) for r in srs]
     torch.cuda.synchronize()
     direct_ms = sa.elapsed_time(sz) / n_stage
     stage_ms = np.array([s["stage_ms"][:5] for s in sstats]).mean(axis=0)
-    engine.set_flags(timing=False)
+    for e_ in engines:
+        e_.set_flags(timing=False)
 
     # ------------------------------------------------------------ e2e through the public API (host buffers)
     e2e = None
@@ -380,11 +421,15 @@ def run_ours(args):
                "steps": n_e, "path": "torch pinned H2D copies + EireneTree.submit_range + D2H of counts and "
                                      "range rows, one stream"}
     elif world == 1 and args.e2e_steps > 0:
-        hb = [wl.batch_arrays(nb + i) for i in range(args.e2e_steps)]
+        if per_tree:
+            _, e_trees, e_tree_of, hb = build_plan(2, args.e2e_steps)
+        else:
+            hb = [wl.batch_arrays(nb + i) for i in range(args.e2e_steps)]
+            e_trees, e_tree_of = [tree], [0] * len(hb)
         pin = [tuple(torch.from_numpy(a).pin_memory() for a in x) for x in hb]
         hres = [torch.empty(batch_n, dtype=torch.uint64).pin_memory() for _ in hb]
-        tk = tree.submit_host(*pin[0], hres[0])   # warm the path
-        tree.results(tk)
+        tk = e_trees[e_tree_of[0]].submit_host(*pin[0], hres[0])   # warm the path
+        e_trees[e_tree_of[0]].results(tk)
         # first DMA touch of each freshly pinned buffer (IOMMU / page mapping) is a
         # one-time cost a serving process with long-lived staging buffers never
         # pays: touch every buffer once, untimed (no batch is run)
@@ -396,9 +441,9 @@ def run_ours(args):
         a = torch.cuda.Event(enable_timing=True)
         z = torch.cuda.Event(enable_timing=True)
         a.record(stream)
-        tks = [tree.submit_host(*pin[i], hres[i]) for i in range(1, len(pin))]
-        for t_ in tks:
-            tree.results(t_)   # waits for the batch's D2H (library's d2h stream)
+        tks = [(e_trees[e_tree_of[i]], e_trees[e_tree_of[i]].submit_host(*pin[i], hres[i])) for i in range(1, len(pin))]
+        for tr_, t_ in tks:
+            tr_.results(t_)   # waits for the batch's D2H (library's d2h stream)
         z.record(stream)       # after the last results() returned: covers every H2D, kernel and D2H
         torch.cuda.synchronize()
         e_ms = a.elapsed_time(z)
@@ -421,14 +466,18 @@ def run_ours(args):
     roof = None
     if rank == 0 and world == 1 and args.cpu_batches > 0:
         import oracle
-        ref = oracle.BTreeOracle(16)
-        t0 = time.time()
-        ref.load(wl.keys, wl.vals)
-        load_s = time.time() - t0
         n_check = min(args.cpu_batches, nb)
+        refs = {}
+        t0 = time.time()
+        for b in range(n_check):   # one oracle per tree (fresh-tree configs), bulk load untimed
+            if step_tree[b] not in refs:
+                refs[step_tree[b]] = oracle.BTreeOracle(16)
+                refs[step_tree[b]].load(wls[step_tree[b]].keys, wls[step_tree[b]].vals)
+        load_s = time.time() - t0
         cpu_t = 0.0
         bad = 0
         for b in range(n_check):
+            ref = refs[step_tree[b]]
             o, k, v = host_batches[b]
             a = time.perf_counter()
             if cap:
@@ -451,13 +500,14 @@ def run_ours(args):
         peaks = load_peaks()
         dom = int(np.argmax(stage_ms))
         if cap:
-            ab = [algorithmic_bytes_range(wl.keys, *host_batches[b], 16, cap)["bytes"]
+            ab = [algorithmic_bytes_range(wls[step_tree[b]].keys, *host_batches[b], 16, cap)["bytes"]
                   for b in range(args.warmup, min(nb, args.warmup + 4))]
             bytes_per = float(np.mean(ab))
             ms = stage_ms[2]
             kern = "range_kernel"
         elif stage_names[dom] == "query" or args.roofline_kernel == "query":
-            ab = [algorithmic_bytes_query(wl.keys, *host_batches[b][:2], 16)["bytes"] for b in range(args.warmup, min(nb, args.warmup + 4))]
+            ab = [algorithmic_bytes_query(wls[step_tree[b]].keys, *host_batches[b][:2], 16)["bytes"]
+                  for b in range(args.warmup, min(nb, args.warmup + 4))]
             bytes_per = float(np.mean(ab))
             ms = stage_ms[2]
             kern = "query_kernel"
@@ -468,11 +518,21 @@ def run_ours(args):
             bytes_per = batch_n * 20 + d * 17
             ms = stage_ms[1]
             kern = "group_kernel"
+        elif stage_names[dom] == "update":
+            # per issued write: its W-list entry (key, op, val, seg, leaf, slot: 26 B) and the
+            # returned old value (8 B); per touched leaf (leaf run) its 256 B block read and
+            # written back; per new leaf 256 B written (batch stats of the stage region)
+            lr = float(np.mean([x["leaf_runs"] for x in sstats]))
+            nlf = float(np.mean([x["new_leaves"] for x in sstats]))
+            iw = float(np.mean([x["issued_w"] for x in sstats]))
+            bytes_per = iw * 34 + lr * 512 + nlf * 256
+            ms = stage_ms[3]
+            kern = "update_kernel"
         else:
-            # bucket scatter: key 8 B + op 1 B read, 12 B written per request (+ hist pass 8 B)
-            bytes_per = batch_n * (8 + 9 + 12)
+            # distribution: key 8 B + op 1 B read, 12 B written per request
+            bytes_per = batch_n * (8 + 1 + 12)
             ms = stage_ms[0]
-            kern = "bsort_hist_kernel + bsort_scatter_kernel"
+            kern = "bsort_dist_kernel"
         ach = bytes_per / (ms * 1e-3) / 1e9
         # measured DRAM traffic of the same kernel per launch, from the committed
         # ncu capture (tools/ncu_traffic.sh -> profiles/traffic.json); null if absent

@@ -175,6 +175,13 @@ int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops_dev, const uin
                               uint32_t cap, uint64_t* range_keys_dev, uint64_t* range_vals_dev,
                               eirene_stream_t stream, uint64_t* ticket);
 
+/* Optional warm-up: captures and instantiates the CUDA graph that batches of
+ * exactly n requests (with_ranges != 0: submitted by eirene_submit_batch_range)
+ * replay, without launching anything and without touching the tree, so that
+ * the first such batch does not pay the capture.  A handle keeps graphs for a
+ * few distinct sizes.  Errors: EINVAL (n == 0 or n > max_batch), ECUDA. */
+int eirene_prepare_batch(eirene_handle h, uint32_t n, int with_ranges);
+
 /* Waits for batch `ticket` and returns its status (EIRENE_OK, EINVAL, EFULL);
  * fills *stats if non-NULL.  ESTATE if the ticket is unknown or too old (the
  * handle remembers the last 64 batches). */

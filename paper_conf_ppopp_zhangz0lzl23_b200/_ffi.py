@@ -56,6 +56,7 @@ _SIGS = {
     "eirene_bulk_load": (_int, [_vp, _vp, _vp, _u64, ctypes.c_float, _vp]),
     "eirene_submit_batch": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _vp, ctypes.POINTER(_u64)]),
     "eirene_submit_batch_host": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _vp, ctypes.POINTER(_u64)]),
+    "eirene_prepare_batch": (_int, [_vp, _u32, _int]),
     "eirene_submit_batch_range": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _u32, _vp, _vp, _vp, ctypes.POINTER(_u64)]),
     "eirene_results": (_int, [_vp, _u64, ctypes.POINTER(eirene_batch_stats)]),
     "eirene_scan": (_int, [_vp, _u64, _u64, _vp, _vp, _u64, ctypes.POINTER(_u64), _vp]),

@@ -257,6 +257,11 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->up.entA_child, nb + 64);
   AL(h->up.entB_key, nb + 64);
   AL(h->up.entB_child, nb + 64);
+  AL(h->up.slots[0], nb / 32 + 32768);
+  AL(h->up.slots[1], nb / 32 + 32768);
+  AL(h->up.eparent, nb + 64);
+  AL(h->up.nemask[0], 4096);
+  AL(h->up.nemask[1], 4096);
   AL(h->st_ops, HOST_SLOTS * nb);
   AL(h->st_keys, HOST_SLOTS * nb);
   AL(h->st_vals, HOST_SLOTS * nb);
@@ -386,13 +391,18 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals
 
 static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                        uint64_t* results, cudaStream_t st, uint64_t* vals_stage, uint64_t* ticket,
-                       uint64_t* rkeys = nullptr, uint64_t* rvals = nullptr, uint32_t rcap = 0) {
-  const bool range = rkeys != nullptr;
+                       uint64_t* rkeys = nullptr, uint64_t* rvals = nullptr, uint32_t rcap = 0,
+                       bool prepare_only = false, bool prepare_range = false) {
+  const bool range = rkeys != nullptr || prepare_range;
   CK(cudaSetDevice(h->cfg.device));
-  const uint64_t tk = h->next_ticket++;
-  Rec& r = h->ring[tk % RING];
-  r.ticket = tk;
-  r.used = true;
+  if (prepare_only && (!h->use_graphs || (h->cfg.flags & EIRENE_F_TIMING))) return EIRENE_OK;
+  const uint64_t tk = prepare_only ? 0 : h->next_ticket++;
+  Rec scratch_rec;
+  Rec& r = prepare_only ? scratch_rec : h->ring[tk % RING];
+  if (!prepare_only) {
+    r.ticket = tk;
+    r.used = true;
+  }
   r.n = n;
   r.timing = (h->cfg.flags & EIRENE_F_TIMING) != 0;
   int launches = 0;
@@ -471,6 +481,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       e.launches = launches;
       g = &e;
     }
+    if (prepare_only) return EIRENE_OK;   // graph captured and instantiated, nothing launched
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
                       const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
                       &rkeys, &rvals, &rcap};
@@ -498,6 +509,13 @@ int eirene_submit_batch(eirene_handle h, const uint8_t* ops, const uint64_t* key
   if (!h || !ops || !keys || !vals || !results || !ticket) return EIRENE_EINVAL;
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   return submit_impl(h, ops, keys, vals, n, results, reinterpret_cast<cudaStream_t>(stream), nullptr, ticket);
+}
+
+int eirene_prepare_batch(eirene_handle h, uint32_t n, int with_ranges) {
+  if (!h || n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
+  uint64_t tk = 0;
+  return submit_impl(h, nullptr, nullptr, nullptr, n, nullptr, nullptr, nullptr, &tk, nullptr, nullptr, 0, true,
+                     with_ranges != 0);
 }
 
 int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,

@@ -373,8 +373,13 @@ void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_
     // fused single launch; slices of whole 512-request rows per CTA
     const uint32_t rows = (n + D_THREADS - 1) / D_THREADS;
     const uint32_t per_cta = ((rows + grid - 1) / grid) * D_THREADS;
-    bsort_dist_kernel<<<grid, D_THREADS, 0, st>>>(A, n, G, per_cta, key_lo, key_hi, b.bcount, b.gstart, b.cursor,
-                                                  b.kA, b.pA, ctl);
+    // cooperative launch: the grid barrier needs every CTA co-resident, which a plain
+    // launch does not guarantee when other kernels share the device
+    void* args[] = {const_cast<BatchArgs**>(&A), &n, const_cast<uint32_t*>(&G), const_cast<uint32_t*>(&per_cta),
+                    &key_lo, &key_hi, const_cast<uint32_t**>(&b.bcount), const_cast<uint32_t**>(&b.gstart),
+                    const_cast<uint32_t**>(&b.cursor), const_cast<uint64_t**>(&b.kA), const_cast<uint32_t**>(&b.pA),
+                    &ctl};
+    cudaLaunchCooperativeKernel(reinterpret_cast<void*>(bsort_dist_kernel), dim3(grid), dim3(D_THREADS), args, 0, st);
     *launches += 1;
     return;
   }

@@ -63,6 +63,10 @@ struct BatchCtl {
   uint32_t nlong, gbar;   // gbar: grid barrier of bsort_dist_kernel
   uint32_t nrange, nart;  // range queries in the batch; artificial queries resolved
   uint32_t hot_ctr;       // hot-key timestamp bitmaps claimed by oversized groups
+  uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
+  uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
+  uint32_t lvl_ent[MAX_LEVELS];   // separator entries produced for level L+1 (update kernel)
+  unsigned long long uprof[24];   // diagnostic (EIRENE_UPDATE_PROF): update-kernel phase timestamps
   unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
   uint32_t dbg[8];   // watchdog diagnostics
 };
@@ -285,6 +289,9 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
 struct UpdParams {
   uint32_t threshold;
   uint32_t flags;
+  uint2* slots[2];      // per producer unit (base, n) of the level-synchronous separator lists
+  uint32_t* eparent;    // [n] parent node of each entry position (lookup step)
+  uint32_t* nemask[2];  // nonempty-producer bitmaps of the upper levels (one bit per warp)
   uint64_t* entA_key;
   uint32_t* entA_child;
   uint64_t* entB_key;

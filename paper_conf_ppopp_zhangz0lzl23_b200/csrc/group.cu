@@ -1093,11 +1093,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     }
     __syncthreads();
     const uint32_t sH = S.seg0 + a_nh, wH = S.w0 + a_nw, pos0 = base + sp_lo;
-    const unsigned long long th0 = g.prof ? gtime_ns() : 0;
     hot_pass2(g, S.hot_bits, hc, sH, pos0);
-    if ((g.prof & 1) && tid == 0)
-      printf("[hot prof] ticket %u h %u pass2 %.1f us, rest emit before %.1f us\n", b, hc.total, (gtime_ns() - th0) * 1e-3,
-             (th0 - tp3) * 1e-3);
     if (tid == 0) {
       const uint64_t hk = S.hk;
       g.istart[sH] = pos0;

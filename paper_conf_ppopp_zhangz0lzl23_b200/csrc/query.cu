@@ -62,7 +62,8 @@ __device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_
 __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
-                                                        const uint32_t* __restrict__ wseg, uint32_t* __restrict__ wleaf,
+                                                        const uint32_t* __restrict__ wseg,
+                                                        const uint8_t* __restrict__ wop, uint32_t* __restrict__ wleaf,
                                                         uint8_t* __restrict__ wslot, uint64_t* __restrict__ old,
                                                         const uint32_t* __restrict__ spay,
                                                         const uint32_t* __restrict__ pinfo,
@@ -97,6 +98,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
     uint32_t seg;
+    bool ins = false;   // an upsert of an absent key: the only request that can split a leaf
     if (isq) {
       seg = qseg[i];
     } else {
@@ -104,6 +106,11 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
       seg = wseg[w];
       wleaf[w] = node;
       wslot[w] = s >= 0 ? (uint8_t)s : (uint8_t)255;
+      ins = s < 0 && wop[w] != OP_DELETE;
+    }
+    {
+      const uint32_t m = __ballot_sync(__activemask(), ins);
+      if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&ctl->nins, (uint32_t)__popc(m));
     }
     old[seg] = v;
     const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
@@ -148,6 +155,12 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
     if (dbgprint)
       printf("[eirene dbg] %u %u %u %u %u %u %u %u\n", ctl->dbg[0], ctl->dbg[1], ctl->dbg[2], ctl->dbg[3],
              ctl->dbg[4], ctl->dbg[5], ctl->dbg[6], ctl->dbg[7]);
+    if (ctl->uprof[0]) {   // EIRENE_UPDATE_PROF: update-kernel phases (us since its start)
+      printf("[upd prof] entries %u %u %u %u %u | t:", ctl->lvl_ent[0], ctl->lvl_ent[1], ctl->lvl_ent[2],
+             ctl->lvl_ent[3], ctl->lvl_ent[4]);
+      for (int i = 1; i < 24 && ctl->uprof[i]; ++i) printf(" %.1f", (ctl->uprof[i] - ctl->uprof[0]) * 1e-3);
+      printf("\n");
+    }
   }
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
@@ -378,7 +391,7 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
   // one resident wave: 8 CTAs of 256 threads per SM at <= 32 registers
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
-  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wleaf, c.wslot, c.old, spay, c.pinfo,
+  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay, c.pinfo,
                                        c.istart, c.longseg, A, t, ctl);
   ++*launches;
 }

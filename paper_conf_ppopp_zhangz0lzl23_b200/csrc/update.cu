@@ -49,6 +49,9 @@ struct Ctx {
   bool regroup;
   bool stats;
   BatchCtl* ctl;
+  uint2* slots[2];      // level-synchronous propagation: per producer unit (base, n)
+  uint32_t* eparent;    // parent found for each entry position (lookup step)
+  uint32_t* nemask[2];  // nonempty producer bitmaps of the upper levels
 };
 
 struct WarpStats {
@@ -81,7 +84,7 @@ __device__ bool watchdog(const Ctx& C, WarpStats& ws, uint32_t where, uint32_t a
 constexpr uint32_t LEAF_TAG = 0x80000000u;
 
 __device__ __forceinline__ void backoff(uint32_t retry) {
-  uint32_t ns = 32u << (retry < 8 ? retry : 8);
+  uint32_t ns = 32u << (retry < 5 ? retry : 5);   // <= 1 us: lock holders finish in about that
   __nanosleep(ns);
 }
 
@@ -575,8 +578,46 @@ __device__ void insert_up(const Ctx& C, uint32_t L0, uint32_t eb0, uint32_t m0, 
   }
 }
 
+// Separator entries of a warp's leaf splits, gathered at [base, base + n) of
+// the level-0 entry buffer and inserted into the parents together (one parent
+// lock per parent instead of one per split leaf).  Each leaf_apply writes its
+// k-1 entries at [b, b+k-1) inside its own run [b, e); runs are processed in
+// key order, so the entries are compacted leftwards in key order.
+struct SepAcc {
+  uint32_t base = NIL, n = 0;
+};
+__device__ void acc_entries_buf(uint64_t* EK, uint32_t* EC, SepAcc& A, uint32_t b, uint32_t cnt) {
+  const int lane = lane_id();
+  if (A.base == NIL) A.base = b;
+  const uint32_t dst = A.base + A.n;
+  if (dst != b) {
+    for (uint32_t x0 = 0; x0 < cnt; x0 += 32) {   // dst < b: a forward copy in warp chunks is safe
+      const uint32_t x = x0 + lane;
+      uint64_t k = 0;
+      uint32_t c = 0;
+      if (x < cnt) {
+        k = ld_cg(EK + b + x);
+        c = ld_cg(EC + b + x);
+      }
+      __syncwarp();
+      if (x < cnt) {
+        EK[dst + x] = k;
+        EC[dst + x] = c;
+      }
+      __syncwarp();
+    }
+    __threadfence();
+    __syncwarp();
+  }
+  A.n += cnt;
+}
+__device__ __forceinline__ void acc_entries(const Ctx& C, SepAcc& A, uint32_t b, uint32_t cnt) {
+  acc_entries_buf(C.eK[0], C.eC[0], A, b, cnt);
+}
+
 // One run of writes [b, e) whose first key was located in leaf `hint`.
-__device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint, WarpStats& ws) {
+// Separators of its leaf splits are added to `acc` (inserted by the caller).
+__device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint, WarpStats& ws, SepAcc& acc) {
   const int lane = lane_id();
   const Tree& t = C.t;
   uint32_t retry = 0;
@@ -615,7 +656,7 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
               rooted = true;
             }
             unlock(vp, v + 2u);   // split: version + 1 step
-            if (!rooted) insert_up(C, 0, b, k - 1, ws);
+            if (!rooted) acc_entries(C, acc, b, k - 1);
           } else {
             unlock(vp, v);
           }
@@ -637,9 +678,279 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
   }
 }
 
-__global__ void __launch_bounds__(128) update_kernel(Ctx C) {
+
+// ---------------------------------------------------------------- level-synchronous separators
+// Under a split storm (cfg1: every leaf splits; cfg4) per-warp upward
+// insertion makes every warp whose leaves share a parent queue on that
+// parent's lock, and every split parent's warp queue on the grandparent's,
+// up to the root.  When the batch can split (some issued upsert targets an
+// absent key, ctl->nins), the kernel is a persistent grid and separators go
+// up one level at a time instead (the regrouping of a4 applied to the inner
+// levels):
+//   level 0: every warp applies its leaf runs; each 32-write chunk leaves its
+//            separators contiguous at [base, base+n) of entry buffer 0 and
+//            records (base, n) in slots[0][chunk] -- chunk order = key order;
+//   lookup : (grid barrier) every entry's parent at level L+1, by an
+//            unprotected per-thread descent of the level-quiescent tree;
+//   apply  : (grid barrier) the entries of one parent form one segment; the
+//            warp whose unit range holds the segment's first entry owns it,
+//            gathers it (in place, leftwards), locks the parent, validates its
+//            fences (Alg.1:38) and merges the whole segment (inner_apply,
+//            multi-way split); the next level's separators are recorded per
+//            warp in slots[1 - x].  A root split builds the new root(s).
+// Owners are unique per parent, so the locks are uncontended; a failed
+// validation (not expected) falls back to insert_up's optimistic / STM retry.
+__device__ int g_uprof = 0;   // diagnostic: print the phase times of the level-synchronous path
+__device__ void grid_barrier(BatchCtl* ctl, uint32_t& gen) {
+  const uint32_t bi = gen / gridDim.x;
+  if (g_uprof && blockIdx.x == 0 && threadIdx.x == 0 && 2 * bi + 2 < 24) ctl->uprof[2 * bi + 1] = gtime_ns();
+  __syncthreads();
+  gen += gridDim.x;
+  if (threadIdx.x == 0) {
+    __threadfence();
+    atomicAdd(&ctl->ubar, 1u);
+    SpinGuard sg;
+    while (ld_acquire(&ctl->ubar) < gen) {
+      __nanosleep(64);
+      if (sg.stuck(ctl)) break;
+    }
+    if (g_uprof && blockIdx.x == 0 && 2 * bi + 2 < 24) ctl->uprof[2 * bi + 2] = gtime_ns();
+  }
+  __syncthreads();
+}
+
+// Node at level `target` (>= 1) whose fences hold k: one thread, unprotected
+// (the inner levels are quiescent during a lookup step), B-link move-right.
+__device__ uint32_t descend_thread(const Tree& t, uint64_t k, uint32_t target) {
+  const unsigned long long rw = ld_acquire64(&t.hdr->root_word);
+  const uint32_t height = (uint32_t)(rw >> 32);
+  uint32_t node = (uint32_t)rw;
+  if (height == 0 || target + 1 > height) return NIL;
+  uint32_t lvl = height - 1;
+  for (int steps = 0; steps < 4096; ++steps) {
+    const NodeMeta* m = t.imeta + node;
+    const uint64_t hi = ld_cg(&m->hi);
+    const uint32_t nxt = ld_cg(&m->next);
+    if (k >= hi && nxt != NIL) {
+      node = nxt;
+      continue;
+    }
+    if (lvl == target) return node;
+    const uint64_t* kl = t.ikeys + (size_t)node * FAN;
+    uint32_t c = 0;
+#pragma unroll
+    for (int i = 0; i < FAN - 1; ++i) c += ld_cg(kl + i) <= k ? 1u : 0u;
+    node = ld_cg(t.ichild + (size_t)node * FAN + c);
+    --lvl;
+  }
+  return NIL;
+}
+
+// Nonempty-unit bitmaps of the upper levels (producer = warp): first set unit
+// >= from (U if none) / last set unit < before (NIL if none), 1024 units per step.
+__device__ uint32_t mask_next(const uint32_t* mk, uint32_t U, uint32_t from) {
+  const int lane = lane_id();
+  for (uint32_t wb = from >> 5; wb * 32 < U; wb += 32) {
+    const uint32_t w = wb + lane;
+    uint32_t word = w * 32 < U ? ld_cg(mk + w) : 0u;
+    if (w == (from >> 5)) word &= ~((1u << (from & 31)) - 1u);
+    const uint32_t bm = __ballot_sync(FULL, word != 0);
+    if (bm) {
+      const int l = __ffs(bm) - 1;
+      const uint32_t wd = __shfl_sync(FULL, word, l);
+      const uint32_t unit = (wb + l) * 32 + (__ffs(wd) - 1);
+      return unit < U ? unit : U;
+    }
+  }
+  return U;
+}
+__device__ uint32_t mask_prev(const uint32_t* mk, uint32_t before) {
+  const int lane = lane_id();
+  for (int64_t we = (int64_t)((before + 31) >> 5); we > 0; we -= 32) {
+    const int64_t w = we - 32 + lane;
+    uint32_t word = w >= 0 ? ld_cg(mk + w) : 0u;
+    if (w == (int64_t)(before >> 5)) word &= (1u << (before & 31)) - 1u;
+    if (w > (int64_t)(before >> 5)) word = 0;
+    const uint32_t bm = __ballot_sync(FULL, word != 0);
+    if (bm) {
+      const int l = 31 - __clz(bm);
+      const uint32_t wd = __shfl_sync(FULL, word, l);
+      return (uint32_t)(we - 32 + l) * 32 + (31 - __clz(wd));
+    }
+  }
+  return NIL;
+}
+
+// units [u0, u1) of a level's producer list, for this warp
+__device__ __forceinline__ void unit_range(uint32_t U, uint32_t gw, uint32_t nwarps, uint32_t& u0, uint32_t& u1) {
+  u0 = (uint32_t)(((unsigned long long)U * gw) / nwarps);
+  u1 = (uint32_t)(((unsigned long long)U * (gw + 1)) / nwarps);
+}
+
+// Propagate the separators of level L (entries in buffer L&1, producer list
+// slots[x] with U units) up to the root.
+__device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps, uint32_t& gen, WarpStats& ws) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  for (uint32_t L = 0; L + 1 < MAX_LEVELS; ++L) {
+    grid_barrier(C.ctl, gen);
+    if (ld_cg(&C.ctl->lvl_ent[L]) == 0) return;   // uniform: read after the barrier by every warp
+    const uint2* sl = C.slots[L & 1];
+    uint2* sn = C.slots[(L + 1) & 1];
+    uint64_t* K = C.eK[L & 1];
+    uint32_t* Ch = C.eC[L & 1];
+    uint64_t* K2 = C.eK[(L + 1) & 1];
+    uint32_t* Ch2 = C.eC[(L + 1) & 1];
+    uint32_t u0, u1;
+    unit_range(U, gw, nwarps, u0, u1);
+    // the next level's nonempty mask (its producers are warps): cleared here, before the apply step
+    if ((gw & 31) == 0 && lane == 0) C.nemask[(L + 1) & 1][gw >> 5] = 0u;
+    // lookup step: parent of every entry (lanes over units, then over a unit's entries)
+    for (uint32_t ub = u0; ub < u1; ub += 32) {
+      const uint32_t u = ub + lane;
+      const uint2 su = u < u1 ? sl[u] : make_uint2(0, 0);
+      for (uint32_t x = 0; x < su.y; ++x) C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
+    }
+    grid_barrier(C.ctl, gen);
+    // apply step
+    SepAcc nxt;
+    // parent of the last entry before my range (the owner test of my first entry)
+    uint32_t prevP = NIL;
+    const uint32_t* mk = C.nemask[L & 1];   // (L >= 1: nonempty producers)
+    if (L > 0) {
+      const uint32_t pu = mask_prev(mk, u0);
+      if (pu != NIL) {
+        const uint2 su = sl[pu];
+        prevP = ld_cg(C.eparent + su.x + su.y - 1);
+      }
+    }
+    for (uint32_t ue = L > 0 ? 0u : u0; ue > 0;) {   // level 0: nearest nonempty chunk before u0, 32 per step
+      const uint32_t ub = ue > 32 ? ue - 32 : 0;
+      const uint32_t uu = ub + lane;
+      const uint2 su = uu < ue ? sl[uu] : make_uint2(0, 0);
+      const uint32_t ne = __ballot_sync(FULL, su.y != 0);
+      if (ne) {
+        const int hl = 31 - __clz(ne);
+        const uint32_t bx = __shfl_sync(FULL, su.x, hl), by = __shfl_sync(FULL, su.y, hl);
+        prevP = ld_cg(C.eparent + bx + by - 1);
+        break;
+      }
+      ue = ub;
+    }
+    // next unit >= from with entries (U if none), 32 units per step
+    auto next_nonempty = [&](uint32_t from) -> uint32_t {
+      if (L > 0) return mask_next(mk, U, from);
+      for (uint32_t ub = from; ub < U; ub += 32) {
+        const uint32_t uu = ub + lane;
+        const bool ne = uu < U && sl[uu].y != 0;
+        const uint32_t bm = __ballot_sync(FULL, ne);
+        if (bm) return ub + __ffs(bm) - 1;
+      }
+      return U;
+    };
+    uint32_t u = u0, x = 0;   // cursor: entry x of unit u
+    while (u < u1 && !ws.dead) {
+      const uint2 su = sl[u];
+      if (x >= su.y) {
+        u = next_nonempty(u + 1);
+        x = 0;
+        continue;
+      }
+      const uint32_t hpos = su.x + x;
+      const uint32_t P = ld_cg(C.eparent + hpos);
+      if (P == prevP) {   // continues a segment owned by an earlier warp / segment
+        ++x;
+        continue;
+      }
+      // a segment head in my range: gather its entries to [hpos, hpos + m)
+      uint32_t m = 0, cu = u, cx = x;
+      for (;;) {
+        if (cu >= U) break;
+        const uint2 sc = sl[cu];
+        if (cx >= sc.y) {
+          cu = next_nonempty(cu + 1);
+          cx = 0;
+          continue;
+        }
+        // entries cx.. of unit cu with parent P (lane-parallel, stops at the first other parent)
+        const uint32_t avail = sc.y - cx;
+        uint32_t take = 0;
+        for (uint32_t b0 = 0; b0 < avail; b0 += 32) {
+          const uint32_t q = b0 + lane;
+          const bool same = q < avail && ld_cg(C.eparent + sc.x + cx + q) == P;
+          const uint32_t bm = __ballot_sync(FULL, q < avail && !same);
+          const uint32_t upto = bm ? (uint32_t)(__ffs(bm) - 1) : min(32u, avail - b0);
+          // move [b0, b0 + upto) to [hpos + m + b0, ...) (leftwards or in place)
+          uint64_t kk = 0;
+          uint32_t cc = 0;
+          if ((uint32_t)lane < upto) {
+            kk = ld_cg(K + sc.x + cx + b0 + lane);
+            cc = ld_cg(Ch + sc.x + cx + b0 + lane);
+          }
+          __syncwarp();
+          if ((uint32_t)lane < upto) {
+            K[hpos + m + b0 + lane] = kk;
+            Ch[hpos + m + b0 + lane] = cc;
+          }
+          __syncwarp();
+          take = b0 + upto;
+          if (bm) break;
+        }
+        m += take;
+        cx += take;
+        if (cx < sc.y) break;   // another parent's entry: the segment ends here
+      }
+      __threadfence();
+      __syncwarp();
+      // lock the parent, validate, merge the whole segment
+      uint32_t* vp = &t.imeta[P].version;
+      uint32_t v;
+      bool done = false;
+      if (P != NIL && try_lock(vp, &v)) {
+        const size_t pb = (size_t)P * FAN;
+        const uint64_t pk = lane < FAN ? ld_cg(t.ikeys + pb + lane) : KEY_MAX;
+        const uint32_t pc = lane < FAN ? ld_cg(t.ichild + pb + lane) : NIL;
+        const uint32_t cP = ld_cg(&t.imeta[P].count);
+        const uint64_t plo = ld_cg(&t.imeta[P].lo), phi = ld_cg(&t.imeta[P].hi);
+        const uint32_t pnext = ld_cg(&t.imeta[P].next);
+        const uint64_t s0 = ld_cg(K + hpos), s1 = ld_cg(K + hpos + m - 1);
+        if (s0 >= plo && s1 < phi) {
+          uint32_t next_m = inner_apply(C, P, L + 1, pk, pc, cP, plo, phi, pnext, K, Ch, K2, Ch2, hpos, m, ws);
+          if (next_m > 0 && is_root(t, P, L + 1)) {
+            build_root(C, L + 1, P, plo, phi, K2, Ch2, K, Ch, hpos, next_m, ws);
+            next_m = 0;
+          }
+          unlock(vp, v + 2u);
+          if (next_m) acc_entries_buf(K2, Ch2, nxt, hpos, next_m);
+          done = true;
+        } else {
+          unlock(vp, v);
+        }
+      }
+      if (!done) {   // not expected: the generic optimistic / STM path, one level at a time upward
+        ws.retries += 1;
+        insert_up(C, L, hpos, m, ws);
+      }
+      prevP = P;
+      u = cu;
+      x = cx;
+      if (u >= u1) break;   // the segment ran past my range: the rest belongs to it
+    }
+    if (lane == 0) {
+      sn[gw] = make_uint2(nxt.base == NIL ? 0u : nxt.base, nxt.n);
+      if (nxt.n) {
+        atomicAdd(&C.ctl->lvl_ent[L + 1], nxt.n);
+        atomicOr(&C.nemask[(L + 1) & 1][gw >> 5], 1u << (gw & 31));
+      }
+    }
+    U = nwarps;
+  }
+}
+
+__global__ void __launch_bounds__(128, 8) update_kernel(Ctx C) {
   const BatchCtl* ctl = C.ctl;
-  if (ctl->invalid || ctl->status != 0) return;
+  if (ctl->invalid || ctl->status != 0) return;   // (uniform: every CTA leaves, no barrier is reached)
+  if (g_uprof && blockIdx.x == 0 && threadIdx.x == 0) C.ctl->uprof[0] = gtime_ns();
   const uint32_t nw = ctl->nw;
   const int lane = lane_id();
   const uint32_t gw = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -647,6 +958,10 @@ __global__ void __launch_bounds__(128) update_kernel(Ctx C) {
   const Tree& t = C.t;
   WarpStats ws;
   ws.t0 = gtime_ns();
+  SepAcc acc;
+  // level-synchronous separators when the batch can split (launch: resident grid)
+  const bool lsync = C.regroup && C.slots[0] != nullptr && ctl->nins > 0;
+  const uint32_t nchunks = (nw + 31) / 32;
   if (C.regroup) {
     for (uint32_t chunk = gw; chunk * 32 < nw; chunk += nwarps) {
       const uint32_t base = chunk * 32;
@@ -722,12 +1037,29 @@ __global__ void __launch_bounds__(128) update_kernel(Ctx C) {
             if (s + 32 >= nw) e = nw;
           }
         }
-        process_run(C, b, e, leaf, ws);
+        process_run(C, b, e, leaf, ws, acc);
         if (ws.dead) break;
       }
+      if (lsync) {
+        if (lane == 0) {
+          C.slots[0][chunk] = make_uint2(acc.base == NIL ? 0u : acc.base, acc.n);
+          if (acc.n) atomicAdd(&C.ctl->lvl_ent[0], acc.n);
+        }
+      } else if (acc.n && !ws.dead) {
+        insert_up(C, 0, acc.base, acc.n, ws);
+      }
+      acc = SepAcc{};
+    }
+    if (lsync) {
+      uint32_t gen = 0;
+      levels_up(C, nchunks, gw, nwarps, gen, ws);
     }
   } else {
-    for (uint32_t j = gw; j < nw && !ws.dead; j += nwarps) process_run(C, j, j + 1, C.wleaf[j], ws);
+    for (uint32_t j = gw; j < nw && !ws.dead; j += nwarps) {
+      SepAcc one;
+      process_run(C, j, j + 1, C.wleaf[j], ws, one);
+      if (one.n && !ws.dead) insert_up(C, 0, one.base, one.n, ws);
+    }
   }
   if (C.stats) {
     // reduce the counters per CTA first: one global atomic per CTA and counter
@@ -773,15 +1105,38 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
   C.regroup = (p.flags & EIRENE_F_REGROUP) != 0;
   C.stats = (p.flags & EIRENE_F_STATS) != 0;
   C.ctl = ctl;
+  C.slots[0] = p.slots[0];
+  C.slots[1] = p.slots[1];
+  C.eparent = p.eparent;
+  C.nemask[0] = p.nemask[0];
+  C.nemask[1] = p.nemask[1];
   const uint32_t warps_needed = C.regroup ? (n + 31) / 32 : n;
   uint32_t blocks = (warps_needed + 3) / 4;
-  blocks = std::min<uint32_t>(blocks, (uint32_t)num_sms * 8u);
+  // the level-synchronous phases need every CTA resident (grid barriers)
+  static int per_sm = -1;
+  if (per_sm < 0 && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, update_kernel, 128, 0) != cudaSuccess)
+    per_sm = 0;
+  const uint32_t resident = (uint32_t)num_sms * (uint32_t)std::max(per_sm, 0);
+  blocks = std::min<uint32_t>(blocks, resident ? resident : (uint32_t)num_sms * 4u);
   if (blocks < 1) blocks = 1;
+  static const bool no_lsync = std::getenv("EIRENE_NO_LSYNC") != nullptr;   // A/B: per-warp insertion only
+  if (!resident || no_lsync) C.slots[0] = nullptr;   // no residency guarantee: per-warp insertion only
   static const char* serial = std::getenv("EIRENE_UPDATE_SERIAL");   // debug: one warp, no concurrency
+  static bool prof_set = false;
+  if (!prof_set) {
+    const int on = std::getenv("EIRENE_UPDATE_PROF") != nullptr;
+    cudaMemcpyToSymbol(g_uprof, &on, sizeof(int));
+    prof_set = true;
+  }
   if (serial) {
     update_kernel<<<1, 32, 0, st>>>(C);
   } else {
-    update_kernel<<<blocks, 128, 0, st>>>(C);
+    if (C.slots[0]) {   // grid barriers: cooperative launch (co-residency guaranteed)
+      void* args[] = {&C};
+      cudaLaunchCooperativeKernel(reinterpret_cast<void*>(update_kernel), dim3(blocks), dim3(128), args, 0, st);
+    } else {
+      update_kernel<<<blocks, 128, 0, st>>>(C);
+    }
   }
   ++*launches;
 }

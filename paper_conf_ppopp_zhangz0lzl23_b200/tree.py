@@ -104,6 +104,10 @@ class EireneTree:
                                           self._stream(stream), ctypes.byref(tk)), "eirene_submit_batch")
         return tk.value
 
+    def prepare(self, n: int, ranges: bool = False):
+        """Capture the batch graph for n-request batches ahead of the first one (no launch)."""
+        check(self._L.eirene_prepare_batch(self._h, n, 1 if ranges else 0), "eirene_prepare_batch")
+
     def submit_range(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor,
                      cap: int, range_keys: torch.Tensor, range_vals: torch.Tensor, stream=None) -> int:
         """Batch that may hold range queries (op RANGE = 4, key = l, val = u, inclusive):

@@ -188,10 +188,12 @@ def make_batch(loaded: np.ndarray, n: int, fracs: dict[int, float], dist: str, s
 # ---------------------------------------------------------------- configs
 # BASELINE.json configs[0..4] == cfg1..cfg5; seed = 0xE1E2E3E4 + cfg.
 CONFIGS = {
-    1: dict(tree=1 << 16, batch=1 << 16, fracs={QUERY: 0.5, INSERT: 0.5}, dist="uniform"),
+    # per_tree: steps per freshly bulk-loaded tree in the bench (cfg1 one batch
+    # per fresh tree, cfg4 ~4 insert-heavy batches per seed until >= 2^22 live keys)
+    1: dict(tree=1 << 16, batch=1 << 16, fracs={QUERY: 0.5, INSERT: 0.5}, dist="uniform", per_tree=1),
     2: dict(tree=1 << 24, batch=1 << 20, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="uniform"),
     3: dict(tree=1 << 24, batch=1 << 20, fracs={QUERY: 0.5, UPDATE: 0.5}, dist="zipf"),
-    4: dict(tree=1 << 20, batch=1 << 20, fracs={INSERT: 0.9, DELETE: 0.1}, dist="uniform"),
+    4: dict(tree=1 << 20, batch=1 << 20, fracs={INSERT: 0.9, DELETE: 0.1}, dist="uniform", per_tree=4),
     5: dict(tree=1 << 28, batch=1 << 24, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="zipf"),
     # the paper's pure range-query workload (Fig.13), length 8
     6: dict(tree=1 << 24, batch=1 << 20, fracs={RANGE: 1.0}, dist="uniform", range_len=8),

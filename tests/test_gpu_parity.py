@@ -376,3 +376,23 @@ def test_route_partition_unpermute(dev):
     assert np.array_equal(sops.cpu().numpy(), ops[order])
     back = t.route_unpermute(skeys, perm)
     assert np.array_equal(back.cpu().numpy(), ks)
+
+
+def test_prepare_batch_then_submit(dev):
+    """eirene_prepare_batch captures the graph without touching the tree; the
+    batches that follow replay it and stay bit-exact."""
+    rng = np.random.default_rng(77)
+    keys, vals = _rand_keys(rng, 5000)
+    t = make_tree(dev, keys, vals)
+    t.prepare(4096)
+    t.prepare(4096, ranges=True)
+    k, v = t.scan()
+    assert np.array_equal(k.cpu().numpy(), keys) and np.array_equal(v.cpu().numpy(), vals)
+    ref = oracle.MapOracle()
+    ref.load(keys, vals)
+    for b in range(3):
+        ops = rng.integers(0, 4, 4096).astype(np.uint8)
+        ks = np.where(rng.random(4096) < 0.5, keys[rng.integers(0, keys.size, 4096)],
+                      rng.integers(1, 1 << 40, 4096, dtype=np.uint64))
+        vs = rng.integers(0, 1 << 62, 4096, dtype=np.uint64)
+        run_and_compare(t, ref, ops, ks, vs, dev)
