@@ -72,3 +72,14 @@ def test_product_package_never_imports_oracle():
         if f.endswith((".cpp", ".h")):
             text = open(os.path.join(root, "oracle", f)).read()
             assert "eirene.h\"" not in text.replace("eirene_oracle.h\"", "") and "csrc" not in text.split("*/")[-1]
+
+
+def test_range_and_prepare_argument_checks_without_gpu(libpath):
+    """The range entry point and the graph warm-up validate their arguments on
+    the host (EINVAL) before touching the device."""
+    L = _ffi.lib()
+    tk = ctypes.c_uint64()
+    assert L.eirene_submit_batch_range(None, None, None, None, 1, None, 8, None, None, None,
+                                       ctypes.byref(tk)) == _ffi.EIRENE_EINVAL
+    assert L.eirene_prepare_batch(None, 16, 0) == _ffi.EIRENE_EINVAL
+    assert _ffi.EIRENE_RANGE == 4
