@@ -223,6 +223,12 @@ def run_ours(args):
     if cap and world > 1:
         raise SystemExit("range-query configs run on one GPU (DESIGN.md §7)")
 
+    # query traversal: the default (one key-sorted request per thread, path
+    # sharing) or the paper's iteration warps + range field (ablation)
+    qmode = {"iterwarp": args.query_mode == "iterwarp", "iter_rgs": args.iter_rgs}
+    if args.query_mode != "default" and world > 1:
+        raise SystemExit("--query-mode iterwarp runs on one GPU")
+
     # ------------------------------------------------------------ inputs
     t_gen = time.time()
     per_tree = C.get("per_tree", 0)
@@ -239,7 +245,7 @@ def run_ours(args):
                     for t in range(ntr)]
             trees_ = []
             for w_ in wls_:
-                tr = EireneTree(max_keys=tree_n + per_tree * batch_n + (1 << 12), max_batch=batch_n)
+                tr = EireneTree(max_keys=tree_n + per_tree * batch_n + (1 << 12), max_batch=batch_n, **qmode)
                 tr.bulk_load(torch.from_numpy(w_.keys).to(dev), torch.from_numpy(w_.vals).to(dev))
                 tr.prepare(batch_n, bool(cap))   # graph capture outside every timed region
                 trees_.append(tr)
@@ -253,7 +259,7 @@ def run_ours(args):
             wl = W.Workload(cfg, tree=tree_n, batch=batch_n)
             keys_d = torch.from_numpy(wl.keys).to(dev)
             vals_d = torch.from_numpy(wl.vals).to(dev)
-            tree = EireneTree(max_keys=max(tree_n * 2, 1 << 20), max_batch=batch_n)
+            tree = EireneTree(max_keys=max(tree_n * 2, 1 << 20), max_batch=batch_n, **qmode)
             tree.bulk_load(keys_d, vals_d)
             del keys_d, vals_d
             wls, trees, step_tree = [wl], [tree], [0] * nb
@@ -576,6 +582,13 @@ def run_ours(args):
             "parity": parity,
             "setup_s": gen_s,
         }
+        if args.query_mode == "iterwarp":
+            tot = lambda f: int(sum(s_[f] for s_ in stats[args.warmup:]))   # noqa: E731
+            issued = tot("issued_q") + tot("issued_w")
+            line["config"]["query_mode"] = f"iterwarp (iter_rgs {args.iter_rgs or 'auto'})"
+            line["traversal"] = {"rg_vertical": tot("rg_vertical"), "rg_horizontal": tot("rg_horizontal"),
+                                 "steps_per_issued": tot("trav_steps") / max(1, issued),
+                                 "vertical_steps_per_issued": float(stats[-1]["height"])}
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
@@ -595,6 +608,9 @@ def main():
     ap.add_argument("--ref-sample", type=int, default=1 << 18)
     ap.add_argument("--roofline-kernel", default="auto")
     ap.add_argument("--backend", default="nccl", choices=["nccl", "gloo"])
+    ap.add_argument("--query-mode", default="default", choices=["default", "iterwarp"],
+                    help="iterwarp: the paper's iteration warps + range field (ablation)")
+    ap.add_argument("--iter-rgs", type=int, default=0, help="RGs per iteration warp (0 = auto)")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

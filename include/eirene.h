@@ -64,7 +64,13 @@ enum {
   EIRENE_F_STATS = 1u << 1,     /* count retries / STM fallbacks / splits on the device           */
   EIRENE_F_FORCE_STM = 1u << 2, /* every traversal in the update kernel is STM-protected
                                    (equivalent to retry_threshold = 0, Alg.1:28-33)               */
-  EIRENE_F_TIMING = 1u << 3     /* record per-stage CUDA events (eirene_batch_stats.stage_ms)     */
+  EIRENE_F_TIMING = 1u << 3,    /* record per-stage CUDA events (eirene_batch_stats.stage_ms)     */
+  EIRENE_F_ITERWARP = 1u << 4   /* query kernel: the paper's iteration warps with a per-leaf range
+                                   field (RF) choosing vertical (root-to-leaf) or horizontal
+                                   (leaf-link) traversal per request group (Fig.6);
+                                   off = one key-sorted request per thread with path sharing (the
+                                   default).  Results are identical either way;
+                                   with EIRENE_F_STATS the batch stats report the decisions      */
 };
 
 typedef struct {
@@ -76,10 +82,13 @@ typedef struct {
   uint32_t flags;             /* EIRENE_F_*                                                    */
   uint64_t key_lo, key_hi;    /* key range owned by this tree (shard), [key_lo, key_hi);
                                  0 .. UINT64_MAX for a single GPU                              */
+  uint32_t iter_rgs;          /* EIRENE_F_ITERWARP: request groups (32 issued requests each) per
+                                 iteration warp; 0 = spread the RGs evenly over the resident
+                                 warps                                           */
 } eirene_config;
 
 /* Fills *cfg with the defaults: device 0, fanout 16, max_keys 2^24,
- * max_batch 2^20, retry_threshold 4, flags REGROUP|STATS, range [0, UINT64_MAX). */
+ * max_batch 2^20, retry_threshold 4, flags REGROUP|STATS, range [0, UINT64_MAX), iter_rgs 0. */
 void eirene_default_config(eirene_config* cfg);
 
 typedef struct eirene_tree* eirene_handle;
@@ -104,6 +113,11 @@ typedef struct {
                                  [5], [6] unused, [7] total                                    */
   uint64_t ranges;            /* range queries in the batch (eirene_submit_batch_range)         */
   uint64_t artificial;        /* artificial queries resolved for them               */
+  uint64_t trav_steps;        /* EIRENE_F_ITERWARP|STATS: nodes visited by the issued requests'
+                                 traversals (vertical: height; horizontal: 1 + links followed;
+                                 Fig.10 "traversal steps"); 0 otherwise            */
+  uint64_t rg_vertical;       /* EIRENE_F_ITERWARP|STATS: request groups traversed from the root */
+  uint64_t rg_horizontal;     /* ... and along the leaf links from the iteration warp's buffer  */
 } eirene_batch_stats;
 
 /* Creates a tree (one empty leaf) on cfg->device and allocates every pool and

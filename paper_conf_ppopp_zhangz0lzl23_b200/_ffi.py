@@ -18,7 +18,7 @@ HEADER = os.path.join(ROOT, "include", "eirene.h")
 
 EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECUDA = 0, -1, -2, -3, -4, -5
 EIRENE_QUERY, EIRENE_UPDATE, EIRENE_INSERT, EIRENE_DELETE, EIRENE_RANGE = 0, 1, 2, 3, 4
-EIRENE_F_REGROUP, EIRENE_F_STATS, EIRENE_F_FORCE_STM, EIRENE_F_TIMING = 1, 2, 4, 8
+EIRENE_F_REGROUP, EIRENE_F_STATS, EIRENE_F_FORCE_STM, EIRENE_F_TIMING, EIRENE_F_ITERWARP = 1, 2, 4, 8, 16
 NOT_FOUND = 0xFFFFFFFFFFFFFFFF
 
 _u64 = ctypes.c_uint64
@@ -29,7 +29,8 @@ _int = ctypes.c_int
 
 class eirene_config(ctypes.Structure):
     _fields_ = [("device", ctypes.c_int), ("fanout", _u32), ("max_keys", _u64), ("max_batch", _u32),
-                ("retry_threshold", _u32), ("flags", _u32), ("key_lo", _u64), ("key_hi", _u64)]
+                ("retry_threshold", _u32), ("flags", _u32), ("key_lo", _u64), ("key_hi", _u64),
+                ("iter_rgs", _u32)]
 
 
 class eirene_batch_stats(ctypes.Structure):
@@ -37,7 +38,8 @@ class eirene_batch_stats(ctypes.Structure):
                 ("issued_w", _u64), ("leaf_runs", _u64), ("retries", _u64), ("stm_fallbacks", _u64),
                 ("leaf_splits", _u64), ("inner_splits", _u64), ("new_leaves", _u64), ("new_inner", _u64),
                 ("height", _u32), ("launches", _u32), ("stage_ms", ctypes.c_float * 8),
-                ("ranges", _u64), ("artificial", _u64)]
+                ("ranges", _u64), ("artificial", _u64), ("trav_steps", _u64), ("rg_vertical", _u64),
+                ("rg_horizontal", _u64)]
 
     def to_dict(self) -> dict:
         d = {f: getattr(self, f) for f, _ in self._fields_ if f != "stage_ms"}

@@ -55,6 +55,7 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
     m.count = 0;
     m.level = 0;
     t.lmeta[0] = m;
+    t.lrf[0] = KEY_MAX;   // no leaf `height` links to the right
     TreeHdr* h = t.hdr;
     h->root_word = (1ull << 32) | 0ull;
     h->leaf_count = 1;
@@ -230,6 +231,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(t.lkeys, leaf_cap * LSTRIDE);   // keys and values of a leaf share one 256 B block
   if (e == cudaSuccess) t.lvals = t.lkeys + FAN;
   AL(t.lmeta, leaf_cap);
+  AL(t.lrf, leaf_cap);
   AL(t.ikeys, inner_cap * FAN);
   AL(t.ichild, inner_cap * FAN);
   AL(t.imeta, inner_cap);
@@ -446,7 +448,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     const uint32_t* spay = h->bs.pB;
     stage("group");
     if (timing) rec(2, s);
-    launch_query(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, s, &launches);
+    launch_query(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, h->cfg.flags, h->cfg.iter_rgs, s, &launches);
     if (range) launch_range(n, h->cb, spay, h->bs.kB, h->dargs, h->t, ctl, h->num_sms, s, &launches);
     stage("query");
     if (timing) rec(3, s);
@@ -602,6 +604,9 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) 
     stats->launches = (uint32_t)r.launches;
     stats->ranges = c.nrange;
     stats->artificial = c.nart;
+    stats->trav_steps = c.trav_steps;
+    stats->rg_vertical = c.rg_vertical;
+    stats->rg_horizontal = c.rg_horizontal;
     if (r.timing) {
       for (int s = 0; s + 1 < NSTAGE; ++s) cudaEventElapsedTime(&stats->stage_ms[s], r.st[s], r.st[s + 1]);
       cudaEventElapsedTime(&stats->stage_ms[7], r.st[0], r.st[NSTAGE - 1]);

@@ -65,6 +65,8 @@ struct BatchCtl {
   uint32_t hot_ctr;       // hot-key timestamp bitmaps claimed by oversized groups
   uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
   uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
+  uint32_t rg_vertical, rg_horizontal;   // EIRENE_F_ITERWARP: RGs traversed vertically / horizontally
+  unsigned long long trav_steps;         // EIRENE_F_ITERWARP: traversal steps of the issued requests
   uint32_t lvl_ent[MAX_LEVELS];   // separator entries produced for level L+1 (update kernel)
   unsigned long long uprof[24];   // diagnostic (EIRENE_UPDATE_PROF): update-kernel phase timestamps
   unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
@@ -121,6 +123,7 @@ struct Tree {
   uint64_t* lkeys;   // leaf L: keys at lkeys[L * LSTRIDE + s]
   uint64_t* lvals;   // = lkeys + FAN: values at lvals[L * LSTRIDE + s]
   NodeMeta* lmeta;
+  uint64_t* lrf;     // range field of every leaf (EIRENE_F_ITERWARP)
   uint64_t* ikeys;
   uint32_t* ichild;
   NodeMeta* imeta;
@@ -284,7 +287,7 @@ constexpr int GROUP_STATUS_WORDS = NBINS;   // >= bsort_groups(n) for every n
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches);
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
-                  int num_sms, cudaStream_t st, int* launches);
+                  int num_sms, uint32_t flags, uint32_t iter_rgs, cudaStream_t st, int* launches);
 
 struct UpdParams {
   uint32_t threshold;

@@ -59,6 +59,69 @@ __device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_
   return s;
 }
 
+// Everything after the locate of issued request i (list position i < nq:
+// query, else write i - nq) at leaf `node`, slot s (-1 = absent), value v:
+// the write's leaf/slot for the update kernel, the segment's old value, and
+// the fused RESULT_CAL of its pending positions (long segments queued).
+struct QueryIO {
+  const uint32_t* __restrict__ qseg;
+  const uint32_t* __restrict__ wseg;
+  const uint8_t* __restrict__ wop;
+  uint32_t* __restrict__ wleaf;
+  uint8_t* __restrict__ wslot;
+  uint64_t* __restrict__ old;
+  const uint32_t* __restrict__ spay;
+  const uint32_t* __restrict__ pinfo;
+  const uint32_t* __restrict__ istart;
+  uint32_t* __restrict__ longseg;
+};
+
+__device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, uint32_t nq, uint32_t node, int s,
+                                       uint64_t v, uint64_t* __restrict__ results, BatchCtl* __restrict__ ctl) {
+  const uint32_t* __restrict__ qseg = io.qseg;
+  const uint32_t* __restrict__ wseg = io.wseg;
+  const uint8_t* __restrict__ wop = io.wop;
+  uint32_t* __restrict__ wleaf = io.wleaf;
+  uint8_t* __restrict__ wslot = io.wslot;
+  uint64_t* __restrict__ old = io.old;
+  const uint32_t* __restrict__ spay = io.spay;
+  const uint32_t* __restrict__ pinfo = io.pinfo;
+  const uint32_t* __restrict__ istart = io.istart;
+  uint32_t* __restrict__ longseg = io.longseg;
+  uint32_t seg;
+  bool ins = false;   // an upsert of an absent key: the only request that can split a leaf
+  if (isq) {
+    seg = qseg[i];
+  } else {
+    const uint32_t w = i - nq;
+    seg = wseg[w];
+    wleaf[w] = node;
+    wslot[w] = s >= 0 ? (uint8_t)s : (uint8_t)255;
+    ins = s < 0 && wop[w] != OP_DELETE;
+  }
+  {
+    const uint32_t m = __ballot_sync(__activemask(), ins);
+    if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&ctl->nins, (uint32_t)__popc(m));
+  }
+  old[seg] = v;
+  const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
+  if (p1 - p0 <= SHORT_SEG) {
+    if (isq) {   // an all-query segment: every position is pending
+      for (uint32_t p = p0; p < p1; ++p) results[spay[p] >> 2] = v;
+    } else {     // positions up to (and including) the first write are pending
+      for (uint32_t p = p0; p < p1; ++p)
+        if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
+    }
+  } else {   // work items of RCHUNK positions: (segment, chunk) pairs
+    const uint32_t nc = (p1 - p0 + RCHUNK - 1) / RCHUNK;
+    const uint32_t at = atomicAdd(&ctl->nlong, nc);
+    for (uint32_t c = 0; c < nc; ++c) {
+      longseg[2 * (at + c)] = seg;
+      longseg[2 * (at + c) + 1] = c;
+    }
+  }
+}
+
 __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
@@ -97,38 +160,107 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
     }
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
-    uint32_t seg;
-    bool ins = false;   // an upsert of an absent key: the only request that can split a leaf
-    if (isq) {
-      seg = qseg[i];
-    } else {
-      const uint32_t w = i - nq;
-      seg = wseg[w];
-      wleaf[w] = node;
-      wslot[w] = s >= 0 ? (uint8_t)s : (uint8_t)255;
-      ins = s < 0 && wop[w] != OP_DELETE;
-    }
-    {
-      const uint32_t m = __ballot_sync(__activemask(), ins);
-      if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&ctl->nins, (uint32_t)__popc(m));
-    }
-    old[seg] = v;
-    const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
-    if (p1 - p0 <= SHORT_SEG) {
-      if (isq) {   // an all-query segment: every position is pending
-        for (uint32_t p = p0; p < p1; ++p) results[spay[p] >> 2] = v;
-      } else {     // positions up to (and including) the first write are pending
-        for (uint32_t p = p0; p < p1; ++p)
-          if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
+    retire(QueryIO{qseg, wseg, wop, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
+           results, ctl);
+  }
+}
+
+// Locality-aware warp reorganisation the paper's way (§5, P:1380-1512,
+// Fig.6): an ablation of the default traversal above (EIRENE_F_ITERWARP).
+// Request groups (RGs) are 32 consecutive issued requests of the key-sorted
+// query list, then of the write list; an ITERATION WARP runs `iter` adjacent
+// RGs one after the other -- iter = iter_rgs, or with 0 the RGs
+// evenly spread over the resident warps.  The warp keeps a
+// buffer (leaf, RF): the first RG, or one whose MAXIMAL key exceeds the
+// buffered RF, descends from the root (vertical, `height`
+// nodes); otherwise every lane walks the leaf links from the buffered leaf
+// (horizontal, 1 + links nodes).  The buffer then holds the leaf
+// of the RG's maximal key and its RF.  RF(leaf) = lo fence of
+// the leaf `height` links to the right (reading 22, set at bulk load and
+// inherited by split-off leaves); a walk longer than `height` repairs the
+// start leaf's RF lazily.  Correctness never depends on RF: a
+// horizontal walk starts at the leaf of a smaller key of the same sorted list
+// and follows B-link `next` pointers until k < hi, so RF only chooses the
+// cheaper way.  With EIRENE_F_STATS the kernel counts vertical / horizontal
+// RGs and traversal steps (Fig.10).
+__global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* __restrict__ qkey,
+                                                                 const uint64_t* __restrict__ wkey, QueryIO io,
+                                                                 const BatchArgs* __restrict__ A, Tree t,
+                                                                 BatchCtl* __restrict__ ctl, uint32_t iter_rgs,
+                                                                 uint32_t stats) {
+  if (ctl->invalid || ctl->status != 0) return;
+  uint64_t* __restrict__ results = A->results;
+  const uint32_t nq = ctl->nq, nw = ctl->nw;
+  const uint32_t rq = (nq + 31) / 32, nrg = rq + (nw + 31) / 32;
+  const unsigned long long rw = t.hdr->root_word;
+  const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
+  const uint32_t lane = threadIdx.x & 31;
+  const uint32_t nwarps = (gridDim.x * blockDim.x) >> 5;
+  const uint32_t iter = iter_rgs ? iter_rgs : max(1u, (nrg + nwarps - 1) / nwarps);
+  const uint64_t pl = pol_evict_last(), pf = pol_evict_first();
+  unsigned long long nsteps = 0;
+  uint32_t nvert = 0, nhor = 0;
+  for (uint32_t w = (blockIdx.x * blockDim.x + threadIdx.x) >> 5; (uint64_t)w * iter < nrg; w += nwarps) {
+    uint32_t buf_leaf = NIL;   // empty buffer: the first RG traverses vertically
+    uint64_t buf_rf = 0;
+    const uint64_t rend = (uint64_t)w * iter + iter;
+    const uint32_t r1 = rend < nrg ? (uint32_t)rend : nrg;
+    for (uint32_t r = w * iter; r < r1; ++r) {
+      const bool isq = r < rq;
+      if (r == rq) buf_leaf = NIL;   // the write list starts over at small keys
+      const uint32_t base = (isq ? r : r - rq) * 32;
+      const uint32_t cnt = min(32u, (isq ? nq : nw) - base);
+      const bool act = lane < cnt;
+      const uint64_t* __restrict__ kl = isq ? qkey : wkey;
+      const uint64_t kmax = kl[base + cnt - 1];   // sorted list: the RG's maximal key
+      const uint64_t k = act ? kl[base + lane] : kmax;
+      const bool vertical = buf_leaf == NIL || kmax > buf_rf;
+      uint32_t node, steps;
+      uint64_t rep = 0;
+      if (vertical) {
+        node = root;
+        for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
+          const uint64_t* kp = t.ikeys + (size_t)node * FAN;
+          ulonglong4 kv[4];
+#pragma unroll
+          for (int x = 0; x < 4; ++x) kv[x] = ldg256_l1(kp + 4 * x, pl);
+          uint32_t c = 0;
+#pragma unroll
+          for (int x = 0; x < 4; ++x) c += (kv[x].x <= k) + (kv[x].y <= k) + (kv[x].z <= k) + (kv[x].w <= k);
+          node = ldg32_pol(t.ichild + (size_t)node * FAN + c, pl);
+        }
+        steps = height;
+      } else {
+        node = buf_leaf;
+        steps = 1;
+        while (k >= t.lmeta[node].hi) {   // the tree is quiescent here
+          node = t.lmeta[node].next;
+          if (++steps == height + 1) rep = t.lmeta[node].lo;   // the leaf `height` links right of the start
+        }
       }
-    } else {   // work items of RCHUNK positions: (segment, chunk) pairs
-      const uint32_t nc = (p1 - p0 + RCHUNK - 1) / RCHUNK;
-      const uint32_t at = atomicAdd(&ctl->nlong, nc);
-      for (uint32_t c = 0; c < nc; ++c) {
-        longseg[2 * (at + c)] = seg;
-        longseg[2 * (at + c) + 1] = c;
+      const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
+      const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
+      if (act) retire(io, isq ? base + lane : nq + base + lane, isq, nq, node, s, v, results, ctl);
+      __syncwarp();
+      const uint32_t top = __shfl_sync(FULL, node, cnt - 1);
+      const uint32_t rm = __ballot_sync(FULL, act && steps > height);
+      if (rm) {   // lazy RF repair of the start leaf; every such lane found the same leaf
+        rep = shfl64(rep, __ffs(rm) - 1);
+        if (lane == 0) t.lrf[buf_leaf] = rep;
+      }
+      buf_rf = (rm && top == buf_leaf) ? rep : __ldcg(reinterpret_cast<const unsigned long long*>(t.lrf + top));
+      buf_leaf = top;
+      if (stats) {
+        nsteps += __reduce_add_sync(FULL, act ? steps : 0u);
+        nvert += vertical ? 1u : 0u;
+        nhor += vertical ? 0u : 1u;
       }
     }
+  }
+  if (stats && lane == 0 && (nvert | nhor)) {
+    atomicAdd(&ctl->trav_steps, nsteps);
+    atomicAdd(&ctl->rg_vertical, nvert);
+    atomicAdd(&ctl->rg_horizontal, nhor);
   }
 }
 
@@ -387,12 +519,20 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
 }  // namespace
 
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
-                  int num_sms, cudaStream_t st, int* launches) {
+                  int num_sms, uint32_t flags, uint32_t iter_rgs, cudaStream_t st, int* launches) {
   // one resident wave: 8 CTAs of 256 threads per SM at <= 32 registers
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
-  query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay, c.pinfo,
-                                       c.istart, c.longseg, A, t, ctl);
+  if (flags & EIRENE_F_ITERWARP) {
+    // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
+    const int iblocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 4u);
+    query_iterwarp_kernel<<<iblocks < 1 ? 1 : iblocks, 256, 0, st>>>(
+        c.qkey, c.wkey, QueryIO{c.qseg, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
+        A, t, ctl, iter_rgs, (flags & EIRENE_F_STATS) ? 1u : 0u);
+  } else {
+    query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay,
+                                         c.pinfo, c.istart, c.longseg, A, t, ctl);
+  }
   ++*launches;
 }
 

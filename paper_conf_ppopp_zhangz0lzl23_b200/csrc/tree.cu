@@ -42,6 +42,14 @@ __global__ void build_leaves_kernel(const uint64_t* __restrict__ keys, const uin
   }
 }
 
+// Range field of every bulk-loaded leaf (reading 22): the min
+// key (= lo fence) of the leaf `height` links to the right, KEY_MAX past the
+// end of the chain.  Bulk-loaded leaf ids are their chain positions.
+__global__ void build_rf_kernel(Tree t, uint32_t L, uint32_t height) {
+  const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i < L) t.lrf[i] = (uint64_t)i + height < L ? t.lmeta[i + height].lo : KEY_MAX;
+}
+
 // One inner level over nc children with consecutive ids [cbase, cbase+nc)
 // (leaves when child_level == 0), nn = ceil(nc/16) nodes, even distribution.
 __global__ void build_inner_kernel(Tree t, uint32_t child_level, uint32_t cbase, uint32_t nc, uint32_t nbase,
@@ -172,6 +180,8 @@ int build_tree(Tree t, const uint64_t* keys, const uint64_t* vals, uint64_t n, i
   hdr.inner_count = nbase;
   hdr.root_word = ((unsigned long long)(level + 1) << 32) | cbase;
   *height_out = level + 1;
+  build_rf_kernel<<<(L + 255) / 256, 256, 0, st>>>(t, L, level + 1);
+  ++*launches;
   cudaMemcpyAsync(t.hdr, &hdr, sizeof(hdr), cudaMemcpyHostToDevice, st);
   cudaStreamSynchronize(st);
   return EIRENE_OK;

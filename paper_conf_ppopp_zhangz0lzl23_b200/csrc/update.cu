@@ -368,6 +368,7 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
       mt.count = bs + (q < rem ? 1u : 0u);
       mt.level = 0;
       t.lmeta[id] = mt;
+      t.lrf[id] = t.lrf[X];   // split-off leaves inherit the RF (repaired lazily)
     }
     __threadfence();
     __syncwarp();

@@ -41,7 +41,8 @@ class EireneTree:
 
     def __init__(self, max_keys: int = 1 << 24, max_batch: int = 1 << 20, device: int | None = None,
                  retry_threshold: int = 4, regroup: bool = True, stats: bool = True, force_stm: bool = False,
-                 timing: bool = False, key_lo: int = 0, key_hi: int = U64_MAX):
+                 timing: bool = False, key_lo: int = 0, key_hi: int = U64_MAX, iterwarp: bool = False,
+                 iter_rgs: int = 0):
         L = _ffi.lib()
         if device is None:
             device = torch.cuda.current_device()
@@ -53,7 +54,9 @@ class EireneTree:
         cfg.max_batch = max_batch
         cfg.retry_threshold = retry_threshold
         cfg.flags = ((_ffi.EIRENE_F_REGROUP if regroup else 0) | (_ffi.EIRENE_F_STATS if stats else 0) |
-                     (_ffi.EIRENE_F_FORCE_STM if force_stm else 0) | (_ffi.EIRENE_F_TIMING if timing else 0))
+                     (_ffi.EIRENE_F_FORCE_STM if force_stm else 0) | (_ffi.EIRENE_F_TIMING if timing else 0) |
+                     (_ffi.EIRENE_F_ITERWARP if iterwarp else 0))
+        cfg.iter_rgs = iter_rgs
         cfg.key_lo = key_lo
         cfg.key_hi = key_hi
         self.cfg = cfg
@@ -184,10 +187,11 @@ class EireneTree:
         return rc, nk.value
 
     def set_flags(self, regroup: bool | None = None, stats: bool | None = None, force_stm: bool | None = None,
-                  timing: bool | None = None):
+                  timing: bool | None = None, iterwarp: bool | None = None):
         f = self.cfg.flags
         for on, bit in ((regroup, _ffi.EIRENE_F_REGROUP), (stats, _ffi.EIRENE_F_STATS),
-                        (force_stm, _ffi.EIRENE_F_FORCE_STM), (timing, _ffi.EIRENE_F_TIMING)):
+                        (force_stm, _ffi.EIRENE_F_FORCE_STM), (timing, _ffi.EIRENE_F_TIMING),
+                        (iterwarp, _ffi.EIRENE_F_ITERWARP)):
             if on is not None:
                 f = (f | bit) if on else (f & ~bit)
         self.cfg.flags = f
