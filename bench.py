@@ -215,6 +215,12 @@ def run_ours(args):
         tree_n = args.tree
     if args.batch:
         batch_n = args.batch
+    # cfg5: ONE 2^28-key tree and 2^24-request global batches at
+    # every N -- strong scaling; the other configs are per-GPU sizes (weak)
+    strong = bool(C.get("strong")) and world > 1
+    if strong:
+        tree_n //= world
+        batch_n //= world
     nb = args.warmup + args.steps
     stream = torch.cuda.current_stream(dev)
     # range-query workload: eirene_submit_batch_range with
@@ -556,8 +562,8 @@ def run_ours(args):
         line = {
             "metric": "requests/sec per batch", "value": value, "unit": "Greq/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps,
-            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64",
-            "data": "synthetic",
+            "higher_is_better": True, "scaling": "strong" if C.get("strong") else "weak", "vs_baseline": None,
+            "dtype": "u64", "data": "synthetic",
             "config": {"workload": f"cfg{cfg}: {tree_n * world} u64 keys (fanout 16, fill 1.0), "
                                    f"{batch_n * world}-request batches, "
                                    + ", ".join(f"{int(p * 100)}% {['query', 'update', 'insert', 'delete', 'range'][o]}"

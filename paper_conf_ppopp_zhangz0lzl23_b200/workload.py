@@ -194,7 +194,7 @@ CONFIGS = {
     2: dict(tree=1 << 24, batch=1 << 20, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="uniform"),
     3: dict(tree=1 << 24, batch=1 << 20, fracs={QUERY: 0.5, UPDATE: 0.5}, dist="zipf"),
     4: dict(tree=1 << 20, batch=1 << 20, fracs={INSERT: 0.9, DELETE: 0.1}, dist="uniform", per_tree=4),
-    5: dict(tree=1 << 28, batch=1 << 24, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="zipf"),
+    5: dict(tree=1 << 28, batch=1 << 24, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="zipf", strong=True),
     # the paper's pure range-query workload (Fig.13), length 8
     6: dict(tree=1 << 24, batch=1 << 20, fracs={RANGE: 1.0}, dist="uniform", range_len=8),
 }
