@@ -70,10 +70,12 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
 __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys,
                                                         const uint64_t* vals_src, uint64_t* vals_stage,
                                                         uint64_t* results, BatchCtl* ctl_out, uint4* zero,
-                                                        uint32_t zero_n16, uint64_t* rkeys, uint64_t* rvals,
-                                                        uint32_t rcap) {
+                                                        uint32_t zero_n16, uint4* zero2, uint32_t zero2_n16,
+                                                        uint64_t* rkeys, uint64_t* rvals, uint32_t rcap) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
     zero[i] = make_uint4(0, 0, 0, 0);
+  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero2_n16; i += gridDim.x * blockDim.x)
+    zero2[i] = make_uint4(0, 0, 0, 0);
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     dst->ops = ops;
     dst->keys = keys;
@@ -128,6 +130,12 @@ struct eirene_tree {
   UpdParams up{};
   unsigned char* zero_region = nullptr;
   size_t zero_bytes = 0;
+  // the two-kernel bucket sort of batches > 2^22 requests (16384 bins): its
+  // bin counts, group cursors and group look-back words, zeroed only for them
+  unsigned char* zero_large = nullptr;
+  size_t zero_large_bytes = 0;
+  BSortBufs bsL{};
+  CombBufs cbL{};
   BatchCtl* ctl = nullptr;
   BatchCtl* host_ctl = nullptr;   // pinned [RING]: landing buffer of eirene_results
   BatchCtl* ctl_ring = nullptr;   // device [RING]: each batch's final BatchCtl (written by result_long)
@@ -277,8 +285,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   }
   AL(h->route_lb, ((nb + 2047) / 2048) * 64);
   AL(h->route_ctr, 1);
-  AL(h->bs.gstart, NBINS + 1);
-  AL(h->bs.bin2grp, NBINS);
+  AL(h->bs.gstart, NBINS_MAX + 1);
+  AL(h->bs.bin2grp, NBINS_MAX);
   AL(h->dargs, 1);
   AL(h->ctl_ring, RING);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
@@ -294,9 +302,15 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     const size_t o_gh = bump(sizeof(uint32_t) * 8 * 256);
     const size_t o_bc = bump(sizeof(uint32_t) * NBINS);
     const size_t o_cu = bump(sizeof(uint32_t) * NBINS);
-    const size_t o_gs = bump(sizeof(unsigned long long) * GROUP_STATUS_WORDS);
+    const size_t o_gs = bump(sizeof(unsigned long long) * NBINS);
     h->zero_bytes = off;
     AL(h->zero_region, off);
+    off = 0;
+    const size_t l_bc = bump(sizeof(uint32_t) * NBINS_L);
+    const size_t l_cu = bump(sizeof(uint32_t) * NBINS_L);
+    const size_t l_gs = bump(sizeof(unsigned long long) * NBINS_L);
+    h->zero_large_bytes = off;
+    if (nb > (1u << 22)) AL(h->zero_large, off);
     if (e == cudaSuccess) {
       h->ctl = reinterpret_cast<BatchCtl*>(h->zero_region + o_ctl);
       h->sb.ghist = reinterpret_cast<uint32_t*>(h->zero_region + o_gh);
@@ -307,6 +321,13 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
       h->bs.kB = h->sb.kB;
       h->bs.pB = h->sb.pB;
       h->cb.group_status = reinterpret_cast<unsigned long long*>(h->zero_region + o_gs);
+      h->bsL = h->bs;
+      h->cbL = h->cb;
+      if (h->zero_large) {
+        h->bsL.bcount = reinterpret_cast<uint32_t*>(h->zero_large + l_bc);
+        h->bsL.cursor = reinterpret_cast<uint32_t*>(h->zero_large + l_cu);
+        h->cbL.group_status = reinterpret_cast<unsigned long long*>(h->zero_large + l_gs);
+      }
     }
   }
 #undef AL
@@ -378,6 +399,7 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals
   int launches = 0;
   uint32_t* flag = &h->ctl->invalid;
   CK(cudaMemsetAsync(h->zero_region, 0, h->zero_bytes, st));
+  if (h->zero_large) CK(cudaMemsetAsync(h->zero_large, 0, h->zero_large_bytes, st));
   launch_validate_bulk(keys, vals, n, h->cfg.key_lo, h->cfg.key_hi, flag, st, &launches);
   uint32_t bad = 0;
   CK(cudaMemcpyAsync(&bad, flag, sizeof(uint32_t), cudaMemcpyDeviceToHost, st));
@@ -432,19 +454,24 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   BatchCtl* ctl_slot = h->ctl_ring + tk % RING;
   uint4* zero16 = reinterpret_cast<uint4*>(h->zero_region);
   uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
+  const bool large = n > (1u << 22);   // two-kernel bucket sort with 16384 bins (bsort.cu)
+  uint4* zero2 = reinterpret_cast<uint4*>(large ? h->zero_large : h->zero_region);
+  uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
+  const BSortBufs& bsn = large ? h->bsL : h->bs;
+  const CombBufs& cbn = large ? h->cbL : h->cb;
   auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
     set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
-                                                   zero_n16, rkeys, rvals, rcap);
+                                                   zero_n16, zero2, zero2_n16, rkeys, rvals, rcap);
     ++launches;
     if (args_node) {
       cudaError_t e = last_node(s, args_node);
       if (e != cudaSuccess) return e;
     }
     if (timing) rec(0, s);
-    launch_bucket_sort(h->dargs, n, h->cfg.key_lo, h->cfg.key_hi, h->bs, ctl, h->num_sms, s, &launches);
+    launch_bucket_sort(h->dargs, n, h->cfg.key_lo, h->cfg.key_hi, bsn, ctl, h->num_sms, s, &launches);
     stage("sort");
     if (timing) rec(1, s);
-    launch_group(h->dargs, n, h->bs, h->cb, h->t, ctl, h->num_sms, s, &launches);
+    launch_group(h->dargs, n, bsn, cbn, h->t, ctl, h->num_sms, s, &launches);
     const uint32_t* spay = h->bs.pB;
     stage("group");
     if (timing) rec(2, s);
@@ -486,7 +513,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     if (prepare_only) return EIRENE_OK;   // graph captured and instantiated, nothing launched
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
                       const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
-                      &rkeys, &rvals, &rcap};
+                      &zero2, &zero2_n16, &rkeys, &rvals, &rcap};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
     p.gridDim = dim3(SET_ARGS_CTAS);

@@ -5,7 +5,8 @@
 // Requests must end up ordered by (key, logical timestamp); the payload of a
 // request is ts<<2 | op and ts is unique, so ordering by (key, payload) is the
 // (key, timestamp) order and this pass need not be stable.
-//   K0 hist    : histogram of the top BIN_BITS key bits (4096 bins); the last
+//   K0 hist    : histogram of the top bits of key - key_lo (bin_of: 4096 bins in
+//                the fused kernel, 16384 above 2^22 requests); the last
 //                CTA to finish scans the bins and cuts them into G groups of
 //                ~n/G requests each (a bin never straddles two groups):
 //                group(bin) = floor((excl(bin) + cnt(bin)/2) * G / n), and
@@ -42,35 +43,38 @@ constexpr int S_ITEMS = 8;
 constexpr int S_TILE = S_THREADS * S_ITEMS;      // 2048
 
 __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* __restrict__ A, uint32_t n,
-                                                               uint32_t G, uint32_t* __restrict__ bcount,
+                                                               uint32_t G, uint64_t key_lo, uint32_t bshift,
+                                                               uint32_t* __restrict__ bcount,
                                                                uint16_t* __restrict__ bin2grp,
                                                                uint32_t* __restrict__ gstart,
                                                                uint32_t* __restrict__ cursor, BatchCtl* ctl) {
-  __shared__ uint32_t h[2 * NBINS];   // two copies (even / odd warps); reused by the last CTA
+  extern __shared__ __align__(16) uint32_t h[];   // [2 * NBINS_L]: counts; the last CTA's cut (groups, prefixes)
   __shared__ uint32_t s_last;
   __shared__ uint32_t wsum[H_THREADS / 32];
   __shared__ uint32_t s_total;
   const uint64_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  for (uint32_t i = tid; i < 2 * NBINS; i += H_THREADS) h[i] = 0;
+  for (uint32_t i = tid; i < NBINS_L; i += H_THREADS) h[i] = 0;
   __syncthreads();
-  uint32_t* hw = h + (warp & 1) * NBINS;
-  const uint32_t t0 = blockIdx.x * (H_THREADS * H_ITEMS);
-  uint64_t k[H_ITEMS];
-  bool pt[H_ITEMS];   // point request (range queries do not enter the sort)
+  // grid-stride over tiles of H_THREADS * H_ITEMS requests: one flush of the
+  // CTA's histogram for all its tiles
+  for (uint32_t t0 = blockIdx.x * (H_THREADS * H_ITEMS); t0 < n; t0 += gridDim.x * (H_THREADS * H_ITEMS)) {
+    uint64_t k[H_ITEMS];
+    bool pt[H_ITEMS];   // point request (range queries do not enter the sort)
 #pragma unroll
-  for (int j = 0; j < H_ITEMS; ++j) {
-    const uint32_t i = t0 + j * H_THREADS + tid;
-    k[j] = i < n ? keys[i] : 0;
-    pt[j] = i < n && ops[i] != OP_RANGE;
+    for (int j = 0; j < H_ITEMS; ++j) {
+      const uint32_t i = t0 + j * H_THREADS + tid;
+      k[j] = i < n ? keys[i] : 0;
+      pt[j] = i < n && ops[i] != OP_RANGE;
+    }
+#pragma unroll
+    for (int j = 0; j < H_ITEMS; ++j)
+      if (pt[j]) atomicAdd(&h[bin_of(k[j], key_lo, bshift, NBINS_L)], 1u);
   }
-#pragma unroll
-  for (int j = 0; j < H_ITEMS; ++j)
-    if (pt[j]) atomicAdd(&hw[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
   __syncthreads();
-  for (uint32_t i = tid; i < NBINS; i += H_THREADS) {
-    const uint32_t c = h[i] + h[NBINS + i];
+  for (uint32_t i = tid; i < NBINS_L; i += H_THREADS) {
+    const uint32_t c = h[i];
     if (c) atomicAdd(&bcount[i], c);
   }
   __syncthreads();
@@ -81,8 +85,8 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
   __syncthreads();
   if (!s_last) return;
   __threadfence();
-  // last CTA: exclusive scan of the bins (16 per thread), then the group cut
-  constexpr int PER = NBINS / H_THREADS;
+  // last CTA: exclusive scan of the bins (32 per thread), then the group cut
+  constexpr int PER = NBINS_L / H_THREADS;
   uint32_t cnt[PER];
   uint32_t s = 0;
 #pragma unroll
@@ -103,9 +107,9 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
   if (tid == H_THREADS - 1) s_total = run + s;   // point requests in the batch
   __syncthreads();
   const uint32_t total = s_total;
-  uint32_t* sg = h;            // group of every bin
-  uint32_t* se = h + NBINS;    // exclusive prefix of every bin
-  const bool identity = G == (uint32_t)NBINS;
+  uint32_t* sg = h;              // group of every bin
+  uint32_t* se = h + NBINS_L;    // exclusive prefix of every bin
+  const bool identity = G == (uint32_t)NBINS_L;
 #pragma unroll
   for (int j = 0; j < PER; ++j) {
     const uint32_t bin = tid * PER + j;
@@ -119,14 +123,14 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
   }
   __syncthreads();
   // group g starts at the first bin mapped to it (empty groups start where the next one does)
-  for (uint32_t bin = tid; bin < (uint32_t)NBINS; bin += H_THREADS) {
+  for (uint32_t bin = tid; bin < (uint32_t)NBINS_L; bin += H_THREADS) {
     const uint32_t g = sg[bin];
     const uint32_t gp = bin ? sg[bin - 1] : 0xFFFFFFFFu;
     for (uint32_t q = gp + 1; q <= g; ++q) {
       gstart[q] = se[bin];
       cursor[q] = se[bin];
     }
-    if (bin == NBINS - 1)
+    if (bin == NBINS_L - 1)
       for (uint32_t q = g + 1; q <= G; ++q) gstart[q] = total;
   }
 }
@@ -137,18 +141,18 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
 // scatter.  Request validation rides on this pass: it reads
 // every key and op anyway, and the value only of writes.
 __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
-    const BatchArgs* __restrict__ A, uint32_t n, uint32_t G, uint64_t key_lo, uint64_t key_hi,
+    const BatchArgs* __restrict__ A, uint32_t n, uint32_t G, uint64_t key_lo, uint64_t key_hi, uint32_t bshift,
     const uint16_t* __restrict__ bin2grp, uint32_t* __restrict__ cursor, uint64_t* __restrict__ kout,
     uint32_t* __restrict__ pout, BatchCtl* ctl) {
   extern __shared__ __align__(16) unsigned char smem[];
-  uint16_t* s_b2g = reinterpret_cast<uint16_t*>(smem);           // [NBINS]
-  uint32_t* hist = reinterpret_cast<uint32_t*>(s_b2g + NBINS);   // [G] tile counts, then global base
+  uint16_t* s_b2g = reinterpret_cast<uint16_t*>(smem);             // [NBINS_L]
+  uint32_t* hist = reinterpret_cast<uint32_t*>(s_b2g + NBINS_L);   // [G] tile counts, then global base
   const uint64_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
   const uint64_t* __restrict__ vals = A->vals_src;
   uint64_t* __restrict__ vstage = A->vals_stage;
   const int tid = threadIdx.x;
-  for (uint32_t i = tid; i < (uint32_t)NBINS; i += S_THREADS) s_b2g[i] = bin2grp[i];
+  for (uint32_t i = tid; i < (uint32_t)NBINS_L; i += S_THREADS) s_b2g[i] = bin2grp[i];
   for (uint32_t i = tid; i < G; i += S_THREADS) hist[i] = 0;
   const uint32_t t0 = blockIdx.x * S_TILE;
   uint64_t k[S_ITEMS];
@@ -177,7 +181,7 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
 #pragma unroll
   for (int j = 0; j < S_ITEMS; ++j) {
     const uint32_t i = t0 + j * S_THREADS + tid;
-    g[j] = s_b2g[(uint32_t)(k[j] >> (64 - BIN_BITS))];
+    g[j] = s_b2g[bin_of(k[j], key_lo, bshift, NBINS_L)];
     r[j] = (i < n && o[j] != OP_RANGE) ? atomicAdd(&hist[g[j]], 1u) : 0u;
   }
   __syncthreads();
@@ -210,7 +214,7 @@ constexpr int D_THREADS = 512;
 constexpr int D_ITEMS = 8;
 __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
     const BatchArgs* __restrict__ A, uint32_t n, uint32_t G, uint32_t per_cta, uint64_t key_lo, uint64_t key_hi,
-    uint32_t* __restrict__ bcount, uint32_t* __restrict__ gstart, uint32_t* __restrict__ cursor,
+    uint32_t bshift, uint32_t* __restrict__ bcount, uint32_t* __restrict__ gstart, uint32_t* __restrict__ cursor,
     uint64_t* __restrict__ kout, uint32_t* __restrict__ pout, BatchCtl* ctl) {
   __shared__ uint32_t h[NBINS];        // bin counts; then bin -> group
   __shared__ uint32_t gs[NBINS + 1];   // exclusive bin prefix; then group starts / bases
@@ -243,7 +247,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
     if (vstage && i < t1 && up) vstage[i] = v;
     bad |= i < t1 && request_invalid(o[j], k[j], v, up, rok, key_lo, key_hi);
     nr += i < t1 && o[j] == OP_RANGE;
-    if (i < t1 && o[j] != OP_RANGE) atomicAdd(&h[(uint32_t)(k[j] >> (64 - BIN_BITS))], 1u);
+    if (i < t1 && o[j] != OP_RANGE) atomicAdd(&h[bin_of(k[j], key_lo, bshift, NBINS)], 1u);
   }
   if (__any_sync(FULL, bad) && lane == 0) atomicOr(&ctl->invalid, 1u);
   if (rok) count_ranges(nr, ctl);
@@ -322,7 +326,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   uint32_t* th = h + NBINS - G;   // bins are no longer needed once g is known per item
   uint32_t g[D_ITEMS], r[D_ITEMS];
 #pragma unroll
-  for (int j = 0; j < D_ITEMS; ++j) g[j] = h[(uint32_t)(k[j] >> (64 - BIN_BITS))];
+  for (int j = 0; j < D_ITEMS; ++j) g[j] = h[bin_of(k[j], key_lo, bshift, NBINS)];
   __syncthreads();
   for (uint32_t q = tid; q < G; q += D_THREADS) th[q] = 0;
   __syncthreads();
@@ -352,12 +356,14 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
 
 uint32_t bsort_groups(uint32_t n, int num_sms) {
   // two resident group CTAs per SM when n allows; ~3.5K requests per group
-  // otherwise (bounded by the bins: above 2^22 requests every bin is a group)
-  if (n > (1u << 22)) return NBINS;
+  // otherwise.  Up to 2^22 requests the fused kernel cuts 4096 bins; above,
+  // the two-kernel path cuts 16384 (every group still fits shared memory
+  // unless one key holds more than a group's worth of requests)
   uint32_t g = (n + 3583) / 3584;
   const uint32_t par = std::min<uint32_t>(2u * (uint32_t)num_sms, (n + 255) / 256);
   g = std::max(g, par);
-  return std::max(1u, std::min(g, (uint32_t)NBINS / 2));
+  const uint32_t cap = n > (1u << 22) ? (uint32_t)NBINS_L : (uint32_t)NBINS / 2;
+  return std::max(1u, std::min(g, cap));
 }
 
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
@@ -369,24 +375,35 @@ void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_
       dist_per_sm = 0;
   }
   const uint32_t grid = (uint32_t)num_sms * (uint32_t)dist_per_sm;
-  if (G < NBINS && grid > 0 && (uint64_t)grid * D_THREADS * D_ITEMS >= n) {
+  if (n <= (1u << 22) && grid > 0 && (uint64_t)grid * D_THREADS * D_ITEMS >= n) {
+    uint32_t bshift = bin_shift(key_lo, key_hi, BIN_BITS);
     // fused single launch; slices of whole 512-request rows per CTA
     const uint32_t rows = (n + D_THREADS - 1) / D_THREADS;
     const uint32_t per_cta = ((rows + grid - 1) / grid) * D_THREADS;
     // cooperative launch: the grid barrier needs every CTA co-resident, which a plain
     // launch does not guarantee when other kernels share the device
     void* args[] = {const_cast<BatchArgs**>(&A), &n, const_cast<uint32_t*>(&G), const_cast<uint32_t*>(&per_cta),
-                    &key_lo, &key_hi, const_cast<uint32_t**>(&b.bcount), const_cast<uint32_t**>(&b.gstart),
+                    &key_lo, &key_hi, &bshift, const_cast<uint32_t**>(&b.bcount), const_cast<uint32_t**>(&b.gstart),
                     const_cast<uint32_t**>(&b.cursor), const_cast<uint64_t**>(&b.kA), const_cast<uint32_t**>(&b.pA),
                     &ctl};
     cudaLaunchCooperativeKernel(reinterpret_cast<void*>(bsort_dist_kernel), dim3(grid), dim3(D_THREADS), args, 0, st);
     *launches += 1;
     return;
   }
-  bsort_hist_kernel<<<(n + H_THREADS * H_ITEMS - 1) / (H_THREADS * H_ITEMS), H_THREADS, 0, st>>>(
-      A, n, G, b.bcount, b.bin2grp, b.gstart, b.cursor, ctl);
-  const size_t sm = NBINS * sizeof(uint16_t) + (size_t)G * sizeof(uint32_t);
-  bsort_scatter_kernel<<<(n + S_TILE - 1) / S_TILE, S_THREADS, sm, st>>>(A, n, G, key_lo, key_hi, b.bin2grp,
+  const uint32_t bshift = bin_shift(key_lo, key_hi, BIN_BITS_L);
+  static bool attr = false;
+  const size_t hsm = 2 * NBINS_L * sizeof(uint32_t);
+  const size_t ssm = NBINS_L * sizeof(uint16_t) + (size_t)NBINS_L * sizeof(uint32_t);
+  if (!attr) {
+    cudaFuncSetAttribute(bsort_hist_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsm);
+    cudaFuncSetAttribute(bsort_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ssm);
+    attr = true;
+  }
+  const uint32_t tiles = (n + H_THREADS * H_ITEMS - 1) / (H_THREADS * H_ITEMS);
+  bsort_hist_kernel<<<std::max(1u, std::min(tiles, (uint32_t)num_sms)), H_THREADS, hsm, st>>>(
+      A, n, G, key_lo, bshift, b.bcount, b.bin2grp, b.gstart, b.cursor, ctl);
+  const size_t sm = NBINS_L * sizeof(uint16_t) + (size_t)G * sizeof(uint32_t);
+  bsort_scatter_kernel<<<(n + S_TILE - 1) / S_TILE, S_THREADS, sm, st>>>(A, n, G, key_lo, key_hi, bshift, b.bin2grp,
                                                                          b.cursor, b.kA, b.pA, ctl);
   *launches += 2;
 }

@@ -245,17 +245,33 @@ void launch_sort(const uint64_t* keys, const uint8_t* ops, const uint32_t* pay_i
 size_t sort_lookback_words(uint32_t max_n);
 
 // Batch request sort (bsort.cu): bucket by the top bits, sort buckets in smem.
-constexpr int BIN_BITS = 12;                  // bucket-sort bins = top key bits
+constexpr int BIN_BITS = 12;                  // bucket-sort bins = top bits of (key - key_lo) (fused path)
 constexpr int NBINS = 1 << BIN_BITS;
+constexpr int BIN_BITS_L = 14;                // bins of the two-kernel path (batches > 2^22 requests)
+constexpr int NBINS_L = 1 << BIN_BITS_L;
+constexpr int NBINS_MAX = NBINS_L;
+// Bin of key k: the top `bits` bits of k - key_lo over the shard's range, so a
+// shard of a multi-GPU tree (a fraction of the key space) still spreads its
+// keys over all the bins.  Out-of-range keys (invalid requests, rejected
+// later) are clamped.  shift = max(0, bits(key_hi - key_lo - 1) - bits).
+__host__ __device__ __forceinline__ uint32_t bin_of(uint64_t k, uint64_t key_lo, uint32_t shift, uint32_t nbins) {
+  const uint64_t d = k >= key_lo ? (k - key_lo) >> shift : 0ull;
+  return d < nbins ? (uint32_t)d : nbins - 1u;
+}
+inline uint32_t bin_shift(uint64_t key_lo, uint64_t key_hi, int bits) {
+  const uint64_t r = key_hi - key_lo - 1;   // key_hi > key_lo
+  const int rb = r ? 64 - __builtin_clzll(r) : 0;
+  return (uint32_t)(rb > bits ? rb - bits : 0);
+}
 struct BSortBufs {
   uint64_t* kA;      // [n] grouped (unordered inside a group)
   uint32_t* pA;
   uint64_t* kB;      // [n] scratch for oversized groups
   uint32_t* pB;      // [n] sorted payloads (output)
-  uint32_t* bcount;  // [NBINS] zeroed per batch
-  uint16_t* bin2grp; // [NBINS]
-  uint32_t* gstart;  // [NBINS + 1] group starts
-  uint32_t* cursor;  // [NBINS] group fill cursors (zeroed per batch)
+  uint32_t* bcount;  // [NBINS_MAX] zeroed per batch
+  uint16_t* bin2grp; // [NBINS_MAX]
+  uint32_t* gstart;  // [NBINS_MAX + 1] group starts
+  uint32_t* cursor;  // [NBINS_MAX] group fill cursors (zeroed per batch)
 };
 uint32_t bsort_groups(uint32_t n, int num_sms);
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
@@ -281,7 +297,7 @@ struct CombBufs {
 };
 constexpr int HOT_SLOTS = 64;
 constexpr uint32_t SHORT_SEG = 32;
-constexpr int GROUP_STATUS_WORDS = NBINS;   // >= bsort_groups(n) for every n
+constexpr int GROUP_STATUS_WORDS = NBINS_MAX;   // >= bsort_groups(n) for every n
 
 // bucket finish (sort in smem) + combine + partition, one CTA per bucket (group.cu)
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,

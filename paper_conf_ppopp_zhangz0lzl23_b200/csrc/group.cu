@@ -431,7 +431,7 @@ __device__ void l2_pass_pay(const uint32_t* ps, uint32_t* pd, uint32_t cnt, int 
 // of key - kmin, ping-pong between the group's two L2 ranges.  Returns the
 // range that holds the result (0: ks/ps, 1: kd/pd).
 __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int tsbits, GSmem& S,
-                       uint32_t* bits, uint32_t hot_words) {
+                       uint32_t* hot_base, uint32_t* hot_ctr, uint32_t nreq, uint32_t hot_words) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint64_t c0 = ks[0], c1 = ks[cnt / 3], c2 = ks[(2 * (uint64_t)cnt) / 3];
   uint64_t mn = KEY_MAX, mx = 0;
@@ -476,7 +476,20 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
   const uint64_t hk = (n0 >= n1 && n0 >= n2) ? c0 : (n1 >= n2 ? c1 : c2);
   const uint32_t hcnt = max(n0, max(n1, n2));
   if (cnt - hcnt <= (uint32_t)G_CAP) {
-    // split: the rest into S.k / S.p, hk's payloads into kd (as u32 scratch)
+    // split: the rest into S.k / S.p, hk's payloads into kd (as u32 scratch).
+    // A timestamp bitmap costs O(n / 32) words whatever hk's count; LSD passes
+    // over hk's payloads cost O(hcnt): the bitmap (a slot of HOT_SLOTS) only
+    // for keys holding more than n / 128 requests -- at most 128 of them
+    if (tid == 0) {
+      uint32_t* b = nullptr;
+      if (hot_base && hcnt > max((uint32_t)G_CAP, nreq >> 7)) {
+        const uint32_t slot = atomicAdd(hot_ctr, 1u);
+        if (slot < (uint32_t)HOT_SLOTS) b = hot_base + (size_t)slot * 3 * hot_words;
+      }
+      S.hot_bits = b;
+    }
+    __syncthreads();
+    uint32_t* bits = S.hot_bits;
     uint32_t* hs = reinterpret_cast<uint32_t*>(kd);
     if (tid == 0) {
       S.r_nh = 0;   // rest
@@ -962,12 +975,8 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   int mode = 0;   // 0: small / L2-sorted group, 2: SPLIT (rest in smem, hot key in a bitmap)
   uint32_t sp_o = 0, sp_h = 0, sp_lo = 0;
   if (!small) {
-    if (tid == 0) {
-      const uint32_t slot = atomicAdd(&ctl->hot_ctr, 1u);
-      S.hot_bits = slot < (uint32_t)HOT_SLOTS ? g.hot_bits + (size_t)slot * 3 * g.hot_words : nullptr;
-    }
-    __syncthreads();
-    const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S, S.hot_bits, g.hot_words);
+    const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S, g.hot_bits,
+                              &ctl->hot_ctr, g.n, g.hot_words);
     if (where == 2) {
       mode = 2;
       sp_o = S.r_nh;

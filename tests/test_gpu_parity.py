@@ -396,3 +396,38 @@ def test_prepare_batch_then_submit(dev):
                       rng.integers(1, 1 << 40, 4096, dtype=np.uint64))
         vs = rng.integers(0, 1 << 62, 4096, dtype=np.uint64)
         run_and_compare(t, ref, ops, ks, vs, dev)
+
+
+@pytest.mark.parametrize("zipf", [False, True])
+def test_large_batch_two_kernel_sort(dev, zipf):
+    """A batch above 2^22 requests (ragged size) takes the two-kernel bucket sort
+    with 16384 bins (bsort.cu); with Zipf keys several groups are oversized."""
+    from paper_conf_ppopp_zhangz0lzl23_b200 import workload as W
+    n = (1 << 22) + 4097
+    w = W.Workload(3 if zipf else 2, tree=1 << 20, batch=n)
+    t = make_tree(dev, w.keys, w.vals, max_keys=1 << 22, max_batch=n)
+    ref = oracle.MapOracle(); ref.load(w.keys, w.vals)
+    for b in range(2):
+        ops, keys, vals = w.batch_arrays(b)
+        run_and_compare(t, ref, ops, keys, vals, dev, check_scan=(b == 1))
+    t.close()
+
+
+def test_narrow_shard_key_range(dev):
+    """A shard owning a 2^40-wide slice of the key space: bins are taken over
+    [key_lo, key_hi), not over the top bits of the key (bin_of)."""
+    lo = 1 << 60
+    rng = np.random.default_rng(77)
+    keys = np.unique(rng.integers(lo, lo + (1 << 40), 50000, dtype=np.uint64))
+    vals = rng.integers(0, 1 << 62, keys.size, dtype=np.uint64)
+    t = make_tree(dev, keys, vals, max_batch=1 << 17, key_lo=lo, key_hi=lo + (1 << 40))
+    ref = oracle.MapOracle(); ref.load(keys, vals)
+    n = 1 << 17
+    for b in range(2):
+        ops = rng.integers(0, 4, n).astype(np.uint8)
+        ks = np.where(rng.random(n) < 0.7, rng.choice(keys, n),
+                      rng.integers(lo, lo + (1 << 40), n, dtype=np.uint64)).astype(np.uint64)
+        vs = rng.integers(0, 1 << 62, n, dtype=np.uint64)
+        run_and_compare(t, ref, ops, ks, vs, dev)
+    assert t.check_invariants()[0] == 0
+    t.close()
