@@ -139,6 +139,54 @@ def algorithmic_bytes_range(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarra
             "bytes": int(nr * (1 + 8 + 8 + 8) + int(cnt.sum()) * 16 + lines * 128 + sectors * 32)}
 
 
+def random_access_counts(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, per_leaf: int) -> dict:
+    """Random HBM touches of one batch on the bulk-loaded shape:
+    every issued request (one per distinct key, query or write) reads its leaf's
+    128 B key line (distinct leaves counted once) and, if its key is present,
+    one 32 B value sector (distinct sectors once); every issued write writes
+    one 32 B value sector.  Streamed bytes per request: op 1 + key 8 +
+    result 8, + 8 per upsert value."""
+    uk = np.unique(keys)
+    wk = np.unique(keys[ops != W.QUERY])
+    pos = np.searchsorted(loaded, uk)
+    hit = (pos < loaded.size) & (loaded[np.minimum(pos, loaded.size - 1)] == uk)
+    leaf = pos // per_leaf
+    n = keys.size
+    ups = int(np.sum((ops == W.UPDATE) | (ops == W.INSERT)))
+    return {"lines": np.unique(leaf).size / n, "sectors": np.unique(leaf[hit] * 4 + (pos[hit] % per_leaf) // 4).size / n,
+            "writes": wk.size / n, "bio": (n * 17 + ups * 8) / n}
+
+
+def probe_random_access(dev, stream, pool_gib: int = 4, n: int = 1 << 24, reps: int = 3) -> dict:
+    """Random accesses per second of this GPU's HBM (eirene_probe_gather: 128 B
+    line reads, 32 B sector reads, 32 B sector writes over a pool >> L2),
+    best of `reps`, CUDA events on the launching stream."""
+    import ctypes
+
+    import torch
+
+    from paper_conf_ppopp_zhangz0lzl23_b200 import _ffi
+    L = _ffi.lib()
+    pool = torch.empty(pool_gib << 30, dtype=torch.uint8, device=dev)
+    out = {}
+    for kind, name in ((0, "R128"), (1, "R32"), (2, "R32w")):
+        best = 0.0
+        for r in range(reps + 1):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            rc = L.eirene_probe_gather(ctypes.c_void_p(pool.data_ptr()), pool.numel(), n, kind, 77 + r,
+                                       ctypes.c_void_p(stream.cuda_stream))
+            e1.record(stream)
+            stream.synchronize()
+            if rc != 0:
+                raise RuntimeError(f"eirene_probe_gather rc={rc}")
+            if r:   # first launch is a warm-up
+                best = max(best, n / (e0.elapsed_time(e1) * 1e-3))
+        out[name] = best
+    del pool
+    return out
+
+
 def run_reference(args):
     """--impl reference: the CPU oracle (sequential B+tree, 1 thread) as it stands,
     each step a bounded sample of the same workload."""
@@ -176,7 +224,7 @@ def run_reference(args):
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
         "config": {"workload": f"cfg{cfg}: {W.CONFIGS[cfg]['tree']} keys, batch sample {sample} of "
                                f"{W.CONFIGS[cfg]['batch']} requests", "cfg": cfg},
-        "cpu_baseline": {"value": v, "unit": "Greq/s", "cores": 1, "kind": "oracle",
+        "cpu_baseline": {"value": v, "unit": "Greq/s", "cores": 1, "host_cores": os.cpu_count(), "kind": "oracle",
                          "sample": f"{args.steps} batches x first {sample} requests; oracle B+tree bulk load "
                                    f"{load_s:.1f}s untimed"},
         "e2e": {"value": v, "unit": "Greq/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
@@ -476,6 +524,7 @@ def run_ours(args):
     parity = None
     cpu = None
     roof = None
+    rar = None
     if rank == 0 and world == 1 and args.cpu_batches > 0:
         import oracle
         n_check = min(args.cpu_batches, nb)
@@ -505,7 +554,7 @@ def run_ours(args):
                 col = np.arange(cap)[None, :] < want.astype(np.int64)[:, None]
                 bad += int(np.sum((gk != wk) & col)) + int(np.sum((gv != wv) & col))
         parity = {"batches_checked": n_check, "mismatches": bad, "vs": "oracle B+tree, every request, bit-exact"}
-        cpu = {"value": n_check * batch_n / cpu_t / 1e9, "unit": "Greq/s", "cores": 1, "kind": "oracle",
+        cpu = {"value": n_check * batch_n / cpu_t / 1e9, "unit": "Greq/s", "cores": 1, "host_cores": os.cpu_count(), "kind": "oracle",
                "sample": f"first {n_check} batches of the same workload ({n_check * batch_n} requests), "
                          f"sequential B+tree, 1 thread; bulk load {load_s:.1f}s untimed"}
         # roofline of the dominant kernel
@@ -557,6 +606,22 @@ def run_ours(args):
         roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s",
                 "frac": ach / peaks["hbm_gbs"], "traffic": traffic, "traffic_source": traffic_src, "kernel": kern,
                 "stage_ms": ms, "algorithmic_bytes_per_launch": bytes_per, "peak_source": peaks["source"]}
+        # whole-path random-access roofline (BASELINE north_star) on
+        # the bulk-loaded shape: 1 / (L/R128 + S/R32 + Wr/R32w + B_io/BW) req/s
+        if not cap and not per_tree and args.ra_probe:
+            rates = probe_random_access(dev, stream)
+            cs = [random_access_counts(wls[0].keys, *host_batches[b][:2], 16)
+                  for b in range(args.warmup, min(nb, args.warmup + 4))]
+            c = {k: float(np.mean([x[k] for x in cs])) for k in cs[0]}
+            t_req = (c["lines"] / rates["R128"] + c["sectors"] / rates["R32"] + c["writes"] / rates["R32w"]
+                     + c["bio"] / (peaks["hbm_gbs"] * 1e9))
+            rar = {"roofline_Greq_s": 1.0 / t_req / 1e9, "achieved_Greq_s": value,
+                   "frac": value / (1.0 / t_req / 1e9),
+                   "per_request": {"leaf_lines": c["lines"], "value_sectors": c["sectors"],
+                                   "value_writes": c["writes"], "streamed_bytes": c["bio"]},
+                   "rates_per_s": rates,
+                   "probe": "eirene_probe_gather: 2^24 uniformly random 128 B line reads / 32 B sector reads / "
+                            "32 B sector writes over a 4 GiB pool, best of 3, CUDA events"}
 
     if rank == 0:
         line = {
@@ -584,6 +649,7 @@ def run_ours(args):
             "clocks": clocks.summary(),
             "e2e": e2e,
             "roofline": roof,
+            "random_access_roofline": rar,
             "cpu_baseline": cpu,
             "parity": parity,
             "setup_s": gen_s,
@@ -617,6 +683,7 @@ def main():
     ap.add_argument("--query-mode", default="default", choices=["default", "iterwarp"],
                     help="iterwarp: the paper's iteration warps + range field (ablation)")
     ap.add_argument("--iter-rgs", type=int, default=0, help="RGs per iteration warp (0 = auto)")
+    ap.add_argument("--ra-probe", type=int, default=1, help="measure the random-access roofline (1) or not (0)")
     args = ap.parse_args()
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")

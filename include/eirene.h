@@ -234,6 +234,18 @@ int eirene_get_info(eirene_handle h, eirene_tree_info* info);
  * launched directly so that stage events can be recorded between them. */
 int eirene_set_flags(eirene_handle h, uint32_t flags);
 
+/* Measurement helper (not part of the request path): launches one random-access
+ * probe on `stream` over the caller's device buffer pool_dev[pool_bytes]
+ * (128 B aligned, ideally far larger than L2): n uniformly random accesses,
+ * kind 0 = 128 B line reads (the leaf key line of a lookup), 1 = 32 B sector
+ * reads (a value sector), 2 = 32 B sector writes (an in-place value update).
+ * The caller times it with events on `stream`; accesses/s are the
+ * denominators of the random-access roofline of SURVEY §8(d) (BASELINE
+ * north_star).  Kind 2 overwrites pool contents.  EINVAL for a null / short /
+ * misaligned pool or an unknown kind; ECUDA if the launch fails. */
+int eirene_probe_gather(void* pool_dev, uint64_t pool_bytes, uint32_t n, int kind, uint64_t seed,
+                        eirene_stream_t stream);
+
 /* Frees every device and host resource of the handle (waits for pending work). */
 int eirene_destroy(eirene_handle h);
 

@@ -65,6 +65,7 @@ _SIGS = {
     "eirene_check_invariants": (_int, [_vp, ctypes.POINTER(_u64)]),
     "eirene_get_info": (_int, [_vp, ctypes.POINTER(eirene_tree_info)]),
     "eirene_set_flags": (_int, [_vp, _u32]),
+    "eirene_probe_gather": (_int, [_vp, _u64, _u32, ctypes.c_int, _u64, _vp]),
     "eirene_destroy": (_int, [_vp]),
     "eirene_strerror": (ctypes.c_char_p, [_int]),
     "eirene_last_cuda_error": (ctypes.c_char_p, []),

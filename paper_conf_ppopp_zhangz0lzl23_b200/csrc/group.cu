@@ -68,6 +68,7 @@ struct GSmem {
   uint32_t seg0, w0, ticket;
   uint32_t h_cnt[G_WARPS], h_lw[G_WARPS], h_lp[G_WARPS];   // hot_pass1 per-warp results
   uint64_t hk;                 // split-off hot key of an oversized group
+  unsigned long long prof_t[2];  // EIRENE_GROUP_PROF timestamps (diagnostic)
   uint32_t* hot_bits;          // its timestamp bitmap slot (null: none free)
 };
 
@@ -430,6 +431,114 @@ __device__ void l2_pass_pay(const uint32_t* ps, uint32_t* pd, uint32_t cnt, int 
 // in (kd, pd).  Otherwise: stable LSD on the timestamp bits, then on the bits
 // of key - kmin, ping-pong between the group's two L2 ranges.  Returns the
 // range that holds the result (0: ks/ps, 1: kd/pd).
+// An oversized group with no dominant key (cnt > G_CAP, its largest key run
+// leaves more than G_CAP others): cut its key range [kmin, kmax] into parts of
+// <= G_CAP requests with a histogram of (k - kmin) >> shift over SB_N bins --
+// part(bin) = floor(prefix(bin) / T), T = G_CAP - largest bin, so a part never
+// exceeds T + largest bin -- scatter the requests into their parts (key
+// ranges, ascending) in kd / pd, then sort every part in shared memory and
+// write it back in place: three passes over the group instead of up to 11
+// LSD passes.  Returns false (nothing written) if it would take more than
+// PART_MAX parts (a bin of nearly G_CAP requests).
+constexpr uint32_t PART_MAX = 64;
+__device__ bool range_partition_sort(const uint64_t* ks, const uint32_t* ps, uint64_t* kd, uint32_t* pd,
+                                     uint32_t cnt, uint64_t kmin, uint64_t range, GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int bits = 64 - __clzll((long long)range);
+  const int shift = bits > SB_BITS ? bits - SB_BITS : 0;
+  for (int i = tid; i <= SB_N; i += G_THREADS) S.sb[i] = 0;
+  __syncthreads();
+  for (uint32_t i0 = tid; i0 < cnt; i0 += 8 * G_THREADS) {   // 8 loads in flight per thread
+    uint64_t kk[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const uint32_t i = i0 + u * G_THREADS;
+      kk[u] = i < cnt ? ks[i] : kmin;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u)
+      if (i0 + u * G_THREADS < cnt) atomicAdd(&S.sb[(uint32_t)((kk[u] - kmin) >> shift)], 1u);
+  }
+  __syncthreads();
+  // exclusive prefix of the bins (8 per thread) and the largest bin
+  constexpr int PER = SB_N / G_THREADS;
+  uint32_t loc[PER], sum = 0, mx = 0;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    loc[j] = S.sb[tid * PER + j];
+    sum += loc[j];
+    mx = max(mx, loc[j]);
+  }
+  uint32_t x = sum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) mx = max(mx, __shfl_xor_sync(FULL, mx, o));
+  if (lane == 31) S.wsum[warp] = x;
+  if (lane == 0) S.wcmax[warp] = mx;
+  __syncthreads();
+  uint32_t run = x - sum, big = 0;
+  for (int w = 0; w < G_WARPS; ++w) {
+    if (w < warp) run += S.wsum[w];
+    big = max(big, S.wcmax[w]);
+  }
+  const uint32_t T = big < (uint32_t)G_CAP ? (uint32_t)G_CAP - big : 0u;
+  const uint32_t parts = T ? (cnt + T - 1) / T : 0xFFFFFFFFu;
+  if (parts > PART_MAX) return false;   // (uniform: every thread computed the same)
+  // part starts: the prefix of the first bin of each part
+  if (tid <= (int)PART_MAX) S.dhist[tid] = cnt;   // empty parts start at the end
+  __syncthreads();
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    const uint32_t q = min(run / T, parts - 1);
+    if (loc[j]) atomicMin(&S.dhist[q], run);   // part start = prefix of its first nonempty bin
+    S.sb[tid * PER + j] = q;                              // bin -> part
+    run += loc[j];
+  }
+  __syncthreads();
+  if (tid == 0) {   // empty parts start where the next nonempty one does
+    for (int q = (int)parts - 1; q >= 0; --q) S.dhist[q] = min(S.dhist[q], S.dhist[q + 1]);
+    for (uint32_t q = 0; q < parts; ++q) S.whist[q] = S.dhist[q];   // fill cursors
+  }
+  __syncthreads();
+  for (uint32_t i0 = tid; i0 < cnt; i0 += 4 * G_THREADS) {   // scatter into the parts (order inside a part: any)
+    uint64_t kk[4];
+    uint32_t pp[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t i = i0 + u * G_THREADS;
+      kk[u] = i < cnt ? ks[i] : 0;
+      pp[u] = i < cnt ? ps[i] : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      if (i0 + u * G_THREADS < cnt) {
+        const uint32_t q = S.sb[(uint32_t)((kk[u] - kmin) >> shift)];
+        const uint32_t pos = atomicAdd(&S.whist[q], 1u);
+        kd[pos] = kk[u];
+        pd[pos] = pp[u];
+      }
+    }
+  }
+  __threadfence_block();
+  __syncthreads();
+  for (uint32_t q = 0; q < parts; ++q) {
+    const uint32_t b0 = S.dhist[q], m = S.dhist[q + 1] - b0;
+    __syncthreads();   // (every thread read the part bounds before smem_sort reuses S)
+    if (m < 2) continue;
+    smem_sort(kd + b0, pd + b0, m, S);
+    for (uint32_t i = tid; i < m; i += G_THREADS) {
+      kd[b0 + i] = S.k[i];
+      pd[b0 + i] = S.p[i];
+    }
+    __syncthreads();
+  }
+  return true;
+}
+
 __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, uint32_t cnt, int tsbits, GSmem& S,
                        uint32_t* hot_base, uint32_t* hot_ctr, uint32_t nreq, uint32_t hot_words) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -569,6 +678,7 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
     __syncthreads();
     return 1;
   }
+  if (range && range_partition_sort(ks, ps, kd, pd, cnt, kmin, range, S)) return 1;
   const int tpass = (tsbits + 7) / 8;
   const int passes = tpass + (range ? (64 - __clzll((long long)range) + 7) / 8 : 0);
   for (int pass = 0; pass < passes; ++pass) {
@@ -1065,6 +1175,9 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
         const uint32_t inc = __ballot_sync(FULL, fl == 2);
         const uint32_t need = inc ? ((2u << (__ffs(inc) - 1)) - 1u) : FULL;
         if (__ballot_sync(FULL, fl == 0) & need) {
+          // a predecessor has not published: back off (a waiting group's spin
+          // would otherwise keep the L2 busy under the slow groups it waits for)
+          __nanosleep(256);
           if (sg.stuck(ctl)) break;
           continue;
         }
@@ -1102,7 +1215,9 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     }
     __syncthreads();
     const uint32_t sH = S.seg0 + a_nh, wH = S.w0 + a_nw, pos0 = base + sp_lo;
+    if ((g.prof & 1) && tid == 0) S.prof_t[0] = gtime_ns();
     hot_pass2(g, S.hot_bits, hc, sH, pos0);
+    if ((g.prof & 1) && tid == 0) S.prof_t[1] = gtime_ns();
     if (tid == 0) {
       const uint64_t hk = S.hk;
       g.istart[sH] = pos0;
@@ -1136,8 +1251,9 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   if ((g.prof & 1) && tid == 0) {
     const unsigned long long tp4 = gtime_ns();
     if (tp4 - tp0 > 20000)
-      printf("[group prof] ticket %u cnt %u mode %d sort %.1f sweep1 %.1f lookback %.1f emit %.1f us\n", b, cnt, mode,
-             (tp1 - tp0) * 1e-3, (tp2 - tp1) * 1e-3, (tp3 - tp2) * 1e-3, (tp4 - tp3) * 1e-3);
+      printf("[group prof] ticket %u cnt %u mode %d sort %.1f sweep1 %.1f lookback %.1f emit %.1f us hot2 %.1f\n", b,
+             cnt, mode, (tp1 - tp0) * 1e-3, (tp2 - tp1) * 1e-3, (tp3 - tp2) * 1e-3, (tp4 - tp3) * 1e-3,
+             mode == 2 ? (S.prof_t[1] - S.prof_t[0]) * 1e-3 : 0.0);
   }
 }
 

@@ -13,7 +13,10 @@ want = ["gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum
         "dram__throughput.avg.pct_of_peak_sustained_elapsed", "lts__throughput.avg.pct_of_peak_sustained_elapsed",
         "sm__throughput.avg.pct_of_peak_sustained_elapsed", "sm__warps_active.avg.pct_of_peak_sustained_active",
         "launch__registers_per_thread", "launch__grid_size", "lts__t_sector_hit_rate.pct",
-        "smsp__thread_inst_executed_per_inst_executed.ratio"]
+        "smsp__thread_inst_executed_per_inst_executed.ratio", "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
+        "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum",
+        "l1tex__t_requests_pipe_lsu_mem_global_op_atom.sum", "smsp__inst_executed_op_branch.sum",
+        "smsp__branch_targets_threads_divergent.sum", "lts__t_sectors_srcunit_tex_op_read.sum"]
 idx = {w: h.index(w) for w in want if w in h}
 stall = [i for i, c in enumerate(h) if c.startswith("smsp__average_warps_issue_stalled_") and c.endswith("_per_issue_active.ratio")]
 ki = h.index("Kernel Name")
@@ -28,4 +31,16 @@ for r in rows[2:]:
           f"sm%={d.get('sm__throughput.avg.pct_of_peak_sustained_elapsed')} warps%={d.get('sm__warps_active.avg.pct_of_peak_sustained_active')} "
           f"regs={d.get('launch__registers_per_thread')} grid={d.get('launch__grid_size')} l2hit={d.get('lts__t_sector_hit_rate.pct')} "
           f"simt={d.get('smsp__thread_inst_executed_per_inst_executed.ratio')}")
+    def num(k):
+        try:
+            return float(d.get(k, "").replace(",", ""))
+        except ValueError:
+            return None
+    sec, req = num("l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum"), num("l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum")
+    print(f"    dram%(gpu)={d.get('gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed')} "
+          f"ld sectors/request={sec / req if sec and req else None} "
+          f"atom requests={d.get('l1tex__t_requests_pipe_lsu_mem_global_op_atom.sum')} "
+          f"branches={d.get('smsp__inst_executed_op_branch.sum')} "
+          f"divergent branch targets={d.get('smsp__branch_targets_threads_divergent.sum')} "
+          f"L2 read sectors from L1={d.get('lts__t_sectors_srcunit_tex_op_read.sum')}")
     print("    stalls:", ", ".join(f"{n}={v:.1f}" for v, n in st))
