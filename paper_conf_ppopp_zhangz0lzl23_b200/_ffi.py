@@ -13,7 +13,8 @@ import re
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
-LIB_PATH = os.path.join(PKG, "libeirene.so")
+# EIRENE_LIB: an alternative build of the same library (A/B experiments); default: the in-tree one
+LIB_PATH = os.environ.get("EIRENE_LIB") or os.path.join(PKG, "libeirene.so")
 HEADER = os.path.join(ROOT, "include", "eirene.h")
 
 EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECUDA = 0, -1, -2, -3, -4, -5

@@ -165,6 +165,11 @@ __device__ __forceinline__ uint32_t atom_cas_acquire(uint32_t* p, uint32_t cmp, 
   asm volatile("atom.acquire.gpu.global.cas.b32 %0, [%1], %2, %3;" : "=r"(old) : "l"(p), "r"(cmp), "r"(val) : "memory");
   return old;
 }
+__device__ __forceinline__ uint32_t atom_or_acquire(uint32_t* p, uint32_t val) {
+  uint32_t old;
+  asm volatile("atom.acquire.gpu.global.or.b32 %0, [%1], %2;" : "=r"(old) : "l"(p), "r"(val) : "memory");
+  return old;
+}
 __device__ __forceinline__ void st_release(uint32_t* p, uint32_t v) {
   asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }

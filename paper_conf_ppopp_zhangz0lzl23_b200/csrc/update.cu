@@ -100,9 +100,9 @@ __device__ __forceinline__ NodeMeta* meta_of(const Tree& t, uint32_t node, bool 
 // lanes' subsequent (L2-coherent) reads after it.
 __device__ __forceinline__ bool try_lock(uint32_t* vp, uint32_t* v_out) {
   uint32_t v = 0, ok = 0;
-  if (lane_id() == 0) {
-    v = ld_relaxed(vp);
-    ok = (!(v & 1u) && atom_cas_acquire(vp, v, v | 1u) == v) ? 1u : 0u;
+  if (lane_id() == 0) {   // test-and-set: one round trip (setting an already set lock bit changes nothing)
+    v = atom_or_acquire(vp, 1u);
+    ok = (v & 1u) ? 0u : 1u;
   }
   ok = shfl32(ok, 0);
   v = shfl32(v, 0);
@@ -263,12 +263,11 @@ __device__ void build_root(const Ctx& C, uint32_t L, uint32_t id0, uint64_t lo0,
 // k = ceil(t/16) leaves (X + k-1 fresh), entries (first key, leaf) for the
 // parent written to (Ek, Ec)[b .. b+k-2].  Returns k.
 __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e, uint64_t X_hi, uint32_t X_next,
-                               uint64_t* Ek, uint32_t* Ec, WarpStats& ws) {
+                               uint64_t okey, uint64_t oval, uint64_t* Ek, uint32_t* Ec, WarpStats& ws) {
+  // okey / oval: X's key and value of slot `lane` (lanes < 16), loaded by the caller under the lock
   const int lane = lane_id();
   const Tree& t = C.t;
   const size_t xb = (size_t)X * LSTRIDE;
-  const uint64_t okey = lane < FAN ? ld_cg(t.lkeys + xb + lane) : KEY_MAX;
-  const uint64_t oval = lane < FAN ? ld_cg(t.lvals + xb + lane) : 0;
   const uint32_t c = __popc(__ballot_sync(FULL, okey != KEY_MAX));
 
   uint32_t mmask = 0, U = 0, ups_before = 0;
@@ -355,7 +354,9 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
       if (s >= sz) t.lkeys[(size_t)(q == 0 ? X : first + q - 1) * LSTRIDE + s] = KEY_MAX;
     }
   }
-  __threadfence();
+  // (no fence here: the new leaves are unreachable until X links them below,
+  // X itself is read only under its lock; __syncwarp orders the lanes' Ek
+  // writes before the meta loop reads them)
   __syncwarp();
   if (k > 1) {
     for (uint32_t q = 1 + lane; q < k; q += 32) {
@@ -382,8 +383,7 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
   } else if (lane == 0) {
     t.lmeta[X].count = tout;
   }
-  __threadfence();
-  __syncwarp();
+  __syncwarp();   // published by the caller's unlock (a release)
   return k;
 }
 
@@ -607,8 +607,7 @@ __device__ void acc_entries_buf(uint64_t* EK, uint32_t* EC, SepAcc& A, uint32_t 
       }
       __syncwarp();
     }
-    __threadfence();
-    __syncwarp();
+    // (no fence: the entries are read by this warp, or by others after a grid barrier)
   }
   A.n += cnt;
 }
@@ -635,8 +634,13 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
     if (X != NIL && X < t.leaf_cap) {
       uint32_t* vp = &t.lmeta[X].version;
       uint32_t v;
-      if (try_lock(vp, &v)) {   // leafvers == leaf.version: the CAS expects v (Alg.1:35-38)
+      if (try_lock(vp, &v)) {   // leafvers = the version the lock saw (Alg.1:35-38)
+        // every read of X the run needs, issued together (one round trip)
         const uint64_t lo = ld_cg(&t.lmeta[X].lo), hi = ld_cg(&t.lmeta[X].hi);
+        const uint32_t nxt = ld_cg(&t.lmeta[X].next);
+        const size_t xb = (size_t)X * LSTRIDE;
+        const uint64_t okey = lane < FAN ? ld_cg(t.lkeys + xb + lane) : KEY_MAX;
+        const uint64_t oval = lane < FAN ? ld_cg(t.lvals + xb + lane) : 0;
         if (k0 >= lo && k0 < hi) {
           uint32_t e2 = e;
           for (uint32_t base = b; base < e; base += 32) {
@@ -647,8 +651,7 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
               break;
             }
           }
-          const uint32_t nxt = ld_cg(&t.lmeta[X].next);
-          const uint32_t k = leaf_apply(C, X, b, e2, hi, nxt, C.eK[0], C.eC[0], ws);
+          const uint32_t k = leaf_apply(C, X, b, e2, hi, nxt, okey, oval, C.eK[0], C.eC[0], ws);
           ws.runs += 1;
           if (k > 1) {
             bool rooted = false;
@@ -948,7 +951,10 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
   }
 }
 
-__global__ void __launch_bounds__(128, 8) update_kernel(Ctx C) {
+#ifndef UPD_MINB
+#define UPD_MINB 8   // resident CTAs per SM the register budget is fitted to (A/B builds: -DUPD_MINB=n)
+#endif
+__global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
   const BatchCtl* ctl = C.ctl;
   if (ctl->invalid || ctl->status != 0) return;   // (uniform: every CTA leaves, no barrier is reached)
   if (g_uprof && blockIdx.x == 0 && threadIdx.x == 0) C.ctl->uprof[0] = gtime_ns();
