@@ -431,3 +431,34 @@ def test_narrow_shard_key_range(dev):
         run_and_compare(t, ref, ops, ks, vs, dev)
     assert t.check_invariants()[0] == 0
     t.close()
+
+
+def test_edge_batches(dev):
+    """Degenerate batches: a single request, extreme valid keys (0 and UINT64_MAX - 1)
+    and values (UINT64_MAX - 1), queries / deletes on an empty tree, a batch of exactly
+    max_batch requests, all-delete batches that empty the tree and a refill."""
+    rng = np.random.default_rng(11)
+    t = make_tree(dev, np.empty(0, np.uint64), np.empty(0, np.uint64), max_keys=1 << 14, max_batch=4096)
+    ref = oracle.MapOracle()
+    top = np.uint64(0xFFFFFFFFFFFFFFFE)
+    # empty tree: queries and deletes of absent keys
+    run_and_compare(t, ref, np.array([0, 3, 0], np.uint8), np.array([0, 5, top], np.uint64),
+                    np.zeros(3, np.uint64), dev)
+    # one request at a time, extreme keys and values
+    for op, k, v in [(2, 0, top), (2, top, 1), (0, 0, 0), (1, top, top), (0, top, 0), (3, 0, 0), (0, 0, 0)]:
+        run_and_compare(t, ref, np.array([op], np.uint8), np.array([k], np.uint64), np.array([v], np.uint64), dev)
+    # exactly max_batch requests over a small key set (long segments, splits from a 1-key tree)
+    n = 4096
+    ops = rng.integers(0, 4, n).astype(np.uint8)
+    ks = rng.integers(0, 600, n, dtype=np.uint64) * np.uint64(0x9E3779B97F4A7C15 >> 4)
+    vs = rng.integers(0, 1 << 63, n, dtype=np.uint64)
+    run_and_compare(t, ref, ops, ks, vs, dev)
+    # delete everything, then query it all, then refill
+    live, _ = ref.scan()
+    d = np.resize(live, n) if live.size else np.zeros(n, np.uint64)
+    run_and_compare(t, ref, np.full(n, 3, np.uint8), d, np.zeros(n, np.uint64), dev)
+    run_and_compare(t, ref, np.zeros(n, np.uint8), d, np.zeros(n, np.uint64), dev)
+    assert ref.size() == 0
+    run_and_compare(t, ref, np.full(n, 2, np.uint8), d, vs, dev)
+    assert t.check_invariants()[0] == 0
+    t.close()
