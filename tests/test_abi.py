@@ -83,3 +83,12 @@ def test_range_and_prepare_argument_checks_without_gpu(libpath):
                                        ctypes.byref(tk)) == _ffi.EIRENE_EINVAL
     assert L.eirene_prepare_batch(None, 16, 0) == _ffi.EIRENE_EINVAL
     assert _ffi.EIRENE_RANGE == 4
+
+
+def test_probe_gather_argument_checks(libpath):
+    """eirene_probe_gather validates its arguments before any device call."""
+    L = _ffi.lib()
+    assert L.eirene_probe_gather(None, 1 << 20, 16, 0, 1, None) == _ffi.EIRENE_EINVAL
+    assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 1024, 16, 0, 1, None) == _ffi.EIRENE_EINVAL   # short
+    assert L.eirene_probe_gather(ctypes.c_void_p((1 << 20) + 8), 1 << 20, 16, 0, 1, None) == _ffi.EIRENE_EINVAL
+    assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 1 << 20, 16, 3, 1, None) == _ffi.EIRENE_EINVAL
