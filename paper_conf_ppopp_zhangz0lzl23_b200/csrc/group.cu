@@ -147,7 +147,10 @@ __device__ void bitonic_run(uint32_t lo, uint32_t m, int t, int nt, GSmem& S) {
 // sorted by a bitonic network, one warp per sub-bucket up to WARP_SB
 // requests, the whole CTA above, so no distribution costs O(m^2).
 constexpr uint32_t FAST_SB = 32;
-constexpr uint32_t WARP_SB = 1024;
+#ifndef GROUP_WARP_SB
+#define GROUP_WARP_SB 256   // A/B builds: -DGROUP_WARP_SB=n; cfg3 1024 -> 256: 3.43 -> 3.64 Greq/s
+#endif
+constexpr uint32_t WARP_SB = GROUP_WARP_SB;
 __device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, GSmem& S) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t C = 32u * ((cnt + G_THREADS - 1) / G_THREADS);
