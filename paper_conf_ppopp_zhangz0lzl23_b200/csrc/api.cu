@@ -258,6 +258,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->cb.wseg, nb);
   AL(h->cb.wleaf, nb);
   AL(h->cb.wslot, nb);
+  AL(h->cb.wparent, nb);
   AL(h->cb.old, nb);
   AL(h->cb.istart, nb + 1);
   AL(h->cb.longseg, nb + 64);   // (segment, chunk) pairs of the long segments

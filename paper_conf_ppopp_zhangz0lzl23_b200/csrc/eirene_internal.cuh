@@ -293,6 +293,7 @@ struct CombBufs {
   uint32_t* wseg;
   uint32_t* wleaf;
   uint8_t* wslot;             // [n] slot of the write's key in its leaf at locate time, 255 = absent
+  uint32_t* wparent;          // [n] the write's leaf's parent (level-1 node) at locate time, NIL if the root is a leaf
   uint64_t* old;              // [n] old value per segment
   uint32_t* istart;           // [n+1] sorted position of each segment's first request (+ n at nseg)
   uint32_t* longseg;          // [n] segments longer than SHORT_SEG, finished by result_long_kernel

@@ -127,7 +127,8 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
                                                         const uint8_t* __restrict__ wop, uint32_t* __restrict__ wleaf,
-                                                        uint8_t* __restrict__ wslot, uint64_t* __restrict__ old,
+                                                        uint8_t* __restrict__ wslot, uint32_t* __restrict__ wparent,
+                                                        uint64_t* __restrict__ old,
                                                         const uint32_t* __restrict__ spay,
                                                         const uint32_t* __restrict__ pinfo,
                                                         const uint32_t* __restrict__ istart,
@@ -143,8 +144,9 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += stride) {
     const bool isq = i < nq;
     const uint64_t k = isq ? qkey[i] : wkey[i - nq];
-    uint32_t node = root;
+    uint32_t node = root, parent = NIL;
     for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
+      parent = node;   // after the loop: the leaf's parent (the level-1 node)
       // a 128 B separator line is four 256-bit loads (LDG.E.ENL2.256), then
       // the one child pointer: loading the whole child line alongside the keys
       // (one round trip per level instead of two) measured slower, as did two
@@ -160,6 +162,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
     }
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
+    if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
     retire(QueryIO{qseg, wseg, wop, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
            results, ctl);
   }
@@ -184,7 +187,8 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
 // cheaper way.  With EIRENE_F_STATS the kernel counts vertical / horizontal
 // RGs and traversal steps (Fig.10).
 __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* __restrict__ qkey,
-                                                                 const uint64_t* __restrict__ wkey, QueryIO io,
+                                                                 const uint64_t* __restrict__ wkey,
+                                                                 uint32_t* __restrict__ wparent, QueryIO io,
                                                                  const BatchArgs* __restrict__ A, Tree t,
                                                                  BatchCtl* __restrict__ ctl, uint32_t iter_rgs,
                                                                  uint32_t stats) {
@@ -215,11 +219,12 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
       const uint64_t kmax = kl[base + cnt - 1];   // sorted list: the RG's maximal key
       const uint64_t k = act ? kl[base + lane] : kmax;
       const bool vertical = buf_leaf == NIL || kmax > buf_rf;
-      uint32_t node, steps;
+      uint32_t node, steps, parent = NIL;   // parent: known after a vertical descent only
       uint64_t rep = 0;
       if (vertical) {
         node = root;
         for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
+          parent = node;
           const uint64_t* kp = t.ikeys + (size_t)node * FAN;
           ulonglong4 kv[4];
 #pragma unroll
@@ -240,6 +245,7 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
       }
       const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
       const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
+      if (act && !isq) wparent[base + lane] = parent;
       if (act) retire(io, isq ? base + lane : nq + base + lane, isq, nq, node, s, v, results, ctl);
       __syncwarp();
       const uint32_t top = __shfl_sync(FULL, node, cnt - 1);
@@ -527,11 +533,11 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
     // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
     const int iblocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 4u);
     query_iterwarp_kernel<<<iblocks < 1 ? 1 : iblocks, 256, 0, st>>>(
-        c.qkey, c.wkey, QueryIO{c.qseg, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
+        c.qkey, c.wkey, c.wparent, QueryIO{c.qseg, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
         A, t, ctl, iter_rgs, (flags & EIRENE_F_STATS) ? 1u : 0u);
   } else {
-    query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay,
-                                         c.pinfo, c.istart, c.longseg, A, t, ctl);
+    query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wleaf, c.wslot, c.wparent, c.old,
+                                         spay, c.pinfo, c.istart, c.longseg, A, t, ctl);
   }
   ++*launches;
 }

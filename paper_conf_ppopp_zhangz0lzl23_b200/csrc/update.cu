@@ -41,6 +41,7 @@ struct Ctx {
   const uint32_t* wseg;
   const uint32_t* wleaf;
   const uint8_t* wslot;
+  const uint32_t* wparent;   // the leaf's parent at locate time (level-0 parent hints), NIL if unknown
   uint64_t* old;
   uint64_t* eK[2];    // entry ping-pong buffers: separators to insert at the next level
   uint32_t* eC[2];
@@ -611,8 +612,15 @@ __device__ void acc_entries_buf(uint64_t* EK, uint32_t* EC, SepAcc& A, uint32_t 
   }
   A.n += cnt;
 }
-__device__ __forceinline__ void acc_entries(const Ctx& C, SepAcc& A, uint32_t b, uint32_t cnt) {
+// Level-0 entries of a split leaf, with their parent hint for the level-
+// synchronous lookup (the leaf's parent recorded by the locate traversal; the
+// inner levels do not change before that lookup, and the apply step validates
+// the parent's fences anyway).
+__device__ __forceinline__ void acc_entries(const Ctx& C, SepAcc& A, uint32_t b, uint32_t cnt, uint32_t parent) {
+  const uint32_t dst = (A.base == NIL ? b : A.base + A.n);
   acc_entries_buf(C.eK[0], C.eC[0], A, b, cnt);
+  if (C.eparent)
+    for (uint32_t x = lane_id(); x < cnt; x += 32) C.eparent[dst + x] = parent;
 }
 
 // One run of writes [b, e) whose first key was located in leaf `hint`.
@@ -620,6 +628,7 @@ __device__ __forceinline__ void acc_entries(const Ctx& C, SepAcc& A, uint32_t b,
 __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint, WarpStats& ws, SepAcc& acc) {
   const int lane = lane_id();
   const Tree& t = C.t;
+  const uint32_t hint0 = hint, b0 = b;   // the run's located leaf and first write
   uint32_t retry = 0;
   while (b < e && !ws.dead) {
     const uint64_t k0 = C.wkey[b];
@@ -660,7 +669,8 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
               rooted = true;
             }
             unlock(vp, v + 2u);   // split: version + 1 step
-            if (!rooted) acc_entries(C, acc, b, k - 1);
+            // parent hint: X was the located leaf (first try) and the inner levels are unchanged
+            if (!rooted) acc_entries(C, acc, b, k - 1, X == hint0 ? C.wparent[b0] : NIL);
           } else {
             unlock(vp, v);
           }
@@ -813,7 +823,11 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
     for (uint32_t ub = u0; ub < u1; ub += 32) {
       const uint32_t u = ub + lane;
       const uint2 su = u < u1 ? sl[u] : make_uint2(0, 0);
-      for (uint32_t x = 0; x < su.y; ++x) C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
+      for (uint32_t x = 0; x < su.y; ++x) {
+        // level 0: entries carry their parent hint (acc_entries); look up the rest
+        if (L == 0 && ld_cg(C.eparent + su.x + x) != NIL) continue;
+        C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
+      }
     }
     grid_barrier(C.ctl, gen);
     // apply step
@@ -1102,6 +1116,7 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
   C.wseg = c.wseg;
   C.wleaf = c.wleaf;
   C.wslot = c.wslot;
+  C.wparent = c.wparent;
   C.old = c.old;
   C.eK[0] = p.entA_key;
   C.eC[0] = p.entA_child;
