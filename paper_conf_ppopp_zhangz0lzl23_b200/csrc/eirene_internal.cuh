@@ -65,6 +65,7 @@ struct BatchCtl {
   uint32_t hot_ctr;       // hot-key timestamp bitmaps claimed by oversized groups
   uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
   uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
+  uint32_t uchunk;        // update kernel: next 32-write chunk (dynamic, level-synchronous mode)
   uint32_t rg_vertical, rg_horizontal;   // EIRENE_F_ITERWARP: RGs traversed vertically / horizontally
   unsigned long long trav_steps;         // EIRENE_F_ITERWARP: traversal steps of the issued requests
   uint32_t lvl_ent[MAX_LEVELS];   // separator entries produced for level L+1 (update kernel)

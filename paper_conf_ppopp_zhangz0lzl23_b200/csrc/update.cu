@@ -984,7 +984,16 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
   const bool lsync = C.regroup && C.slots[0] != nullptr && ctl->nins > 0;
   const uint32_t nchunks = (nw + 31) / 32;
   if (C.regroup) {
-    for (uint32_t chunk = gw; chunk * 32 < nw; chunk += nwarps) {
+    // Under a split storm a chunk's cost varies with its leaf runs and splits:
+    // chunks are handed out dynamically (a warp takes the next one when done) so
+    // the level-0 phase ends at the average warp's time, not the unluckiest one's
+    auto next_chunk = [&]() -> uint32_t {
+      uint32_t c = 0;
+      if (lane == 0) c = atomicAdd(&C.ctl->uchunk, 1u);
+      return __shfl_sync(FULL, c, 0);
+    };
+    for (uint32_t chunk = lsync ? next_chunk() : gw; chunk * 32 < nw;
+         chunk = lsync ? next_chunk() : chunk + nwarps) {
       const uint32_t base = chunk * 32;
       const uint32_t j = base + lane;
       const bool act = j < nw;
