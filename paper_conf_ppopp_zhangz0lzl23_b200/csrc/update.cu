@@ -820,13 +820,21 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
     // the next level's nonempty mask (its producers are warps): cleared here, before the apply step
     if ((gw & 31) == 0 && lane == 0) C.nemask[(L + 1) & 1][gw >> 5] = 0u;
     // lookup step: parent of every entry (lanes over units, then over a unit's entries)
-    for (uint32_t ub = u0; ub < u1; ub += 32) {
-      const uint32_t u = ub + lane;
-      const uint2 su = u < u1 ? sl[u] : make_uint2(0, 0);
-      for (uint32_t x = 0; x < su.y; ++x) {
-        // level 0: entries carry their parent hint (acc_entries); look up the rest
-        if (L == 0 && ld_cg(C.eparent + su.x + x) != NIL) continue;
-        C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
+    if (L == 0) {   // many small units (chunks): lanes over units
+      for (uint32_t ub = u0; ub < u1; ub += 32) {
+        const uint32_t u = ub + lane;
+        const uint2 su = u < u1 ? sl[u] : make_uint2(0, 0);
+        for (uint32_t x = 0; x < su.y; ++x) {
+          // level 0: entries carry their parent hint (acc_entries); look up the rest
+          if (ld_cg(C.eparent + su.x + x) != NIL) continue;
+          C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
+        }
+      }
+    } else {        // one unit per warp (its own entries): lanes over the unit's entries
+      for (uint32_t u = u0; u < u1; ++u) {
+        const uint2 su = sl[u];
+        for (uint32_t x = lane; x < su.y; x += 32)
+          C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
       }
     }
     grid_barrier(C.ctl, gen);
