@@ -303,7 +303,10 @@ struct CombBufs {
   uint32_t hot_words;         // >= max_batch / 32, a multiple of 4
 };
 constexpr int HOT_SLOTS = 64;
-constexpr uint32_t SHORT_SEG = 32;
+#ifndef EIRENE_SHORT_SEG
+#define EIRENE_SHORT_SEG 32   // A/B builds: -DEIRENE_SHORT_SEG=n
+#endif
+constexpr uint32_t SHORT_SEG = EIRENE_SHORT_SEG;
 constexpr int GROUP_STATUS_WORDS = NBINS_MAX;   // >= bsort_groups(n) for every n
 
 // bucket finish (sort in smem) + combine + partition, one CTA per bucket (group.cu)
