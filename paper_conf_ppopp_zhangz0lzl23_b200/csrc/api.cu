@@ -271,8 +271,9 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->up.slots[0], nb / 32 + 32768);
   AL(h->up.slots[1], nb / 32 + 32768);
   AL(h->up.eparent, nb + 64);
-  AL(h->up.nemask[0], 4096);
-  AL(h->up.nemask[1], 4096);
+  AL(h->up.flat_key, nb + 64);
+  AL(h->up.flat_child, nb + 64);
+  AL(h->up.flat_off, nb / 32 + 32768);
   AL(h->st_ops, HOST_SLOTS * nb);
   AL(h->st_keys, HOST_SLOTS * nb);
   AL(h->st_vals, HOST_SLOTS * nb);

@@ -66,6 +66,7 @@ struct BatchCtl {
   uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
   uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
   uint32_t uchunk;        // update kernel: next 32-write chunk (dynamic, level-synchronous mode)
+  uint32_t flat_total;    // update kernel: entries of the current upper level (flattened)
   uint32_t rg_vertical, rg_horizontal;   // EIRENE_F_ITERWARP: RGs traversed vertically / horizontally
   unsigned long long trav_steps;         // EIRENE_F_ITERWARP: traversal steps of the issued requests
   uint32_t lvl_ent[MAX_LEVELS];   // separator entries produced for level L+1 (update kernel)
@@ -320,11 +321,13 @@ struct UpdParams {
   uint32_t flags;
   uint2* slots[2];      // per producer unit (base, n) of the level-synchronous separator lists
   uint32_t* eparent;    // [n] parent node of each entry position (lookup step)
-  uint32_t* nemask[2];  // nonempty-producer bitmaps of the upper levels (one bit per warp)
   uint64_t* entA_key;
   uint32_t* entA_child;
   uint64_t* entB_key;
   uint32_t* entB_child;
+  uint64_t* flat_key;   // [n] an upper level's entries, concatenated in producer (= key) order
+  uint32_t* flat_child;
+  uint32_t* flat_off;   // [producers] exclusive prefix of the producers' entry counts
 };
 void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms,
                    cudaStream_t st, int* launches);

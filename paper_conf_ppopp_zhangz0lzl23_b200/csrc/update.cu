@@ -52,7 +52,9 @@ struct Ctx {
   BatchCtl* ctl;
   uint2* slots[2];      // level-synchronous propagation: per producer unit (base, n)
   uint32_t* eparent;    // parent found for each entry position (lookup step)
-  uint32_t* nemask[2];  // nonempty producer bitmaps of the upper levels
+  uint64_t* flat_key;   // upper levels: the level's entries concatenated in key order
+  uint32_t* flat_child;
+  uint32_t* flat_off;   // per producer warp: offset of its entries in the flat list
 };
 
 struct WarpStats {
@@ -712,6 +714,11 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
 //            fences (Alg.1:38) and merges the whole segment (inner_apply,
 //            multi-way split); the next level's separators are recorded per
 //            warp in slots[1 - x].  A root split builds the new root(s).
+// Levels >= 1 (few entries, produced by owner warps): the producers' lists are
+// first concatenated in key order into one flat list (per-CTA totals, a scan
+// by CTA 0, every warp copies its list and looks its entries' parents up), so
+// each parent's entries are contiguous; a warp owns the segments whose first
+// entry falls in its slice of the flat list (no gather).
 // Owners are unique per parent, so the locks are uncontended; a failed
 // validation (not expected) falls back to insert_up's optimistic / STM retry.
 __device__ int g_uprof = 0;   // diagnostic: print the phase times of the level-synchronous path
@@ -760,41 +767,6 @@ __device__ uint32_t descend_thread(const Tree& t, uint64_t k, uint32_t target) {
   return NIL;
 }
 
-// Nonempty-unit bitmaps of the upper levels (producer = warp): first set unit
-// >= from (U if none) / last set unit < before (NIL if none), 1024 units per step.
-__device__ uint32_t mask_next(const uint32_t* mk, uint32_t U, uint32_t from) {
-  const int lane = lane_id();
-  for (uint32_t wb = from >> 5; wb * 32 < U; wb += 32) {
-    const uint32_t w = wb + lane;
-    uint32_t word = w * 32 < U ? ld_cg(mk + w) : 0u;
-    if (w == (from >> 5)) word &= ~((1u << (from & 31)) - 1u);
-    const uint32_t bm = __ballot_sync(FULL, word != 0);
-    if (bm) {
-      const int l = __ffs(bm) - 1;
-      const uint32_t wd = __shfl_sync(FULL, word, l);
-      const uint32_t unit = (wb + l) * 32 + (__ffs(wd) - 1);
-      return unit < U ? unit : U;
-    }
-  }
-  return U;
-}
-__device__ uint32_t mask_prev(const uint32_t* mk, uint32_t before) {
-  const int lane = lane_id();
-  for (int64_t we = (int64_t)((before + 31) >> 5); we > 0; we -= 32) {
-    const int64_t w = we - 32 + lane;
-    uint32_t word = w >= 0 ? ld_cg(mk + w) : 0u;
-    if (w == (int64_t)(before >> 5)) word &= (1u << (before & 31)) - 1u;
-    if (w > (int64_t)(before >> 5)) word = 0;
-    const uint32_t bm = __ballot_sync(FULL, word != 0);
-    if (bm) {
-      const int l = 31 - __clz(bm);
-      const uint32_t wd = __shfl_sync(FULL, word, l);
-      return (uint32_t)(we - 32 + l) * 32 + (31 - __clz(wd));
-    }
-  }
-  return NIL;
-}
-
 // units [u0, u1) of a level's producer list, for this warp
 __device__ __forceinline__ void unit_range(uint32_t U, uint32_t gw, uint32_t nwarps, uint32_t& u0, uint32_t& u1) {
   u0 = (uint32_t)(((unsigned long long)U * gw) / nwarps);
@@ -817,8 +789,72 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
     uint32_t* Ch2 = C.eC[(L + 1) & 1];
     uint32_t u0, u1;
     unit_range(U, gw, nwarps, u0, u1);
-    // the next level's nonempty mask (its producers are warps): cleared here, before the apply step
-    if ((gw & 31) == 0 && lane == 0) C.nemask[(L + 1) & 1][gw >> 5] = 0u;
+    uint32_t ftotal = 0;   // L >= 1: entries of the flattened level
+    if (L > 0) {
+      // Upper levels: the producers are warps (one unit each, key order = warp
+      // order) and a parent's entries come from many of them.  Concatenate the
+      // units into one flat list (CTA 0 scans the counts, barrier, every warp
+      // copies its unit), so every segment is contiguous and the apply step
+      // walks 32-entry units instead of gathering unit by unit.
+      // (1) per CTA: its warps' (= producers') counts and their offsets inside
+      // the CTA; (2) CTA 0 scans the CTA totals; (3) every warp's offset
+      __shared__ uint32_t s_woff[4], s_cta;
+      if (threadIdx.x == 0) {
+        uint32_t run = 0;
+        for (uint32_t w = 0; w < (blockDim.x >> 5); ++w) {
+          s_woff[w] = run;
+          const uint32_t uw = blockIdx.x * (blockDim.x >> 5) + w;
+          run += uw < U ? sl[uw].y : 0u;
+        }
+        C.flat_off[blockIdx.x] = run;   // this CTA's total (scanned by CTA 0 below)
+      }
+      grid_barrier(C.ctl, gen);
+      if (blockIdx.x == 0) {
+        __shared__ uint32_t s_part[128];
+        const uint32_t nc = gridDim.x, per = (nc + blockDim.x - 1) / blockDim.x;
+        const uint32_t a0 = threadIdx.x * per, z0 = min(nc, a0 + per);
+        uint32_t v[16];   // per <= 16 (<= 2048 CTAs)
+        uint32_t sum = 0;
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+          v[q] = (a0 + q < z0) ? ld_cg(C.flat_off + a0 + q) : 0u;
+          sum += v[q];
+        }
+        s_part[threadIdx.x] = sum;
+        __syncthreads();
+        if (threadIdx.x == 0) {
+          uint32_t run = 0;
+          for (uint32_t i = 0; i < blockDim.x; ++i) {
+            const uint32_t c = s_part[i];
+            s_part[i] = run;
+            run += c;
+          }
+          C.ctl->flat_total = run;
+        }
+        __syncthreads();
+        uint32_t run = s_part[threadIdx.x];
+#pragma unroll
+        for (int q = 0; q < 16; ++q) {
+          if (a0 + q < z0) C.flat_off[a0 + q] = run;   // exclusive offset of CTA a0 + q
+          run += v[q];
+        }
+      }
+      grid_barrier(C.ctl, gen);
+      ftotal = ld_cg(&C.ctl->flat_total);
+      // copy my unit into the flat list and look its entries' parents up (lanes over entries)
+      if (threadIdx.x == 0) s_cta = ld_cg(C.flat_off + blockIdx.x);
+      __syncthreads();
+      for (uint32_t u = u0; u < u1; ++u) {   // (u == gw: my own unit)
+        const uint2 su = sl[u];
+        const uint32_t off = s_cta + s_woff[threadIdx.x >> 5];
+        for (uint32_t x = lane; x < su.y; x += 32) {
+          const uint64_t k = ld_cg(K + su.x + x);
+          C.flat_key[off + x] = k;
+          C.flat_child[off + x] = ld_cg(Ch + su.x + x);
+          C.eparent[off + x] = descend_thread(t, k, L + 1);
+        }
+      }
+    }
     // lookup step: parent of every entry (lanes over units, then over a unit's entries)
     if (L == 0) {   // many small units (chunks): lanes over units
       for (uint32_t ub = u0; ub < u1; ub += 32) {
@@ -830,25 +866,25 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
           C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
         }
       }
-    } else {        // one unit per warp (its own entries): lanes over the unit's entries
-      for (uint32_t u = u0; u < u1; ++u) {
-        const uint2 su = sl[u];
-        for (uint32_t x = lane; x < su.y; x += 32)
-          C.eparent[su.x + x] = descend_thread(t, ld_cg(K + su.x + x), L + 1);
-      }
     }
     grid_barrier(C.ctl, gen);
+    // the apply step's units: L = 0 the chunks; L >= 1 32-entry slices of the flat list
+    const uint32_t UA = L > 0 ? (ftotal + 31) / 32 : U;
+    if (L > 0) {
+      K = C.flat_key;
+      Ch = C.flat_child;
+      unit_range(UA, gw, nwarps, u0, u1);
+    }
+    auto unit = [&](uint32_t x) -> uint2 {
+      return L > 0 ? make_uint2(32u * x, min(32u, ftotal - 32u * x)) : sl[x];
+    };
     // apply step
     SepAcc nxt;
     // parent of the last entry before my range (the owner test of my first entry)
     uint32_t prevP = NIL;
-    const uint32_t* mk = C.nemask[L & 1];   // (L >= 1: nonempty producers)
-    if (L > 0) {
-      const uint32_t pu = mask_prev(mk, u0);
-      if (pu != NIL) {
-        const uint2 su = sl[pu];
-        prevP = ld_cg(C.eparent + su.x + su.y - 1);
-      }
+    if (L > 0 && u0 > 0 && u0 <= UA) {   // flat units are all nonempty: the previous one is u0 - 1
+      const uint2 su = unit(u0 - 1);
+      prevP = ld_cg(C.eparent + su.x + su.y - 1);
     }
     for (uint32_t ue = L > 0 ? 0u : u0; ue > 0;) {   // level 0: nearest nonempty chunk before u0, 32 per step
       const uint32_t ub = ue > 32 ? ue - 32 : 0;
@@ -865,7 +901,7 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
     }
     // next unit >= from with entries (U if none), 32 units per step
     auto next_nonempty = [&](uint32_t from) -> uint32_t {
-      if (L > 0) return mask_next(mk, U, from);
+      if (L > 0) return from < UA ? from : UA;
       for (uint32_t ub = from; ub < U; ub += 32) {
         const uint32_t uu = ub + lane;
         const bool ne = uu < U && sl[uu].y != 0;
@@ -874,9 +910,76 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
       }
       return U;
     };
+    // lock the parent P, validate its fences, merge the segment [hpos, hpos + m) of K / Ch
+    auto apply_segment = [&](uint32_t P, uint32_t hpos, uint32_t m) {
+      uint32_t* vp = &t.imeta[P].version;
+      uint32_t v;
+      bool done = false;
+      if (P != NIL && try_lock(vp, &v)) {
+        const size_t pb = (size_t)P * FAN;
+        const uint64_t pk = lane < FAN ? ld_cg(t.ikeys + pb + lane) : KEY_MAX;
+        const uint32_t pc = lane < FAN ? ld_cg(t.ichild + pb + lane) : NIL;
+        const uint32_t cP = ld_cg(&t.imeta[P].count);
+        const uint64_t plo = ld_cg(&t.imeta[P].lo), phi = ld_cg(&t.imeta[P].hi);
+        const uint32_t pnext = ld_cg(&t.imeta[P].next);
+        const uint64_t s0 = ld_cg(K + hpos), s1 = ld_cg(K + hpos + m - 1);
+        if (s0 >= plo && s1 < phi) {
+          uint32_t next_m = inner_apply(C, P, L + 1, pk, pc, cP, plo, phi, pnext, K, Ch, K2, Ch2, hpos, m, ws);
+          if (next_m > 0 && is_root(t, P, L + 1)) {
+            build_root(C, L + 1, P, plo, phi, K2, Ch2, K, Ch, hpos, next_m, ws);
+            next_m = 0;
+          }
+          unlock(vp, v + 2u);
+          if (next_m) acc_entries_buf(K2, Ch2, nxt, hpos, next_m);
+          done = true;
+        } else {
+          unlock(vp, v);
+        }
+      }
+      if (!done) {   // not expected: the generic optimistic / STM path, one level at a time upward
+        ws.retries += 1;
+        if (K != C.eK[L & 1]) {   // flat list: insert_up reads the level's own buffer (free by now)
+          for (uint32_t q = lane; q < m; q += 32) {
+            C.eK[L & 1][hpos + q] = ld_cg(K + hpos + q);
+            C.eC[L & 1][hpos + q] = ld_cg(Ch + hpos + q);
+          }
+          __threadfence();
+          __syncwarp();
+        }
+        insert_up(C, L, hpos, m, ws);
+      }
+    };
+    if (L > 0) {
+      // flat list: this warp owns the segments whose first entry lies in its
+      // slice of the entries; a segment is contiguous, found by one ballot per 32
+      const uint32_t e0 = (uint32_t)(((unsigned long long)ftotal * gw) / nwarps);
+      const uint32_t e1 = (uint32_t)(((unsigned long long)ftotal * (gw + 1)) / nwarps);
+      uint32_t prevE = e0 > 0 ? ld_cg(C.eparent + e0 - 1) : NIL;
+      uint32_t e = e0;
+      while (e < e1 && !ws.dead) {
+        const uint32_t P = ld_cg(C.eparent + e);
+        if (P == prevE) {   // continues a segment owned by an earlier warp
+          ++e;
+          continue;
+        }
+        uint32_t end = ftotal;
+        for (uint32_t b0 = e + 1; b0 < ftotal; b0 += 32) {
+          const uint32_t q = b0 + lane;
+          const uint32_t bm = __ballot_sync(FULL, q < ftotal && ld_cg(C.eparent + q) != P);
+          if (bm) {
+            end = b0 + __ffs(bm) - 1;
+            break;
+          }
+        }
+        apply_segment(P, e, end - e);
+        prevE = P;
+        e = end;
+      }
+      u0 = u1 = 0;   // (the unit loop below has nothing left to do)
+    }
     uint32_t u = u0, x = 0;   // cursor: entry x of unit u
     while (u < u1 && !ws.dead) {
-      const uint2 su = sl[u];
+      const uint2 su = unit(u);
       if (x >= su.y) {
         u = next_nonempty(u + 1);
         x = 0;
@@ -891,8 +994,8 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
       // a segment head in my range: gather its entries to [hpos, hpos + m)
       uint32_t m = 0, cu = u, cx = x;
       for (;;) {
-        if (cu >= U) break;
-        const uint2 sc = sl[cu];
+        if (cu >= UA) break;
+        const uint2 sc = unit(cu);
         if (cx >= sc.y) {
           cu = next_nonempty(cu + 1);
           cx = 0;
@@ -928,35 +1031,7 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
       }
       __threadfence();
       __syncwarp();
-      // lock the parent, validate, merge the whole segment
-      uint32_t* vp = &t.imeta[P].version;
-      uint32_t v;
-      bool done = false;
-      if (P != NIL && try_lock(vp, &v)) {
-        const size_t pb = (size_t)P * FAN;
-        const uint64_t pk = lane < FAN ? ld_cg(t.ikeys + pb + lane) : KEY_MAX;
-        const uint32_t pc = lane < FAN ? ld_cg(t.ichild + pb + lane) : NIL;
-        const uint32_t cP = ld_cg(&t.imeta[P].count);
-        const uint64_t plo = ld_cg(&t.imeta[P].lo), phi = ld_cg(&t.imeta[P].hi);
-        const uint32_t pnext = ld_cg(&t.imeta[P].next);
-        const uint64_t s0 = ld_cg(K + hpos), s1 = ld_cg(K + hpos + m - 1);
-        if (s0 >= plo && s1 < phi) {
-          uint32_t next_m = inner_apply(C, P, L + 1, pk, pc, cP, plo, phi, pnext, K, Ch, K2, Ch2, hpos, m, ws);
-          if (next_m > 0 && is_root(t, P, L + 1)) {
-            build_root(C, L + 1, P, plo, phi, K2, Ch2, K, Ch, hpos, next_m, ws);
-            next_m = 0;
-          }
-          unlock(vp, v + 2u);
-          if (next_m) acc_entries_buf(K2, Ch2, nxt, hpos, next_m);
-          done = true;
-        } else {
-          unlock(vp, v);
-        }
-      }
-      if (!done) {   // not expected: the generic optimistic / STM path, one level at a time upward
-        ws.retries += 1;
-        insert_up(C, L, hpos, m, ws);
-      }
+      apply_segment(P, hpos, m);
       prevP = P;
       u = cu;
       x = cx;
@@ -964,10 +1039,7 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
     }
     if (lane == 0) {
       sn[gw] = make_uint2(nxt.base == NIL ? 0u : nxt.base, nxt.n);
-      if (nxt.n) {
-        atomicAdd(&C.ctl->lvl_ent[L + 1], nxt.n);
-        atomicOr(&C.nemask[(L + 1) & 1][gw >> 5], 1u << (gw & 31));
-      }
+      if (nxt.n) atomicAdd(&C.ctl->lvl_ent[L + 1], nxt.n);
     }
     U = nwarps;
   }
@@ -1147,8 +1219,9 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
   C.slots[0] = p.slots[0];
   C.slots[1] = p.slots[1];
   C.eparent = p.eparent;
-  C.nemask[0] = p.nemask[0];
-  C.nemask[1] = p.nemask[1];
+  C.flat_key = p.flat_key;
+  C.flat_child = p.flat_child;
+  C.flat_off = p.flat_off;
   const uint32_t warps_needed = C.regroup ? (n + 31) / 32 : n;
   uint32_t blocks = (warps_needed + 3) / 4;
   // the level-synchronous phases need every CTA resident (grid barriers)
