@@ -268,7 +268,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->up.entA_child, nb + 64);
   AL(h->up.entB_key, nb + 64);
   AL(h->up.entB_child, nb + 64);
-  AL(h->up.slots[0], nb / 32 + 32768);
+  AL(h->up.slots[0], nb / 16 + 32768);   // level-0 chunks of 16 writes
   AL(h->up.slots[1], nb / 32 + 32768);
   AL(h->up.eparent, nb + 64);
   AL(h->up.flat_key, nb + 64);

@@ -1062,7 +1062,11 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
   SepAcc acc;
   // level-synchronous separators when the batch can split (launch: resident grid)
   const bool lsync = C.regroup && C.slots[0] != nullptr && ctl->nins > 0;
-  const uint32_t nchunks = (nw + 31) / 32;
+  // writes per chunk: a warp takes one chunk at a time and its leaf runs one
+  // after the other; under a split storm (lsync) each run is a long dependent
+  // chain, so chunks of 16 halve the runs a warp applies in a row
+  const uint32_t CH = lsync ? 16u : 32u;
+  const uint32_t nchunks = (nw + CH - 1) / CH;
   if (C.regroup) {
     // Under a split storm a chunk's cost varies with its leaf runs and splits:
     // chunks are handed out dynamically (a warp takes the next one when done) so
@@ -1072,11 +1076,11 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
       if (lane == 0) c = atomicAdd(&C.ctl->uchunk, 1u);
       return __shfl_sync(FULL, c, 0);
     };
-    for (uint32_t chunk = lsync ? next_chunk() : gw; chunk * 32 < nw;
+    for (uint32_t chunk = lsync ? next_chunk() : gw; chunk * CH < nw;
          chunk = lsync ? next_chunk() : chunk + nwarps) {
-      const uint32_t base = chunk * 32;
+      const uint32_t base = chunk * CH;
       const uint32_t j = base + lane;
-      const bool act = j < nw;
+      const bool act = (uint32_t)lane < CH && j < nw;
       const uint32_t lf = act ? C.wleaf[j] : NIL;
       const uint32_t pv = (act && j > 0) ? C.wleaf[j - 1] : NIL;
       const bool head = act && (j == 0 || lf != pv);
@@ -1137,7 +1141,7 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
           e = base + __ffs(later) - 1;
         } else {
           e = nw;
-          for (uint32_t s = base + 32; s < nw; s += 32) {
+          for (uint32_t s = base + CH; s < nw; s += 32) {
             const uint32_t jj = s + lane;
             const uint32_t mk = __ballot_sync(FULL, jj < nw && C.wleaf[jj] != leaf);
             if (mk) {
