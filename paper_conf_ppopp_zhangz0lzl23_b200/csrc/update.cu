@@ -1046,7 +1046,8 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
 }
 
 #ifndef UPD_MINB
-#define UPD_MINB 8   // resident CTAs per SM the register budget is fitted to (A/B builds: -DUPD_MINB=n)
+#define UPD_MINB 6   // resident CTAs per SM the register budget is fitted to (A/B builds: -DUPD_MINB=n;
+                     // r1h: 6 (80 regs, no spills) vs 8 (64 regs, 432 B spills): cfg1 0.389 -> 0.404, cfg2 6.92 -> 7.04)
 #endif
 __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
   const BatchCtl* ctl = C.ctl;
