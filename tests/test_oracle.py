@@ -232,6 +232,52 @@ def test_btree_checker_detects_corruption(kind, code):
     assert t.check() == code
 
 
+# Codes 3 (unequal leaf depth), 4 (fill outside [ceil(F/2), F] below the root,
+# both directions) and 7 (shape: #keys != #values) -- the "fill bounds, uniform
+# leaf depth" invariants of the B+tree that north_star names.
+@pytest.mark.parametrize("F", [3, 4, 5, 16])
+@pytest.mark.parametrize("kind,code", [(4, 4), (7, 7), (8, 4)])
+def test_btree_checker_detects_fill_shape(F, kind, code):
+    rng = np.random.default_rng(100 + F)
+    t = BTreeOracle(F)
+    keys = rng.permutation(np.arange(0, 4000, 2, dtype=np.uint64))
+    t.apply(np.full(keys.size, 2, np.uint8), keys, keys + 1)
+    assert t.check() == 0 and t.height() >= 3
+    assert t.corrupt(kind) == 0
+    assert t.check() == code
+
+
+@pytest.mark.parametrize("F", [3, 5, 16])
+def test_btree_depth_corruption_needs_small_fanout(F):
+    """A depth-only defect (a leaf pushed under a new 2-child inner node, every
+    other invariant intact) exists only when 2 children and 2 half-full leaves
+    are legal: F = 4.  Other fanouts: the hook refuses (F odd: no leaf splits into
+    two legal leaves) or the new node breaks fill first (F = 16: code 4)."""
+    t = BTreeOracle(F)
+    keys = np.random.default_rng(F).permutation(np.arange(0, 4000, 2, dtype=np.uint64))
+    t.apply(np.full(keys.size, 2, np.uint8), keys, keys + 1)
+    rc = t.corrupt(3)
+    if F in (3, 5):
+        assert rc == -1 and t.check() == 0
+    else:
+        assert rc == 0 and t.check() == 4
+
+
+def test_btree_checker_depth_only_violation_is_first_reported():
+    """A tree whose ONLY defect is unequal leaf depth (fill, order, fences, chain
+    and size all valid) must fail with 3, not pass: a checker that never tests
+    depth would accept it."""
+    t = BTreeOracle(4)
+    keys = np.random.default_rng(3).permutation(np.arange(0, 2000, 2, dtype=np.uint64))
+    t.apply(np.full(keys.size, 2, np.uint8), keys, keys + 1)
+    n0 = t.size()
+    assert t.corrupt(3) == 0
+    assert t.size() == n0
+    # every key is still found with its value, in order (the defect is structural only)
+    assert np.array_equal(t.scan(0, 1 << 62)[0], np.sort(keys))
+    assert t.check() == 3
+
+
 def test_combining_vs_map_conflict_heavy():
     rng = np.random.default_rng(11)
     keys, vals = _rand_tree(rng, 200, 0, 400)
