@@ -118,6 +118,13 @@ typedef struct {
                                  Fig.10 "traversal steps"); 0 otherwise            */
   uint64_t rg_vertical;       /* EIRENE_F_ITERWARP|STATS: request groups traversed from the root */
   uint64_t rg_horizontal;     /* ... and along the leaf links from the iteration warp's buffer  */
+  uint64_t device_ns;         /* batch response time on the device: %globaltimer at the start of
+                                 the batch's first kernel to the end of its last one (ns); the
+                                 paper's per-batch time without host
+                                 launch jitter                                                  */
+  uint64_t nins, ndelp;       /* issued inserts of absent keys / deletes of present keys: the
+                                 structural writes left to the update kernel (value overwrites
+                                 of present keys are applied in place by the query kernel)      */
 } eirene_batch_stats;
 
 /* Creates a tree (one empty leaf) on cfg->device and allocates every pool and

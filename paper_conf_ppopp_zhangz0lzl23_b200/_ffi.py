@@ -17,7 +17,8 @@ ROOT = os.path.dirname(PKG)
 LIB_PATH = os.environ.get("EIRENE_LIB") or os.path.join(PKG, "libeirene.so")
 HEADER = os.path.join(ROOT, "include", "eirene.h")
 
-EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECUDA = 0, -1, -2, -3, -4, -5
+EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECUDA, EIRENE_EINTERNAL = (
+    0, -1, -2, -3, -4, -5, -6)
 EIRENE_QUERY, EIRENE_UPDATE, EIRENE_INSERT, EIRENE_DELETE, EIRENE_RANGE = 0, 1, 2, 3, 4
 EIRENE_F_REGROUP, EIRENE_F_STATS, EIRENE_F_FORCE_STM, EIRENE_F_TIMING, EIRENE_F_ITERWARP = 1, 2, 4, 8, 16
 NOT_FOUND = 0xFFFFFFFFFFFFFFFF
@@ -40,7 +41,7 @@ class eirene_batch_stats(ctypes.Structure):
                 ("leaf_splits", _u64), ("inner_splits", _u64), ("new_leaves", _u64), ("new_inner", _u64),
                 ("height", _u32), ("launches", _u32), ("stage_ms", ctypes.c_float * 8),
                 ("ranges", _u64), ("artificial", _u64), ("trav_steps", _u64), ("rg_vertical", _u64),
-                ("rg_horizontal", _u64)]
+                ("rg_horizontal", _u64), ("device_ns", _u64), ("nins", _u64), ("ndelp", _u64)]
 
     def to_dict(self) -> dict:
         d = {f: getattr(self, f) for f, _ in self._fields_ if f != "stage_ms"}

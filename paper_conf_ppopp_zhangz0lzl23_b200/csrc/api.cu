@@ -34,6 +34,22 @@ int cuda_fail(cudaError_t e, const char* where) {
   return EIRENE_ECUDA;
 }
 
+// Makes the handle's device current for the duration of an ABI call and
+// restores the caller's current device on return (the caller's CUDA state is
+// not changed behind its back).
+struct DeviceGuard {
+  int prev = -1;
+  cudaError_t err = cudaSuccess;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) err = cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
 #define CK(expr)                                    \
   do {                                              \
     cudaError_t _e = (expr);                        \
@@ -77,6 +93,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero2_n16; i += gridDim.x * blockDim.x)
     zero2[i] = make_uint4(0, 0, 0, 0);
   if (blockIdx.x == 0 && threadIdx.x == 0) {
+    dst->t0 = gtime_ns();
     dst->ops = ops;
     dst->keys = keys;
     dst->vals = vals_stage ? vals_stage : vals_src;
@@ -195,6 +212,7 @@ const char* eirene_strerror(int code) {
     case EIRENE_EFULL: return "node pools lack headroom for the batch";
     case EIRENE_ESTATE: return "call not valid in this state (or stale ticket)";
     case EIRENE_ECUDA: return "CUDA error (see eirene_last_cuda_error)";
+    case EIRENE_EINTERNAL: return "device watchdog fired: no forward progress (internal error; discard the tree)";
     default: return "unknown error";
   }
 }
@@ -214,7 +232,8 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   if (cfg->fanout != 16 || cfg->max_batch == 0 || cfg->max_batch > (1u << 29) || cfg->key_lo >= cfg->key_hi ||
       cfg->max_keys == 0)
     return EIRENE_EINVAL;
-  CK(cudaSetDevice(cfg->device));
+  DeviceGuard dg_(cfg->device);
+  CK(dg_.err);
   eirene_tree* h = new (std::nothrow) eirene_tree();
   if (!h) return EIRENE_ENOMEM;
   h->cfg = *cfg;
@@ -312,7 +331,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     const size_t l_cu = bump(sizeof(uint32_t) * NBINS_L);
     const size_t l_gs = bump(sizeof(unsigned long long) * NBINS_L);
     h->zero_large_bytes = off;
-    if (nb > (1u << 22)) AL(h->zero_large, off);
+    if (nb > bsort_fused_capacity(h->num_sms)) AL(h->zero_large, off);   // the two-kernel path's region
     if (e == cudaSuccess) {
       h->ctl = reinterpret_cast<BatchCtl*>(h->zero_region + o_ctl);
       h->sb.ghist = reinterpret_cast<uint32_t*>(h->zero_region + o_gh);
@@ -360,7 +379,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
 
 int eirene_destroy(eirene_handle h) {
   if (!h) return EIRENE_EINVAL;
-  cudaSetDevice(h->cfg.device);
+  DeviceGuard dg_(h->cfg.device);
   cudaDeviceSynchronize();
   for (int i = 0; i < RING; ++i) {
     if (h->ring[i].done) cudaEventDestroy(h->ring[i].done);
@@ -392,7 +411,8 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals
   if (h->loaded || h->modified) return EIRENE_ESTATE;
   if (n == 0) return EIRENE_OK;
   if (!keys || !vals || !(leaf_fill > 0.f) || leaf_fill > 1.f) return EIRENE_EINVAL;
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   int per = (int)(16.f * leaf_fill + 0.5f);
   if (per < 1) per = 1;
@@ -420,7 +440,8 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
                        uint64_t* rkeys = nullptr, uint64_t* rvals = nullptr, uint32_t rcap = 0,
                        bool prepare_only = false, bool prepare_range = false) {
   const bool range = rkeys != nullptr || prepare_range;
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   if (prepare_only && (!h->use_graphs || (h->cfg.flags & EIRENE_F_TIMING))) return EIRENE_OK;
   const uint64_t tk = prepare_only ? 0 : h->next_ticket++;
   Rec scratch_rec;
@@ -456,7 +477,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   BatchCtl* ctl_slot = h->ctl_ring + tk % RING;
   uint4* zero16 = reinterpret_cast<uint4*>(h->zero_region);
   uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
-  const bool large = n > (1u << 22);   // two-kernel bucket sort with 16384 bins (bsort.cu)
+  const bool large = !bsort_fused(n, h->num_sms);   // two-kernel bucket sort with 16384 bins (bsort.cu)
   uint4* zero2 = reinterpret_cast<uint4*>(large ? h->zero_large : h->zero_region);
   uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
   const BSortBufs& bsn = large ? h->bsL : h->bs;
@@ -484,7 +505,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
     stage("update");
     if (timing) rec(4, s);
-    launch_result(spay, h->bs.kB, n, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, s, &launches);
+    launch_result(spay, h->bs.kB, n, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, h->num_sms, s, &launches);
     stage("result");
     if (timing) rec(5, s);
     return cudaGetLastError();
@@ -563,7 +584,8 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
   if (!h || !ops || !keys || !vals || !results || !ticket) return EIRENE_EINVAL;
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   // Triple-buffered staging (HOST_SLOTS), three streams: the H2D of this batch (copy
   // stream) overlaps the previous batch's kernels (`st`) and the D2H of its
   // results (d2h stream).  A slot is reused only after the D2H of the batch
@@ -606,6 +628,8 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
 
 int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) {
   if (!h) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   Rec& r = h->ring[ticket % RING];
   if (!r.used || r.ticket != ticket) return EIRENE_ESTATE;
   CK(cudaEventSynchronize(r.done));
@@ -636,6 +660,9 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) 
     stats->trav_steps = c.trav_steps;
     stats->rg_vertical = c.rg_vertical;
     stats->rg_horizontal = c.rg_horizontal;
+    stats->device_ns = c.t_end > c.t_begin ? c.t_end - c.t_begin : 0;
+    stats->nins = c.nins;
+    stats->ndelp = c.ndelp;
     if (r.timing) {
       for (int s = 0; s + 1 < NSTAGE; ++s) cudaEventElapsedTime(&stats->stage_ms[s], r.st[s], r.st[s + 1]);
       cudaEventElapsedTime(&stats->stage_ms[7], r.st[0], r.st[NSTAGE - 1]);
@@ -648,7 +675,8 @@ int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out, u
                 uint64_t* count, eirene_stream_t stream) {
   if (!h || !count) return EIRENE_EINVAL;
   if (cap > 0 && !keys_out && !vals_out) return EIRENE_EINVAL;
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
   TreeHdr hdr;
   CK(cudaMemcpyAsync(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost, st));
@@ -675,7 +703,8 @@ int eirene_set_flags(eirene_handle h, uint32_t flags) {
 
 int eirene_get_info(eirene_handle h, eirene_tree_info* info) {
   if (!h || !info) return EIRENE_EINVAL;
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   TreeHdr hdr;
   CK(cudaMemcpy(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost));
   info->height = (uint32_t)(hdr.root_word >> 32);
@@ -693,7 +722,8 @@ int eirene_get_info(eirene_handle h, eirene_tree_info* info) {
 // Host-side structural check of a quiescent tree (debug utility).
 int eirene_check_invariants(eirene_handle h, uint64_t* n_keys) {
   if (!h) return EIRENE_EINVAL;
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   CK(cudaDeviceSynchronize());
   TreeHdr hdr;
   CK(cudaMemcpy(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost));
@@ -781,7 +811,8 @@ int eirene_route_partition(eirene_handle h, const uint8_t* ops, const uint64_t* 
   if (n > h->cfg.max_batch) return EIRENE_EINVAL;
   if (n > 0 && (!ops || !keys || !vals || !sops || !skeys || !svals || !perm)) return EIRENE_EINVAL;
   if (P > 1 && !splitters) return EIRENE_EINVAL;
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   int launches = 0;
   launch_route_partition(ops, keys, vals, n, splitters, P, sops, skeys, svals, perm, counts, invalid, h->route_lb,
                          h->route_ctr, ++h->route_epoch, reinterpret_cast<cudaStream_t>(stream), &launches);
@@ -794,7 +825,8 @@ int eirene_route_unpermute(eirene_handle h, const uint64_t* recv, const uint32_t
                            eirene_stream_t stream) {
   if (!h) return EIRENE_EINVAL;
   if (n > 0 && (!recv || !perm || !results)) return EIRENE_EINVAL;
-  CK(cudaSetDevice(h->cfg.device));
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
   int launches = 0;
   launch_route_unpermute(recv, perm, n, results, reinterpret_cast<cudaStream_t>(stream), &launches);
   h->launches += launches;

@@ -354,28 +354,43 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
 
 }  // namespace
 
+static uint32_t dist_grid(int num_sms) {
+  static int occ[MAX_DEVICES];
+  const int per_sm = per_device(occ, [] {
+    int v = 0;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, bsort_dist_kernel, D_THREADS, 0) == cudaSuccess ? v
+                                                                                                           : 0;
+  });
+  return (uint32_t)num_sms * (uint32_t)std::max(per_sm, 0);
+}
+
+// The ONE predicate choosing the distribution path (used by the launcher, the
+// group count and the handle's buffer choice in api.cu): the fused kernel
+// (4096 bins, keys held in registers by one resident wave) when the batch fits
+// that wave, else the two-kernel path (16384 bins, its own zeroed region).
+bool bsort_fused(uint32_t n, int num_sms) {
+  const uint32_t grid = dist_grid(num_sms);
+  return grid > 0 && (uint64_t)grid * D_THREADS * D_ITEMS >= n;
+}
+uint64_t bsort_fused_capacity(int num_sms) { return (uint64_t)dist_grid(num_sms) * D_THREADS * D_ITEMS; }
+
 uint32_t bsort_groups(uint32_t n, int num_sms) {
   // two resident group CTAs per SM when n allows; ~3.5K requests per group
-  // otherwise.  Up to 2^22 requests the fused kernel cuts 4096 bins; above,
+  // otherwise.  The fused kernel cuts 4096 bins (at most NBINS / 2 groups);
   // the two-kernel path cuts 16384 (every group still fits shared memory
   // unless one key holds more than a group's worth of requests)
   uint32_t g = (n + 3583) / 3584;
   const uint32_t par = std::min<uint32_t>(2u * (uint32_t)num_sms, (n + 255) / 256);
   g = std::max(g, par);
-  const uint32_t cap = n > (1u << 22) ? (uint32_t)NBINS_L : (uint32_t)NBINS / 2;
+  const uint32_t cap = bsort_fused(n, num_sms) ? (uint32_t)NBINS / 2 : (uint32_t)NBINS_L;
   return std::max(1u, std::min(g, cap));
 }
 
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
                         BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
   const uint32_t G = bsort_groups(n, num_sms);
-  static int dist_per_sm = -1;
-  if (dist_per_sm < 0) {
-    if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&dist_per_sm, bsort_dist_kernel, D_THREADS, 0) != cudaSuccess)
-      dist_per_sm = 0;
-  }
-  const uint32_t grid = (uint32_t)num_sms * (uint32_t)dist_per_sm;
-  if (n <= (1u << 22) && grid > 0 && (uint64_t)grid * D_THREADS * D_ITEMS >= n) {
+  const uint32_t grid = dist_grid(num_sms);
+  if (bsort_fused(n, num_sms)) {
     uint32_t bshift = bin_shift(key_lo, key_hi, BIN_BITS);
     // fused single launch; slices of whole 512-request rows per CTA
     const uint32_t rows = (n + D_THREADS - 1) / D_THREADS;
@@ -391,14 +406,13 @@ void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_
     return;
   }
   const uint32_t bshift = bin_shift(key_lo, key_hi, BIN_BITS_L);
-  static bool attr = false;
   const size_t hsm = 2 * NBINS_L * sizeof(uint32_t);
   const size_t ssm = NBINS_L * sizeof(uint16_t) + (size_t)NBINS_L * sizeof(uint32_t);
-  if (!attr) {
+  static int attr[MAX_DEVICES];
+  per_device(attr, [&] {
     cudaFuncSetAttribute(bsort_hist_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)hsm);
-    cudaFuncSetAttribute(bsort_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ssm);
-    attr = true;
-  }
+    return (int)cudaFuncSetAttribute(bsort_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ssm);
+  });
   const uint32_t tiles = (n + H_THREADS * H_ITEMS - 1) / (H_THREADS * H_ITEMS);
   bsort_hist_kernel<<<std::max(1u, std::min(tiles, (uint32_t)num_sms)), H_THREADS, hsm, st>>>(
       A, n, G, key_lo, bshift, b.bcount, b.bin2grp, b.gstart, b.cursor, ctl);

@@ -64,6 +64,10 @@ struct BatchCtl {
   uint32_t nrange, nart;  // range queries in the batch; artificial queries resolved
   uint32_t hot_ctr;       // hot-key timestamp bitmaps claimed by oversized groups
   uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
+  uint32_t ndelp;         // issued deletes of present keys (query kernel); nins == ndelp == 0 -> every
+                          // issued write was a value overwrite, applied in place by the query kernel
+  uint32_t fin_ctr;       // result_long_kernel: CTAs finished (the last one publishes the BatchCtl)
+  unsigned long long t_begin, t_end;   // %globaltimer (ns) at the batch's first / last kernel
   uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
   uint32_t uchunk;        // update kernel: next 32-write chunk (dynamic, level-synchronous mode)
   uint32_t flat_total;    // update kernel: entries of the current upper level (flattened)
@@ -116,6 +120,7 @@ struct BatchArgs {
   uint64_t* rkeys;      // range-query output (eirene_submit_batch_range), else null: RANGE ops invalid
   uint64_t* rvals;
   uint32_t rcap;
+  unsigned long long t0;   // %globaltimer when the batch's first kernel started (device batch time)
 };
 
 // tile counters
@@ -226,6 +231,25 @@ __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
 
 __host__ __device__ __forceinline__ bool is_write(uint32_t op) { return op != OP_QUERY; }
 
+// ------------------------------------------------------------ per-device host state
+// One-time host-side state (function attributes, occupancy) is per DEVICE:
+// a process may hold handles on several GPUs.  Keyed by the current device
+// (every ABI entry point makes the handle's device current).  0 = not yet
+// computed; a benign race between threads computes the same value twice.
+constexpr int MAX_DEVICES = 64;
+inline int current_device() {
+  int d = 0;
+  cudaGetDevice(&d);
+  return d;
+}
+template <class F>
+inline int per_device(int (&cache)[MAX_DEVICES], F compute) {
+  const int d = current_device();
+  if (d < 0 || d >= MAX_DEVICES) return compute();
+  if (cache[d] == 0) cache[d] = compute() + 1;
+  return cache[d] - 1;
+}
+
 // ------------------------------------------------------------ host-side launchers
 // (defined in the .cu files; called from api.cu)
 struct SortBufs {
@@ -281,6 +305,8 @@ struct BSortBufs {
   uint32_t* cursor;  // [NBINS_MAX] group fill cursors (zeroed per batch)
 };
 uint32_t bsort_groups(uint32_t n, int num_sms);
+bool bsort_fused(uint32_t n, int num_sms);         // the distribution path of an n-request batch
+uint64_t bsort_fused_capacity(int num_sms);        // largest batch of the fused path
 void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_t key_hi, const BSortBufs& b,
                         BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches);
 
@@ -335,9 +361,7 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
 void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const uint64_t* kB, const BatchArgs* A, Tree t,
                   BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches);
 void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const CombBufs& c, const BatchArgs* A,
-                   BatchCtl* ctl,
-                   const TreeHdr* hdr, int dbgprint,
-                   cudaStream_t st, int* launches);
+                   BatchCtl* ctl, const TreeHdr* hdr, int dbgprint, int num_sms, cudaStream_t st, int* launches);
 
 // bulk build / scan
 int build_tree(Tree t, const uint64_t* keys, const uint64_t* vals, uint64_t n, int per_leaf, uint64_t key_lo,

@@ -1264,11 +1264,10 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
 
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(group_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(GSmem));
-    attr = true;
-  }
+  static int attr[MAX_DEVICES];
+  per_device(attr, [] {
+    return (int)cudaFuncSetAttribute(group_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(GSmem));
+  });
   GroupArgs g;
   g.A = A;
   g.kA = b.kA;

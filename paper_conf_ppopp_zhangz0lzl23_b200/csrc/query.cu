@@ -67,6 +67,7 @@ struct QueryIO {
   const uint32_t* __restrict__ qseg;
   const uint32_t* __restrict__ wseg;
   const uint8_t* __restrict__ wop;
+  const uint64_t* __restrict__ wval;
   uint32_t* __restrict__ wleaf;
   uint8_t* __restrict__ wslot;
   uint64_t* __restrict__ old;
@@ -77,7 +78,8 @@ struct QueryIO {
 };
 
 __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, uint32_t nq, uint32_t node, int s,
-                                       uint64_t v, uint64_t* __restrict__ results, BatchCtl* __restrict__ ctl) {
+                                       uint64_t v, uint64_t* __restrict__ results, BatchCtl* __restrict__ ctl,
+                                       uint64_t* __restrict__ lvals) {
   const uint32_t* __restrict__ qseg = io.qseg;
   const uint32_t* __restrict__ wseg = io.wseg;
   const uint8_t* __restrict__ wop = io.wop;
@@ -89,7 +91,8 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
   const uint32_t* __restrict__ istart = io.istart;
   uint32_t* __restrict__ longseg = io.longseg;
   uint32_t seg;
-  bool ins = false;   // an upsert of an absent key: the only request that can split a leaf
+  bool ins = false;    // an upsert of an absent key: the only request that can split a leaf
+  bool delp = false;   // a delete of a present key: removes a key from its leaf
   if (isq) {
     seg = qseg[i];
   } else {
@@ -97,11 +100,24 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
     seg = wseg[w];
     wleaf[w] = node;
     wslot[w] = s >= 0 ? (uint8_t)s : (uint8_t)255;
-    ins = s < 0 && wop[w] != OP_DELETE;
+    const uint32_t op = wop[w];
+    ins = s < 0 && op != OP_DELETE;
+    delp = s >= 0 && op == OP_DELETE;
+    // A value overwrite (upsert of a present key) changes one value slot and
+    // nothing else, so it is applied here, by the thread that located it: the
+    // structure is quiescent during this kernel (the update kernel runs after
+    // it), issued keys are distinct (one issued request per key,
+    // P:728-745), so no concurrent issued query reads this slot, and v above
+    // is already the pre-batch value the write returns.  The update kernel
+    // then only has the structural writes (inserts of absent keys, deletes of
+    // present ones) to do, and re-applies overwrites idempotently.
+    if (s >= 0 && op != OP_DELETE) lvals[(size_t)node * LSTRIDE + s] = io.wval[w];
   }
   {
-    const uint32_t m = __ballot_sync(__activemask(), ins);
+    const uint32_t am = __activemask();
+    const uint32_t m = __ballot_sync(am, ins), md = __ballot_sync(am, delp);
     if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&ctl->nins, (uint32_t)__popc(m));
+    if (md && (threadIdx.x & 31) == __ffs(md) - 1) atomicAdd(&ctl->ndelp, (uint32_t)__popc(md));
   }
   old[seg] = v;
   const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
@@ -126,7 +142,8 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
-                                                        const uint8_t* __restrict__ wop, uint32_t* __restrict__ wleaf,
+                                                        const uint8_t* __restrict__ wop,
+                                                        const uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
                                                         uint8_t* __restrict__ wslot, uint32_t* __restrict__ wparent,
                                                         uint64_t* __restrict__ old,
                                                         const uint32_t* __restrict__ spay,
@@ -163,8 +180,8 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
     if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
-    retire(QueryIO{qseg, wseg, wop, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
-           results, ctl);
+    retire(QueryIO{qseg, wseg, wop, wval, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
+           results, ctl, t.lvals);
   }
 }
 
@@ -246,7 +263,7 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
       const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
       const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
       if (act && !isq) wparent[base + lane] = parent;
-      if (act) retire(io, isq ? base + lane : nq + base + lane, isq, nq, node, s, v, results, ctl);
+      if (act) retire(io, isq ? base + lane : nq + base + lane, isq, nq, node, s, v, results, ctl, t.lvals);
       __syncwarp();
       const uint32_t top = __shfl_sync(FULL, node, cnt - 1);
       const uint32_t rm = __ballot_sync(FULL, act && steps > height);
@@ -284,49 +301,69 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
                                                             const BatchArgs* __restrict__ A,
                                                             BatchCtl* __restrict__ ctl, const TreeHdr* hdr,
                                                             int dbgprint) {
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
-    // end of the batch (the last kernel; nothing below changes ctl): final
-    // status and height, then the whole BatchCtl to the batch's ring slot
-    if (ctl->invalid) ctl->status = EIRENE_EINVAL;
-    ctl->height = (uint32_t)(hdr->root_word >> 32);
-    *A->ctl_out = *ctl;
-    if (dbgprint)
-      printf("[eirene dbg] %u %u %u %u %u %u %u %u\n", ctl->dbg[0], ctl->dbg[1], ctl->dbg[2], ctl->dbg[3],
-             ctl->dbg[4], ctl->dbg[5], ctl->dbg[6], ctl->dbg[7]);
-    if (ctl->uprof[0]) {   // EIRENE_UPDATE_PROF: update-kernel phases (us since its start)
-      printf("[upd prof] entries %u %u %u %u %u | t:", ctl->lvl_ent[0], ctl->lvl_ent[1], ctl->lvl_ent[2],
-             ctl->lvl_ent[3], ctl->lvl_ent[4]);
-      for (int i = 1; i < 24 && ctl->uprof[i]; ++i) printf(" %.1f", (ctl->uprof[i] - ctl->uprof[0]) * 1e-3);
-      printf("\n");
-    }
-  }
-  if (ctl->invalid || ctl->status != 0) return;
-  uint64_t* __restrict__ results = A->results;
-  const uint64_t* __restrict__ vals = A->vals;
-  const uint32_t nl = ctl->nlong;
-  for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
-    const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
-    const uint64_t v = old[s];
-    const uint32_t b = istart[s] + ch * RCHUNK;
-    const uint32_t e = min(istart[s + 1], b + RCHUNK);
-    for (uint32_t p0 = b + threadIdx.x; p0 < e; p0 += 4 * blockDim.x) {   // 4 loads in flight
-      uint32_t pi[4], py[4];
+  if (!(ctl->invalid || ctl->status != 0)) {
+    uint64_t* __restrict__ results = A->results;
+    const uint64_t* __restrict__ vals = A->vals;
+    const uint32_t nl = ctl->nlong;
+    for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
+      const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
+      const uint64_t v = old[s];
+      const uint32_t b = istart[s] + ch * RCHUNK;
+      const uint32_t e = min(istart[s + 1], b + RCHUNK);
+      for (uint32_t p0 = b + threadIdx.x; p0 < e; p0 += 4 * blockDim.x) {   // 4 loads in flight
+        uint32_t pi[4], py[4];
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        const uint32_t p = p0 + u * blockDim.x;
-        pi[u] = p < e ? pinfo[p] : DONE_BIT;
-        py[u] = p < e ? spay[p] : 0u;
-      }
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t p = p0 + u * blockDim.x;
+          pi[u] = p < e ? pinfo[p] : DONE_BIT;
+          py[u] = p < e ? spay[p] : 0u;
+        }
 #pragma unroll
-      for (int u = 0; u < 4; ++u) {
-        if (!(pi[u] & DONE_BIT)) {
-          results[py[u] >> 2] = v;   // no earlier write in the segment: the issued request's value
-        } else if (pi[u] & DEFER_BIT) {   // hot key: the nearest earlier write (its payload in kB)
-          const uint32_t pw = (uint32_t)kB[p0 + u * blockDim.x];
-          results[py[u] >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
+        for (int u = 0; u < 4; ++u) {
+          if (!(pi[u] & DONE_BIT)) {
+            results[py[u] >> 2] = v;   // no earlier write in the segment: the issued request's value
+          } else if (pi[u] & DEFER_BIT) {   // hot key: the nearest earlier write (its payload in kB)
+            const uint32_t pw = (uint32_t)kB[p0 + u * blockDim.x];
+            results[py[u] >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
+          }
         }
       }
     }
+  }
+  // End of the batch (the last kernel): the last CTA to finish stamps the
+  // device end time, sets the final status and height and publishes the whole
+  // BatchCtl to the batch's ring slot (one word per thread).
+  __shared__ uint32_t s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(&ctl->fin_ctr, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  if (threadIdx.x == 0) {
+    if (ld_cg(&ctl->invalid)) ctl->status = EIRENE_EINVAL;
+    ctl->height = (uint32_t)(hdr->root_word >> 32);
+    ctl->t_begin = A->t0;
+    ctl->t_end = gtime_ns();
+  }
+  __syncthreads();
+  {
+    static_assert(sizeof(BatchCtl) % 8 == 0, "BatchCtl is copied as u64 words");
+    const unsigned long long* src = reinterpret_cast<const unsigned long long*>(ctl);
+    unsigned long long* dst = reinterpret_cast<unsigned long long*>(A->ctl_out);
+    for (uint32_t i = threadIdx.x; i < sizeof(BatchCtl) / 8; i += blockDim.x) dst[i] = __ldcg(src + i);
+  }
+  if (threadIdx.x == 0 && dbgprint) {
+    printf("[eirene dbg] %u %u %u %u %u %u %u %u\n", ctl->dbg[0], ctl->dbg[1], ctl->dbg[2], ctl->dbg[3],
+           ctl->dbg[4], ctl->dbg[5], ctl->dbg[6], ctl->dbg[7]);
+  }
+  if (threadIdx.x == 0 && ctl->uprof[0]) {   // EIRENE_UPDATE_PROF: update-kernel phases (us since its start)
+    printf("[upd prof] entries %u %u %u %u %u | t:", ctl->lvl_ent[0], ctl->lvl_ent[1], ctl->lvl_ent[2],
+           ctl->lvl_ent[3], ctl->lvl_ent[4]);
+    for (int i = 1; i < 24 && ctl->uprof[i]; ++i) printf(" %.1f", (ctl->uprof[i] - ctl->uprof[0]) * 1e-3);
+    printf("\n");
   }
 }
 
@@ -386,6 +423,7 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
                                                     const uint32_t* __restrict__ pinfo,
                                                     const uint32_t* __restrict__ istart,
                                                     const uint64_t* __restrict__ kB,
+                                                    const uint64_t* __restrict__ old,
                                                     const BatchArgs* __restrict__ A, Tree t, BatchCtl* __restrict__ ctl) {
   if (ctl->invalid || ctl->status != 0 || ctl->nrange == 0) return;
   const uint8_t* __restrict__ ops = A->ops;
@@ -481,12 +519,17 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
               wk = w < nw ? wkey[w] : KEY_MAX;
             }
             if (c >= cap) break;
-            uint64_t v = ldg64_pol(lv + s, pf);
+            uint64_t v;
             if (wk == k) {
-              v = artificial_query(w, i, v, wseg, istart, spay, pinfo, kB, vals, results);
+              // a written key: its pre-batch value is the one its issued write's
+              // locate retrieved (old[seg]); the slot may already hold the write's
+              // value (overwrites are applied in place by the query kernel)
+              v = artificial_query(w, i, old[wseg[w]], wseg, istart, spay, pinfo, kB, vals, results);
               ++nart;
               ++w;
               wk = w < nw ? wkey[w] : KEY_MAX;
+            } else {
+              v = ldg64_pol(lv + s, pf);
             }
             if (v != KEY_MAX) {
               ok[c] = k;
@@ -533,10 +576,11 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
     // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
     const int iblocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 4u);
     query_iterwarp_kernel<<<iblocks < 1 ? 1 : iblocks, 256, 0, st>>>(
-        c.qkey, c.wkey, c.wparent, QueryIO{c.qseg, c.wseg, c.wop, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
+        c.qkey, c.wkey, c.wparent,
+        QueryIO{c.qseg, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
         A, t, ctl, iter_rgs, (flags & EIRENE_F_STATS) ? 1u : 0u);
   } else {
-    query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wleaf, c.wslot, c.wparent, c.old,
+    query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.wparent, c.old,
                                          spay, c.pinfo, c.istart, c.longseg, A, t, ctl);
   }
   ++*launches;
@@ -546,26 +590,16 @@ void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const uin
                   BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
-  range_kernel<<<blocks, 256, 0, st>>>(n, c.wkey, c.wseg, spay, c.pinfo, c.istart, kB, A, t, ctl);
+  range_kernel<<<blocks, 256, 0, st>>>(n, c.wkey, c.wseg, spay, c.pinfo, c.istart, kB, c.old, A, t, ctl);
   ++*launches;
 }
 
-static int num_long_ctas() {
-  static int n = 0;
-  if (!n) {
-    int dev = 0, sms = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    n = 2 * sms;
-  }
-  return n;
-}
-
 void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const CombBufs& c, const BatchArgs* A,
-                   BatchCtl* ctl,
-                   const TreeHdr* hdr, int dbgprint, cudaStream_t st, int* launches) {
-  (void)n;
-  result_long_kernel<<<num_long_ctas(), 1024, 0, st>>>(spay, kB, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr,
+                   BatchCtl* ctl, const TreeHdr* hdr, int dbgprint, int num_sms, cudaStream_t st, int* launches) {
+  // one 1024-thread CTA per SM: enough for the long segments of a Zipf batch
+  // (RCHUNK work items), cheap when there are none
+  const uint32_t grid = std::max(1u, std::min<uint32_t>((uint32_t)num_sms, (n + 1023) / 1024));
+  result_long_kernel<<<grid, 1024, 0, st>>>(spay, kB, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr,
                                                        dbgprint);
   ++*launches;
 }

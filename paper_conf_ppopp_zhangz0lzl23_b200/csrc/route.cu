@@ -186,11 +186,11 @@ void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint
                             const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
                             uint32_t* perm, uint32_t* counts, uint32_t* invalid, unsigned long long* lookback,
                             uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st, int* launches) {
-  static bool attr = false;
-  if (!attr) {
-    cudaFuncSetAttribute(route_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(RtSmem));
-    attr = true;
-  }
+  static int attr[MAX_DEVICES];
+  per_device(attr, [] {
+    return (int)cudaFuncSetAttribute(route_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sizeof(RtSmem));
+  });
   cudaMemsetAsync(counts, 0, sizeof(uint32_t) * P, st);
   cudaMemsetAsync(tile_ctr, 0, sizeof(uint32_t), st);
   if (n == 0) return;

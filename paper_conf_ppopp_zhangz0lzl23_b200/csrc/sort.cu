@@ -238,11 +238,11 @@ size_t sort_lookback_words(uint32_t max_n) {
 void launch_sort(const uint64_t* keys, const uint8_t* ops, const uint32_t* pay_in, const uint64_t* vals, uint32_t n,
                  uint64_t key_lo, uint64_t key_hi, const SortBufs& b, BatchCtl* ctl, uint32_t epoch_base,
                  cudaStream_t st, int* launches, uint64_t** kout, uint32_t** pout) {
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaFuncSetAttribute(sort_pass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(PassSmem));
-    attr_set = true;
-  }
+  static int attr[MAX_DEVICES];
+  per_device(attr, [] {
+    return (int)cudaFuncSetAttribute(sort_pass_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sizeof(PassSmem));
+  });
   const uint32_t tiles = (n + SORT_TILE - 1) / SORT_TILE;
   int up_blocks = (int)std::min<uint32_t>((n + SORT_THREADS * 8 - 1) / (SORT_THREADS * 8), 148u * 4u);
   if (up_blocks < 1) up_blocks = 1;

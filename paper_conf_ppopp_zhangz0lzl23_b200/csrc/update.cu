@@ -1052,6 +1052,10 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
 __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
   const BatchCtl* ctl = C.ctl;
   if (ctl->invalid || ctl->status != 0) return;   // (uniform: every CTA leaves, no barrier is reached)
+  // every issued write a value overwrite of a present key: all of them were
+  // applied in place by the query kernel's locate (query.cu, retire), nothing
+  // structural is left (uniform)
+  if (ctl->nins == 0 && ctl->ndelp == 0) return;
   if (g_uprof && blockIdx.x == 0 && threadIdx.x == 0) C.ctl->uprof[0] = gtime_ns();
   const uint32_t nw = ctl->nw;
   const int lane = lane_id();
@@ -1230,21 +1234,22 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
   const uint32_t warps_needed = C.regroup ? (n + 31) / 32 : n;
   uint32_t blocks = (warps_needed + 3) / 4;
   // the level-synchronous phases need every CTA resident (grid barriers)
-  static int per_sm = -1;
-  if (per_sm < 0 && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, update_kernel, 128, 0) != cudaSuccess)
-    per_sm = 0;
+  static int occ[MAX_DEVICES];
+  const int per_sm = per_device(occ, [] {
+    int v = 0;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, update_kernel, 128, 0) == cudaSuccess ? v : 0;
+  });
   const uint32_t resident = (uint32_t)num_sms * (uint32_t)std::max(per_sm, 0);
   blocks = std::min<uint32_t>(blocks, resident ? resident : (uint32_t)num_sms * 4u);
   if (blocks < 1) blocks = 1;
   static const bool no_lsync = std::getenv("EIRENE_NO_LSYNC") != nullptr;   // A/B: per-warp insertion only
   if (!resident || no_lsync) C.slots[0] = nullptr;   // no residency guarantee: per-warp insertion only
   static const char* serial = std::getenv("EIRENE_UPDATE_SERIAL");   // debug: one warp, no concurrency
-  static bool prof_set = false;
-  if (!prof_set) {
+  static int prof_set[MAX_DEVICES];
+  per_device(prof_set, [] {
     const int on = std::getenv("EIRENE_UPDATE_PROF") != nullptr;
-    cudaMemcpyToSymbol(g_uprof, &on, sizeof(int));
-    prof_set = true;
-  }
+    return (int)cudaMemcpyToSymbol(g_uprof, &on, sizeof(int));
+  });
   if (serial) {
     update_kernel<<<1, 32, 0, st>>>(C);
   } else {

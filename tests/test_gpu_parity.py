@@ -462,3 +462,84 @@ def test_edge_batches(dev):
     run_and_compare(t, ref, np.full(n, 2, np.uint8), d, vs, dev)
     assert t.check_invariants()[0] == 0
     t.close()
+
+
+def test_efull_rejects_batch_untouched(dev):
+    """Pool headroom: a batch whose worst case (every issued write
+    an insert that splits) exceeds the leaf pool is rejected with EFULL before any
+    kernel modifies the tree; the tree then still serves batches that fit."""
+    from paper_conf_ppopp_zhangz0lzl23_b200._ffi import EIRENE_EFULL
+    rng = np.random.default_rng(21)
+    nb = 4096
+    # leaf_cap = max_keys / 8 + 2 * max_batch + 1024 = 9728 leaves (api.cu); one key per leaf
+    keys = np.arange(1, 9001, dtype=np.uint64) * np.uint64(1 << 20)
+    vals = rng.integers(0, 1 << 62, keys.size, dtype=np.uint64)
+    t = make_tree(dev, keys, vals, max_keys=4096, max_batch=nb, fill=1.0 / 16)
+    assert t.info()["leaves"] == 9000
+    ref = oracle.MapOracle(); ref.load(keys, vals)
+    ops = np.full(nb, 2, np.uint8)
+    ks = keys[:nb] + np.uint64(1)           # 4096 distinct fresh keys: 9000 + 4096 > 9728
+    vs = rng.integers(0, 1 << 62, nb, dtype=np.uint64)
+    res = torch.empty(nb, dtype=torch.uint64, device=dev)
+    st = t.results(t.submit(T(ops, dev), T(ks, dev), T(vs, dev), res), raise_on_error=False)
+    assert st["rc"] == EIRENE_EFULL and st["status"] == EIRENE_EFULL
+    k, v = t.scan()
+    assert np.array_equal(k.cpu().numpy(), keys) and np.array_equal(v.cpu().numpy(), vals)
+    assert t.check_invariants() == (0, keys.size)
+    # a batch within the headroom goes through (mixed, 500 fresh inserts)
+    ops2 = rng.integers(0, 4, nb).astype(np.uint8)
+    ks2 = np.where(np.arange(nb) < 500, ks, keys[rng.integers(0, keys.size, nb)]).astype(np.uint64)
+    run_and_compare(t, ref, ops2, ks2, vs, dev)
+    t.close()
+
+
+@pytest.mark.parametrize("zipf", [False, True])
+def test_two_kernel_sort_size_band(dev, zipf):
+    """Batches above the fused distribution kernel's capacity (one resident
+    wave, ~1.2M requests) but at most 2^22 take the two-kernel path with its
+    own 16384-bin buffers (bsort_fused decides for the launcher, the group
+    count and the buffers alike) -- the per-shard batch of cfg5 at N = 4 / 8."""
+    from paper_conf_ppopp_zhangz0lzl23_b200 import workload as W
+    n = (1 << 21) + 123
+    w = W.Workload(3 if zipf else 2, tree=1 << 20, batch=n)
+    t = make_tree(dev, w.keys, w.vals, max_keys=1 << 22, max_batch=n)
+    ref = oracle.MapOracle(); ref.load(w.keys, w.vals)
+    for b in range(2):
+        ops, keys, vals = w.batch_arrays(b)
+        run_and_compare(t, ref, ops, keys, vals, dev, check_scan=(b == 1))
+    t.close()
+
+
+def test_structural_counts_and_device_time(dev):
+    """nins / ndelp (the structural writes the update kernel is left with; value
+    overwrites are applied in place by the query kernel) equal their definition
+    on the oracle's pre-batch state, and the device batch time is recorded."""
+    rng = np.random.default_rng(5)
+    keys, vals = _rand_keys(rng, 20000)
+    t = make_tree(dev, keys, vals, max_batch=1 << 15)
+    ref = oracle.MapOracle(); ref.load(keys, vals)
+    for b in range(3):
+        n = 1 << 15
+        ops = rng.integers(0, 4, n).astype(np.uint8)
+        if b == 2:
+            ops[ops >= 2] = 1               # overwrites only: the update kernel has nothing left
+        ks = np.where(rng.random(n) < 0.6, keys[rng.integers(0, keys.size, n)],
+                      rng.integers(1, 1 << 40, n, dtype=np.uint64)).astype(np.uint64)
+        vs = rng.integers(0, 1 << 62, n, dtype=np.uint64)
+        pre_k, _ = ref.scan()
+        if b == 2:   # every write on a live key
+            ks[ops == 1] = pre_k[rng.integers(0, pre_k.size, int(np.sum(ops == 1)))]
+        # issued write per key = its last write; structural iff insert of absent / delete of present
+        last = {}
+        for o, k in zip(ops, ks):
+            if o != 0:
+                last[int(k)] = int(o)
+        present = set(int(x) for x in pre_k)
+        want_ins = sum(1 for k, o in last.items() if o != 3 and k not in present)
+        want_delp = sum(1 for k, o in last.items() if o == 3 and k in present)
+        st = run_and_compare(t, ref, ops, ks, vs, dev)
+        assert (st["nins"], st["ndelp"]) == (want_ins, want_delp)
+        if b == 2:
+            assert want_ins == 0 and want_delp == 0
+        assert 0 < st["device_ns"] < 10**9
+    t.close()
