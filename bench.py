@@ -409,6 +409,10 @@ def run_ours(args):
     dev_batch_ms = np.array(dns, dtype=np.float64) / 1e6 if dns and all(x > 0 for x in dns) else None
     if os.environ.get("EIRENE_BENCH_VERBOSE") and dev_batch_ms is not None:
         print("device batch ms:", " ".join(f"{x:.3f}" for x in dev_batch_ms), file=sys.stderr)
+        tb = [s.get("t_begin_ns", 0) for s in stats[args.warmup:]]
+        te = [s.get("t_end_ns", 0) for s in stats[args.warmup:]]
+        print("device gap us:", " ".join(f"{(tb[i + 1] - te[i]) / 1e3:.1f}" for i in range(len(tb) - 1)),
+              file=sys.stderr)
     if world > 1:
         tmax = torch.tensor([elapsed_ms], device=dev)
         dist.all_reduce(tmax, op=dist.ReduceOp.MAX)

@@ -122,6 +122,7 @@ typedef struct {
                                  the batch's first kernel to the end of its last one (ns); the
                                  paper's per-batch time without host
                                  launch jitter                                                  */
+  uint64_t t_begin_ns, t_end_ns;   /* the two %globaltimer stamps of device_ns (gaps between batches) */
   uint64_t nins, ndelp;       /* issued inserts of absent keys / deletes of present keys: the
                                  structural writes left to the update kernel (value overwrites
                                  of present keys are applied in place by the query kernel)      */
@@ -278,6 +279,35 @@ int eirene_route_partition(eirene_handle h, const uint8_t* ops_dev, const uint64
                            int P, uint8_t* send_ops_dev, uint64_t* send_keys_dev,
                            uint64_t* send_vals_dev, uint32_t* perm_dev, uint32_t* counts_dev,
                            uint32_t* invalid_dev, eirene_stream_t stream);
+
+/* The same partition for ONE payload exchange: each request becomes a 24 B
+ * record {key, value, op} (three u64 words) in send_rec_dev[3n], grouped by
+ * destination in timestamp order; perm_dev[n] as above; counts2_dev[2P] (u32)
+ * holds, per destination d, counts2[2d] = requests for shard d and
+ * counts2[2d+1] = 1 if ANY request of this slice is invalid (the validation
+ * of eirene_submit_batch, always on), else 0 -- so a single all-to-all of
+ * [P][2] words gives every rank the receive counts and every rank's validity
+ * flag (the whole global batch is rejected if one is set; SURVEY §8(b),
+ * §8(e)).  `h` provides scratch only.  Asynchronous on `stream`. */
+int eirene_route_partition_packed(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev,
+                                  const uint64_t* vals_dev, uint32_t n, const uint64_t* splitters_dev,
+                                  int P, uint64_t* send_rec_dev, uint32_t* perm_dev, uint32_t* counts2_dev,
+                                  eirene_stream_t stream);
+
+/* Receiver side of the packed exchange: splits n records recv_rec_dev[3n]
+ * (the source ranks' segments concatenated in rank order = timestamp order)
+ * into ops_out_dev[n], keys_out_dev[n], vals_out_dev[n] for
+ * eirene_submit_batch.  Asynchronous on `stream`. */
+int eirene_route_unpack(eirene_handle h, const uint64_t* recv_rec_dev, uint32_t n, uint8_t* ops_out_dev,
+                        uint64_t* keys_out_dev, uint64_t* vals_out_dev, eirene_stream_t stream);
+
+/* Enqueues on `stream` a copy of batch `ticket`'s final status (the value
+ * eirene_results would return) into status_dev (one int32 in device memory),
+ * without a host synchronisation: the multi-GPU layer all-reduces it so that
+ * every rank agrees on the global batch's outcome (EFULL / EINTERNAL on one
+ * shard fails the batch everywhere).  `stream` must be ordered after the
+ * batch's stream.  ESTATE for an unknown or too old ticket. */
+int eirene_batch_status_async(eirene_handle h, uint64_t ticket, int32_t* status_dev, eirene_stream_t stream);
 
 /* Inverse of the partition for the returned results:
  * results_dev[perm_dev[j]] = recv_results_dev[j] for j < n.  Asynchronous. */

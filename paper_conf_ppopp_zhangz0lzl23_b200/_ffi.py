@@ -41,7 +41,7 @@ class eirene_batch_stats(ctypes.Structure):
                 ("leaf_splits", _u64), ("inner_splits", _u64), ("new_leaves", _u64), ("new_inner", _u64),
                 ("height", _u32), ("launches", _u32), ("stage_ms", ctypes.c_float * 8),
                 ("ranges", _u64), ("artificial", _u64), ("trav_steps", _u64), ("rg_vertical", _u64),
-                ("rg_horizontal", _u64), ("device_ns", _u64), ("nins", _u64), ("ndelp", _u64)]
+                ("rg_horizontal", _u64), ("device_ns", _u64), ("t_begin_ns", _u64), ("t_end_ns", _u64), ("nins", _u64), ("ndelp", _u64)]
 
     def to_dict(self) -> dict:
         d = {f: getattr(self, f) for f, _ in self._fields_ if f != "stage_ms"}
@@ -73,6 +73,9 @@ _SIGS = {
     "eirene_last_cuda_error": (ctypes.c_char_p, []),
     "eirene_route_partition": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _int, _vp, _vp, _vp, _vp, _vp, _vp, _vp]),
     "eirene_route_unpermute": (_int, [_vp, _vp, _vp, _u32, _vp, _vp]),
+    "eirene_route_partition_packed": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _int, _vp, _vp, _vp, _vp]),
+    "eirene_route_unpack": (_int, [_vp, _vp, _u32, _vp, _vp, _vp, _vp]),
+    "eirene_batch_status_async": (_int, [_vp, _u64, _vp, _vp]),
 }
 
 _lib = None

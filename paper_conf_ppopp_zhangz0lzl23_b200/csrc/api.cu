@@ -305,7 +305,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->comp_ev[s], cudaEventDisableTiming);
   }
   AL(h->route_lb, ((nb + 2047) / 2048) * 64);
-  AL(h->route_ctr, 1);
+  AL(h->route_ctr, 2);   // [0] scatter tile counter, [1] validity flag of the packed partition
   AL(h->bs.gstart, NBINS_MAX + 1);
   AL(h->bs.bin2grp, NBINS_MAX);
   AL(h->dargs, 1);
@@ -661,6 +661,8 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) 
     stats->rg_vertical = c.rg_vertical;
     stats->rg_horizontal = c.rg_horizontal;
     stats->device_ns = c.t_end > c.t_begin ? c.t_end - c.t_begin : 0;
+    stats->t_begin_ns = c.t_begin;
+    stats->t_end_ns = c.t_end;
     stats->nins = c.nins;
     stats->ndelp = c.ndelp;
     if (r.timing) {
@@ -814,10 +816,54 @@ int eirene_route_partition(eirene_handle h, const uint8_t* ops, const uint64_t* 
   DeviceGuard dg_(h->cfg.device);
   CK(dg_.err);
   int launches = 0;
-  launch_route_partition(ops, keys, vals, n, splitters, P, sops, skeys, svals, perm, counts, invalid, h->route_lb,
-                         h->route_ctr, ++h->route_epoch, reinterpret_cast<cudaStream_t>(stream), &launches);
+  launch_route_partition(ops, keys, vals, n, splitters, P, sops, skeys, svals, nullptr, perm, counts, 1, invalid,
+                         h->route_lb, h->route_ctr, ++h->route_epoch, reinterpret_cast<cudaStream_t>(stream),
+                         &launches);
   h->launches += launches;
   CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+int eirene_route_partition_packed(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
+                                  uint32_t n, const uint64_t* splitters, int P, uint64_t* send_rec, uint32_t* perm,
+                                  uint32_t* counts2, eirene_stream_t stream) {
+  if (!h || P < 1 || P > 64 || !counts2) return EIRENE_EINVAL;
+  if (n > h->cfg.max_batch) return EIRENE_EINVAL;
+  if (n > 0 && (!ops || !keys || !vals || !send_rec || !perm)) return EIRENE_EINVAL;
+  if (P > 1 && !splitters) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  int launches = 0;
+  CK(cudaMemsetAsync(h->route_ctr + 1, 0, sizeof(uint32_t), st));
+  launch_route_partition(ops, keys, vals, n, splitters, P, nullptr, nullptr, nullptr, send_rec, perm, counts2, 2,
+                         h->route_ctr + 1, h->route_lb, h->route_ctr, ++h->route_epoch, st, &launches);
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+int eirene_route_unpack(eirene_handle h, const uint64_t* recv_rec, uint32_t n, uint8_t* ops_out, uint64_t* keys_out,
+                        uint64_t* vals_out, eirene_stream_t stream) {
+  if (!h) return EIRENE_EINVAL;
+  if (n > 0 && (!recv_rec || !ops_out || !keys_out || !vals_out)) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  int launches = 0;
+  launch_route_unpack(recv_rec, n, ops_out, keys_out, vals_out, reinterpret_cast<cudaStream_t>(stream), &launches);
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+int eirene_batch_status_async(eirene_handle h, uint64_t ticket, int32_t* status_dev, eirene_stream_t stream) {
+  if (!h || !status_dev) return EIRENE_EINVAL;
+  const Rec& r = h->ring[ticket % RING];
+  if (!r.used || r.ticket != ticket) return EIRENE_ESTATE;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  CK(cudaMemcpyAsync(status_dev, &h->ctl_ring[ticket % RING].status, sizeof(int32_t), cudaMemcpyDeviceToDevice,
+                     reinterpret_cast<cudaStream_t>(stream)));
   return EIRENE_OK;
 }
 

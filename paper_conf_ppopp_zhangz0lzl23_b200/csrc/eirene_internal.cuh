@@ -372,10 +372,15 @@ int scan_tree(Tree t, uint32_t leaf_count, uint64_t lo, uint64_t hi, uint64_t* k
               uint64_t cap, uint64_t* count, cudaStream_t st, int* launches);
 
 // routing
+// SoA outputs (sops/skeys/svals, counts[P]) or, with rec != null, 24 B records
+// {key, value, op} and counts[2P] = (count, validity flag) per destination
 void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                             const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
-                            uint32_t* perm, uint32_t* counts, uint32_t* invalid, unsigned long long* lookback,
-                            uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st, int* launches);
+                            uint64_t* rec, uint32_t* perm, uint32_t* counts, uint32_t cstride, uint32_t* invalid,
+                            unsigned long long* lookback, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st,
+                            int* launches);
+void launch_route_unpack(const uint64_t* rec, uint32_t n, uint8_t* ops, uint64_t* keys, uint64_t* vals,
+                         cudaStream_t st, int* launches);
 void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,
                             cudaStream_t st, int* launches);
 

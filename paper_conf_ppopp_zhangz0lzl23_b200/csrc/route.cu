@@ -32,7 +32,7 @@ __global__ void __launch_bounds__(RT_THREADS) route_count_kernel(const uint64_t*
                                                                  const uint8_t* __restrict__ ops,
                                                                  const uint64_t* __restrict__ vals, uint32_t n,
                                                                  const uint64_t* __restrict__ splitters, int P,
-                                                                 uint32_t* __restrict__ counts,
+                                                                 uint32_t* __restrict__ counts, uint32_t cstride,
                                                                  uint32_t* __restrict__ invalid) {
   __shared__ uint64_t sp[RT_MAXP];
   __shared__ uint32_t h[RT_MAXP];
@@ -54,7 +54,7 @@ __global__ void __launch_bounds__(RT_THREADS) route_count_kernel(const uint64_t*
   }
   if (__any_sync(FULL, bad) && (tid & 31) == 0) atomicOr(invalid, 1u);
   __syncthreads();
-  if (tid < P && h[tid]) atomicAdd(&counts[tid], h[tid]);
+  if (tid < P && h[tid]) atomicAdd(&counts[tid * cstride], h[tid]);
 }
 
 struct RtSmem {
@@ -73,8 +73,9 @@ struct RtSmem {
 
 __global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
     const uint8_t* __restrict__ ops, const uint64_t* __restrict__ keys, const uint64_t* __restrict__ vals, uint32_t n,
-    const uint64_t* __restrict__ splitters, int P, const uint32_t* __restrict__ counts, uint8_t* __restrict__ sops,
-    uint64_t* __restrict__ skeys, uint64_t* __restrict__ svals, uint32_t* __restrict__ perm,
+    const uint64_t* __restrict__ splitters, int P, uint32_t* __restrict__ counts, uint32_t cstride,
+    const uint32_t* __restrict__ invalid, uint8_t* __restrict__ sops, uint64_t* __restrict__ skeys,
+    uint64_t* __restrict__ svals, uint64_t* __restrict__ rec, uint32_t* __restrict__ perm,
     unsigned long long* __restrict__ lookback, uint32_t epoch, uint32_t* __restrict__ tile_ctr) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   RtSmem& S = *reinterpret_cast<RtSmem*>(smem_raw);
@@ -84,13 +85,18 @@ __global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
     uint32_t run = 0;
     for (int d = 0; d < P; ++d) {
       S.bin_start[d] = run;
-      run += counts[d];
+      run += counts[d * cstride];
     }
   }
   for (int i = tid; i < RT_WARPS * RT_MAXP; i += RT_THREADS) (&S.wh[0][0])[i] = 0;
   if (tid < RT_MAXP) S.sp[tid] = tid < P - 1 ? splitters[tid] : KEY_MAX;
   __syncthreads();
   const uint32_t tile = S.tile_id, base = tile * RT_TILE;
+  // packed mode: every destination's count word is followed by the batch's
+  // validity flag (final: route_count_kernel ran before this kernel), so ONE
+  // exchange of [P][2] words tells every rank the counts and whether the
+  // global batch is rejected
+  if (cstride == 2 && tile == 0 && tid < P) counts[2 * tid + 1] = invalid ? *invalid : 0u;
   const uint32_t wbase = base + warp * (RT_ITEMS * 32);
   uint64_t k[RT_ITEMS];
   uint32_t d[RT_ITEMS], r[RT_ITEMS];
@@ -168,9 +174,15 @@ __global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
   for (uint32_t i = tid; i < tile_n; i += RT_THREADS) {
     const uint64_t key = S.keys[i];
     const uint32_t o = S.bin_base[dest_of(key, S.sp, P)] + i;
-    skeys[o] = key;
-    svals[o] = S.vals[i];
-    sops[o] = S.ops[i];
+    if (rec) {   // one 24 B record {key, value, op} per request: one payload exchange
+      rec[3 * (size_t)o] = key;
+      rec[3 * (size_t)o + 1] = S.vals[i];
+      rec[3 * (size_t)o + 2] = S.ops[i];
+    } else {
+      skeys[o] = key;
+      svals[o] = S.vals[i];
+      sops[o] = S.ops[i];
+    }
     perm[o] = S.idx[i];
   }
 }
@@ -180,25 +192,44 @@ __global__ void unpermute_kernel(const uint64_t* __restrict__ recv, const uint32
   for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) out[perm[j]] = recv[j];
 }
 
+__global__ void unpack_kernel(const uint64_t* __restrict__ rec, uint32_t n, uint8_t* __restrict__ ops,
+                              uint64_t* __restrict__ keys, uint64_t* __restrict__ vals) {
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < n; j += gridDim.x * blockDim.x) {
+    keys[j] = rec[3 * (size_t)j];
+    vals[j] = rec[3 * (size_t)j + 1];
+    ops[j] = (uint8_t)rec[3 * (size_t)j + 2];
+  }
+}
+
 }  // namespace
+
+void launch_route_unpack(const uint64_t* rec, uint32_t n, uint8_t* ops, uint64_t* keys, uint64_t* vals,
+                         cudaStream_t st, int* launches) {
+  if (n == 0) return;
+  int blocks = (int)std::min<uint32_t>((n + 255) / 256, 148u * 8u);
+  unpack_kernel<<<blocks, 256, 0, st>>>(rec, n, ops, keys, vals);
+  ++*launches;
+}
 
 void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                             const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
-                            uint32_t* perm, uint32_t* counts, uint32_t* invalid, unsigned long long* lookback,
-                            uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st, int* launches) {
+                            uint64_t* rec, uint32_t* perm, uint32_t* counts, uint32_t cstride, uint32_t* invalid,
+                            unsigned long long* lookback, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st,
+                            int* launches) {
   static int attr[MAX_DEVICES];
   per_device(attr, [] {
     return (int)cudaFuncSetAttribute(route_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                      (int)sizeof(RtSmem));
   });
-  cudaMemsetAsync(counts, 0, sizeof(uint32_t) * P, st);
+  cudaMemsetAsync(counts, 0, sizeof(uint32_t) * P * cstride, st);
   cudaMemsetAsync(tile_ctr, 0, sizeof(uint32_t), st);
   if (n == 0) return;
   int blocks = (int)std::min<uint32_t>((n + RT_THREADS * 8 - 1) / (RT_THREADS * 8), 148u * 4u);
-  route_count_kernel<<<blocks, RT_THREADS, 0, st>>>(keys, ops, vals, n, splitters, P, counts, invalid);
+  route_count_kernel<<<blocks, RT_THREADS, 0, st>>>(keys, ops, vals, n, splitters, P, counts, cstride, invalid);
   const uint32_t tiles = (n + RT_TILE - 1) / RT_TILE;
-  route_scatter_kernel<<<tiles, RT_THREADS, sizeof(RtSmem), st>>>(ops, keys, vals, n, splitters, P, counts, sops,
-                                                                  skeys, svals, perm, lookback, epoch, tile_ctr);
+  route_scatter_kernel<<<tiles, RT_THREADS, sizeof(RtSmem), st>>>(ops, keys, vals, n, splitters, P, counts, cstride,
+                                                                  invalid, sops, skeys, svals, rec, perm, lookback,
+                                                                  epoch, tile_ctr);
   *launches += 2;
 }
 

@@ -6,14 +6,21 @@ the splitters being equal-count quantiles of the bulk-loaded keys -- and each
 batch needs one exchange step each way:
 
   1. every rank holds the contiguous timestamp slice r of the global batch;
-  2. route_partition (CUDA kernel) stably groups the slice by destination
-     shard (dest = upper_bound(splitters, key)) and counts per destination;
-  3. all_to_all_single on the counts, an all_reduce of the validity flag;
-  4. all_to_all_single on the payload (NCCL over NVLink 5 / NVSwitch);
+  2. route_partition_packed (CUDA kernels) stably groups the slice by
+     destination shard (dest = upper_bound(splitters, key)) into 24 B
+     {key, value, op} records and counts per destination;
+  3. ONE all_to_all_single of (count, validity flag) per destination: the
+     receive counts, and every rank's flag (a bad request anywhere rejects the
+     global batch everywhere, before any shard applies) -- the one host sync;
+  4. ONE all_to_all_single of the records (NCCL over NVLink 5 / NVSwitch),
+     route_unpack on the receiver;
      the receiver's concatenation in source-rank order is timestamp-ordered,
      so the shard's stable (key, ts) sort keeps linearizability (per-key
      locality of linearizability, Herlihy & Wing [17], P:2487-2492);
-  5. the shard runs the single-GPU hot path (eirene_submit_batch);
+  5. the shard runs the single-GPU hot path (eirene_submit_batch); its final
+     status is copied on the device and all-reduced (MIN), so an EFULL /
+     EINTERNAL on one shard fails the global batch on every rank and no rank
+     raises alone while the others wait in a collective;
   6. all_to_all_single returns the results; route_unpermute (CUDA kernel)
      puts them back in the slice's timestamp order.
 
@@ -75,49 +82,99 @@ class ShardedEirene:
         if my_k.size:
             self.engine.bulk_load(torch.from_numpy(my_k).to(self.device), torch.from_numpy(my_v).to(self.device))
         self.splitters = torch.from_numpy(self.splitters_np if self.world > 1 else np.zeros(1, np.uint64)).to(self.device)
-        self.flag = torch.zeros(1, dtype=torch.int32, device=self.device)
 
-    def apply(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor) -> dict:
-        """Process this rank's timestamp slice of a global batch; results in slice order."""
+    def submit(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor) -> "ShardedTicket":
+        """Process this rank's timestamp slice of a global batch; `results` (slice order) is valid once the
+        returned ticket's results() returns.  Collective: every rank calls it for every global batch in the
+        same order.  ONE host synchronisation per batch (the receive counts the payload exchange needs);
+        everything else is stream-ordered on the current stream:
+
+          route_partition_packed -> all_to_all(counts + validity flags) -> [host: counts]
+          -> all_to_all(24 B records) -> route_unpack -> submit (shard's hot path)
+          -> status copy + all_reduce(MIN) -> all_to_all(results) -> route_unpermute
+        """
         P = self.world
-        sops, skeys, svals, perm, counts = self.router.route_partition(ops, keys, vals, self.splitters, P,
-                                                                      invalid=self.flag)
-        recv_counts = torch.empty_like(counts)
+        n = int(ops.numel())
+        rec, perm, cnt2 = self.router.route_partition_packed(ops, keys, vals, self.splitters, P)
+        recv2 = torch.empty_like(cnt2)
         if P > 1:
-            dist.all_to_all_single(recv_counts, counts, group=self.group)
-            dist.all_reduce(self.flag, op=dist.ReduceOp.MAX, group=self.group)
+            dist.all_to_all_single(recv2, cnt2, group=self.group)
         else:
-            recv_counts.copy_(counts)
-        sc = counts.cpu().tolist()
-        rc = recv_counts.cpu().tolist()
-        invalid = int(self.flag.item())
-        self.flag.zero_()
+            recv2.copy_(cnt2)
+        both = torch.cat([cnt2, recv2]).cpu().numpy().astype(np.int64)   # the one host sync
+        sc = both[0:2 * P:2].tolist()
+        rcv = both[2 * P::2].tolist()
+        invalid = int(both[2 * P + 1::2].max())   # every rank's flag: all ranks agree
         if invalid:
-            return {"rc": -1, "status": -1, "n": int(ops.numel()), "launches": 0, "stage_ms": [0.0] * 8}
-        nrecv = int(sum(rc))
+            return ShardedTicket(self, None, None, n, rejected=-1)
+        nrecv = int(sum(rcv))
         dev = self.device
-        rops = torch.empty(nrecv, dtype=torch.uint8, device=dev)
-        rkeys = torch.empty(nrecv, dtype=torch.uint64, device=dev)
-        rvals = torch.empty(nrecv, dtype=torch.uint64, device=dev)
+        rrec = torch.empty(3 * nrecv, dtype=torch.uint64, device=dev)
         if P > 1:
-            dist.all_to_all_single(_i64(rkeys), _i64(skeys), rc, sc, group=self.group)
-            dist.all_to_all_single(_i64(rvals), _i64(svals), rc, sc, group=self.group)
-            dist.all_to_all_single(rops, sops, rc, sc, group=self.group)
+            dist.all_to_all_single(_i64(rrec), _i64(rec), [3 * c for c in rcv], [3 * c for c in sc],
+                                   group=self.group)
         else:
-            rops.copy_(sops)
-            rkeys.copy_(skeys)
-            rvals.copy_(svals)
+            rrec.copy_(rec)
+        rops, rkeys, rvals = self.router.route_unpack(rrec, nrecv)
         rres = torch.empty(nrecv, dtype=torch.uint64, device=dev)
-        st = {"rc": 0, "status": 0, "n": nrecv, "launches": 0, "stage_ms": [0.0] * 8}
+        status = torch.zeros(1, dtype=torch.int32, device=dev)
+        tk = None
         if nrecv:
-            _, st = self.engine.apply(rops, rkeys, rvals, rres)
-        back = torch.empty(int(sum(sc)), dtype=torch.uint64, device=dev)
+            tk = self.engine.submit(rops, rkeys, rvals, rres)
+            self.engine.status_async(tk, status)
         if P > 1:
-            dist.all_to_all_single(_i64(back), _i64(rres), sc, rc, group=self.group)
+            # EFULL / EINTERNAL / CUDA failure on one shard fails the global batch on every rank
+            # (statuses are <= 0: the minimum is the error, if any) -- no rank raises alone
+            dist.all_reduce(status, op=dist.ReduceOp.MIN, group=self.group)
+        back = torch.empty(n, dtype=torch.uint64, device=dev)
+        if P > 1:
+            dist.all_to_all_single(_i64(back), _i64(rres), sc, rcv, group=self.group)
         else:
             back.copy_(rres)
         self.router.route_unpermute(back, perm, out=results)
-        return st
+        # the ticket keeps every buffer of the batch alive until its results are read
+        return ShardedTicket(self, tk, status, n, keep=(rec, perm, rrec, rops, rkeys, rvals, rres, back))
+
+    def apply(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor) -> dict:
+        """submit + results (synchronous convenience)."""
+        return self.submit(ops, keys, vals, results).results()
+
+    def submit_host(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor,
+                    results: torch.Tensor) -> "ShardedTicket":
+        """Host (pinned) slice buffers: H2D of the slice on the current stream, submit, D2H of the results;
+        results are valid once the ticket's results() returns."""
+        dev = self.device
+        d = [torch.empty(x.shape, dtype=x.dtype, device=dev) for x in (ops, keys, vals)]
+        for dst, src in zip(d, (ops, keys, vals)):
+            dst.copy_(src, non_blocking=True)
+        dres = torch.empty(results.shape, dtype=results.dtype, device=dev)
+        t = self.submit(*d, dres)
+        results.copy_(dres, non_blocking=True)
+        t.keep = (t.keep, d, dres)
+        return t
 
     def scan(self):
         return self.engine.scan()
+
+
+class ShardedTicket:
+    """A submitted global batch on this rank.  results() waits for the shard's batch and returns its stats
+    with the GLOBAL status (the minimum over every shard's status, already all-reduced on the device)."""
+
+    def __init__(self, sh: ShardedEirene, tk, status: torch.Tensor | None, n: int, keep=None,
+                 rejected: int | None = None):
+        self.sh, self.tk, self.status, self.n, self.keep = sh, tk, status, n, keep
+        self.fixed = rejected
+
+    def results(self) -> dict:
+        if self.fixed is not None:   # rejected before any shard applied anything (invalid request)
+            return {"rc": self.fixed, "status": self.fixed, "n": self.n, "launches": 0, "stage_ms": [0.0] * 8,
+                    "device_ns": 0}
+        st = {"rc": 0, "status": 0, "n": 0, "launches": 0, "stage_ms": [0.0] * 8, "device_ns": 0}
+        if self.tk is not None:
+            st = self.sh.engine.results(self.tk, raise_on_error=False)
+        g = int(self.status.item())
+        st["shard_status"] = st["status"]
+        st["rc"] = st["status"] = g
+        self.keep = None
+        return st

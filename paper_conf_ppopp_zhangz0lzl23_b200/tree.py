@@ -227,3 +227,33 @@ class EireneTree:
         check(self._L.eirene_route_unpermute(self._h, _ptr(recv), _ptr(perm), n, _ptr(out), self._stream(stream)),
               "eirene_route_unpermute")
         return out
+
+    def route_partition_packed(self, ops, keys, vals, splitters: torch.Tensor | None, P: int, stream=None):
+        """Partition for ONE payload exchange: returns (send_rec u64[3n] of {key, value, op} records grouped by
+        destination, perm int32[n], counts2 int32[2P] = (count, validity flag) per destination)."""
+        n = ops.numel()
+        dev = self.device
+        rec = torch.empty(3 * n, dtype=torch.uint64, device=dev)
+        perm = torch.empty(n, dtype=torch.int32, device=dev)
+        counts2 = torch.empty(2 * P, dtype=torch.int32, device=dev)
+        check(self._L.eirene_route_partition_packed(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n,
+                                                    _ptr(splitters) if splitters is not None else None, P,
+                                                    _ptr(rec), _ptr(perm), _ptr(counts2), self._stream(stream)),
+              "eirene_route_partition_packed")
+        return rec, perm, counts2
+
+    def route_unpack(self, rec: torch.Tensor, n: int, stream=None):
+        """Split n received {key, value, op} records into (ops u8, keys u64, vals u64)."""
+        dev = self.device
+        ops = torch.empty(n, dtype=torch.uint8, device=dev)
+        keys = torch.empty(n, dtype=torch.uint64, device=dev)
+        vals = torch.empty(n, dtype=torch.uint64, device=dev)
+        check(self._L.eirene_route_unpack(self._h, _ptr(rec), n, _ptr(ops), _ptr(keys), _ptr(vals),
+                                          self._stream(stream)), "eirene_route_unpack")
+        return ops, keys, vals
+
+    def status_async(self, ticket: int, out: torch.Tensor, stream=None):
+        """Enqueue a copy of batch `ticket`'s final status into out (int32[1] on the device), no host sync."""
+        check(self._L.eirene_batch_status_async(self._h, ticket, _ptr(out), self._stream(stream)),
+              "eirene_batch_status_async")
+        return out

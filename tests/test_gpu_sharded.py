@@ -23,7 +23,7 @@ def dev():
     return torch.device("cuda", 0)
 
 
-def run_sharded(dev, w, P, nb, per_rank):
+def run_sharded(dev, w, P, nb, per_rank, packed=False):
     from paper_conf_ppopp_zhangz0lzl23_b200.tree import EireneTree
     sp = splitters_for(w.keys, P)
     sp_t = torch.from_numpy(sp if P > 1 else np.zeros(1, np.uint64)).to(dev)
@@ -41,10 +41,17 @@ def run_sharded(dev, w, P, nb, per_rank):
         routed = []
         for r in range(P):     # every source rank partitions its ts-slice
             sl = slice(r * per_rank, (r + 1) * per_rank)
-            so, sk, sv, perm, cnt = trees[r].route_partition(torch.from_numpy(ops[sl].copy()).to(dev),
-                                                             torch.from_numpy(keys[sl].copy()).to(dev),
-                                                             torch.from_numpy(vals[sl].copy()).to(dev), sp_t, P)
-            c = cnt.cpu().numpy()
+            args = (torch.from_numpy(ops[sl].copy()).to(dev), torch.from_numpy(keys[sl].copy()).to(dev),
+                    torch.from_numpy(vals[sl].copy()).to(dev), sp_t, P)
+            if packed:   # 24 B records + (count, validity flag) per destination, unpacked after the "exchange"
+                rec, perm, cnt2 = trees[r].route_partition_packed(*args)
+                c2 = cnt2.cpu().numpy()
+                c = c2[0::2]
+                assert np.all(c2[1::2] == 0)
+                so, sk, sv = trees[r].route_unpack(rec, int(c.sum()))
+            else:
+                so, sk, sv, perm, cnt = trees[r].route_partition(*args)
+                c = cnt.cpu().numpy()
             off = np.concatenate([[0], np.cumsum(c)])
             routed.append((so, sk, sv, perm, off))
         back = [[None] * P for _ in range(P)]
@@ -71,8 +78,9 @@ def run_sharded(dev, w, P, nb, per_rank):
     return out, keys, vals
 
 
+@pytest.mark.parametrize("packed", [False, True])
 @pytest.mark.parametrize("cfg", [2, 3])
-def test_sharded_equals_oracle_for_every_P(dev, cfg):
+def test_sharded_equals_oracle_for_every_P(dev, cfg, packed):
     per_rank = 4096
     nb = 3
     results = {}
@@ -81,7 +89,7 @@ def test_sharded_equals_oracle_for_every_P(dev, cfg):
                        fracs={W.QUERY: 0.5, W.UPDATE: 0.3, W.INSERT: 0.15, W.DELETE: 0.05})
         ref = oracle.MapOracle()
         ref.load(w.keys, w.vals)
-        out, k, v = run_sharded(dev, w, P, nb, per_rank)
+        out, k, v = run_sharded(dev, w, P, nb, per_rank, packed)
         # replay the same batches on the oracle (a fresh generator: the batch
         # stream is a pure function of (cfg, seed, batch index))
         w2 = W.Workload(cfg, tree=1 << 16, batch=P * per_rank,
@@ -93,3 +101,35 @@ def test_sharded_equals_oracle_for_every_P(dev, cfg):
         rk, rv = ref.scan()
         assert np.array_equal(k, rk) and np.array_equal(v, rv), f"P={P}: final state differs"
         results[P] = out
+
+
+def test_packed_partition_flags_invalid_slice(dev):
+    """route_partition_packed: one invalid request in the slice sets the validity
+    word of every destination (so one exchange tells every rank), counts intact."""
+    from paper_conf_ppopp_zhangz0lzl23_b200.tree import EireneTree
+    t = EireneTree(max_keys=1 << 12, max_batch=1 << 12)
+    rng = np.random.default_rng(3)
+    n, P = 3000, 4
+    ops = rng.integers(0, 4, n).astype(np.uint8)
+    keys = rng.integers(1, 1 << 62, n, dtype=np.uint64)
+    vals = rng.integers(0, 1 << 62, n, dtype=np.uint64)
+    sp = np.sort(rng.integers(1, 1 << 62, P - 1, dtype=np.uint64))
+    sp_t = torch.from_numpy(sp).to(dev)
+    for bad in (False, True):
+        o = ops.copy()
+        if bad:
+            o[1234] = 9
+        rec, perm, cnt2 = t.route_partition_packed(torch.from_numpy(o).to(dev), torch.from_numpy(keys).to(dev),
+                                                   torch.from_numpy(vals).to(dev), sp_t, P)
+        c2 = cnt2.cpu().numpy()
+        dest = np.searchsorted(sp, keys, side="right")
+        assert np.array_equal(c2[0::2], np.bincount(dest, minlength=P))
+        assert np.all(c2[1::2] == (1 if bad else 0))
+        r = rec.cpu().numpy().reshape(n, 3)
+        pm = perm.cpu().numpy()
+        assert np.array_equal(r[:, 0], keys[pm]) and np.array_equal(r[:, 1], vals[pm])
+        assert np.array_equal(r[:, 2], o[pm].astype(np.uint64))
+        assert np.all(np.diff(dest[pm]) >= 0)                       # grouped by destination
+        for d in range(P):                                           # stable: timestamp order inside
+            assert np.all(np.diff(pm[dest[pm] == d]) > 0)
+    t.close()

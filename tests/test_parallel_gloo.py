@@ -37,6 +37,19 @@ class CpuRouter:
                 torch.from_numpy(v[order].copy()), torch.from_numpy(order.astype(np.int32)),
                 torch.from_numpy(counts))
 
+    def route_partition_packed(self, ops, keys, vals, splitters, P):
+        o, k, v, perm, counts = self.route_partition(ops, keys, vals, splitters, P)
+        bad = np.zeros(1, np.int32)
+        self.route_partition(ops, keys, vals, splitters, P, invalid=torch.from_numpy(bad))
+        rec = np.stack([k.numpy(), v.numpy(), o.numpy().astype(np.uint64)], axis=1).reshape(-1)
+        c2 = np.stack([counts.numpy(), np.full(P, bad[0], np.int32)], axis=1).reshape(-1)
+        return torch.from_numpy(rec.copy()), perm, torch.from_numpy(c2.astype(np.int32))
+
+    def route_unpack(self, rec, n):
+        r = rec.numpy().reshape(n, 3)
+        return (torch.from_numpy(r[:, 2].astype(np.uint8)), torch.from_numpy(r[:, 0].copy()),
+                torch.from_numpy(r[:, 1].copy()))
+
     def route_unpermute(self, back, perm, out=None):
         res = np.empty(back.numel(), np.uint64)
         res[perm.numpy()] = back.numpy()
@@ -60,6 +73,17 @@ class OracleEngine:
         r = self.m.apply(ops.numpy(), keys.numpy(), vals.numpy())
         results.copy_(torch.from_numpy(r))
         return results, {"rc": 0, "status": 0, "n": int(ops.numel()), "launches": 0, "stage_ms": [0.0] * 8}
+
+    def submit(self, ops, keys, vals, results):
+        self.apply(ops, keys, vals, results)
+        return 1
+
+    def status_async(self, tk, out):
+        out.fill_(0)
+        return out
+
+    def results(self, tk, raise_on_error=True):
+        return {"rc": 0, "status": 0, "n": 0, "launches": 0, "stage_ms": [0.0] * 8}
 
     def scan(self):
         k, v = self.m.scan()
