@@ -242,6 +242,32 @@ def run_reference(args):
     print(json.dumps(line), flush=True)
 
 
+def slice_parity(wl, got_batches, splitters, slice_keys: int) -> dict:
+    """Bit-exact check of the first global batches on key slices (see the caller)."""
+    import oracle
+    K, V = wl.keys, wl.vals
+    starts = [0, max(0, K.size - slice_keys)]
+    for s in splitters:
+        starts.append(int(np.clip(np.searchsorted(K, s) - slice_keys // 2, 0, max(0, K.size - slice_keys))))
+    starts = sorted(set(starts))
+    bad = checked = 0
+    for a in starts:
+        b = min(K.size, a + slice_keys)
+        lo = int(K[a]) if a > 0 else 0
+        hi = int(K[b]) if b < K.size else None
+        ref = oracle.MapOracle()
+        ref.load(K[a:b], V[a:b])
+        for bi, got in enumerate(got_batches):
+            o, k, v = wl.batch_arrays(bi)
+            m = (k >= np.uint64(lo)) & ((k < np.uint64(hi)) if hi is not None else True)
+            want = ref.apply(o[m], k[m], v[m])
+            bad += int(np.sum(got[m] != want))
+            checked += int(m.sum())
+    return {"batches_checked": len(got_batches), "requests_checked": checked, "mismatches": bad,
+            "vs": f"oracle (std::map) on {len(starts)} key slices of {slice_keys} loaded keys (one across every "
+                  f"shard boundary, both ends), every request of the slice, bit-exact"}
+
+
 def run_ours(args):
     import torch
     import torch.distributed as dist
@@ -267,7 +293,10 @@ def run_ours(args):
             dist.init_process_group(args.backend)
         from paper_conf_ppopp_zhangz0lzl23_b200.parallel import ShardedEirene
     cfg = args.config
-    C = W.CONFIGS[cfg]
+    C = dict(W.CONFIGS[cfg])
+    if args.mix:   # YCSB-like mix override (cfg5: A, B, C, U)
+        C["fracs"], C["dist"] = W.MIXES[args.mix]
+    wkw = {"fracs": C["fracs"], "dist": C["dist"]}
     tree_n, batch_n = C["tree"], C["batch"]
     if args.tree:
         tree_n = args.tree
@@ -305,7 +334,7 @@ def run_ours(args):
             if not per_tree:
                 return None
             ntr = (nsteps + per_tree - 1) // per_tree
-            wls_ = [W.Workload(cfg, tree=tree_n, batch=batch_n, seed=W.seed_for(cfg) + 7919 * (1000 * tag + t + 1))
+            wls_ = [W.Workload(cfg, tree=tree_n, batch=batch_n, seed=W.seed_for(cfg) + 7919 * (1000 * tag + t + 1), **wkw)
                     for t in range(ntr)]
             trees_ = []
             for w_ in wls_:
@@ -320,7 +349,7 @@ def run_ours(args):
             wls, trees, step_tree, host_batches = build_plan(0, nb)
             wl, tree = wls[0], trees[0]
         else:
-            wl = W.Workload(cfg, tree=tree_n, batch=batch_n)
+            wl = W.Workload(cfg, tree=tree_n, batch=batch_n, **wkw)
             keys_d = torch.from_numpy(wl.keys).to(dev)
             vals_d = torch.from_numpy(wl.vals).to(dev)
             tree = EireneTree(max_keys=max(tree_n * 2, 1 << 20), max_batch=batch_n, **qmode)
@@ -336,42 +365,50 @@ def run_ours(args):
     else:
         # weak scaling: the global tree holds world * tree_n keys, the global batch
         # world * batch_n requests; rank r owns key range r and ts-slice r
-        wl = W.Workload(cfg, tree=tree_n * world, batch=batch_n * world)
+        wl = W.Workload(cfg, tree=tree_n * world, batch=batch_n * world, **wkw)
         sh = ShardedEirene(wl.keys, wl.vals, max_batch=batch_n, device=dev)
+        for f_ in (0.97, 1.0, 1.03, 1.1):   # graph capture for the likely shard batch size buckets, untimed
+            sh.engine.prepare(min(int(batch_n * f_), batch_n * world))
         host_batches = []
         batches = []
+        sl = slice(rank * batch_n, (rank + 1) * batch_n)
         for b in range(nb):
             o, k, v = wl.batch_arrays(b)
-            sl = slice(rank * batch_n, (rank + 1) * batch_n)
-            host_batches.append((o[sl], k[sl], v[sl]))
-            batches.append(tuple(torch.from_numpy(np.ascontiguousarray(a[sl])).to(dev) for a in (o, k, v)))
+            host_batches.append(tuple(np.ascontiguousarray(a[sl]) for a in (o, k, v)))
+            batches.append(tuple(torch.from_numpy(a).to(dev) for a in host_batches[-1]))
         results = [torch.empty(batch_n, dtype=torch.uint64, device=dev) for _ in range(nb)]
     torch.cuda.synchronize()
     gen_s = time.time() - t_gen
 
     # ------------------------------------------------------------ device-timed run
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(nb)]
+    # per-batch host events between the batches (EIRENE_BENCH_NO_EVENTS=1: none; the device
+    # timestamps of every batch are in its stats either way)
+    host_ev = not os.environ.get("EIRENE_BENCH_NO_EVENTS")
     stats = []
     launches = 0
 
     def step(b, tr_list=None, st_tree=None, bt=None):
         nonlocal launches
         o, k, v = (bt or batches)[b]
-        ev[b][0].record(stream)
+        if host_ev:
+            ev[b][0].record(stream)
         if world == 1:
             tr = (tr_list or trees)[(st_tree or step_tree)[b]]
             if cap:
                 tk = tr.submit_range(o, k, v, results[b], cap, *rrows[b])
             else:
                 tk = tr.submit(o, k, v, results[b])
-            ev[b][1].record(stream)
+            if host_ev:
+                ev[b][1].record(stream)
             return (tr, tk)
-        st = sh.apply(o, k, v, results[b])
-        ev[b][1].record(stream)
-        return st
+        tk = sh.submit(o, k, v, results[b])
+        if host_ev:
+            ev[b][1].record(stream)
+        return tk
 
     def fetch(r):
-        return r[0].results(r[1]) if world == 1 else r
+        return r[0].results(r[1]) if world == 1 else r.results()
 
     for b in range(args.warmup):
         stats.append(fetch(step(b)))
@@ -399,7 +436,8 @@ def run_ours(args):
     for r in tickets:
         stats.append(fetch(r))
     elapsed_ms = t_start.elapsed_time(t_end)
-    per_batch_ms = np.array([ev[b][0].elapsed_time(ev[b][1]) for b in range(args.warmup, nb)])
+    per_batch_ms = (np.array([ev[b][0].elapsed_time(ev[b][1]) for b in range(args.warmup, nb)]) if host_ev
+                    else np.full(args.steps, elapsed_ms / args.steps))
     if os.environ.get("EIRENE_BENCH_VERBOSE"):
         print("per-batch ms:", " ".join(f"{x:.3f}" for x in per_batch_ms), file=sys.stderr)
         print("stage ms per batch:", [[round(x, 3) for x in s["stage_ms"][:5]] for s in stats[args.warmup:]][:8],
@@ -534,16 +572,65 @@ def run_ours(args):
                "steps": n_e, "path": "eirene_submit_batch_host (pinned host buffers; H2D of batch b+1 on the "
                                      "library's copy stream and D2H of batch b-1 on its d2h stream overlap "
                                      "batch b's kernels; upsert values read zero-copy)"}
-    elif world > 1:
-        e2e = {"value": None, "unit": "Greq/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0,
-               "note": "multi-GPU e2e not measured this round"}
+    elif world > 1 and args.e2e_steps > 0:
+        # through the public multi-GPU API with host buffers: every rank copies its
+        # pinned ts-slice in, ShardedEirene routes / applies / returns, the results
+        # slice is copied back; max over ranks of the device-timed region
+        e_hb = []
+        for i in range(args.e2e_steps):
+            o, k, v = wl.batch_arrays(nb + i)
+            e_hb.append(tuple(torch.from_numpy(np.ascontiguousarray(a[sl])).pin_memory() for a in (o, k, v)))
+        hres = [torch.empty(batch_n, dtype=torch.uint64).pin_memory() for _ in e_hb]
+        sh.submit_host(*e_hb[0], hres[0]).results()   # warm the path
+        torch.cuda.synchronize()
+        dist.barrier()
+        a = torch.cuda.Event(enable_timing=True)
+        z = torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        tks = [sh.submit_host(*e_hb[i], hres[i]) for i in range(1, len(e_hb))]
+        for t_ in tks:
+            t_.results()
+        z.record(stream)
+        torch.cuda.synchronize()
+        e_ms = torch.tensor([a.elapsed_time(z)], device=dev)
+        dist.all_reduce(e_ms, op=dist.ReduceOp.MAX)
+        n_e = len(e_hb) - 1
+        ups = np.mean([int(np.count_nonzero((x[0].numpy() == W.UPDATE) | (x[0].numpy() == W.INSERT))) for x in e_hb])
+        e2e = {"value": batch_n * world * n_e / (float(e_ms.item()) * 1e-3) / 1e9, "unit": "Greq/s",
+               "h2d_bytes_per_step": int(world * batch_n * 17), "d2h_bytes_per_step": int(world * batch_n * 8),
+               "steps": n_e, "path": "ShardedEirene.submit_host on every rank: pinned H2D of the rank's slice, "
+                                     "routing + NCCL exchanges + shard batch, D2H of the results slice (one "
+                                     "stream per rank); max over ranks"}
+
+    # ------------------------------------------------------------ parity at N > 1
+    # The first global batches against the oracle on SAMPLED KEY SLICES: requests
+    # on different keys are independent (linearizability is local),
+    # so the oracle loaded with the keys of a slice [lo, hi) and fed the batch's
+    # requests with lo <= key < hi, in timestamp order, must reproduce those
+    # requests' results exactly.  One slice straddles every shard boundary, plus
+    # the two ends of the key space.
+    parity = None
+    if world > 1 and args.cpu_batches > 0:
+        n_check = min(args.cpu_batches, nb)
+        gathered = []
+        for b in range(n_check):
+            t_ = results[b].view(torch.int64)
+            t_ = t_.cpu() if args.backend == "gloo" else t_
+            parts = [torch.empty_like(t_) for _ in range(world)]
+            dist.all_gather(parts, t_)
+            gathered.append(np.concatenate([p.cpu().numpy() for p in parts]).view(np.uint64))
+        if rank == 0:
+            parity = slice_parity(wl, gathered, sh.splitters_np, args.parity_slice)
 
     # ------------------------------------------------------------ parity + CPU baseline (rank 0, N=1)
-    parity = None
     cpu = None
     roof = None
     rar = None
-    if rank == 0 and world == 1 and args.cpu_batches > 0:
+    if rank == 0 and world == 1 and args.cpu_batches > 0 and tree_n > (1 << 25):
+        # (cfg5 at N = 1: a 2^28-key oracle is minutes of CPU; key-slice parity as at N > 1)
+        parity = slice_parity(wl, [results[b].cpu().numpy() for b in range(min(args.cpu_batches, nb))],
+                              np.zeros(0, np.uint64), args.parity_slice)
+    elif rank == 0 and world == 1 and args.cpu_batches > 0:
         import oracle
         n_check = min(args.cpu_batches, nb)
         refs = {}
@@ -641,6 +728,23 @@ def run_ours(args):
                    "probe": "eirene_probe_gather: 2^24 uniformly random 128 B line reads / 32 B sector reads / "
                             "32 B sector writes over a 4 GiB pool, best of 3, CUDA events"}
 
+    if rank == 0 and roof is None and not cap and not per_tree:
+        # the query kernel of rank 0's shard (N > 1, or a tree too large for the full oracle): its
+        # algorithmic bytes from the requests of the timed batches routed to this shard
+        my = wl.keys[(wl.keys >= np.uint64(sh.lo)) & ((wl.keys < np.uint64(sh.hi)) if sh.hi != (1 << 64) - 1
+                                                       else True)] if world > 1 else wl.keys
+        ab = []
+        for b in range(args.warmup, min(nb, args.warmup + 2)):
+            o, k, _ = wl.batch_arrays(b)
+            m = (k >= np.uint64(my[0])) & (k <= np.uint64(my[-1])) if world > 1 else slice(None)
+            ab.append(algorithmic_bytes_query(my, o[m], k[m], 16)["bytes"])
+        peaks = load_peaks()
+        ach = float(np.mean(ab)) / (stage_ms[2] * 1e-3) / 1e9
+        roof = {"bound": "hbm", "achieved": ach, "peak": peaks["hbm_gbs"], "unit": "GB/s", "frac": ach / peaks["hbm_gbs"],
+                "traffic": None, "kernel": "query_kernel" + (" (rank 0's shard)" if world > 1 else ""),
+                "stage_ms": float(stage_ms[2]), "algorithmic_bytes_per_launch": float(np.mean(ab)),
+                "peak_source": peaks["source"]}
+
     if rank == 0:
         line = {
             "metric": "requests/sec per batch", "value": value, "unit": "Greq/s", "n_gpus": world,
@@ -651,6 +755,7 @@ def run_ours(args):
                                    f"{batch_n * world}-request batches, "
                                    + ", ".join(f"{int(p * 100)}% {['query', 'update', 'insert', 'delete', 'range'][o]}"
                                                for o, p in sorted(C['fracs'].items())) + f", {C['dist']} keys"
+                                   + (f" (YCSB-like mix {args.mix})" if args.mix else "")
                                    + (f", range length {cap} (first {cap} pairs returned)" if cap else ""),
                        "cfg": cfg, "global_batch": batch_n * world,
                        "parallelism": f"key-range shards x{world}" if world > 1 else "single GPU",
@@ -702,7 +807,20 @@ def main():
                     help="iterwarp: the paper's iteration warps + range field (ablation)")
     ap.add_argument("--iter-rgs", type=int, default=0, help="RGs per iteration warp (0 = auto)")
     ap.add_argument("--ra-probe", type=int, default=1, help="measure the random-access roofline (1) or not (0)")
+    ap.add_argument("--mix", default="", choices=["", "A", "B", "C", "U"],
+                    help="YCSB-like mix override (cfg5): A 50/50 Zipf, B 95/5 Zipf, C 100%% read Zipf, U 95/5 uniform")
+    ap.add_argument("--parity-slice", type=int, default=1 << 16, help="loaded keys per parity slice (N > 1)")
     args = ap.parse_args()
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        # one process per GPU: relaunch under torch.distributed.run (rank 0 prints the line)
+        import socket
+        s_ = socket.socket()
+        s_.bind(("127.0.0.1", 0))
+        port = s_.getsockname()[1]
+        s_.close()
+        cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+               "--master-addr=127.0.0.1", f"--master-port={port}", os.path.abspath(__file__)] + sys.argv[1:]
+        raise SystemExit(subprocess.call(cmd))
     if args.warmup < 3:
         raise SystemExit("--warmup must be >= 3")
     if args.impl == "reference":

@@ -87,7 +87,8 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
                                                         const uint64_t* vals_src, uint64_t* vals_stage,
                                                         uint64_t* results, BatchCtl* ctl_out, uint4* zero,
                                                         uint32_t zero_n16, uint4* zero2, uint32_t zero2_n16,
-                                                        uint64_t* rkeys, uint64_t* rvals, uint32_t rcap) {
+                                                        uint64_t* rkeys, uint64_t* rvals, uint32_t rcap,
+                                                        uint32_t n) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
     zero[i] = make_uint4(0, 0, 0, 0);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero2_n16; i += gridDim.x * blockDim.x)
@@ -104,6 +105,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
     dst->rkeys = rkeys;
     dst->rvals = rvals;
     dst->rcap = rcap;
+    dst->n = n;
   }
 }
 
@@ -188,6 +190,18 @@ struct eirene_tree {
     return e;
   }
 };
+
+namespace eirene {
+// EIRENE_PDL=0/1 (read once per process): programmatic dependent launch of the
+// batch's kernels 2.. (eirene_internal.cuh)
+bool pdl_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("EIRENE_PDL");
+    return e ? std::atoi(e) != 0 : false;
+  }();
+  return on;
+}
+}  // namespace eirene
 
 extern "C" {
 
@@ -435,6 +449,17 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals
   return rc;
 }
 
+// Size bucket of an n-request batch: exact up to 256, else n rounded up to
+// 1/8 of its power of two (<= 12.5% padding, 8 buckets per octave), at most
+// max_batch.
+static uint32_t size_bucket(uint32_t n, uint32_t max_batch) {
+  if (n <= 256) return n;
+  const int k = 31 - __builtin_clz(n);
+  const uint32_t step = 1u << (k - 3);
+  const uint64_t b = ((uint64_t)n + step - 1) / step * step;
+  return (uint32_t)std::min<uint64_t>(b, max_batch);
+}
+
 static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                        uint64_t* results, cudaStream_t st, uint64_t* vals_stage, uint64_t* ticket,
                        uint64_t* rkeys = nullptr, uint64_t* rvals = nullptr, uint32_t rcap = 0,
@@ -451,6 +476,11 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     r.used = true;
   }
   r.n = n;
+  // Launches (grids, group count, distribution path) and the captured graph
+  // are sized for n's size bucket; the kernels read the batch's own n from
+  // BatchArgs.  Batches of varying size (the shards of a multi-GPU batch)
+  // then replay a handful of graphs instead of capturing one per size.
+  const uint32_t nk = size_bucket(n, h->cfg.max_batch);
   r.timing = (h->cfg.flags & EIRENE_F_TIMING) != 0;
   int launches = 0;
   const uint32_t seq = ++h->batch_seq;
@@ -477,35 +507,35 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   BatchCtl* ctl_slot = h->ctl_ring + tk % RING;
   uint4* zero16 = reinterpret_cast<uint4*>(h->zero_region);
   uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
-  const bool large = !bsort_fused(n, h->num_sms);   // two-kernel bucket sort with 16384 bins (bsort.cu)
+  const bool large = !bsort_fused(nk, h->num_sms);   // two-kernel bucket sort with 16384 bins (bsort.cu)
   uint4* zero2 = reinterpret_cast<uint4*>(large ? h->zero_large : h->zero_region);
   uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
   const BSortBufs& bsn = large ? h->bsL : h->bs;
   const CombBufs& cbn = large ? h->cbL : h->cb;
   auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
     set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
-                                                   zero_n16, zero2, zero2_n16, rkeys, rvals, rcap);
+                                                   zero_n16, zero2, zero2_n16, rkeys, rvals, rcap, n);
     ++launches;
     if (args_node) {
       cudaError_t e = last_node(s, args_node);
       if (e != cudaSuccess) return e;
     }
     if (timing) rec(0, s);
-    launch_bucket_sort(h->dargs, n, h->cfg.key_lo, h->cfg.key_hi, bsn, ctl, h->num_sms, s, &launches);
+    launch_bucket_sort(h->dargs, nk, h->cfg.key_lo, h->cfg.key_hi, bsn, ctl, h->num_sms, s, &launches);
     stage("sort");
     if (timing) rec(1, s);
-    launch_group(h->dargs, n, bsn, cbn, h->t, ctl, h->num_sms, s, &launches);
+    launch_group(h->dargs, nk, bsn, cbn, h->t, ctl, h->num_sms, s, &launches);
     const uint32_t* spay = h->bs.pB;
     stage("group");
     if (timing) rec(2, s);
-    launch_query(n, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, h->cfg.flags, h->cfg.iter_rgs, s, &launches);
-    if (range) launch_range(n, h->cb, spay, h->bs.kB, h->dargs, h->t, ctl, h->num_sms, s, &launches);
+    launch_query(nk, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, h->cfg.flags, h->cfg.iter_rgs, s, &launches);
+    if (range) launch_range(nk, h->cb, spay, h->bs.kB, h->dargs, h->t, ctl, h->num_sms, s, &launches);
     stage("query");
     if (timing) rec(3, s);
-    launch_update(n, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
+    launch_update(nk, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
     stage("update");
     if (timing) rec(4, s);
-    launch_result(spay, h->bs.kB, n, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, h->num_sms, s, &launches);
+    launch_result(spay, h->bs.kB, nk, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, h->num_sms, s, &launches);
     stage("result");
     if (timing) rec(5, s);
     return cudaGetLastError();
@@ -516,7 +546,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     // one captured graph per batch size; a replay updates only the args node
     GraphEntry* g = nullptr;
     for (auto& e : h->graphs)
-      if (e.exec && e.n == n && e.range == range) g = &e;
+      if (e.exec && e.n == nk && e.range == range) g = &e;
     if (!g) {
       GraphEntry& e = h->graphs[h->next_graph++ % MAX_GRAPHS];
       if (e.exec) cudaGraphExecDestroy(e.exec);
@@ -528,7 +558,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       if (ce != cudaSuccess) return cuda_fail(ce, "capture");
       CK(ee);
       CK(cudaGraphInstantiate(&e.exec, e.graph, 0));
-      e.n = n;
+      e.n = nk;
       e.range = range;
       e.launches = launches;
       g = &e;
@@ -536,7 +566,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     if (prepare_only) return EIRENE_OK;   // graph captured and instantiated, nothing launched
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
                       const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
-                      &zero2, &zero2_n16, &rkeys, &rvals, &rcap};
+                      &zero2, &zero2_n16, &rkeys, &rvals, &rcap, &n};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
     p.gridDim = dim3(SET_ARGS_CTAS);

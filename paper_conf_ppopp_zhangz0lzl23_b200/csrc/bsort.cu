@@ -48,8 +48,11 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
                                                                uint16_t* __restrict__ bin2grp,
                                                                uint32_t* __restrict__ gstart,
                                                                uint32_t* __restrict__ cursor, BatchCtl* ctl) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   extern __shared__ __align__(16) uint32_t h[];   // [2 * NBINS_L]: counts; the last CTA's cut (groups, prefixes)
   __shared__ uint32_t s_last;
+  n = A->n;   // the launch is sized for the graph's size bucket; the batch's own size is on the device
   __shared__ uint32_t wsum[H_THREADS / 32];
   __shared__ uint32_t s_total;
   const uint64_t* __restrict__ keys = A->keys;
@@ -144,9 +147,12 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
     const BatchArgs* __restrict__ A, uint32_t n, uint32_t G, uint64_t key_lo, uint64_t key_hi, uint32_t bshift,
     const uint16_t* __restrict__ bin2grp, uint32_t* __restrict__ cursor, uint64_t* __restrict__ kout,
     uint32_t* __restrict__ pout, BatchCtl* ctl) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   extern __shared__ __align__(16) unsigned char smem[];
   uint16_t* s_b2g = reinterpret_cast<uint16_t*>(smem);             // [NBINS_L]
   uint32_t* hist = reinterpret_cast<uint32_t*>(s_b2g + NBINS_L);   // [G] tile counts, then global base
+  n = A->n;
   const uint64_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
   const uint64_t* __restrict__ vals = A->vals_src;
@@ -216,9 +222,12 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
     const BatchArgs* __restrict__ A, uint32_t n, uint32_t G, uint32_t per_cta, uint64_t key_lo, uint64_t key_hi,
     uint32_t bshift, uint32_t* __restrict__ bcount, uint32_t* __restrict__ gstart, uint32_t* __restrict__ cursor,
     uint64_t* __restrict__ kout, uint32_t* __restrict__ pout, BatchCtl* ctl) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   __shared__ uint32_t h[NBINS];        // bin counts; then bin -> group
   __shared__ uint32_t gs[NBINS + 1];   // exclusive bin prefix; then group starts / bases
   __shared__ uint32_t wsum[D_THREADS / 32];
+  n = A->n;   // (per_cta is sized for the graph's size bucket >= n)
   const uint64_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
   const uint64_t* __restrict__ vals = A->vals_src;
@@ -397,11 +406,8 @@ void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_
     const uint32_t per_cta = ((rows + grid - 1) / grid) * D_THREADS;
     // cooperative launch: the grid barrier needs every CTA co-resident, which a plain
     // launch does not guarantee when other kernels share the device
-    void* args[] = {const_cast<BatchArgs**>(&A), &n, const_cast<uint32_t*>(&G), const_cast<uint32_t*>(&per_cta),
-                    &key_lo, &key_hi, &bshift, const_cast<uint32_t**>(&b.bcount), const_cast<uint32_t**>(&b.gstart),
-                    const_cast<uint32_t**>(&b.cursor), const_cast<uint64_t**>(&b.kA), const_cast<uint32_t**>(&b.pA),
-                    &ctl};
-    cudaLaunchCooperativeKernel(reinterpret_cast<void*>(bsort_dist_kernel), dim3(grid), dim3(D_THREADS), args, 0, st);
+    launch_k(bsort_dist_kernel, dim3(grid), dim3(D_THREADS), 0, st, true, true, A, n, G, per_cta, key_lo, key_hi,
+             bshift, b.bcount, b.gstart, b.cursor, b.kA, b.pA, ctl);
     *launches += 1;
     return;
   }
@@ -414,11 +420,11 @@ void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_
     return (int)cudaFuncSetAttribute(bsort_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)ssm);
   });
   const uint32_t tiles = (n + H_THREADS * H_ITEMS - 1) / (H_THREADS * H_ITEMS);
-  bsort_hist_kernel<<<std::max(1u, std::min(tiles, (uint32_t)num_sms)), H_THREADS, hsm, st>>>(
-      A, n, G, key_lo, bshift, b.bcount, b.bin2grp, b.gstart, b.cursor, ctl);
+  launch_k(bsort_hist_kernel, dim3(std::max(1u, std::min(tiles, (uint32_t)num_sms))), dim3(H_THREADS), hsm, st, true,
+           false, A, n, G, key_lo, bshift, b.bcount, b.bin2grp, b.gstart, b.cursor, ctl);
   const size_t sm = NBINS_L * sizeof(uint16_t) + (size_t)G * sizeof(uint32_t);
-  bsort_scatter_kernel<<<(n + S_TILE - 1) / S_TILE, S_THREADS, sm, st>>>(A, n, G, key_lo, key_hi, bshift, b.bin2grp,
-                                                                         b.cursor, b.kA, b.pA, ctl);
+  launch_k(bsort_scatter_kernel, dim3((n + S_TILE - 1) / S_TILE), dim3(S_THREADS), sm, st, true, false, A, n, G,
+           key_lo, key_hi, bshift, (const uint16_t*)b.bin2grp, b.cursor, b.kA, b.pA, ctl);
   *launches += 2;
 }
 

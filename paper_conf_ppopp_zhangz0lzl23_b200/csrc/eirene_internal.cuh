@@ -15,6 +15,7 @@
 #pragma once
 #include <algorithm>
 #include <cstdint>
+#include <utility>
 #include <cuda_runtime.h>
 
 #include "eirene.h"
@@ -121,6 +122,7 @@ struct BatchArgs {
   uint64_t* rvals;
   uint32_t rcap;
   unsigned long long t0;   // %globaltimer when the batch's first kernel started (device batch time)
+  uint32_t n;              // requests in the batch (launches are sized for the graph's size bucket >= n)
 };
 
 // tile counters
@@ -248,6 +250,43 @@ inline int per_device(int (&cache)[MAX_DEVICES], F compute) {
   if (d < 0 || d >= MAX_DEVICES) return compute();
   if (cache[d] == 0) cache[d] = compute() + 1;
   return cache[d] - 1;
+}
+
+// ------------------------------------------------------------ programmatic dependent launch
+// Kernels 2.. of a batch are launched with programmatic stream serialization
+// (PDL, EIRENE_PDL=1): a kernel may be scheduled while its predecessor drains,
+// hiding the launch latency between the batch's kernels.  Every batch kernel
+// starts with pdl_wait() (griddepcontrol.wait: returns once the predecessor
+// grid has completed and its writes are visible; a no-op without PDL) before
+// it touches anything, then pdl_trigger() lets its own successor be scheduled.
+// All batch kernels are single-wave grids, so an early successor never takes
+// SM slots a later wave of its predecessor would need.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, bool pdl,
+                     bool coop, Args&&... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute at[2];
+  unsigned na = 0;
+  if (pdl && pdl_enabled()) {
+    at[na].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[na].val.programmaticStreamSerializationAllowed = 1;
+    ++na;
+  }
+  if (coop) {
+    at[na].id = cudaLaunchAttributeCooperative;
+    at[na].val.cooperative = 1;
+    ++na;
+  }
+  cfg.attrs = at;
+  cfg.numAttrs = na;
+  return cudaLaunchKernelEx(&cfg, kern, std::forward<Args>(args)...);
 }
 
 // ------------------------------------------------------------ host-side launchers

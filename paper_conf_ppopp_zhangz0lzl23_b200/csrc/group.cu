@@ -1060,6 +1060,8 @@ __device__ void hot_pass2(const GroupArgs& g, uint32_t* bits, const HotCarry& c,
 }
 
 __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   extern __shared__ __align__(16) unsigned char smem_raw[];
   GSmem& S = *reinterpret_cast<GSmem*>(smem_raw);
   BatchCtl* ctl = g.ctl;
@@ -1089,7 +1091,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   uint32_t sp_o = 0, sp_h = 0, sp_lo = 0;
   if (!small) {
     const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S, g.hot_bits,
-                              &ctl->hot_ctr, g.n, g.hot_words);
+                              &ctl->hot_ctr, g.A->n, g.hot_words);
     if (where == 2) {
       mode = 2;
       sp_o = S.r_nh;
@@ -1251,6 +1253,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       __syncthreads();
     }
   }
+#ifdef EIRENE_GROUP_PROF_BUILD   // diagnostic builds only: printf in a kernel costs on every launch
   if ((g.prof & 1) && tid == 0) {
     const unsigned long long tp4 = gtime_ns();
     if (tp4 - tp0 > 20000)
@@ -1258,6 +1261,9 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
              cnt, mode, (tp1 - tp0) * 1e-3, (tp2 - tp1) * 1e-3, (tp3 - tp2) * 1e-3, (tp4 - tp3) * 1e-3,
              mode == 2 ? (S.prof_t[1] - S.prof_t[0]) * 1e-3 : 0.0);
   }
+#else
+  (void)tp0; (void)tp1; (void)tp2; (void)tp3;
+#endif
 }
 
 }  // namespace
@@ -1293,7 +1299,7 @@ void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const Comb
   g.prof = prof;
   g.t = t;
   g.ctl = ctl;
-  group_kernel<<<g.nb, G_THREADS, sizeof(GSmem), st>>>(g);
+  launch_k(group_kernel, dim3(g.nb), dim3(G_THREADS), sizeof(GSmem), st, true, false, g);
   ++*launches;
 }
 

@@ -23,6 +23,7 @@
 // order); segments longer than SHORT_SEG are queued for result_long_kernel.
 #include "eirene_internal.cuh"
 #include <cstdio>
+#include <cstdlib>
 
 namespace eirene {
 
@@ -151,6 +152,8 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
                                                         const uint32_t* __restrict__ istart,
                                                         uint32_t* __restrict__ longseg, const BatchArgs* __restrict__ A,
                                                         Tree t, BatchCtl* __restrict__ ctl) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
@@ -209,6 +212,8 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
                                                                  const BatchArgs* __restrict__ A, Tree t,
                                                                  BatchCtl* __restrict__ ctl, uint32_t iter_rgs,
                                                                  uint32_t stats) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw;
@@ -301,6 +306,8 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
                                                             const BatchArgs* __restrict__ A,
                                                             BatchCtl* __restrict__ ctl, const TreeHdr* hdr,
                                                             int dbgprint) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   if (!(ctl->invalid || ctl->status != 0)) {
     uint64_t* __restrict__ results = A->results;
     const uint64_t* __restrict__ vals = A->vals;
@@ -355,11 +362,15 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
     unsigned long long* dst = reinterpret_cast<unsigned long long*>(A->ctl_out);
     for (uint32_t i = threadIdx.x; i < sizeof(BatchCtl) / 8; i += blockDim.x) dst[i] = __ldcg(src + i);
   }
-  if (threadIdx.x == 0 && dbgprint) {
+}
+
+// Diagnostics (EIRENE_DEBUG_SYNC / EIRENE_UPDATE_PROF only): printf lives in
+// its own kernel, launched after the batch, not in the batch's kernels.
+__global__ void debug_print_kernel(const BatchCtl* __restrict__ ctl, int dbgprint) {
+  if (dbgprint)
     printf("[eirene dbg] %u %u %u %u %u %u %u %u\n", ctl->dbg[0], ctl->dbg[1], ctl->dbg[2], ctl->dbg[3],
            ctl->dbg[4], ctl->dbg[5], ctl->dbg[6], ctl->dbg[7]);
-  }
-  if (threadIdx.x == 0 && ctl->uprof[0]) {   // EIRENE_UPDATE_PROF: update-kernel phases (us since its start)
+  if (ctl->uprof[0]) {   // EIRENE_UPDATE_PROF: update-kernel phases (us since its start)
     printf("[upd prof] entries %u %u %u %u %u | t:", ctl->lvl_ent[0], ctl->lvl_ent[1], ctl->lvl_ent[2],
            ctl->lvl_ent[3], ctl->lvl_ent[4]);
     for (int i = 1; i < 24 && ctl->uprof[i]; ++i) printf(" %.1f", (ctl->uprof[i] - ctl->uprof[0]) * 1e-3);
@@ -425,7 +436,10 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
                                                     const uint64_t* __restrict__ kB,
                                                     const uint64_t* __restrict__ old,
                                                     const BatchArgs* __restrict__ A, Tree t, BatchCtl* __restrict__ ctl) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   if (ctl->invalid || ctl->status != 0 || ctl->nrange == 0) return;
+  n = A->n;   // (the grid is sized for the graph's size bucket)
   const uint8_t* __restrict__ ops = A->ops;
   const uint64_t* __restrict__ keys = A->keys;
   const uint64_t* __restrict__ vals = A->vals;
@@ -575,12 +589,12 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
   if (flags & EIRENE_F_ITERWARP) {
     // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
     const int iblocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 4u);
-    query_iterwarp_kernel<<<iblocks < 1 ? 1 : iblocks, 256, 0, st>>>(
+    launch_k(query_iterwarp_kernel, dim3(iblocks < 1 ? 1 : iblocks), dim3(256), 0, st, true, false, 
         c.qkey, c.wkey, c.wparent,
         QueryIO{c.qseg, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
         A, t, ctl, iter_rgs, (flags & EIRENE_F_STATS) ? 1u : 0u);
   } else {
-    query_kernel<<<blocks, 256, 0, st>>>(c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.wparent, c.old,
+    launch_k(query_kernel, dim3(blocks), dim3(256), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.wparent, c.old,
                                          spay, c.pinfo, c.istart, c.longseg, A, t, ctl);
   }
   ++*launches;
@@ -590,7 +604,7 @@ void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const uin
                   BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches) {
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
-  range_kernel<<<blocks, 256, 0, st>>>(n, c.wkey, c.wseg, spay, c.pinfo, c.istart, kB, c.old, A, t, ctl);
+  launch_k(range_kernel, dim3(blocks), dim3(256), 0, st, true, false, n, c.wkey, c.wseg, spay, c.pinfo, c.istart, kB, c.old, A, t, ctl);
   ++*launches;
 }
 
@@ -599,8 +613,10 @@ void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const C
   // one 1024-thread CTA per SM: enough for the long segments of a Zipf batch
   // (RCHUNK work items), cheap when there are none
   const uint32_t grid = std::max(1u, std::min<uint32_t>((uint32_t)num_sms, (n + 1023) / 1024));
-  result_long_kernel<<<grid, 1024, 0, st>>>(spay, kB, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr,
+  launch_k(result_long_kernel, dim3(grid), dim3(1024), 0, st, true, false, spay, kB, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr,
                                                        dbgprint);
+  static const bool uprof = std::getenv("EIRENE_UPDATE_PROF") != nullptr;
+  if (dbgprint || uprof) debug_print_kernel<<<1, 1, 0, st>>>(ctl, dbgprint);
   ++*launches;
 }
 

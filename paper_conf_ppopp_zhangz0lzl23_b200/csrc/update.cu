@@ -77,7 +77,6 @@ __device__ bool watchdog(const Ctx& C, WarpStats& ws, uint32_t where, uint32_t a
       C.ctl->dbg[3] = c;
       C.ctl->dbg[4] = d;
       C.ctl->dbg[5] = (blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-      printf("eirene watchdog: where=%u a=%u b=%u c=%u d=%u warp=%u\n", where, a, b, c, d, C.ctl->dbg[5]);
     }
     return true;
   }
@@ -1050,6 +1049,8 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
                      // r1h: 6 (80 regs, no spills) vs 8 (64 regs, 432 B spills): cfg1 0.389 -> 0.404, cfg2 6.92 -> 7.04)
 #endif
 __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
   const BatchCtl* ctl = C.ctl;
   if (ctl->invalid || ctl->status != 0) return;   // (uniform: every CTA leaves, no barrier is reached)
   // every issued write a value overwrite of a present key: all of them were
@@ -1254,10 +1255,9 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
     update_kernel<<<1, 32, 0, st>>>(C);
   } else {
     if (C.slots[0]) {   // grid barriers: cooperative launch (co-residency guaranteed)
-      void* args[] = {&C};
-      cudaLaunchCooperativeKernel(reinterpret_cast<void*>(update_kernel), dim3(blocks), dim3(128), args, 0, st);
+      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, true, C);
     } else {
-      update_kernel<<<blocks, 128, 0, st>>>(C);
+      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, false, C);
     }
   }
   ++*launches;

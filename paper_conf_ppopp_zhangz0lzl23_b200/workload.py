@@ -200,6 +200,17 @@ CONFIGS = {
 }
 
 
+# YCSB-like mixes of cfg5 (BASELINE configs[4]): workload A
+# (50% read / 50% update, Zipf), B (95 / 5, Zipf), C (100% read, Zipf) and the
+# paper's default 95 / 5 uniform
+MIXES = {
+    "A": (dict({0: 0.5, 1: 0.5}), "zipf"),
+    "B": (dict({0: 0.95, 1: 0.05}), "zipf"),
+    "C": (dict({0: 1.0}), "zipf"),
+    "U": (dict({0: 0.95, 1: 0.05}), "uniform"),
+}
+
+
 def seed_for(cfg: int) -> int:
     return 0xE1E2E3E4 + cfg
 
