@@ -110,19 +110,19 @@ def algorithmic_bytes_query(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarra
     per issued query 8 B key + 4 B seg read + 8 B result write, one 128 B leaf key
     line per distinct leaf touched, one 32 B value sector per distinct (leaf, sector)
     hit.  Valid for batches on the bulk-loaded shape (cfg2 never splits)."""
-    uk, first = np.unique(keys, return_index=True)
+    uk = W.sorted_unique(keys)
     issued_w = np.zeros(uk.size, bool)
     w = ops != W.QUERY
     # a key issues a write iff any write on it
-    wk = np.unique(keys[w])
+    wk = W.sorted_unique(keys[w])
     issued_w[np.searchsorted(uk, wk)] = True
     qk = uk[~issued_w]
     pos = np.searchsorted(loaded, qk)
     hit = (pos < loaded.size) & (loaded[np.minimum(pos, loaded.size - 1)] == qk)
     leaf = pos // per_leaf
     slot = pos % per_leaf
-    lines = np.unique(leaf).size
-    sectors = np.unique(leaf[hit] * 4 + slot[hit] // 4).size
+    lines = W.sorted_unique(leaf).size
+    sectors = W.sorted_unique(leaf[hit] * 4 + slot[hit] // 4).size
     nq = qk.size
     return {"issued_q": int(nq), "leaf_lines": int(lines), "value_sectors": int(sectors),
             "bytes": int(nq * (8 + 4 + 8) + lines * 128 + sectors * 32)}
@@ -142,8 +142,8 @@ def algorithmic_bytes_range(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarra
     idx = np.concatenate([np.arange(a, a + c) for a, c in zip(lo, cnt)]) if cnt.size else np.empty(0, np.int64)
     leaf = idx // per_leaf
     # the walk reads the leaf of l even when it holds no key of the range
-    lines = np.unique(np.concatenate([leaf, np.minimum(lo, loaded.size - 1) // per_leaf])).size
-    sectors = np.unique(leaf * 4 + (idx % per_leaf) // 4).size
+    lines = W.sorted_unique(np.concatenate([leaf, np.minimum(lo, loaded.size - 1) // per_leaf])).size
+    sectors = W.sorted_unique(leaf * 4 + (idx % per_leaf) // 4).size
     nr = int(r.sum())
     return {"ranges": nr, "pairs": int(cnt.sum()), "leaf_lines": int(lines), "value_sectors": int(sectors),
             "bytes": int(nr * (1 + 8 + 8 + 8) + int(cnt.sum()) * 16 + lines * 128 + sectors * 32)}
@@ -156,14 +156,14 @@ def random_access_counts(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, 
     one 32 B value sector (distinct sectors once); every issued write writes
     one 32 B value sector.  Streamed bytes per request: op 1 + key 8 +
     result 8, + 8 per upsert value."""
-    uk = np.unique(keys)
-    wk = np.unique(keys[ops != W.QUERY])
+    uk = W.sorted_unique(keys)
+    wk = W.sorted_unique(keys[ops != W.QUERY])
     pos = np.searchsorted(loaded, uk)
     hit = (pos < loaded.size) & (loaded[np.minimum(pos, loaded.size - 1)] == uk)
     leaf = pos // per_leaf
     n = keys.size
     ups = int(np.sum((ops == W.UPDATE) | (ops == W.INSERT)))
-    return {"lines": np.unique(leaf).size / n, "sectors": np.unique(leaf[hit] * 4 + (pos[hit] % per_leaf) // 4).size / n,
+    return {"lines": W.sorted_unique(leaf).size / n, "sectors": W.sorted_unique(leaf[hit] * 4 + (pos[hit] % per_leaf) // 4).size / n,
             "writes": wk.size / n, "bio": (n * 17 + ups * 8) / n}
 
 
@@ -382,9 +382,11 @@ def run_ours(args):
 
     # ------------------------------------------------------------ device-timed run
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(nb)]
-    # per-batch host events between the batches (EIRENE_BENCH_NO_EVENTS=1: none; the device
-    # timestamps of every batch are in its stats either way)
-    host_ev = not os.environ.get("EIRENE_BENCH_NO_EVENTS")
+    # Per-batch response times come from the device timestamps in every batch's stats
+    # (%globaltimer, BatchCtl t_begin / t_end).  Host CUDA events around each submit
+    # (EIRENE_BENCH_HOST_EVENTS=1) cost ~5 us of stream gap per batch (measured r2c:
+    # inter-batch gap 11 us -> 5.5 us without them), so the timed region only has its two.
+    host_ev = bool(os.environ.get("EIRENE_BENCH_HOST_EVENTS"))
     stats = []
     launches = 0
 
@@ -680,7 +682,7 @@ def run_ours(args):
         elif stage_names[dom] == "group":
             # bucket read 12 B + sorted payload 4 B + pinfo 4 B per request; one issued entry per key
             o0, k0 = host_batches[args.warmup][:2]
-            d = len(np.unique(k0))
+            d = len(W.sorted_unique(k0))
             bytes_per = batch_n * 20 + d * 17
             ms = stage_ms[1]
             kern = "group_kernel"
@@ -765,7 +767,8 @@ def run_ours(args):
                                              "its last kernel (BatchCtl t_begin / t_end), per timed batch")
             if dev_batch_ms is not None else spread(per_batch_ms, "CUDA events around each submit"),
             "batch_ms_host_events": spread(per_batch_ms, "CUDA events recorded on the submit stream around each "
-                                                         "submit (includes any host-side launch gap)"),
+                                                         "submit (includes any host-side launch gap)") if host_ev
+            else None,
             "stage_ms": {n: float(x) for n, x in zip(stage_names, stage_ms)},
             "stage_region_ms_per_step": direct_ms,
             "gpu_launches": launches,

@@ -254,6 +254,13 @@ int eirene_set_flags(eirene_handle h, uint32_t flags);
 int eirene_probe_gather(void* pool_dev, uint64_t pool_bytes, uint32_t n, int kind, uint64_t seed,
                         eirene_stream_t stream);
 
+/* Diagnostic: copies min(n_words, 2*512*8) u64 %globaltimer stamps of the
+ * last batch's distribution (kernel 0) and group (kernel 1) kernels,
+ * [kernel][CTA][phase], to host memory `out` (synchronises the device).  Only
+ * builds compiled with -DEIRENE_PHASE_PROF write them (tools/phase_prof.py);
+ * otherwise the buffer stays zero. */
+int eirene_debug_phases(eirene_handle h, uint64_t* out, uint32_t n_words);
+
 /* Frees every device and host resource of the handle (waits for pending work). */
 int eirene_destroy(eirene_handle h);
 

@@ -76,6 +76,7 @@ _SIGS = {
     "eirene_route_partition_packed": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _int, _vp, _vp, _vp, _vp]),
     "eirene_route_unpack": (_int, [_vp, _vp, _u32, _vp, _vp, _vp, _vp]),
     "eirene_batch_status_async": (_int, [_vp, _u64, _vp, _vp]),
+    "eirene_debug_phases": (_int, [_vp, _vp, _u32]),
 }
 
 _lib = None

@@ -40,7 +40,12 @@ def _stale(target: str, deps) -> bool:
     return any(os.path.getmtime(d) > t for d in deps)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, variant: str = "", defines: tuple = ()) -> str:
+    """Build libeirene.so; a `variant` (A/B or diagnostic build, e.g. -DEIRENE_PHASE_PROF) goes to
+    _build_<variant>/ and libeirene_<variant>.so, selected at run time with EIRENE_LIB."""
+    OBJ = os.path.join(PKG, "_build" + (f"_{variant}" if variant else ""))
+    LIB = os.path.join(PKG, f"libeirene_{variant}.so" if variant else "libeirene.so")
+    flags = FLAGS + [f"-D{d}" for d in defines]
     os.makedirs(OBJ, exist_ok=True)
     headers = glob.glob(os.path.join(CSRC, "*.cuh")) + [os.path.join(INCLUDE, "eirene.h")]
     jobs = []
@@ -49,7 +54,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         obj = os.path.join(OBJ, os.path.basename(src)[:-3] + ".o")
         objs.append(obj)
         if force or _stale(obj, [src] + headers):
-            cmd = [NVCC, *ARCH, *FLAGS, "-Xptxas", "-v", "-c", src, "-o", obj]
+            cmd = [NVCC, *ARCH, *flags, "-Xptxas", "-v", "-c", src, "-o", obj]
             jobs.append((src, cmd))
 
     def run(job):
@@ -79,4 +84,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
 
 if __name__ == "__main__":
-    build(force="--force" in sys.argv, verbose=True)
+    # python -m paper_conf_ppopp_zhangz0lzl23_b200.build [--force] [--variant NAME -DX ...]
+    a = sys.argv[1:]
+    var = a[a.index("--variant") + 1] if "--variant" in a else ""
+    build(force="--force" in a, verbose=True, variant=var, defines=tuple(x[2:] for x in a if x.startswith("-D")))

@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
                                                         uint64_t* results, BatchCtl* ctl_out, uint4* zero,
                                                         uint32_t zero_n16, uint4* zero2, uint32_t zero2_n16,
                                                         uint64_t* rkeys, uint64_t* rvals, uint32_t rcap,
-                                                        uint32_t n) {
+                                                        uint32_t n, unsigned long long* phase) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
     zero[i] = make_uint4(0, 0, 0, 0);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero2_n16; i += gridDim.x * blockDim.x)
@@ -106,6 +106,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
     dst->rvals = rvals;
     dst->rcap = rcap;
     dst->n = n;
+    dst->phase = phase;
   }
 }
 
@@ -141,6 +142,7 @@ struct eirene_tree {
   SortBufs sb{};
   BSortBufs bs{};
   BatchArgs* dargs = nullptr;
+  unsigned long long* phase = nullptr;   // diagnostic phase stamps (filled by -DEIRENE_PHASE_PROF builds)
   cudaStream_t cap_stream = nullptr;
   GraphEntry graphs[MAX_GRAPHS];
   uint32_t next_graph = 0;
@@ -323,6 +325,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->bs.gstart, NBINS_MAX + 1);
   AL(h->bs.bin2grp, NBINS_MAX);
   AL(h->dargs, 1);
+  AL(h->phase, 2 * PROF_CTAS * PROF_PHASES);
   AL(h->ctl_ring, RING);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
@@ -514,7 +517,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   const CombBufs& cbn = large ? h->cbL : h->cb;
   auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
     set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
-                                                   zero_n16, zero2, zero2_n16, rkeys, rvals, rcap, n);
+                                                   zero_n16, zero2, zero2_n16, rkeys, rvals, rcap, n, h->phase);
     ++launches;
     if (args_node) {
       cudaError_t e = last_node(s, args_node);
@@ -566,7 +569,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     if (prepare_only) return EIRENE_OK;   // graph captured and instantiated, nothing launched
     void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
                       const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
-                      &zero2, &zero2_n16, &rkeys, &rvals, &rcap, &n};
+                      &zero2, &zero2_n16, &rkeys, &rvals, &rcap, &n, &h->phase};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
     p.gridDim = dim3(SET_ARGS_CTAS);
@@ -718,6 +721,16 @@ int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out, u
   h->launches += launches;
   if (rc == EIRENE_ECUDA) return cuda_fail(cudaGetLastError(), "eirene_scan");
   return rc;
+}
+
+int eirene_debug_phases(eirene_handle h, uint64_t* out, uint32_t n_words) {
+  if (!h || !out) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  CK(cudaDeviceSynchronize());
+  const uint32_t m = std::min<uint32_t>(n_words, 2 * PROF_CTAS * PROF_PHASES);
+  CK(cudaMemcpy(out, h->phase, sizeof(uint64_t) * m, cudaMemcpyDeviceToHost));
+  return EIRENE_OK;
 }
 
 int eirene_set_flags(eirene_handle h, uint32_t flags) {

@@ -36,6 +36,15 @@ __device__ __forceinline__ void count_ranges(uint32_t nr, BatchCtl* ctl) {
   if (nr && (threadIdx.x & 31) == 0) atomicAdd(&ctl->nrange, nr);
 }
 
+// Group of a bin whose requests' midpoint has prefix x: floor(x * G / total),
+// clamped.  Any monotone non-decreasing map of x gives a valid cut (a bin never
+// straddles groups, groups stay key ranges in order); a float multiply is that
+// and costs one instruction instead of a 64-bit division per bin.  Every CTA
+// computes it from the same inputs, so all agree.
+__device__ __forceinline__ uint32_t group_of(uint32_t x, float gscale, uint32_t G) {
+  return min(G - 1u, (uint32_t)__fmul_rz((float)x, gscale));
+}
+
 constexpr int H_THREADS = 512;
 constexpr int H_ITEMS = 16;                      // 8192 requests per CTA
 constexpr int S_THREADS = 256;
@@ -113,12 +122,11 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
   uint32_t* sg = h;              // group of every bin
   uint32_t* se = h + NBINS_L;    // exclusive prefix of every bin
   const bool identity = G == (uint32_t)NBINS_L;
+  const float gscale = (float)G / (float)max(total, 1u);
 #pragma unroll
   for (int j = 0; j < PER; ++j) {
     const uint32_t bin = tid * PER + j;
-    const uint32_t g = identity ? bin
-                                : (uint32_t)min((unsigned long long)(G - 1),
-                                                ((unsigned long long)run + cnt[j] / 2) * G / max(total, 1u));
+    const uint32_t g = identity ? bin : group_of(run + cnt[j] / 2, gscale, G);
     sg[bin] = g;
     se[bin] = run;
     bin2grp[bin] = (uint16_t)g;
@@ -228,6 +236,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   __shared__ uint32_t gs[NBINS + 1];   // exclusive bin prefix; then group starts / bases
   __shared__ uint32_t wsum[D_THREADS / 32];
   n = A->n;   // (per_cta is sized for the graph's size bucket >= n)
+  EIRENE_PHASE(A, 0, blockIdx.x, 0);
   const uint64_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
   const uint64_t* __restrict__ vals = A->vals_src;
@@ -261,10 +270,12 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   if (__any_sync(FULL, bad) && lane == 0) atomicOr(&ctl->invalid, 1u);
   if (rok) count_ranges(nr, ctl);
   __syncthreads();
+  EIRENE_PHASE(A, 0, blockIdx.x, 1);
   for (uint32_t i = tid; i < NBINS; i += D_THREADS)
     if (h[i]) atomicAdd(&bcount[i], h[i]);
   // grid barrier (all CTAs are resident: the grid is one occupancy wave)
   __syncthreads();
+  EIRENE_PHASE(A, 0, blockIdx.x, 2);
   if (tid == 0) {
     __threadfence();
     atomicAdd(&ctl->gbar, 1u);
@@ -273,6 +284,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
       if (sg.stuck(ctl)) break;
   }
   __syncthreads();
+  EIRENE_PHASE(A, 0, blockIdx.x, 3);
   // phase 2: the group cut, as in bsort_hist_kernel's last CTA
   constexpr int PER = NBINS / D_THREADS;
   uint32_t cnt[PER];
@@ -297,12 +309,11 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   __syncthreads();
   const uint32_t total = s_total;
   const bool identity = G == (uint32_t)NBINS;
+  const float gscale = (float)G / (float)max(total, 1u);
 #pragma unroll
   for (int j = 0; j < PER; ++j) {
     const uint32_t bin = tid * PER + j;
-    const uint32_t g = identity ? bin
-                                : (uint32_t)min((unsigned long long)(G - 1),
-                                                ((unsigned long long)run + cnt[j] / 2) * G / max(total, 1u));
+    const uint32_t g = identity ? bin : group_of(run + cnt[j] / 2, gscale, G);
     h[bin] = g;
     gs[bin] = run;
     run += cnt[j];
@@ -331,6 +342,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   __syncthreads();
   if (blockIdx.x == 0)
     for (uint32_t q = tid; q <= G; q += D_THREADS) gstart[q] = gs[q];
+  EIRENE_PHASE(A, 0, blockIdx.x, 4);
   // phase 3: tile histogram over the groups (reuses the tail of h as counters)
   uint32_t* th = h + NBINS - G;   // bins are no longer needed once g is known per item
   uint32_t g[D_ITEMS], r[D_ITEMS];
@@ -350,6 +362,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
     th[q] = c ? gs[q] + atomicAdd(&cursor[q], c) : 0u;
   }
   __syncthreads();
+  EIRENE_PHASE(A, 0, blockIdx.x, 5);
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
@@ -359,6 +372,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
       pout[pos] = (i << 2) | o[j];
     }
   }
+  EIRENE_PHASE(A, 0, blockIdx.x, 6);
 }
 
 }  // namespace

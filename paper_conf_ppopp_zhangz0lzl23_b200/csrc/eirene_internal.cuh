@@ -31,6 +31,7 @@ constexpr uint32_t DONE_BIT = 0x80000000u;    // pinfo: an earlier write of the 
 constexpr uint32_t DEFER_BIT = 0x40000000u;   // pinfo (hot-key segments): that early result is written by
                                               // result_long_kernel from the nearest write's payload in kB
 constexpr uint32_t SEG_MASK = 0x3FFFFFFFu;
+constexpr uint32_t Q_SINGLE = 0x80000000u;    // qseg entry of a one-request query segment: Q_SINGLE | its timestamp
 constexpr uint32_t RCHUNK = 4096;             // result_long_kernel work item: positions of one long segment
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 
@@ -123,7 +124,23 @@ struct BatchArgs {
   uint32_t rcap;
   unsigned long long t0;   // %globaltimer when the batch's first kernel started (device batch time)
   uint32_t n;              // requests in the batch (launches are sized for the graph's size bucket >= n)
+  unsigned long long* phase;   // diagnostic builds (-DEIRENE_PHASE_PROF): [kernel][CTA][phase] %globaltimer stamps
 };
+
+// Phase timestamps of the distribution / group kernels (diagnostic builds only:
+// -DEIRENE_PHASE_PROF; read back with eirene_debug_phases).
+constexpr int PROF_CTAS = 512, PROF_PHASES = 8;
+#ifdef EIRENE_PHASE_PROF
+#define EIRENE_PHASE(A, k, cta, i)                                                                   \
+  do {                                                                                            \
+    if (threadIdx.x == 0 && (A)->phase && (cta) < PROF_CTAS)                                       \
+      (A)->phase[((size_t)(k) * PROF_CTAS + (cta)) * PROF_PHASES + (i)] = gtime_ns();             \
+  } while (0)
+#else
+#define EIRENE_PHASE(A, k, cta, i) \
+  do {                             \
+  } while (0)
+#endif
 
 // tile counters
 enum { TC_SORT0 = 0, TC_GROUP = 8, TC_ROUTE = 10, TC_SCAN = 11, TC_HIST = 12 };

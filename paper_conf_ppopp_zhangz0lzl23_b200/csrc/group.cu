@@ -872,7 +872,10 @@ __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uin
       } else {      // all-query segment: its last query
         const uint32_t qi = seg - wi;
         g.qkey[qi] = k;
-        g.qseg[qi] = seg;
+        // a one-request segment (head and tail) carries its timestamp instead of
+        // its segment index: the query kernel writes results[ts] directly, with
+        // no istart / sorted-payload reads and no old[seg] (RESULT_CAL)
+        g.qseg[qi] = head ? (Q_SINGLE | (p >> 2)) : seg;
       }
     }
     nh += __popc(H);
@@ -1070,6 +1073,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   if (tid == 0) S.ticket = atomicAdd(&ctl->tile_ctr[TC_GROUP], 1u);
   __syncthreads();
   const uint32_t b = S.ticket;
+  EIRENE_PHASE(g.A, 1, b, 0);
   const unsigned long long tp0 = g.prof ? gtime_ns() : 0;
   const uint32_t base = g.gstart[b];
   const uint32_t cnt = g.gstart[b + 1] - base;
@@ -1104,6 +1108,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       P = (where ? g.pB : g.pA) + base;
     }
   }
+  EIRENE_PHASE(g.A, 1, b, 1);
   const unsigned long long tp1 = g.prof ? gtime_ns() : 0;
   // an oversized group is walked in rounds of G_CAP positions copied to smem
   auto load_round = [&](uint32_t r0, uint32_t r1) {
@@ -1161,6 +1166,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     c_lw = S.r_lw;
     c_nw = S.r_nw;
   }
+  EIRENE_PHASE(g.A, 1, b, 2);
   const unsigned long long tp2 = g.prof ? gtime_ns() : 0;
   // decoupled look-back over the buckets (ticket order) on (heads << 31 | writes)
   if (warp == 0) {
@@ -1210,6 +1216,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     }
   }
   __syncthreads();
+  EIRENE_PHASE(g.A, 1, b, 3);
   const unsigned long long tp3 = g.prof ? gtime_ns() : 0;
   // sweep 2: emit (a small bucket reuses the carries of its single round)
   if (mode == 2) {
@@ -1253,6 +1260,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       __syncthreads();
     }
   }
+  EIRENE_PHASE(g.A, 1, b, 4);
 #ifdef EIRENE_GROUP_PROF_BUILD   // diagnostic builds only: printf in a kernel costs on every launch
   if ((g.prof & 1) && tid == 0) {
     const unsigned long long tp4 = gtime_ns();

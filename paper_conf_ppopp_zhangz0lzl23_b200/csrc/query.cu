@@ -96,6 +96,10 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
   bool delp = false;   // a delete of a present key: removes a key from its leaf
   if (isq) {
     seg = qseg[i];
+    if (seg & Q_SINGLE) {   // the segment's only request: its result, nothing else
+      results[seg & ~Q_SINGLE] = v;
+      return;
+    }
   } else {
     const uint32_t w = i - nq;
     seg = wseg[w];
@@ -120,7 +124,9 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
     if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&ctl->nins, (uint32_t)__popc(m));
     if (md && (threadIdx.x & 31) == __ffs(md) - 1) atomicAdd(&ctl->ndelp, (uint32_t)__popc(md));
   }
-  old[seg] = v;
+  // old[seg] (the pre-batch value) is read by result_long_kernel for long
+  // segments and by the range kernel for written keys only
+  if (!isq) old[seg] = v;
   const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
   if (p1 - p0 <= SHORT_SEG) {
     if (isq) {   // an all-query segment: every position is pending
@@ -130,6 +136,7 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
         if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
     }
   } else {   // work items of RCHUNK positions: (segment, chunk) pairs
+    if (isq) old[seg] = v;
     const uint32_t nc = (p1 - p0 + RCHUNK - 1) / RCHUNK;
     const uint32_t at = atomicAdd(&ctl->nlong, nc);
     for (uint32_t c = 0; c < nc; ++c) {
