@@ -226,15 +226,37 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
 // read of the keys instead of two of each.
 constexpr int D_THREADS = 512;
 constexpr int D_ITEMS = 8;
+constexpr int D_TILE = D_THREADS * D_ITEMS;   // >= per_cta
+constexpr int D_GMAX = NBINS / 2;             // groups of the fused path
+// Dynamic shared memory of the fused kernel (two CTAs per SM).  The tile
+// staging arrays overlay the bin arrays, which are dead by the time the tile
+// is staged.
+struct DSmem {
+  union {
+    struct {
+      uint32_t h[NBINS];        // local bin counts; global counts; then bin -> group
+      uint32_t gs[NBINS + 4];   // exclusive bin prefix; then group starts
+    } b;
+    uint64_t sk[D_TILE];        // the tile's keys in group order (staged scatter)
+  } u;
+  uint32_t sp[D_TILE];          // ... their payloads
+  uint16_t sg[D_TILE];          // ... their groups
+  uint32_t th[D_GMAX];          // tile count per group; then local offsets
+  uint32_t gb[D_GMAX];          // global position of the tile's first request of each group
+  uint32_t wsum[D_THREADS / 32];
+  uint32_t total;
+};
+
 __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
     const BatchArgs* __restrict__ A, uint32_t n, uint32_t G, uint32_t per_cta, uint64_t key_lo, uint64_t key_hi,
     uint32_t bshift, uint32_t* __restrict__ bcount, uint32_t* __restrict__ gstart, uint32_t* __restrict__ cursor,
     uint64_t* __restrict__ kout, uint32_t* __restrict__ pout, BatchCtl* ctl) {
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
-  __shared__ uint32_t h[NBINS];        // bin counts; then bin -> group
-  __shared__ uint32_t gs[NBINS + 1];   // exclusive bin prefix; then group starts / bases
-  __shared__ uint32_t wsum[D_THREADS / 32];
+  extern __shared__ __align__(16) unsigned char dsm_raw[];
+  DSmem& S = *reinterpret_cast<DSmem*>(dsm_raw);
+  uint32_t* h = S.u.b.h;
+  uint32_t* gs = S.u.b.gs;
   n = A->n;   // (per_cta is sized for the graph's size bucket >= n)
   EIRENE_PHASE(A, 0, blockIdx.x, 0);
   const uint64_t* __restrict__ keys = A->keys;
@@ -285,52 +307,51 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   }
   __syncthreads();
   EIRENE_PHASE(A, 0, blockIdx.x, 3);
-  // phase 2: the group cut, as in bsort_hist_kernel's last CTA
+  // phase 2: the group cut, as in bsort_hist_kernel's last CTA.  Every CTA
+  // needs all 4096 global counts: staged into shared memory with coalesced
+  // 16 B loads (296 CTAs reading the same 16 KB as strided 4 B loads hammered
+  // the same L2 lines: 7-11 us, r2d phase profile)
+  for (uint32_t i = tid; i < NBINS / 4; i += D_THREADS)
+    reinterpret_cast<uint4*>(h)[i] = __ldcg(reinterpret_cast<const uint4*>(bcount) + i);
+  __syncthreads();
   constexpr int PER = NBINS / D_THREADS;
   uint32_t cnt[PER];
   uint32_t sum = 0;
-#pragma unroll
-  for (int j = 0; j < PER; ++j) {
-    cnt[j] = ld_cg(bcount + tid * PER + j);
-    sum += cnt[j];
+  {
+    const uint4 a = reinterpret_cast<const uint4*>(h)[2 * tid], b = reinterpret_cast<const uint4*>(h)[2 * tid + 1];
+    cnt[0] = a.x; cnt[1] = a.y; cnt[2] = a.z; cnt[3] = a.w;
+    cnt[4] = b.x; cnt[5] = b.y; cnt[6] = b.z; cnt[7] = b.w;
   }
+#pragma unroll
+  for (int j = 0; j < PER; ++j) sum += cnt[j];
   uint32_t x = sum;
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
     const uint32_t y = __shfl_up_sync(FULL, x, d);
     if (lane >= d) x += y;
   }
-  if (lane == 31) wsum[warp] = x;
+  if (lane == 31) S.wsum[warp] = x;
   __syncthreads();
   uint32_t run = x - sum;
-  for (int w = 0; w < warp; ++w) run += wsum[w];
-  __shared__ uint32_t s_total;
-  if (tid == D_THREADS - 1) s_total = run + sum;   // point requests in the batch
+  for (int w = 0; w < warp; ++w) run += S.wsum[w];
+  if (tid == D_THREADS - 1) S.total = run + sum;   // point requests in the batch
   __syncthreads();
-  const uint32_t total = s_total;
+  const uint32_t total = S.total;
   const bool identity = G == (uint32_t)NBINS;
   const float gscale = (float)G / (float)max(total, 1u);
-#pragma unroll
-  for (int j = 0; j < PER; ++j) {
-    const uint32_t bin = tid * PER + j;
-    const uint32_t g = identity ? bin : group_of(run + cnt[j] / 2, gscale, G);
-    h[bin] = g;
-    gs[bin] = run;
-    run += cnt[j];
-  }
-  __syncthreads();
-  // group starts into registers of the bins' threads, then gs[] = group starts
   uint32_t gq[PER], ge[PER];
 #pragma unroll
   for (int j = 0; j < PER; ++j) {
     const uint32_t bin = tid * PER + j;
-    gq[j] = h[bin];
-    ge[j] = gs[bin];
+    gq[j] = identity ? bin : group_of(run + cnt[j] / 2, gscale, G);
+    ge[j] = run;
+    h[bin] = gq[j];
+    run += cnt[j];
   }
-  const uint32_t gprev = tid ? h[tid * PER - 1] : 0xFFFFFFFFu;
   __syncthreads();
+  // group g starts at the prefix of its first bin (empty groups: where the next one does)
   {
-    uint32_t gp = gprev;
+    uint32_t gp = tid ? h[tid * PER - 1] : 0xFFFFFFFFu;
 #pragma unroll
     for (int j = 0; j < PER; ++j) {
       for (uint32_t q = gp + 1; q <= gq[j]; ++q) gs[q] = ge[j];
@@ -343,34 +364,83 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   if (blockIdx.x == 0)
     for (uint32_t q = tid; q <= G; q += D_THREADS) gstart[q] = gs[q];
   EIRENE_PHASE(A, 0, blockIdx.x, 4);
-  // phase 3: tile histogram over the groups (reuses the tail of h as counters)
-  uint32_t* th = h + NBINS - G;   // bins are no longer needed once g is known per item
+  // phase 3: group of every item; tile histogram over the groups
   uint32_t g[D_ITEMS], r[D_ITEMS];
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) g[j] = h[bin_of(k[j], key_lo, bshift, NBINS)];
-  __syncthreads();
-  for (uint32_t q = tid; q < G; q += D_THREADS) th[q] = 0;
+  for (uint32_t q = tid; q < G; q += D_THREADS) S.th[q] = 0;
   __syncthreads();
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
-    r[j] = (i < t1 && o[j] != OP_RANGE) ? atomicAdd(&th[g[j]], 1u) : 0u;
+    r[j] = (i < t1 && o[j] != OP_RANGE) ? atomicAdd(&S.th[g[j]], 1u) : 0u;
   }
   __syncthreads();
-  for (uint32_t q = tid; q < G; q += D_THREADS) {
-    const uint32_t c = th[q];
-    th[q] = c ? gs[q] + atomicAdd(&cursor[q], c) : 0u;
+  // per group: one global atomic for the tile's base in the group, and the
+  // exclusive scan of the tile's counts (local offsets of the group-ordered tile)
+  for (uint32_t q = tid; q < G; q += D_THREADS) {   // (one atomic per thread: all in flight together)
+    const uint32_t c = S.th[q];
+    if (c) S.gb[q] = gs[q] + atomicAdd(&cursor[q], c);
   }
-  __syncthreads();
+  {
+    constexpr int GPER = D_GMAX / D_THREADS;   // 4 groups per thread
+    uint32_t c[GPER], lsum = 0;
+#pragma unroll
+    for (int j = 0; j < GPER; ++j) {
+      const uint32_t q = tid * GPER + j;
+      c[j] = q < G ? S.th[q] : 0u;
+      lsum += c[j];
+    }
+    uint32_t y = lsum;
+#pragma unroll
+    for (int d = 1; d < 32; d <<= 1) {
+      const uint32_t z = __shfl_up_sync(FULL, y, d);
+      if (lane >= d) y += z;
+    }
+    __syncthreads();   // (S.wsum reuse)
+    if (lane == 31) S.wsum[warp] = y;
+    __syncthreads();
+    uint32_t lr = y - lsum;
+    for (int w = 0; w < warp; ++w) lr += S.wsum[w];
+#pragma unroll
+    for (int j = 0; j < GPER; ++j) {
+      const uint32_t q = tid * GPER + j;
+      if (q < G) S.th[q] = lr;
+      lr += c[j];
+    }
+  }
+  __syncthreads();   // (the bin arrays are dead from here: the staging overlays them)
   EIRENE_PHASE(A, 0, blockIdx.x, 5);
+  // staged scatter: the tile in group order in shared memory, then every
+  // group's run written out contiguously (coalesced instead of one scattered
+  // 8 B + 4 B store per request)
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
     if (i < t1 && o[j] != OP_RANGE) {
-      const uint32_t pos = th[g[j]] + r[j];
-      kout[pos] = k[j];
-      pout[pos] = (i << 2) | o[j];
+      const uint32_t lp = S.th[g[j]] + r[j];
+      S.u.sk[lp] = k[j];
+      S.sp[lp] = (i << 2) | o[j];
+      S.sg[lp] = (uint16_t)g[j];
     }
+  }
+  __syncthreads();
+  uint32_t tcount = 0;   // point requests of the tile
+#pragma unroll
+  for (int j = 0; j < D_ITEMS; ++j) {
+    const uint32_t i = t0 + j * D_THREADS + tid;
+    tcount += (i < t1 && o[j] != OP_RANGE) ? 1u : 0u;
+  }
+  tcount = __reduce_add_sync(FULL, tcount);
+  if (lane == 0) S.wsum[warp] = tcount;
+  __syncthreads();
+  uint32_t tot = 0;
+  for (int w = 0; w < D_THREADS / 32; ++w) tot += S.wsum[w];
+  for (uint32_t lp = tid; lp < tot; lp += D_THREADS) {
+    const uint32_t q = S.sg[lp];
+    const uint32_t pos = S.gb[q] + (lp - S.th[q]);
+    kout[pos] = S.u.sk[lp];
+    pout[pos] = S.sp[lp];
   }
   EIRENE_PHASE(A, 0, blockIdx.x, 6);
 }
@@ -381,8 +451,11 @@ static uint32_t dist_grid(int num_sms) {
   static int occ[MAX_DEVICES];
   const int per_sm = per_device(occ, [] {
     int v = 0;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, bsort_dist_kernel, D_THREADS, 0) == cudaSuccess ? v
-                                                                                                           : 0;
+    cudaFuncSetAttribute(bsort_dist_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(DSmem));
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, bsort_dist_kernel, D_THREADS, sizeof(DSmem)) ==
+                   cudaSuccess
+               ? v
+               : 0;
   });
   return (uint32_t)num_sms * (uint32_t)std::max(per_sm, 0);
 }
@@ -420,7 +493,7 @@ void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_
     const uint32_t per_cta = ((rows + grid - 1) / grid) * D_THREADS;
     // cooperative launch: the grid barrier needs every CTA co-resident, which a plain
     // launch does not guarantee when other kernels share the device
-    launch_k(bsort_dist_kernel, dim3(grid), dim3(D_THREADS), 0, st, true, true, A, n, G, per_cta, key_lo, key_hi,
+    launch_k(bsort_dist_kernel, dim3(grid), dim3(D_THREADS), sizeof(DSmem), st, true, true, A, n, G, per_cta, key_lo, key_hi,
              bshift, b.bcount, b.gstart, b.cursor, b.kA, b.pA, ctl);
     *launches += 1;
     return;
