@@ -318,7 +318,7 @@ def run_ours(args):
 
     # query traversal: the default (one key-sorted request per thread, path
     # sharing) or the paper's iteration warps + range field (ablation)
-    qmode = {"iterwarp": args.query_mode == "iterwarp", "iter_rgs": args.iter_rgs}
+    qmode = {"iterwarp": args.query_mode == "iterwarp", "iter_rgs": args.iter_rgs, "pipeline": bool(args.pipeline)}
     if args.query_mode != "default" and world > 1:
         raise SystemExit("--query-mode iterwarp runs on one GPU")
 
@@ -430,6 +430,8 @@ def run_ours(args):
         tickets = []
         for b in range(args.warmup, nb):
             tickets.append(step(b))
+        if world == 1 and args.pipeline:   # the last batch ends on the library's back stream
+            tickets[-1][0].stream_wait(tickets[-1][1], stream)
         t_end.record(stream)
         torch.cuda.synchronize()
         if world > 1:
@@ -813,6 +815,8 @@ def main():
     ap.add_argument("--mix", default="", choices=["", "A", "B", "C", "U"],
                     help="YCSB-like mix override (cfg5): A 50/50 Zipf, B 95/5 Zipf, C 100%% read Zipf, U 95/5 uniform")
     ap.add_argument("--parity-slice", type=int, default=1 << 16, help="loaded keys per parity slice (N > 1)")
+    ap.add_argument("--pipeline", type=int, default=0,
+                    help="1: cross-batch pipelining (EIRENE_F_PIPELINE, SURVEY 8(f) NEXT(3))")
     args = ap.parse_args()
     if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
         # one process per GPU: relaunch under torch.distributed.run (rank 0 prints the line)

@@ -65,12 +65,21 @@ enum {
   EIRENE_F_FORCE_STM = 1u << 2, /* every traversal in the update kernel is STM-protected
                                    (equivalent to retry_threshold = 0, Alg.1:28-33)               */
   EIRENE_F_TIMING = 1u << 3,    /* record per-stage CUDA events (eirene_batch_stats.stage_ms)     */
-  EIRENE_F_ITERWARP = 1u << 4   /* query kernel: the paper's iteration warps with a per-leaf range
+  EIRENE_F_ITERWARP = 1u << 4,  /* query kernel: the paper's iteration warps with a per-leaf range
                                    field (RF) choosing vertical (root-to-leaf) or horizontal
                                    (leaf-link) traversal per request group (Fig.6);
                                    off = one key-sorted request per thread with path sharing (the
                                    default).  Results are identical either way;
                                    with EIRENE_F_STATS the batch stats report the decisions      */
+  EIRENE_F_PIPELINE = 1u << 5   /* (at create) cross-batch pipelining, §8(f) NEXT(3): the front
+                                   of batch b+1 (distribution, group sort, combine, partition --
+                                   nothing that reads the tree) runs on the caller's stream while
+                                   the back of batch b (query, update, RESULT_CAL) runs on the
+                                   handle's back stream; backs stay in submission order, so
+                                   query(b+1) follows update(b).  Double-buffers the
+                                   front->back scratch.  A batch's results are then NOT ordered on
+                                   the caller's stream: use eirene_results or
+                                   eirene_stream_wait_batch before consuming them there        */
 };
 
 typedef struct {
@@ -203,6 +212,13 @@ int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops_dev, const uin
  * the first such batch does not pay the capture.  A handle keeps graphs for a
  * few distinct sizes.  Errors: EINVAL (n == 0 or n > max_batch), ECUDA. */
 int eirene_prepare_batch(eirene_handle h, uint32_t n, int with_ranges);
+
+/* Makes `stream` wait (on the device, no host synchronisation) until batch
+ * `ticket` has finished, so work enqueued on `stream` afterwards may consume
+ * its results.  Needed with EIRENE_F_PIPELINE, where a batch ends on the
+ * handle's back stream; a no-op ordering otherwise.  ESTATE for an unknown or
+ * too old ticket. */
+int eirene_stream_wait_batch(eirene_handle h, uint64_t ticket, eirene_stream_t stream);
 
 /* Waits for batch `ticket` and returns its status (EIRENE_OK, EINVAL, EFULL);
  * fills *stats if non-NULL.  ESTATE if the ticket is unknown or too old (the

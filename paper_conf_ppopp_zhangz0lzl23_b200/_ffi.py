@@ -21,6 +21,7 @@ EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECU
     0, -1, -2, -3, -4, -5, -6)
 EIRENE_QUERY, EIRENE_UPDATE, EIRENE_INSERT, EIRENE_DELETE, EIRENE_RANGE = 0, 1, 2, 3, 4
 EIRENE_F_REGROUP, EIRENE_F_STATS, EIRENE_F_FORCE_STM, EIRENE_F_TIMING, EIRENE_F_ITERWARP = 1, 2, 4, 8, 16
+EIRENE_F_PIPELINE = 32
 NOT_FOUND = 0xFFFFFFFFFFFFFFFF
 
 _u64 = ctypes.c_uint64
@@ -77,6 +78,7 @@ _SIGS = {
     "eirene_route_unpack": (_int, [_vp, _vp, _u32, _vp, _vp, _vp, _vp]),
     "eirene_batch_status_async": (_int, [_vp, _u64, _vp, _vp]),
     "eirene_debug_phases": (_int, [_vp, _vp, _u32]),
+    "eirene_stream_wait_batch": (_int, [_vp, _u64, _vp]),
 }
 
 _lib = None

@@ -123,6 +123,25 @@ struct GraphEntry {
   int launches = 0;                 // kernels in the graph
 };
 
+// One set of the buffers a batch's front (distribution + group: sort, combine,
+// partition) hands to its back (query, range, update, RESULT_CAL), plus the
+// per-batch control region.  Lane 0 always exists; with EIRENE_F_PIPELINE a
+// second lane lets the front of batch b+1 run while the back of batch b runs
+// (§8(f) NEXT(3)): the front never reads the tree, only the back does, and
+// backs stay in submission order (query(b+1) after update(b)).
+struct Lane {
+  BSortBufs bs{}, bsL{};
+  CombBufs cb{}, cbL{};
+  BatchArgs* dargs = nullptr;
+  BatchCtl* ctl = nullptr;
+  unsigned char* zero_region = nullptr;
+  unsigned char* zero_large = nullptr;
+  GraphEntry fg[MAX_GRAPHS], bg[MAX_GRAPHS];   // pipelined mode: front / back graphs per size bucket
+  uint32_t next_fg = 0, next_bg = 0;
+  cudaEvent_t front_done = nullptr, back_done = nullptr;
+  bool used = false;
+};
+
 struct Rec {
   uint64_t ticket = 0;
   bool used = false;
@@ -145,6 +164,11 @@ struct eirene_tree {
   unsigned long long* phase = nullptr;   // diagnostic phase stamps (filled by -DEIRENE_PHASE_PROF builds)
   cudaStream_t cap_stream = nullptr;
   GraphEntry graphs[MAX_GRAPHS];
+  Lane lanes[2];
+  int nlanes = 1;
+  uint32_t lane_seq = 0;
+  cudaStream_t back_stream = nullptr;   // pipelined mode: the backs of all batches, in order
+  cudaEvent_t last_done = nullptr;      // pipelined mode: the last submitted batch's end
   uint32_t next_graph = 0;
   bool use_graphs = std::getenv("EIRENE_NO_GRAPHS") == nullptr;
   CombBufs cb{};
@@ -368,6 +392,76 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
       }
     }
   }
+  // lane 0 = the buffers above; lane 1 (EIRENE_F_PIPELINE) = its own copy of
+  // every buffer a front hands to its back and of the control regions
+  if (e == cudaSuccess) {
+    Lane& L0 = h->lanes[0];
+    L0.bs = h->bs;
+    L0.bsL = h->bsL;
+    L0.cb = h->cb;
+    L0.cbL = h->cbL;
+    L0.dargs = h->dargs;
+    L0.ctl = h->ctl;
+    L0.zero_region = h->zero_region;
+    L0.zero_large = h->zero_large;
+  }
+  if (e == cudaSuccess && (cfg->flags & EIRENE_F_PIPELINE)) {
+    Lane& L1 = h->lanes[1];
+    L1 = h->lanes[0];
+    uint64_t *kB = nullptr, *qkey = nullptr, *wkey = nullptr, *wval = nullptr;
+    uint32_t *pB = nullptr, *pinfo = nullptr, *istart = nullptr, *qseg = nullptr, *wseg = nullptr;
+    uint8_t* wop = nullptr;
+    AL(kB, nb);
+    AL(pB, nb);
+    AL(pinfo, nb);
+    AL(istart, nb + 1);
+    AL(qkey, nb);
+    AL(qseg, nb);
+    AL(wkey, nb);
+    AL(wop, nb);
+    AL(wval, nb);
+    AL(wseg, nb);
+    AL(L1.dargs, 1);
+    AL(L1.zero_region, h->zero_bytes);
+    if (h->zero_large) AL(L1.zero_large, h->zero_large_bytes);
+    if (e == cudaSuccess) {
+      const ptrdiff_t dz = L1.zero_region - h->zero_region;
+      const ptrdiff_t dl = h->zero_large ? L1.zero_large - h->zero_large : 0;
+      auto rz = [&](auto* p) { return reinterpret_cast<decltype(p)>(reinterpret_cast<unsigned char*>(p) + dz); };
+      auto rl = [&](auto* p) { return reinterpret_cast<decltype(p)>(reinterpret_cast<unsigned char*>(p) + dl); };
+      L1.ctl = rz(h->ctl);
+      for (BSortBufs* b : {&L1.bs, &L1.bsL}) {
+        b->kB = kB;
+        b->pB = pB;
+      }
+      L1.bs.bcount = rz(h->bs.bcount);
+      L1.bs.cursor = rz(h->bs.cursor);
+      if (h->zero_large) {
+        L1.bsL.bcount = rl(h->bsL.bcount);
+        L1.bsL.cursor = rl(h->bsL.cursor);
+      }
+      for (CombBufs* c : {&L1.cb, &L1.cbL}) {
+        c->pinfo = pinfo;
+        c->istart = istart;
+        c->qkey = qkey;
+        c->qseg = qseg;
+        c->wkey = wkey;
+        c->wop = wop;
+        c->wval = wval;
+        c->wseg = wseg;
+      }
+      L1.cb.group_status = rz(h->cb.group_status);
+      if (h->zero_large) L1.cbL.group_status = rl(h->cbL.group_status);
+      h->nlanes = 2;
+      e = cudaMemset(L1.zero_region, 0, h->zero_bytes);
+      if (e == cudaSuccess && L1.zero_large) e = cudaMemset(L1.zero_large, 0, h->zero_large_bytes);
+      if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->back_stream, cudaStreamNonBlocking);
+    }
+  }
+  for (int l = 0; l < h->nlanes && e == cudaSuccess; ++l) {
+    e = cudaEventCreateWithFlags(&h->lanes[l].front_done, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&h->lanes[l].back_done, cudaEventDisableTiming);
+  }
 #undef AL
   if (e == cudaSuccess) e = cudaMallocHost(reinterpret_cast<void**>(&h->host_ctl), sizeof(BatchCtl) * RING);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->res_stream, cudaStreamNonBlocking);
@@ -408,6 +502,16 @@ int eirene_destroy(eirene_handle h) {
     if (g.graph) cudaGraphDestroy(g.graph);
   }
   if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
+  for (auto& L : h->lanes) {
+    for (GraphEntry* ge : {L.fg, L.bg})
+      for (int i = 0; i < MAX_GRAPHS; ++i) {
+        if (ge[i].exec) cudaGraphExecDestroy(ge[i].exec);
+        if (ge[i].graph) cudaGraphDestroy(ge[i].graph);
+      }
+    if (L.front_done) cudaEventDestroy(L.front_done);
+    if (L.back_done) cudaEventDestroy(L.back_done);
+  }
+  if (h->back_stream) cudaStreamDestroy(h->back_stream);
   if (h->h2d_stream) cudaStreamDestroy(h->h2d_stream);
   if (h->d2h_stream) cudaStreamDestroy(h->d2h_stream);
   for (int s = 0; s < HOST_SLOTS; ++s) {
@@ -463,14 +567,61 @@ static uint32_t size_bucket(uint32_t n, uint32_t max_batch) {
   return (uint32_t)std::min<uint64_t>(b, max_batch);
 }
 
+static cudaError_t capture_node(cudaStream_t s, cudaGraphNode_t* out) {
+  cudaStreamCaptureStatus cs;
+  const cudaGraphNode_t* deps = nullptr;
+  size_t nd = 0;
+  cudaError_t e = cudaStreamGetCaptureInfo(s, &cs, nullptr, nullptr, &deps, &nd);
+  if (e != cudaSuccess) return e;
+  if (nd != 1) return cudaErrorStreamCaptureInvalidated;
+  *out = deps[0];
+  return cudaSuccess;
+}
+
+}  // extern "C"
+
+// The graph of `table` for (size bucket, range), captured from `enqueue` on
+// first use (kept: up to MAX_GRAPHS per table).
+template <class F>
+static int get_graph(eirene_handle h, GraphEntry* table, uint32_t& next, uint32_t nk, bool range, bool want_args,
+                     F&& enqueue, GraphEntry** out) {
+  for (int i = 0; i < MAX_GRAPHS; ++i)
+    if (table[i].exec && table[i].n == nk && table[i].range == range) {
+      *out = &table[i];
+      return EIRENE_OK;
+    }
+  GraphEntry& e = table[next++ % MAX_GRAPHS];
+  if (e.exec) cudaGraphExecDestroy(e.exec);
+  if (e.graph) cudaGraphDestroy(e.graph);
+  e = GraphEntry{};
+  int launches = 0;
+  CK(cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeRelaxed));
+  cudaError_t ce = enqueue(h->cap_stream, want_args ? &e.args_node : nullptr, &launches);
+  cudaError_t ee = cudaStreamEndCapture(h->cap_stream, &e.graph);
+  if (ce != cudaSuccess) return cuda_fail(ce, "capture");
+  CK(ee);
+  CK(cudaGraphInstantiate(&e.exec, e.graph, 0));
+  e.n = nk;
+  e.range = range;
+  e.launches = launches;
+  *out = &e;
+  return EIRENE_OK;
+}
+
+extern "C" {
+
 static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
                        uint64_t* results, cudaStream_t st, uint64_t* vals_stage, uint64_t* ticket,
                        uint64_t* rkeys = nullptr, uint64_t* rvals = nullptr, uint32_t rcap = 0,
-                       bool prepare_only = false, bool prepare_range = false) {
+                       bool prepare_only = false, bool prepare_range = false, cudaStream_t* end_stream = nullptr) {
   const bool range = rkeys != nullptr || prepare_range;
   DeviceGuard dg_(h->cfg.device);
   CK(dg_.err);
   if (prepare_only && (!h->use_graphs || (h->cfg.flags & EIRENE_F_TIMING))) return EIRENE_OK;
+  static const bool dbg = std::getenv("EIRENE_DEBUG_SYNC") != nullptr;
+  const bool timing = (h->cfg.flags & EIRENE_F_TIMING) != 0;
+  // cross-batch pipelining (EIRENE_F_PIPELINE): graph replays only
+  const bool pipe = h->nlanes == 2 && h->use_graphs && !timing && !dbg;
   const uint64_t tk = prepare_only ? 0 : h->next_ticket++;
   Rec scratch_rec;
   Rec& r = prepare_only ? scratch_rec : h->ring[tk % RING];
@@ -479,95 +630,69 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     r.used = true;
   }
   r.n = n;
-  // Launches (grids, group count, distribution path) and the captured graph
+  // Launches (grids, group count, distribution path) and the captured graphs
   // are sized for n's size bucket; the kernels read the batch's own n from
   // BatchArgs.  Batches of varying size (the shards of a multi-GPU batch)
   // then replay a handful of graphs instead of capturing one per size.
   const uint32_t nk = size_bucket(n, h->cfg.max_batch);
-  r.timing = (h->cfg.flags & EIRENE_F_TIMING) != 0;
-  int launches = 0;
+  r.timing = timing;
   const uint32_t seq = ++h->batch_seq;
-  BatchCtl* ctl = h->ctl;
-  static const bool dbg = std::getenv("EIRENE_DEBUG_SYNC") != nullptr;
-  auto stage = [&](const char* name) {
+  auto stage = [&](const char* name, cudaStream_t s) {
     if (!dbg) return;
-    cudaError_t e = cudaStreamSynchronize(st);
+    cudaError_t e = cudaStreamSynchronize(s);
     std::fprintf(stderr, "[eirene] batch %u stage %s done: %s\n", seq, name, cudaGetErrorString(e));
-  };
-  // The pipeline: a tiny node that publishes this batch's pointers to the
-  // device-side BatchArgs, then every kernel of Alg.1 reading them from there.
-  auto last_node = [](cudaStream_t s, cudaGraphNode_t* out) -> cudaError_t {
-    cudaStreamCaptureStatus cs;
-    const cudaGraphNode_t* deps = nullptr;
-    size_t nd = 0;
-    cudaError_t e = cudaStreamGetCaptureInfo(s, &cs, nullptr, nullptr, &deps, &nd);
-    if (e != cudaSuccess) return e;
-    if (nd != 1) return cudaErrorStreamCaptureInvalidated;
-    *out = deps[0];
-    return cudaSuccess;
   };
   auto rec = [&](int i, cudaStream_t s) { cudaEventRecord(r.st[i], s); };
   BatchCtl* ctl_slot = h->ctl_ring + tk % RING;
-  uint4* zero16 = reinterpret_cast<uint4*>(h->zero_region);
-  uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
   const bool large = !bsort_fused(nk, h->num_sms);   // two-kernel bucket sort with 16384 bins (bsort.cu)
-  uint4* zero2 = reinterpret_cast<uint4*>(large ? h->zero_large : h->zero_region);
-  uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
-  const BSortBufs& bsn = large ? h->bsL : h->bs;
-  const CombBufs& cbn = large ? h->cbL : h->cb;
-  auto enqueue = [&](cudaStream_t s, bool timing, cudaGraphNode_t* args_node) -> cudaError_t {
-    set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(h->dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
+  // The front of a batch: a tiny node publishing its pointers to the lane's
+  // device-side BatchArgs (and zeroing the lane's control region), then the
+  // distribution and group kernels (sort Alg.1:10, combine Alg.1:11, partition
+  // Alg.1:3).  Nothing in it reads the tree.
+  auto front = [&](Lane& L, cudaStream_t s, cudaGraphNode_t* args_node, int* nl) -> cudaError_t {
+    uint4* zero16 = reinterpret_cast<uint4*>(L.zero_region);
+    const uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
+    uint4* zero2 = reinterpret_cast<uint4*>(large ? L.zero_large : L.zero_region);
+    const uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
+    set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(L.dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
                                                    zero_n16, zero2, zero2_n16, rkeys, rvals, rcap, n, h->phase);
-    ++launches;
+    ++*nl;
     if (args_node) {
-      cudaError_t e = last_node(s, args_node);
+      cudaError_t e = capture_node(s, args_node);
       if (e != cudaSuccess) return e;
     }
     if (timing) rec(0, s);
-    launch_bucket_sort(h->dargs, nk, h->cfg.key_lo, h->cfg.key_hi, bsn, ctl, h->num_sms, s, &launches);
-    stage("sort");
+    launch_bucket_sort(L.dargs, nk, h->cfg.key_lo, h->cfg.key_hi, large ? L.bsL : L.bs, L.ctl, h->num_sms, s, nl);
+    stage("sort", s);
     if (timing) rec(1, s);
-    launch_group(h->dargs, nk, bsn, cbn, h->t, ctl, h->num_sms, s, &launches);
-    const uint32_t* spay = h->bs.pB;
-    stage("group");
+    launch_group(L.dargs, nk, large ? L.bsL : L.bs, large ? L.cbL : L.cb, h->t, L.ctl, h->num_sms, s, nl);
+    stage("group", s);
+    return cudaGetLastError();
+  };
+  // The back: query (Alg.1:15-21; it checks the pool headroom first), range,
+  // update (Alg.1:23-46), RESULT_CAL (Alg.1:6) -- the kernels that read or
+  // change the tree.
+  auto back = [&](Lane& L, cudaStream_t s, int* nl) -> cudaError_t {
+    const uint32_t* spay = L.bs.pB;
     if (timing) rec(2, s);
-    launch_query(nk, h->cb, spay, h->dargs, h->t, ctl, h->num_sms, h->cfg.flags, h->cfg.iter_rgs, s, &launches);
-    if (range) launch_range(nk, h->cb, spay, h->bs.kB, h->dargs, h->t, ctl, h->num_sms, s, &launches);
-    stage("query");
+    launch_query(nk, L.cb, spay, L.dargs, h->t, L.ctl, h->num_sms, h->cfg.flags, h->cfg.iter_rgs, s, nl);
+    if (range) launch_range(nk, L.cb, spay, L.bs.kB, L.dargs, h->t, L.ctl, h->num_sms, s, nl);
+    stage("query", s);
     if (timing) rec(3, s);
-    launch_update(nk, h->cb, h->t, ctl, h->up, h->num_sms, s, &launches);
-    stage("update");
+    launch_update(nk, L.cb, h->t, L.ctl, h->up, h->num_sms, s, nl);
+    stage("update", s);
     if (timing) rec(4, s);
-    launch_result(spay, h->bs.kB, nk, h->cb, h->dargs, ctl, h->t.hdr, dbg ? 1 : 0, h->num_sms, s, &launches);
-    stage("result");
+    launch_result(spay, L.bs.kB, nk, L.cb, L.dargs, L.ctl, h->t.hdr, dbg ? 1 : 0, h->num_sms, s, nl);
+    stage("result", s);
     if (timing) rec(5, s);
     return cudaGetLastError();
   };
-  if (dbg || r.timing || !h->use_graphs) {   // per-stage events: direct launches
-    CK(enqueue(st, r.timing, nullptr));
-  } else {
-    // one captured graph per batch size; a replay updates only the args node
-    GraphEntry* g = nullptr;
-    for (auto& e : h->graphs)
-      if (e.exec && e.n == nk && e.range == range) g = &e;
-    if (!g) {
-      GraphEntry& e = h->graphs[h->next_graph++ % MAX_GRAPHS];
-      if (e.exec) cudaGraphExecDestroy(e.exec);
-      if (e.graph) cudaGraphDestroy(e.graph);
-      e = GraphEntry{};
-      CK(cudaStreamBeginCapture(h->cap_stream, cudaStreamCaptureModeRelaxed));
-      cudaError_t ce = enqueue(h->cap_stream, false, &e.args_node);
-      cudaError_t ee = cudaStreamEndCapture(h->cap_stream, &e.graph);
-      if (ce != cudaSuccess) return cuda_fail(ce, "capture");
-      CK(ee);
-      CK(cudaGraphInstantiate(&e.exec, e.graph, 0));
-      e.n = nk;
-      e.range = range;
-      e.launches = launches;
-      g = &e;
-    }
-    if (prepare_only) return EIRENE_OK;   // graph captured and instantiated, nothing launched
-    void* params[] = {&h->dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
+  auto set_args_params = [&](GraphEntry* g, Lane& L) -> int {
+    uint4* zero16 = reinterpret_cast<uint4*>(L.zero_region);
+    uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
+    uint4* zero2 = reinterpret_cast<uint4*>(large ? L.zero_large : L.zero_region);
+    uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
+    void* params[] = {&L.dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
                       const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
                       &zero2, &zero2_n16, &rkeys, &rvals, &rcap, &n, &h->phase};
     cudaKernelNodeParams p{};
@@ -578,10 +703,70 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     p.kernelParams = params;
     p.extra = nullptr;
     CK(cudaGraphExecKernelNodeSetParams(g->exec, g->args_node, &p));
-    CK(cudaGraphLaunch(g->exec, st));
-    launches = g->launches;
+    return EIRENE_OK;
+  };
+  int launches = 0;
+  cudaStream_t end = st;
+  if (pipe) {
+    // front of this batch on the caller's stream, back on the handle's back stream
+    auto fq = [&](cudaStream_t s, cudaGraphNode_t* an, int* nl) { return front(h->lanes[0], s, an, nl); };
+    if (prepare_only) {
+      for (int l = 0; l < 2; ++l) {
+        Lane& L = h->lanes[l];
+        GraphEntry *gf, *gb;
+        int rc = get_graph(h, L.fg, L.next_fg, nk, range, true,
+                           [&](cudaStream_t s, cudaGraphNode_t* an, int* nl) { return front(L, s, an, nl); }, &gf);
+        if (rc != EIRENE_OK) return rc;
+        rc = get_graph(h, L.bg, L.next_bg, nk, range, false,
+                       [&](cudaStream_t s, cudaGraphNode_t*, int* nl) { return back(L, s, nl); }, &gb);
+        if (rc != EIRENE_OK) return rc;
+      }
+      (void)fq;
+      return EIRENE_OK;
+    }
+    Lane& L = h->lanes[h->lane_seq++ & 1];
+    GraphEntry *gf, *gb;
+    int rc = get_graph(h, L.fg, L.next_fg, nk, range, true,
+                       [&](cudaStream_t s, cudaGraphNode_t* an, int* nl) { return front(L, s, an, nl); }, &gf);
+    if (rc != EIRENE_OK) return rc;
+    rc = get_graph(h, L.bg, L.next_bg, nk, range, false,
+                   [&](cudaStream_t s, cudaGraphNode_t*, int* nl) { return back(L, s, nl); }, &gb);
+    if (rc != EIRENE_OK) return rc;
+    if (L.used) CK(cudaStreamWaitEvent(st, L.back_done, 0));   // the back of batch b-2 released this lane
+    rc = set_args_params(gf, L);
+    if (rc != EIRENE_OK) return rc;
+    CK(cudaGraphLaunch(gf->exec, st));
+    CK(cudaEventRecord(L.front_done, st));
+    CK(cudaStreamWaitEvent(h->back_stream, L.front_done, 0));
+    CK(cudaGraphLaunch(gb->exec, h->back_stream));
+    CK(cudaEventRecord(L.back_done, h->back_stream));
+    L.used = true;
+    launches = gf->launches + gb->launches;
+    end = h->back_stream;
+  } else {
+    Lane& L = h->lanes[0];
+    if (h->nlanes == 2 && h->last_done) CK(cudaStreamWaitEvent(st, h->last_done, 0));   // pipelined batches first
+    auto whole = [&](cudaStream_t s, cudaGraphNode_t* an, int* nl) -> cudaError_t {
+      cudaError_t e = front(L, s, an, nl);
+      return e != cudaSuccess ? e : back(L, s, nl);
+    };
+    if (dbg || timing || !h->use_graphs) {   // per-stage events: direct launches
+      CK(whole(st, nullptr, &launches));
+    } else {
+      // one captured graph per batch size bucket; a replay updates only the args node
+      GraphEntry* g = nullptr;
+      int rc = get_graph(h, h->graphs, h->next_graph, nk, range, true, whole, &g);
+      if (rc != EIRENE_OK) return rc;
+      if (prepare_only) return EIRENE_OK;   // graph captured and instantiated, nothing launched
+      rc = set_args_params(g, L);
+      if (rc != EIRENE_OK) return rc;
+      CK(cudaGraphLaunch(g->exec, st));
+      launches = g->launches;
+    }
   }
-  CK(cudaEventRecord(r.done, st));
+  CK(cudaEventRecord(r.done, end));
+  if (h->nlanes == 2) h->last_done = r.done;
+  if (end_stream) *end_stream = end;
   r.launches = launches;
   h->launches += launches;
   h->modified = true;
@@ -647,9 +832,11 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
   CK(cudaEventRecord(h->h2d_done[s], h->h2d_stream));
   CK(cudaStreamWaitEvent(st, h->h2d_done[s], 0));
   uint64_t tk = 0;
-  int rc = submit_impl(h, h->st_ops + off, h->st_keys + off, vsrc, n, h->st_res + off, st, vstage, &tk);
+  cudaStream_t end = st;   // (the handle's back stream when pipelined)
+  int rc = submit_impl(h, h->st_ops + off, h->st_keys + off, vsrc, n, h->st_res + off, st, vstage, &tk, nullptr,
+                       nullptr, 0, false, false, &end);
   if (rc != EIRENE_OK) return rc;
-  CK(cudaEventRecord(h->comp_ev[s], st));
+  CK(cudaEventRecord(h->comp_ev[s], end));
   CK(cudaStreamWaitEvent(h->d2h_stream, h->comp_ev[s], 0));
   CK(cudaMemcpyAsync(results, h->st_res + off, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, h->d2h_stream));
   CK(cudaEventRecord(h->comp_done[s], h->d2h_stream));
@@ -713,6 +900,7 @@ int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out, u
   DeviceGuard dg_(h->cfg.device);
   CK(dg_.err);
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  if (h->nlanes == 2 && h->last_done) CK(cudaStreamWaitEvent(st, h->last_done, 0));   // pipelined batches first
   TreeHdr hdr;
   CK(cudaMemcpyAsync(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost, st));
   CK(cudaStreamSynchronize(st));
@@ -743,6 +931,23 @@ int eirene_set_flags(eirene_handle h, uint32_t flags) {
     if (g.graph) cudaGraphDestroy(g.graph);
     g = GraphEntry{};
   }
+  for (auto& L : h->lanes)
+    for (GraphEntry* ge : {L.fg, L.bg})
+      for (int i = 0; i < MAX_GRAPHS; ++i) {
+        if (ge[i].exec) cudaGraphExecDestroy(ge[i].exec);
+        if (ge[i].graph) cudaGraphDestroy(ge[i].graph);
+        ge[i] = GraphEntry{};
+      }
+  return EIRENE_OK;
+}
+
+int eirene_stream_wait_batch(eirene_handle h, uint64_t ticket, eirene_stream_t stream) {
+  if (!h) return EIRENE_EINVAL;
+  const Rec& r = h->ring[ticket % RING];
+  if (!r.used || r.ticket != ticket) return EIRENE_ESTATE;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  CK(cudaStreamWaitEvent(reinterpret_cast<cudaStream_t>(stream), r.done, 0));
   return EIRENE_OK;
 }
 
@@ -751,6 +956,7 @@ int eirene_get_info(eirene_handle h, eirene_tree_info* info) {
   DeviceGuard dg_(h->cfg.device);
   CK(dg_.err);
   TreeHdr hdr;
+  if (h->back_stream) CK(cudaStreamSynchronize(h->back_stream));
   CK(cudaMemcpy(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost));
   info->height = (uint32_t)(hdr.root_word >> 32);
   info->root = (uint32_t)hdr.root_word;
@@ -905,6 +1111,7 @@ int eirene_batch_status_async(eirene_handle h, uint64_t ticket, int32_t* status_
   if (!r.used || r.ticket != ticket) return EIRENE_ESTATE;
   DeviceGuard dg_(h->cfg.device);
   CK(dg_.err);
+  CK(cudaStreamWaitEvent(reinterpret_cast<cudaStream_t>(stream), r.done, 0));   // (pipelined: ends elsewhere)
   CK(cudaMemcpyAsync(status_dev, &h->ctl_ring[ticket % RING].status, sizeof(int32_t), cudaMemcpyDeviceToDevice,
                      reinterpret_cast<cudaStream_t>(stream)));
   return EIRENE_OK;

@@ -269,6 +269,27 @@ inline int per_device(int (&cache)[MAX_DEVICES], F compute) {
   return cache[d] - 1;
 }
 
+// Worst-case node demand of the update kernel (EFULL pre-check, SURVEY
+// §8(b)), checked by the query kernel before anything changes (the front of a
+// pipelined batch must not read the tree): new leaves <= issued writes; new inner nodes at level l+1 <=
+// min(N_l, (I_l + N_l) / 8) because every node created by an even multi-way
+// split keeps >= 8 children, plus root growth.
+__device__ __forceinline__ bool headroom_ok(const Tree& t, uint32_t nw) {
+  const TreeHdr* h = t.hdr;
+  const uint32_t height = (uint32_t)(h->root_word >> 32);
+  unsigned long long need_leaf = nw;
+  unsigned long long N = nw, inner = 0;
+  for (uint32_t l = 0; l + 1 < height && N > 0; ++l) {
+    unsigned long long I = h->level_count[l];
+    unsigned long long Nn = min(N, (I + N) / 8 + 1);
+    inner += Nn;
+    N = Nn;
+  }
+  inner += 2 * (N + 1) + 64;   // new root levels
+  return (unsigned long long)h->leaf_count + need_leaf <= t.leaf_cap &&
+         (unsigned long long)h->inner_count + inner <= t.inner_cap;
+}
+
 // ------------------------------------------------------------ programmatic dependent launch
 // Kernels 2.. of a batch are launched with programmatic stream serialization
 // (PDL, EIRENE_PDL=1): a kernel may be scheduled while its predecessor drains,

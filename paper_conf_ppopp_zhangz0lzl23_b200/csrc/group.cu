@@ -695,26 +695,6 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
   return passes & 1;
 }
 
-// Worst-case node demand of the update kernel (EFULL pre-check, SURVEY
-// §8(b)): new leaves <= issued writes; new inner nodes at level l+1 <=
-// min(N_l, (I_l + N_l) / 8) because every node created by an even multi-way
-// split keeps >= 8 children, plus root growth.
-__device__ bool headroom_ok(const Tree& t, uint32_t nw) {
-  const TreeHdr* h = t.hdr;
-  const uint32_t height = (uint32_t)(h->root_word >> 32);
-  unsigned long long need_leaf = nw;
-  unsigned long long N = nw, inner = 0;
-  for (uint32_t l = 0; l + 1 < height && N > 0; ++l) {
-    unsigned long long I = h->level_count[l];
-    unsigned long long Nn = min(N, (I + N) / 8 + 1);
-    inner += Nn;
-    N = Nn;
-  }
-  inner += 2 * (N + 1) + 64;   // new root levels
-  return (unsigned long long)h->leaf_count + need_leaf <= t.leaf_cap &&
-         (unsigned long long)h->inner_count + inner <= t.inner_cap;
-}
-
 struct GroupArgs {
   const BatchArgs* A;
   uint64_t* kA;                 // bucketed requests (bsort scatter output)
@@ -1205,13 +1185,12 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       const uint32_t seg0 = (uint32_t)(excl >> 31), w0 = (uint32_t)(excl & ((1u << 31) - 1));
       S.seg0 = seg0;
       S.w0 = w0;
-      if (b + 1 == g.nb) {   // last bucket: batch totals + headroom check
+      if (b + 1 == g.nb) {   // last bucket: batch totals (the pool headroom is checked by the query kernel)
         const uint32_t nseg = seg0 + c_nh, nw = w0 + c_nw;
         ctl->nseg = nseg;
         ctl->nw = nw;
         ctl->nq = nseg - nw;
         g.istart[nseg] = g.gstart[g.nb];   // point requests (range queries are not sorted)
-        if (!headroom_ok(g.t, nw)) ctl->status = EIRENE_EFULL;
       }
     }
   }

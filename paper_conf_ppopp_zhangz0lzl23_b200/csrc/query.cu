@@ -164,6 +164,12 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
+  // pool headroom for the batch's worst case (every CTA computes the same
+  // answer from the same tree header: none of them changes anything if it fails)
+  if (!headroom_ok(t, nw)) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = EIRENE_EFULL;
+    return;
+  }
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
   const uint32_t stride = gridDim.x * blockDim.x;
@@ -224,6 +230,10 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
   if (ctl->invalid || ctl->status != 0) return;
   uint64_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw;
+  if (!headroom_ok(t, nw)) {
+    if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = EIRENE_EFULL;
+    return;
+  }
   const uint32_t rq = (nq + 31) / 32, nrg = rq + (nw + 31) / 32;
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;

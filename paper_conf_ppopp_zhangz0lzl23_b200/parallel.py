@@ -121,7 +121,7 @@ class ShardedEirene:
         tk = None
         if nrecv:
             tk = self.engine.submit(rops, rkeys, rvals, rres)
-            self.engine.status_async(tk, status)
+            self.engine.status_async(tk, status)   # (orders the current stream after the batch)
         if P > 1:
             # EFULL / EINTERNAL / CUDA failure on one shard fails the global batch on every rank
             # (statuses are <= 0: the minimum is the error, if any) -- no rank raises alone

@@ -42,7 +42,7 @@ class EireneTree:
     def __init__(self, max_keys: int = 1 << 24, max_batch: int = 1 << 20, device: int | None = None,
                  retry_threshold: int = 4, regroup: bool = True, stats: bool = True, force_stm: bool = False,
                  timing: bool = False, key_lo: int = 0, key_hi: int = U64_MAX, iterwarp: bool = False,
-                 iter_rgs: int = 0):
+                 iter_rgs: int = 0, pipeline: bool = False):
         L = _ffi.lib()
         if device is None:
             device = torch.cuda.current_device()
@@ -55,7 +55,7 @@ class EireneTree:
         cfg.retry_threshold = retry_threshold
         cfg.flags = ((_ffi.EIRENE_F_REGROUP if regroup else 0) | (_ffi.EIRENE_F_STATS if stats else 0) |
                      (_ffi.EIRENE_F_FORCE_STM if force_stm else 0) | (_ffi.EIRENE_F_TIMING if timing else 0) |
-                     (_ffi.EIRENE_F_ITERWARP if iterwarp else 0))
+                     (_ffi.EIRENE_F_ITERWARP if iterwarp else 0) | (_ffi.EIRENE_F_PIPELINE if pipeline else 0))
         cfg.iter_rgs = iter_rgs
         cfg.key_lo = key_lo
         cfg.key_hi = key_hi
@@ -153,6 +153,11 @@ class EireneTree:
                                                self._stream(stream), ctypes.byref(tk)), "eirene_submit_batch_host")
         return tk.value
 
+    def stream_wait(self, ticket: int, stream=None):
+        """Order `stream` (default: current) after batch `ticket` on the device (needed with pipeline=True
+        before consuming its results there)."""
+        check(self._L.eirene_stream_wait_batch(self._h, ticket, self._stream(stream)), "eirene_stream_wait_batch")
+
     def results(self, ticket: int, raise_on_error: bool = True) -> dict:
         st = _ffi.eirene_batch_stats()
         rc = self._L.eirene_results(self._h, ticket, ctypes.byref(st))
@@ -191,7 +196,7 @@ class EireneTree:
         f = self.cfg.flags
         for on, bit in ((regroup, _ffi.EIRENE_F_REGROUP), (stats, _ffi.EIRENE_F_STATS),
                         (force_stm, _ffi.EIRENE_F_FORCE_STM), (timing, _ffi.EIRENE_F_TIMING),
-                        (iterwarp, _ffi.EIRENE_F_ITERWARP)):
+                        (iterwarp, _ffi.EIRENE_F_ITERWARP)):   # (pipelining is fixed at create)
             if on is not None:
                 f = (f | bit) if on else (f & ~bit)
         self.cfg.flags = f

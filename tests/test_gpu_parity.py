@@ -544,3 +544,43 @@ def test_structural_counts_and_device_time(dev):
             assert want_ins == 0 and want_delp == 0
         assert 0 < st["device_ns"] < 10**9
     t.close()
+
+
+@pytest.mark.parametrize("cfg", [2, 3])
+def test_pipelined_batches_in_flight(dev, cfg):
+    """EIRENE_F_PIPELINE (§8(f) NEXT(3)): the front (sort, combine, partition) of
+    batch b+1 overlaps the back (query, update, RESULT_CAL) of batch b.  Many
+    batches are submitted before any result is read; every result and the final
+    state must equal the oracle's (backs in submission order), and a
+    non-pipelined batch and a scan afterwards must see every pipelined one."""
+    rng = np.random.default_rng(40 + cfg)
+    w = W.Workload(cfg, tree=1 << 16, batch=1 << 14,
+                   fracs={W.QUERY: 0.5, W.UPDATE: 0.25, W.INSERT: 0.2, W.DELETE: 0.05})
+    t = make_tree(dev, w.keys, w.vals, max_keys=1 << 18, max_batch=1 << 14, pipeline=True)
+    ref = oracle.MapOracle(); ref.load(w.keys, w.vals)
+    nb = 9
+    host = [w.batch_arrays(b) for b in range(nb)]
+    outs, tks = [], []
+    for b in range(nb):
+        n = (1 << 14) - int(rng.integers(0, 3000))   # ragged sizes: several graph buckets
+        o, k, v = (T(a[:n], dev) for a in host[b])
+        res = torch.empty(n, dtype=torch.uint64, device=dev)
+        tks.append(t.submit(o, k, v, res))
+        outs.append((res, n, (o, k, v)))
+    for b in range(nb):
+        st = t.results(tks[b])
+        res, n, _ = outs[b]
+        want = ref.apply(host[b][0][:n], host[b][1][:n], host[b][2][:n])
+        got = res.cpu().numpy()
+        assert np.array_equal(got, want), f"batch {b}: {int(np.sum(got != want))} differ"
+    k, v = t.scan()
+    rk, rv = ref.scan()
+    assert np.array_equal(k.cpu().numpy(), rk) and np.array_equal(v.cpu().numpy(), rv)
+    # the host-buffer path on a pipelined handle
+    o, k_, v_ = w.batch_arrays(50)
+    pin = [torch.from_numpy(a).pin_memory() for a in (o, k_, v_)]
+    hres = torch.empty(o.size, dtype=torch.uint64).pin_memory()
+    t.results(t.submit_host(*pin, hres))
+    assert np.array_equal(hres.numpy(), ref.apply(o, k_, v_))
+    assert t.check_invariants() == (0, ref.size())
+    t.close()
