@@ -167,31 +167,36 @@ def random_access_counts(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, 
             "writes": wk.size / n, "bio": (n * 17 + ups * 8) / n}
 
 
-def probe_random_access(dev, stream, pool_gib: int = 4, n: int = 1 << 24, reps: int = 3) -> dict:
-    """Random accesses per second of this GPU's HBM (eirene_probe_gather: 128 B
-    line reads, 32 B sector reads, 32 B sector writes over a pool >> L2),
-    best of `reps`, CUDA events on the launching stream."""
+def probe_random_access(dev, stream, pool_bytes: int, n: int = 1 << 24, n_leaf: int = 1 << 20,
+                        reps: int = 3) -> dict:
+    """Random accesses per second of this GPU's HBM (eirene_probe_gather) over a
+    pool the size of the leaf pool (power of two >= the tree's leaf blocks, so the
+    TLB reach matches): R128 = 128 B line reads, R32 = 32 B sector reads, R32w =
+    32 B sector writes (uniformly random), R_leaf = the query kernel's leaf access
+    (key line + dependent value sector of a 256 B block) at a key-sorted batch's
+    order and density (n_leaf blocks visited ascending).  Best of `reps`, CUDA
+    events on the launching stream."""
     import ctypes
 
     import torch
 
     from paper_conf_ppopp_zhangz0lzl23_b200 import _ffi
     L = _ffi.lib()
-    pool = torch.empty(pool_gib << 30, dtype=torch.uint8, device=dev)
-    out = {}
-    for kind, name in ((0, "R128"), (1, "R32"), (2, "R32w")):
+    pool = torch.empty(pool_bytes, dtype=torch.uint8, device=dev)
+    out = {"pool_bytes": pool_bytes}
+    for kind, name, cnt in ((0, "R128", n), (1, "R32", n), (2, "R32w", n), (3, "R_leaf", n_leaf)):
         best = 0.0
         for r in range(reps + 1):
             e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            rc = L.eirene_probe_gather(ctypes.c_void_p(pool.data_ptr()), pool.numel(), n, kind, 77 + r,
+            rc = L.eirene_probe_gather(ctypes.c_void_p(pool.data_ptr()), pool.numel(), cnt, kind, 77 + r,
                                        ctypes.c_void_p(stream.cuda_stream))
             e1.record(stream)
             stream.synchronize()
             if rc != 0:
                 raise RuntimeError(f"eirene_probe_gather rc={rc}")
             if r:   # first launch is a warm-up
-                best = max(best, n / (e0.elapsed_time(e1) * 1e-3))
+                best = max(best, cnt / (e0.elapsed_time(e1) * 1e-3))
         out[name] = best
     del pool
     return out
@@ -717,20 +722,38 @@ def run_ours(args):
                 "stage_ms": ms, "algorithmic_bytes_per_launch": bytes_per, "peak_source": peaks["source"]}
         # whole-path random-access roofline (BASELINE north_star) on
         # the bulk-loaded shape: 1 / (L/R128 + S/R32 + Wr/R32w + B_io/BW) req/s
-        if not cap and not per_tree and args.ra_probe:
-            rates = probe_random_access(dev, stream)
+        if not cap and not per_tree:
             cs = [random_access_counts(wls[0].keys, *host_batches[b][:2], 16)
                   for b in range(args.warmup, min(nb, args.warmup + 4))]
             c = {k: float(np.mean([x[k] for x in cs])) for k in cs[0]}
-            t_req = (c["lines"] / rates["R128"] + c["sectors"] / rates["R32"] + c["writes"] / rates["R32w"]
-                     + c["bio"] / (peaks["hbm_gbs"] * 1e9))
+            # whole-path HBM streaming roofline: algorithmic bytes per request =
+            # B_io + leaf lines x 128 + value sectors x 32 + written sectors x 32, at the measured peak
+            b_req = c["bio"] + 128 * c["lines"] + 32 * c["sectors"] + 32 * c["writes"]
+            stream_roof = peaks["hbm_gbs"] * 1e9 / b_req / 1e9
+            roof["streaming"] = {"roofline_Greq_s": stream_roof, "frac": value / stream_roof,
+                                 "bytes_per_request": b_req}
+        if not cap and not per_tree and args.ra_probe:
+            n_leaves = (tree_n + 15) // 16
+            pool_bytes = 1 << int(np.ceil(np.log2(max(n_leaves * 256, 1 << 20))))
+            n_leaf = int(round(c["lines"] * batch_n))
+            rates = probe_random_access(dev, stream, pool_bytes, n_leaf=n_leaf)
+            # whole path: every leaf visited (key line + one value sector: R_leaf), the further
+            # value sectors (R32), the written sectors (R32w), the streamed bytes (BW)
+            t_req = (c["lines"] / rates["R_leaf"] + max(0.0, c["sectors"] - c["lines"]) / rates["R32"]
+                     + c["writes"] / rates["R32w"] + c["bio"] / (peaks["hbm_gbs"] * 1e9))
+            q_rate = n_leaf / (stage_ms[2] * 1e-3)   # the query kernel's leaf visits per second
             rar = {"roofline_Greq_s": 1.0 / t_req / 1e9, "achieved_Greq_s": value,
                    "frac": value / (1.0 / t_req / 1e9),
+                   "query_kernel": {"leaf_visits_per_s": q_rate, "probe_R_leaf": rates["R_leaf"],
+                                    "frac": q_rate / rates["R_leaf"]},
+                   "streaming_frac": value / stream_roof,
                    "per_request": {"leaf_lines": c["lines"], "value_sectors": c["sectors"],
                                    "value_writes": c["writes"], "streamed_bytes": c["bio"]},
                    "rates_per_s": rates,
-                   "probe": "eirene_probe_gather: 2^24 uniformly random 128 B line reads / 32 B sector reads / "
-                            "32 B sector writes over a 4 GiB pool, best of 3, CUDA events"}
+                   "probe": f"eirene_probe_gather over a {pool_bytes >> 20} MiB pool (the leaf pool's size, "
+                            "power-of-two masks): 2^24 uniformly random 128 B line reads / 32 B sector reads / "
+                            f"32 B sector writes, and {n_leaf} leaf visits (128 B key line + dependent 32 B value "
+                            "sector) in key-sorted batch order; best of 3, CUDA events"}
 
     if rank == 0 and roof is None and not cap and not per_tree:
         # the query kernel of rank 0's shard (N > 1, or a tree too large for the full oracle): its

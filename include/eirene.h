@@ -260,13 +260,16 @@ int eirene_set_flags(eirene_handle h, uint32_t flags);
 
 /* Measurement helper (not part of the request path): launches one random-access
  * probe on `stream` over the caller's device buffer pool_dev[pool_bytes]
- * (128 B aligned, ideally far larger than L2): n uniformly random accesses,
- * kind 0 = 128 B line reads (the leaf key line of a lookup), 1 = 32 B sector
- * reads (a value sector), 2 = 32 B sector writes (an in-place value update).
- * The caller times it with events on `stream`; accesses/s are the
- * denominators of the random-access roofline of SURVEY §8(d) (BASELINE
- * north_star).  Kind 2 overwrites pool contents.  EINVAL for a null / short /
- * misaligned pool or an unknown kind; ECUDA if the launch fails. */
+ * (256 B aligned, a power of two bytes): n accesses, kind 0 = uniformly random
+ * 128 B line reads, 1 = random 32 B sector reads (a value sector), 2 = random
+ * 32 B sector writes (an in-place value update), 3 = the query kernel's leaf
+ * access: the 128 B key line of a 256 B leaf block then, dependent on it, one
+ * 32 B sector of the block's value line, at a key-sorted batch's order and
+ * density (access i visits block ~ i * blocks / n, ascending).  The caller
+ * times it with events on `stream`; accesses/s are the denominators of the
+ * random-access roofline of SURVEY §8(d) (BASELINE north_star).  Kind 2
+ * overwrites pool contents.  EINVAL for a null / misaligned / non-power-of-two
+ * pool or an unknown kind; ECUDA if the launch fails. */
 int eirene_probe_gather(void* pool_dev, uint64_t pool_bytes, uint32_t n, int kind, uint64_t seed,
                         eirene_stream_t stream);
 

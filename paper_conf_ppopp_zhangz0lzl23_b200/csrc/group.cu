@@ -70,6 +70,12 @@ struct GSmem {
   uint64_t hk;                 // split-off hot key of an oversized group
   unsigned long long prof_t[2];  // EIRENE_GROUP_PROF timestamps (diagnostic)
   uint32_t* hot_bits;          // its timestamp bitmap slot (null: none free)
+  // hot_run_sort: timestamp-bucket counters, provisional payloads, the run's other keys
+  uint32_t tcnt[SB_N + 1];
+  uint32_t tpay[G_CAP];
+  uint64_t ck[32];
+  uint32_t cp[32];
+  uint32_t hr_lt, hr_eq, hr_nc, hr_cm;
 };
 
 __device__ __forceinline__ bool kp_less(uint64_t ka, uint32_t pa, uint64_t kb, uint32_t pb) {
@@ -151,7 +157,137 @@ constexpr uint32_t FAST_SB = 32;
 #define GROUP_WARP_SB 256   // A/B builds: -DGROUP_WARP_SB=n; cfg3 1024 -> 256: 3.43 -> 3.64 Greq/s
 #endif
 constexpr uint32_t WARP_SB = GROUP_WARP_SB;
-__device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, GSmem& S) {
+// Exclusive scan of a[0..SB_N) in place (SB_N / G_THREADS per thread), a[SB_N] = total.
+__device__ void block_scan_sbn(uint32_t* a, GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  constexpr int PER = SB_N / G_THREADS;
+  uint32_t loc[PER], sum = 0;
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    loc[j] = a[tid * PER + j];
+    sum += loc[j];
+  }
+  uint32_t x = sum;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) S.wsum[warp] = x;
+  __syncthreads();
+  uint32_t run = x - sum;
+  for (int w = 0; w < warp; ++w) run += S.wsum[w];
+#pragma unroll
+  for (int j = 0; j < PER; ++j) {
+    a[tid * PER + j] = run;
+    run += loc[j];
+  }
+  if (tid == G_THREADS - 1) a[SB_N] = run;
+  __syncthreads();
+}
+
+// A big sub-bucket S.k/S.p[lo, lo + m) (m <= G_CAP) dominated by one key hk
+// (a hot key: Zipf).  hk's requests -- equal keys -- only need timestamp
+// order: a counting sort on the top SB_BITS bits of the timestamp, then a rank
+// fix inside each timestamp bucket; the few other requests of the sub-bucket
+// (<= 32) are ranked against each other directly.  About ten CTA barriers
+// instead of a bitonic network's log2(m)(log2(m)+1)/2 (78 at m = 4096).
+// Returns false, having changed nothing, if the sub-bucket holds more than 32
+// other requests or a timestamp bucket more than FAST_SB (the caller then
+// sorts it with the bitonic network).  CTA-uniform.
+constexpr uint32_t FAST_SB_ = 32;
+__device__ __noinline__ bool hot_run_sort(uint32_t lo, uint32_t m, int tsbits, GSmem& S) {
+  const int tid = threadIdx.x, lane = tid & 31;
+  const uint64_t hk = S.k[lo + m / 2];   // a member: the dominant key with high probability
+  uint64_t kr[G_ITEMS];
+  uint32_t pr[G_ITEMS], r[G_ITEMS];
+  uint32_t lt = 0, eq = 0;
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = tid + j * G_THREADS;
+    const bool v = i < m;
+    kr[j] = v ? S.k[lo + i] : hk;
+    pr[j] = v ? S.p[lo + i] : 0u;
+    lt += (v && kr[j] < hk) ? 1u : 0u;
+    eq += (v && kr[j] == hk) ? 1u : 0u;
+  }
+  if (tid == 0) {
+    S.hr_lt = 0;
+    S.hr_eq = 0;
+    S.hr_nc = 0;
+    S.hr_cm = 0;
+  }
+  for (int i = tid; i <= SB_N; i += G_THREADS) S.tcnt[i] = 0;
+  __syncthreads();
+  lt = __reduce_add_sync(FULL, lt);
+  eq = __reduce_add_sync(FULL, eq);
+  if (lane == 0) {
+    if (lt) atomicAdd(&S.hr_lt, lt);
+    if (eq) atomicAdd(&S.hr_eq, eq);
+  }
+  const int tsh = tsbits > SB_BITS ? tsbits - SB_BITS : 0;
+  uint32_t cm = 0;
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = tid + j * G_THREADS;
+    r[j] = 0;
+    if (i < m) {
+      if (kr[j] == hk) {
+        r[j] = atomicAdd(&S.tcnt[(pr[j] >> 2) >> tsh], 1u);
+        cm = max(cm, r[j] + 1);
+      } else {
+        const uint32_t c = atomicAdd(&S.hr_nc, 1u);
+        if (c < 32) {
+          S.ck[c] = kr[j];
+          S.cp[c] = pr[j];
+        }
+      }
+    }
+  }
+  cm = __reduce_max_sync(FULL, cm);
+  if (lane == 0 && cm) atomicMax(&S.hr_cm, cm);
+  __syncthreads();
+  const uint32_t nlt = S.hr_lt, neq = S.hr_eq, nc = S.hr_nc;
+  if (nc > 32 || S.hr_cm > FAST_SB_) {
+    __syncthreads();   // (everyone read the verdict before the caller reuses S)
+    return false;
+  }
+  block_scan_sbn(S.tcnt, S);   // timestamp bucket starts among hk's requests
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j)
+    if (tid + j * G_THREADS < m && kr[j] == hk) S.tpay[S.tcnt[(pr[j] >> 2) >> tsh] + r[j]] = pr[j];
+  __syncthreads();
+  uint32_t pos[G_ITEMS];
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j) {
+    const uint32_t i = tid + j * G_THREADS;
+    pos[j] = 0xFFFFFFFFu;
+    if (i >= m) continue;
+    if (kr[j] == hk) {
+      const uint32_t b = (pr[j] >> 2) >> tsh, s0 = S.tcnt[b], s1 = S.tcnt[b + 1];
+      uint32_t less = 0;
+      for (uint32_t x = s0; x < s1; ++x) less += S.tpay[x] < pr[j];
+      pos[j] = lo + nlt + s0 + less;
+    } else {
+      const bool low = kr[j] < hk;
+      uint32_t less = 0;
+      for (uint32_t x = 0; x < nc; ++x)
+        less += ((S.ck[x] < hk) == low && kp_less(S.ck[x], S.cp[x], kr[j], pr[j])) ? 1u : 0u;
+      pos[j] = (low ? lo : lo + nlt + neq) + less;
+    }
+  }
+  __syncthreads();   // every read of the run done before it is rewritten
+#pragma unroll
+  for (int j = 0; j < G_ITEMS; ++j)
+    if (pos[j] != 0xFFFFFFFFu) {
+      S.k[pos[j]] = kr[j];
+      S.p[pos[j]] = pr[j];
+    }
+  __syncthreads();
+  return true;
+}
+
+__device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, int tsbits, GSmem& S) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t C = 32u * ((cnt + G_THREADS - 1) / G_THREADS);
   const uint32_t wb = warp * C;
@@ -269,7 +405,7 @@ __device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, 
   __syncthreads();
   for (uint32_t e = 0; e < nbig; ++e) {
     const uint32_t x = S.whist[e], lo = S.sb[x], m = S.sb[x + 1] - lo;
-    if (m > WARP_SB) bitonic_run<true>(lo, m, tid, G_THREADS, S);
+    if (m > WARP_SB && !hot_run_sort(lo, m, tsbits, S)) bitonic_run<true>(lo, m, tid, G_THREADS, S);
   }
   __syncthreads();
 }
@@ -445,7 +581,7 @@ __device__ void l2_pass_pay(const uint32_t* ps, uint32_t* pd, uint32_t cnt, int 
 // PART_MAX parts (a bin of nearly G_CAP requests).
 constexpr uint32_t PART_MAX = 64;
 __device__ bool range_partition_sort(const uint64_t* ks, const uint32_t* ps, uint64_t* kd, uint32_t* pd,
-                                     uint32_t cnt, uint64_t kmin, uint64_t range, GSmem& S) {
+                                     uint32_t cnt, uint64_t kmin, uint64_t range, int tsbits, GSmem& S) {
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const int bits = 64 - __clzll((long long)range);
   const int shift = bits > SB_BITS ? bits - SB_BITS : 0;
@@ -532,7 +668,7 @@ __device__ bool range_partition_sort(const uint64_t* ks, const uint32_t* ps, uin
     const uint32_t b0 = S.dhist[q], m = S.dhist[q + 1] - b0;
     __syncthreads();   // (every thread read the part bounds before smem_sort reuses S)
     if (m < 2) continue;
-    smem_sort(kd + b0, pd + b0, m, S);
+    smem_sort(kd + b0, pd + b0, m, tsbits, S);
     for (uint32_t i = tid; i < m; i += G_THREADS) {
       kd[b0 + i] = S.k[i];
       pd[b0 + i] = S.p[i];
@@ -653,7 +789,7 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
     }
     __syncthreads();
     const uint32_t o = S.r_nh, h = S.r_lw, lo = S.r_nw;
-    if (o > 1) smem_sort(S.k, S.p, o, S);
+    if (o > 1) smem_sort(S.k, S.p, o, tsbits, S);
     __syncthreads();
     if (bits) {   // SPLIT: the rest stays sorted in S.k / S.p, hk in the bitmap
       if (tid == 0) {
@@ -681,7 +817,7 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
     __syncthreads();
     return 1;
   }
-  if (range && range_partition_sort(ks, ps, kd, pd, cnt, kmin, range, S)) return 1;
+  if (range && range_partition_sort(ks, ps, kd, pd, cnt, kmin, range, tsbits, S)) return 1;
   const int tpass = (tsbits + 7) / 8;
   const int passes = tpass + (range ? (64 - __clzll((long long)range) + 7) / 8 : 0);
   for (int pass = 0; pass < passes; ++pass) {
@@ -1065,7 +1201,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       S.k[0] = g.kA[base];
       S.p[0] = g.pA[base];
     } else if (cnt > 1) {
-      smem_sort(g.kA + base, g.pA + base, cnt, S);
+      smem_sort(g.kA + base, g.pA + base, cnt, g.tsbits, S);
     }
     __syncthreads();
     K = S.k;
