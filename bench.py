@@ -105,11 +105,13 @@ def spread(ms: np.ndarray, source: str) -> dict:
 
 
 
-def algorithmic_bytes_query(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, per_leaf: int) -> dict:
+def algorithmic_bytes_query(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, per_leaf: int,
+                            kb: int = 8) -> dict:
     """Algorithmic HBM bytes of the QUERY kernel for one cfg2 batch:
     per issued query 8 B key + 4 B seg read + 8 B result write, one 128 B leaf key
     line per distinct leaf touched, one 32 B value sector per distinct (leaf, sector)
-    hit.  Valid for batches on the bulk-loaded shape (cfg2 never splits)."""
+    hit.  Valid for batches on the bulk-loaded shape (cfg2 never splits).  kb = bytes per key
+    and value (8; 4 for the 32-bit build: a 64 B key line, 8 values per sector)."""
     uk = W.sorted_unique(keys)
     issued_w = np.zeros(uk.size, bool)
     w = ops != W.QUERY
@@ -122,10 +124,11 @@ def algorithmic_bytes_query(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarra
     leaf = pos // per_leaf
     slot = pos % per_leaf
     lines = W.sorted_unique(leaf).size
-    sectors = W.sorted_unique(leaf[hit] * 4 + slot[hit] // 4).size
+    vps = 32 // kb
+    sectors = W.sorted_unique(leaf[hit] * 4 + slot[hit] // vps).size
     nq = qk.size
     return {"issued_q": int(nq), "leaf_lines": int(lines), "value_sectors": int(sectors),
-            "bytes": int(nq * (8 + 4 + 8) + lines * 128 + sectors * 32)}
+            "bytes": int(nq * (kb + 4 + kb) + lines * 16 * kb + sectors * 32)}
 
 
 def algorithmic_bytes_range(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, vals: np.ndarray,
@@ -149,7 +152,8 @@ def algorithmic_bytes_range(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarra
             "bytes": int(nr * (1 + 8 + 8 + 8) + int(cnt.sum()) * 16 + lines * 128 + sectors * 32)}
 
 
-def random_access_counts(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, per_leaf: int) -> dict:
+def random_access_counts(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, per_leaf: int,
+                         kb: int = 8) -> dict:
     """Random HBM touches of one batch on the bulk-loaded shape:
     every issued request (one per distinct key, query or write) reads its leaf's
     128 B key line (distinct leaves counted once) and, if its key is present,
@@ -163,8 +167,10 @@ def random_access_counts(loaded: np.ndarray, ops: np.ndarray, keys: np.ndarray, 
     leaf = pos // per_leaf
     n = keys.size
     ups = int(np.sum((ops == W.UPDATE) | (ops == W.INSERT)))
-    return {"lines": W.sorted_unique(leaf).size / n, "sectors": W.sorted_unique(leaf[hit] * 4 + (pos[hit] % per_leaf) // 4).size / n,
-            "writes": wk.size / n, "bio": (n * 17 + ups * 8) / n}
+    vps = 32 // kb
+    return {"lines": W.sorted_unique(leaf).size / n,
+            "sectors": W.sorted_unique(leaf[hit] * 4 + (pos[hit] % per_leaf) // vps).size / n,
+            "writes": wk.size / n, "bio": (n * (1 + 2 * kb) + ups * kb) / n, "line_bytes": 16 * kb}
 
 
 def probe_random_access(dev, stream, pool_bytes: int, n: int = 1 << 24, n_leaf: int = 1 << 20,
@@ -302,6 +308,21 @@ def run_ours(args):
     if args.mix:   # YCSB-like mix override (cfg5: A, B, C, U)
         C["fracs"], C["dist"] = W.MIXES[args.mix]
     wkw = {"fracs": C["fracs"], "dist": C["dist"]}
+    # cfg7: the 32-bit key / value build, libeirene32.so
+    kbits = C.get("key_bits", 64)
+    kb = kbits // 8
+    kdt = torch.uint32 if kbits == 32 else torch.uint64
+    if kbits == 32 and world > 1:
+        raise SystemExit("the 32-bit key build runs on one GPU (multi-GPU routing is 64-bit)")
+
+    def tnp(a):   # host array -> tensor of the key width (ops stay u8)
+        return torch.from_numpy(a.astype(np.uint32) if (kbits == 32 and a.dtype == np.uint64) else a)
+
+    def widen_np(r):   # results of the 32-bit build as the oracle's u64 (NOT_FOUND = all ones)
+        r = np.asarray(r).astype(np.uint64)
+        if kbits == 32:
+            r[r == np.uint64(0xFFFFFFFF)] = np.uint64(0xFFFFFFFFFFFFFFFF)
+        return r
     tree_n, batch_n = C["tree"], C["batch"]
     if args.tree:
         tree_n = args.tree
@@ -323,7 +344,8 @@ def run_ours(args):
 
     # query traversal: the default (one key-sorted request per thread, path
     # sharing) or the paper's iteration warps + range field (ablation)
-    qmode = {"iterwarp": args.query_mode == "iterwarp", "iter_rgs": args.iter_rgs, "pipeline": bool(args.pipeline)}
+    qmode = {"iterwarp": args.query_mode == "iterwarp", "iter_rgs": args.iter_rgs, "pipeline": bool(args.pipeline),
+             "key_bits": kbits}
     if args.query_mode != "default" and world > 1:
         raise SystemExit("--query-mode iterwarp runs on one GPU")
 
@@ -344,7 +366,7 @@ def run_ours(args):
             trees_ = []
             for w_ in wls_:
                 tr = EireneTree(max_keys=tree_n + per_tree * batch_n + (1 << 12), max_batch=batch_n, **qmode)
-                tr.bulk_load(torch.from_numpy(w_.keys).to(dev), torch.from_numpy(w_.vals).to(dev))
+                tr.bulk_load(tnp(w_.keys).to(dev), tnp(w_.vals).to(dev))
                 tr.prepare(batch_n, bool(cap))   # graph capture outside every timed region
                 trees_.append(tr)
             hb_ = [wls_[s_ // per_tree].batch_arrays(s_ % per_tree) for s_ in range(nsteps)]
@@ -355,18 +377,18 @@ def run_ours(args):
             wl, tree = wls[0], trees[0]
         else:
             wl = W.Workload(cfg, tree=tree_n, batch=batch_n, **wkw)
-            keys_d = torch.from_numpy(wl.keys).to(dev)
-            vals_d = torch.from_numpy(wl.vals).to(dev)
+            keys_d = tnp(wl.keys).to(dev)
+            vals_d = tnp(wl.vals).to(dev)
             tree = EireneTree(max_keys=max(tree_n * 2, 1 << 20), max_batch=batch_n, **qmode)
             tree.bulk_load(keys_d, vals_d)
             del keys_d, vals_d
             wls, trees, step_tree = [wl], [tree], [0] * nb
             host_batches = [wl.batch_arrays(b) for b in range(nb)]
-        batches = [tuple(torch.from_numpy(a).to(dev) for a in hb) for hb in host_batches]
-        results = [torch.empty(batch_n, dtype=torch.uint64, device=dev) for _ in range(nb)]
+        batches = [tuple(tnp(a).to(dev) for a in hb) for hb in host_batches]
+        results = [torch.empty(batch_n, dtype=kdt, device=dev) for _ in range(nb)]
         if cap:
-            rrows = [(torch.empty(batch_n * cap, dtype=torch.uint64, device=dev),
-                      torch.empty(batch_n * cap, dtype=torch.uint64, device=dev)) for _ in range(nb)]
+            rrows = [(torch.empty(batch_n * cap, dtype=kdt, device=dev),
+                      torch.empty(batch_n * cap, dtype=kdt, device=dev)) for _ in range(nb)]
     else:
         # weak scaling: the global tree holds world * tree_n keys, the global batch
         # world * batch_n requests; rank r owns key range r and ts-slice r
@@ -479,7 +501,7 @@ def run_ours(args):
         _, s_trees, s_tree_of, s_hb = build_plan(1, n_stage)
         # (indexed from args.warmup like the single-tree region: results[0..warmup) keep
         # the parity batches)
-        s_batches = [None] * args.warmup + [tuple(torch.from_numpy(a).to(dev) for a in hb) for hb in s_hb]
+        s_batches = [None] * args.warmup + [tuple(tnp(a).to(dev) for a in hb) for hb in s_hb]
         s_tree_of = [0] * args.warmup + s_tree_of
         engines = s_trees
         stage_step = lambda i: step(args.warmup + i, s_trees, s_tree_of, s_batches)  # noqa: E731
@@ -510,15 +532,15 @@ def run_ours(args):
         # the inputs, submit_range, D2H of the counts and the range rows, all on
         # the submit stream inside the timed region (no overlap across steps)
         hb = [wl.batch_arrays(nb + i) for i in range(args.e2e_steps)]
-        pin = [tuple(torch.from_numpy(a).pin_memory() for a in x) for x in hb]
-        hout = [(torch.empty(batch_n, dtype=torch.uint64).pin_memory(),
-                 torch.empty(batch_n * cap, dtype=torch.uint64).pin_memory(),
-                 torch.empty(batch_n * cap, dtype=torch.uint64).pin_memory()) for _ in hb]
-        dbuf = [torch.empty(batch_n, dtype=torch.uint8, device=dev), torch.empty(batch_n, dtype=torch.uint64, device=dev),
-                torch.empty(batch_n, dtype=torch.uint64, device=dev)]
-        dres = torch.empty(batch_n, dtype=torch.uint64, device=dev)
-        drk = torch.empty(batch_n * cap, dtype=torch.uint64, device=dev)
-        drv = torch.empty(batch_n * cap, dtype=torch.uint64, device=dev)
+        pin = [tuple(tnp(a).pin_memory() for a in x) for x in hb]
+        hout = [(torch.empty(batch_n, dtype=kdt).pin_memory(),
+                 torch.empty(batch_n * cap, dtype=kdt).pin_memory(),
+                 torch.empty(batch_n * cap, dtype=kdt).pin_memory()) for _ in hb]
+        dbuf = [torch.empty(batch_n, dtype=torch.uint8, device=dev), torch.empty(batch_n, dtype=kdt, device=dev),
+                torch.empty(batch_n, dtype=kdt, device=dev)]
+        dres = torch.empty(batch_n, dtype=kdt, device=dev)
+        drk = torch.empty(batch_n * cap, dtype=kdt, device=dev)
+        drv = torch.empty(batch_n * cap, dtype=kdt, device=dev)
 
         def e2e_step(i):
             for d_, h_ in zip(dbuf, pin[i]):
@@ -551,8 +573,8 @@ def run_ours(args):
         else:
             hb = [wl.batch_arrays(nb + i) for i in range(args.e2e_steps)]
             e_trees, e_tree_of = [tree], [0] * len(hb)
-        pin = [tuple(torch.from_numpy(a).pin_memory() for a in x) for x in hb]
-        hres = [torch.empty(batch_n, dtype=torch.uint64).pin_memory() for _ in hb]
+        pin = [tuple(tnp(a).pin_memory() for a in x) for x in hb]
+        hres = [torch.empty(batch_n, dtype=kdt).pin_memory() for _ in hb]
         tk = e_trees[e_tree_of[0]].submit_host(*pin[0], hres[0])   # warm the path
         e_trees[e_tree_of[0]].results(tk)
         # first DMA touch of each freshly pinned buffer (IOMMU / page mapping) is a
@@ -577,7 +599,7 @@ def run_ours(args):
         # read zero-copy from the pinned buffer by the distribution kernel
         ups = np.mean([int(np.count_nonzero((x[0] == W.UPDATE) | (x[0] == W.INSERT))) for x in hb[1:]])
         e2e = {"value": batch_n * n_e / (e_ms * 1e-3) / 1e9, "unit": "Greq/s",
-               "h2d_bytes_per_step": int(batch_n * 9 + 8 * ups), "d2h_bytes_per_step": int(batch_n * 8),
+               "h2d_bytes_per_step": int(batch_n * (1 + kb) + kb * ups), "d2h_bytes_per_step": int(batch_n * kb),
                "steps": n_e, "path": "eirene_submit_batch_host (pinned host buffers; H2D of batch b+1 on the "
                                      "library's copy stream and D2H of batch b-1 on its d2h stream overlap "
                                      "batch b's kernels; upsert values read zero-copy)"}
@@ -660,7 +682,7 @@ def run_ours(args):
             else:
                 want = ref.apply(o, k, v)
             cpu_t += time.perf_counter() - a
-            got = results[b].cpu().numpy()
+            got = widen_np(results[b].cpu().numpy())
             bad += int(np.sum(got != want))
             if cap:
                 gk = rrows[b][0].view(batch_n, cap).cpu().numpy()
@@ -681,7 +703,7 @@ def run_ours(args):
             ms = stage_ms[2]
             kern = "range_kernel"
         elif stage_names[dom] == "query" or args.roofline_kernel == "query":
-            ab = [algorithmic_bytes_query(wls[step_tree[b]].keys, *host_batches[b][:2], 16)["bytes"]
+            ab = [algorithmic_bytes_query(wls[step_tree[b]].keys, *host_batches[b][:2], 16, kb)["bytes"]
                   for b in range(args.warmup, min(nb, args.warmup + 4))]
             bytes_per = float(np.mean(ab))
             ms = stage_ms[2]
@@ -723,16 +745,16 @@ def run_ours(args):
         # whole-path random-access roofline (BASELINE north_star) on
         # the bulk-loaded shape: 1 / (L/R128 + S/R32 + Wr/R32w + B_io/BW) req/s
         if not cap and not per_tree:
-            cs = [random_access_counts(wls[0].keys, *host_batches[b][:2], 16)
+            cs = [random_access_counts(wls[0].keys, *host_batches[b][:2], 16, kb)
                   for b in range(args.warmup, min(nb, args.warmup + 4))]
             c = {k: float(np.mean([x[k] for x in cs])) for k in cs[0]}
             # whole-path HBM streaming roofline: algorithmic bytes per request =
             # B_io + leaf lines x 128 + value sectors x 32 + written sectors x 32, at the measured peak
-            b_req = c["bio"] + 128 * c["lines"] + 32 * c["sectors"] + 32 * c["writes"]
+            b_req = c["bio"] + c["line_bytes"] * c["lines"] + 32 * c["sectors"] + 32 * c["writes"]
             stream_roof = peaks["hbm_gbs"] * 1e9 / b_req / 1e9
             roof["streaming"] = {"roofline_Greq_s": stream_roof, "frac": value / stream_roof,
                                  "bytes_per_request": b_req}
-        if not cap and not per_tree and args.ra_probe:
+        if not cap and not per_tree and args.ra_probe and kbits == 64:
             n_leaves = (tree_n + 15) // 16
             pool_bytes = 1 << int(np.ceil(np.log2(max(n_leaves * 256, 1 << 20))))
             n_leaf = int(round(c["lines"] * batch_n))
@@ -777,8 +799,8 @@ def run_ours(args):
             "metric": "requests/sec per batch", "value": value, "unit": "Greq/s", "n_gpus": world,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": elapsed_ms / args.steps,
             "higher_is_better": True, "scaling": "strong" if C.get("strong") else "weak", "vs_baseline": None,
-            "dtype": "u64", "data": "synthetic",
-            "config": {"workload": f"cfg{cfg}: {tree_n * world} u64 keys (fanout 16, fill 1.0), "
+            "dtype": "u32" if kbits == 32 else "u64", "data": "synthetic",
+            "config": {"workload": f"cfg{cfg}: {tree_n * world} u{kbits} keys (fanout 16, fill 1.0), "
                                    f"{batch_n * world}-request batches, "
                                    + ", ".join(f"{int(p * 100)}% {['query', 'update', 'insert', 'delete', 'range'][o]}"
                                                for o, p in sorted(C['fracs'].items())) + f", {C['dist']} keys"

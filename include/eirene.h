@@ -38,9 +38,22 @@ extern "C" {
 
 typedef struct CUstream_st* eirene_stream_t;   /* == cudaStream_t; NULL = legacy default stream */
 
-/* Result sentinel (null).  UINT64_MAX is also reserved as a key and
- * as a written value; requests using it are rejected with EIRENE_EINVAL. */
+/* Key / value width.  libeirene.so: 64-bit keys and values (BASELINE configs).
+ * Built with -DEIRENE_KEY32 (libeirene32.so): 32-bit keys
+ * and values, the paper's record width -- the leaves and inner nodes
+ * hold 32-bit keys, so a leaf key line is 64 B and a value sector 8 values.
+ * Every key / value / result pointer of the single-GPU API below is
+ * eirene_key_t; the multi-GPU routing calls are 64-bit only.
+ * Result sentinel (null): the all-ones value of the width.  It is
+ * also reserved as a key and as a written value; requests using it are
+ * rejected with EIRENE_EINVAL. */
+#ifdef EIRENE_KEY32
+typedef uint32_t eirene_key_t;
+#define EIRENE_NOT_FOUND UINT32_MAX
+#else
+typedef uint64_t eirene_key_t;
 #define EIRENE_NOT_FOUND UINT64_MAX
+#endif
 
 enum {
   EIRENE_OK = 0,
@@ -149,7 +162,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out);
  * and speed only (§8(c) reading 13).  Valid only on a freshly created tree
  * (ESTATE otherwise).  Synchronous with respect to `stream`; EINVAL if the
  * device check of the keys fails (tree left empty). */
-int eirene_bulk_load(eirene_handle h, const uint64_t* keys_dev, const uint64_t* vals_dev,
+int eirene_bulk_load(eirene_handle h, const eirene_key_t* keys_dev, const eirene_key_t* vals_dev,
                      uint64_t n, float leaf_fill, eirene_stream_t stream);
 
 /* Submits one batch of n requests (Alg.1:1-7): ops_dev[n] (u8, EIRENE_*),
@@ -165,8 +178,8 @@ int eirene_bulk_load(eirene_handle h, const uint64_t* keys_dev, const uint64_t* 
  * Invalid requests (op > 3, key == UINT64_MAX or outside [key_lo, key_hi),
  * upsert value == UINT64_MAX) are detected on the device: the batch then
  * leaves the tree untouched and eirene_results reports EINVAL. */
-int eirene_submit_batch(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev,
-                        const uint64_t* vals_dev, uint32_t n, uint64_t* results_dev,
+int eirene_submit_batch(eirene_handle h, const uint8_t* ops_dev, const eirene_key_t* keys_dev,
+                        const eirene_key_t* vals_dev, uint32_t n, eirene_key_t* results_dev,
                         eirene_stream_t stream, uint64_t* ticket);
 
 /* Same batch from HOST buffers.  ops and keys are copied host->device into
@@ -179,8 +192,8 @@ int eirene_submit_batch(eirene_handle h, const uint8_t* ops_dev, const uint64_t*
  * values are copied.  The copies run at full speed only from pinned memory.
  * Results are valid after eirene_results(ticket); keep every buffer alive
  * until then. */
-int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops_host, const uint64_t* keys_host,
-                             const uint64_t* vals_host, uint32_t n, uint64_t* results_host,
+int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops_host, const eirene_key_t* keys_host,
+                             const eirene_key_t* vals_host, uint32_t n, eirene_key_t* results_host,
                              eirene_stream_t stream, uint64_t* ticket);
 
 /* Same as eirene_submit_batch, and the batch may also hold range queries
@@ -201,9 +214,9 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops_host, const uin
  * that key's timestamp-sorted segment.  Not accepted by the multi-GPU
  * routing (EINVAL there).  Errors as eirene_submit_batch, plus EINVAL for
  * cap == 0, cap > 4096 or null range buffers. */
-int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev,
-                              const uint64_t* vals_dev, uint32_t n, uint64_t* results_dev,
-                              uint32_t cap, uint64_t* range_keys_dev, uint64_t* range_vals_dev,
+int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops_dev, const eirene_key_t* keys_dev,
+                              const eirene_key_t* vals_dev, uint32_t n, eirene_key_t* results_dev,
+                              uint32_t cap, eirene_key_t* range_keys_dev, eirene_key_t* range_vals_dev,
                               eirene_stream_t stream, uint64_t* ticket);
 
 /* Optional warm-up: captures and instantiates the CUDA graph that batches of
@@ -230,8 +243,8 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats);
  * keys_out_dev / vals_out_dev (either may be NULL when cap == 0) and the total
  * to *count.  Synchronous with respect to `stream`.  Used for parity and as
  * the save half of save/restore (bulk_load is the restore half). */
-int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out_dev,
-                uint64_t* vals_out_dev, uint64_t cap, uint64_t* count, eirene_stream_t stream);
+int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, eirene_key_t* keys_out_dev,
+                eirene_key_t* vals_out_dev, uint64_t cap, uint64_t* count, eirene_stream_t stream);
 
 /* Debug: copies the node pools to the host and checks the structural
  * invariants of the quiescent tree: keys strictly increasing in every node,

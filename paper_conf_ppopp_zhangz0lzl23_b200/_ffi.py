@@ -15,6 +15,8 @@ PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 # EIRENE_LIB: an alternative build of the same library (A/B experiments); default: the in-tree one
 LIB_PATH = os.environ.get("EIRENE_LIB") or os.path.join(PKG, "libeirene.so")
+# the 32-bit key / value build (-DEIRENE_KEY32): same API, eirene_key_t = uint32_t
+LIB32_PATH = os.environ.get("EIRENE_LIB32") or os.path.join(PKG, "libeirene32.so")
 HEADER = os.path.join(ROOT, "include", "eirene.h")
 
 EIRENE_OK, EIRENE_EINVAL, EIRENE_ENOMEM, EIRENE_EFULL, EIRENE_ESTATE, EIRENE_ECUDA, EIRENE_EINTERNAL = (
@@ -81,7 +83,7 @@ _SIGS = {
     "eirene_stream_wait_batch": (_int, [_vp, _u64, _vp]),
 }
 
-_lib = None
+_libs: dict = {}
 
 
 def header_functions() -> list[str]:
@@ -92,20 +94,20 @@ def header_functions() -> list[str]:
     return sorted(set(re.findall(r"\b(eirene_[a-z_]+)\s*\(", text)))
 
 
-def lib() -> ctypes.CDLL:
-    """Load libeirene.so (raises if it was not built)."""
-    global _lib
-    if _lib is None:
-        if not os.path.exists(LIB_PATH):
-            raise RuntimeError(f"{LIB_PATH} is missing: run `python -m paper_conf_ppopp_zhangz0lzl23_b200.build` "
+def lib(key_bits: int = 64) -> ctypes.CDLL:
+    """Load libeirene.so (key_bits 64) or libeirene32.so (32); raises if it was not built."""
+    if key_bits not in _libs:
+        path = {64: LIB_PATH, 32: LIB32_PATH}[key_bits]
+        if not os.path.exists(path):
+            raise RuntimeError(f"{path} is missing: run `python -m paper_conf_ppopp_zhangz0lzl23_b200.build` "
                                "(there is no CPU fallback)")
-        L = ctypes.CDLL(LIB_PATH)
+        L = ctypes.CDLL(path)
         for name, (res, args) in _SIGS.items():
             fn = getattr(L, name)
             fn.restype = res
             fn.argtypes = args
-        _lib = L
-    return _lib
+        _libs[key_bits] = L
+    return _libs[key_bits]
 
 
 class EireneError(RuntimeError):

@@ -44,7 +44,7 @@ def build(force: bool = False, verbose: bool = False, variant: str = "", defines
     """Build libeirene.so; a `variant` (A/B or diagnostic build, e.g. -DEIRENE_PHASE_PROF) goes to
     _build_<variant>/ and libeirene_<variant>.so, selected at run time with EIRENE_LIB."""
     OBJ = os.path.join(PKG, "_build" + (f"_{variant}" if variant else ""))
-    LIB = os.path.join(PKG, f"libeirene_{variant}.so" if variant else "libeirene.so")
+    LIB = os.path.join(PKG, {"": "libeirene.so", "32": "libeirene32.so"}.get(variant, f"libeirene_{variant}.so"))
     flags = FLAGS + [f"-D{d}" for d in defines]
     os.makedirs(OBJ, exist_ok=True)
     headers = glob.glob(os.path.join(CSRC, "*.cuh")) + [os.path.join(INCLUDE, "eirene.h")]
@@ -83,8 +83,17 @@ def build(force: bool = False, verbose: bool = False, variant: str = "", defines
     return LIB
 
 
+def build_all(force: bool = False, verbose: bool = False) -> list[str]:
+    """The product libraries: libeirene.so (64-bit keys / values) and libeirene32.so
+    (-DEIRENE_KEY32: 32-bit keys / values)."""
+    return [build(force, verbose), build(force, verbose, variant="32", defines=("EIRENE_KEY32",))]
+
+
 if __name__ == "__main__":
     # python -m paper_conf_ppopp_zhangz0lzl23_b200.build [--force] [--variant NAME -DX ...]
     a = sys.argv[1:]
     var = a[a.index("--variant") + 1] if "--variant" in a else ""
-    build(force="--force" in a, verbose=True, variant=var, defines=tuple(x[2:] for x in a if x.startswith("-D")))
+    if var or any(x.startswith("-D") for x in a):
+        build(force="--force" in a, verbose=True, variant=var, defines=tuple(x[2:] for x in a if x.startswith("-D")))
+    else:
+        build_all(force="--force" in a, verbose=True)

@@ -83,11 +83,11 @@ __global__ void init_empty_kernel(Tree t, uint64_t key_lo, uint64_t key_hi) {
 
 // First node of the batch graph: zero the per-batch control region (BatchCtl,
 // bin counts, group look-back words) and publish the batch's pointers.
-__global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const uint8_t* ops, const uint64_t* keys,
-                                                        const uint64_t* vals_src, uint64_t* vals_stage,
-                                                        uint64_t* results, BatchCtl* ctl_out, uint4* zero,
+__global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const uint8_t* ops, const tkey_t* keys,
+                                                        const tkey_t* vals_src, tkey_t* vals_stage,
+                                                        tkey_t* results, BatchCtl* ctl_out, uint4* zero,
                                                         uint32_t zero_n16, uint4* zero2, uint32_t zero2_n16,
-                                                        uint64_t* rkeys, uint64_t* rvals, uint32_t rcap,
+                                                        tkey_t* rkeys, tkey_t* rvals, uint32_t rcap,
                                                         uint32_t n, unsigned long long* phase) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
     zero[i] = make_uint4(0, 0, 0, 0);
@@ -190,9 +190,9 @@ struct eirene_tree {
   bool slot_used[HOST_SLOTS] = {};
   uint32_t host_slot = 0;
   uint8_t* st_ops = nullptr;
-  uint64_t* st_keys = nullptr;
-  uint64_t* st_vals = nullptr;
-  uint64_t* st_res = nullptr;
+  tkey_t* st_keys = nullptr;
+  tkey_t* st_vals = nullptr;
+  tkey_t* st_res = nullptr;
   unsigned long long* route_lb = nullptr;
   uint32_t* route_ctr = nullptr;
   uint32_t route_epoch = 0;
@@ -272,6 +272,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   if (cfg->fanout != 16 || cfg->max_batch == 0 || cfg->max_batch > (1u << 29) || cfg->key_lo >= cfg->key_hi ||
       cfg->max_keys == 0)
     return EIRENE_EINVAL;
+  if (sizeof(tkey_t) == 4 && cfg->key_lo >= 0xFFFFFFFFull) return EIRENE_EINVAL;   // (32-bit keys: empty range)
   DeviceGuard dg_(cfg->device);
   CK(dg_.err);
   eirene_tree* h = new (std::nothrow) eirene_tree();
@@ -526,7 +527,7 @@ int eirene_destroy(eirene_handle h) {
   return EIRENE_OK;
 }
 
-int eirene_bulk_load(eirene_handle h, const uint64_t* keys, const uint64_t* vals, uint64_t n, float leaf_fill,
+int eirene_bulk_load(eirene_handle h, const tkey_t* keys, const tkey_t* vals, uint64_t n, float leaf_fill,
                      eirene_stream_t stream) {
   if (!h) return EIRENE_EINVAL;
   if (h->loaded || h->modified) return EIRENE_ESTATE;
@@ -610,9 +611,9 @@ static int get_graph(eirene_handle h, GraphEntry* table, uint32_t& next, uint32_
 
 extern "C" {
 
-static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
-                       uint64_t* results, cudaStream_t st, uint64_t* vals_stage, uint64_t* ticket,
-                       uint64_t* rkeys = nullptr, uint64_t* rvals = nullptr, uint32_t rcap = 0,
+static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, const tkey_t* vals, uint32_t n,
+                       tkey_t* results, cudaStream_t st, tkey_t* vals_stage, uint64_t* ticket,
+                       tkey_t* rkeys = nullptr, tkey_t* rvals = nullptr, uint32_t rcap = 0,
                        bool prepare_only = false, bool prepare_range = false, cudaStream_t* end_stream = nullptr) {
   const bool range = rkeys != nullptr || prepare_range;
   DeviceGuard dg_(h->cfg.device);
@@ -662,7 +663,9 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
       if (e != cudaSuccess) return e;
     }
     if (timing) rec(0, s);
-    launch_bucket_sort(L.dargs, nk, h->cfg.key_lo, h->cfg.key_hi, large ? L.bsL : L.bs, L.ctl, h->num_sms, s, nl);
+    // (32-bit keys: the bins span [key_lo, min(key_hi, 2^32)), not the 64-bit range)
+    const uint64_t bin_hi = sizeof(tkey_t) == 4 ? std::min<uint64_t>(h->cfg.key_hi, 1ull << 32) : h->cfg.key_hi;
+    launch_bucket_sort(L.dargs, nk, h->cfg.key_lo, bin_hi, large ? L.bsL : L.bs, L.ctl, h->num_sms, s, nl);
     stage("sort", s);
     if (timing) rec(1, s);
     launch_group(L.dargs, nk, large ? L.bsL : L.bs, large ? L.cbL : L.cb, h->t, L.ctl, h->num_sms, s, nl);
@@ -692,8 +695,8 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
     uint32_t zero_n16 = (uint32_t)(h->zero_bytes / 16);
     uint4* zero2 = reinterpret_cast<uint4*>(large ? L.zero_large : L.zero_region);
     uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
-    void* params[] = {&L.dargs, const_cast<uint8_t**>(&ops), const_cast<uint64_t**>(&keys),
-                      const_cast<uint64_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
+    void* params[] = {&L.dargs, const_cast<uint8_t**>(&ops), const_cast<tkey_t**>(&keys),
+                      const_cast<tkey_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
                       &zero2, &zero2_n16, &rkeys, &rvals, &rcap, &n, &h->phase};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
@@ -774,8 +777,8 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const uint64_t* keys
   return EIRENE_OK;
 }
 
-int eirene_submit_batch(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
-                        uint64_t* results, eirene_stream_t stream, uint64_t* ticket) {
+int eirene_submit_batch(eirene_handle h, const uint8_t* ops, const tkey_t* keys, const tkey_t* vals, uint32_t n,
+                        tkey_t* results, eirene_stream_t stream, uint64_t* ticket) {
   if (!h || !ops || !keys || !vals || !results || !ticket) return EIRENE_EINVAL;
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   return submit_impl(h, ops, keys, vals, n, results, reinterpret_cast<cudaStream_t>(stream), nullptr, ticket);
@@ -788,17 +791,17 @@ int eirene_prepare_batch(eirene_handle h, uint32_t n, int with_ranges) {
                      with_ranges != 0);
 }
 
-int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
-                              uint32_t n, uint64_t* results, uint32_t cap, uint64_t* range_keys,
-                              uint64_t* range_vals, eirene_stream_t stream, uint64_t* ticket) {
+int eirene_submit_batch_range(eirene_handle h, const uint8_t* ops, const tkey_t* keys, const tkey_t* vals,
+                              uint32_t n, tkey_t* results, uint32_t cap, tkey_t* range_keys,
+                              tkey_t* range_vals, eirene_stream_t stream, uint64_t* ticket) {
   if (!h || !ops || !keys || !vals || !results || !ticket || !range_keys || !range_vals) return EIRENE_EINVAL;
   if (n == 0 || n > h->cfg.max_batch || cap == 0 || cap > 4096) return EIRENE_EINVAL;
   return submit_impl(h, ops, keys, vals, n, results, reinterpret_cast<cudaStream_t>(stream), nullptr, ticket,
                      range_keys, range_vals, cap);
 }
 
-int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals,
-                             uint32_t n, uint64_t* results, eirene_stream_t stream, uint64_t* ticket) {
+int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const tkey_t* keys, const tkey_t* vals,
+                             uint32_t n, tkey_t* results, eirene_stream_t stream, uint64_t* ticket) {
   if (!h || !ops || !keys || !vals || !results || !ticket) return EIRENE_EINVAL;
   if (n == 0 || n > h->cfg.max_batch) return EIRENE_EINVAL;
   cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
@@ -815,18 +818,18 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
   const size_t off = (size_t)s * h->cfg.max_batch;
   if (h->slot_used[s]) CK(cudaStreamWaitEvent(h->h2d_stream, h->comp_done[s], 0));
   CK(cudaMemcpyAsync(h->st_ops + off, ops, n, cudaMemcpyHostToDevice, h->h2d_stream));
-  CK(cudaMemcpyAsync(h->st_keys + off, keys, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, h->h2d_stream));
+  CK(cudaMemcpyAsync(h->st_keys + off, keys, sizeof(tkey_t) * n, cudaMemcpyHostToDevice, h->h2d_stream));
   cudaPointerAttributes pa{};
   const bool pinned = cudaPointerGetAttributes(&pa, vals) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
                       pa.devicePointer != nullptr;
   cudaGetLastError();   // (clear a pageable-pointer query error, if any)
-  const uint64_t* vsrc;
-  uint64_t* vstage = nullptr;
+  const tkey_t* vsrc;
+  tkey_t* vstage = nullptr;
   if (pinned) {
-    vsrc = static_cast<const uint64_t*>(pa.devicePointer);
+    vsrc = static_cast<const tkey_t*>(pa.devicePointer);
     vstage = h->st_vals + off;
   } else {
-    CK(cudaMemcpyAsync(h->st_vals + off, vals, sizeof(uint64_t) * n, cudaMemcpyHostToDevice, h->h2d_stream));
+    CK(cudaMemcpyAsync(h->st_vals + off, vals, sizeof(tkey_t) * n, cudaMemcpyHostToDevice, h->h2d_stream));
     vsrc = h->st_vals + off;
   }
   CK(cudaEventRecord(h->h2d_done[s], h->h2d_stream));
@@ -838,7 +841,7 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const uint64_t
   if (rc != EIRENE_OK) return rc;
   CK(cudaEventRecord(h->comp_ev[s], end));
   CK(cudaStreamWaitEvent(h->d2h_stream, h->comp_ev[s], 0));
-  CK(cudaMemcpyAsync(results, h->st_res + off, sizeof(uint64_t) * n, cudaMemcpyDeviceToHost, h->d2h_stream));
+  CK(cudaMemcpyAsync(results, h->st_res + off, sizeof(tkey_t) * n, cudaMemcpyDeviceToHost, h->d2h_stream));
   CK(cudaEventRecord(h->comp_done[s], h->d2h_stream));
   CK(cudaEventRecord(h->ring[tk % RING].done, h->d2h_stream));   // eirene_results waits for the D2H too
   h->slot_used[s] = true;
@@ -893,7 +896,7 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) 
   return c.status;
 }
 
-int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, uint64_t* keys_out, uint64_t* vals_out, uint64_t cap,
+int eirene_scan(eirene_handle h, uint64_t lo, uint64_t hi, tkey_t* keys_out, tkey_t* vals_out, uint64_t cap,
                 uint64_t* count, eirene_stream_t stream) {
   if (!h || !count) return EIRENE_EINVAL;
   if (cap > 0 && !keys_out && !vals_out) return EIRENE_EINVAL;
@@ -979,13 +982,14 @@ int eirene_check_invariants(eirene_handle h, uint64_t* n_keys) {
   TreeHdr hdr;
   CK(cudaMemcpy(&hdr, h->t.hdr, sizeof(hdr), cudaMemcpyDeviceToHost));
   const uint32_t L = hdr.leaf_count, I = hdr.inner_count;
-  std::vector<uint64_t> lk((size_t)L * FAN), ik((size_t)I * FAN);
+  std::vector<tkey_t> lk((size_t)L * FAN), ik((size_t)I * FAN);
   std::vector<uint32_t> ic((size_t)I * FAN);
   std::vector<NodeMeta> lm(L), im(I);
-  CK(cudaMemcpy2D(lk.data(), FAN * 8, h->t.lkeys, LSTRIDE * 8, FAN * 8, L, cudaMemcpyDeviceToHost));
+  CK(cudaMemcpy2D(lk.data(), FAN * sizeof(tkey_t), h->t.lkeys, LSTRIDE * sizeof(tkey_t), FAN * sizeof(tkey_t), L,
+                   cudaMemcpyDeviceToHost));
   CK(cudaMemcpy(lm.data(), h->t.lmeta, lm.size() * sizeof(NodeMeta), cudaMemcpyDeviceToHost));
   if (I) {
-    CK(cudaMemcpy(ik.data(), h->t.ikeys, ik.size() * 8, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(ik.data(), h->t.ikeys, ik.size() * sizeof(tkey_t), cudaMemcpyDeviceToHost));
     CK(cudaMemcpy(ic.data(), h->t.ichild, ic.size() * 4, cudaMemcpyDeviceToHost));
     CK(cudaMemcpy(im.data(), h->t.imeta, im.size() * sizeof(NodeMeta), cudaMemcpyDeviceToHost));
   }
@@ -1009,7 +1013,7 @@ int eirene_check_invariants(eirene_handle h, uint64_t* n_keys) {
       uint64_t prev = 0;
       bool first = true, ended = false;
       for (int s = 0; s < FAN; ++s) {
-        const uint64_t k = lk[(size_t)f.node * FAN + s];
+        const uint64_t k = widen(lk[(size_t)f.node * FAN + s]);
         if (k == KEY_MAX) { ended = true; continue; }
         if (ended) return 15;               // key after padding
         if (!first && !(prev < k)) return 16;   // strictly increasing
@@ -1028,19 +1032,20 @@ int eirene_check_invariants(eirene_handle h, uint64_t* n_keys) {
     if (m.lo != f.lo || m.hi != f.hi) return 14;
     const uint32_t c = m.count;
     if (c < 1 || c > FAN) return 20;
-    const uint64_t* K = &ik[(size_t)f.node * FAN];
+    const tkey_t* Kr = &ik[(size_t)f.node * FAN];
+    auto K = [&](uint32_t i) { return widen(Kr[i]); };
     const uint32_t* Cc = &ic[(size_t)f.node * FAN];
     for (uint32_t i = 0; i + 1 < c; ++i) {
-      if (K[i] == KEY_MAX) return 21;
-      if (i > 0 && !(K[i - 1] < K[i])) return 16;
-      if (K[i] <= f.lo || K[i] >= f.hi) return 17;
+      if (K(i) == KEY_MAX) return 21;
+      if (i > 0 && !(K(i - 1) < K(i))) return 16;
+      if (K(i) <= f.lo || K(i) >= f.hi) return 17;
     }
     for (uint32_t i = c - 1; i < FAN; ++i)
-      if (K[i] != KEY_MAX) return 21;
+      if (K(i) != KEY_MAX) return 21;
     // push children right-to-left so the leftmost is visited first
     for (int i = (int)c - 1; i >= 0; --i) {
-      const uint64_t clo = i == 0 ? f.lo : K[i - 1];
-      const uint64_t chi = (uint32_t)i + 1 < c ? K[i] : f.hi;
+      const uint64_t clo = i == 0 ? f.lo : K(i - 1);
+      const uint64_t chi = (uint32_t)i + 1 < c ? K(i) : f.hi;
       stack.push_back({Cc[i], f.level - 1, clo, chi});
     }
   }

@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
   n = A->n;   // the launch is sized for the graph's size bucket; the batch's own size is on the device
   __shared__ uint32_t wsum[H_THREADS / 32];
   __shared__ uint32_t s_total;
-  const uint64_t* __restrict__ keys = A->keys;
+  const tkey_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   for (uint32_t i = tid; i < NBINS_L; i += H_THREADS) h[i] = 0;
@@ -77,7 +77,7 @@ __global__ void __launch_bounds__(H_THREADS) bsort_hist_kernel(const BatchArgs* 
 #pragma unroll
     for (int j = 0; j < H_ITEMS; ++j) {
       const uint32_t i = t0 + j * H_THREADS + tid;
-      k[j] = i < n ? keys[i] : 0;
+      k[j] = i < n ? widen(keys[i]) : 0;
       pt[j] = i < n && ops[i] != OP_RANGE;
     }
 #pragma unroll
@@ -161,10 +161,10 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
   uint16_t* s_b2g = reinterpret_cast<uint16_t*>(smem);             // [NBINS_L]
   uint32_t* hist = reinterpret_cast<uint32_t*>(s_b2g + NBINS_L);   // [G] tile counts, then global base
   n = A->n;
-  const uint64_t* __restrict__ keys = A->keys;
+  const tkey_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
-  const uint64_t* __restrict__ vals = A->vals_src;
-  uint64_t* __restrict__ vstage = A->vals_stage;
+  const tkey_t* __restrict__ vals = A->vals_src;
+  tkey_t* __restrict__ vstage = A->vals_stage;
   const int tid = threadIdx.x;
   for (uint32_t i = tid; i < (uint32_t)NBINS_L; i += S_THREADS) s_b2g[i] = bin2grp[i];
   for (uint32_t i = tid; i < G; i += S_THREADS) hist[i] = 0;
@@ -174,7 +174,7 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
 #pragma unroll
   for (int j = 0; j < S_ITEMS; ++j) {
     const uint32_t i = t0 + j * S_THREADS + tid;
-    k[j] = i < n ? keys[i] : 0;
+    k[j] = i < n ? widen(keys[i]) : 0;
     o[j] = i < n ? (uint32_t)ops[i] : 0u;
   }
   bool bad = false;
@@ -184,7 +184,7 @@ __global__ void __launch_bounds__(S_THREADS) bsort_scatter_kernel(
   for (int j = 0; j < S_ITEMS; ++j) {
     const uint32_t i = t0 + j * S_THREADS + tid;
     const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
-    const uint64_t v = (i < n && up) ? vals[i] : 0;
+    const uint64_t v = (i < n && up) ? widen(vals[i]) : 0;
     if (vstage && i < n && up) vstage[i] = v;
     bad |= i < n && request_invalid(o[j], k[j], v, up, rok, key_lo, key_hi);
     nr += i < n && o[j] == OP_RANGE;
@@ -259,10 +259,10 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   uint32_t* gs = S.u.b.gs;
   n = A->n;   // (per_cta is sized for the graph's size bucket >= n)
   EIRENE_PHASE(A, 0, blockIdx.x, 0);
-  const uint64_t* __restrict__ keys = A->keys;
+  const tkey_t* __restrict__ keys = A->keys;
   const uint8_t* __restrict__ ops = A->ops;
-  const uint64_t* __restrict__ vals = A->vals_src;
-  uint64_t* __restrict__ vstage = A->vals_stage;
+  const tkey_t* __restrict__ vals = A->vals_src;
+  tkey_t* __restrict__ vstage = A->vals_stage;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   for (uint32_t i = tid; i < NBINS; i += D_THREADS) h[i] = 0;
   __syncthreads();
@@ -273,7 +273,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
 #pragma unroll
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
-    k[j] = i < t1 ? keys[i] : 0;
+    k[j] = i < t1 ? widen(keys[i]) : 0;
     o[j] = i < t1 ? (uint32_t)ops[i] : 0u;
   }
   bool bad = false;
@@ -283,7 +283,7 @@ __global__ void __launch_bounds__(D_THREADS, 2) bsort_dist_kernel(
   for (int j = 0; j < D_ITEMS; ++j) {
     const uint32_t i = t0 + j * D_THREADS + tid;
     const bool up = (o[j] == OP_UPDATE || o[j] == OP_INSERT);
-    const uint64_t v = (i < t1 && up) ? vals[i] : 0;
+    const uint64_t v = (i < t1 && up) ? widen(vals[i]) : 0;
     if (vstage && i < t1 && up) vstage[i] = v;
     bad |= i < t1 && request_invalid(o[j], k[j], v, up, rok, key_lo, key_hi);
     nr += i < t1 && o[j] == OP_RANGE;

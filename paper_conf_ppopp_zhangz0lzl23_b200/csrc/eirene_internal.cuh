@@ -23,8 +23,17 @@
 namespace eirene {
 
 constexpr int FAN = 16;
-constexpr int LSTRIDE = 2 * FAN;   // u64 words per leaf block (keys, then values)
+constexpr int LSTRIDE = 2 * FAN;   // tkey_t words per leaf block (keys, then values)
 constexpr uint64_t KEY_MAX = ~0ull;
+// Storage type of keys and values in the tree and in the caller's batch arrays
+// (eirene_key_t: 64 bits, or 32 with -DEIRENE_KEY32 -- SURVEY §8(f) NEXT(4)).
+// Kernels compute on 64-bit keys: a stored key is zero-extended on load (every
+// valid key, and the padding TKEY_MAX above them, keep their order) and
+// narrowed on store (KEY_MAX -> TKEY_MAX); widen() maps the padding / NOT_FOUND
+// sentinel to KEY_MAX where a loaded word is compared with it.
+typedef eirene_key_t tkey_t;
+constexpr tkey_t TKEY_MAX = (tkey_t)~(tkey_t)0;
+__host__ __device__ __forceinline__ uint64_t widen(tkey_t x) { return x == TKEY_MAX ? KEY_MAX : (uint64_t)x; }
 constexpr uint32_t NIL = 0xFFFFFFFFu;
 constexpr int MAX_LEVELS = 32;
 constexpr uint32_t DONE_BIT = 0x80000000u;    // pinfo: an earlier write of the segment decides the result
@@ -113,14 +122,14 @@ struct SpinGuard {
 // updating that single node (api.cu).
 struct BatchArgs {
   const uint8_t* ops;
-  const uint64_t* keys;
-  const uint64_t* vals;        // values as read by the kernels after the distribution pass
-  uint64_t* results;
-  const uint64_t* vals_src;    // where the distribution pass reads the values of upserts
-  uint64_t* vals_stage;        // non-null: it also copies them here (== vals); host path, zero-copy
+  const tkey_t* keys;
+  const tkey_t* vals;        // values as read by the kernels after the distribution pass
+  tkey_t* results;
+  const tkey_t* vals_src;    // where the distribution pass reads the values of upserts
+  tkey_t* vals_stage;        // non-null: it also copies them here (== vals); host path, zero-copy
   BatchCtl* ctl_out;    // device ring slot: the batch's final BatchCtl is copied here at the end
-  uint64_t* rkeys;      // range-query output (eirene_submit_batch_range), else null: RANGE ops invalid
-  uint64_t* rvals;
+  tkey_t* rkeys;        // range-query output (eirene_submit_batch_range), else null: RANGE ops invalid
+  tkey_t* rvals;
   uint32_t rcap;
   unsigned long long t0;   // %globaltimer when the batch's first kernel started (device batch time)
   uint32_t n;              // requests in the batch (launches are sized for the graph's size bucket >= n)
@@ -146,11 +155,11 @@ constexpr int PROF_CTAS = 512, PROF_PHASES = 8;
 enum { TC_SORT0 = 0, TC_GROUP = 8, TC_ROUTE = 10, TC_SCAN = 11, TC_HIST = 12 };
 
 struct Tree {
-  uint64_t* lkeys;   // leaf L: keys at lkeys[L * LSTRIDE + s]
-  uint64_t* lvals;   // = lkeys + FAN: values at lvals[L * LSTRIDE + s]
+  tkey_t* lkeys;     // leaf L: keys at lkeys[L * LSTRIDE + s]
+  tkey_t* lvals;     // = lkeys + FAN: values at lvals[L * LSTRIDE + s]
   NodeMeta* lmeta;
   uint64_t* lrf;     // range field of every leaf (EIRENE_F_ITERWARP)
-  uint64_t* ikeys;
+  tkey_t* ikeys;
   uint32_t* ichild;
   NodeMeta* imeta;
   TreeHdr* hdr;
@@ -235,6 +244,11 @@ __device__ __forceinline__ uint64_t ldg64_pol(const uint64_t* p, uint64_t pol) {
   asm volatile("ld.global.nc.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
   return v;
 }
+__device__ __forceinline__ uint64_t ldg64_pol(const uint32_t* p, uint64_t pol) {   // (32-bit keys: zero-extended)
+  uint32_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
 __device__ __forceinline__ uint32_t ldg32_pol(const uint32_t* p, uint64_t pol) {
   uint32_t v;
   asm volatile("ld.global.nc.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
@@ -243,6 +257,76 @@ __device__ __forceinline__ uint32_t ldg32_pol(const uint32_t* p, uint64_t pol) {
 __device__ __forceinline__ void st64_pol(uint64_t* p, uint64_t v, uint64_t pol) {
   asm volatile("st.global.L2::cache_hint.u64 [%0], %1, %2;" ::"l"(p), "l"(v), "l"(pol) : "memory");
 }
+__device__ __forceinline__ void st64_pol(uint32_t* p, uint64_t v, uint64_t pol) {   // (32-bit keys: narrowed)
+  asm volatile("st.global.L2::cache_hint.u32 [%0], %1, %2;" ::"l"(p), "r"((uint32_t)v), "l"(pol) : "memory");
+}
+
+// The 16 keys of a node line (a 128 B line of u64 keys, or 64 B of u32 keys)
+// in registers, with 256-bit loads: Line16::at(s) = key s zero-extended.
+struct Line16 {
+  static constexpr int NW = FAN * (int)sizeof(tkey_t) / 32;   // 256-bit words: 4 (u64 keys) or 2 (u32)
+  ulonglong4 w[NW];
+  __device__ __forceinline__ void load(const tkey_t* p, uint64_t pol) {   // L1 no-allocate (leaves)
+#pragma unroll
+    for (int x = 0; x < NW; ++x) w[x] = ldg256_pol(reinterpret_cast<const uint64_t*>(p) + 4 * x, pol);
+  }
+  __device__ __forceinline__ void load_l1(const tkey_t* p, uint64_t pol) {   // L1-allocating (inner nodes)
+#pragma unroll
+    for (int x = 0; x < NW; ++x) {
+      const uint64_t* q = reinterpret_cast<const uint64_t*>(p) + 4 * x;
+      asm volatile("ld.global.nc.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+                   : "=l"(w[x].x), "=l"(w[x].y), "=l"(w[x].z), "=l"(w[x].w) : "l"(q), "l"(pol));
+    }
+  }
+  __device__ __forceinline__ uint64_t at(uint32_t s) const {
+    if constexpr (sizeof(tkey_t) == 8) {
+      const ulonglong4 q = (s < 8) ? ((s < 4) ? w[0] : w[1]) : ((s < 12) ? w[2 % NW] : w[3 % NW]);
+      const uint32_t r = s & 3;
+      return r == 0 ? q.x : r == 1 ? q.y : r == 2 ? q.z : q.w;
+    } else {
+      const ulonglong4 q = (s < 8) ? w[0] : w[1];
+      const uint32_t r = (s & 7) >> 1;
+      const uint64_t x = r == 0 ? q.x : r == 1 ? q.y : r == 2 ? q.z : q.w;
+      return (s & 1) ? (x >> 32) : (x & 0xFFFFFFFFull);
+    }
+  }
+  // number of keys <= k (the child index of k in an inner node: padding is above every key)
+  __device__ __forceinline__ uint32_t count_le(uint64_t k) const {
+    uint32_t c = 0;
+#pragma unroll
+    for (int x = 0; x < NW; ++x) {
+      const uint64_t q[4] = {w[x].x, w[x].y, w[x].z, w[x].w};
+#pragma unroll
+      for (int y = 0; y < 4; ++y) {
+        if constexpr (sizeof(tkey_t) == 8) {
+          c += q[y] <= k;
+        } else {
+          c += (q[y] & 0xFFFFFFFFull) <= k;
+          c += (q[y] >> 32) <= k;
+        }
+      }
+    }
+    return c;
+  }
+  // slot of key k (a valid key: never the padding), -1 if absent
+  __device__ __forceinline__ int find(uint64_t k) const {
+    int s = -1;
+#pragma unroll
+    for (int x = 0; x < NW; ++x) {
+      const uint64_t q[4] = {w[x].x, w[x].y, w[x].z, w[x].w};
+#pragma unroll
+      for (int y = 0; y < 4; ++y) {
+        if constexpr (sizeof(tkey_t) == 8) {
+          if (q[y] == k) s = 4 * x + y;
+        } else {
+          if ((q[y] & 0xFFFFFFFFull) == k) s = 8 * x + 2 * y;
+          if ((q[y] >> 32) == k) s = 8 * x + 2 * y + 1;
+        }
+      }
+    }
+    return s;
+  }
+};
 
 __device__ __forceinline__ uint64_t shfl64(uint64_t v, int src) {
   return __shfl_sync(FULL, (unsigned long long)v, src);
@@ -441,11 +525,11 @@ void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const C
                    BatchCtl* ctl, const TreeHdr* hdr, int dbgprint, int num_sms, cudaStream_t st, int* launches);
 
 // bulk build / scan
-int build_tree(Tree t, const uint64_t* keys, const uint64_t* vals, uint64_t n, int per_leaf, uint64_t key_lo,
+int build_tree(Tree t, const tkey_t* keys, const tkey_t* vals, uint64_t n, int per_leaf, uint64_t key_lo,
                uint64_t key_hi, cudaStream_t st, int* launches, uint32_t* height_out);
-void launch_validate_bulk(const uint64_t* keys, const uint64_t* vals, uint64_t n, uint64_t key_lo, uint64_t key_hi,
+void launch_validate_bulk(const tkey_t* keys, const tkey_t* vals, uint64_t n, uint64_t key_lo, uint64_t key_hi,
                           uint32_t* flag, cudaStream_t st, int* launches);
-int scan_tree(Tree t, uint32_t leaf_count, uint64_t lo, uint64_t hi, uint64_t* keys_out, uint64_t* vals_out,
+int scan_tree(Tree t, uint32_t leaf_count, uint64_t lo, uint64_t hi, tkey_t* keys_out, tkey_t* vals_out,
               uint64_t cap, uint64_t* count, cudaStream_t st, int* launches);
 
 // routing

@@ -937,8 +937,8 @@ __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uin
                            uint32_t r0, uint32_t r1, bool write_spay, GSmem& S,
                            uint32_t split_lo = 0xFFFFFFFFu, uint32_t split_h = 0, uint32_t split_w = 0) {
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  const uint64_t* __restrict__ vals = g.A->vals;
-  uint64_t* __restrict__ results = g.A->results;
+  const tkey_t* __restrict__ vals = g.A->vals;
+  tkey_t* __restrict__ results = g.A->results;
   const uint32_t len = r1 - r0;
   const uint32_t C = 32u * ((len + G_THREADS - 1) / G_THREADS);
   const uint32_t wb = r0 + warp * C;
@@ -1161,8 +1161,8 @@ __device__ void hot_pass2(const GroupArgs& g, uint32_t* bits, const HotCarry& c,
     }
   }
   __syncthreads();
-  const uint64_t* __restrict__ vals = g.A->vals;
-  uint64_t* __restrict__ results = g.A->results;
+  const tkey_t* __restrict__ vals = g.A->vals;
+  tkey_t* __restrict__ results = g.A->results;
   const uint32_t e = pos0 + c.total;
   for (uint32_t q0 = pos0 + tid; q0 < e && !defer; q0 += 8 * G_THREADS) {   // 8 in flight per thread
     uint32_t pw[8], py[8];

@@ -29,35 +29,20 @@ namespace eirene {
 
 namespace {
 
-// inner-node separator line: L1-allocating (lanes of neighbouring warps walk
-// shared upper nodes) with an L2 policy (evict_last: re-read every batch)
-__device__ __forceinline__ ulonglong4 ldg256_l1(const uint64_t* p, uint64_t pol) {
-  ulonglong4 v;
-  asm volatile("ld.global.nc.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
-               : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p), "l"(pol));
-  return v;
+// Child index of key k in inner node `node`: its separator line (Line16:
+// 256-bit loads, L1-allocating -- lanes of neighbouring warps walk shared upper
+// nodes -- with an L2 policy, evict_last: re-read every batch).
+__device__ __forceinline__ uint32_t child_slot(const Tree& t, uint32_t node, uint64_t k, uint64_t pol) {
+  Line16 l;
+  l.load_l1(t.ikeys + (size_t)node * FAN, pol);
+  return l.count_le(k);
 }
-// key s of a 16-key line held in registers (selects, no local memory)
-__device__ __forceinline__ uint64_t pick16(const ulonglong4 (&kv)[4], uint32_t s) {
-  const ulonglong4 q = (s < 8) ? ((s < 4) ? kv[0] : kv[1]) : ((s < 12) ? kv[2] : kv[3]);
-  const uint32_t r = s & 3;
-  return r == 0 ? q.x : r == 1 ? q.y : r == 2 ? q.z : q.w;
-}
-// Slot of key k in a 16-key leaf line (4 x 256-bit loads, L2 evict_first:
-// leaves are touched once per batch), -1 if absent.
-__device__ __forceinline__ int slot16(const uint64_t* __restrict__ line, uint64_t k, uint64_t pol) {
-  ulonglong4 v[4];
-#pragma unroll
-  for (int i = 0; i < 4; ++i) v[i] = ldg256_pol(line + 4 * i, pol);
-  int s = -1;
-#pragma unroll
-  for (int i = 0; i < 4; ++i) {
-    if (v[i].x == k) s = 4 * i;
-    if (v[i].y == k) s = 4 * i + 1;
-    if (v[i].z == k) s = 4 * i + 2;
-    if (v[i].w == k) s = 4 * i + 3;
-  }
-  return s;
+// Slot of key k in a 16-key leaf line (256-bit loads, L2 evict_first: leaves
+// are touched once per batch), -1 if absent.
+__device__ __forceinline__ int slot16(const tkey_t* __restrict__ line, uint64_t k, uint64_t pol) {
+  Line16 l;
+  l.load(line, pol);
+  return l.find(k);
 }
 
 // Everything after the locate of issued request i (list position i < nq:
@@ -79,8 +64,8 @@ struct QueryIO {
 };
 
 __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, uint32_t nq, uint32_t node, int s,
-                                       uint64_t v, uint64_t* __restrict__ results, BatchCtl* __restrict__ ctl,
-                                       uint64_t* __restrict__ lvals) {
+                                       uint64_t v, tkey_t* __restrict__ results, BatchCtl* __restrict__ ctl,
+                                       tkey_t* __restrict__ lvals) {
   const uint32_t* __restrict__ qseg = io.qseg;
   const uint32_t* __restrict__ wseg = io.wseg;
   const uint8_t* __restrict__ wop = io.wop;
@@ -162,7 +147,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   if (ctl->invalid || ctl->status != 0) return;
-  uint64_t* __restrict__ results = A->results;
+  tkey_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
   // pool headroom for the batch's worst case (every CTA computes the same
   // answer from the same tree header: none of them changes anything if it fails)
@@ -184,14 +169,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
       // the one child pointer: loading the whole child line alongside the keys
       // (one round trip per level instead of two) measured slower, as did two
       // or four interleaved traversals per thread (tools/ab.py)
-      const uint64_t* kl = t.ikeys + (size_t)node * FAN;
-      ulonglong4 kv[4];
-#pragma unroll
-      for (int x = 0; x < 4; ++x) kv[x] = ldg256_l1(kl + 4 * x, pl);
-      uint32_t c = 0;
-#pragma unroll
-      for (int x = 0; x < 4; ++x) c += (kv[x].x <= k) + (kv[x].y <= k) + (kv[x].z <= k) + (kv[x].w <= k);
-      node = ldg32_pol(t.ichild + (size_t)node * FAN + c, pl);
+      node = ldg32_pol(t.ichild + (size_t)node * FAN + child_slot(t, node, k, pl), pl);
     }
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
@@ -228,7 +206,7 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   if (ctl->invalid || ctl->status != 0) return;
-  uint64_t* __restrict__ results = A->results;
+  tkey_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw;
   if (!headroom_ok(t, nw)) {
     if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = EIRENE_EFULL;
@@ -264,14 +242,7 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
         node = root;
         for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
           parent = node;
-          const uint64_t* kp = t.ikeys + (size_t)node * FAN;
-          ulonglong4 kv[4];
-#pragma unroll
-          for (int x = 0; x < 4; ++x) kv[x] = ldg256_l1(kp + 4 * x, pl);
-          uint32_t c = 0;
-#pragma unroll
-          for (int x = 0; x < 4; ++x) c += (kv[x].x <= k) + (kv[x].y <= k) + (kv[x].z <= k) + (kv[x].w <= k);
-          node = ldg32_pol(t.ichild + (size_t)node * FAN + c, pl);
+          node = ldg32_pol(t.ichild + (size_t)node * FAN + child_slot(t, node, k, pl), pl);
         }
         steps = height;
       } else {
@@ -326,8 +297,8 @@ __global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __res
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   if (!(ctl->invalid || ctl->status != 0)) {
-    uint64_t* __restrict__ results = A->results;
-    const uint64_t* __restrict__ vals = A->vals;
+    tkey_t* __restrict__ results = A->results;
+    const tkey_t* __restrict__ vals = A->vals;
     const uint32_t nl = ctl->nlong;
     for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
       const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
@@ -421,8 +392,8 @@ __device__ __forceinline__ uint64_t artificial_query(uint32_t w, uint32_t t, uin
                                                      const uint32_t* __restrict__ spay,
                                                      const uint32_t* __restrict__ pinfo,
                                                      const uint64_t* __restrict__ kB,
-                                                     const uint64_t* __restrict__ vals,
-                                                     const uint64_t* __restrict__ results) {
+                                                     const tkey_t* __restrict__ vals,
+                                                     const tkey_t* __restrict__ results) {
   const uint32_t seg = wseg[w];
   uint32_t lo = istart[seg], hi = istart[seg + 1];
   const uint32_t p0 = lo;
@@ -442,7 +413,7 @@ __device__ __forceinline__ uint64_t artificial_query(uint32_t w, uint32_t t, uin
     const uint32_t pw = (uint32_t)kB[lo - 1];
     return ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
   }
-  return ld_cg(results + (pj >> 2));
+  return widen(ld_cg(results + (pj >> 2)));
 }
 
 __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_t* __restrict__ wkey,
@@ -458,11 +429,11 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
   if (ctl->invalid || ctl->status != 0 || ctl->nrange == 0) return;
   n = A->n;   // (the grid is sized for the graph's size bucket)
   const uint8_t* __restrict__ ops = A->ops;
-  const uint64_t* __restrict__ keys = A->keys;
-  const uint64_t* __restrict__ vals = A->vals;
-  uint64_t* __restrict__ results = A->results;
-  uint64_t* __restrict__ rkeys = A->rkeys;
-  uint64_t* __restrict__ rvals = A->rvals;
+  const tkey_t* __restrict__ keys = A->keys;
+  const tkey_t* __restrict__ vals = A->vals;
+  tkey_t* __restrict__ results = A->results;
+  tkey_t* __restrict__ rkeys = A->rkeys;
+  tkey_t* __restrict__ rvals = A->rvals;
   const uint32_t cap = A->rcap;
   const uint32_t nw = ctl->nw;
   const unsigned long long rw = t.hdr->root_word;
@@ -472,9 +443,9 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
     if (ops[i] != OP_RANGE) continue;
-    const uint64_t l = keys[i], u = vals[i];
-    uint64_t* __restrict__ ok = rkeys + (size_t)i * cap;
-    uint64_t* __restrict__ ov = rvals + (size_t)i * cap;
+    const uint64_t l = widen(keys[i]), u = widen(vals[i]);
+    tkey_t* __restrict__ ok = rkeys + (size_t)i * cap;
+    tkey_t* __restrict__ ov = rvals + (size_t)i * cap;
     uint32_t c = 0;
     if (l <= u && l != KEY_MAX) {   // (no key is UINT64_MAX; the descent needs l < the separator padding)
       // written keys >= l: lower_bound over the key-sorted issued writes
@@ -488,33 +459,22 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
       // leaf of l
       uint32_t node = root;
       for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
-        const uint64_t* kl = t.ikeys + (size_t)node * FAN;
-        ulonglong4 kv[4];
-#pragma unroll
-        for (int x = 0; x < 4; ++x) kv[x] = ldg256_l1(kl + 4 * x, pl);
-        uint32_t cc = 0;
-#pragma unroll
-        for (int x = 0; x < 4; ++x) cc += (kv[x].x <= l) + (kv[x].y <= l) + (kv[x].z <= l) + (kv[x].w <= l);
-        node = ldg32_pol(t.ichild + (size_t)node * FAN + cc, pl);
+        node = ldg32_pol(t.ichild + (size_t)node * FAN + child_slot(t, node, l, pl), pl);
       }
       // walk the leaf chain, merged with the written keys
       for (;;) {
-        const uint64_t* lk = t.lkeys + (size_t)node * LSTRIDE;
-        const uint64_t* lv = lk + FAN;
-        ulonglong4 kv[4];
-#pragma unroll
-        for (int x = 0; x < 4; ++x) kv[x] = ldg256_pol(lk + 4 * x, pf);
-        // slots [s0, s1) hold the leaf's keys in [l, u] (keys ascending, KEY_MAX padded)
+        const tkey_t* lk = t.lkeys + (size_t)node * LSTRIDE;
+        const tkey_t* lv = lk + FAN;
+        Line16 kv;
+        kv.load(lk, pf);
+        // slots [s0, s1) hold the leaf's keys in [l, u] (keys ascending, padding last)
         uint32_t s0 = 0, s1 = 0, nk = 0;
 #pragma unroll
-        for (int x = 0; x < 4; ++x) {
-          const uint64_t q[4] = {kv[x].x, kv[x].y, kv[x].z, kv[x].w};
-#pragma unroll
-          for (int y = 0; y < 4; ++y) {
-            s0 += q[y] < l;
-            s1 += q[y] <= u && q[y] != KEY_MAX;
-            nk += q[y] != KEY_MAX;
-          }
+        for (uint32_t j = 0; j < (uint32_t)FAN; ++j) {
+          const uint64_t q = widen((tkey_t)kv.at(j));
+          s0 += q < l;
+          s1 += q <= u && q != KEY_MAX;
+          nk += q != KEY_MAX;
         }
         if (wk > u) {
           // no written key left in [l, u]: the pairs come straight from the leaf;
@@ -524,19 +484,22 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
           // keys first (their registers die), then the value chunks that hold slots [s0, e)
 #pragma unroll
           for (uint32_t j = 0; j < (uint32_t)FAN; ++j)
-            if (j >= s0 && j < e) st64_pol(ok + c + (j - s0), pick16(kv, j), pf);
+            if (j >= s0 && j < e) st64_pol(ok + c + (j - s0), kv.at(j), pf);
+          // the value chunks (256 bits each) that hold slots [s0, e)
+          constexpr uint32_t PER = 32 / sizeof(tkey_t);
 #pragma unroll
-          for (int x = 0; x < 4; ++x) {
-            kv[x] = make_ulonglong4(0, 0, 0, 0);
-            if (4u * x < e && 4u * x + 4 > s0) kv[x] = ldg256_pol(lv + 4 * x, pf);
+          for (int x = 0; x < Line16::NW; ++x) {
+            kv.w[x] = make_ulonglong4(0, 0, 0, 0);
+            if (PER * x < e && PER * x + PER > s0)
+              kv.w[x] = ldg256_pol(reinterpret_cast<const uint64_t*>(lv) + 4 * x, pf);
           }
 #pragma unroll
           for (uint32_t j = 0; j < (uint32_t)FAN; ++j)
-            if (j >= s0 && j < e) st64_pol(ov + c + (j - s0), pick16(kv, j), pf);
+            if (j >= s0 && j < e) st64_pol(ov + c + (j - s0), kv.at(j), pf);
           c += take;
         } else {
           for (uint32_t s = s0; s < s1 && c < cap; ++s) {
-            const uint64_t k = pick16(kv, s);
+            const uint64_t k = kv.at(s);
             // written keys before k are absent from the pre-batch tree
             while (wk < k && c < cap) {
               const uint64_t v = artificial_query(w, i, KEY_MAX, wseg, istart, spay, pinfo, kB, vals, results);

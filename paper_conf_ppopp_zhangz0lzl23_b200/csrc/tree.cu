@@ -8,19 +8,19 @@ namespace eirene {
 
 namespace {
 
-__global__ void validate_bulk_kernel(const uint64_t* __restrict__ keys, const uint64_t* __restrict__ vals, uint64_t n,
+__global__ void validate_bulk_kernel(const tkey_t* __restrict__ keys, const tkey_t* __restrict__ vals, uint64_t n,
                                      uint64_t key_lo, uint64_t key_hi, uint32_t* flag) {
   const uint64_t stride = (uint64_t)gridDim.x * blockDim.x;
   bool bad = false;
   for (uint64_t i = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += stride) {
-    const uint64_t k = keys[i];
-    bad |= k == KEY_MAX || k < key_lo || k >= key_hi || vals[i] == KEY_MAX || (i > 0 && !(keys[i - 1] < k));
+    const uint64_t k = widen(keys[i]);
+    bad |= k == KEY_MAX || k < key_lo || k >= key_hi || widen(vals[i]) == KEY_MAX || (i > 0 && !(keys[i - 1] < k));
   }
   if (__any_sync(FULL, bad) && (threadIdx.x & 31) == 0) atomicOr(flag, 1u);
 }
 
 // Leaves: leaf q holds keys [q*per, min((q+1)*per, n)); fences from the keys.
-__global__ void build_leaves_kernel(const uint64_t* __restrict__ keys, const uint64_t* __restrict__ vals, uint64_t n,
+__global__ void build_leaves_kernel(const tkey_t* __restrict__ keys, const tkey_t* __restrict__ vals, uint64_t n,
                                     uint32_t per, uint32_t L, uint64_t key_lo, uint64_t key_hi, Tree t) {
   const uint64_t gid = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const uint64_t leaf = gid / FAN;
@@ -91,7 +91,7 @@ __global__ void leaf_count_kernel(Tree t, const uint32_t* __restrict__ order, ui
   const uint32_t leaf = order[i];
   uint64_t c = 0;
   for (int s = 0; s < FAN; ++s) {
-    const uint64_t k = t.lkeys[(size_t)leaf * LSTRIDE + s];
+    const uint64_t k = widen(t.lkeys[(size_t)leaf * LSTRIDE + s]);
     c += (k != KEY_MAX && k >= lo && k <= hi) ? 1 : 0;
   }
   cnt[i] = c;
@@ -130,14 +130,14 @@ __global__ void __launch_bounds__(1024) excl_scan_u64_kernel(uint64_t* __restric
 }
 
 __global__ void leaf_emit_kernel(Tree t, const uint32_t* __restrict__ order, const uint64_t* __restrict__ off,
-                                 uint32_t lc, uint64_t lo, uint64_t hi, uint64_t* __restrict__ ko,
-                                 uint64_t* __restrict__ vo, uint64_t cap) {
+                                 uint32_t lc, uint64_t lo, uint64_t hi, tkey_t* __restrict__ ko,
+                                 tkey_t* __restrict__ vo, uint64_t cap) {
   const uint32_t i = blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= lc) return;
   const uint32_t leaf = order[i];
   uint64_t o = off[i];
   for (int s = 0; s < FAN; ++s) {
-    const uint64_t k = t.lkeys[(size_t)leaf * LSTRIDE + s];
+    const uint64_t k = widen(t.lkeys[(size_t)leaf * LSTRIDE + s]);
     if (k != KEY_MAX && k >= lo && k <= hi) {
       if (o < cap) {
         if (ko) ko[o] = k;
@@ -150,7 +150,7 @@ __global__ void leaf_emit_kernel(Tree t, const uint32_t* __restrict__ order, con
 
 }  // namespace
 
-int build_tree(Tree t, const uint64_t* keys, const uint64_t* vals, uint64_t n, int per, uint64_t key_lo,
+int build_tree(Tree t, const tkey_t* keys, const tkey_t* vals, uint64_t n, int per, uint64_t key_lo,
                uint64_t key_hi, cudaStream_t st, int* launches, uint32_t* height_out) {
   // caller has validated and zeroed; per in [1, 16]
   const uint64_t L64 = (n + per - 1) / per;
@@ -187,7 +187,7 @@ int build_tree(Tree t, const uint64_t* keys, const uint64_t* vals, uint64_t n, i
   return EIRENE_OK;
 }
 
-void launch_validate_bulk(const uint64_t* keys, const uint64_t* vals, uint64_t n, uint64_t key_lo, uint64_t key_hi,
+void launch_validate_bulk(const tkey_t* keys, const tkey_t* vals, uint64_t n, uint64_t key_lo, uint64_t key_hi,
                           uint32_t* flag, cudaStream_t st, int* launches) {
   unsigned blocks = (unsigned)std::min<uint64_t>((n + 255) / 256, 148ull * 16ull);
   if (blocks < 1) blocks = 1;
@@ -195,7 +195,7 @@ void launch_validate_bulk(const uint64_t* keys, const uint64_t* vals, uint64_t n
   ++*launches;
 }
 
-int scan_tree(Tree t, uint32_t lc, uint64_t lo, uint64_t hi, uint64_t* ko, uint64_t* vo, uint64_t cap,
+int scan_tree(Tree t, uint32_t lc, uint64_t lo, uint64_t hi, tkey_t* ko, tkey_t* vo, uint64_t cap,
               uint64_t* count, cudaStream_t st, int* launches) {
   *count = 0;
   if (lc == 0 || lo > hi) return EIRENE_OK;

@@ -153,7 +153,7 @@ __device__ uint32_t descend(const Ctx& C, uint64_t k, uint32_t target, bool stm)
     uint32_t child = NIL;
     if (!right && lvl > target) {
       const size_t nb = (size_t)node * FAN;
-      const uint64_t key = lane < FAN ? ld_cg(t.ikeys + nb + lane) : KEY_MAX;
+      const uint64_t key = lane < FAN ? widen(ld_cg(t.ikeys + nb + lane)) : KEY_MAX;
       const uint32_t ch = lane < FAN ? ld_cg(t.ichild + nb + lane) : NIL;
       const uint32_t idx = __popc(__ballot_sync(FULL, lane < FAN - 1 && key <= k));
       child = shfl32(ch, idx);
@@ -535,7 +535,7 @@ __device__ void insert_up(const Ctx& C, uint32_t L0, uint32_t eb0, uint32_t m0, 
         uint32_t v;
         if (try_lock(vp, &v)) {
           const size_t pb = (size_t)P * FAN;
-          const uint64_t pk = lane < FAN ? ld_cg(t.ikeys + pb + lane) : KEY_MAX;
+          const uint64_t pk = lane < FAN ? widen(ld_cg(t.ikeys + pb + lane)) : KEY_MAX;
           const uint32_t pc = lane < FAN ? ld_cg(t.ichild + pb + lane) : NIL;
           const uint32_t cP = ld_cg(&t.imeta[P].count);
           const uint64_t plo = ld_cg(&t.imeta[P].lo), phi = ld_cg(&t.imeta[P].hi);
@@ -649,8 +649,8 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
         const uint64_t lo = ld_cg(&t.lmeta[X].lo), hi = ld_cg(&t.lmeta[X].hi);
         const uint32_t nxt = ld_cg(&t.lmeta[X].next);
         const size_t xb = (size_t)X * LSTRIDE;
-        const uint64_t okey = lane < FAN ? ld_cg(t.lkeys + xb + lane) : KEY_MAX;
-        const uint64_t oval = lane < FAN ? ld_cg(t.lvals + xb + lane) : 0;
+        const uint64_t okey = lane < FAN ? widen(ld_cg(t.lkeys + xb + lane)) : KEY_MAX;
+        const uint64_t oval = lane < FAN ? widen(ld_cg(t.lvals + xb + lane)) : 0;
         if (k0 >= lo && k0 < hi) {
           uint32_t e2 = e;
           for (uint32_t base = b; base < e; base += 32) {
@@ -756,7 +756,7 @@ __device__ uint32_t descend_thread(const Tree& t, uint64_t k, uint32_t target) {
       continue;
     }
     if (lvl == target) return node;
-    const uint64_t* kl = t.ikeys + (size_t)node * FAN;
+    const tkey_t* kl = t.ikeys + (size_t)node * FAN;
     uint32_t c = 0;
 #pragma unroll
     for (int i = 0; i < FAN - 1; ++i) c += ld_cg(kl + i) <= k ? 1u : 0u;
@@ -916,7 +916,7 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
       bool done = false;
       if (P != NIL && try_lock(vp, &v)) {
         const size_t pb = (size_t)P * FAN;
-        const uint64_t pk = lane < FAN ? ld_cg(t.ikeys + pb + lane) : KEY_MAX;
+        const uint64_t pk = lane < FAN ? widen(ld_cg(t.ikeys + pb + lane)) : KEY_MAX;
         const uint32_t pc = lane < FAN ? ld_cg(t.ichild + pb + lane) : NIL;
         const uint32_t cP = ld_cg(&t.imeta[P].count);
         const uint64_t plo = ld_cg(&t.imeta[P].lo), phi = ld_cg(&t.imeta[P].hi);
@@ -1123,7 +1123,7 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
       bool ok = true;
       if (fast) {
         const size_t at = (size_t)lf * LSTRIDE + sl;
-        if (ld_cg(t.lkeys + at) == C.wkey[j]) {
+        if (widen(ld_cg(t.lkeys + at)) == C.wkey[j]) {
           t.lvals[at] = C.wval[j];
         } else {
           ok = false;

@@ -42,8 +42,12 @@ class EireneTree:
     def __init__(self, max_keys: int = 1 << 24, max_batch: int = 1 << 20, device: int | None = None,
                  retry_threshold: int = 4, regroup: bool = True, stats: bool = True, force_stm: bool = False,
                  timing: bool = False, key_lo: int = 0, key_hi: int = U64_MAX, iterwarp: bool = False,
-                 iter_rgs: int = 0, pipeline: bool = False):
-        L = _ffi.lib()
+                 iter_rgs: int = 0, pipeline: bool = False, key_bits: int = 64):
+        # key_bits 32: libeirene32.so (32-bit keys and values); tensors torch.uint32
+        L = _ffi.lib(key_bits)
+        self.key_bits = key_bits
+        self.kdtype = torch.uint32 if key_bits == 32 else torch.uint64
+        self.not_found = (1 << key_bits) - 1
         if device is None:
             device = torch.cuda.current_device()
         self.device = torch.device("cuda", device)
@@ -90,8 +94,8 @@ class EireneTree:
 
     # ---------------------------------------------------------------- ABI calls
     def bulk_load(self, keys: torch.Tensor, vals: torch.Tensor, leaf_fill: float = 1.0, stream=None):
-        _need(keys, torch.uint64, self.device, "keys")
-        _need(vals, torch.uint64, self.device, "vals", keys.numel())
+        _need(keys, self.kdtype, self.device, "keys")
+        _need(vals, self.kdtype, self.device, "vals", keys.numel())
         check(self._L.eirene_bulk_load(self._h, _ptr(keys), _ptr(vals), keys.numel(), leaf_fill,
                                        self._stream(stream)), "eirene_bulk_load")
 
@@ -99,9 +103,9 @@ class EireneTree:
                stream=None) -> int:
         n = ops.numel()
         _need(ops, torch.uint8, self.device, "ops")
-        _need(keys, torch.uint64, self.device, "keys", n)
-        _need(vals, torch.uint64, self.device, "vals", n)
-        _need(results, torch.uint64, self.device, "results", n)
+        _need(keys, self.kdtype, self.device, "keys", n)
+        _need(vals, self.kdtype, self.device, "vals", n)
+        _need(results, self.kdtype, self.device, "results", n)
         tk = ctypes.c_uint64()
         check(self._L.eirene_submit_batch(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n, _ptr(results),
                                           self._stream(stream), ctypes.byref(tk)), "eirene_submit_batch")
@@ -117,11 +121,11 @@ class EireneTree:
         range_keys / range_vals are [n, cap] u64; row i receives the first results[i] pairs of R(l, u)."""
         n = ops.numel()
         _need(ops, torch.uint8, self.device, "ops")
-        _need(keys, torch.uint64, self.device, "keys", n)
-        _need(vals, torch.uint64, self.device, "vals", n)
-        _need(results, torch.uint64, self.device, "results", n)
-        _need(range_keys, torch.uint64, self.device, "range_keys", n * cap)
-        _need(range_vals, torch.uint64, self.device, "range_vals", n * cap)
+        _need(keys, self.kdtype, self.device, "keys", n)
+        _need(vals, self.kdtype, self.device, "vals", n)
+        _need(results, self.kdtype, self.device, "results", n)
+        _need(range_keys, self.kdtype, self.device, "range_keys", n * cap)
+        _need(range_vals, self.kdtype, self.device, "range_vals", n * cap)
         tk = ctypes.c_uint64()
         check(self._L.eirene_submit_batch_range(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n, _ptr(results), cap,
                                                 _ptr(range_keys), _ptr(range_vals), self._stream(stream),
@@ -131,9 +135,9 @@ class EireneTree:
     def apply_range(self, ops, keys, vals, cap: int, stream=None):
         """submit_range + results: returns (results, range_keys [n, cap], range_vals [n, cap], stats)."""
         n = ops.numel()
-        res = torch.empty(n, dtype=torch.uint64, device=self.device)
-        rk = torch.zeros((n, cap), dtype=torch.uint64, device=self.device)
-        rv = torch.zeros((n, cap), dtype=torch.uint64, device=self.device)
+        res = torch.empty(n, dtype=self.kdtype, device=self.device)
+        rk = torch.zeros((n, cap), dtype=self.kdtype, device=self.device)
+        rv = torch.zeros((n, cap), dtype=self.kdtype, device=self.device)
         tk = self.submit_range(ops, keys, vals, res, cap, rk, rv, stream)
         return res, rk, rv, self.results(tk)
 
@@ -145,9 +149,9 @@ class EireneTree:
         n = ops.numel()
         cpu = torch.device("cpu")
         _need(ops, torch.uint8, cpu, "ops")
-        _need(keys, torch.uint64, cpu, "keys", n)
-        _need(vals, torch.uint64, cpu, "vals", n)
-        _need(results, torch.uint64, cpu, "results", n)
+        _need(keys, self.kdtype, cpu, "keys", n)
+        _need(vals, self.kdtype, cpu, "vals", n)
+        _need(results, self.kdtype, cpu, "results", n)
         tk = ctypes.c_uint64()
         check(self._L.eirene_submit_batch_host(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n, _ptr(results),
                                                self._stream(stream), ctypes.byref(tk)), "eirene_submit_batch_host")
@@ -170,17 +174,18 @@ class EireneTree:
     def apply(self, ops, keys, vals, results=None, stream=None):
         """submit + results: returns (results tensor, stats dict)."""
         if results is None:
-            results = torch.empty(ops.numel(), dtype=torch.uint64, device=self.device)
+            results = torch.empty(ops.numel(), dtype=self.kdtype, device=self.device)
         tk = self.submit(ops, keys, vals, results, stream)
         return results, self.results(tk)
 
     def scan(self, lo: int = 0, hi: int = U64_MAX - 1, stream=None):
+        hi = min(hi, self.not_found - 1)
         cnt = ctypes.c_uint64()
         s = self._stream(stream)
         check(self._L.eirene_scan(self._h, lo, hi, None, None, 0, ctypes.byref(cnt), s), "eirene_scan")
         n = cnt.value
-        k = torch.empty(max(n, 1), dtype=torch.uint64, device=self.device)
-        v = torch.empty(max(n, 1), dtype=torch.uint64, device=self.device)
+        k = torch.empty(max(n, 1), dtype=self.kdtype, device=self.device)
+        v = torch.empty(max(n, 1), dtype=self.kdtype, device=self.device)
         check(self._L.eirene_scan(self._h, lo, hi, _ptr(k), _ptr(v), n, ctypes.byref(cnt), s), "eirene_scan")
         return k[:n], v[:n]
 

@@ -74,27 +74,35 @@ def sorted_unique(a: np.ndarray) -> np.ndarray:
     return s[keep]
 
 
-def loaded_keys(n: int, seed: int) -> tuple[np.ndarray, np.ndarray]:
-    """n distinct EVEN u64 keys (sorted) and their values (never UINT64_MAX)."""
+def loaded_keys(n: int, seed: int, key_bits: int = 64) -> tuple[np.ndarray, np.ndarray]:
+    """n distinct EVEN keys (sorted) and their values (never the all-ones NOT_FOUND);
+    key_bits 32: 32-bit keys and values (the u32 variant)."""
     keys = np.empty(0, dtype=np.uint64)
     start = 0
     while keys.size < n:
         need = n - keys.size
-        draw = rand_u64(seed, S_LOAD_KEY, start, need + need // 64 + 16) & ~np.uint64(1)
+        draw = rand_u64(seed, S_LOAD_KEY, start, need + need // 64 + 16)
+        if key_bits == 32:
+            draw >>= np.uint64(32)
+        draw &= ~np.uint64(1)
         start += draw.size
         keys = sorted_unique(np.concatenate([keys, draw]))
     if keys.size > n:
         # drop a seeded random subset so the kept keys stay uniform
         drop = np.argsort(rand_u64(seed, S_LOAD_KEY ^ 0x55, 0, keys.size))[: keys.size - n]
         keys = np.delete(keys, drop)
-    vals = rand_u64(seed, S_LOAD_VAL, 0, n) >> np.uint64(1)
+    vals = rand_u64(seed, S_LOAD_VAL, 0, n) >> np.uint64(1 if key_bits == 64 else 33)
     return keys, vals
 
 
-def fresh_keys(seed: int, batch: int, count: int) -> np.ndarray:
+def fresh_keys(seed: int, batch: int, count: int, key_bits: int = 64) -> np.ndarray:
     """Fresh insert keys: odd, so disjoint from the (even) loaded keys."""
-    k = rand_u64(seed, S_FRESH, batch << 32, count) | np.uint64(1)
-    k[k == U64_MAX] ^= np.uint64(2)
+    k = rand_u64(seed, S_FRESH, batch << 32, count)
+    if key_bits == 32:
+        k >>= np.uint64(32)
+    k |= np.uint64(1)
+    top = np.uint64(U64_MAX if key_bits == 64 else 0xFFFFFFFF)
+    k[k == top] ^= np.uint64(2)
     return k
 
 
@@ -161,7 +169,8 @@ def shuffled_ops(n: int, fracs: dict[int, float], seed: int, batch: int) -> np.n
 
 
 def make_batch(loaded: np.ndarray, n: int, fracs: dict[int, float], dist: str, seed: int,
-               batch: int, zipf: Zipf | None = None, live: np.ndarray | None = None, range_len: int = 8):
+               batch: int, zipf: Zipf | None = None, live: np.ndarray | None = None, range_len: int = 8,
+               key_bits: int = 64):
     """One request batch: (ops u8[n], keys u64[n], vals u64[n]).
 
     QUERY/UPDATE keys are drawn from `loaded` (uniform or scrambled Zipf);
@@ -181,12 +190,12 @@ def make_batch(loaded: np.ndarray, n: int, fracs: dict[int, float], dist: str, s
         raise ValueError(dist)
     keys[sel] = loaded[idx]
     ins = ops == INSERT
-    keys[ins] = fresh_keys(seed, batch, int(ins.sum()))
+    keys[ins] = fresh_keys(seed, batch, int(ins.sum()), key_bits)
     dele = ops == DELETE
     if dele.any():
         pool = live if live is not None else loaded
         keys[dele] = pool[uniform_index(rand_u64(seed, S_DEL, batch << 32, int(dele.sum())), len(pool))]
-    vals = rand_u64(seed, S_WVAL, batch << 32, n) >> np.uint64(1)
+    vals = rand_u64(seed, S_WVAL, batch << 32, n) >> np.uint64(1 if key_bits == 64 else 33)
     vals[ops == QUERY] = 0
     rng_ = ops == RANGE
     if rng_.any():
@@ -209,6 +218,9 @@ CONFIGS = {
     5: dict(tree=1 << 28, batch=1 << 24, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="zipf", strong=True),
     # the paper's pure range-query workload (Fig.13), length 8
     6: dict(tree=1 << 24, batch=1 << 20, fracs={RANGE: 1.0}, dist="uniform", range_len=8),
+    # the paper's default workload with its record width -- 32-bit keys and
+    # values, 2^23-key tree, 1M-request batches, 95% query / 5% update, uniform
+    7: dict(tree=1 << 23, batch=1 << 20, fracs={QUERY: 0.95, UPDATE: 0.05}, dist="uniform", key_bits=32),
 }
 
 
@@ -233,8 +245,9 @@ class Workload:
 
     def __init__(self, cfg: int, tree: int | None = None, batch: int | None = None,
                  fracs: dict | None = None, dist: str | None = None, seed: int | None = None,
-                 range_len: int | None = None):
+                 range_len: int | None = None, key_bits: int | None = None):
         c = dict(CONFIGS[cfg])
+        self.key_bits = key_bits or c.get("key_bits", 64)
         self.range_len = range_len or c.get("range_len", 8)
         self.cfg = cfg
         self.tree = tree or c["tree"]
@@ -242,13 +255,13 @@ class Workload:
         self.fracs = fracs or c["fracs"]
         self.dist = dist or c["dist"]
         self.seed = seed_for(cfg) if seed is None else seed
-        self.keys, self.vals = loaded_keys(self.tree, self.seed)
+        self.keys, self.vals = loaded_keys(self.tree, self.seed, self.key_bits)
         self.zipf = Zipf(self.tree) if self.dist == "zipf" else None
         self.live = self.keys if DELETE in self.fracs else None
 
     def batch_arrays(self, b: int):
         ops, keys, vals = make_batch(self.keys, self.batch, self.fracs, self.dist, self.seed, b,
-                                     zipf=self.zipf, live=self.live, range_len=self.range_len)
+                                     zipf=self.zipf, live=self.live, range_len=self.range_len, key_bits=self.key_bits)
         if self.live is not None:
             # live-key snapshot for the next batch (generator bookkeeping only)
             ins = keys[ops == INSERT]

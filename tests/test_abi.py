@@ -32,6 +32,24 @@ def test_exports_are_c_linkage(libpath):
         assert n in exported, n
 
 
+def test_key32_library_exports_the_same_abi(libpath):
+    """libeirene32.so (-DEIRENE_KEY32) exports the same C ABI
+    with 32-bit keys / values; it builds for sm_100a only."""
+    from paper_conf_ppopp_zhangz0lzl23_b200.build import build_all
+    p32 = build_all()[1]
+    assert p32.endswith("libeirene32.so")
+    L = ctypes.CDLL(p32)
+    assert not [n for n in _ffi.header_functions() if not hasattr(L, n)]
+    out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", p32], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+    L32 = _ffi.lib(32)
+    h = ctypes.c_void_p()
+    cfg = _ffi.eirene_config()
+    L32.eirene_default_config(ctypes.byref(cfg))
+    cfg.key_lo = 1 << 32   # no 32-bit key lies at or above 2^32 - 1
+    assert L32.eirene_create(ctypes.byref(cfg), ctypes.byref(h)) == _ffi.EIRENE_EINVAL
+
+
 def test_sm100a_code_only(libpath):
     out = subprocess.run(["/usr/local/cuda/bin/cuobjdump", "--list-elf", libpath], capture_output=True,
                          text=True).stdout
@@ -91,4 +109,5 @@ def test_probe_gather_argument_checks(libpath):
     assert L.eirene_probe_gather(None, 1 << 20, 16, 0, 1, None) == _ffi.EIRENE_EINVAL
     assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 1024, 16, 0, 1, None) == _ffi.EIRENE_EINVAL   # short
     assert L.eirene_probe_gather(ctypes.c_void_p((1 << 20) + 8), 1 << 20, 16, 0, 1, None) == _ffi.EIRENE_EINVAL
-    assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 1 << 20, 16, 3, 1, None) == _ffi.EIRENE_EINVAL
+    assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 1 << 20, 16, 4, 1, None) == _ffi.EIRENE_EINVAL   # kind
+    assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 3 << 20, 16, 0, 1, None) == _ffi.EIRENE_EINVAL   # not 2^k
