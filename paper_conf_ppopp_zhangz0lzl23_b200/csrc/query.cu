@@ -37,6 +37,31 @@ __device__ __forceinline__ uint32_t child_slot(const Tree& t, uint32_t node, uin
   l.load_l1(t.ikeys + (size_t)node * FAN, pol);
   return l.count_le(k);
 }
+// The value of a located key (one 32 B value sector of its leaf).  A/B builds:
+// -DEIRENE_VAL_LOAD=1: L1 no-allocate; 2: plain coherent load; 0 (default):
+// read-only path with the evict_first L2 policy.
+#ifndef EIRENE_VAL_LOAD
+#define EIRENE_VAL_LOAD 0
+#endif
+__device__ __forceinline__ uint64_t load_value(const tkey_t* p, uint64_t pol) {
+#if EIRENE_VAL_LOAD == 1
+  if constexpr (sizeof(tkey_t) == 8) {
+    uint64_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+    return v;
+  } else {
+    uint32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+  }
+#elif EIRENE_VAL_LOAD == 2
+  (void)pol;
+  return *p;
+#else
+  return ldg64_pol(p, pol);
+#endif
+}
+
 // Slot of key k in a 16-key leaf line (256-bit loads, L2 evict_first: leaves
 // are touched once per batch), -1 if absent.
 __device__ __forceinline__ int slot16(const tkey_t* __restrict__ line, uint64_t k, uint64_t pol) {
@@ -172,7 +197,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
       node = ldg32_pol(t.ichild + (size_t)node * FAN + child_slot(t, node, k, pl), pl);
     }
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
-    const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
+    const uint64_t v = s >= 0 ? load_value(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
     if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
     retire(QueryIO{qseg, wseg, wop, wval, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
            results, ctl, t.lvals);
@@ -254,7 +279,7 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
         }
       }
       const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
-      const uint64_t v = s >= 0 ? ldg64_pol(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
+      const uint64_t v = s >= 0 ? load_value(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
       if (act && !isq) wparent[base + lane] = parent;
       if (act) retire(io, isq ? base + lane : nq + base + lane, isq, nq, node, s, v, results, ctl, t.lvals);
       __syncwarp();
