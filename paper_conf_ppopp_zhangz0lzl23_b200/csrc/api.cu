@@ -110,7 +110,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
   }
 }
 
-// kernels in one batch graph: set_args, 1-2 sort, group, query, update, result_long
+// kernels in one batch graph: set_args, 1-2 sort, group, query, (range), update + result phase
 constexpr int SET_ARGS_CTAS = 4;
 constexpr int MAX_GRAPHS = 8;
 
@@ -183,7 +183,7 @@ struct eirene_tree {
   CombBufs cbL{};
   BatchCtl* ctl = nullptr;
   BatchCtl* host_ctl = nullptr;   // pinned [RING]: landing buffer of eirene_results
-  BatchCtl* ctl_ring = nullptr;   // device [RING]: each batch's final BatchCtl (written by result_long)
+  BatchCtl* ctl_ring = nullptr;   // device [RING]: each batch's final BatchCtl (written by the update kernel's result phase)
   cudaStream_t res_stream = nullptr;
   cudaStream_t h2d_stream = nullptr, d2h_stream = nullptr;
   cudaEvent_t h2d_done[HOST_SLOTS] = {}, comp_ev[HOST_SLOTS] = {}, comp_done[HOST_SLOTS] = {};
@@ -682,10 +682,12 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
     if (range) launch_range(nk, L.cb, spay, L.bs.kB, L.dargs, h->t, L.ctl, h->num_sms, s, nl);
     stage("query", s);
     if (timing) rec(3, s);
-    launch_update(nk, L.cb, h->t, L.ctl, h->up, h->num_sms, s, nl);
+    const ResultArgs ra{spay, L.bs.kB, L.cb.pinfo, L.cb.istart, L.cb.longseg, L.cb.old, L.dargs, L.ctl, h->t.hdr};
+    launch_update(nk, L.cb, h->t, L.ctl, h->up, ra, h->num_sms, s, nl);
     stage("update", s);
     if (timing) rec(4, s);
-    launch_result(spay, L.bs.kB, nk, L.cb, L.dargs, L.ctl, h->t.hdr, dbg ? 1 : 0, h->num_sms, s, nl);
+    if (dbg) launch_result(L.ctl, 1, s);
+    else launch_result(L.ctl, 0, s);
     stage("result", s);
     if (timing) rec(5, s);
     return cudaGetLastError();

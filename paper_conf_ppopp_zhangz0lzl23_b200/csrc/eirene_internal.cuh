@@ -38,10 +38,10 @@ constexpr uint32_t NIL = 0xFFFFFFFFu;
 constexpr int MAX_LEVELS = 32;
 constexpr uint32_t DONE_BIT = 0x80000000u;    // pinfo: an earlier write of the segment decides the result
 constexpr uint32_t DEFER_BIT = 0x40000000u;   // pinfo (hot-key segments): that early result is written by
-                                              // result_long_kernel from the nearest write's payload in kB
+                                              // result phase from the nearest write's payload in kB
 constexpr uint32_t SEG_MASK = 0x3FFFFFFFu;
 constexpr uint32_t Q_SINGLE = 0x80000000u;    // qseg entry of a one-request query segment: Q_SINGLE | its timestamp
-constexpr uint32_t RCHUNK = 4096;             // result_long_kernel work item: positions of one long segment
+constexpr uint32_t RCHUNK = 4096;             // result phase work item: positions of one long segment
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 
 enum { OP_QUERY = 0, OP_UPDATE = 1, OP_INSERT = 2, OP_DELETE = 3, OP_RANGE = 4 };
@@ -77,7 +77,7 @@ struct BatchCtl {
   uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
   uint32_t ndelp;         // issued deletes of present keys (query kernel); nins == ndelp == 0 -> every
                           // issued write was a value overwrite, applied in place by the query kernel
-  uint32_t fin_ctr;       // result_long_kernel: CTAs finished (the last one publishes the BatchCtl)
+  uint32_t fin_ctr;       // update kernel's result phase: CTAs finished (the last one publishes the BatchCtl)
   unsigned long long t_begin, t_end;   // %globaltimer (ns) at the batch's first / last kernel
   uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
   uint32_t uchunk;        // update kernel: next 32-write chunk (dynamic, level-synchronous mode)
@@ -485,7 +485,7 @@ struct CombBufs {
   uint32_t* wparent;          // [n] the write's leaf's parent (level-1 node) at locate time, NIL if the root is a leaf
   uint64_t* old;              // [n] old value per segment
   uint32_t* istart;           // [n+1] sorted position of each segment's first request (+ n at nseg)
-  uint32_t* longseg;          // [n] segments longer than SHORT_SEG, finished by result_long_kernel
+  uint32_t* longseg;          // [n] segments longer than SHORT_SEG, finished by the result phase
   uint32_t* hot_bits;         // [HOT_SLOTS][3][hot_words] timestamp bitmaps of hot keys: present, op bit 0,
                               // op bit 1 (all zero between batches)
   uint32_t hot_words;         // >= max_batch / 32, a multiple of 4
@@ -516,13 +516,15 @@ struct UpdParams {
   uint32_t* flat_child;
   uint32_t* flat_off;   // [producers] exclusive prefix of the producers' entry counts
 };
-void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms,
-                   cudaStream_t st, int* launches);
+struct ResultArgs;
+// update kernel (Alg.1:23-46), then the result phase (long-segment RESULT_CAL, Alg.1:6, and the
+// batch's final BatchCtl): the batch's last kernel
+void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, const ResultArgs& r,
+                   int num_sms, cudaStream_t st, int* launches);
 // range queries R(l, u): between the query and the update kernel
 void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const uint64_t* kB, const BatchArgs* A, Tree t,
                   BatchCtl* ctl, int num_sms, cudaStream_t st, int* launches);
-void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const CombBufs& c, const BatchArgs* A,
-                   BatchCtl* ctl, const TreeHdr* hdr, int dbgprint, int num_sms, cudaStream_t st, int* launches);
+void launch_result(const BatchCtl* ctl, int dbgprint, cudaStream_t st);   // diagnostics print only
 
 // bulk build / scan
 int build_tree(Tree t, const tkey_t* keys, const tkey_t* vals, uint64_t n, int per_leaf, uint64_t key_lo,
@@ -544,5 +546,91 @@ void launch_route_unpack(const uint64_t* rec, uint32_t n, uint8_t* ops, uint64_t
                          cudaStream_t st, int* launches);
 void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,
                             cudaStream_t st, int* launches);
+
+// RESULT_CAL is fused into the query kernel: every issued
+// request scatters the value it retrieved to the pending positions of its own
+// segment.  The segments longer than SHORT_SEG (hot keys) are queued instead
+// and finished here, work items of RCHUNK positions spread over the CTAs, so a
+// 56K-request Zipf key does not serialise one thread.
+struct ResultArgs {
+  const uint32_t* spay;
+  const uint64_t* kB;
+  const uint32_t* pinfo;
+  const uint32_t* istart;
+  const uint32_t* longseg;
+  const uint64_t* old;
+  const BatchArgs* A;
+  BatchCtl* ctl;
+  const TreeHdr* hdr;
+};
+// Run by every CTA of the batch's last kernel (the update kernel), after its
+// structural work: the long segments need only the query kernel's old values,
+// so they need no grid barrier after the updates.
+__device__ __forceinline__ void result_phase(const ResultArgs& R) {
+  const uint32_t* __restrict__ spay = R.spay;
+  const uint64_t* __restrict__ kB = R.kB;
+  const uint32_t* __restrict__ pinfo = R.pinfo;
+  const uint32_t* __restrict__ istart = R.istart;
+  const uint32_t* __restrict__ longseg = R.longseg;
+  const uint64_t* __restrict__ old = R.old;
+  const BatchArgs* __restrict__ A = R.A;
+  BatchCtl* __restrict__ ctl = R.ctl;
+  const TreeHdr* hdr = R.hdr;
+  if (!(ctl->invalid || ctl->status != 0)) {
+    tkey_t* __restrict__ results = A->results;
+    const tkey_t* __restrict__ vals = A->vals;
+    const uint32_t nl = ctl->nlong;
+    for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
+      const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
+      const uint64_t v = old[s];
+      const uint32_t b = istart[s] + ch * RCHUNK;
+      const uint32_t e = min(istart[s + 1], b + RCHUNK);
+      for (uint32_t p0 = b + threadIdx.x; p0 < e; p0 += 4 * blockDim.x) {   // 4 loads in flight
+        uint32_t pi[4], py[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          const uint32_t p = p0 + u * blockDim.x;
+          pi[u] = p < e ? pinfo[p] : DONE_BIT;
+          py[u] = p < e ? spay[p] : 0u;
+        }
+#pragma unroll
+        for (int u = 0; u < 4; ++u) {
+          if (!(pi[u] & DONE_BIT)) {
+            results[py[u] >> 2] = v;   // no earlier write in the segment: the issued request's value
+          } else if (pi[u] & DEFER_BIT) {   // hot key: the nearest earlier write (its payload in kB)
+            const uint32_t pw = (uint32_t)kB[p0 + u * blockDim.x];
+            results[py[u] >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
+          }
+        }
+      }
+    }
+  }
+  // End of the batch (the last kernel): the last CTA to finish stamps the
+  // device end time, sets the final status and height and publishes the whole
+  // BatchCtl to the batch's ring slot (one word per thread).
+  __shared__ uint32_t s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(&ctl->fin_ctr, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  if (threadIdx.x == 0) {
+    if (ld_cg(&ctl->invalid)) ctl->status = EIRENE_EINVAL;
+    ctl->height = (uint32_t)(hdr->root_word >> 32);
+    ctl->t_begin = A->t0;
+    ctl->t_end = gtime_ns();
+  }
+  __syncthreads();
+  {
+    static_assert(sizeof(BatchCtl) % 8 == 0, "BatchCtl is copied as u64 words");
+    const unsigned long long* src = reinterpret_cast<const unsigned long long*>(ctl);
+    unsigned long long* dst = reinterpret_cast<unsigned long long*>(A->ctl_out);
+    for (uint32_t i = threadIdx.x; i < sizeof(BatchCtl) / 8; i += blockDim.x) dst[i] = __ldcg(src + i);
+  }
+}
+
 
 }  // namespace eirene

@@ -1090,7 +1090,7 @@ __device__ HotCarry hot_pass1(const GroupArgs& g, const uint32_t* bits, GSmem& S
 
 // Pass 2 + results; sH = the hot segment's index, pos0 = its first sorted position.
 // The early results of the DONE positions are written here only for a short
-// segment; a long one's positions are marked DEFER and result_long_kernel,
+// segment; a long one's positions are marked DEFER and the result phase,
 // which spreads long segments over many CTAs, writes them.
 // Pass 2 walks the bitmaps warp-contiguously (warp w owns the words of
 // threads [32w, 32w + 32) of pass 1, lanes read consecutive words), so the
@@ -1102,7 +1102,7 @@ __device__ void hot_pass2(const GroupArgs& g, uint32_t* bits, const HotCarry& c,
   const uint32_t wbeg = min(W, (uint32_t)(tid & ~31) * PW), wend = min(W, wbeg + 32u * PW);
   // the warp's carries = those of its lane 0 in pass 1
   uint32_t rank = __shfl_sync(FULL, c.rank, 0), prev = __shfl_sync(FULL, c.lw, 0);
-  // a long hot segment's early results are left to result_long_kernel (many CTAs)
+  // a long hot segment's early results are left to the result phase (many CTAs)
   const bool defer = c.total > SHORT_SEG;
   const uint32_t dbits = DONE_BIT | (defer ? DEFER_BIT : 0u);
   constexpr int D = 4;   // steps whose loads are issued together

@@ -20,7 +20,7 @@
 // RESULT_CAL: the un-issued requests of a segment that have no
 // earlier write take the retrieved value.  The thread that retrieved it
 // scatters it to its segment's pending positions (results in timestamp
-// order); segments longer than SHORT_SEG are queued for result_long_kernel.
+// order); segments longer than SHORT_SEG are queued for the update kernel's result phase.
 #include "eirene_internal.cuh"
 #include <cstdio>
 #include <cstdlib>
@@ -134,7 +134,7 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
     if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&ctl->nins, (uint32_t)__popc(m));
     if (md && (threadIdx.x & 31) == __ffs(md) - 1) atomicAdd(&ctl->ndelp, (uint32_t)__popc(md));
   }
-  // old[seg] (the pre-batch value) is read by result_long_kernel for long
+  // old[seg] (the pre-batch value) is read by the result phase for long
   // segments and by the range kernel for written keys only
   if (!isq) old[seg] = v;
   const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
@@ -196,6 +196,9 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
       // or four interleaved traversals per thread (tools/ab.py)
       node = ldg32_pol(t.ichild + (size_t)node * FAN + child_slot(t, node, k, pl), pl);
     }
+#if EIRENE_VAL_LOAD == 3   // A/B: the leaf's value line prefetched into L2 alongside its key line
+    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(t.lvals + (size_t)node * LSTRIDE));
+#endif
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? load_value(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
     if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
@@ -302,78 +305,6 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
     atomicAdd(&ctl->trav_steps, nsteps);
     atomicAdd(&ctl->rg_vertical, nvert);
     atomicAdd(&ctl->rg_horizontal, nhor);
-  }
-}
-
-// RESULT_CAL is fused into the query kernel: every issued request scatters
-// the value it retrieved to the pending positions of its own segment.  The
-// segments longer than SHORT_SEG (hot keys) are queued instead and finished
-// here with one CTA per segment, so a 56K-request Zipf key does not serialise
-// one thread.
-__global__ void __launch_bounds__(1024) result_long_kernel(const uint32_t* __restrict__ spay,
-                                                            const uint64_t* __restrict__ kB,
-                                                            const uint32_t* __restrict__ pinfo,
-                                                            const uint32_t* __restrict__ istart,
-                                                            const uint32_t* __restrict__ longseg,
-                                                            const uint64_t* __restrict__ old,
-                                                            const BatchArgs* __restrict__ A,
-                                                            BatchCtl* __restrict__ ctl, const TreeHdr* hdr,
-                                                            int dbgprint) {
-  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
-  pdl_trigger();
-  if (!(ctl->invalid || ctl->status != 0)) {
-    tkey_t* __restrict__ results = A->results;
-    const tkey_t* __restrict__ vals = A->vals;
-    const uint32_t nl = ctl->nlong;
-    for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
-      const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
-      const uint64_t v = old[s];
-      const uint32_t b = istart[s] + ch * RCHUNK;
-      const uint32_t e = min(istart[s + 1], b + RCHUNK);
-      for (uint32_t p0 = b + threadIdx.x; p0 < e; p0 += 4 * blockDim.x) {   // 4 loads in flight
-        uint32_t pi[4], py[4];
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          const uint32_t p = p0 + u * blockDim.x;
-          pi[u] = p < e ? pinfo[p] : DONE_BIT;
-          py[u] = p < e ? spay[p] : 0u;
-        }
-#pragma unroll
-        for (int u = 0; u < 4; ++u) {
-          if (!(pi[u] & DONE_BIT)) {
-            results[py[u] >> 2] = v;   // no earlier write in the segment: the issued request's value
-          } else if (pi[u] & DEFER_BIT) {   // hot key: the nearest earlier write (its payload in kB)
-            const uint32_t pw = (uint32_t)kB[p0 + u * blockDim.x];
-            results[py[u] >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
-          }
-        }
-      }
-    }
-  }
-  // End of the batch (the last kernel): the last CTA to finish stamps the
-  // device end time, sets the final status and height and publishes the whole
-  // BatchCtl to the batch's ring slot (one word per thread).
-  __shared__ uint32_t s_last;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-    s_last = atomicAdd(&ctl->fin_ctr, 1u) == gridDim.x - 1;
-  }
-  __syncthreads();
-  if (!s_last) return;
-  __threadfence();
-  if (threadIdx.x == 0) {
-    if (ld_cg(&ctl->invalid)) ctl->status = EIRENE_EINVAL;
-    ctl->height = (uint32_t)(hdr->root_word >> 32);
-    ctl->t_begin = A->t0;
-    ctl->t_end = gtime_ns();
-  }
-  __syncthreads();
-  {
-    static_assert(sizeof(BatchCtl) % 8 == 0, "BatchCtl is copied as u64 words");
-    const unsigned long long* src = reinterpret_cast<const unsigned long long*>(ctl);
-    unsigned long long* dst = reinterpret_cast<unsigned long long*>(A->ctl_out);
-    for (uint32_t i = threadIdx.x; i < sizeof(BatchCtl) / 8; i += blockDim.x) dst[i] = __ldcg(src + i);
   }
 }
 
@@ -613,16 +544,11 @@ void launch_range(uint32_t n, const CombBufs& c, const uint32_t* spay, const uin
   ++*launches;
 }
 
-void launch_result(const uint32_t* spay, const uint64_t* kB, uint32_t n, const CombBufs& c, const BatchArgs* A,
-                   BatchCtl* ctl, const TreeHdr* hdr, int dbgprint, int num_sms, cudaStream_t st, int* launches) {
-  // one 1024-thread CTA per SM: enough for the long segments of a Zipf batch
-  // (RCHUNK work items), cheap when there are none
-  const uint32_t grid = std::max(1u, std::min<uint32_t>((uint32_t)num_sms, (n + 1023) / 1024));
-  launch_k(result_long_kernel, dim3(grid), dim3(1024), 0, st, true, false, spay, kB, c.pinfo, c.istart, c.longseg, c.old, A, ctl, hdr,
-                                                       dbgprint);
+void launch_result(const BatchCtl* ctl, int dbgprint, cudaStream_t st) {
+  // (RESULT_CAL of the long segments and the batch's BatchCtl are the update
+  // kernel's last phase, result_phase; only the diagnostics print is left here)
   static const bool uprof = std::getenv("EIRENE_UPDATE_PROF") != nullptr;
   if (dbgprint || uprof) debug_print_kernel<<<1, 1, 0, st>>>(ctl, dbgprint);
-  ++*launches;
 }
 
 }  // namespace eirene

@@ -1048,15 +1048,26 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
 #define UPD_MINB 6   // resident CTAs per SM the register budget is fitted to (A/B builds: -DUPD_MINB=n;
                      // r1h: 6 (80 regs, no spills) vs 8 (64 regs, 432 B spills): cfg1 0.389 -> 0.404, cfg2 6.92 -> 7.04)
 #endif
-__global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
+__device__ __forceinline__ void update_body(const Ctx& C);
+
+// The batch's last kernel: the structural writes (Alg.1:23-46), then every
+// CTA's share of the long-segment RESULT_CAL and the batch's BatchCtl
+// (result_phase, eirene_internal.cuh) -- one launch for both.
+__global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C, ResultArgs R) {
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   const BatchCtl* ctl = C.ctl;
-  if (ctl->invalid || ctl->status != 0) return;   // (uniform: every CTA leaves, no barrier is reached)
-  // every issued write a value overwrite of a present key: all of them were
-  // applied in place by the query kernel's locate (query.cu, retire), nothing
-  // structural is left (uniform)
-  if (ctl->nins == 0 && ctl->ndelp == 0) return;
+  // skipped (uniformly: every CTA reads the same flags before any changes them)
+  // for a rejected batch, and when every issued write was a value overwrite of
+  // a present key: all of them were applied in place by the query kernel's
+  // locate (query.cu, retire), nothing structural is left
+  const bool skip = ctl->invalid || ctl->status != 0 || (ctl->nins == 0 && ctl->ndelp == 0);
+  if (!skip) update_body(C);
+  result_phase(R);
+}
+
+__device__ __forceinline__ void update_body(const Ctx& C) {
+  const BatchCtl* ctl = C.ctl;
   if (g_uprof && blockIdx.x == 0 && threadIdx.x == 0) C.ctl->uprof[0] = gtime_ns();
   const uint32_t nw = ctl->nw;
   const int lane = lane_id();
@@ -1205,8 +1216,8 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C) {
 
 }  // namespace
 
-void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, int num_sms, cudaStream_t st,
-                   int* launches) {
+void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdParams p, const ResultArgs& r,
+                   int num_sms, cudaStream_t st, int* launches) {
   Ctx C;
   C.t = t;
   C.wkey = c.wkey;
@@ -1252,12 +1263,12 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
     return (int)cudaMemcpyToSymbol(g_uprof, &on, sizeof(int));
   });
   if (serial) {
-    update_kernel<<<1, 32, 0, st>>>(C);
+    update_kernel<<<1, 32, 0, st>>>(C, r);
   } else {
     if (C.slots[0]) {   // grid barriers: cooperative launch (co-residency guaranteed)
-      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, true, C);
+      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, true, C, r);
     } else {
-      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, false, C);
+      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, false, C, r);
     }
   }
   ++*launches;
