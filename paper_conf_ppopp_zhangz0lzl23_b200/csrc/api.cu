@@ -88,7 +88,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
                                                         tkey_t* results, BatchCtl* ctl_out, uint4* zero,
                                                         uint32_t zero_n16, uint4* zero2, uint32_t zero2_n16,
                                                         tkey_t* rkeys, tkey_t* rvals, uint32_t rcap,
-                                                        uint32_t n, unsigned long long* phase) {
+                                                        uint32_t n, unsigned long long* phase, uint32_t seq) {
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero_n16; i += gridDim.x * blockDim.x)
     zero[i] = make_uint4(0, 0, 0, 0);
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < zero2_n16; i += gridDim.x * blockDim.x)
@@ -107,6 +107,7 @@ __global__ void __launch_bounds__(1024) set_args_kernel(BatchArgs* dst, const ui
     dst->rcap = rcap;
     dst->n = n;
     dst->phase = phase;
+    dst->seq = seq;
   }
 }
 
@@ -194,6 +195,8 @@ struct eirene_tree {
   tkey_t* st_vals = nullptr;
   tkey_t* st_res = nullptr;
   unsigned long long* route_lb = nullptr;
+  unsigned long long* hot_lb = nullptr;   // result phase's look-back over the deferred hot keys' chunks
+  uint32_t hot_chunks = 0;
   uint32_t* route_ctr = nullptr;
   uint32_t route_epoch = 0;
   Rec ring[RING];
@@ -324,6 +327,9 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->cb.longseg, nb + 64);   // (segment, chunk) pairs of the long segments
   h->cb.hot_words = (uint32_t)(((nb + 127) / 128) * 4);   // multiple of 4 (uint4 access)
   AL(h->cb.hot_bits, (size_t)HOT_SLOTS * 3 * h->cb.hot_words);
+  AL(h->cb.hot_seg, HOT_SLOTS);
+  h->hot_chunks = (h->cb.hot_words + HOT_CHW - 1) / HOT_CHW;
+  AL(h->hot_lb, (size_t)HOT_SLOTS * h->hot_chunks);   // epoch-tagged: never needs zeroing between batches
   AL(h->up.entA_key, nb + 64);
   AL(h->up.entA_child, nb + 64);
   AL(h->up.entB_key, nb + 64);
@@ -422,6 +428,9 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     AL(wop, nb);
     AL(wval, nb);
     AL(wseg, nb);
+    uint32_t *hbits = nullptr, *hseg = nullptr;   // hot-key bitmaps: set by the front, walked by the back
+    AL(hbits, (size_t)HOT_SLOTS * 3 * h->cb.hot_words);
+    AL(hseg, HOT_SLOTS);
     AL(L1.dargs, 1);
     AL(L1.zero_region, h->zero_bytes);
     if (h->zero_large) AL(L1.zero_large, h->zero_large_bytes);
@@ -450,11 +459,14 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
         c->wop = wop;
         c->wval = wval;
         c->wseg = wseg;
+        c->hot_bits = hbits;
+        c->hot_seg = hseg;
       }
       L1.cb.group_status = rz(h->cb.group_status);
       if (h->zero_large) L1.cbL.group_status = rl(h->cbL.group_status);
       h->nlanes = 2;
       e = cudaMemset(L1.zero_region, 0, h->zero_bytes);
+      if (e == cudaSuccess) e = cudaMemset(hbits, 0, sizeof(uint32_t) * HOT_SLOTS * 3 * h->cb.hot_words);
       if (e == cudaSuccess && L1.zero_large) e = cudaMemset(L1.zero_large, 0, h->zero_large_bytes);
       if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->back_stream, cudaStreamNonBlocking);
     }
@@ -471,6 +483,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
     for (int s = 0; s < NSTAGE && e == cudaSuccess; ++s) e = cudaEventCreate(&h->ring[i].st[s]);
   }
   if (e == cudaSuccess) e = cudaMemset(h->cb.hot_bits, 0, sizeof(uint32_t) * HOT_SLOTS * 3 * h->cb.hot_words);
+  if (e == cudaSuccess) e = cudaMemset(h->hot_lb, 0, sizeof(unsigned long long) * HOT_SLOTS * h->hot_chunks);
   if (e == cudaSuccess) e = cudaMemset(h->sb.lookback, 0, sizeof(unsigned long long) * sort_tiles * 256);
   if (e == cudaSuccess) e = cudaMemset(h->route_lb, 0, sizeof(unsigned long long) * ((nb + 2047) / 2048) * 64);
   if (e == cudaSuccess) {
@@ -656,7 +669,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
     uint4* zero2 = reinterpret_cast<uint4*>(large ? L.zero_large : L.zero_region);
     const uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
     set_args_kernel<<<SET_ARGS_CTAS, 1024, 0, s>>>(L.dargs, ops, keys, vals, vals_stage, results, ctl_slot, zero16,
-                                                   zero_n16, zero2, zero2_n16, rkeys, rvals, rcap, n, h->phase);
+                                                   zero_n16, zero2, zero2_n16, rkeys, rvals, rcap, n, h->phase, seq);
     ++*nl;
     if (args_node) {
       cudaError_t e = capture_node(s, args_node);
@@ -682,7 +695,9 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
     if (range) launch_range(nk, L.cb, spay, L.bs.kB, L.dargs, h->t, L.ctl, h->num_sms, s, nl);
     stage("query", s);
     if (timing) rec(3, s);
-    const ResultArgs ra{spay, L.bs.kB, L.cb.pinfo, L.cb.istart, L.cb.longseg, L.cb.old, L.dargs, L.ctl, h->t.hdr};
+    const ResultArgs ra{spay,          L.bs.kB,  L.cb.pinfo,       L.cb.istart,    L.cb.longseg,
+                        L.cb.old,      L.dargs,  L.ctl,            h->t.hdr,       L.cb.hot_bits,
+                        L.cb.hot_words, L.cb.hot_seg, h->hot_lb,   h->hot_chunks};
     launch_update(nk, L.cb, h->t, L.ctl, h->up, ra, h->num_sms, s, nl);
     stage("update", s);
     if (timing) rec(4, s);
@@ -699,7 +714,7 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
     uint32_t zero2_n16 = large ? (uint32_t)(h->zero_large_bytes / 16) : 0u;
     void* params[] = {&L.dargs, const_cast<uint8_t**>(&ops), const_cast<tkey_t**>(&keys),
                       const_cast<tkey_t**>(&vals), &vals_stage, &results, &ctl_slot, &zero16, &zero_n16,
-                      &zero2, &zero2_n16, &rkeys, &rvals, &rcap, &n, &h->phase};
+                      &zero2, &zero2_n16, &rkeys, &rvals, &rcap, &n, &h->phase, const_cast<uint32_t*>(&seq)};
     cudaKernelNodeParams p{};
     p.func = reinterpret_cast<void*>(set_args_kernel);
     p.gridDim = dim3(SET_ARGS_CTAS);

@@ -41,7 +41,8 @@ constexpr uint32_t DEFER_BIT = 0x40000000u;   // pinfo (hot-key segments): that 
                                               // result phase from the nearest write's payload in kB
 constexpr uint32_t SEG_MASK = 0x3FFFFFFFu;
 constexpr uint32_t Q_SINGLE = 0x80000000u;    // qseg entry of a one-request query segment: Q_SINGLE | its timestamp
-constexpr uint32_t RCHUNK = 4096;             // result phase work item: positions of one long segment
+constexpr uint32_t RCHUNK = 512;              // result phase work item: positions of one long segment
+                                              // (4 per thread of the update kernel's 128-thread CTAs)
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 
 enum { OP_QUERY = 0, OP_UPDATE = 1, OP_INSERT = 2, OP_DELETE = 3, OP_RANGE = 4 };
@@ -74,6 +75,7 @@ struct BatchCtl {
   uint32_t nlong, gbar;   // gbar: grid barrier of bsort_dist_kernel
   uint32_t nrange, nart;  // range queries in the batch; artificial queries resolved
   uint32_t hot_ctr;       // hot-key timestamp bitmaps claimed by oversized groups
+  uint32_t hot_item;      // result phase: next (hot key, bitmap chunk) work item
   uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
   uint32_t ndelp;         // issued deletes of present keys (query kernel); nins == ndelp == 0 -> every
                           // issued write was a value overwrite, applied in place by the query kernel
@@ -134,6 +136,7 @@ struct BatchArgs {
   unsigned long long t0;   // %globaltimer when the batch's first kernel started (device batch time)
   uint32_t n;              // requests in the batch (launches are sized for the graph's size bucket >= n)
   unsigned long long* phase;   // diagnostic builds (-DEIRENE_PHASE_PROF): [kernel][CTA][phase] %globaltimer stamps
+  uint32_t seq;                // the handle's batch sequence number (epoch of the result phase's look-back)
 };
 
 // Phase timestamps of the distribution / group kernels (diagnostic builds only:
@@ -489,6 +492,7 @@ struct CombBufs {
   uint32_t* hot_bits;         // [HOT_SLOTS][3][hot_words] timestamp bitmaps of hot keys: present, op bit 0,
                               // op bit 1 (all zero between batches)
   uint32_t hot_words;         // >= max_batch / 32, a multiple of 4
+  uint32_t* hot_seg;          // [HOT_SLOTS] segment of each hot key whose bitmap the result phase walks
 };
 constexpr int HOT_SLOTS = 64;
 #ifndef EIRENE_SHORT_SEG
@@ -562,7 +566,13 @@ struct ResultArgs {
   const BatchArgs* A;
   BatchCtl* ctl;
   const TreeHdr* hdr;
+  uint32_t* hot_bits;             // deferred hot keys: bitmap slots [HOT_SLOTS][3][hot_words] (cleared here)
+  uint32_t hot_words;
+  const uint32_t* hot_seg;        // [HOT_SLOTS] their segments
+  unsigned long long* hot_lb;     // [HOT_SLOTS][HOT_CHUNKS_MAX] epoch-tagged look-back words
+  uint32_t hot_chunks;            // chunks per slot (hot_words / HOT_CHW, rounded up)
 };
+constexpr uint32_t HOT_CHW = 1024;   // bitmap words (32K timestamps) per result-phase work item
 // Run by every CTA of the batch's last kernel (the update kernel), after its
 // structural work: the long segments need only the query kernel's old values,
 // so they need no grid barrier after the updates.
@@ -576,12 +586,22 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
   const BatchArgs* __restrict__ A = R.A;
   BatchCtl* __restrict__ ctl = R.ctl;
   const TreeHdr* hdr = R.hdr;
+  __shared__ uint32_t s_hseg[HOT_SLOTS];
+  __shared__ uint32_t s_item, s_red[32];
+  const uint32_t njobs = min(ld_cg(&ctl->hot_ctr), (uint32_t)HOT_SLOTS);
+  // (a deferred hot key's segment is walked below, not through its positions)
+  const uint32_t nhot = A->rkeys == nullptr ? njobs : 0u;
+  for (uint32_t j = threadIdx.x; j < nhot; j += blockDim.x) s_hseg[j] = ld_cg(R.hot_seg + j);
+  __syncthreads();
   if (!(ctl->invalid || ctl->status != 0)) {
     tkey_t* __restrict__ results = A->results;
     const tkey_t* __restrict__ vals = A->vals;
     const uint32_t nl = ctl->nlong;
     for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
       const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
+      bool hotseg = false;
+      for (uint32_t j = 0; j < nhot; ++j) hotseg |= s_hseg[j] == s;
+      if (hotseg) continue;   // (uniform in the CTA)
       const uint64_t v = old[s];
       const uint32_t b = istart[s] + ch * RCHUNK;
       const uint32_t e = min(istart[s + 1], b + RCHUNK);
@@ -602,6 +622,102 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
             results[py[u] >> 2] = ((pw & 3) == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
           }
         }
+      }
+    }
+  }
+  if (!ctl->invalid) {   // (the group kernel set the bits of any valid batch: walk them even if it failed later)
+    tkey_t* __restrict__ results = A->results;
+    const tkey_t* __restrict__ vals = A->vals;
+    const bool ok = ctl->status == 0;
+    // Deferred hot keys (SPLIT groups, group.cu): the bits of slot j are the key's
+    // requests in timestamp order (present / op bit 0 / op bit 1 bitmaps over
+    // [0, n)).  Work items (slot, chunk of HOT_CHW words) are taken in order; a
+    // request's result is the value of the nearest earlier write of the key
+    // (NOT_FOUND if a delete) or, with none, the pre-batch value old[seg]
+    // (P:746-758); the nearest earlier write across chunks comes
+    // from an epoch-tagged decoupled look-back (max of write payloads).
+    const uint32_t C = R.hot_chunks, W = R.hot_words, items = nhot * C;
+    const unsigned long long ep = (unsigned long long)(A->seq & 0x3FFFFFFFu) << 34;
+    const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
+    for (;;) {
+      __syncthreads();
+      if (threadIdx.x == 0) s_item = atomicAdd(&ctl->hot_item, 1u);
+      __syncthreads();
+      const uint32_t item = s_item;
+      if (item >= items) break;
+      const uint32_t j = item / C, c = item - j * C;
+      uint32_t* bits = R.hot_bits + (size_t)j * 3 * W;
+      const uint32_t sH = s_hseg[j];
+      const uint32_t w0 = c * HOT_CHW, w1 = min(W, w0 + HOT_CHW);
+      const uint32_t PW = (HOT_CHW + blockDim.x - 1) / blockDim.x;
+      const uint32_t tw0 = min(w1, w0 + threadIdx.x * PW), tw1 = min(w1, tw0 + PW);
+      // pass 1: this thread's last write payload (0: none)
+      uint32_t lw = 0;
+      for (uint32_t x = tw0; x < tw1; ++x) {
+        const uint32_t wm = __ldcg(bits + x) & (__ldcg(bits + W + x) | __ldcg(bits + 2 * W + x));
+        if (wm) {
+          const uint32_t tb = 31 - __clz(wm);
+          lw = ((x * 32 + tb) << 2) | ((__ldcg(bits + W + x) >> tb) & 1u) | (((__ldcg(bits + 2 * W + x) >> tb) & 1u) << 1);
+        }
+      }
+      // exclusive max-scan over the threads (ascending word ranges), chunk aggregate
+      uint32_t inc = lw;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, inc, o);
+        if ((int)lane >= o) inc = max(inc, y);
+      }
+      if (lane == 31) s_red[warp] = inc;
+      __syncthreads();
+      uint32_t before = 0, agg = 0;
+      for (uint32_t w = 0; w < nwarp; ++w) {
+        if (w < warp) before = max(before, s_red[w]);
+        agg = max(agg, s_red[w]);
+      }
+      const uint32_t excl = max(before, __shfl_up_sync(FULL, inc, 1) * (lane ? 1u : 0u));
+      // look-back over the slot's earlier chunks: the nearest write before this chunk
+      __shared__ uint32_t s_carry;
+      if (threadIdx.x == 0) {
+        unsigned long long* lb = R.hot_lb + (size_t)j * C;
+        uint32_t carry = 0;
+        if (c == 0) {
+          st_relaxed64(lb, ep | (2ull << 32) | agg);
+        } else {
+          st_relaxed64(lb + c, ep | (1ull << 32) | agg);
+          SpinGuard sg;
+          for (int32_t pc = (int32_t)c - 1; pc >= 0;) {
+            const unsigned long long wv = ld_relaxed64(lb + pc);
+            const uint32_t fl = (uint32_t)(wv >> 32) & 3u;
+            if ((wv & ~((1ull << 34) - 1)) != ep || fl == 0) {   // not yet published this batch
+              if (sg.stuck(ctl)) break;
+              continue;
+            }
+            carry = max(carry, (uint32_t)wv);
+            if (fl == 2) break;
+            --pc;
+          }
+          st_relaxed64(lb + c, ep | (2ull << 32) | max(carry, agg));
+        }
+        s_carry = carry;
+      }
+      __syncthreads();
+      // pass 2: every request of the thread's words, in timestamp order
+      uint32_t pv = max(s_carry, excl);
+      const uint64_t vold = ok ? old[sH] : 0;
+      for (uint32_t x = tw0; x < tw1; ++x) {
+        const uint32_t pw = __ldcg(bits + x);
+        if (!pw) continue;
+        const uint32_t b0 = __ldcg(bits + W + x), b1 = __ldcg(bits + 2 * W + x);
+        for (uint32_t m = pw; m; m &= m - 1) {
+          const uint32_t tb = __ffs(m) - 1;
+          const uint32_t op = ((b0 >> tb) & 1u) | (((b1 >> tb) & 1u) << 1);
+          const uint32_t ts = x * 32 + tb;
+          if (ok) results[ts] = pv ? (((pv & 3) == OP_DELETE) ? KEY_MAX : (uint64_t)vals[pv >> 2]) : vold;
+          if (op) pv = (ts << 2) | op;
+        }
+        bits[x] = 0u;   // leave the slot clean for the next batch
+        bits[W + x] = 0u;
+        bits[2 * W + x] = 0u;
       }
     }
   }

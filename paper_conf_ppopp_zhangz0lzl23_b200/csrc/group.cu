@@ -76,6 +76,7 @@ struct GSmem {
   uint64_t ck[32];
   uint32_t cp[32];
   uint32_t hr_lt, hr_eq, hr_nc, hr_cm;
+  uint32_t hot_lastw, hot_lastp, hot_slot;   // split-off hot key: last write / last payload, bitmap slot
 };
 
 __device__ __forceinline__ bool kp_less(uint64_t ka, uint32_t pa, uint64_t kb, uint32_t pb) {
@@ -730,9 +731,13 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
     // for keys holding more than n / 128 requests -- at most 128 of them
     if (tid == 0) {
       uint32_t* b = nullptr;
+      S.hot_slot = 0xFFFFFFFFu;
       if (hot_base && hcnt > max((uint32_t)G_CAP, nreq >> 7)) {
         const uint32_t slot = atomicAdd(hot_ctr, 1u);
-        if (slot < (uint32_t)HOT_SLOTS) b = hot_base + (size_t)slot * 3 * hot_words;
+        if (slot < (uint32_t)HOT_SLOTS) {
+          b = hot_base + (size_t)slot * 3 * hot_words;
+          S.hot_slot = slot;
+        }
       }
       S.hot_bits = b;
     }
@@ -743,8 +748,11 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
       S.r_nh = 0;   // rest
       S.r_lw = 0;   // hk
       S.r_nw = 0;   // rest below hk
+      S.hot_lastw = 0;   // hk's last write payload (0: none; a write's op bits are never 0)
+      S.hot_lastp = 0;   // hk's last payload
     }
     __syncthreads();
+    uint32_t my_lw = 0, my_lp = 0;
     for (uint32_t b0 = 0; b0 < cnt; b0 += 8 * G_THREADS) {   // 8 loads in flight per thread
       uint64_t kk[8];
       uint32_t pp[8];
@@ -771,6 +779,8 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
         bh = __shfl_sync(FULL, bh, 0);
         bo = __shfl_sync(FULL, bo, 0);
         if (hot) {
+          my_lp = max(my_lp, p);
+          if (p & 3) my_lw = max(my_lw, p);
           if (bits) {   // timestamp bitmaps: the set bits ARE the hot key's requests in timestamp order
             const uint32_t ts = p >> 2, wd = ts >> 5, bit = 1u << (ts & 31);
             atomicOr(bits + wd, bit);
@@ -786,6 +796,12 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
           S.p[x] = p;
         }
       }
+    }
+    my_lw = __reduce_max_sync(FULL, my_lw);
+    my_lp = __reduce_max_sync(FULL, my_lp);
+    if (lane == 0) {
+      if (my_lw) atomicMax(&S.hot_lastw, my_lw);
+      if (my_lp) atomicMax(&S.hot_lastp, my_lp);
     }
     __syncthreads();
     const uint32_t o = S.r_nh, h = S.r_lw, lo = S.r_nw;
@@ -851,6 +867,7 @@ struct GroupArgs {
   unsigned long long* status;   // [nb] look-back words (zeroed per batch)
   uint32_t* hot_bits;           // [HOT_SLOTS][hot_words] timestamp bitmaps, zero between uses
   uint32_t hot_words;
+  uint32_t* hot_seg;            // [HOT_SLOTS] segment of each deferred hot key (result phase)
   int prof;                     // EIRENE_GROUP_PROF: print the phases of slow groups (diagnostic)
   Tree t;
   BatchCtl* ctl;
@@ -1208,6 +1225,10 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     P = S.p;
   }
   int mode = 0;   // 0: small / L2-sorted group, 2: SPLIT (rest in smem, hot key in a bitmap)
+  // SPLIT groups of a batch without range queries hand the hot key's bitmap to
+  // the result phase (multi-CTA); range batches need the segment's positions
+  // (artificial queries binary-search them) and walk it here (hot_pass2)
+  const bool deferred = g.A->rkeys == nullptr;
   uint32_t sp_o = 0, sp_h = 0, sp_lo = 0;
   if (!small) {
     const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S, g.hot_bits,
@@ -1267,9 +1288,14 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       c_nw = S.r_nw;
     }
     __syncthreads();
-    hc = hot_pass1(g, S.hot_bits, S);
-    hot_w = hc.last_w ? 1u : 0u;
-    hot_last = hc.last_w ? hc.last_w : hc.last_p;   // issue rule: the last write, else the last query
+    if (deferred) {   // the aggregate came with the split scan; the bitmap walk is the result phase's
+      hot_w = S.hot_lastw ? 1u : 0u;
+      hot_last = S.hot_lastw ? S.hot_lastw : S.hot_lastp;
+    } else {
+      hc = hot_pass1(g, S.hot_bits, S);
+      hot_w = hc.last_w ? 1u : 0u;
+      hot_last = hc.last_w ? hc.last_w : hc.last_p;   // issue rule: the last write, else the last query
+    }
     c_nh += 1;
     c_nw += hot_w;
     __syncthreads();
@@ -1343,11 +1369,15 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
     __syncthreads();
     const uint32_t sH = S.seg0 + a_nh, wH = S.w0 + a_nw, pos0 = base + sp_lo;
     if ((g.prof & 1) && tid == 0) S.prof_t[0] = gtime_ns();
-    hot_pass2(g, S.hot_bits, hc, sH, pos0);
+    if (!deferred) hot_pass2(g, S.hot_bits, hc, sH, pos0);
     if ((g.prof & 1) && tid == 0) S.prof_t[1] = gtime_ns();
     if (tid == 0) {
       const uint64_t hk = S.hk;
       g.istart[sH] = pos0;
+      // deferred: the segment's positions (pinfo, sorted payloads) are not
+      // written; every result of it comes from the result phase's walk of the
+      // bitmap slot, spread over many CTAs (result_phase, eirene_internal.cuh)
+      if (deferred) g.hot_seg[S.hot_slot] = sH;
       if (hot_w) {   // issue rule: the segment's last write
         const uint32_t opw = hot_last & 3;
         g.wkey[wH] = hk;
@@ -1418,6 +1448,7 @@ void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const Comb
   g.status = c.group_status;
   g.hot_bits = c.hot_bits;
   g.hot_words = c.hot_words;
+  g.hot_seg = c.hot_seg;
   static const int prof = std::getenv("EIRENE_GROUP_PROF") ? std::atoi(std::getenv("EIRENE_GROUP_PROF")) : 0;
   g.prof = prof;
   g.t = t;

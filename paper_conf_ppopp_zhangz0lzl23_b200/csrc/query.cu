@@ -196,9 +196,6 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
       // or four interleaved traversals per thread (tools/ab.py)
       node = ldg32_pol(t.ichild + (size_t)node * FAN + child_slot(t, node, k, pl), pl);
     }
-#if EIRENE_VAL_LOAD == 3   // A/B: the leaf's value line prefetched into L2 alongside its key line
-    asm volatile("prefetch.global.L2::evict_last [%0];" ::"l"(t.lvals + (size_t)node * LSTRIDE));
-#endif
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? load_value(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
     if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
