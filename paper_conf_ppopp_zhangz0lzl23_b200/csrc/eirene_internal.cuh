@@ -79,7 +79,8 @@ struct BatchCtl {
   uint32_t nins;          // issued upserts of absent keys (query kernel): 0 -> no split is possible
   uint32_t ndelp;         // issued deletes of present keys (query kernel); nins == ndelp == 0 -> every
                           // issued write was a value overwrite, applied in place by the query kernel
-  uint32_t fin_ctr;       // update kernel's result phase: CTAs finished (the last one publishes the BatchCtl)
+  uint32_t fin_ctr;       // update kernel's result phase: residue classes finished (the last publishes the BatchCtl)
+  uint32_t fin_sub[16];   // ... CTAs finished per residue class blockIdx % 16
   unsigned long long t_begin, t_end;   // %globaltimer (ns) at the batch's first / last kernel
   uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
   uint32_t uchunk;        // update kernel: next 32-write chunk (dynamic, level-synchronous mode)
@@ -639,7 +640,7 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
     const uint32_t C = R.hot_chunks, W = R.hot_words, items = nhot * C;
     const unsigned long long ep = (unsigned long long)(A->seq & 0x3FFFFFFFu) << 34;
     const uint32_t lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nwarp = blockDim.x >> 5;
-    for (;;) {
+    for (; items;) {   // (no deferred hot key: no ticket atomics at all)
       __syncthreads();
       if (threadIdx.x == 0) s_item = atomicAdd(&ctl->hot_item, 1u);
       __syncthreads();
@@ -724,11 +725,20 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
   // End of the batch (the last kernel): the last CTA to finish stamps the
   // device end time, sets the final status and height and publishes the whole
   // BatchCtl to the batch's ring slot (one word per thread).
+  // two-level arrival count (16 counters, then one): ~gridDim/16 same-address
+  // atomics per counter instead of gridDim on one
   __shared__ uint32_t s_last;
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
-    s_last = atomicAdd(&ctl->fin_ctr, 1u) == gridDim.x - 1;
+    const uint32_t grp = blockIdx.x & 15u, gsize = (gridDim.x + 15u - grp) / 16u;   // CTAs with this residue
+    bool last = false;
+    if (atomicAdd(&ctl->fin_sub[grp], 1u) == gsize - 1) {   // the last of its residue class
+      __threadfence();
+      const uint32_t ngrp = min(16u, gridDim.x);
+      last = atomicAdd(&ctl->fin_ctr, 1u) == ngrp - 1;
+    }
+    s_last = last;
   }
   __syncthreads();
   if (!s_last) return;
