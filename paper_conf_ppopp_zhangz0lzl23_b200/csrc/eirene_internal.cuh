@@ -589,15 +589,21 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
   const TreeHdr* hdr = R.hdr;
   __shared__ uint32_t s_hseg[HOT_SLOTS];
   __shared__ uint32_t s_item, s_red[32];
-  const uint32_t njobs = min(ld_cg(&ctl->hot_ctr), (uint32_t)HOT_SLOTS);
+  // the batch's scalars, loaded together (independent loads: one round trip)
+  const uint32_t c_invalid = ld_cg(&ctl->invalid), c_status = ld_cg(reinterpret_cast<const uint32_t*>(&ctl->status));
+  const uint32_t c_nlong = ld_cg(&ctl->nlong), c_hot = ld_cg(&ctl->hot_ctr);
+  const bool c_range = A->rkeys != nullptr;
+  const uint32_t njobs = min(c_hot, (uint32_t)HOT_SLOTS);
   // (a deferred hot key's segment is walked below, not through its positions)
-  const uint32_t nhot = A->rkeys == nullptr ? njobs : 0u;
-  for (uint32_t j = threadIdx.x; j < nhot; j += blockDim.x) s_hseg[j] = ld_cg(R.hot_seg + j);
-  __syncthreads();
-  if (!(ctl->invalid || ctl->status != 0)) {
+  const uint32_t nhot = c_range ? 0u : njobs;
+  if (nhot) {   // (uniform)
+    for (uint32_t j = threadIdx.x; j < nhot; j += blockDim.x) s_hseg[j] = ld_cg(R.hot_seg + j);
+    __syncthreads();
+  }
+  if (!(c_invalid || c_status != 0)) {
     tkey_t* __restrict__ results = A->results;
     const tkey_t* __restrict__ vals = A->vals;
-    const uint32_t nl = ctl->nlong;
+    const uint32_t nl = c_nlong;
     for (uint32_t x = blockIdx.x; x < nl; x += gridDim.x) {
       const uint32_t s = longseg[2 * x], ch = longseg[2 * x + 1];
       bool hotseg = false;
@@ -626,10 +632,10 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
       }
     }
   }
-  if (!ctl->invalid) {   // (the group kernel set the bits of any valid batch: walk them even if it failed later)
+  if (!c_invalid && nhot) {   // (the group kernel set the bits of any valid batch: walk them even if it failed later)
     tkey_t* __restrict__ results = A->results;
     const tkey_t* __restrict__ vals = A->vals;
-    const bool ok = ctl->status == 0;
+    const bool ok = c_status == 0;
     // Deferred hot keys (SPLIT groups, group.cu): the bits of slot j are the key's
     // requests in timestamp order (present / op bit 0 / op bit 1 bitmaps over
     // [0, n)).  Work items (slot, chunk of HOT_CHW words) are taken in order; a
@@ -731,6 +737,9 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
   __syncthreads();
   if (threadIdx.x == 0) {
     __threadfence();
+#ifdef EIRENE_FIN_FLAT
+    s_last = atomicAdd(&ctl->fin_ctr, 1u) == gridDim.x - 1;
+#else
     const uint32_t grp = blockIdx.x & 15u, gsize = (gridDim.x + 15u - grp) / 16u;   // CTAs with this residue
     bool last = false;
     if (atomicAdd(&ctl->fin_sub[grp], 1u) == gsize - 1) {   // the last of its residue class
@@ -739,6 +748,7 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
       last = atomicAdd(&ctl->fin_ctr, 1u) == ngrp - 1;
     }
     s_last = last;
+#endif
   }
   __syncthreads();
   if (!s_last) return;
