@@ -122,6 +122,7 @@ struct GraphEntry {
   cudaGraphExec_t exec = nullptr;
   cudaGraphNode_t args_node = nullptr;
   int launches = 0;                 // kernels in the graph
+  bool cond = false;                // the update kernel is a conditional node (may not run)
 };
 
 // One set of the buffers a batch's front (distribution + group: sort, combine,
@@ -147,6 +148,7 @@ struct Rec {
   uint64_t ticket = 0;
   bool used = false;
   bool timing = false;
+  bool cond = false;      // its graph's update kernel is conditional
   uint32_t n = 0;
   int launches = 0;
   cudaEvent_t done = nullptr;
@@ -164,6 +166,8 @@ struct eirene_tree {
   BatchArgs* dargs = nullptr;
   unsigned long long* phase = nullptr;   // diagnostic phase stamps (filled by -DEIRENE_PHASE_PROF builds)
   cudaStream_t cap_stream = nullptr;
+  cudaStream_t cap_stream2 = nullptr;   // captures the body of the update kernel's conditional node
+  bool use_cond = std::getenv("EIRENE_NO_COND") == nullptr;   // A/B: always launch the update kernel
   GraphEntry graphs[MAX_GRAPHS];
   Lane lanes[2];
   int nlanes = 1;
@@ -359,6 +363,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   AL(h->phase, 2 * PROF_CTAS * PROF_PHASES);
   AL(h->ctl_ring, RING);
   if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream, cudaStreamNonBlocking);
+  if (e == cudaSuccess) e = cudaStreamCreateWithFlags(&h->cap_stream2, cudaStreamNonBlocking);
   // one contiguous region zeroed before every batch: BatchCtl | ghist | comb/part status
   {
     size_t off = 0;
@@ -516,6 +521,7 @@ int eirene_destroy(eirene_handle h) {
     if (g.graph) cudaGraphDestroy(g.graph);
   }
   if (h->cap_stream) cudaStreamDestroy(h->cap_stream);
+  if (h->cap_stream2) cudaStreamDestroy(h->cap_stream2);
   for (auto& L : h->lanes) {
     for (GraphEntry* ge : {L.fg, L.bg})
       for (int i = 0; i < MAX_GRAPHS; ++i) {
@@ -657,6 +663,8 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
     std::fprintf(stderr, "[eirene] batch %u stage %s done: %s\n", seq, name, cudaGetErrorString(e));
   };
   auto rec = [&](int i, cudaStream_t s) { cudaEventRecord(r.st[i], s); };
+  bool cond_captured = false;   // set by `back` when it captured a conditional update node
+  bool* cond_out = &cond_captured;
   BatchCtl* ctl_slot = h->ctl_ring + tk % RING;
   const bool large = !bsort_fused(nk, h->num_sms);   // two-kernel bucket sort with 16384 bins (bsort.cu)
   // The front of a batch: a tiny node publishing its pointers to the lane's
@@ -688,17 +696,58 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
   // The back: query (Alg.1:15-21; it checks the pool headroom first), range,
   // update (Alg.1:23-46), RESULT_CAL (Alg.1:6) -- the kernels that read or
   // change the tree.
-  auto back = [&](Lane& L, cudaStream_t s, int* nl) -> cudaError_t {
+  // capture: the update kernel becomes the body of a conditional graph node
+  // that the query kernel's last CTA switches on only when there is anything
+  // left for it (structural writes, long segments, deferred hot keys); else
+  // the query kernel ends the batch (query_end, query.cu).  Not for range
+  // batches (their range kernel sits between the two).
+  auto back = [&](Lane& L, cudaStream_t s, int* nl, bool capture) -> cudaError_t {
     const uint32_t* spay = L.bs.pB;
+    const bool cond_mode = capture && !range && h->use_cond;
+    cudaGraphConditionalHandle cond = 0;
+    cudaGraph_t cg = nullptr;
+    if (cond_mode) {
+      cudaStreamCaptureStatus cs;
+      cudaError_t e = cudaStreamGetCaptureInfo(s, &cs, nullptr, &cg, nullptr, nullptr);
+      if (e == cudaSuccess) e = cudaGraphConditionalHandleCreate(&cond, cg, 0, cudaGraphCondAssignDefault);
+      if (e != cudaSuccess) return e;
+    }
     if (timing) rec(2, s);
-    launch_query(nk, L.cb, spay, L.dargs, h->t, L.ctl, h->num_sms, h->cfg.flags, h->cfg.iter_rgs, s, nl);
+    launch_query(nk, L.cb, spay, L.dargs, h->t, L.ctl, h->num_sms, h->cfg.flags, h->cfg.iter_rgs, cond,
+                 cond_mode ? 1 : 0, s, nl);
     if (range) launch_range(nk, L.cb, spay, L.bs.kB, L.dargs, h->t, L.ctl, h->num_sms, s, nl);
     stage("query", s);
     if (timing) rec(3, s);
     const ResultArgs ra{spay,          L.bs.kB,  L.cb.pinfo,       L.cb.istart,    L.cb.longseg,
                         L.cb.old,      L.dargs,  L.ctl,            h->t.hdr,       L.cb.hot_bits,
                         L.cb.hot_words, L.cb.hot_seg, h->hot_lb,   h->hot_chunks};
-    launch_update(nk, L.cb, h->t, L.ctl, h->up, ra, h->num_sms, s, nl);
+    cudaStream_t us = s;
+    if (cond_mode) {
+      cudaStreamCaptureStatus cs;
+      const cudaGraphNode_t* deps = nullptr;
+      size_t nd = 0;
+      cudaError_t e = cudaStreamGetCaptureInfo(s, &cs, nullptr, &cg, &deps, &nd);
+      cudaGraphNodeParams cp{};
+      cp.type = cudaGraphNodeTypeConditional;
+      cp.conditional.handle = cond;
+      cp.conditional.type = cudaGraphCondTypeIf;
+      cp.conditional.size = 1;
+      cudaGraphNode_t cn = nullptr;
+      if (e == cudaSuccess) e = cudaGraphAddNode(&cn, cg, deps, nd, &cp);
+      if (e == cudaSuccess) e = cudaStreamUpdateCaptureDependencies(s, &cn, 1, cudaStreamSetCaptureDependencies);
+      if (e == cudaSuccess)
+        e = cudaStreamBeginCaptureToGraph(h->cap_stream2, cp.conditional.phGraph_out[0], nullptr, nullptr, 0,
+                                          cudaStreamCaptureModeRelaxed);
+      if (e != cudaSuccess) return e;
+      us = h->cap_stream2;
+    }
+    launch_update(nk, L.cb, h->t, L.ctl, h->up, ra, h->num_sms, us, nl);
+    if (cond_mode) {
+      cudaGraph_t body = nullptr;
+      cudaError_t e = cudaStreamEndCapture(h->cap_stream2, &body);
+      if (e != cudaSuccess) return e;
+      *cond_out = true;
+    }
     stage("update", s);
     if (timing) rec(4, s);
     if (dbg) launch_result(L.ctl, 1, s);
@@ -738,8 +787,10 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
                            [&](cudaStream_t s, cudaGraphNode_t* an, int* nl) { return front(L, s, an, nl); }, &gf);
         if (rc != EIRENE_OK) return rc;
         rc = get_graph(h, L.bg, L.next_bg, nk, range, false,
-                       [&](cudaStream_t s, cudaGraphNode_t*, int* nl) { return back(L, s, nl); }, &gb);
+                       [&](cudaStream_t s, cudaGraphNode_t*, int* nl) { return back(L, s, nl, true); }, &gb);
         if (rc != EIRENE_OK) return rc;
+        if (cond_captured) gb->cond = true;
+        cond_captured = false;
       }
       (void)fq;
       return EIRENE_OK;
@@ -750,8 +801,9 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
                        [&](cudaStream_t s, cudaGraphNode_t* an, int* nl) { return front(L, s, an, nl); }, &gf);
     if (rc != EIRENE_OK) return rc;
     rc = get_graph(h, L.bg, L.next_bg, nk, range, false,
-                   [&](cudaStream_t s, cudaGraphNode_t*, int* nl) { return back(L, s, nl); }, &gb);
+                   [&](cudaStream_t s, cudaGraphNode_t*, int* nl) { return back(L, s, nl, true); }, &gb);
     if (rc != EIRENE_OK) return rc;
+    if (cond_captured) gb->cond = true;
     if (L.used) CK(cudaStreamWaitEvent(st, L.back_done, 0));   // the back of batch b-2 released this lane
     rc = set_args_params(gf, L);
     if (rc != EIRENE_OK) return rc;
@@ -762,13 +814,14 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
     CK(cudaEventRecord(L.back_done, h->back_stream));
     L.used = true;
     launches = gf->launches + gb->launches;
+    r.cond = gb->cond;
     end = h->back_stream;
   } else {
     Lane& L = h->lanes[0];
     if (h->nlanes == 2 && h->last_done) CK(cudaStreamWaitEvent(st, h->last_done, 0));   // pipelined batches first
     auto whole = [&](cudaStream_t s, cudaGraphNode_t* an, int* nl) -> cudaError_t {
       cudaError_t e = front(L, s, an, nl);
-      return e != cudaSuccess ? e : back(L, s, nl);
+      return e != cudaSuccess ? e : back(L, s, nl, an != nullptr);
     };
     if (dbg || timing || !h->use_graphs) {   // per-stage events: direct launches
       CK(whole(st, nullptr, &launches));
@@ -777,11 +830,13 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
       GraphEntry* g = nullptr;
       int rc = get_graph(h, h->graphs, h->next_graph, nk, range, true, whole, &g);
       if (rc != EIRENE_OK) return rc;
+      if (cond_captured) g->cond = true;
       if (prepare_only) return EIRENE_OK;   // graph captured and instantiated, nothing launched
       rc = set_args_params(g, L);
       if (rc != EIRENE_OK) return rc;
       CK(cudaGraphLaunch(g->exec, st));
       launches = g->launches;
+      r.cond = g->cond;
     }
   }
   CK(cudaEventRecord(r.done, end));
@@ -894,7 +949,8 @@ int eirene_results(eirene_handle h, uint64_t ticket, eirene_batch_stats* stats) 
     stats->new_leaves = c.new_leaves;
     stats->new_inner = c.new_inner;
     stats->height = c.height;
-    stats->launches = (uint32_t)r.launches;
+    // (a conditional update kernel that did not run is not counted)
+    stats->launches = (uint32_t)r.launches - ((r.cond && !c.upd_ran) ? 1u : 0u);
     stats->ranges = c.nrange;
     stats->artificial = c.nart;
     stats->trav_steps = c.trav_steps;

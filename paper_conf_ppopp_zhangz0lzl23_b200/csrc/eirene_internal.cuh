@@ -81,6 +81,8 @@ struct BatchCtl {
                           // issued write was a value overwrite, applied in place by the query kernel
   uint32_t fin_ctr;       // update kernel's result phase: residue classes finished (the last publishes the BatchCtl)
   uint32_t fin_sub[16];   // ... CTAs finished per residue class blockIdx % 16
+  uint32_t qfin_ctr, qfin_sub[16];   // the same for the query kernel (graph mode: it may end the batch)
+  uint32_t upd_ran;       // the update kernel ran (its conditional graph node was switched on)
   unsigned long long t_begin, t_end;   // %globaltimer (ns) at the batch's first / last kernel
   uint32_t ubar;          // grid barrier of the update kernel's level-synchronous phases
   uint32_t uchunk;        // update kernel: next 32-write chunk (dynamic, level-synchronous mode)
@@ -505,8 +507,11 @@ constexpr int GROUP_STATUS_WORDS = NBINS_MAX;   // >= bsort_groups(n) for every 
 // bucket finish (sort in smem) + combine + partition, one CTA per bucket (group.cu)
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
                   int num_sms, cudaStream_t st, int* launches);
+// cond / use_cond: graph mode -- the query kernel's last CTA sets the
+// conditional node around the update kernel (or ends the batch itself)
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
-                  int num_sms, uint32_t flags, uint32_t iter_rgs, cudaStream_t st, int* launches);
+                  int num_sms, uint32_t flags, uint32_t iter_rgs, cudaGraphConditionalHandle cond, int use_cond,
+                  cudaStream_t st, int* launches);
 
 struct UpdParams {
   uint32_t threshold;
@@ -557,6 +562,55 @@ void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t
 // segment.  The segments longer than SHORT_SEG (hot keys) are queued instead
 // and finished here, work items of RCHUNK positions spread over the CTAs, so a
 // 56K-request Zipf key does not serialise one thread.
+// True in exactly one CTA of the grid: the last to arrive (CTA-uniform; call
+// with every thread).  Two levels -- 16 counters by blockIdx % 16, then one --
+// so no address takes more than ~gridDim / 16 same-address atomics.
+__device__ __forceinline__ bool last_cta(uint32_t* sub16, uint32_t* top) {
+  __shared__ uint32_t s_last;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const uint32_t grp = blockIdx.x & 15u, gsize = (gridDim.x + 15u - grp) / 16u;   // CTAs with this residue
+    bool last = false;
+    if (atomicAdd(&sub16[grp], 1u) == gsize - 1) {   // the last of its residue class
+      __threadfence();
+      last = atomicAdd(top, 1u) == min(16u, gridDim.x) - 1;
+    }
+    s_last = last;
+  }
+  __syncthreads();
+  const bool last = s_last;
+  if (last) __threadfence();
+  return last;
+}
+
+// End of a batch, by the last CTA of its last kernel: the device end time, the
+// final status and height, and the whole BatchCtl copied to the batch's ring
+// slot (one word per thread).
+__device__ __forceinline__ void publish_batch(BatchCtl* ctl, const BatchArgs* A, const TreeHdr* hdr) {
+  if (threadIdx.x == 0) {
+    if (ld_cg(&ctl->invalid)) ctl->status = EIRENE_EINVAL;
+    ctl->height = (uint32_t)(hdr->root_word >> 32);
+    ctl->t_begin = A->t0;
+    ctl->t_end = gtime_ns();
+  }
+  __syncthreads();
+  static_assert(sizeof(BatchCtl) % 8 == 0, "BatchCtl is copied as u64 words");
+  const unsigned long long* src = reinterpret_cast<const unsigned long long*>(ctl);
+  unsigned long long* dst = reinterpret_cast<unsigned long long*>(A->ctl_out);
+  for (uint32_t i = threadIdx.x; i < sizeof(BatchCtl) / 8; i += blockDim.x) dst[i] = __ldcg(src + i);
+}
+
+// Whether the update kernel has anything to do once the query kernel has run:
+// structural writes, long segments, or deferred hot-key bitmaps (whose bits
+// must be walked -- and cleared -- even when the batch failed after the group
+// kernel).  Read by the query kernel's last CTA (graph conditional node).
+__device__ __forceinline__ bool update_needed(const BatchCtl* ctl, const BatchArgs* A) {
+  const uint32_t inv = ld_cg(&ctl->invalid), st = ld_cg(reinterpret_cast<const uint32_t*>(&ctl->status));
+  const bool hot = A->rkeys == nullptr && ld_cg(&ctl->hot_ctr) > 0;
+  return !inv && (hot || (st == 0 && (ld_cg(&ctl->nins) | ld_cg(&ctl->ndelp) | ld_cg(&ctl->nlong)) != 0));
+}
+
 struct ResultArgs {
   const uint32_t* spay;
   const uint64_t* kB;
@@ -590,8 +644,9 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
   __shared__ uint32_t s_hseg[HOT_SLOTS];
   __shared__ uint32_t s_item, s_red[32];
   // the batch's scalars, loaded together (independent loads: one round trip)
-  const uint32_t c_invalid = ld_cg(&ctl->invalid), c_status = ld_cg(reinterpret_cast<const uint32_t*>(&ctl->status));
-  const uint32_t c_nlong = ld_cg(&ctl->nlong), c_hot = ld_cg(&ctl->hot_ctr);
+  // (plain loads: ctl was read at the kernel's start, written only by earlier kernels)
+  const uint32_t c_invalid = ctl->invalid, c_status = (uint32_t)ctl->status;
+  const uint32_t c_nlong = ctl->nlong, c_hot = ctl->hot_ctr;
   const bool c_range = A->rkeys != nullptr;
   const uint32_t njobs = min(c_hot, (uint32_t)HOT_SLOTS);
   // (a deferred hot key's segment is walked below, not through its positions)
@@ -728,44 +783,8 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
       }
     }
   }
-  // End of the batch (the last kernel): the last CTA to finish stamps the
-  // device end time, sets the final status and height and publishes the whole
-  // BatchCtl to the batch's ring slot (one word per thread).
-  // two-level arrival count (16 counters, then one): ~gridDim/16 same-address
-  // atomics per counter instead of gridDim on one
-  __shared__ uint32_t s_last;
-  __syncthreads();
-  if (threadIdx.x == 0) {
-    __threadfence();
-#ifdef EIRENE_FIN_FLAT
-    s_last = atomicAdd(&ctl->fin_ctr, 1u) == gridDim.x - 1;
-#else
-    const uint32_t grp = blockIdx.x & 15u, gsize = (gridDim.x + 15u - grp) / 16u;   // CTAs with this residue
-    bool last = false;
-    if (atomicAdd(&ctl->fin_sub[grp], 1u) == gsize - 1) {   // the last of its residue class
-      __threadfence();
-      const uint32_t ngrp = min(16u, gridDim.x);
-      last = atomicAdd(&ctl->fin_ctr, 1u) == ngrp - 1;
-    }
-    s_last = last;
-#endif
-  }
-  __syncthreads();
-  if (!s_last) return;
-  __threadfence();
-  if (threadIdx.x == 0) {
-    if (ld_cg(&ctl->invalid)) ctl->status = EIRENE_EINVAL;
-    ctl->height = (uint32_t)(hdr->root_word >> 32);
-    ctl->t_begin = A->t0;
-    ctl->t_end = gtime_ns();
-  }
-  __syncthreads();
-  {
-    static_assert(sizeof(BatchCtl) % 8 == 0, "BatchCtl is copied as u64 words");
-    const unsigned long long* src = reinterpret_cast<const unsigned long long*>(ctl);
-    unsigned long long* dst = reinterpret_cast<unsigned long long*>(A->ctl_out);
-    for (uint32_t i = threadIdx.x; i < sizeof(BatchCtl) / 8; i += blockDim.x) dst[i] = __ldcg(src + i);
-  }
+  // End of the batch (the last kernel): the last CTA to finish publishes it
+  if (last_cta(ctl->fin_sub, &ctl->fin_ctr)) publish_batch(ctl, A, hdr);
 }
 
 

@@ -156,7 +156,7 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
   }
 }
 
-__global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restrict__ qkey,
+__device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
@@ -169,8 +169,6 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
                                                         const uint32_t* __restrict__ istart,
                                                         uint32_t* __restrict__ longseg, const BatchArgs* __restrict__ A,
                                                         Tree t, BatchCtl* __restrict__ ctl) {
-  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
-  pdl_trigger();
   if (ctl->invalid || ctl->status != 0) return;
   tkey_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw, total = nq + nw;
@@ -204,6 +202,42 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
   }
 }
 
+// End of the query kernel in graph mode (cond != 0): its last CTA decides
+// whether the batch's update kernel -- a conditional graph node -- runs at all
+// (structural writes, long segments or deferred hot keys left); if not, it ends
+// the batch itself (publish_batch), so a read-mostly batch is four kernels.
+__device__ __forceinline__ void query_end(BatchCtl* ctl, const BatchArgs* A, const TreeHdr* hdr,
+                                          cudaGraphConditionalHandle cond) {
+  if (!last_cta(ctl->qfin_sub, &ctl->qfin_ctr)) return;
+  __shared__ uint32_t s_need;
+  if (threadIdx.x == 0) {
+    s_need = update_needed(ctl, A) ? 1u : 0u;
+    if (s_need) cudaGraphSetConditional(cond, 1u);
+  }
+  __syncthreads();
+  if (!s_need) publish_batch(ctl, A, hdr);
+}
+
+__global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restrict__ qkey,
+                                                        const uint32_t* __restrict__ qseg,
+                                                        const uint64_t* __restrict__ wkey,
+                                                        const uint32_t* __restrict__ wseg,
+                                                        const uint8_t* __restrict__ wop,
+                                                        const uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
+                                                        uint8_t* __restrict__ wslot, uint32_t* __restrict__ wparent,
+                                                        uint64_t* __restrict__ old,
+                                                        const uint32_t* __restrict__ spay,
+                                                        const uint32_t* __restrict__ pinfo,
+                                                        const uint32_t* __restrict__ istart,
+                                                        uint32_t* __restrict__ longseg, const BatchArgs* __restrict__ A,
+                                                        Tree t, BatchCtl* __restrict__ ctl,
+                                                        cudaGraphConditionalHandle cond, int use_cond) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
+  query_body(qkey, qseg, wkey, wseg, wop, wval, wleaf, wslot, wparent, old, spay, pinfo, istart, longseg, A, t, ctl);
+  if (use_cond) query_end(ctl, A, t.hdr, cond);
+}
+
 // Locality-aware warp reorganisation the paper's way (§5, P:1380-1512,
 // Fig.6): an ablation of the default traversal above (EIRENE_F_ITERWARP).
 // Request groups (RGs) are 32 consecutive issued requests of the key-sorted
@@ -222,14 +256,12 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
 // and follows B-link `next` pointers until k < hi, so RF only chooses the
 // cheaper way.  With EIRENE_F_STATS the kernel counts vertical / horizontal
 // RGs and traversal steps (Fig.10).
-__global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* __restrict__ qkey,
+__device__ __forceinline__ void query_iterwarp_body(const uint64_t* __restrict__ qkey,
                                                                  const uint64_t* __restrict__ wkey,
                                                                  uint32_t* __restrict__ wparent, QueryIO io,
                                                                  const BatchArgs* __restrict__ A, Tree t,
                                                                  BatchCtl* __restrict__ ctl, uint32_t iter_rgs,
                                                                  uint32_t stats) {
-  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
-  pdl_trigger();
   if (ctl->invalid || ctl->status != 0) return;
   tkey_t* __restrict__ results = A->results;
   const uint32_t nq = ctl->nq, nw = ctl->nw;
@@ -303,6 +335,19 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
     atomicAdd(&ctl->rg_vertical, nvert);
     atomicAdd(&ctl->rg_horizontal, nhor);
   }
+}
+
+__global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* __restrict__ qkey,
+                                                                 const uint64_t* __restrict__ wkey,
+                                                                 uint32_t* __restrict__ wparent, QueryIO io,
+                                                                 const BatchArgs* __restrict__ A, Tree t,
+                                                                 BatchCtl* __restrict__ ctl, uint32_t iter_rgs,
+                                                                 uint32_t stats, cudaGraphConditionalHandle cond,
+                                                                 int use_cond) {
+  pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
+  pdl_trigger();
+  query_iterwarp_body(qkey, wkey, wparent, io, A, t, ctl, iter_rgs, stats);
+  if (use_cond) query_end(ctl, A, t.hdr, cond);
 }
 
 // Diagnostics (EIRENE_DEBUG_SYNC / EIRENE_UPDATE_PROF only): printf lives in
@@ -515,7 +560,8 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
 }  // namespace
 
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
-                  int num_sms, uint32_t flags, uint32_t iter_rgs, cudaStream_t st, int* launches) {
+                  int num_sms, uint32_t flags, uint32_t iter_rgs, cudaGraphConditionalHandle cond, int use_cond,
+                  cudaStream_t st, int* launches) {
   // one resident wave: 8 CTAs of 256 threads per SM at <= 32 registers
   int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
   if (blocks < 1) blocks = 1;
@@ -525,10 +571,10 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
     launch_k(query_iterwarp_kernel, dim3(iblocks < 1 ? 1 : iblocks), dim3(256), 0, st, true, false, 
         c.qkey, c.wkey, c.wparent,
         QueryIO{c.qseg, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
-        A, t, ctl, iter_rgs, (flags & EIRENE_F_STATS) ? 1u : 0u);
+        A, t, ctl, iter_rgs, (flags & EIRENE_F_STATS) ? 1u : 0u, cond, use_cond);
   } else {
     launch_k(query_kernel, dim3(blocks), dim3(256), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.wparent, c.old,
-                                         spay, c.pinfo, c.istart, c.longseg, A, t, ctl);
+                                         spay, c.pinfo, c.istart, c.longseg, A, t, ctl, cond, use_cond);
   }
   ++*launches;
 }

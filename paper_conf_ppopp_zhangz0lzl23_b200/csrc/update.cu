@@ -1062,6 +1062,7 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C, ResultArgs
   // a present key: all of them were applied in place by the query kernel's
   // locate (query.cu, retire), nothing structural is left
   const bool skip = ctl->invalid || ctl->status != 0 || (ctl->nins == 0 && ctl->ndelp == 0);
+  if (blockIdx.x == 0 && threadIdx.x == 0) C.ctl->upd_ran = 1;
   if (!skip) update_body(C);
   result_phase(R);
 }
