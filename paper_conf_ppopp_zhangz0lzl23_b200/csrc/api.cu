@@ -167,7 +167,9 @@ struct eirene_tree {
   unsigned long long* phase = nullptr;   // diagnostic phase stamps (filled by -DEIRENE_PHASE_PROF builds)
   cudaStream_t cap_stream = nullptr;
   cudaStream_t cap_stream2 = nullptr;   // captures the body of the update kernel's conditional node
-  bool use_cond = std::getenv("EIRENE_NO_COND") == nullptr;   // A/B: always launch the update kernel
+  // EIRENE_COND=1: the update kernel as a conditional graph node (measured r2: device batch time -2 us but the
+  // gap between graph launches +8 us on cfg2 -- off by default)
+  bool use_cond = std::getenv("EIRENE_COND") != nullptr;
   GraphEntry graphs[MAX_GRAPHS];
   Lane lanes[2];
   int nlanes = 1;

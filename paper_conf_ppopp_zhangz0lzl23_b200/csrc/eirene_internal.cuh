@@ -41,7 +41,10 @@ constexpr uint32_t DEFER_BIT = 0x40000000u;   // pinfo (hot-key segments): that 
                                               // result phase from the nearest write's payload in kB
 constexpr uint32_t SEG_MASK = 0x3FFFFFFFu;
 constexpr uint32_t Q_SINGLE = 0x80000000u;    // qseg entry of a one-request query segment: Q_SINGLE | its timestamp
-constexpr uint32_t RCHUNK = 512;              // result phase work item: positions of one long segment
+#ifndef EIRENE_RCHUNK
+#define EIRENE_RCHUNK 512
+#endif
+constexpr uint32_t RCHUNK = EIRENE_RCHUNK;    // result phase work item: positions of one long segment
                                               // (4 per thread of the update kernel's 128-thread CTAs)
 constexpr uint32_t FULL = 0xFFFFFFFFu;
 
@@ -650,7 +653,13 @@ __device__ __forceinline__ void result_phase(const ResultArgs& R) {
   const bool c_range = A->rkeys != nullptr;
   const uint32_t njobs = min(c_hot, (uint32_t)HOT_SLOTS);
   // (a deferred hot key's segment is walked below, not through its positions)
+#ifdef EIRENE_NO_HOTDEFER
+  const uint32_t nhot = 0;
+  (void)c_range;
+  (void)njobs;
+#else
   const uint32_t nhot = c_range ? 0u : njobs;
+#endif
   if (nhot) {   // (uniform)
     for (uint32_t j = threadIdx.x; j < nhot; j += blockDim.x) s_hseg[j] = ld_cg(R.hot_seg + j);
     __syncthreads();

@@ -1228,7 +1228,11 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   // SPLIT groups of a batch without range queries hand the hot key's bitmap to
   // the result phase (multi-CTA); range batches need the segment's positions
   // (artificial queries binary-search them) and walk it here (hot_pass2)
+#ifdef EIRENE_NO_HOTDEFER
+  const bool deferred = false;
+#else
   const bool deferred = g.A->rkeys == nullptr;
+#endif
   uint32_t sp_o = 0, sp_h = 0, sp_lo = 0;
   if (!small) {
     const int where = l2_sort(g.kA + base, g.pA + base, g.kB + base, g.pB + base, cnt, g.tsbits, S, g.hot_bits,
