@@ -334,6 +334,7 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   h->cb.hot_words = (uint32_t)(((nb + 127) / 128) * 4);   // multiple of 4 (uint4 access)
   AL(h->cb.hot_bits, (size_t)HOT_SLOTS * 3 * h->cb.hot_words);
   AL(h->cb.hot_seg, HOT_SLOTS);
+  AL(h->cb.grec, (size_t)NBINS_MAX * 4);   // GroupRec per group (the two-phase group stage)
   h->hot_chunks = (h->cb.hot_words + HOT_CHW - 1) / HOT_CHW;
   AL(h->hot_lb, (size_t)HOT_SLOTS * h->hot_chunks);   // epoch-tagged: never needs zeroing between batches
   AL(h->up.entA_key, nb + 64);
@@ -691,7 +692,9 @@ static int submit_impl(eirene_handle h, const uint8_t* ops, const tkey_t* keys, 
     launch_bucket_sort(L.dargs, nk, h->cfg.key_lo, bin_hi, large ? L.bsL : L.bs, L.ctl, h->num_sms, s, nl);
     stage("sort", s);
     if (timing) rec(1, s);
-    launch_group(L.dargs, nk, large ? L.bsL : L.bs, large ? L.cbL : L.cb, h->t, L.ctl, h->num_sms, s, nl);
+    // (range batches keep the one-kernel stage: their hot keys are walked by the group kernel)
+    launch_group(L.dargs, nk, large ? L.bsL : L.bs, large ? L.cbL : L.cb, h->t, L.ctl, h->num_sms,
+                 !range && group_two_phase(nk, h->num_sms), s, nl);
     stage("group", s);
     return cudaGetLastError();
   };

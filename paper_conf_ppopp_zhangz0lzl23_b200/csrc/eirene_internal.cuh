@@ -161,7 +161,7 @@ constexpr int PROF_CTAS = 512, PROF_PHASES = 8;
 #endif
 
 // tile counters
-enum { TC_SORT0 = 0, TC_GROUP = 8, TC_ROUTE = 10, TC_SCAN = 11, TC_HIST = 12 };
+enum { TC_SORT0 = 0, TC_GROUP = 8, TC_GROUP2 = 9, TC_ROUTE = 10, TC_SCAN = 11, TC_HIST = 12 };
 
 struct Tree {
   tkey_t* lkeys;     // leaf L: keys at lkeys[L * LSTRIDE + s]
@@ -499,6 +499,7 @@ struct CombBufs {
                               // op bit 1 (all zero between batches)
   uint32_t hot_words;         // >= max_batch / 32, a multiple of 4
   uint32_t* hot_seg;          // [HOT_SLOTS] segment of each hot key whose bitmap the result phase walks
+  uint4* grec;                // [NBINS_MAX][3] per-group records of the two-phase group stage (multi-wave batches)
 };
 constexpr int HOT_SLOTS = 64;
 #ifndef EIRENE_SHORT_SEG
@@ -508,8 +509,12 @@ constexpr uint32_t SHORT_SEG = EIRENE_SHORT_SEG;
 constexpr int GROUP_STATUS_WORDS = NBINS_MAX;   // >= bsort_groups(n) for every n
 
 // bucket finish (sort in smem) + combine + partition, one CTA per bucket (group.cu)
+// two_phase: a batch of more groups than are co-resident (several waves) and no
+// range queries runs the group stage as two kernels -- sort + totals, then
+// look-back + emit -- so that no CTA waits for a later wave's slow group
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
-                  int num_sms, cudaStream_t st, int* launches);
+                  int num_sms, bool two_phase, cudaStream_t st, int* launches);
+bool group_two_phase(uint32_t n, int num_sms);   // the batch has more groups than one wave
 // cond / use_cond: graph mode -- the query kernel's last CTA sets the
 // conditional node around the update kernel (or ends the batch itself)
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,

@@ -869,6 +869,8 @@ struct GroupArgs {
   uint32_t hot_words;
   uint32_t* hot_seg;            // [HOT_SLOTS] segment of each deferred hot key (result phase)
   int prof;                     // EIRENE_GROUP_PROF: print the phases of slow groups (diagnostic)
+  int phase;                    // 0: one kernel; 1: phase 1 of the two-phase group stage
+  uint4* grec;                  // [nb] GroupRec (two-phase)
   Tree t;
   BatchCtl* ctl;
 };
@@ -1195,6 +1197,188 @@ __device__ void hot_pass2(const GroupArgs& g, uint32_t* bits, const HotCarry& c,
   }
 }
 
+// Per-group record from phase 1 to phase 2 of the two-phase group stage.
+struct alignas(16) GroupRec {
+  uint64_t hk;          // SPLIT: the hot key
+  uint32_t where;       // 0: sorted in kA / pA, 1: in kB / pB, 2: SPLIT (the rest sorted in kB / pB [0, sp_o))
+  uint32_t c_nh, c_nw;  // the group's key segments and issued writes (its look-back aggregate)
+  uint32_t sp_o, sp_h, sp_lo, a_nh, a_nw, hot_w, hot_last, hot_slot;
+};
+static_assert(sizeof(GroupRec) == 4 * sizeof(uint4), "grec holds 4 uint4 per group");
+
+// Round [r0, r1) of a group sorted in L2 (K, P), copied to shared memory.
+__device__ GView load_round(const uint64_t* K, const uint32_t* P, uint32_t r0, uint32_t r1, GSmem& S) {
+  const int tid = threadIdx.x;
+  __syncthreads();
+  for (uint32_t i0 = r0 + tid; i0 < r1; i0 += 8 * G_THREADS) {   // 8 loads in flight per thread
+    uint64_t kk[8];
+    uint32_t pp[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const uint32_t i = i0 + u * G_THREADS;
+      kk[u] = i < r1 ? K[i] : 0;
+      pp[u] = i < r1 ? P[i] : 0;
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      const uint32_t i = i0 + u * G_THREADS;
+      if (i < r1) {
+        S.k[i - r0] = kk[u];
+        S.p[i - r0] = pp[u];
+      }
+    }
+  }
+  __syncthreads();
+  return GView{K, P, S.k, S.p, r0, r1};
+}
+
+// Decoupled look-back over the buckets (ticket order) on (heads << 31 | writes)
+// -> S.seg0, S.w0 (the last bucket also writes the batch totals).
+__device__ void group_lookback(const GroupArgs& g, uint32_t b, uint32_t c_nh, uint32_t c_nw, GSmem& S) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  BatchCtl* ctl = g.ctl;
+  if (warp == 0) {
+    const unsigned long long tot = ((unsigned long long)c_nh << 31) | c_nw;
+    unsigned long long* my = g.status + b;
+    unsigned long long excl = 0;
+    if (b == 0) {
+      if (lane == 0) st_relaxed64(my, F_INC | tot);
+    } else {
+      if (lane == 0) st_relaxed64(my, F_AGG | tot);
+      SpinGuard sg;
+      int32_t pt = (int32_t)b - 1;
+      for (;;) {
+        const int32_t idx = pt - lane;
+        const unsigned long long w = idx >= 0 ? ld_relaxed64(g.status + idx) : F_INC;
+        const uint32_t fl = (uint32_t)(w >> 62);
+        const uint32_t inc = __ballot_sync(FULL, fl == 2);
+        const uint32_t need = inc ? ((2u << (__ffs(inc) - 1)) - 1u) : FULL;
+        if (__ballot_sync(FULL, fl == 0) & need) {
+          // a predecessor has not published: back off (a waiting group's spin
+          // would otherwise keep the L2 busy under the slow groups it waits for)
+          __nanosleep(256);
+          if (sg.stuck(ctl)) break;
+          continue;
+        }
+        unsigned long long a = ((need >> lane) & 1u) ? (w & F_VAL) : 0ull;
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(FULL, a, o);
+        excl += a;
+        if (inc) break;
+        pt -= 32;
+      }
+      if (lane == 0) st_relaxed64(my, F_INC | (excl + tot));
+    }
+    if (lane == 0) {
+      const uint32_t seg0 = (uint32_t)(excl >> 31), w0 = (uint32_t)(excl & ((1u << 31) - 1));
+      S.seg0 = seg0;
+      S.w0 = w0;
+      if (b + 1 == g.nb) {   // last bucket: batch totals (the pool headroom is checked by the query kernel)
+        const uint32_t nseg = seg0 + c_nh, nw = w0 + c_nw;
+        ctl->nseg = nseg;
+        ctl->nw = nw;
+        ctl->nq = nseg - nw;
+        g.istart[nseg] = g.gstart[g.nb];   // point requests (range queries are not sorted)
+      }
+    }
+  }
+  __syncthreads();
+}
+
+// Sweep 2 of a SPLIT group: the rest (sorted in S.k / S.p [0, sp_o)) around the
+// hot key's segment (sp_h positions after the sp_lo smaller ones).
+__device__ void emit_split(const GroupArgs& g, GSmem& S, uint32_t base, uint32_t sp_o, uint32_t sp_lo, uint32_t sp_h,
+                           uint32_t hot_w, uint32_t hot_last, uint32_t a_nh, uint32_t a_nw, bool deferred,
+                           const HotCarry& hc) {
+  const int tid = threadIdx.x;
+  const GView V{S.k, S.p, S.k, S.p, 0, sp_o};
+  if (sp_o) {
+    round_scan(V, sp_o, 0, sp_o, 0, 0, 0, S);
+    round_emit(g, V, sp_o, base, 0, sp_o, true, S, sp_lo, sp_h, hot_w);
+  }
+  __syncthreads();
+  const uint32_t sH = S.seg0 + a_nh, wH = S.w0 + a_nw, pos0 = base + sp_lo;
+  if ((g.prof & 1) && tid == 0) S.prof_t[0] = gtime_ns();
+  if (!deferred) hot_pass2(g, S.hot_bits, hc, sH, pos0);
+  if ((g.prof & 1) && tid == 0) S.prof_t[1] = gtime_ns();
+  if (tid == 0) {
+    const uint64_t hk = S.hk;
+    g.istart[sH] = pos0;
+    // deferred: the segment's positions (pinfo, sorted payloads) are not
+    // written; every result of it comes from the result phase's walk of the
+    // bitmap slot, spread over many CTAs (result_phase, eirene_internal.cuh)
+    if (deferred) g.hot_seg[S.hot_slot] = sH;
+    if (hot_w) {   // issue rule: the segment's last write
+      const uint32_t opw = hot_last & 3;
+      g.wkey[wH] = hk;
+      g.wop[wH] = (uint8_t)opw;
+      g.wval[wH] = (opw == OP_DELETE) ? KEY_MAX : g.A->vals[hot_last >> 2];
+      g.wseg[wH] = sH;
+    } else {       // all-query segment: its last query
+      g.qkey[sH - wH] = hk;
+      g.qseg[sH - wH] = sH;
+    }
+  }
+}
+
+// Sweep 2 of a group sorted in L2 (K, P), walked in rounds of G_CAP positions.
+__device__ void emit_rounds(const GroupArgs& g, GSmem& S, const uint64_t* K, const uint32_t* P, uint32_t cnt,
+                            uint32_t base) {
+  const bool write_spay = P != g.pB + base;
+  uint32_t c_nh = 0, c_lw = 0, c_nw = 0;
+  for (uint32_t r0 = 0; r0 < cnt; r0 += G_CAP) {
+    const uint32_t r1 = min(cnt, r0 + (uint32_t)G_CAP);
+    const GView V = load_round(K, P, r0, r1, S);
+    round_scan(V, cnt, r0, r1, c_nh, c_lw, c_nw, S);
+    round_emit(g, V, cnt, base, r0, r1, write_spay, S);
+    c_nh = S.r_nh;
+    c_lw = S.r_lw;
+    c_nw = S.r_nw;
+    __syncthreads();
+  }
+}
+
+// Phase 2 of the two-phase group stage: look-back on the aggregates phase 1
+// published, then the emit sweep over the group phase 1 left sorted in L2.
+__device__ void group_phase2(const GroupArgs& g, GSmem& S, uint32_t b) {
+  const int tid = threadIdx.x;
+  const GroupRec r = reinterpret_cast<const GroupRec*>(g.grec)[b];
+  const uint32_t base = g.gstart[b];
+  const uint32_t cnt = g.gstart[b + 1] - base;
+  if (r.where == 2) {
+    for (uint32_t i = tid; i < r.sp_o; i += G_THREADS) {
+      S.k[i] = __ldcg(g.kB + base + i);
+      S.p[i] = __ldcg(g.pB + base + i);
+    }
+    if (tid == 0) {
+      S.hk = r.hk;
+      S.hot_slot = r.hot_slot;
+    }
+  }
+  group_lookback(g, b, r.c_nh, r.c_nw, S);   // (ends with a barrier)
+  if (r.where == 2)
+    emit_split(g, S, base, r.sp_o, r.sp_lo, r.sp_h, r.hot_w, r.hot_last, r.a_nh, r.a_nw, true, HotCarry{});
+  else
+    emit_rounds(g, S, (r.where ? g.kB : g.kA) + base, (r.where ? g.pB : g.pA) + base, cnt, base);
+}
+
+// Phase 2 of the two-phase group stage (its own kernel: its register budget
+// stays out of group_kernel's).
+__global__ void __launch_bounds__(G_THREADS, 2) group_emit_kernel(GroupArgs g) {
+  pdl_wait();
+  pdl_trigger();
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  GSmem& S = *reinterpret_cast<GSmem*>(smem_raw);
+  if (g.ctl->invalid) return;
+  if (threadIdx.x == 0) S.ticket = atomicAdd(&g.ctl->tile_ctr[TC_GROUP2], 1u);
+  __syncthreads();
+  group_phase2(g, S, S.ticket);
+}
+
+// g.phase 0: the whole group stage in one kernel; 1: phase 1 of the two-phase
+// stage of a multi-wave batch (phase 1 never waits for another group, so a
+// slow group holds only its own SM slot; phase 2's look-back finds every
+// aggregate published).
 __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
@@ -1202,7 +1386,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   GSmem& S = *reinterpret_cast<GSmem*>(smem_raw);
   BatchCtl* ctl = g.ctl;
   if (ctl->invalid) return;
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int tid = threadIdx.x;
   if (tid == 0) S.ticket = atomicAdd(&ctl->tile_ctr[TC_GROUP], 1u);
   __syncthreads();
   const uint32_t b = S.ticket;
@@ -1251,30 +1435,6 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   }
   EIRENE_PHASE(g.A, 1, b, 1);
   const unsigned long long tp1 = g.prof ? gtime_ns() : 0;
-  // an oversized group is walked in rounds of G_CAP positions copied to smem
-  auto load_round = [&](uint32_t r0, uint32_t r1) {
-    __syncthreads();
-    for (uint32_t i0 = r0 + tid; i0 < r1; i0 += 8 * G_THREADS) {   // 8 loads in flight per thread
-      uint64_t kk[8];
-      uint32_t pp[8];
-#pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        const uint32_t i = i0 + u * G_THREADS;
-        kk[u] = i < r1 ? K[i] : 0;
-        pp[u] = i < r1 ? P[i] : 0;
-      }
-#pragma unroll
-      for (int u = 0; u < 8; ++u) {
-        const uint32_t i = i0 + u * G_THREADS;
-        if (i < r1) {
-          S.k[i - r0] = kk[u];
-          S.p[i - r0] = pp[u];
-        }
-      }
-    }
-    __syncthreads();
-    return GView{K, P, S.k, S.p, r0, r1};
-  };
   // sweep 1: bucket totals (heads, write segments)
   uint32_t c_nh = 0, c_lw = 0, c_nw = 0;
   uint32_t a_nh = 0, a_nw = 0, hot_w = 0, hot_last = 0;   // SPLIT: rest below hk; hk's issue
@@ -1306,7 +1466,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   }
   for (uint32_t r0 = 0; mode == 0 && r0 < cnt; r0 += G_CAP) {
     const uint32_t r1 = min(cnt, r0 + (uint32_t)G_CAP);
-    const GView V = small ? GView{K, P, K, P, 0, cnt} : load_round(r0, r1);
+    const GView V = small ? GView{K, P, K, P, 0, cnt} : load_round(K, P, r0, r1, S);
     round_scan(V, cnt, r0, r1, c_nh, c_lw, c_nw, S);
     c_nh = S.r_nh;
     c_lw = S.r_lw;
@@ -1314,101 +1474,46 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   }
   EIRENE_PHASE(g.A, 1, b, 2);
   const unsigned long long tp2 = g.prof ? gtime_ns() : 0;
-  // decoupled look-back over the buckets (ticket order) on (heads << 31 | writes)
-  if (warp == 0) {
-    const unsigned long long tot = ((unsigned long long)c_nh << 31) | c_nw;
-    unsigned long long* my = g.status + b;
-    unsigned long long excl = 0;
-    if (b == 0) {
-      if (lane == 0) st_relaxed64(my, F_INC | tot);
-    } else {
-      if (lane == 0) st_relaxed64(my, F_AGG | tot);
-      SpinGuard sg;
-      int32_t pt = (int32_t)b - 1;
-      for (;;) {
-        const int32_t idx = pt - lane;
-        const unsigned long long w = idx >= 0 ? ld_relaxed64(g.status + idx) : F_INC;
-        const uint32_t fl = (uint32_t)(w >> 62);
-        const uint32_t inc = __ballot_sync(FULL, fl == 2);
-        const uint32_t need = inc ? ((2u << (__ffs(inc) - 1)) - 1u) : FULL;
-        if (__ballot_sync(FULL, fl == 0) & need) {
-          // a predecessor has not published: back off (a waiting group's spin
-          // would otherwise keep the L2 busy under the slow groups it waits for)
-          __nanosleep(256);
-          if (sg.stuck(ctl)) break;
-          continue;
-        }
-        unsigned long long a = ((need >> lane) & 1u) ? (w & F_VAL) : 0ull;
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) a += __shfl_xor_sync(FULL, a, o);
-        excl += a;
-        if (inc) break;
-        pt -= 32;
-      }
-      if (lane == 0) st_relaxed64(my, F_INC | (excl + tot));
-    }
-    if (lane == 0) {
-      const uint32_t seg0 = (uint32_t)(excl >> 31), w0 = (uint32_t)(excl & ((1u << 31) - 1));
-      S.seg0 = seg0;
-      S.w0 = w0;
-      if (b + 1 == g.nb) {   // last bucket: batch totals (the pool headroom is checked by the query kernel)
-        const uint32_t nseg = seg0 + c_nh, nw = w0 + c_nw;
-        ctl->nseg = nseg;
-        ctl->nw = nw;
-        ctl->nq = nseg - nw;
-        g.istart[nseg] = g.gstart[g.nb];   // point requests (range queries are not sorted)
+  if (g.phase == 1) {
+    // phase 1 of two (batches without range queries: deferred hot keys): leave
+    // the sorted group in L2 for phase 2 and publish the aggregate -- no wait
+    const uint32_t where = mode == 2 ? 2u : (small || K == g.kB + base) ? 1u : 0u;
+    if (small || mode == 2) {
+      const uint32_t m = small ? cnt : sp_o;
+      for (uint32_t i = tid; i < m; i += G_THREADS) {
+        g.kB[base + i] = S.k[i];
+        g.pB[base + i] = S.p[i];
       }
     }
+    if (tid == 0) {
+      GroupRec r;
+      r.hk = mode == 2 ? S.hk : 0;
+      r.where = where;
+      r.c_nh = c_nh;
+      r.c_nw = c_nw;
+      r.sp_o = sp_o;
+      r.sp_h = sp_h;
+      r.sp_lo = sp_lo;
+      r.a_nh = a_nh;
+      r.a_nw = a_nw;
+      r.hot_w = hot_w;
+      r.hot_last = hot_last;
+      r.hot_slot = mode == 2 ? S.hot_slot : 0u;
+      reinterpret_cast<GroupRec*>(g.grec)[b] = r;
+      st_relaxed64(g.status + b, F_AGG | (((unsigned long long)c_nh << 31) | c_nw));
+    }
+    return;
   }
-  __syncthreads();
+  group_lookback(g, b, c_nh, c_nw, S);
   EIRENE_PHASE(g.A, 1, b, 3);
   const unsigned long long tp3 = g.prof ? gtime_ns() : 0;
   // sweep 2: emit (a small bucket reuses the carries of its single round)
-  if (mode == 2) {
-    const GView V{K, P, K, P, 0, sp_o};
-    if (sp_o) {
-      round_scan(V, sp_o, 0, sp_o, 0, 0, 0, S);
-      round_emit(g, V, sp_o, base, 0, sp_o, true, S, sp_lo, sp_h, hot_w);
-    }
-    __syncthreads();
-    const uint32_t sH = S.seg0 + a_nh, wH = S.w0 + a_nw, pos0 = base + sp_lo;
-    if ((g.prof & 1) && tid == 0) S.prof_t[0] = gtime_ns();
-    if (!deferred) hot_pass2(g, S.hot_bits, hc, sH, pos0);
-    if ((g.prof & 1) && tid == 0) S.prof_t[1] = gtime_ns();
-    if (tid == 0) {
-      const uint64_t hk = S.hk;
-      g.istart[sH] = pos0;
-      // deferred: the segment's positions (pinfo, sorted payloads) are not
-      // written; every result of it comes from the result phase's walk of the
-      // bitmap slot, spread over many CTAs (result_phase, eirene_internal.cuh)
-      if (deferred) g.hot_seg[S.hot_slot] = sH;
-      if (hot_w) {   // issue rule: the segment's last write
-        const uint32_t opw = hot_last & 3;
-        g.wkey[wH] = hk;
-        g.wop[wH] = (uint8_t)opw;
-        g.wval[wH] = (opw == OP_DELETE) ? KEY_MAX : g.A->vals[hot_last >> 2];
-        g.wseg[wH] = sH;
-      } else {       // all-query segment: its last query
-        g.qkey[sH - wH] = hk;
-        g.qseg[sH - wH] = sH;
-      }
-    }
-  } else if (small) {
+  if (mode == 2)
+    emit_split(g, S, base, sp_o, sp_lo, sp_h, hot_w, hot_last, a_nh, a_nw, deferred, hc);
+  else if (small) {
     if (cnt) round_emit(g, GView{K, P, K, P, 0, cnt}, cnt, base, 0, cnt, true, S);
-  } else {
-    const bool write_spay = P != g.pB + base;
-    c_nh = c_lw = c_nw = 0;
-    for (uint32_t r0 = 0; r0 < cnt; r0 += G_CAP) {
-      const uint32_t r1 = min(cnt, r0 + (uint32_t)G_CAP);
-      const GView V = load_round(r0, r1);
-      round_scan(V, cnt, r0, r1, c_nh, c_lw, c_nw, S);
-      round_emit(g, V, cnt, base, r0, r1, write_spay, S);
-      c_nh = S.r_nh;
-      c_lw = S.r_lw;
-      c_nw = S.r_nw;
-      __syncthreads();
-    }
-  }
+  } else
+    emit_rounds(g, S, K, P, cnt, base);
   EIRENE_PHASE(g.A, 1, b, 4);
 #ifdef EIRENE_GROUP_PROF_BUILD   // diagnostic builds only: printf in a kernel costs on every launch
   if ((g.prof & 1) && tid == 0) {
@@ -1425,8 +1530,10 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
 
 }  // namespace
 
+bool group_two_phase(uint32_t n, int num_sms) { return bsort_groups(n, num_sms) > 2u * (uint32_t)num_sms; }
+
 void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const CombBufs& c, Tree t, BatchCtl* ctl,
-                  int num_sms, cudaStream_t st, int* launches) {
+                  int num_sms, bool two_phase, cudaStream_t st, int* launches) {
   static int attr[MAX_DEVICES];
   per_device(attr, [] {
     return (int)cudaFuncSetAttribute(group_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(GSmem));
@@ -1455,10 +1562,24 @@ void launch_group(const BatchArgs* A, uint32_t n, const BSortBufs& b, const Comb
   g.hot_seg = c.hot_seg;
   static const int prof = std::getenv("EIRENE_GROUP_PROF") ? std::atoi(std::getenv("EIRENE_GROUP_PROF")) : 0;
   g.prof = prof;
+  g.grec = c.grec;
   g.t = t;
   g.ctl = ctl;
+  if (!two_phase) {
+    g.phase = 0;
+    launch_k(group_kernel, dim3(g.nb), dim3(G_THREADS), sizeof(GSmem), st, true, false, g);
+    ++*launches;
+    return;
+  }
+  static int attr2[MAX_DEVICES];
+  per_device(attr2, [] {
+    return (int)cudaFuncSetAttribute(group_emit_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                     (int)sizeof(GSmem));
+  });
+  g.phase = 1;
   launch_k(group_kernel, dim3(g.nb), dim3(G_THREADS), sizeof(GSmem), st, true, false, g);
-  ++*launches;
+  launch_k(group_emit_kernel, dim3(g.nb), dim3(G_THREADS), sizeof(GSmem), st, true, false, g);
+  *launches += 2;
 }
 
 }  // namespace eirene

@@ -511,6 +511,24 @@ def test_two_kernel_sort_size_band(dev, zipf):
     t.close()
 
 
+@pytest.mark.parametrize("n", [1_100_000, (1 << 21) + 77])
+def test_two_phase_group_stage(dev, n):
+    """More groups than one resident wave (2 per SM): the group stage runs as
+    two kernels -- sort + aggregates, then look-back + emit (group.cu) -- on
+    Zipf keys with every op kind, so small, L2-sorted and SPLIT (hot-key
+    bitmap) groups all cross the phase boundary; n = 1.1M stays on the fused
+    distribution kernel, 2^21 + 77 takes the two-kernel one."""
+    from paper_conf_ppopp_zhangz0lzl23_b200 import workload as W
+    w = W.Workload(3, tree=1 << 20, batch=n, fracs={0: 0.4, 1: 0.2, 2: 0.3, 3: 0.1})
+    t = make_tree(dev, w.keys, w.vals, max_keys=1 << 22, max_batch=n)
+    ref = oracle.MapOracle(); ref.load(w.keys, w.vals)
+    for b in range(2):
+        ops, keys, vals = w.batch_arrays(b)
+        run_and_compare(t, ref, ops, keys, vals, dev, check_scan=(b == 1))
+    assert t.check_invariants()[0] == 0
+    t.close()
+
+
 def test_structural_counts_and_device_time(dev):
     """nins / ndelp (the structural writes the update kernel is left with; value
     overwrites are applied in place by the query kernel) equal their definition
