@@ -88,6 +88,23 @@ struct QueryIO {
   uint32_t* __restrict__ longseg;
 };
 
+// A/B switch for the query kernel's result stores (EIRENE_RES_ST): 0 plain,
+// 1 L2 evict_last (a result sector stays in L2 until its four results are
+// written instead of being written back partially), 2 none (diagnostic:
+// wrong results, traffic only)
+#ifndef EIRENE_RES_ST
+#define EIRENE_RES_ST 0
+#endif
+__device__ __forceinline__ void st_result(tkey_t* p, uint64_t v) {
+#if EIRENE_RES_ST == 1
+  st64_pol(p, v, pol_evict_last());
+#elif EIRENE_RES_ST == 2
+  (void)p; (void)v;
+#else
+  *p = (tkey_t)v;
+#endif
+}
+
 __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, uint32_t nq, uint32_t node, int s,
                                        uint64_t v, tkey_t* __restrict__ results, BatchCtl* __restrict__ ctl,
                                        tkey_t* __restrict__ lvals) {
@@ -107,7 +124,7 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
   if (isq) {
     seg = qseg[i];
     if (seg & Q_SINGLE) {   // the segment's only request: its result, nothing else
-      results[seg & ~Q_SINGLE] = v;
+      st_result(results + (seg & ~Q_SINGLE), v);
       return;
     }
   } else {
@@ -140,10 +157,10 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
   const uint32_t p0 = istart[seg], p1 = istart[seg + 1];
   if (p1 - p0 <= SHORT_SEG) {
     if (isq) {   // an all-query segment: every position is pending
-      for (uint32_t p = p0; p < p1; ++p) results[spay[p] >> 2] = v;
+      for (uint32_t p = p0; p < p1; ++p) st_result(results + (spay[p] >> 2), v);
     } else {     // positions up to (and including) the first write are pending
       for (uint32_t p = p0; p < p1; ++p)
-        if (!(pinfo[p] & DONE_BIT)) results[spay[p] >> 2] = v;
+        if (!(pinfo[p] & DONE_BIT)) st_result(results + (spay[p] >> 2), v);
     }
   } else {   // work items of RCHUNK positions: (segment, chunk) pairs
     if (isq) old[seg] = v;
@@ -218,6 +235,9 @@ __device__ __forceinline__ void query_end(BatchCtl* ctl, const BatchArgs* A, con
   if (!s_need) publish_batch(ctl, A, hdr);
 }
 
+// The graph-mode variant with the conditional update node (EIRENE_COND) is a
+// kernel of its own: a kernel that references the device graph API is not
+// profiled by ncu inside a graph, and the default path should be.
 __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
@@ -230,12 +250,29 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
                                                         const uint32_t* __restrict__ pinfo,
                                                         const uint32_t* __restrict__ istart,
                                                         uint32_t* __restrict__ longseg, const BatchArgs* __restrict__ A,
-                                                        Tree t, BatchCtl* __restrict__ ctl,
-                                                        cudaGraphConditionalHandle cond, int use_cond) {
+                                                        Tree t, BatchCtl* __restrict__ ctl) {
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   query_body(qkey, qseg, wkey, wseg, wop, wval, wleaf, wslot, wparent, old, spay, pinfo, istart, longseg, A, t, ctl);
-  if (use_cond) query_end(ctl, A, t.hdr, cond);
+}
+__global__ void __launch_bounds__(256, 8) query_cond_kernel(const uint64_t* __restrict__ qkey,
+                                                        const uint32_t* __restrict__ qseg,
+                                                        const uint64_t* __restrict__ wkey,
+                                                        const uint32_t* __restrict__ wseg,
+                                                        const uint8_t* __restrict__ wop,
+                                                        const uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
+                                                        uint8_t* __restrict__ wslot, uint32_t* __restrict__ wparent,
+                                                        uint64_t* __restrict__ old,
+                                                        const uint32_t* __restrict__ spay,
+                                                        const uint32_t* __restrict__ pinfo,
+                                                        const uint32_t* __restrict__ istart,
+                                                        uint32_t* __restrict__ longseg, const BatchArgs* __restrict__ A,
+                                                        Tree t, BatchCtl* __restrict__ ctl,
+                                                        cudaGraphConditionalHandle cond) {
+  pdl_wait();
+  pdl_trigger();
+  query_body(qkey, qseg, wkey, wseg, wop, wval, wleaf, wslot, wparent, old, spay, pinfo, istart, longseg, A, t, ctl);
+  query_end(ctl, A, t.hdr, cond);
 }
 
 // Locality-aware warp reorganisation the paper's way (§5, P:1380-1512,
@@ -342,12 +379,21 @@ __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* 
                                                                  uint32_t* __restrict__ wparent, QueryIO io,
                                                                  const BatchArgs* __restrict__ A, Tree t,
                                                                  BatchCtl* __restrict__ ctl, uint32_t iter_rgs,
-                                                                 uint32_t stats, cudaGraphConditionalHandle cond,
-                                                                 int use_cond) {
+                                                                 uint32_t stats) {
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   query_iterwarp_body(qkey, wkey, wparent, io, A, t, ctl, iter_rgs, stats);
-  if (use_cond) query_end(ctl, A, t.hdr, cond);
+}
+__global__ void __launch_bounds__(256, 4) query_iterwarp_cond_kernel(const uint64_t* __restrict__ qkey,
+                                                                      const uint64_t* __restrict__ wkey,
+                                                                      uint32_t* __restrict__ wparent, QueryIO io,
+                                                                      const BatchArgs* __restrict__ A, Tree t,
+                                                                      BatchCtl* __restrict__ ctl, uint32_t iter_rgs,
+                                                                      uint32_t stats, cudaGraphConditionalHandle cond) {
+  pdl_wait();
+  pdl_trigger();
+  query_iterwarp_body(qkey, wkey, wparent, io, A, t, ctl, iter_rgs, stats);
+  query_end(ctl, A, t.hdr, cond);
 }
 
 // Diagnostics (EIRENE_DEBUG_SYNC / EIRENE_UPDATE_PROF only): printf lives in
@@ -568,13 +614,21 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
   if (flags & EIRENE_F_ITERWARP) {
     // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
     const int iblocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 4u);
-    launch_k(query_iterwarp_kernel, dim3(iblocks < 1 ? 1 : iblocks), dim3(256), 0, st, true, false, 
-        c.qkey, c.wkey, c.wparent,
-        QueryIO{c.qseg, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg},
-        A, t, ctl, iter_rgs, (flags & EIRENE_F_STATS) ? 1u : 0u, cond, use_cond);
+    const dim3 g(iblocks < 1 ? 1 : iblocks);
+    const QueryIO io{c.qseg, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg};
+    const uint32_t stats = (flags & EIRENE_F_STATS) ? 1u : 0u;
+    if (use_cond)
+      launch_k(query_iterwarp_cond_kernel, g, dim3(256), 0, st, true, false, c.qkey, c.wkey, c.wparent, io, A, t, ctl,
+               iter_rgs, stats, cond);
+    else
+      launch_k(query_iterwarp_kernel, g, dim3(256), 0, st, true, false, c.qkey, c.wkey, c.wparent, io, A, t, ctl,
+               iter_rgs, stats);
+  } else if (use_cond) {
+    launch_k(query_cond_kernel, dim3(blocks), dim3(256), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop,
+             c.wval, c.wleaf, c.wslot, c.wparent, c.old, spay, c.pinfo, c.istart, c.longseg, A, t, ctl, cond);
   } else {
-    launch_k(query_kernel, dim3(blocks), dim3(256), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.wparent, c.old,
-                                         spay, c.pinfo, c.istart, c.longseg, A, t, ctl, cond, use_cond);
+    launch_k(query_kernel, dim3(blocks), dim3(256), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval,
+             c.wleaf, c.wslot, c.wparent, c.old, spay, c.pinfo, c.istart, c.longseg, A, t, ctl);
   }
   ++*launches;
 }
