@@ -39,6 +39,9 @@ namespace eirene {
 
 namespace {
 
+#define GROUP_PRAGMA(x) _Pragma(#x)
+#define GROUP_UNROLL_(n) GROUP_PRAGMA(unroll n)
+
 constexpr int G_THREADS = 512;
 constexpr int G_WARPS = G_THREADS / 32;
 constexpr int G_ITEMS = 8;
@@ -288,7 +291,20 @@ __device__ __noinline__ bool hot_run_sort(uint32_t lo, uint32_t m, int tsbits, G
   return true;
 }
 
-__device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, int tsbits, GSmem& S) {
+#ifdef EIRENE_RANK_UNROLL   // A/B: the in-sub-bucket rank loop of smem_sort unrolled (loads in flight together)
+#define RANK_UNROLL GROUP_UNROLL_(EIRENE_RANK_UNROLL)
+#else
+#define RANK_UNROLL
+#endif
+// (A, b: the phase stamps of diagnostic builds, -DEIRENE_PHASE_PROF; null elsewhere)
+__device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, int tsbits, GSmem& S,
+                          const BatchArgs* A = nullptr, uint32_t b = 0) {
+#ifdef EIRENE_PHASE_PROF
+#define SS_PHASE(i) \
+  if (A) EIRENE_PHASE(A, 1, b, i)
+#else
+#define SS_PHASE(i) (void)A, (void)b
+#endif
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t C = 32u * ((cnt + G_THREADS - 1) / G_THREADS);
   const uint32_t wb = warp * C;
@@ -308,6 +324,7 @@ __device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, 
   }
   for (int i = tid; i <= SB_N; i += G_THREADS) S.sb[i] = 0;
   key_range(mn, mx, S);   // (its barriers also order the sb zeroing)
+  SS_PHASE(5);
   const uint64_t kmin = S.kmin, range = S.kmax - S.kmin;
   const int bits = 64 - __clzll((long long)range);
   const int shift = bits > SB_BITS ? bits - SB_BITS : 0;
@@ -356,6 +373,7 @@ __device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, 
     if (tid == 0) S.sb[SB_N] = cnt;
   }
   __syncthreads();
+  SS_PHASE(6);
 #pragma unroll
   for (int j = 0; j < G_ITEMS; ++j) {
     const uint32_t i = wb + 32 * j + lane;
@@ -375,6 +393,7 @@ __device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, 
       const uint32_t lo = S.sb[x], hi = S.sb[x + 1];
       if (hi - lo <= FAST_SB) {
         uint32_t less = 0;
+        RANK_UNROLL
         for (uint32_t m = lo; m < hi; ++m) less += kp_less(S.k[m], S.p[m], kr[j], pr[j]);
         r[j] = lo + less;
       }
@@ -389,6 +408,8 @@ __device__ void smem_sort(const uint64_t* ks, const uint32_t* ps, uint32_t cnt, 
     }
   }
   __syncthreads();
+  SS_PHASE(7);
+#undef SS_PHASE
   if (S.cmax <= FAST_SB) return;
   // big sub-buckets: list them, then bitonic-sort each in place
   if (tid == 0) S.r_nh = 0;
@@ -888,6 +909,17 @@ struct GView {
   __device__ __forceinline__ uint32_t p(uint32_t x) const { return x - c0 < c1 - c0 ? Ps[x - c0] : Pg[x]; }
 };
 
+// A/B switch: unrolling of the warps' 32-position steps (independent smem loads
+// of several steps in flight); EIRENE_GROUP_UNROLL=n
+#ifndef EIRENE_GROUP_UNROLL
+#define EIRENE_GROUP_UNROLL 2   // (A/B r2s: 2 > 1, 4)
+#endif
+#if EIRENE_GROUP_UNROLL > 1
+#define GROUP_UNROLL GROUP_UNROLL_(EIRENE_GROUP_UNROLL)
+#else
+#define GROUP_UNROLL
+#endif
+
 // Round [r0, r1) of a bucket walked by 16 warps: pass 1 (heads, last write per
 // warp), warp scan, pass 2 (write segments ending in each warp), warp scan.
 // Leaves the exclusive per-warp carries in S.c_* and the carry-out in S.r_*.
@@ -899,6 +931,7 @@ __device__ void round_scan(const GView& V, uint32_t cnt, uint32_t r0, uint32_t r
   const uint32_t wb = r0 + warp * C;
   const uint32_t we = min(r1, wb + C);
   uint32_t nh = 0, lw = 0;
+  GROUP_UNROLL
   for (uint32_t b = wb; b < we; b += 32) {
     const uint32_t x = b + lane;
     const bool valid = x < we;
@@ -926,6 +959,7 @@ __device__ void round_scan(const GView& V, uint32_t cnt, uint32_t r0, uint32_t r
   }
   __syncthreads();
   uint32_t lwc = S.c_lw[warp], nwt = 0;
+  GROUP_UNROLL
   for (uint32_t b = wb; b < we; b += 32) {
     const uint32_t x = b + lane;
     const bool valid = x < we;
@@ -964,6 +998,7 @@ __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uin
   const uint32_t we = min(r1, wb + C);
   const uint32_t seg0 = S.seg0, w0 = S.w0;
   uint32_t nh = S.c_nh[warp], lwc = S.c_lw[warp], nwc = S.c_nw[warp];
+  GROUP_UNROLL
   for (uint32_t b = wb; b < we; b += 32) {
     const uint32_t x = b + lane;
     const bool valid = x < we;
@@ -1002,7 +1037,7 @@ __device__ void round_emit(const GroupArgs& g, const GView& V, uint32_t cnt, uin
         const uint32_t opw = pw & 3;
         g.wkey[wi] = k;
         g.wop[wi] = (uint8_t)opw;
-        g.wval[wi] = (opw == OP_DELETE) ? KEY_MAX : vals[pw >> 2];
+        g.wval[wi] = pw >> 2;   // its timestamp: the query kernel's locate gathers the value (WVAL_TS)
         g.wseg[wi] = seg;
       } else {      // all-query segment: its last query
         const uint32_t qi = seg - wi;
@@ -1312,7 +1347,7 @@ __device__ void emit_split(const GroupArgs& g, GSmem& S, uint32_t base, uint32_t
       const uint32_t opw = hot_last & 3;
       g.wkey[wH] = hk;
       g.wop[wH] = (uint8_t)opw;
-      g.wval[wH] = (opw == OP_DELETE) ? KEY_MAX : g.A->vals[hot_last >> 2];
+      g.wval[wH] = hot_last >> 2;   // (timestamp, as above)
       g.wseg[wH] = sH;
     } else {       // all-query segment: its last query
       g.qkey[sH - wH] = hk;
@@ -1402,7 +1437,7 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
       S.k[0] = g.kA[base];
       S.p[0] = g.pA[base];
     } else if (cnt > 1) {
-      smem_sort(g.kA + base, g.pA + base, cnt, g.tsbits, S);
+      smem_sort(g.kA + base, g.pA + base, cnt, g.tsbits, S, g.A, b);
     }
     __syncthreads();
     K = S.k;

@@ -78,7 +78,8 @@ struct QueryIO {
   const uint32_t* __restrict__ qseg;
   const uint32_t* __restrict__ wseg;
   const uint8_t* __restrict__ wop;
-  const uint64_t* __restrict__ wval;
+  uint64_t* __restrict__ wval;      // in: the issued write's timestamp; out: its value (WVAL_TS)
+  const tkey_t* __restrict__ vals;  // the batch's values
   uint32_t* __restrict__ wleaf;
   uint8_t* __restrict__ wslot;
   uint64_t* __restrict__ old;
@@ -135,6 +136,11 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
     const uint32_t op = wop[w];
     ins = s < 0 && op != OP_DELETE;
     delp = s >= 0 && op == OP_DELETE;
+    // WVAL_TS: the group kernel left the issued write's timestamp in wval; its
+    // value is gathered from the batch here (off the group kernel's critical
+    // path) and stored back for the update kernel
+    const uint64_t wv = op == OP_DELETE ? KEY_MAX : (uint64_t)io.vals[io.wval[w]];
+    io.wval[w] = wv;
     // A value overwrite (upsert of a present key) changes one value slot and
     // nothing else, so it is applied here, by the thread that located it: the
     // structure is quiescent during this kernel (the update kernel runs after
@@ -143,7 +149,7 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
     // is already the pre-batch value the write returns.  The update kernel
     // then only has the structural writes (inserts of absent keys, deletes of
     // present ones) to do, and re-applies overwrites idempotently.
-    if (s >= 0 && op != OP_DELETE) lvals[(size_t)node * LSTRIDE + s] = io.wval[w];
+    if (s >= 0 && op != OP_DELETE) lvals[(size_t)node * LSTRIDE + s] = wv;
   }
   {
     const uint32_t am = __activemask();
@@ -178,7 +184,7 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
                                                         const uint8_t* __restrict__ wop,
-                                                        const uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
+                                                        uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
                                                         uint8_t* __restrict__ wslot, uint32_t* __restrict__ wparent,
                                                         uint64_t* __restrict__ old,
                                                         const uint32_t* __restrict__ spay,
@@ -214,7 +220,7 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
     const uint64_t v = s >= 0 ? load_value(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
     if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
-    retire(QueryIO{qseg, wseg, wop, wval, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
+    retire(QueryIO{qseg, wseg, wop, wval, A->vals, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
            results, ctl, t.lvals);
   }
 }
@@ -243,7 +249,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
                                                         const uint8_t* __restrict__ wop,
-                                                        const uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
+                                                        uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
                                                         uint8_t* __restrict__ wslot, uint32_t* __restrict__ wparent,
                                                         uint64_t* __restrict__ old,
                                                         const uint32_t* __restrict__ spay,
@@ -260,7 +266,7 @@ __global__ void __launch_bounds__(256, 8) query_cond_kernel(const uint64_t* __re
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
                                                         const uint8_t* __restrict__ wop,
-                                                        const uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
+                                                        uint64_t* __restrict__ wval, uint32_t* __restrict__ wleaf,
                                                         uint8_t* __restrict__ wslot, uint32_t* __restrict__ wparent,
                                                         uint64_t* __restrict__ old,
                                                         const uint32_t* __restrict__ spay,
@@ -301,6 +307,7 @@ __device__ __forceinline__ void query_iterwarp_body(const uint64_t* __restrict__
                                                                  uint32_t stats) {
   if (ctl->invalid || ctl->status != 0) return;
   tkey_t* __restrict__ results = A->results;
+  io.vals = A->vals;   // (the batch's pointers live on the device)
   const uint32_t nq = ctl->nq, nw = ctl->nw;
   if (!headroom_ok(t, nw)) {
     if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = EIRENE_EFULL;
@@ -615,7 +622,7 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
     // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
     const int iblocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 4u);
     const dim3 g(iblocks < 1 ? 1 : iblocks);
-    const QueryIO io{c.qseg, c.wseg, c.wop, c.wval, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg};
+    const QueryIO io{c.qseg, c.wseg, c.wop, c.wval, nullptr, c.wleaf, c.wslot, c.old, spay, c.pinfo, c.istart, c.longseg};
     const uint32_t stats = (flags & EIRENE_F_STATS) ? 1u : 0u;
     if (use_cond)
       launch_k(query_iterwarp_cond_kernel, g, dim3(256), 0, st, true, false, c.qkey, c.wkey, c.wparent, io, A, t, ctl,

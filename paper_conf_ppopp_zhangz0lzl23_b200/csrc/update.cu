@@ -1057,6 +1057,16 @@ __global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C, ResultArgs
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   const BatchCtl* ctl = C.ctl;
+  // nothing at all left (no structural write, long segment or deferred hot
+  // key; the common case of a read-mostly batch): CTA 0 ends the batch at
+  // once, no arrival counting, the other CTAs just exit
+  if (!update_needed(ctl, R.A)) {
+    if (blockIdx.x == 0) {
+      if (threadIdx.x == 0) C.ctl->upd_ran = 1;
+      publish_batch(C.ctl, R.A, R.hdr);
+    }
+    return;
+  }
   // skipped (uniformly: every CTA reads the same flags before any changes them)
   // for a rejected batch, and when every issued write was a value overwrite of
   // a present key: all of them were applied in place by the query kernel's

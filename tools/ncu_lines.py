@@ -26,8 +26,14 @@ for x in csv.reader(io.StringIO(out)):
     si = hdr.index("Warp Stall Sampling (All Samples)")
     ei = hdr.index("Instructions Executed")
     if x[si].isdigit():
-        data.append((int(x[si]), f"{f}:{x[0]}", x[ei], x[1].strip()))
+        st = sorted(((float(x[j] or 0), hdr[j][6:]) for j in range(len(hdr))
+                     if hdr[j].startswith("stall_") and "Not Issued" not in hdr[j] and x[j] not in ("", "-")),
+                    reverse=True)
+        xs = hdr.index("L1 Wavefronts Shared Excessive") if "L1 Wavefronts Shared Excessive" in hdr else None
+        exc = x[xs] if xs is not None else ""
+        why = " ".join(f"{n}:{int(v)}" for v, n in st[:3] if v > 0)
+        data.append((int(x[si]), f"{f}:{x[0]}", x[ei], x[1].strip(), why, exc))
 tot = sum(d[0] for d in data) or 1
 print("samples", tot)
-for a, loc, e, s in sorted(data, reverse=True)[:top]:
-    print(f"{a:6d} {100 * a / tot:5.1f}% {loc:24s} exec={e:>9s} {s[:80]}")
+for a, loc, e, s, why, exc in sorted(data, reverse=True)[:top]:
+    print(f"{a:6d} {100 * a / tot:5.1f}% {loc:24s} exec={e:>9s} [{why}] smem_excess={exc} | {s[:70]}")

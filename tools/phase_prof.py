@@ -24,7 +24,7 @@ wl = W.Workload(cfg, tree=C["tree"], batch=C["batch"])
 t = EireneTree(max_keys=max(2 * C["tree"], 1 << 20), max_batch=C["batch"])
 t.bulk_load(torch.from_numpy(wl.keys).to(dev), torch.from_numpy(wl.vals).to(dev))
 names = {0: ["start", "hist", "bcount atomics", "barrier", "cut", "tile hist+cursor", "scatter"],
-         1: ["ticket", "sort", "sweep1", "lookback", "emit"]}
+         1: ["ticket", "sort", "sweep1", "lookback", "emit", "ss:loaded+range", "ss:scan", "ss:rank"]}
 acc = {0: [], 1: []}
 for b in range(6):
     o, k, v = (torch.from_numpy(x).to(dev) for x in wl.batch_arrays(b))
