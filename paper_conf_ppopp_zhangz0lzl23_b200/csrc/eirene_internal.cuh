@@ -241,11 +241,42 @@ __device__ __forceinline__ uint64_t pol_evict_first() {
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
   return p;
 }
-// read-only (nc) loads with an L2 policy; 256-bit loads skip L1 allocation
+// read-only (nc) loads with an L2 policy; 256-bit loads skip L1 allocation.
+// A/B (EIRENE_LEAF_PF=128): the leaf line loads with an explicit 128 B L2 fetch size
 __device__ __forceinline__ ulonglong4 ldg256_pol(const uint64_t* p, uint64_t pol) {
   ulonglong4 v;
+#if defined(EIRENE_LEAF_PF) && EIRENE_LEAF_PF == 128
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::128B.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+               : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p), "l"(pol));
+#elif defined(EIRENE_LEAF_PF) && EIRENE_LEAF_PF == 64
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.L2::64B.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
+               : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p), "l"(pol));
+#else
   asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u64 {%0,%1,%2,%3}, [%4], %5;"
                : "=l"(v.x), "=l"(v.y), "=l"(v.z), "=l"(v.w) : "l"(p), "l"(pol));
+#endif
+  return v;
+}
+// one value with an explicit 64 B L2 fetch size (A/B: EIRENE_VAL_LOAD=4)
+__device__ __forceinline__ uint64_t ldg64_pol_64b(const uint64_t* p, uint64_t pol) {
+  uint64_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.L2::64B.u64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ uint64_t ldg64_pol_64b(const uint32_t* p, uint64_t pol) {
+  uint32_t v;
+  asm volatile("ld.global.nc.L2::cache_hint.L2::64B.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
+// ... and without an eviction policy (data re-read later in the batch: the write values)
+__device__ __forceinline__ uint64_t ldg64_64b(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.global.nc.L2::64B.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ uint64_t ldg64_64b(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.global.nc.L2::64B.u32 %0, [%1];" : "=r"(v) : "l"(p));
   return v;
 }
 __device__ __forceinline__ uint64_t ldg64_pol(const uint64_t* p, uint64_t pol) {

@@ -41,7 +41,7 @@ __device__ __forceinline__ uint32_t child_slot(const Tree& t, uint32_t node, uin
 // -DEIRENE_VAL_LOAD=1: L1 no-allocate; 2: plain coherent load; 0 (default):
 // read-only path with the evict_first L2 policy.
 #ifndef EIRENE_VAL_LOAD
-#define EIRENE_VAL_LOAD 0
+#define EIRENE_VAL_LOAD 4   // r2u: the default fetch of a value sector was 128 B (207 -> 174 MB per cfg2 launch)
 #endif
 __device__ __forceinline__ uint64_t load_value(const tkey_t* p, uint64_t pol) {
 #if EIRENE_VAL_LOAD == 1
@@ -54,6 +54,8 @@ __device__ __forceinline__ uint64_t load_value(const tkey_t* p, uint64_t pol) {
     asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.u32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
     return v;
   }
+#elif EIRENE_VAL_LOAD == 4
+  return ldg64_pol_64b(p, pol);
 #elif EIRENE_VAL_LOAD == 2
   (void)pol;
   return *p;
@@ -139,7 +141,7 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
     // WVAL_TS: the group kernel left the issued write's timestamp in wval; its
     // value is gathered from the batch here (off the group kernel's critical
     // path) and stored back for the update kernel
-    const uint64_t wv = op == OP_DELETE ? KEY_MAX : (uint64_t)io.vals[io.wval[w]];
+    const uint64_t wv = op == OP_DELETE ? KEY_MAX : ldg64_64b(io.vals + io.wval[w]);
     io.wval[w] = wv;
     // A value overwrite (upsert of a present key) changes one value slot and
     // nothing else, so it is applied here, by the thread that located it: the
@@ -217,8 +219,16 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
       // or four interleaved traversals per thread (tools/ab.py)
       node = ldg32_pol(t.ichild + (size_t)node * FAN + child_slot(t, node, k, pl), pl);
     }
+#if defined(EIRENE_QDIAG) && EIRENE_QDIAG == 2   // diagnostic (traffic only, wrong results): no leaf loads
+    const int s = -1;
+#else
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
+#endif
+#if defined(EIRENE_QDIAG) && EIRENE_QDIAG == 1   // diagnostic: no value load
+    const uint64_t v = s >= 0 ? 0ull : KEY_MAX;
+#else
     const uint64_t v = s >= 0 ? load_value(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
+#endif
     if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
     retire(QueryIO{qseg, wseg, wop, wval, A->vals, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
            results, ctl, t.lvals);
