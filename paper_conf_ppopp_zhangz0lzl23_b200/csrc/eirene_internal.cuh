@@ -63,10 +63,18 @@ struct NodeMeta {
 };
 static_assert(sizeof(NodeMeta) == 32, "meta is 32 B");
 
+// The allocation counters sit on lines of their own: under a split storm
+// every split leaf's warp does an atomic on leaf_count, and the root word is
+// read by every descent.  level_count[0] is not maintained by the update
+// kernel (leaves are never freed: it equals leaf_count, which is what
+// headroom_ok uses for level 0).
 struct TreeHdr {
   unsigned long long root_word;          // (height << 32) | root id; height 1 = leaf root
-  uint32_t leaf_count, inner_count;      // pool allocation counters
-  uint32_t level_count[MAX_LEVELS];      // nodes per level (EFULL bound)
+  uint32_t pad0[30];
+  uint32_t leaf_count;                   // leaf pool allocation counter
+  uint32_t pad1[31];
+  uint32_t inner_count;                  // inner pool allocation counter
+  uint32_t level_count[MAX_LEVELS];      // nodes per level (EFULL bound; [0] see above)
 };
 
 // Per-batch device scalars; zeroed (cudaMemsetAsync) before every batch.
@@ -404,7 +412,7 @@ __device__ __forceinline__ bool headroom_ok(const Tree& t, uint32_t nw) {
   unsigned long long need_leaf = nw;
   unsigned long long N = nw, inner = 0;
   for (uint32_t l = 0; l + 1 < height && N > 0; ++l) {
-    unsigned long long I = h->level_count[l];
+    unsigned long long I = l == 0 ? h->leaf_count : h->level_count[l];
     unsigned long long Nn = min(N, (I + N) / 8 + 1);
     inner += Nn;
     N = Nn;

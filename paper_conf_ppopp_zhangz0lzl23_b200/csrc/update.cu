@@ -62,6 +62,7 @@ struct WarpStats {
                      new_inner = 0;
   unsigned long long t0 = 0;
   bool dead = false;
+  bool leaf_root = true;   // the tree had height 1 at the kernel's start (else no leaf is ever the root)
 };
 
 // Watchdog (see eirene_internal.cuh): true if this warp must give up.
@@ -313,7 +314,6 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
   const uint32_t tout = c - __popc(mmask) + U;
   const uint32_t k = tout <= FAN ? 1u : (tout + FAN - 1) / FAN;
   const uint32_t first = k > 1 ? warp_alloc(&t.hdr->leaf_count, k - 1) : 0u;
-  if (k > 1 && lane == 0) atomicAdd(&t.hdr->level_count[0], k - 1);
   const uint32_t bs = tout / k, rem = tout % k, big = rem * (bs + 1);
   auto place = [&](uint32_t f, uint64_t key, uint64_t val) {
     uint32_t q, start;
@@ -665,7 +665,7 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
           ws.runs += 1;
           if (k > 1) {
             bool rooted = false;
-            if (is_root(t, X, 0)) {
+            if (ws.leaf_root && is_root(t, X, 0)) {
               build_root(C, 0, X, lo, hi, C.eK[0], C.eC[0], C.eK[1], C.eC[1], b, k - 1, ws);
               rooted = true;
             }
@@ -1087,6 +1087,7 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
   const Tree& t = C.t;
   WarpStats ws;
   ws.t0 = gtime_ns();
+  ws.leaf_root = (uint32_t)(ld_acquire64(&t.hdr->root_word) >> 32) <= 1;   // (heights never shrink)
   SepAcc acc;
   // level-synchronous separators when the batch can split (launch: resident grid)
   const bool lsync = C.regroup && C.slots[0] != nullptr && ctl->nins > 0;
