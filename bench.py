@@ -393,7 +393,7 @@ def run_ours(args):
         # weak scaling: the global tree holds world * tree_n keys, the global batch
         # world * batch_n requests; rank r owns key range r and ts-slice r
         wl = W.Workload(cfg, tree=tree_n * world, batch=batch_n * world, **wkw)
-        sh = ShardedEirene(wl.keys, wl.vals, max_batch=batch_n, device=dev)
+        sh = ShardedEirene(wl.keys, wl.vals, max_batch=batch_n, device=dev, fused=args.route == "fused")
         for f_ in (0.97, 1.0, 1.03, 1.1):   # graph capture for the likely shard batch size buckets, untimed
             sh.engine.prepare(min(int(batch_n * f_), batch_n * world))
         host_batches = []
@@ -630,7 +630,9 @@ def run_ours(args):
         e2e = {"value": batch_n * world * n_e / (float(e_ms.item()) * 1e-3) / 1e9, "unit": "Greq/s",
                "h2d_bytes_per_step": int(world * batch_n * 17), "d2h_bytes_per_step": int(world * batch_n * 8),
                "steps": n_e, "path": "ShardedEirene.submit_host on every rank: pinned H2D of the rank's slice, "
-                                     "routing + NCCL exchanges + shard batch, D2H of the results slice (one "
+                                     + ("fused push routing (partition kernel storing into the peers' arenas, "
+                                        "results pushed back) " if args.route == "fused" else
+                                        "routing + NCCL exchanges ") + "+ shard batch, D2H of the results slice (one "
                                      "stream per rank); max over ranks"}
 
     # ------------------------------------------------------------ parity at N > 1
@@ -807,7 +809,9 @@ def run_ours(args):
                                    + (f" (YCSB-like mix {args.mix})" if args.mix else "")
                                    + (f", range length {cap} (first {cap} pairs returned)" if cap else ""),
                        "cfg": cfg, "global_batch": batch_n * world,
-                       "parallelism": f"key-range shards x{world}" if world > 1 else "single GPU",
+                       "parallelism": (f"key-range shards x{world}, "
+                                       + ("fused push over peer memory" if args.route == "fused"
+                                          else "NCCL all-to-all")) if world > 1 else "single GPU",
                        "l2": "distinct input/result buffers per step (steps x 25 MiB >> 126 MB L2); "
                              "inner levels stay L2-resident across batches (steady state)"},
             "batch_ms": spread(dev_batch_ms, "device %globaltimer: start of the batch's first kernel to the end of "
@@ -860,6 +864,9 @@ def main():
     ap.add_argument("--mix", default="", choices=["", "A", "B", "C", "U"],
                     help="YCSB-like mix override (cfg5): A 50/50 Zipf, B 95/5 Zipf, C 100%% read Zipf, U 95/5 uniform")
     ap.add_argument("--parity-slice", type=int, default=1 << 16, help="loaded keys per parity slice (N > 1)")
+    ap.add_argument("--route", default="fused", choices=["nccl", "fused"],
+                    help="N > 1 exchange: NCCL all-to-all, or the fused push into the peers' arenas over CUDA IPC "
+                         "peer memory (SURVEY 8(f) NEXT(3))")
     ap.add_argument("--pipeline", type=int, default=0,
                     help="1: cross-batch pipelining (EIRENE_F_PIPELINE, SURVEY 8(f) NEXT(3))")
     args = ap.parse_args()

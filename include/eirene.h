@@ -354,6 +354,62 @@ int eirene_route_unpermute(eirene_handle h, const uint64_t* recv_results_dev,
                            const uint32_t* perm_dev, uint32_t n, uint64_t* results_dev,
                            eirene_stream_t stream);
 
+/* ---- fused routing over peer memory (one-shot NVLink
+ * push fusing route_partition with the exchange; §8(e) steps 2-8).  Each rank
+ * owns a receive ARENA in device memory: P source slots {count, invalid flag,
+ * start, epoch} (u32 x4), cap result words (this rank's slice, partition
+ * order) and P x cap 24 B records.  The partition kernel stores every request
+ * directly into its destination's arena (peer memory over NVLink 5 /
+ * NVSwitch, mapped by CUDA IPC; in one process, any device pointers), so no
+ * payload collective runs: the caller only orders the ranks with a barrier
+ * (e.g. a one-word NCCL all_reduce on the same stream) after eirene_route_push
+ * and after eirene_route_push_results.  Every rank calls every function for
+ * every global batch in the same order, with the same P and cap. ---------- */
+#define EIRENE_IPC_HANDLE_BYTES 64
+
+/* Allocates this rank's arena for P ranks (1 <= P <= 64), rank `rank`, at
+ * most `cap` requests per rank slice (the source's n of eirene_route_push).
+ * *arena_dev_out = its device address; if ipc_handle_out != NULL it receives
+ * EIRENE_IPC_HANDLE_BYTES of CUDA IPC handle for the other processes.  Freed
+ * by eirene_destroy.  ESTATE if the handle already has an arena. */
+int eirene_route_arena_create(eirene_handle h, int P, int rank, uint32_t cap, void** arena_dev_out,
+                              void* ipc_handle_out);
+/* Maps a peer process's arena (its IPC handle) into this process:
+ * *arena_dev_out = the address to pass to eirene_route_arena_connect.
+ * Unmapped by eirene_destroy. */
+int eirene_route_arena_open_ipc(eirene_handle h, const void* ipc_handle, void** arena_dev_out);
+/* peer_arenas (host array of P device addresses; entry `rank` = this rank's own
+ * arena): the destinations of the pushes.  Synchronous. */
+int eirene_route_arena_connect(eirene_handle h, void* const* peer_arenas);
+/* Source side (steps 2+4 fused): the stable partition of eirene_route_partition
+ * (dest = upper_bound(splitters, key), perm_dev[n] as there, validation of
+ * eirene_submit_batch) whose scatter stores each request as a {key, value, op}
+ * record into arena(dest).rec[rank][j], j its index among this slice's
+ * requests for dest (timestamp order); then every destination's slot [rank]
+ * gets {count, invalid, start of dest's segment in perm order, epoch}.
+ * n <= cap.  Asynchronous on `stream`; the pushes are complete (system-scope
+ * fenced) when the stream reaches its end. */
+int eirene_route_push(eirene_handle h, const uint8_t* ops_dev, const uint64_t* keys_dev, const uint64_t* vals_dev,
+                      uint32_t n, const uint64_t* splitters_dev, uint32_t* perm_dev, eirene_stream_t stream);
+/* Receiver side, after the barrier that follows every rank's push: reads the
+ * P slots (ONE host synchronisation of `stream`), sets *n_out = requests
+ * received and *invalid_out = 1 if any source's slice holds an invalid request
+ * (then nothing is written: every rank sees the same flags, so all reject the
+ * global batch), else compacts the records in source-rank order (= timestamp
+ * order) into ops/keys/vals_out[*n_out] (n_cap entries
+ * available) for eirene_submit_batch.  EINTERNAL if a source's slot does not
+ * carry this batch's epoch (its push never arrived). */
+int eirene_route_pull(eirene_handle h, uint8_t* ops_out_dev, uint64_t* keys_out_dev, uint64_t* vals_out_dev,
+                      uint32_t n_cap, uint32_t* n_out, uint32_t* invalid_out, eirene_stream_t stream);
+/* Receiver side: the shard's results_dev[*n_out of the last pull] (pulled
+ * order) stored back into every source's arena at its partition positions
+ * (step 7).  Asynchronous; the caller's barrier must follow it. */
+int eirene_route_push_results(eirene_handle h, const uint64_t* results_dev, eirene_stream_t stream);
+/* Source side, after that barrier: results_dev[perm_dev[j]] = arena.res[j] for
+ * j < n (step 8).  Asynchronous. */
+int eirene_route_unpermute_arena(eirene_handle h, const uint32_t* perm_dev, uint32_t n, uint64_t* results_dev,
+                                 eirene_stream_t stream);
+
 #ifdef __cplusplus
 }
 #endif

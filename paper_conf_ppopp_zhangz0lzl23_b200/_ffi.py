@@ -57,6 +57,8 @@ class eirene_tree_info(ctypes.Structure):
                 ("inner_cap", _u64), ("launches", _u64), ("device_bytes", _u64)]
 
 
+EIRENE_IPC_HANDLE_BYTES = 64   # include/eirene.h
+
 _SIGS = {
     "eirene_default_config": (None, [ctypes.POINTER(eirene_config)]),
     "eirene_create": (_int, [ctypes.POINTER(eirene_config), ctypes.POINTER(_vp)]),
@@ -81,6 +83,13 @@ _SIGS = {
     "eirene_batch_status_async": (_int, [_vp, _u64, _vp, _vp]),
     "eirene_debug_phases": (_int, [_vp, _vp, _u32]),
     "eirene_stream_wait_batch": (_int, [_vp, _u64, _vp]),
+    "eirene_route_arena_create": (_int, [_vp, _int, _int, _u32, ctypes.POINTER(_vp), _vp]),
+    "eirene_route_arena_open_ipc": (_int, [_vp, _vp, ctypes.POINTER(_vp)]),
+    "eirene_route_arena_connect": (_int, [_vp, _vp]),
+    "eirene_route_push": (_int, [_vp, _vp, _vp, _vp, _u32, _vp, _vp, _vp]),
+    "eirene_route_pull": (_int, [_vp, _vp, _vp, _vp, _u32, ctypes.POINTER(_u32), ctypes.POINTER(_u32), _vp]),
+    "eirene_route_push_results": (_int, [_vp, _vp, _vp]),
+    "eirene_route_unpermute_arena": (_int, [_vp, _vp, _u32, _vp, _vp]),
 }
 
 _libs: dict = {}

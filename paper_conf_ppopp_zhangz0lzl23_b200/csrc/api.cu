@@ -213,6 +213,24 @@ struct eirene_tree {
   uint64_t launches = 0;
   size_t device_bytes = 0;
   std::vector<void*> allocs;
+  // fused routing (eirene_route_arena_*): this rank's receive arena, the P
+  // peers' arenas (IPC-mapped or, in one process, plain device pointers)
+  struct Arena {
+    void* base = nullptr;
+    uint32_t P = 0, me = 0, cap = 0, epoch = 0;
+    uint32_t* cnt = nullptr;        // [P] uint4 {count, invalid, start, epoch} written by the sources
+    uint64_t* res = nullptr;        // [cap] results pushed back by the shards (this rank's partition order)
+    uint64_t* rec = nullptr;        // [P][cap][3] records pushed by the sources
+    uint32_t* lcnt = nullptr;       // [64] local per-destination counts of the push
+    uint32_t* linv = nullptr;       // validity flag of the push
+    uint64_t** d_prec = nullptr;    // device tables [P]: peers' rec / res / cnt
+    uint64_t** d_pres = nullptr;
+    uint32_t** d_pcnt = nullptr;
+    uint32_t* h_cnt = nullptr;      // pinned [P * 4]
+    uint32_t pushed_n = 0;          // largest per-source count of the last pull (grid sizing)
+    bool connected = false;
+    std::vector<void*> opened;      // IPC mappings to close
+  } ar;
 
   template <class T>
   cudaError_t dalloc(T** p, size_t count) {
@@ -261,7 +279,7 @@ const char* eirene_strerror(int code) {
     case EIRENE_EFULL: return "node pools lack headroom for the batch";
     case EIRENE_ESTATE: return "call not valid in this state (or stale ticket)";
     case EIRENE_ECUDA: return "CUDA error (see eirene_last_cuda_error)";
-    case EIRENE_EINTERNAL: return "device watchdog fired: no forward progress (internal error; discard the tree)";
+    case EIRENE_EINTERNAL: return "internal error: the device watchdog fired (no forward progress; discard the tree) or a peer's routed push never arrived";
     default: return "unknown error";
   }
 }
@@ -542,6 +560,8 @@ int eirene_destroy(eirene_handle h) {
     if (h->comp_done[s]) cudaEventDestroy(h->comp_done[s]);
     if (h->comp_ev[s]) cudaEventDestroy(h->comp_ev[s]);
   }
+  for (void* p : h->ar.opened) cudaIpcCloseMemHandle(p);
+  if (h->ar.h_cnt) cudaFreeHost(h->ar.h_cnt);
   for (void* p : h->allocs) cudaFree(p);
   if (h->host_ctl) cudaFreeHost(h->host_ctl);
   if (h->res_stream) cudaStreamDestroy(h->res_stream);
@@ -1208,6 +1228,166 @@ int eirene_route_unpermute(eirene_handle h, const uint64_t* recv, const uint32_t
   CK(dg_.err);
   int launches = 0;
   launch_route_unpermute(recv, perm, n, results, reinterpret_cast<cudaStream_t>(stream), &launches);
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+// ---------------------------------------------------------------- fused routing over peer memory
+// Arena layout (identical on every rank): [0, 1024) the P source slots
+// {count, invalid, start, epoch}; [1024, ..) res[cap]; then rec[P][cap][3].
+static size_t arena_res_off() { return 1024; }
+static size_t arena_rec_off(uint32_t cap) { return 1024 + (((size_t)cap * 8 + 255) / 256) * 256; }
+static size_t arena_bytes(uint32_t P, uint32_t cap) { return arena_rec_off(cap) + (size_t)P * cap * 24; }
+
+int eirene_route_arena_create(eirene_handle h, int P, int rank, uint32_t cap, void** arena_dev_out,
+                              void* ipc_handle_out) {
+  if (!h || P < 1 || P > 64 || rank < 0 || rank >= P || cap == 0 || !arena_dev_out) return EIRENE_EINVAL;
+  if (h->ar.base) return EIRENE_ESTATE;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  auto& A = h->ar;
+  unsigned char* base = nullptr;
+  CK(h->dalloc(&base, arena_bytes((uint32_t)P, cap)));
+  CK(cudaMemset(base, 0, 1024));
+  A.base = base;
+  A.P = (uint32_t)P;
+  A.me = (uint32_t)rank;
+  A.cap = cap;
+  A.cnt = reinterpret_cast<uint32_t*>(base);
+  A.res = reinterpret_cast<uint64_t*>(base + arena_res_off());
+  A.rec = reinterpret_cast<uint64_t*>(base + arena_rec_off(cap));
+  CK(h->dalloc(&A.lcnt, 64));
+  CK(h->dalloc(&A.linv, 1));
+  CK(h->dalloc(&A.d_prec, 64));
+  CK(h->dalloc(&A.d_pres, 64));
+  CK(h->dalloc(&A.d_pcnt, 64));
+  CK(cudaMallocHost(reinterpret_cast<void**>(&A.h_cnt), sizeof(uint32_t) * 4 * 64));
+  *arena_dev_out = base;
+  if (ipc_handle_out) {
+    cudaIpcMemHandle_t ih;
+    CK(cudaIpcGetMemHandle(&ih, base));
+    std::memcpy(ipc_handle_out, &ih, sizeof(ih));
+  }
+  return EIRENE_OK;
+}
+
+int eirene_route_arena_open_ipc(eirene_handle h, const void* ipc_handle, void** arena_dev_out) {
+  if (!h || !ipc_handle || !arena_dev_out) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  cudaIpcMemHandle_t ih;
+  std::memcpy(&ih, ipc_handle, sizeof(ih));
+  void* p = nullptr;
+  CK(cudaIpcOpenMemHandle(&p, ih, cudaIpcMemLazyEnablePeerAccess));
+  h->ar.opened.push_back(p);
+  *arena_dev_out = p;
+  return EIRENE_OK;
+}
+
+int eirene_route_arena_connect(eirene_handle h, void* const* peer_arenas) {
+  if (!h || !peer_arenas) return EIRENE_EINVAL;
+  auto& A = h->ar;
+  if (!A.base) return EIRENE_ESTATE;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  uint64_t* prec[64];
+  uint64_t* pres[64];
+  uint32_t* pcnt[64];
+  for (uint32_t d = 0; d < A.P; ++d) {
+    unsigned char* b = static_cast<unsigned char*>(peer_arenas[d]);
+    if (!b) return EIRENE_EINVAL;
+    prec[d] = reinterpret_cast<uint64_t*>(b + arena_rec_off(A.cap));
+    pres[d] = reinterpret_cast<uint64_t*>(b + arena_res_off());
+    pcnt[d] = reinterpret_cast<uint32_t*>(b);
+  }
+  CK(cudaMemcpy(A.d_prec, prec, sizeof(void*) * A.P, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(A.d_pres, pres, sizeof(void*) * A.P, cudaMemcpyHostToDevice));
+  CK(cudaMemcpy(A.d_pcnt, pcnt, sizeof(void*) * A.P, cudaMemcpyHostToDevice));
+  A.connected = true;
+  return EIRENE_OK;
+}
+
+int eirene_route_push(eirene_handle h, const uint8_t* ops, const uint64_t* keys, const uint64_t* vals, uint32_t n,
+                      const uint64_t* splitters, uint32_t* perm, eirene_stream_t stream) {
+  if (!h) return EIRENE_EINVAL;
+  auto& A = h->ar;
+  if (!A.connected) return EIRENE_ESTATE;
+  if (n > A.cap || n > h->cfg.max_batch) return EIRENE_EINVAL;
+  if (n > 0 && (!ops || !keys || !vals || !perm)) return EIRENE_EINVAL;
+  if (A.P > 1 && !splitters) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  int launches = 0;
+  CK(cudaMemsetAsync(A.linv, 0, sizeof(uint32_t), st));
+  launch_route_partition(ops, keys, vals, n, splitters, (int)A.P, nullptr, nullptr, nullptr, nullptr, perm, A.lcnt, 1,
+                         A.linv, h->route_lb, h->route_ctr, ++h->route_epoch, st, &launches, A.d_prec, A.me, A.cap);
+  launch_push_counts(A.lcnt, A.linv, (int)A.P, A.me, A.d_pcnt, ++A.epoch, st, &launches);
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+int eirene_route_pull(eirene_handle h, uint8_t* ops_out, uint64_t* keys_out, uint64_t* vals_out, uint32_t n_cap,
+                      uint32_t* n_out, uint32_t* invalid_out, eirene_stream_t stream) {
+  if (!h || !n_out || !invalid_out) return EIRENE_EINVAL;
+  auto& A = h->ar;
+  if (!A.connected) return EIRENE_ESTATE;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  cudaStream_t st = reinterpret_cast<cudaStream_t>(stream);
+  CK(cudaMemcpyAsync(A.h_cnt, A.cnt, sizeof(uint32_t) * 4 * A.P, cudaMemcpyDeviceToHost, st));
+  CK(cudaStreamSynchronize(st));   // the one host synchronisation of a fused-routing batch
+  uint64_t n = 0;
+  uint32_t inv = 0, mx = 0;
+  for (uint32_t s = 0; s < A.P; ++s) {
+    const uint32_t* e = A.h_cnt + 4 * s;
+    if (e[3] != A.epoch) return EIRENE_EINTERNAL;   // a source's push of this batch never arrived
+    n += e[0];
+    inv |= e[1];
+    mx = std::max(mx, e[0]);
+  }
+  *invalid_out = inv;
+  *n_out = (uint32_t)std::min<uint64_t>(n, 0xFFFFFFFFull);
+  A.pushed_n = 0;
+  if (inv) return EIRENE_OK;
+  if (n > n_cap || n > h->cfg.max_batch) return EIRENE_EINVAL;
+  if (n > 0 && (!ops_out || !keys_out || !vals_out)) return EIRENE_EINVAL;
+  int launches = 0;
+  launch_pull_unpack(A.cnt, A.rec, A.cap, (int)A.P, mx, ops_out, keys_out, vals_out, st, &launches);
+  A.pushed_n = mx;
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+int eirene_route_push_results(eirene_handle h, const uint64_t* results, eirene_stream_t stream) {
+  if (!h) return EIRENE_EINVAL;
+  auto& A = h->ar;
+  if (!A.connected) return EIRENE_ESTATE;
+  if (A.pushed_n > 0 && !results) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  int launches = 0;
+  launch_push_results(A.cnt, results, (int)A.P, A.pushed_n, A.d_pres, reinterpret_cast<cudaStream_t>(stream),
+                      &launches);
+  A.pushed_n = 0;
+  h->launches += launches;
+  CK(cudaGetLastError());
+  return EIRENE_OK;
+}
+
+int eirene_route_unpermute_arena(eirene_handle h, const uint32_t* perm, uint32_t n, uint64_t* results,
+                                 eirene_stream_t stream) {
+  if (!h) return EIRENE_EINVAL;
+  auto& A = h->ar;
+  if (!A.connected) return EIRENE_ESTATE;
+  if (n > A.cap || (n > 0 && (!perm || !results))) return EIRENE_EINVAL;
+  DeviceGuard dg_(h->cfg.device);
+  CK(dg_.err);
+  int launches = 0;
+  launch_route_unpermute(A.res, perm, n, results, reinterpret_cast<cudaStream_t>(stream), &launches);
   h->launches += launches;
   CK(cudaGetLastError());
   return EIRENE_OK;

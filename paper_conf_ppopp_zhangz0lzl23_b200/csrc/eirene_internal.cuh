@@ -598,7 +598,14 @@ void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint
                             const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
                             uint64_t* rec, uint32_t* perm, uint32_t* counts, uint32_t cstride, uint32_t* invalid,
                             unsigned long long* lookback, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st,
-                            int* launches);
+                            int* launches, uint64_t* const* peer_rec = nullptr, uint32_t me = 0, uint32_t cap = 0);
+// fused push over peer memory (NVLink): counts / arena compaction / results back
+void launch_push_counts(const uint32_t* counts, const uint32_t* invalid, int P, uint32_t me, uint32_t* const* peer_cnt,
+                        uint32_t epoch, cudaStream_t st, int* launches);
+void launch_pull_unpack(const uint32_t* cnt, const uint64_t* rec, uint32_t cap, int P, uint32_t max_per_src,
+                        uint8_t* ops, uint64_t* keys, uint64_t* vals, cudaStream_t st, int* launches);
+void launch_push_results(const uint32_t* cnt, const uint64_t* res, int P, uint32_t max_per_src,
+                         uint64_t* const* peer_res, cudaStream_t st, int* launches);
 void launch_route_unpack(const uint64_t* rec, uint32_t n, uint8_t* ops, uint64_t* keys, uint64_t* vals,
                          cudaStream_t st, int* launches);
 void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,

@@ -68,6 +68,7 @@ struct RtSmem {
   uint32_t cnt[RT_MAXP];
   uint32_t bin_base[RT_MAXP];
   uint32_t bin_start[RT_MAXP];
+  uint64_t* prec[RT_MAXP];   // fused push: destination d's receive arena records (peer memory)
   uint32_t tile_id;
 };
 
@@ -76,7 +77,8 @@ __global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
     const uint64_t* __restrict__ splitters, int P, uint32_t* __restrict__ counts, uint32_t cstride,
     const uint32_t* __restrict__ invalid, uint8_t* __restrict__ sops, uint64_t* __restrict__ skeys,
     uint64_t* __restrict__ svals, uint64_t* __restrict__ rec, uint32_t* __restrict__ perm,
-    unsigned long long* __restrict__ lookback, uint32_t epoch, uint32_t* __restrict__ tile_ctr) {
+    unsigned long long* __restrict__ lookback, uint32_t epoch, uint32_t* __restrict__ tile_ctr,
+    uint64_t* const* __restrict__ peer_rec, uint32_t me, uint32_t cap) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
   RtSmem& S = *reinterpret_cast<RtSmem*>(smem_raw);
   const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
@@ -90,6 +92,7 @@ __global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
   }
   for (int i = tid; i < RT_WARPS * RT_MAXP; i += RT_THREADS) (&S.wh[0][0])[i] = 0;
   if (tid < RT_MAXP) S.sp[tid] = tid < P - 1 ? splitters[tid] : KEY_MAX;
+  if (peer_rec && tid < P) S.prec[tid] = peer_rec[tid];
   __syncthreads();
   const uint32_t tile = S.tile_id, base = tile * RT_TILE;
   // packed mode: every destination's count word is followed by the batch's
@@ -173,8 +176,14 @@ __global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
   const uint32_t tile_n = min((uint32_t)RT_TILE, n - base);
   for (uint32_t i = tid; i < tile_n; i += RT_THREADS) {
     const uint64_t key = S.keys[i];
-    const uint32_t o = S.bin_base[dest_of(key, S.sp, P)] + i;
-    if (rec) {   // one 24 B record {key, value, op} per request: one payload exchange
+    const uint32_t d = dest_of(key, S.sp, P);
+    const uint32_t o = S.bin_base[d] + i;
+    if (peer_rec) {   // fused push: straight into destination d's arena, region of source `me`
+      uint64_t* dst = S.prec[d] + 3 * ((size_t)me * cap + (o - S.bin_start[d]));
+      dst[0] = key;
+      dst[1] = S.vals[i];
+      dst[2] = S.ops[i];
+    } else if (rec) {   // one 24 B record {key, value, op} per request: one payload exchange
       rec[3 * (size_t)o] = key;
       rec[3 * (size_t)o + 1] = S.vals[i];
       rec[3 * (size_t)o + 2] = S.ops[i];
@@ -185,6 +194,58 @@ __global__ void __launch_bounds__(RT_THREADS) route_scatter_kernel(
     }
     perm[o] = S.idx[i];
   }
+  // (the records must be visible to the peer once this kernel is complete: the
+  // caller's barrier -- an NCCL collective on the same stream -- follows it)
+  if (peer_rec) __threadfence_system();
+}
+
+// Fused push, after the scatter: source `me` tells every destination d how
+// many records it pushed, whether its slice holds an invalid request, where
+// d's segment starts in its own partition order (the results come back
+// there) and the batch epoch, in d's arena slot [me]: {count, invalid,
+// start, epoch}.  Written for every d (also count 0), so a receiver always
+// hears from every source.
+__global__ void push_counts_kernel(const uint32_t* __restrict__ counts, const uint32_t* __restrict__ invalid, int P,
+                                   uint32_t me, uint32_t* const* __restrict__ peer_cnt, uint32_t epoch) {
+  const int d = threadIdx.x;
+  if (d < P) {
+    uint32_t start = 0;
+    for (int x = 0; x < d; ++x) start += counts[x];
+    uint4* dst = reinterpret_cast<uint4*>(peer_cnt[d]) + me;
+    *dst = make_uint4(counts[d], invalid ? *invalid : 0u, start, epoch);
+    __threadfence_system();
+  }
+}
+
+// Receiver: the P sources' records in its arena, rx_rec[src][0, cnt_src),
+// compacted in source-rank (= timestamp) order into the shard's SoA batch.
+__global__ void pull_unpack_kernel(const uint4* __restrict__ cnt, const uint64_t* __restrict__ rec, uint32_t cap,
+                                   uint8_t* __restrict__ ops, uint64_t* __restrict__ keys,
+                                   uint64_t* __restrict__ vals) {
+  const uint32_t src = blockIdx.y;
+  uint32_t off = 0;
+  for (uint32_t x = 0; x < src; ++x) off += cnt[x].x;
+  const uint32_t c = cnt[src].x;
+  const uint64_t* r = rec + 3 * (size_t)src * cap;
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < c; j += gridDim.x * blockDim.x) {
+    keys[off + j] = r[3 * (size_t)j];
+    vals[off + j] = r[3 * (size_t)j + 1];
+    ops[off + j] = (uint8_t)r[3 * (size_t)j + 2];
+  }
+}
+
+// Receiver: the shard's results (source-rank order) pushed back into every
+// source's arena at the position its partition gave them (start_src + j).
+__global__ void push_results_kernel(const uint4* __restrict__ cnt, const uint64_t* __restrict__ res,
+                                    uint64_t* const* __restrict__ peer_res) {
+  const uint32_t src = blockIdx.y;
+  uint32_t off = 0;
+  for (uint32_t x = 0; x < src; ++x) off += cnt[x].x;
+  const uint4 e = cnt[src];
+  uint64_t* dst = peer_res[src] + e.z;
+  for (uint32_t j = blockIdx.x * blockDim.x + threadIdx.x; j < e.x; j += gridDim.x * blockDim.x)
+    dst[j] = res[off + j];
+  __threadfence_system();
 }
 
 __global__ void unpermute_kernel(const uint64_t* __restrict__ recv, const uint32_t* __restrict__ perm, uint32_t n,
@@ -215,7 +276,7 @@ void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint
                             const uint64_t* splitters, int P, uint8_t* sops, uint64_t* skeys, uint64_t* svals,
                             uint64_t* rec, uint32_t* perm, uint32_t* counts, uint32_t cstride, uint32_t* invalid,
                             unsigned long long* lookback, uint32_t* tile_ctr, uint32_t epoch, cudaStream_t st,
-                            int* launches) {
+                            int* launches, uint64_t* const* peer_rec, uint32_t me, uint32_t cap) {
   static int attr[MAX_DEVICES];
   per_device(attr, [] {
     return (int)cudaFuncSetAttribute(route_scatter_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -229,8 +290,30 @@ void launch_route_partition(const uint8_t* ops, const uint64_t* keys, const uint
   const uint32_t tiles = (n + RT_TILE - 1) / RT_TILE;
   route_scatter_kernel<<<tiles, RT_THREADS, sizeof(RtSmem), st>>>(ops, keys, vals, n, splitters, P, counts, cstride,
                                                                   invalid, sops, skeys, svals, rec, perm, lookback,
-                                                                  epoch, tile_ctr);
+                                                                  epoch, tile_ctr, peer_rec, me, cap);
   *launches += 2;
+}
+
+void launch_push_counts(const uint32_t* counts, const uint32_t* invalid, int P, uint32_t me, uint32_t* const* peer_cnt,
+                        uint32_t epoch, cudaStream_t st, int* launches) {
+  push_counts_kernel<<<1, 64, 0, st>>>(counts, invalid, P, me, peer_cnt, epoch);
+  ++*launches;
+}
+
+void launch_pull_unpack(const uint32_t* cnt, const uint64_t* rec, uint32_t cap, int P, uint32_t max_per_src,
+                        uint8_t* ops, uint64_t* keys, uint64_t* vals, cudaStream_t st, int* launches) {
+  if (max_per_src == 0) return;
+  const dim3 grid(std::max(1u, std::min<uint32_t>((max_per_src + 255) / 256, 148u * 8u / (uint32_t)P)), P);
+  pull_unpack_kernel<<<grid, 256, 0, st>>>(reinterpret_cast<const uint4*>(cnt), rec, cap, ops, keys, vals);
+  ++*launches;
+}
+
+void launch_push_results(const uint32_t* cnt, const uint64_t* res, int P, uint32_t max_per_src,
+                         uint64_t* const* peer_res, cudaStream_t st, int* launches) {
+  if (max_per_src == 0) return;
+  const dim3 grid(std::max(1u, std::min<uint32_t>((max_per_src + 255) / 256, 148u * 8u / (uint32_t)P)), P);
+  push_results_kernel<<<grid, 256, 0, st>>>(reinterpret_cast<const uint4*>(cnt), res, peer_res);
+  ++*launches;
 }
 
 void launch_route_unpermute(const uint64_t* recv, const uint32_t* perm, uint32_t n, uint64_t* results,

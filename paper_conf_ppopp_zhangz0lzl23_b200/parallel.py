@@ -24,6 +24,15 @@ batch needs one exchange step each way:
   6. all_to_all_single returns the results; route_unpermute (CUDA kernel)
      puts them back in the slice's timestamp order.
 
+With fused=True (bench.py's default at N > 1) steps 2-4 and 6 run over peer
+memory instead: every rank's receive arena is mapped
+into every other rank by CUDA IPC (NVLink 5 / NVSwitch), the partition kernel
+stores each request straight into its destination's arena
+(eirene_route_push), the shard pulls its records after a one-word barrier
+(eirene_route_pull: the one host sync) and pushes the results straight back
+(eirene_route_push_results); the status all-reduce is the second barrier.
+No payload collective runs at all.
+
 The engine (per-shard tree) and router are injectable so the host-side logic
 (splitters, count exchange, concatenation order, inverse permutation) can be
 tested on CPU with the gloo backend; the product path uses EireneTree and its
@@ -63,7 +72,7 @@ class ShardedEirene:
     """
 
     def __init__(self, keys: np.ndarray, vals: np.ndarray, max_batch: int, device=None, group=None,
-                 engine=None, router=None, **tree_kw):
+                 engine=None, router=None, fused: bool = False, **tree_kw):
         self.group = group
         self.world = dist.get_world_size(group) if dist.is_initialized() else 1
         self.rank = dist.get_rank(group) if dist.is_initialized() else 0
@@ -82,6 +91,55 @@ class ShardedEirene:
         if my_k.size:
             self.engine.bulk_load(torch.from_numpy(my_k).to(self.device), torch.from_numpy(my_v).to(self.device))
         self.splitters = torch.from_numpy(self.splitters_np if self.world > 1 else np.zeros(1, np.uint64)).to(self.device)
+        self.fused = fused
+        if fused:
+            self._connect_arenas()
+
+    def _connect_arenas(self):
+        """Fused routing: every rank's receive arena, mapped into every other rank's
+        process over CUDA IPC (peer memory over NVLink 5 / NVSwitch), so the partition kernel pushes the
+        requests straight into their shards and the shards push the results straight back."""
+        addr, ipc = self.engine.route_arena_create(self.world, self.rank, self.max_batch)
+        handles = [ipc]
+        if self.world > 1:
+            handles = [None] * self.world
+            dist.all_gather_object(handles, ipc, group=self.group)
+        addrs = [addr if r == self.rank else self.engine.route_arena_open_ipc(handles[r]) for r in range(self.world)]
+        self.engine.route_arena_connect(addrs)
+        self._tok = torch.zeros(1, dtype=torch.int32, device=self.device)
+
+    def _barrier(self):
+        """Stream-ordered barrier: no rank passes it before every rank's preceding kernels (its pushes into
+        the peers' arenas) are complete."""
+        if self.world > 1:
+            dist.all_reduce(self._tok, group=self.group)
+
+    def _submit_fused(self, ops, keys, vals, results) -> "ShardedTicket":
+        """One global batch with the fused push: partition + peer stores (no payload collective), barrier,
+        pull (the one host sync), the shard's batch, results pushed back, barrier (the status all-reduce),
+        unpermute from the arena."""
+        P, n, dev = self.world, int(ops.numel()), self.device
+        perm = torch.empty(n, dtype=torch.int32, device=dev)
+        self.engine.route_push(ops, keys, vals, self.splitters, perm)
+        self._barrier()
+        cap = P * self.max_batch
+        rops = torch.empty(cap, dtype=torch.uint8, device=dev)
+        rkeys = torch.empty(cap, dtype=torch.uint64, device=dev)
+        rvals = torch.empty(cap, dtype=torch.uint64, device=dev)
+        nrecv, invalid = self.engine.route_pull(rops, rkeys, rvals)
+        if invalid:   # every rank saw every source's flag: all reject the global batch
+            return ShardedTicket(self, None, None, n, rejected=-1)
+        rres = torch.empty(max(nrecv, 1), dtype=torch.uint64, device=dev)
+        status = torch.zeros(1, dtype=torch.int32, device=dev)
+        tk = None
+        if nrecv:
+            tk = self.engine.submit(rops[:nrecv], rkeys[:nrecv], rvals[:nrecv], rres[:nrecv])
+            self.engine.status_async(tk, status)   # (orders the current stream after the batch)
+        self.engine.route_push_results(rres)
+        if P > 1:   # the status all-reduce doubles as the barrier after the result pushes
+            dist.all_reduce(status, op=dist.ReduceOp.MIN, group=self.group)
+        self.engine.route_unpermute_arena(perm, results)
+        return ShardedTicket(self, tk, status, n, keep=(perm, rops, rkeys, rvals, rres))
 
     def submit(self, ops: torch.Tensor, keys: torch.Tensor, vals: torch.Tensor, results: torch.Tensor) -> "ShardedTicket":
         """Process this rank's timestamp slice of a global batch; `results` (slice order) is valid once the
@@ -93,6 +151,8 @@ class ShardedEirene:
           -> all_to_all(24 B records) -> route_unpack -> submit (shard's hot path)
           -> status copy + all_reduce(MIN) -> all_to_all(results) -> route_unpermute
         """
+        if self.fused:
+            return self._submit_fused(ops, keys, vals, results)
         P = self.world
         n = int(ops.numel())
         rec, perm, cnt2 = self.router.route_partition_packed(ops, keys, vals, self.splitters, P)

@@ -262,6 +262,50 @@ class EireneTree:
                                           self._stream(stream)), "eirene_route_unpack")
         return ops, keys, vals
 
+    # ------------------------------------------- fused routing over peer memory (NEXT(3))
+    def route_arena_create(self, P: int, rank: int, cap: int) -> tuple[int, bytes]:
+        """This rank's receive arena: (device address, CUDA IPC handle bytes)."""
+        addr = ctypes.c_void_p()
+        ipc = ctypes.create_string_buffer(_ffi.EIRENE_IPC_HANDLE_BYTES)
+        check(self._L.eirene_route_arena_create(self._h, P, rank, cap, ctypes.byref(addr), ipc),
+              "eirene_route_arena_create")
+        return int(addr.value), bytes(ipc.raw)
+
+    def route_arena_open_ipc(self, handle: bytes) -> int:
+        addr = ctypes.c_void_p()
+        buf = ctypes.create_string_buffer(bytes(handle), _ffi.EIRENE_IPC_HANDLE_BYTES)
+        check(self._L.eirene_route_arena_open_ipc(self._h, buf, ctypes.byref(addr)), "eirene_route_arena_open_ipc")
+        return int(addr.value)
+
+    def route_arena_connect(self, peer_addrs: list[int]):
+        arr = (ctypes.c_void_p * len(peer_addrs))(*peer_addrs)
+        check(self._L.eirene_route_arena_connect(self._h, arr), "eirene_route_arena_connect")
+
+    def route_push(self, ops, keys, vals, splitters: torch.Tensor | None, perm: torch.Tensor, stream=None):
+        """Partition this slice and store every request into its destination's arena; perm int32[n] out."""
+        n = ops.numel()
+        check(self._L.eirene_route_push(self._h, _ptr(ops), _ptr(keys), _ptr(vals), n,
+                                        _ptr(splitters) if splitters is not None else None, _ptr(perm),
+                                        self._stream(stream)), "eirene_route_push")
+
+    def route_pull(self, ops, keys, vals, stream=None) -> tuple[int, int]:
+        """Compact the records pushed to this rank into ops/keys/vals (capacity = their length);
+        returns (n, invalid).  One host synchronisation."""
+        n = _ffi._u32()
+        inv = _ffi._u32()
+        check(self._L.eirene_route_pull(self._h, _ptr(ops), _ptr(keys), _ptr(vals), ops.numel(), ctypes.byref(n),
+                                        ctypes.byref(inv), self._stream(stream)), "eirene_route_pull")
+        return int(n.value), int(inv.value)
+
+    def route_push_results(self, results: torch.Tensor | None, stream=None):
+        check(self._L.eirene_route_push_results(self._h, _ptr(results) if results is not None else None,
+                                                self._stream(stream)), "eirene_route_push_results")
+
+    def route_unpermute_arena(self, perm: torch.Tensor, out: torch.Tensor, stream=None):
+        check(self._L.eirene_route_unpermute_arena(self._h, _ptr(perm), perm.numel(), _ptr(out),
+                                                   self._stream(stream)), "eirene_route_unpermute_arena")
+        return out
+
     def status_async(self, ticket: int, out: torch.Tensor, stream=None):
         """Enqueue a copy of batch `ticket`'s final status into out (int32[1] on the device), no host sync."""
         check(self._L.eirene_batch_status_async(self._h, ticket, _ptr(out), self._stream(stream)),
