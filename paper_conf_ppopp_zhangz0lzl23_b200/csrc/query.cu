@@ -78,6 +78,53 @@ __device__ __forceinline__ int slot16(const tkey_t* __restrict__ line, uint64_t 
   return l.find(k);
 }
 
+#ifndef EIRENE_QCOOP
+#define EIRENE_QCOOP 0   // A/B: warp-cooperative leaf search (KPL lanes read one leaf's key line)
+#endif
+// Warp-cooperative leaf search: the 32 lanes' leaves are read KPL lanes per
+// leaf line (each lane one 32 B sector), 32/KPL leaves per 256-bit load
+// instruction, so every L1 tag lookup of a leaf load serves a whole line
+// instead of one sector of 32 different lines; the KPL lanes of a leaf compare
+// their keys with the owner's key (shuffled) and the owner collects the slot
+// by ballot.  All KPL loads are issued before any compare.
+__device__ __forceinline__ int slot16_coop(const tkey_t* __restrict__ lkeys, uint32_t node, uint64_t k, uint64_t pol) {
+  constexpr int KPL = FAN * (int)sizeof(tkey_t) / 32;   // lanes per leaf line: 4 (u64 keys) or 2 (u32)
+  constexpr int LPR = 32 / KPL;                          // leaves per round
+  constexpr int KPW = 32 / (int)sizeof(tkey_t);          // keys per 32 B sector
+  const uint32_t lane = threadIdx.x & 31u, g = lane / KPL, part = lane % KPL;
+  ulonglong4 q[KPL];
+  uint64_t kt[KPL];
+#pragma unroll
+  for (int r = 0; r < KPL; ++r) {
+    const uint32_t src = LPR * r + g;
+    const uint32_t leaf = __shfl_sync(FULL, node, src);
+    kt[r] = __shfl_sync(FULL, k, src);
+    q[r] = ldg256_pol(reinterpret_cast<const uint64_t*>(lkeys + (size_t)leaf * LSTRIDE) + 4 * part, pol);
+  }
+  int s = -1;
+  const uint32_t my_r = lane / LPR, my_g = lane % LPR;
+#pragma unroll
+  for (int r = 0; r < KPL; ++r) {
+    const uint64_t w[4] = {q[r].x, q[r].y, q[r].z, q[r].w};
+    int li = -1;
+#pragma unroll
+    for (int y = 0; y < 4; ++y) {
+      if constexpr (sizeof(tkey_t) == 8) {
+        if (w[y] == kt[r]) li = y;
+      } else {
+        if ((w[y] & 0xFFFFFFFFull) == kt[r]) li = 2 * y;
+        if ((w[y] >> 32) == kt[r]) li = 2 * y + 1;
+      }
+    }
+    const uint32_t b = __ballot_sync(FULL, li >= 0);
+    const uint32_t bits = (b >> (KPL * my_g)) & ((1u << KPL) - 1u);
+    const int sub = bits ? __ffs(bits) - 1 : 0;
+    const int lsrc = __shfl_sync(FULL, li, KPL * my_g + sub);
+    if ((int)my_r == r && bits) s = sub * KPW + lsrc;
+  }
+  return s;
+}
+
 // Everything after the locate of issued request i (list position i < nq:
 // query, else write i - nq) at leaf `node`, slot s (-1 = absent), value v:
 // the write's leaf/slot for the update kernel, the segment's old value, and
@@ -212,7 +259,17 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
   const uint64_t pl = pol_evict_last(), pf = pol_evict_first();
-#if EIRENE_QRUN
+#if EIRENE_QCOOP
+  // Warp-uniform steps of 32 consecutive issued requests (lanes with i >= total
+  // ride along with a dummy key, so the leaf search can shuffle over the warp)
+  const uint32_t lane = threadIdx.x & 31u;
+  const uint32_t wstride = gridDim.x * blockDim.x;
+  for (uint32_t i0 = blockIdx.x * blockDim.x + (threadIdx.x & ~31u); i0 < total; i0 += wstride) {
+    const uint32_t i = i0 + lane;
+    const bool valid = i < total;
+    const bool isq = i < nq;
+    const uint64_t k = !valid ? 0ull : isq ? qkey[i] : wkey[i - nq];
+#elif EIRENE_QRUN
   // every thread takes a contiguous run of the key-sorted list: its next key
   // is the neighbour of the last one, so the inner nodes it walks again (the
   // level-1 and level-2 nodes, L2 round trips on a first visit) are L1 hits
@@ -223,8 +280,10 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
   const uint32_t stride = gridDim.x * blockDim.x;
   for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < total; i += stride) {
 #endif
+#if !EIRENE_QCOOP
     const bool isq = i < nq;
     const uint64_t k = isq ? qkey[i] : wkey[i - nq];
+#endif
     uint32_t node = root, parent = NIL;
     for (uint32_t lvl = height - 1; lvl > 0; --lvl) {
       parent = node;   // after the loop: the leaf's parent (the level-1 node)
@@ -241,6 +300,8 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
     }
 #if defined(EIRENE_QDIAG) && EIRENE_QDIAG == 2   // diagnostic (traffic only, wrong results): no leaf loads
     const int s = -1;
+#elif EIRENE_QCOOP
+    const int s = slot16_coop(t.lkeys, node, k, pf);
 #else
     const int s = slot16(t.lkeys + (size_t)node * LSTRIDE, k, pf);
 #endif
@@ -248,6 +309,9 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
     const uint64_t v = s >= 0 ? 0ull : KEY_MAX;
 #else
     const uint64_t v = s >= 0 ? load_value(t.lvals + (size_t)node * LSTRIDE + s, pf) : KEY_MAX;
+#endif
+#if EIRENE_QCOOP
+    if (!valid) continue;
 #endif
     if (!isq) wparent[i - nq] = parent;   // (the parent hint of the update kernel's first level)
     retire(QueryIO{qseg, wseg, wop, wval, A->vals, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,

@@ -260,61 +260,83 @@ __device__ void build_root(const Ctx& C, uint32_t L, uint32_t id0, uint64_t lo0,
   }
 }
 
-// Merge writes [b, e) (key-sorted, all inside the locked leaf X's fences) into
-// X.  Every write returns the value X held for its key (old[seg]), NOT_FOUND if
-// absent.  Result t keys; t <= 16 stays in X, else an even multi-way split into
-// k = ceil(t/16) leaves (X + k-1 fresh), entries (first key, leaf) for the
-// parent written to (Ek, Ec)[b .. b+k-2].  Returns k.
-__device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e, uint64_t X_hi, uint32_t X_next,
-                               uint64_t okey, uint64_t oval, uint64_t* Ek, uint32_t* Ec, WarpStats& ws) {
-  // okey / oval: X's key and value of slot `lane` (lanes < 16), loaded by the caller under the lock
-  const int lane = lane_id();
-  const Tree& t = C.t;
-  const size_t xb = (size_t)X * LSTRIDE;
-  const uint32_t c = __popc(__ballot_sync(FULL, okey != KEY_MAX));
-
-  uint32_t mmask = 0, U = 0, ups_before = 0;
+// The merge of writes [b, e) into a leaf whose c keys are okey (slot `lane`,
+// lanes < 16): which of the leaf's keys the writes hit (mmask), how many
+// upserts (U), per leaf key the upserts before it (ups_before, lanes < c), and
+// whether every write is a value overwrite of a present key (inplace).
+struct LeafPlan {
+  uint32_t c = 0, mmask = 0, U = 0, ups_before = 0;
   bool inplace = true;
+};
+// #leaf keys < wk: the leaf's keys sit sorted in lanes 0..15 (KEY_MAX padding
+// above), so a 5-step binary search over shuffles
+__device__ __forceinline__ uint32_t rank16(uint64_t okey, uint64_t wk) {
+  uint32_t lo = 0;
+#pragma unroll
+  for (uint32_t s = 8; s > 0; s >>= 1)
+    if (shfl64(okey, lo + s - 1) < wk) lo += s;
+  if (shfl64(okey, lo) < wk) ++lo;   // (only reachable at lo == 15)
+  return lo;
+}
+// #active write lanes whose key < ok (the step's write keys are ascending over the lanes, KEY_MAX when inactive)
+__device__ __forceinline__ uint32_t rank32(uint64_t wk, uint64_t ok) {
+  uint32_t lo = 0;
+#pragma unroll
+  for (uint32_t s = 16; s > 0; s >>= 1)
+    if (shfl64(wk, lo + s - 1) < ok) lo += s;
+  if (shfl64(wk, lo & 31u) < ok) ++lo;   // (only reachable at lo == 31)
+  return lo;
+}
+__device__ __forceinline__ LeafPlan leaf_plan(const Ctx& C, uint32_t b, uint32_t e, uint64_t okey) {
+  const int lane = lane_id();
+  LeafPlan L;
+  L.c = __popc(__ballot_sync(FULL, okey != KEY_MAX));
   for (uint32_t base = b; base < e; base += 32) {
     const uint32_t j = base + lane;
     const bool act = j < e;
     const uint64_t wk = act ? C.wkey[j] : KEY_MAX;
     const uint32_t wo = act ? C.wop[j] : 0;
-    uint32_t lo = 0;
-#pragma unroll
-    for (int i = 0; i < FAN; ++i) lo += shfl64(okey, i) < wk ? 1u : 0u;
-    const uint64_t at = shfl64(okey, lo);
-    const uint64_t ov = shfl64(oval, lo);
-    const bool match = act && lo < c && at == wk;
+    const uint32_t lo = rank16(okey, wk);
+    const uint64_t at = shfl64(okey, lo & 15u);
+    const bool match = act && lo < L.c && at == wk;
     const bool ups = act && wo != OP_DELETE;
-    mmask |= __reduce_or_sync(FULL, match ? (1u << lo) : 0u);
+    L.mmask |= __reduce_or_sync(FULL, match ? (1u << lo) : 0u);
     const uint32_t um = __ballot_sync(FULL, ups);
-    U += __popc(um);
-    if (__any_sync(FULL, act && !(match && ups))) inplace = false;
-    if (c > 0 && um) {
-      for (uint32_t i = 0; i < c; ++i) {
-        const uint64_t oi = shfl64(okey, i);
-        const uint32_t bm = __ballot_sync(FULL, ups && wk < oi);
-        if (lane == (int)i) ups_before += __popc(bm);
-      }
+    L.U += __popc(um);
+    if (__any_sync(FULL, act && !(match && ups))) L.inplace = false;
+    if (L.c > 0 && um) {   // upserts before leaf key `lane`: the writes below it, counted over um
+      const uint32_t p = rank32(wk, okey);
+      if (lane < (int)L.c) L.ups_before += __popc(p >= 32 ? um : (um & ((1u << p) - 1u)));
     }
   }
-  if (inplace) {   // only value overwrites of present keys: no structural change
-    for (uint32_t base = b; base < e; base += 32) {
-      const uint32_t j = base + lane;
-      const bool act = j < e;
-      const uint64_t wk = act ? C.wkey[j] : KEY_MAX;
-      uint32_t lo = 0;
-#pragma unroll
-      for (int i = 0; i < FAN; ++i) lo += shfl64(okey, i) < wk ? 1u : 0u;
-      if (act) t.lvals[xb + lo] = C.wval[j];
-    }
-    return 1;   // ordered before the release by unlock()
+  return L;
+}
+
+// Only value overwrites of present keys: no structural change.
+__device__ __forceinline__ void leaf_overwrite(const Ctx& C, uint32_t X, uint32_t b, uint32_t e, uint64_t okey) {
+  const int lane = lane_id();
+  for (uint32_t base = b; base < e; base += 32) {
+    const uint32_t j = base + lane;
+    const bool act = j < e;
+    const uint64_t wk = act ? C.wkey[j] : KEY_MAX;
+    const uint32_t lo = rank16(okey, wk);
+    if (act) C.t.lvals[(size_t)X * LSTRIDE + lo] = C.wval[j];
   }
-  const uint32_t tout = c - __popc(mmask) + U;
-  const uint32_t k = tout <= FAN ? 1u : (tout + FAN - 1) / FAN;
-  const uint32_t first = k > 1 ? warp_alloc(&t.hdr->leaf_count, k - 1) : 0u;
+}
+
+// The merged sequence (tout keys) written over X and k-1 fresh leaves
+// first.. (even multi-way split); entries (first key, leaf) for the parent
+// to (Ek, Ec)[b .. b+k-2] if Ek != null.  Returns, in every lane, the first
+// key of the second leaf (k > 1).
+__device__ uint64_t leaf_place(const Ctx& C, uint32_t X, uint32_t first, uint32_t b, uint32_t e, uint64_t okey,
+                               uint64_t oval, const LeafPlan& L, uint32_t tout, uint32_t k, uint64_t* Ek,
+                               uint32_t* Ec) {
+  const int lane = lane_id();
+  const Tree& t = C.t;
   const uint32_t bs = tout / k, rem = tout % k, big = rem * (bs + 1);
+  const uint32_t mmask = L.mmask;
+  uint64_t k1 = 0;   // this lane placed slot 0 of leaf 1
+  bool has1 = false;
   auto place = [&](uint32_t f, uint64_t key, uint64_t val) {
     uint32_t q, start;
     if (f < big) {
@@ -329,21 +351,25 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
     t.lkeys[(size_t)id * LSTRIDE + slot] = key;
     t.lvals[(size_t)id * LSTRIDE + slot] = val;
     if (q > 0 && slot == 0) {
-      Ek[b + q - 1] = key;
-      Ec[b + q - 1] = id;
+      if (Ek) {
+        Ek[b + q - 1] = key;
+        Ec[b + q - 1] = id;
+      }
+      if (q == 1) {
+        k1 = key;
+        has1 = true;
+      }
     }
   };
-  if (lane < (int)c && !((mmask >> lane) & 1u))
-    place(lane - __popc(mmask & ((1u << lane) - 1u)) + ups_before, okey, oval);
+  if (lane < (int)L.c && !((mmask >> lane) & 1u))
+    place(lane - __popc(mmask & ((1u << lane) - 1u)) + L.ups_before, okey, oval);
   uint32_t urun = 0;
   for (uint32_t base = b; base < e; base += 32) {
     const uint32_t j = base + lane;
     const bool act = j < e;
     const uint64_t wk = act ? C.wkey[j] : KEY_MAX;
     const uint32_t wo = act ? C.wop[j] : 0;
-    uint32_t lo = 0;
-#pragma unroll
-    for (int i = 0; i < FAN; ++i) lo += shfl64(okey, i) < wk ? 1u : 0u;
+    const uint32_t lo = rank16(okey, wk);
     const bool ups = act && wo != OP_DELETE;
     const uint32_t um = __ballot_sync(FULL, ups);
     if (ups) place(lo - __popc(mmask & ((1u << lo) - 1u)) + urun + __popc(um & lanemask_lt()), wk, C.wval[j]);
@@ -356,6 +382,31 @@ __device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e,
       if (s >= sz) t.lkeys[(size_t)(q == 0 ? X : first + q - 1) * LSTRIDE + s] = KEY_MAX;
     }
   }
+  const uint32_t h1 = __ballot_sync(FULL, has1);
+  return h1 ? shfl64(k1, __ffs(h1) - 1) : 0ull;
+}
+
+// Merge writes [b, e) (key-sorted, all inside the locked leaf X's fences) into
+// X.  Every write returns the value X held for its key (old[seg], retrieved by
+// the query kernel), NOT_FOUND if absent.  Result t keys; t <= 16 stays in X,
+// else an even multi-way split into k = ceil(t/16) leaves (X + k-1 fresh),
+// entries (first key, leaf) for the parent written to (Ek, Ec)[b .. b+k-2].
+// Returns k.
+__device__ uint32_t leaf_apply(const Ctx& C, uint32_t X, uint32_t b, uint32_t e, uint64_t X_hi, uint32_t X_next,
+                               uint64_t okey, uint64_t oval, uint64_t* Ek, uint32_t* Ec, WarpStats& ws) {
+  // okey / oval: X's key and value of slot `lane` (lanes < 16), loaded by the caller under the lock
+  const int lane = lane_id();
+  const Tree& t = C.t;
+  const LeafPlan L = leaf_plan(C, b, e, okey);
+  if (L.inplace) {   // only value overwrites of present keys: no structural change
+    leaf_overwrite(C, X, b, e, okey);
+    return 1;   // ordered before the release by unlock()
+  }
+  const uint32_t tout = L.c - __popc(L.mmask) + L.U;
+  const uint32_t k = tout <= FAN ? 1u : (tout + FAN - 1) / FAN;
+  const uint32_t first = k > 1 ? warp_alloc(&t.hdr->leaf_count, k - 1) : 0u;
+  const uint32_t bs = tout / k, rem = tout % k;
+  leaf_place(C, X, first, b, e, okey, oval, L, tout, k, Ek, Ec);
   // (no fence here: the new leaves are unreachable until X links them below,
   // X itself is read only under its lock; __syncwarp orders the lanes' Ek
   // writes before the meta loop reads them)
@@ -433,11 +484,10 @@ __device__ uint32_t inner_apply(const Ctx& C, uint32_t P, uint32_t L, uint64_t p
   for (uint32_t base = 0; base < m; base += 32) {
     const uint32_t x = base + lane;
     const uint64_t ek = x < m ? ld_cg(K + eb + x) : KEY_MAX;
-    for (uint32_t i = 1; i < cP; ++i) {   // entries are > plo, so child 0 stays first
-      const uint64_t li = shfl64(pk, i - 1);
-      const uint32_t bm = __ballot_sync(FULL, ek < li);
-      if (lane == (int)i) below += __popc(bm);
-    }
+    // child i >= 1: the entries below its left separator pk[i-1] (entries are
+    // > plo, so child 0 stays first); the entries ascend over the lanes
+    const uint32_t p = rank32(ek, my_low);
+    if (lane >= 1 && lane < (int)cP) below += p;
   }
   // padding first (disjoint from the element slots below)
   for (uint32_t q0 = 0; q0 < kp; q0 += 2) {
@@ -457,9 +507,7 @@ __device__ uint32_t inner_apply(const Ctx& C, uint32_t P, uint32_t L, uint64_t p
     const bool act = x < m;
     const uint64_t ek = act ? ld_cg(K + eb + x) : KEY_MAX;
     const uint32_t ec = act ? ld_cg(Ch + eb + x) : NIL;
-    uint32_t lt = 0;
-#pragma unroll
-    for (int i = 0; i < FAN - 1; ++i) lt += shfl64(pk, i) < ek ? 1u : 0u;   // pk[>= cP-1] == KEY_MAX
+    const uint32_t lt = rank16(pk, ek);   // pk[>= cP-1] == KEY_MAX
     if (act) place(x + 1 + lt, ec, ek);
   }
   __threadfence();
@@ -693,6 +741,155 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
   }
 }
 
+
+#ifndef UPD_BATCH
+#define UPD_BATCH 1   // A/B: 0 = every leaf run of a chunk through process_run, one after the other
+#endif
+// Split storms (level-synchronous mode): the leaf runs of one chunk that end
+// inside it (head lanes `bm`, run of lane h = [base + h, eL_h), leaf lf_h,
+// key order = lane order) applied TOGETHER, so the chunk pays each round trip
+// of Alg.1:34-45 once instead of once per run: every leaf locked at once
+// (test-and-set per lane), every locked leaf's fences and key/value block read
+// at once (into shared memory), one allocation for all splits, one fence, all
+// links and releases at once.  Each run holds <= 16 writes, so it leaves at
+// most two leaves (k <= 2: one separator entry).  A run whose lock is busy or
+// whose keys fall outside the leaf's fences (Alg.1:40-43) is released
+// untouched and returned in the mask for process_run (retry / STM).  Per lane
+// h of a split run: ek = the new leaf's first key, nid = its id.
+__device__ uint32_t batched_runs(const Ctx& C, uint32_t base, uint32_t bm, uint32_t eL, uint32_t lf, WarpStats& ws,
+                                 uint64_t& ek, uint32_t& nid, bool& split) {
+  __shared__ uint64_t s_lk[4][16][2 * FAN];   // [warp of the CTA][run head lane][key 0-15, value 0-15]
+  const int lane = lane_id();
+  const uint32_t w4 = (threadIdx.x >> 5) & 3u;
+  const Tree& t = C.t;
+  const bool mine = ((bm >> lane) & 1u) && lf < t.leaf_cap;
+  uint32_t* vp = &t.lmeta[mine ? lf : 0].version;
+  uint32_t v = 0;
+  bool got = false;
+  if (mine) {   // TX_BEGIN for every run at once (eager ownership, Alg.1:37)
+    v = atom_or_acquire(vp, 1u);
+    got = !(v & 1u);
+  }
+  __syncwarp();
+  uint64_t lo = 0, hi = 0, k0 = 0, kl = 0;
+  uint32_t nxt = NIL;
+  if (got) {   // leafvers / fences / link, and the run's first and last key (Alg.1:35-38)
+    lo = ld_cg(&t.lmeta[lf].lo);
+    hi = ld_cg(&t.lmeta[lf].hi);
+    nxt = ld_cg(&t.lmeta[lf].next);
+    k0 = C.wkey[base + lane];
+    kl = C.wkey[eL - 1];
+  }
+  const uint32_t gm = __ballot_sync(FULL, got);
+  for (uint32_t m = gm; m;) {   // the locked leaves' key + value blocks, four in flight per lane
+    int r[4];
+    uint64_t x[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      r[u] = m ? __ffs(m) - 1 : -1;
+      if (m) m &= m - 1;
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint32_t X = __shfl_sync(FULL, lf, r[u] < 0 ? 0 : r[u]);
+      x[u] = r[u] >= 0 ? widen(ld_cg(t.lkeys + (size_t)X * LSTRIDE + lane)) : 0ull;   // (values follow the keys)
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u)
+      if (r[u] >= 0) s_lk[w4][r[u]][lane] = x[u];
+  }
+  __syncwarp();
+  const bool ok = got && k0 >= lo && k0 < hi && kl < hi;   // key in range(leaf) (Alg.1:38)
+  if (got && !ok) st_release(vp, v);                         // abort, untouched (Alg.1:40-43)
+  const uint32_t om = __ballot_sync(FULL, ok);
+  // plan: every run's size after the merge -> in place (0), one leaf (1) or two
+  // (2); the plan is kept (lane r: c, mmask; smem: upserts before each leaf key)
+  __shared__ uint8_t s_ub[4][16][FAN];
+  uint32_t tout_l = 0, k_l = 1, c_l = 0, mm_l = 0;
+  for (uint32_t m = om; m; m &= m - 1) {
+    const int r = __ffs(m) - 1;
+    const uint32_t re = __shfl_sync(FULL, eL, r);
+    const uint64_t okey = lane < FAN ? s_lk[w4][r][lane] : KEY_MAX;
+    const LeafPlan L = leaf_plan(C, base + r, re, okey);
+    const uint32_t tout = L.c - __popc(L.mmask) + L.U;
+    if (lane < FAN) s_ub[w4][r][lane] = (uint8_t)L.ups_before;
+    if (lane == r) {
+      tout_l = tout;
+      k_l = L.inplace ? 0u : (tout <= FAN ? 1u : 2u);
+      c_l = L.c;
+      mm_l = L.mmask;
+    }
+  }
+  __syncwarp();
+  const uint32_t sm = __ballot_sync(FULL, ok && k_l == 2);
+  const uint32_t first = sm ? warp_alloc(&t.hdr->leaf_count, __popc(sm)) : 0u;   // one allocation for all splits
+  nid = first + __popc(sm & lanemask_lt());
+  for (uint32_t m = om; m; m &= m - 1) {   // the merges (stores only)
+    const int r = __ffs(m) - 1;
+    const uint32_t re = __shfl_sync(FULL, eL, r), X = __shfl_sync(FULL, lf, r);
+    const uint32_t kr = __shfl_sync(FULL, k_l, r), tr = __shfl_sync(FULL, tout_l, r), idr = __shfl_sync(FULL, nid, r);
+    const uint64_t okey = lane < FAN ? s_lk[w4][r][lane] : KEY_MAX;
+    if (kr == 0) {
+      leaf_overwrite(C, X, base + r, re, okey);
+      continue;
+    }
+    const uint64_t oval = lane < FAN ? s_lk[w4][r][FAN + lane] : 0ull;
+    LeafPlan L;
+    L.c = __shfl_sync(FULL, c_l, r);
+    L.mmask = __shfl_sync(FULL, mm_l, r);
+    L.ups_before = lane < FAN ? s_ub[w4][r][lane] : 0u;
+    L.inplace = false;
+    const uint64_t k1 = leaf_place(C, X, idr, base + r, re, okey, oval, L, tr, kr, nullptr, nullptr);
+    if (lane == r) ek = k1;
+  }
+  split = (sm >> lane) & 1u;
+  __syncwarp();
+  if (split) {   // the fresh leaves' meta: unreachable until X links them below
+    NodeMeta mt;
+    mt.version = 0;
+    mt.lo = ek;
+    mt.hi = hi;
+    mt.next = nxt;
+    mt.count = tout_l / 2;
+    mt.level = 0;
+    t.lmeta[nid] = mt;
+    t.lrf[nid] = t.lrf[lf];   // (inherits the RF, repaired lazily)
+  }
+  if (sm) __threadfence();    // one fence for every split of the chunk
+  __syncwarp();
+  if (ok) {
+    if (split) {
+      t.lmeta[lf].hi = ek;
+      t.lmeta[lf].next = nid;
+      t.lmeta[lf].count = tout_l - tout_l / 2;
+    } else if (k_l == 1) {
+      t.lmeta[lf].count = tout_l;
+    }
+  }
+  __syncwarp();   // every lane's stores into the leaves happen-before the releases
+  if (ok) st_release(vp, split ? v + 2u : v);   // a split: version + 1 step
+  __syncwarp();
+  ws.runs += __popc(om);
+  ws.leaf_splits += __popc(sm);
+  ws.new_leaves += __popc(sm);
+  return bm & ~om;
+}
+
+// Level-0 entries of split runs (lanes in sm, one entry each: (ek, nid)) appended
+// to the chunk's list in key (= lane) order; parent hint = the located leaf's parent.
+__device__ __forceinline__ void append_entries(const Ctx& C, SepAcc& A, uint32_t base, uint32_t sm, uint64_t ek,
+                                               uint32_t nid) {
+  if (!sm) return;
+  const int lane = lane_id();
+  if (A.base == NIL) A.base = base + __ffs(sm) - 1;
+  const uint32_t dst = A.base + A.n + __popc(sm & lanemask_lt());   // <= the run's own first write
+  if ((sm >> lane) & 1u) {
+    C.eK[0][dst] = ek;
+    C.eC[0][dst] = nid;
+    if (C.eparent) C.eparent[dst] = C.wparent[base + lane];
+  }
+  A.n += __popc(sm);
+}
 
 // ---------------------------------------------------------------- level-synchronous separators
 // Under a split storm (cfg1: every leaf splits; cfg4) per-warp upward
@@ -1159,6 +1356,36 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
       const uint32_t fastm = __ballot_sync(FULL, fast);
       ws.runs += __popc(fastm & allheads);
       uint32_t heads = allheads & ~fastm;
+#if UPD_BATCH
+      // the runs ending inside the chunk, applied together (first attempts are
+      // optimistic: not with FORCE_STM / THRESHOLD 0, whose first attempt is STM)
+      if (lsync && !ws.leaf_root && !C.force_stm && C.threshold > 0) {
+        const uint32_t later_l = allheads & ~((2u << lane) - 1u);
+        const bool cand = ((heads >> lane) & 1u) && later_l != 0;
+        const uint32_t eL = cand ? base + __ffs(later_l) - 1 : 0u;
+        const uint32_t bm = __ballot_sync(FULL, cand);
+        if (__popc(bm) >= 2) {
+          uint64_t ek = 0;
+          uint32_t nid = 0;
+          bool split = false;
+          const uint32_t fail = batched_runs(C, base, bm, eL, lf, ws, ek, nid, split);
+          const uint32_t sm = __ballot_sync(FULL, split);
+          if (!fail) {
+            append_entries(C, acc, base, sm, ek, nid);
+          } else {   // (rare) key order kept: failed runs through process_run in place
+            for (uint32_t m = bm; m && !ws.dead; m &= m - 1) {
+              const int r = __ffs(m) - 1;
+              if ((fail >> r) & 1u) {
+                process_run(C, base + r, __shfl_sync(FULL, eL, r), __shfl_sync(FULL, lf, r), ws, acc);
+              } else {
+                append_entries(C, acc, base, sm & (1u << r), ek, nid);
+              }
+            }
+          }
+          heads &= ~bm;
+        }
+      }
+#endif
       while (heads) {
         const int h = __ffs(heads) - 1;
         heads &= heads - 1;
