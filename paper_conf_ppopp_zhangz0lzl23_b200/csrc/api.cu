@@ -917,8 +917,9 @@ int eirene_submit_batch_host(eirene_handle h, const uint8_t* ops, const tkey_t* 
   CK(cudaMemcpyAsync(h->st_ops + off, ops, n, cudaMemcpyHostToDevice, h->h2d_stream));
   CK(cudaMemcpyAsync(h->st_keys + off, keys, sizeof(tkey_t) * n, cudaMemcpyHostToDevice, h->h2d_stream));
   cudaPointerAttributes pa{};
-  const bool pinned = cudaPointerGetAttributes(&pa, vals) == cudaSuccess && pa.type == cudaMemoryTypeHost &&
-                      pa.devicePointer != nullptr;
+  static const bool vals_copy = std::getenv("EIRENE_VALS_COPY") != nullptr;   // A/B: always copy the values
+  const bool pinned = !vals_copy && cudaPointerGetAttributes(&pa, vals) == cudaSuccess &&
+                      pa.type == cudaMemoryTypeHost && pa.devicePointer != nullptr;
   cudaGetLastError();   // (clear a pageable-pointer query error, if any)
   const tkey_t* vsrc;
   tkey_t* vstage = nullptr;

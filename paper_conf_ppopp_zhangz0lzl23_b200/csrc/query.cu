@@ -79,7 +79,11 @@ __device__ __forceinline__ int slot16(const tkey_t* __restrict__ line, uint64_t 
 }
 
 #ifndef EIRENE_QCOOP
-#define EIRENE_QCOOP 0   // A/B: warp-cooperative leaf search (KPL lanes read one leaf's key line)
+#ifdef EIRENE_KEY32
+#define EIRENE_QCOOP 0   // (32-bit keys: a leaf line is two sectors; A/B pending)
+#else
+#define EIRENE_QCOOP 1   // warp-cooperative leaf search (r3h: cfg2 query 56.8 -> 54.6 us; 0 = per-lane line loads)
+#endif
 #endif
 // Warp-cooperative leaf search: the 32 lanes' leaves are read KPL lanes per
 // leaf line (each lane one 32 B sector), 32/KPL leaves per 256-bit load

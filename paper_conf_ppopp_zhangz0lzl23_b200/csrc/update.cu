@@ -1297,11 +1297,20 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
     // Under a split storm a chunk's cost varies with its leaf runs and splits:
     // chunks are handed out dynamically (a warp takes the next one when done) so
     // the level-0 phase ends at the average warp's time, not the unluckiest one's
+    // (one chunk per claim: claiming 4 at a time, r3i, made cfg4's update 513 -> 532 us -- the
+    // tail imbalance costs more than the claims' atomics on one address)
+    const uint32_t G = 1u;
+    uint32_t c_next = 0, c_end = 0;
     auto next_chunk = [&]() -> uint32_t {
-      uint32_t c = 0;
-      if (lane == 0) c = atomicAdd(&C.ctl->uchunk, 1u);
-      return __shfl_sync(FULL, c, 0);
+      if (c_next == c_end) {
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(&C.ctl->uchunk, G);
+        c_next = __shfl_sync(FULL, c, 0);
+        c_end = c_next + G;
+      }
+      return c_next++;
     };
+    uint32_t lvl0 = 0;   // this warp's level-0 entries (one atomic per warp, not per chunk)
     for (uint32_t chunk = lsync ? next_chunk() : gw; chunk * CH < nw;
          chunk = lsync ? next_chunk() : chunk + nwarps) {
       const uint32_t base = chunk * CH;
@@ -1413,7 +1422,7 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
       if (lsync) {
         if (lane == 0) {
           C.slots[0][chunk] = make_uint2(acc.base == NIL ? 0u : acc.base, acc.n);
-          if (acc.n) atomicAdd(&C.ctl->lvl_ent[0], acc.n);
+          lvl0 += acc.n;
         }
       } else if (acc.n && !ws.dead) {
         insert_up(C, 0, acc.base, acc.n, ws);
@@ -1421,6 +1430,7 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
       acc = SepAcc{};
     }
     if (lsync) {
+      if (lane == 0 && lvl0) atomicAdd(&C.ctl->lvl_ent[0], lvl0);   // (read after the grid barrier)
       uint32_t gen = 0;
       levels_up(C, nchunks, gw, nwarps, gen, ws);
     }
