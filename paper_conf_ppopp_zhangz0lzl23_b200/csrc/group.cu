@@ -72,6 +72,7 @@ struct GSmem {
   uint32_t h_cnt[G_WARPS], h_lw[G_WARPS], h_lp[G_WARPS];   // hot_pass1 per-warp results
   uint64_t hk;                 // split-off hot key of an oversized group
   unsigned long long prof_t[2];  // EIRENE_GROUP_PROF timestamps (diagnostic)
+  unsigned long long prof_l[4];  // ... inside l2_sort: range pass, split pass, rest sorted
   uint32_t* hot_bits;          // its timestamp bitmap slot (null: none free)
   // hot_run_sort: timestamp-bucket counters, provisional payloads, the run's other keys
   uint32_t tcnt[SB_N + 1];
@@ -736,6 +737,9 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
     S.w_nw[warp] = n2;
   }
   key_range(mn, mx, S);   // (its barriers publish the per-warp counts)
+#ifdef EIRENE_GROUP_PROF_BUILD
+  if (tid == 0) S.prof_l[0] = gtime_ns();
+#endif
   n0 = n1 = n2 = 0;
   for (int w = 0; w < G_WARPS; ++w) {
     n0 += S.w_nh[w];
@@ -825,9 +829,15 @@ __device__ int l2_sort(uint64_t* ks, uint32_t* ps, uint64_t* kd, uint32_t* pd, u
       if (my_lp) atomicMax(&S.hot_lastp, my_lp);
     }
     __syncthreads();
+#ifdef EIRENE_GROUP_PROF_BUILD
+    if (tid == 0) S.prof_l[1] = gtime_ns();
+#endif
     const uint32_t o = S.r_nh, h = S.r_lw, lo = S.r_nw;
     if (o > 1) smem_sort(S.k, S.p, o, tsbits, S);
     __syncthreads();
+#ifdef EIRENE_GROUP_PROF_BUILD
+    if (tid == 0) S.prof_l[2] = gtime_ns();
+#endif
     if (bits) {   // SPLIT: the rest stays sorted in S.k / S.p, hk in the bitmap
       if (tid == 0) {
         S.r_nh = o;
@@ -1554,8 +1564,11 @@ __global__ void __launch_bounds__(G_THREADS, 2) group_kernel(GroupArgs g) {
   if ((g.prof & 1) && tid == 0) {
     const unsigned long long tp4 = gtime_ns();
     if (tp4 - tp0 > 20000)
-      printf("[group prof] ticket %u cnt %u mode %d sort %.1f sweep1 %.1f lookback %.1f emit %.1f us hot2 %.1f\n", b,
-             cnt, mode, (tp1 - tp0) * 1e-3, (tp2 - tp1) * 1e-3, (tp3 - tp2) * 1e-3, (tp4 - tp3) * 1e-3,
+      printf("[group prof] ticket %u cnt %u mode %d sort %.1f (range %.1f split %.1f rest %.1f, rest %u hot %u) "
+             "sweep1 %.1f lookback %.1f emit %.1f us hot2 %.1f\n", b,
+             cnt, mode, (tp1 - tp0) * 1e-3, small ? 0.0 : (S.prof_l[0] - tp0) * 1e-3,
+             mode == 2 ? (S.prof_l[1] - S.prof_l[0]) * 1e-3 : 0.0, mode == 2 ? (S.prof_l[2] - S.prof_l[1]) * 1e-3 : 0.0,
+             sp_o, sp_h, (tp2 - tp1) * 1e-3, (tp3 - tp2) * 1e-3, (tp4 - tp3) * 1e-3,
              mode == 2 ? (S.prof_t[1] - S.prof_t[0]) * 1e-3 : 0.0);
   }
 #else
