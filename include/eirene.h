@@ -183,7 +183,7 @@ int eirene_submit_batch(eirene_handle h, const uint8_t* ops_dev, const eirene_ke
                         eirene_stream_t stream, uint64_t* ticket);
 
 /* Same batch from HOST buffers.  ops and keys are copied host->device into
- * handle-owned double-buffered staging on the handle's copy stream (which
+ * handle-owned triple-buffered staging on the handle's copy stream (which
  * overlaps the previous batch's kernels); the pipeline runs on `stream`; the
  * results are copied device->host on the handle's d2h stream.  If vals_host is
  * pinned (page-locked, device-mapped under UVA) it is not copied: the

@@ -1,12 +1,17 @@
 // api.cu -- the C ABI (include/eirene.h): handle, pools, batch sequencing.
 //
-// A batch (Alg.1:1-7) is a fixed chain of kernels on the caller's stream:
-//   memset(batch scratch) -> sort upsweep + 8 digit passes (Alg.1:10)
-//   -> combine (Alg.1:11) -> partition (Alg.1:3) -> query + write-locate
-//   (Alg.1:4) -> update (Alg.1:5) -> RESULT_CAL (Alg.1:6) -> finalize
-// followed by an async copy of the batch's device scalars into a pinned ring
-// slot and an event; eirene_results() waits on that event.  No allocation and
-// no host synchronisation happen inside submit.
+// A batch (Alg.1:1-7) is one CUDA graph replay of five kernels on the
+// caller's stream:
+//   set_args (zero the control region, publish the batch's pointers)
+//   -> bsort_dist (key-range bucket distribution, Alg.1:10)
+//   -> group (per-group smem sort + combine + partition, Alg.1:10-11, 3)
+//   -> query (Alg.1:4, with the write locate and RESULT_CAL of short segments)
+//   -> update (Alg.1:5, then the result phase: long segments, deferred hot
+//      keys, the BatchCtl publish into a device ring slot).
+// eirene_results() waits on the batch's event and fetches its BatchCtl off the
+// pipeline.  No allocation and no host synchronisation happen inside submit.
+// Graphs are captured per size bucket; pipelined handles (EIRENE_F_PIPELINE)
+// split each batch into a front and a back graph on two streams (§7.2).
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>

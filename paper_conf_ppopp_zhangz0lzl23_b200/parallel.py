@@ -128,6 +128,9 @@ class ShardedEirene:
         rvals = torch.empty(cap, dtype=torch.uint64, device=dev)
         nrecv, invalid = self.engine.route_pull(rops, rkeys, rvals)
         if invalid:   # every rank saw every source's flag: all reject the global batch
+            # (a barrier still: no source may push the next batch into an arena before its owner has read
+            # this batch's slots)
+            self._barrier()
             return ShardedTicket(self, None, None, n, rejected=-1)
         rres = torch.empty(max(nrecv, 1), dtype=torch.uint64, device=dev)
         status = torch.zeros(1, dtype=torch.int32, device=dev)

@@ -111,3 +111,23 @@ def test_probe_gather_argument_checks(libpath):
     assert L.eirene_probe_gather(ctypes.c_void_p((1 << 20) + 8), 1 << 20, 16, 0, 1, None) == _ffi.EIRENE_EINVAL
     assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 1 << 20, 16, 4, 1, None) == _ffi.EIRENE_EINVAL   # kind
     assert L.eirene_probe_gather(ctypes.c_void_p(1 << 20), 3 << 20, 16, 0, 1, None) == _ffi.EIRENE_EINVAL   # not 2^k
+
+
+def test_fused_routing_argument_checks_without_gpu(libpath):
+    """The fused-routing calls reject a null handle or null outputs on the host (EINVAL)
+    before touching the device; the IPC handle size is the header's."""
+    L = _ffi.lib()
+    addr = ctypes.c_void_p()
+    n = ctypes.c_uint32()
+    inv = ctypes.c_uint32()
+    E = _ffi.EIRENE_EINVAL
+    assert L.eirene_route_arena_create(None, 2, 0, 1024, ctypes.byref(addr), None) == E
+    assert L.eirene_route_arena_open_ipc(None, None, ctypes.byref(addr)) == E
+    assert L.eirene_route_arena_connect(None, None) == E
+    assert L.eirene_route_push(None, None, None, None, 0, None, None, None) == E
+    assert L.eirene_route_pull(None, None, None, None, 0, ctypes.byref(n), ctypes.byref(inv), None) == E
+    assert L.eirene_route_push_results(None, None, None) == E
+    assert L.eirene_route_unpermute_arena(None, None, 0, None, None) == E
+    with open(_ffi.HEADER) as f:
+        assert "#define EIRENE_IPC_HANDLE_BYTES 64" in f.read()
+    assert _ffi.EIRENE_IPC_HANDLE_BYTES == 64

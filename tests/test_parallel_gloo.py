@@ -90,6 +90,97 @@ class OracleEngine:
         return torch.from_numpy(k), torch.from_numpy(v)
 
 
+class OracleArenaEngine(OracleEngine):
+    """OracleEngine plus a CPU stand-in of the fused-routing arena calls (include/eirene.h contract): each rank's
+    arena is a POSIX shared-memory segment {P x (count, invalid, start, epoch) u32, cap result u64, P x cap x 3
+    record u64}; its name plays the IPC handle, so the peers' "pushes" are plain stores into it."""
+
+    def __init__(self):
+        super().__init__()
+        self.views = {}
+        self.shms = []
+        self.epoch = 0
+
+    def _view(self, shm, P, cap):
+        buf = shm.buf
+        cnt = np.ndarray((P, 4), np.uint32, buf, 0)
+        res = np.ndarray((cap,), np.uint64, buf, 1024)
+        rec = np.ndarray((P, cap, 3), np.uint64, buf, 1024 + 8 * cap)
+        return cnt, res, rec
+
+    def route_arena_create(self, P, rank, cap):
+        from multiprocessing import shared_memory
+        shm = shared_memory.SharedMemory(create=True, size=1024 + 8 * cap + 24 * P * cap)
+        self.shms.append(shm)
+        self.P, self.me, self.cap = P, rank, cap
+        np.ndarray((1024,), np.uint8, shm.buf, 0)[:] = 0
+        key = len(self.views) + 1
+        self.views[key] = self._view(shm, P, cap)
+        return key, shm.name.encode().ljust(64, b"\0")
+
+    def route_arena_open_ipc(self, handle):
+        from multiprocessing import shared_memory
+        shm = shared_memory.SharedMemory(name=handle.rstrip(b"\0").decode())
+        self.shms.append(shm)
+        key = len(self.views) + 1
+        self.views[key] = self._view(shm, self.P, self.cap)
+        return key
+
+    def route_arena_connect(self, addrs):
+        self.peers = [self.views[a] for a in addrs]
+        self.own = self.peers[self.me]
+
+    def route_push(self, ops, keys, vals, splitters, perm):
+        P = self.P
+        o, k, v, pm, counts = CpuRouter().route_partition(ops, keys, vals, splitters, P)
+        bad = np.zeros(1, np.int32)
+        CpuRouter().route_partition(ops, keys, vals, splitters, P, invalid=torch.from_numpy(bad))
+        perm.copy_(pm)
+        self.epoch += 1
+        start = np.concatenate([[0], np.cumsum(counts.numpy())])
+        for d in range(P):
+            c = int(counts[d])
+            rec = self.peers[d][2]
+            rec[self.me, :c, 0] = k.numpy()[start[d]:start[d] + c]
+            rec[self.me, :c, 1] = v.numpy()[start[d]:start[d] + c]
+            rec[self.me, :c, 2] = o.numpy()[start[d]:start[d] + c]
+            self.peers[d][0][self.me] = (c, bad[0], start[d], self.epoch)
+
+    def route_pull(self, ops, keys, vals):
+        cnt, _, rec = self.own
+        assert np.all(cnt[:, 3] == self.epoch), "a peer's push never arrived"
+        if cnt[:, 1].any():
+            return int(cnt[:, 0].sum()), 1
+        parts = [rec[s, :cnt[s, 0]] for s in range(self.P)]
+        r = np.concatenate(parts) if parts else np.zeros((0, 3), np.uint64)
+        n = r.shape[0]
+        keys[:n].copy_(torch.from_numpy(r[:, 0].copy()))
+        vals[:n].copy_(torch.from_numpy(r[:, 1].copy()))
+        ops[:n].copy_(torch.from_numpy(r[:, 2].astype(np.uint8)))
+        return n, 0
+
+    def route_push_results(self, results):
+        cnt = self.own[0]
+        off = 0
+        for s in range(self.P):
+            c, st = int(cnt[s, 0]), int(cnt[s, 2])
+            self.peers[s][1][st:st + c] = results.numpy()[off:off + c]
+            off += c
+
+    def route_unpermute_arena(self, perm, out):
+        res = np.empty(perm.numel(), np.uint64)
+        res[perm.numpy()] = self.own[1][:perm.numel()]
+        out.copy_(torch.from_numpy(res))
+        return out
+
+    def close_arenas(self):
+        for shm in self.shms[1:]:
+            shm.close()
+        if self.shms:
+            self.shms[0].close()
+            self.shms[0].unlink()
+
+
 def _free_port():
     s = socket.socket()
     s.bind(("127.0.0.1", 0))
@@ -98,7 +189,7 @@ def _free_port():
     return p
 
 
-def _worker(rank, world, port, outdir):
+def _worker(rank, world, port, outdir, fused=False):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), RANK=str(rank), WORLD_SIZE=str(world))
     dist.init_process_group("gloo", rank=rank, world_size=world)
     try:
@@ -107,7 +198,8 @@ def _worker(rank, world, port, outdir):
         from paper_conf_ppopp_zhangz0lzl23_b200.parallel import ShardedEirene
         w = W.Workload(2, tree=1 << 12, batch=world * 1024,
                        fracs={W.QUERY: 0.5, W.UPDATE: 0.2, W.INSERT: 0.2, W.DELETE: 0.1})
-        sh = ShardedEirene(w.keys, w.vals, max_batch=1024, device="cpu", engine=OracleEngine(), router=CpuRouter())
+        eng = OracleArenaEngine() if fused else OracleEngine()
+        sh = ShardedEirene(w.keys, w.vals, max_batch=1024, device="cpu", engine=eng, router=CpuRouter(), fused=fused)
         ref = oracle.MapOracle()
         ref.load(w.keys, w.vals)
         bad = 0
@@ -137,14 +229,20 @@ def _worker(rank, world, port, outdir):
         untouched = np.array_equal(k2.numpy(), k.numpy()) and np.array_equal(v2.numpy(), v.numpy())
         with open(os.path.join(outdir, f"r{rank}.txt"), "w") as f:
             f.write(f"{bad} {int(same)} {st['status']} {int(untouched)}\n")
+        dist.barrier()
+        if fused:
+            eng.close_arenas()
     finally:
         dist.destroy_process_group()
 
 
-def test_sharded_two_ranks_gloo():
+@pytest.mark.parametrize("fused", [False, True])
+def test_sharded_two_ranks_gloo(fused):
+    """fused=True: the fused push over the ranks' arenas (ShardedEirene._submit_fused: push, barrier, pull,
+    shard batch, results pushed back, status all-reduce as the second barrier, unpermute)."""
     world = 2
     with tempfile.TemporaryDirectory() as d:
-        mp.spawn(_worker, args=(world, _free_port(), d), nprocs=world, join=True)
+        mp.spawn(_worker, args=(world, _free_port(), d, fused), nprocs=world, join=True)
         for r in range(world):
             bad, same, st, untouched = open(os.path.join(d, f"r{r}.txt")).read().split()
             assert bad == "0", f"rank {r}: {bad} results differ from the oracle"
