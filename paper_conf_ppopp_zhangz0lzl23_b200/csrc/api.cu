@@ -12,6 +12,7 @@
 // pipeline.  No allocation and no host synchronisation happen inside submit.
 // Graphs are captured per size bucket; pipelined handles (EIRENE_F_PIPELINE)
 // split each batch into a front and a back graph on two streams (§7.2).
+#include <atomic>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -218,6 +219,7 @@ struct eirene_tree {
   uint64_t launches = 0;
   size_t device_bytes = 0;
   std::vector<void*> allocs;
+  bool counted_pipelined = false;   // counted in g_pipelined_handles (cooperative grid launches while > 0)
   // fused routing (eirene_route_arena_*): this rank's receive arena, the P
   // peers' arenas (IPC-mapped or, in one process, plain device pointers)
   struct Arena {
@@ -258,6 +260,20 @@ bool pdl_enabled() {
     return e ? std::atoi(e) != 0 : false;
   }();
   return on;
+}
+// EIRENE_COOP=0/1 (read once per process): cooperative launches of the
+// grid-barrier kernels (default off: eirene_internal.cuh, launch_k)
+// (also on while any pipelined handle exists in the process: its front's
+// distribution kernel and its back's update kernel run concurrently on two
+// streams, and two plain grid-barrier kernels could each hold the SMs the
+// other needs)
+std::atomic<int> g_pipelined_handles{0};
+bool coop_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("EIRENE_COOP");
+    return e ? std::atoi(e) != 0 : false;
+  }();
+  return on || g_pipelined_handles.load(std::memory_order_relaxed) > 0;
 }
 }  // namespace eirene
 
@@ -529,6 +545,10 @@ int eirene_create(const eirene_config* cfg, eirene_handle* out) {
   }
   h->up.threshold = cfg->retry_threshold;
   h->up.flags = cfg->flags;
+  if (cfg->flags & EIRENE_F_PIPELINE) {
+    eirene::g_pipelined_handles.fetch_add(1);
+    h->counted_pipelined = true;
+  }
   *out = h;
   return EIRENE_OK;
 }
@@ -565,6 +585,7 @@ int eirene_destroy(eirene_handle h) {
     if (h->comp_done[s]) cudaEventDestroy(h->comp_done[s]);
     if (h->comp_ev[s]) cudaEventDestroy(h->comp_ev[s]);
   }
+  if (h->counted_pipelined) eirene::g_pipelined_handles.fetch_sub(1);
   for (void* p : h->ar.opened) cudaIpcCloseMemHandle(p);
   if (h->ar.h_cnt) cudaFreeHost(h->ar.h_cnt);
   for (void* p : h->allocs) cudaFree(p);

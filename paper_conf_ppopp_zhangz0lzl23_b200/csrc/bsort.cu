@@ -491,8 +491,8 @@ void launch_bucket_sort(const BatchArgs* A, uint32_t n, uint64_t key_lo, uint64_
     // fused single launch; slices of whole 512-request rows per CTA
     const uint32_t rows = (n + D_THREADS - 1) / D_THREADS;
     const uint32_t per_cta = ((rows + grid - 1) / grid) * D_THREADS;
-    // cooperative launch: the grid barrier needs every CTA co-resident, which a plain
-    // launch does not guarantee when other kernels share the device
+    // one resident wave with a grid barrier: every CTA co-resident (a cooperative
+    // launch only with EIRENE_COOP=1; see launch_k for why a plain launch is safe here)
     launch_k(bsort_dist_kernel, dim3(grid), dim3(D_THREADS), sizeof(DSmem), st, true, true, A, n, G, per_cta, key_lo, key_hi,
              bshift, b.bcount, b.gstart, b.cursor, b.kA, b.pA, ctl);
     *launches += 1;

@@ -434,6 +434,7 @@ __device__ __forceinline__ bool headroom_ok(const Tree& t, uint32_t nw) {
 __device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
 __device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
 bool pdl_enabled();
+bool coop_enabled();
 template <typename... KArgs, typename... Args>
 cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st, bool pdl,
                      bool coop, Args&&... args) {
@@ -449,6 +450,17 @@ cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem,
     at[na].val.programmaticStreamSerializationAllowed = 1;
     ++na;
   }
+  // The two grid-barrier kernels (distribution, update) run grids sized to the
+  // occupancy calculator's co-resident capacity.  By default they are launched
+  // WITHOUT the cooperative attribute (r3o: cfg2 9.03 -> 9.24 G req/s, the
+  // cooperative launch cost ~2.5 us per batch): every CTA of such a grid fits
+  // on the device at once, and no kernel that may share the device with it (the
+  // library's own: a pipelined front, routing kernels, NCCL's -- stream-ordered
+  // around it) waits on it, so every CTA is eventually scheduled and the
+  // barrier completes.  A foreign kernel holding SMs indefinitely would make the
+  // barrier wait; the device watchdog then ends the batch with EINTERNAL instead
+  // of hanging.  EIRENE_COOP=1 restores cooperative launches (shared devices).
+  if (coop && !coop_enabled()) coop = false;
   if (coop) {
     at[na].id = cudaLaunchAttributeCooperative;
     at[na].val.cooperative = 1;

@@ -1514,7 +1514,7 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
   if (serial) {
     update_kernel<<<1, 32, 0, st>>>(C, r);
   } else {
-    if (C.slots[0]) {   // grid barriers: cooperative launch (co-residency guaranteed)
+    if (C.slots[0]) {   // grid barriers: a resident-sized grid (cooperative only with EIRENE_COOP=1, launch_k)
       launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, true, C, r);
     } else {
       launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, false, C, r);
