@@ -342,7 +342,15 @@ __device__ __forceinline__ void query_end(BatchCtl* ctl, const BatchArgs* A, con
 // The graph-mode variant with the conditional update node (EIRENE_COND) is a
 // kernel of its own: a kernel that references the device graph API is not
 // profiled by ncu inside a graph, and the default path should be.
-__global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restrict__ qkey,
+#ifndef EIRENE_QMINB
+#ifdef EIRENE_KEY32
+#define EIRENE_QMINB 8   // resident CTAs per SM the query kernel's registers are fitted to (8: 32 registers)
+#else
+#define EIRENE_QMINB 6   // (64-bit keys, cooperative leaf search: 40 registers; r3r: 8 / 6 / 5 / 4 CTAs per SM ->
+                         // cfg2 9.20 / 9.26 / 9.12 / 9.13 G req/s, cfg3 query 43.4 -> 40.9 us at 6)
+#endif
+#endif
+__global__ void __launch_bounds__(256, EIRENE_QMINB) query_kernel(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
@@ -359,7 +367,7 @@ __global__ void __launch_bounds__(256, 8) query_kernel(const uint64_t* __restric
   pdl_trigger();
   query_body(qkey, qseg, wkey, wseg, wop, wval, wleaf, wslot, wparent, old, spay, pinfo, istart, longseg, A, t, ctl);
 }
-__global__ void __launch_bounds__(256, 8) query_cond_kernel(const uint64_t* __restrict__ qkey,
+__global__ void __launch_bounds__(256, EIRENE_QMINB) query_cond_kernel(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
@@ -713,8 +721,8 @@ __global__ void __launch_bounds__(256, 4) range_kernel(uint32_t n, const uint64_
 void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const BatchArgs* A, Tree t, BatchCtl* ctl,
                   int num_sms, uint32_t flags, uint32_t iter_rgs, cudaGraphConditionalHandle cond, int use_cond,
                   cudaStream_t st, int* launches) {
-  // one resident wave: 8 CTAs of 256 threads per SM at <= 32 registers
-  int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * 8u);
+  // one resident wave: EIRENE_QMINB (8) CTAs of 256 threads per SM at <= 32 registers
+  int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * (uint32_t)EIRENE_QMINB);
   if (blocks < 1) blocks = 1;
   if (flags & EIRENE_F_ITERWARP) {
     // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
