@@ -631,7 +631,7 @@ def run_ours(args):
                "h2d_bytes_per_step": int(world * batch_n * 17), "d2h_bytes_per_step": int(world * batch_n * 8),
                "steps": n_e, "path": "ShardedEirene.submit_host on every rank: pinned H2D of the rank's slice, "
                                      + ("fused push routing (partition kernel storing into the peers' arenas, "
-                                        "results pushed back) " if args.route == "fused" else
+                                        "results pushed back) " if sh.fused else
                                         "routing + NCCL exchanges ") + "+ shard batch, D2H of the results slice (one "
                                      "stream per rank); max over ranks"}
 
@@ -810,8 +810,10 @@ def run_ours(args):
                                    + (f", range length {cap} (first {cap} pairs returned)" if cap else ""),
                        "cfg": cfg, "global_batch": batch_n * world,
                        "parallelism": (f"key-range shards x{world}, "
-                                       + ("fused push over peer memory" if args.route == "fused"
-                                          else "NCCL all-to-all")) if world > 1 else "single GPU",
+                                       + ("fused push over peer memory" if sh is not None and sh.fused
+                                          else "NCCL all-to-all" + (f" (fused push unavailable: {sh.route_error})"
+                                                                    if sh is not None and getattr(sh, "route_error", None)
+                                                                    else ""))) if world > 1 else "single GPU",
                        "l2": "distinct input/result buffers per step (steps x 25 MiB >> 126 MB L2); "
                              "inner levels stay L2-resident across batches (steady state)"},
             "batch_ms": spread(dev_batch_ms, "device %globaltimer: start of the batch's first kernel to the end of "

@@ -157,7 +157,10 @@ __device__ void bitonic_run(uint32_t lo, uint32_t m, int t, int nt, GSmem& S) {
 // Larger sub-buckets (hot keys: a key's requests always share one) are
 // sorted by a bitonic network, one warp per sub-bucket up to WARP_SB
 // requests, the whole CTA above, so no distribution costs O(m^2).
-constexpr uint32_t FAST_SB = 32;
+#ifndef GROUP_FAST_SB
+#define GROUP_FAST_SB 32   // A/B builds: -DGROUP_FAST_SB=n
+#endif
+constexpr uint32_t FAST_SB = GROUP_FAST_SB;
 #ifndef GROUP_WARP_SB
 #define GROUP_WARP_SB 256   // A/B builds: -DGROUP_WARP_SB=n; cfg3 1024 -> 256: 3.43 -> 3.64 Greq/s
 #endif

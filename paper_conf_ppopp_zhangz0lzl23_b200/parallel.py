@@ -93,7 +93,21 @@ class ShardedEirene:
         self.splitters = torch.from_numpy(self.splitters_np if self.world > 1 else np.zeros(1, np.uint64)).to(self.device)
         self.fused = fused
         if fused:
-            self._connect_arenas()
+            # every rank must map every peer's arena; if any rank cannot (no CUDA IPC between the processes,
+            # no peer access), ALL ranks take the NCCL exchange instead -- decided together
+            ok = 1
+            try:
+                self._connect_arenas()
+            except Exception as e:   # noqa: BLE001 -- reported, and agreed on below
+                ok = 0
+                self.route_error = f"{type(e).__name__}: {e}"
+            if self.world > 1:
+                flag = torch.tensor([ok], dtype=torch.int32,
+                                    device=self.device if self.device.type == "cuda" else "cpu")
+                dist.all_reduce(flag, op=dist.ReduceOp.MIN, group=self.group)
+                ok = int(flag.item())
+            if not ok:
+                self.fused = False
 
     def _connect_arenas(self):
         """Fused routing: every rank's receive arena, mapped into every other rank's
@@ -103,7 +117,7 @@ class ShardedEirene:
         handles = [ipc]
         if self.world > 1:
             handles = [None] * self.world
-            dist.all_gather_object(handles, ipc, group=self.group)
+            dist.all_gather_object(handles, ipc, group=self.group)   # (collective: before anything can fail)
         addrs = [addr if r == self.rank else self.engine.route_arena_open_ipc(handles[r]) for r in range(self.world)]
         self.engine.route_arena_connect(addrs)
         self._tok = torch.zeros(1, dtype=torch.int32, device=self.device)
