@@ -742,6 +742,7 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
 }
 
 
+constexpr uint32_t UPD_LSYNC_CH = 16;   // writes per level-0 chunk under a split storm (r3t: 32 slower on cfg1)
 #ifndef UPD_BATCH
 #define UPD_BATCH 1   // A/B: 0 = every leaf run of a chunk through process_run, one after the other
 #endif
@@ -758,7 +759,7 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
 // h of a split run: ek = the new leaf's first key, nid = its id.
 __device__ uint32_t batched_runs(const Ctx& C, uint32_t base, uint32_t bm, uint32_t eL, uint32_t lf, WarpStats& ws,
                                  uint64_t& ek, uint32_t& nid, bool& split) {
-  __shared__ uint64_t s_lk[4][16][2 * FAN];   // [warp of the CTA][run head lane][key 0-15, value 0-15]
+  __shared__ uint64_t s_lk[4][UPD_LSYNC_CH][2 * FAN];   // [warp of the CTA][run head lane][key 0-15, value 0-15]
   const int lane = lane_id();
   const uint32_t w4 = (threadIdx.x >> 5) & 3u;
   const Tree& t = C.t;
@@ -804,7 +805,7 @@ __device__ uint32_t batched_runs(const Ctx& C, uint32_t base, uint32_t bm, uint3
   const uint32_t om = __ballot_sync(FULL, ok);
   // plan: every run's size after the merge -> in place (0), one leaf (1) or two
   // (2); the plan is kept (lane r: c, mmask; smem: upserts before each leaf key)
-  __shared__ uint8_t s_ub[4][16][FAN];
+  __shared__ uint8_t s_ub[4][UPD_LSYNC_CH][FAN];
   uint32_t tout_l = 0, k_l = 1, c_l = 0, mm_l = 0;
   for (uint32_t m = om; m; m &= m - 1) {
     const int r = __ffs(m) - 1;
@@ -1291,7 +1292,7 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
   // writes per chunk: a warp takes one chunk at a time and its leaf runs one
   // after the other; under a split storm (lsync) each run is a long dependent
   // chain, so chunks of 16 halve the runs a warp applies in a row
-  const uint32_t CH = lsync ? 16u : 32u;
+  const uint32_t CH = lsync ? (uint32_t)UPD_LSYNC_CH : 32u;
   const uint32_t nchunks = (nw + CH - 1) / CH;
   if (C.regroup) {
     // Under a split storm a chunk's cost varies with its leaf runs and splits:
@@ -1370,8 +1371,9 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
       // optimistic: not with FORCE_STM / THRESHOLD 0, whose first attempt is STM)
       if (lsync && !ws.leaf_root && !C.force_stm && C.threshold > 0) {
         const uint32_t later_l = allheads & ~((2u << lane) - 1u);
-        const bool cand = ((heads >> lane) & 1u) && later_l != 0;
+        bool cand = ((heads >> lane) & 1u) && later_l != 0;
         const uint32_t eL = cand ? base + __ffs(later_l) - 1 : 0u;
+        cand = cand && eL - (base + lane) <= (uint32_t)FAN;   // <= 16 writes: at most two leaves (batched_runs)
         const uint32_t bm = __ballot_sync(FULL, cand);
         if (__popc(bm) >= 2) {
           uint64_t ek = 0;

@@ -143,6 +143,26 @@ def test_cfg1_inserts_split_every_leaf(dev):
     assert rc == 0 and nk == ref.size()
 
 
+def test_cfg4_full_size_growth(dev):
+    """cfg4 at full size, as the bench runs it: a 2^20-key tree grown by four 2^20-request batches of 90% insert /
+    10% delete (toward 2^22 keys: split storms on every batch, level-synchronous propagation, batched leaf runs);
+    every result and the final scan bit-exact, invariants intact."""
+    w = W.Workload(4)
+    C = W.CONFIGS[4]
+    t = make_tree(dev, w.keys, w.vals, max_keys=C["tree"] + C["per_tree"] * C["batch"] + (1 << 12),
+                  max_batch=C["batch"])
+    ref = oracle.MapOracle(); ref.load(w.keys, w.vals)
+    splits = 0
+    for b in range(C["per_tree"]):
+        ops, keys, vals = w.batch_arrays(b)
+        st = run_and_compare(t, ref, ops, keys, vals, dev, check_scan=b + 1 == C["per_tree"])
+        splits += st["leaf_splits"]
+    assert splits > C["batch"] // 8   # (the storm did happen)
+    rc, nk = t.check_invariants()
+    assert rc == 0 and nk == ref.size()
+    t.close()
+
+
 @pytest.mark.parametrize("regroup", [True, False])
 @pytest.mark.parametrize("threshold,force", [(4, False), (0, False), (1, False), (1 << 30, False), (4, True)])
 def test_structural_mix_threshold_and_regroup(dev, regroup, threshold, force):
