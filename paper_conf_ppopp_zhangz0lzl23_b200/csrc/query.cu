@@ -342,6 +342,9 @@ __device__ __forceinline__ void query_end(BatchCtl* ctl, const BatchArgs* A, con
 // The graph-mode variant with the conditional update node (EIRENE_COND) is a
 // kernel of its own: a kernel that references the device graph API is not
 // profiled by ncu inside a graph, and the default path should be.
+#ifndef EIRENE_QTHREADS
+#define EIRENE_QTHREADS 256   // query-kernel CTA size (A/B builds: 768 with EIRENE_QMINB=2)
+#endif
 #ifndef EIRENE_QMINB
 #ifdef EIRENE_KEY32
 #define EIRENE_QMINB 8   // resident CTAs per SM the query kernel's registers are fitted to (8: 32 registers)
@@ -350,7 +353,7 @@ __device__ __forceinline__ void query_end(BatchCtl* ctl, const BatchArgs* A, con
                          // cfg2 9.20 / 9.26 / 9.12 / 9.13 G req/s, cfg3 query 43.4 -> 40.9 us at 6)
 #endif
 #endif
-__global__ void __launch_bounds__(256, EIRENE_QMINB) query_kernel(const uint64_t* __restrict__ qkey,
+__global__ void __launch_bounds__(EIRENE_QTHREADS, EIRENE_QMINB) query_kernel(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
@@ -367,7 +370,7 @@ __global__ void __launch_bounds__(256, EIRENE_QMINB) query_kernel(const uint64_t
   pdl_trigger();
   query_body(qkey, qseg, wkey, wseg, wop, wval, wleaf, wslot, wparent, old, spay, pinfo, istart, longseg, A, t, ctl);
 }
-__global__ void __launch_bounds__(256, EIRENE_QMINB) query_cond_kernel(const uint64_t* __restrict__ qkey,
+__global__ void __launch_bounds__(EIRENE_QTHREADS, EIRENE_QMINB) query_cond_kernel(const uint64_t* __restrict__ qkey,
                                                         const uint32_t* __restrict__ qseg,
                                                         const uint64_t* __restrict__ wkey,
                                                         const uint32_t* __restrict__ wseg,
@@ -722,7 +725,8 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
                   int num_sms, uint32_t flags, uint32_t iter_rgs, cudaGraphConditionalHandle cond, int use_cond,
                   cudaStream_t st, int* launches) {
   // one resident wave: EIRENE_QMINB (8) CTAs of 256 threads per SM at <= 32 registers
-  int blocks = (int)std::min<uint32_t>((n + 255) / 256, (uint32_t)num_sms * (uint32_t)EIRENE_QMINB);
+  int blocks = (int)std::min<uint32_t>((n + EIRENE_QTHREADS - 1) / EIRENE_QTHREADS,
+                                       (uint32_t)num_sms * (uint32_t)EIRENE_QMINB);
   if (blocks < 1) blocks = 1;
   if (flags & EIRENE_F_ITERWARP) {
     // <= 64 registers (the RG loop keeps the buffer and the lane's state): 4 resident CTAs per SM
@@ -737,10 +741,10 @@ void launch_query(uint32_t n, const CombBufs& c, const uint32_t* spay, const Bat
       launch_k(query_iterwarp_kernel, g, dim3(256), 0, st, true, false, c.qkey, c.wkey, c.wparent, io, A, t, ctl,
                iter_rgs, stats);
   } else if (use_cond) {
-    launch_k(query_cond_kernel, dim3(blocks), dim3(256), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop,
+    launch_k(query_cond_kernel, dim3(blocks), dim3(EIRENE_QTHREADS), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop,
              c.wval, c.wleaf, c.wslot, c.wparent, c.old, spay, c.pinfo, c.istart, c.longseg, A, t, ctl, cond);
   } else {
-    launch_k(query_kernel, dim3(blocks), dim3(256), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval,
+    launch_k(query_kernel, dim3(blocks), dim3(EIRENE_QTHREADS), 0, st, true, false, c.qkey, c.qseg, c.wkey, c.wseg, c.wop, c.wval,
              c.wleaf, c.wslot, c.wparent, c.old, spay, c.pinfo, c.istart, c.longseg, A, t, ctl);
   }
   ++*launches;

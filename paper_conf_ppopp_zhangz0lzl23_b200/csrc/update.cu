@@ -29,6 +29,10 @@
 
 #include "eirene_internal.cuh"
 
+#ifndef UPD_THREADS
+#define UPD_THREADS 128   // update-kernel CTA: 4 warps, six per SM (r3w: one 768-thread CTA per SM: cfg1 update 103 -> 111 us)
+#endif
+
 namespace eirene {
 
 namespace {
@@ -743,6 +747,9 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
 
 
 constexpr uint32_t UPD_LSYNC_CH = 16;   // writes per level-0 chunk under a split storm (r3t: 32 slower on cfg1)
+// Dynamic shared memory of batched_runs: per warp, the key + value blocks of up
+// to UPD_LSYNC_CH locked leaves and the kept plan (upserts before each key)
+constexpr size_t UPD_SMEM_PER_WARP = (size_t)UPD_LSYNC_CH * (2 * FAN * sizeof(uint64_t) + FAN);
 #ifndef UPD_BATCH
 #define UPD_BATCH 1   // A/B: 0 = every leaf run of a chunk through process_run, one after the other
 #endif
@@ -759,9 +766,13 @@ constexpr uint32_t UPD_LSYNC_CH = 16;   // writes per level-0 chunk under a spli
 // h of a split run: ek = the new leaf's first key, nid = its id.
 __device__ uint32_t batched_runs(const Ctx& C, uint32_t base, uint32_t bm, uint32_t eL, uint32_t lf, WarpStats& ws,
                                  uint64_t& ek, uint32_t& nid, bool& split) {
-  __shared__ uint64_t s_lk[4][UPD_LSYNC_CH][2 * FAN];   // [warp of the CTA][run head lane][key 0-15, value 0-15]
+  // [run head lane][key 0-15, value 0-15] of this warp (dynamic shared memory, UPD_SMEM_PER_WARP per warp)
+  extern __shared__ __align__(16) unsigned char upd_smem[];
   const int lane = lane_id();
-  const uint32_t w4 = (threadIdx.x >> 5) & 3u;
+  const uint32_t wi = threadIdx.x >> 5;
+  uint64_t (*s_lk)[2 * FAN] = reinterpret_cast<uint64_t (*)[2 * FAN]>(upd_smem + wi * UPD_SMEM_PER_WARP);
+  uint8_t (*s_ub)[FAN] = reinterpret_cast<uint8_t (*)[FAN]>(upd_smem + wi * UPD_SMEM_PER_WARP +
+                                                            (size_t)UPD_LSYNC_CH * 2 * FAN * sizeof(uint64_t));
   const Tree& t = C.t;
   const bool mine = ((bm >> lane) & 1u) && lf < t.leaf_cap;
   uint32_t* vp = &t.lmeta[mine ? lf : 0].version;
@@ -797,7 +808,7 @@ __device__ uint32_t batched_runs(const Ctx& C, uint32_t base, uint32_t bm, uint3
     }
 #pragma unroll
     for (int u = 0; u < 4; ++u)
-      if (r[u] >= 0) s_lk[w4][r[u]][lane] = x[u];
+      if (r[u] >= 0) s_lk[r[u]][lane] = x[u];
   }
   __syncwarp();
   const bool ok = got && k0 >= lo && k0 < hi && kl < hi;   // key in range(leaf) (Alg.1:38)
@@ -805,15 +816,14 @@ __device__ uint32_t batched_runs(const Ctx& C, uint32_t base, uint32_t bm, uint3
   const uint32_t om = __ballot_sync(FULL, ok);
   // plan: every run's size after the merge -> in place (0), one leaf (1) or two
   // (2); the plan is kept (lane r: c, mmask; smem: upserts before each leaf key)
-  __shared__ uint8_t s_ub[4][UPD_LSYNC_CH][FAN];
   uint32_t tout_l = 0, k_l = 1, c_l = 0, mm_l = 0;
   for (uint32_t m = om; m; m &= m - 1) {
     const int r = __ffs(m) - 1;
     const uint32_t re = __shfl_sync(FULL, eL, r);
-    const uint64_t okey = lane < FAN ? s_lk[w4][r][lane] : KEY_MAX;
+    const uint64_t okey = lane < FAN ? s_lk[r][lane] : KEY_MAX;
     const LeafPlan L = leaf_plan(C, base + r, re, okey);
     const uint32_t tout = L.c - __popc(L.mmask) + L.U;
-    if (lane < FAN) s_ub[w4][r][lane] = (uint8_t)L.ups_before;
+    if (lane < FAN) s_ub[r][lane] = (uint8_t)L.ups_before;
     if (lane == r) {
       tout_l = tout;
       k_l = L.inplace ? 0u : (tout <= FAN ? 1u : 2u);
@@ -829,16 +839,16 @@ __device__ uint32_t batched_runs(const Ctx& C, uint32_t base, uint32_t bm, uint3
     const int r = __ffs(m) - 1;
     const uint32_t re = __shfl_sync(FULL, eL, r), X = __shfl_sync(FULL, lf, r);
     const uint32_t kr = __shfl_sync(FULL, k_l, r), tr = __shfl_sync(FULL, tout_l, r), idr = __shfl_sync(FULL, nid, r);
-    const uint64_t okey = lane < FAN ? s_lk[w4][r][lane] : KEY_MAX;
+    const uint64_t okey = lane < FAN ? s_lk[r][lane] : KEY_MAX;
     if (kr == 0) {
       leaf_overwrite(C, X, base + r, re, okey);
       continue;
     }
-    const uint64_t oval = lane < FAN ? s_lk[w4][r][FAN + lane] : 0ull;
+    const uint64_t oval = lane < FAN ? s_lk[r][FAN + lane] : 0ull;
     LeafPlan L;
     L.c = __shfl_sync(FULL, c_l, r);
     L.mmask = __shfl_sync(FULL, mm_l, r);
-    L.ups_before = lane < FAN ? s_ub[w4][r][lane] : 0u;
+    L.ups_before = lane < FAN ? s_ub[r][lane] : 0u;
     L.inplace = false;
     const uint64_t k1 = leaf_place(C, X, idr, base + r, re, okey, oval, L, tr, kr, nullptr, nullptr);
     if (lane == r) ek = k1;
@@ -995,7 +1005,7 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
       // walks 32-entry units instead of gathering unit by unit.
       // (1) per CTA: its warps' (= producers') counts and their offsets inside
       // the CTA; (2) CTA 0 scans the CTA totals; (3) every warp's offset
-      __shared__ uint32_t s_woff[4], s_cta;
+      __shared__ uint32_t s_woff[UPD_THREADS / 32], s_cta;
       if (threadIdx.x == 0) {
         uint32_t run = 0;
         for (uint32_t w = 0; w < (blockDim.x >> 5); ++w) {
@@ -1007,7 +1017,7 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
       }
       grid_barrier(C.ctl, gen);
       if (blockIdx.x == 0) {
-        __shared__ uint32_t s_part[128];
+        __shared__ uint32_t s_part[UPD_THREADS];
         const uint32_t nc = gridDim.x, per = (nc + blockDim.x - 1) / blockDim.x;
         const uint32_t a0 = threadIdx.x * per, z0 = min(nc, a0 + per);
         uint32_t v[16];   // per <= 16 (<= 2048 CTAs)
@@ -1243,35 +1253,51 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
 }
 
 #ifndef UPD_MINB
+#if UPD_THREADS == 128
 #define UPD_MINB 6   // resident CTAs per SM the register budget is fitted to (A/B builds: -DUPD_MINB=n;
                      // r1h: 6 (80 regs, no spills) vs 8 (64 regs, 432 B spills): cfg1 0.389 -> 0.404, cfg2 6.92 -> 7.04)
+#else
+#define UPD_MINB 1   // one CTA of UPD_THREADS per SM (the same 24 warps at 80 registers)
+#endif
 #endif
 __device__ __forceinline__ void update_body(const Ctx& C);
 
 // The batch's last kernel: the structural writes (Alg.1:23-46), then every
 // CTA's share of the long-segment RESULT_CAL and the batch's BatchCtl
 // (result_phase, eirene_internal.cuh) -- one launch for both.
-__global__ void __launch_bounds__(128, UPD_MINB) update_kernel(Ctx C, ResultArgs R) {
+__global__ void __launch_bounds__(UPD_THREADS, UPD_MINB) update_kernel(Ctx C, ResultArgs R) {
   pdl_wait();   // predecessor kernel complete, its writes visible (no-op without PDL)
   pdl_trigger();
   const BatchCtl* ctl = C.ctl;
-  // nothing at all left (no structural write, long segment or deferred hot
-  // key; the common case of a read-mostly batch): CTA 0 ends the batch at
-  // once, no arrival counting, the other CTAs just exit
-  if (!update_needed(ctl, R.A)) {
+  // What is left, read by ONE thread per CTA (every thread of every CTA
+  // loading the same flags made a same-address load storm: r3v, a no-op update
+  // kernel took 11 us with 3552 warps loading, 7.5 us with 592):
+  //   0: nothing (no structural write, long segment or deferred hot key; the
+  //      common case of a read-mostly batch): CTA 0 ends the batch at once, no
+  //      arrival counting, the other CTAs just exit;
+  //   1: the result phase only: a rejected batch, or every issued write was a
+  //      value overwrite of a present key, all applied in place by the query
+  //      kernel's locate (query.cu, retire) -- nothing structural is left;
+  //   2: structural writes, then the result phase.
+  // (Uniform: every CTA reads the same flags before any changes them.)
+  __shared__ uint32_t s_mode;
+  if (threadIdx.x == 0) {
+    uint32_t m = 0;
+    if (update_needed(ctl, R.A))
+      m = (ctl->invalid || ctl->status != 0 || (ctl->nins == 0 && ctl->ndelp == 0)) ? 1u : 2u;
+    s_mode = m;
+  }
+  __syncthreads();
+  const uint32_t mode = s_mode;
+  if (mode == 0) {
     if (blockIdx.x == 0) {
       if (threadIdx.x == 0) C.ctl->upd_ran = 1;
       publish_batch(C.ctl, R.A, R.hdr);
     }
     return;
   }
-  // skipped (uniformly: every CTA reads the same flags before any changes them)
-  // for a rejected batch, and when every issued write was a value overwrite of
-  // a present key: all of them were applied in place by the query kernel's
-  // locate (query.cu, retire), nothing structural is left
-  const bool skip = ctl->invalid || ctl->status != 0 || (ctl->nins == 0 && ctl->ndelp == 0);
   if (blockIdx.x == 0 && threadIdx.x == 0) C.ctl->upd_ran = 1;
-  if (!skip) update_body(C);
+  if (mode == 2) update_body(C);
   result_phase(R);
 }
 
@@ -1495,15 +1521,24 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
   C.flat_child = p.flat_child;
   C.flat_off = p.flat_off;
   const uint32_t warps_needed = C.regroup ? (n + 31) / 32 : n;
-  uint32_t blocks = (warps_needed + 3) / 4;
+  constexpr uint32_t WPC = UPD_THREADS / 32;
+  const size_t dsm = WPC * UPD_SMEM_PER_WARP;
+  uint32_t blocks = (warps_needed + WPC - 1) / WPC;
+  static int attr[MAX_DEVICES];
+  per_device(attr, [dsm] {
+    return (int)cudaFuncSetAttribute(update_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)dsm);
+  });
   // the level-synchronous phases need every CTA resident (grid barriers)
   static int occ[MAX_DEVICES];
-  const int per_sm = per_device(occ, [] {
+  const int per_sm = per_device(occ, [dsm] {
     int v = 0;
-    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, update_kernel, 128, 0) == cudaSuccess ? v : 0;
+    return cudaOccupancyMaxActiveBlocksPerMultiprocessor(&v, update_kernel, UPD_THREADS, dsm) == cudaSuccess ? v : 0;
   });
   const uint32_t resident = (uint32_t)num_sms * (uint32_t)std::max(per_sm, 0);
   blocks = std::min<uint32_t>(blocks, resident ? resident : (uint32_t)num_sms * 4u);
+#ifdef UPD_MAXCTAS   // diagnostic: launch-overhead floor of the update kernel
+  blocks = std::min<uint32_t>(blocks, (uint32_t)UPD_MAXCTAS);
+#endif
   if (blocks < 1) blocks = 1;
   static const bool no_lsync = std::getenv("EIRENE_NO_LSYNC") != nullptr;   // A/B: per-warp insertion only
   if (!resident || no_lsync) C.slots[0] = nullptr;   // no residency guarantee: per-warp insertion only
@@ -1514,12 +1549,12 @@ void launch_update(uint32_t n, const CombBufs& c, Tree t, BatchCtl* ctl, UpdPara
     return (int)cudaMemcpyToSymbol(g_uprof, &on, sizeof(int));
   });
   if (serial) {
-    update_kernel<<<1, 32, 0, st>>>(C, r);
+    update_kernel<<<1, 32, dsm, st>>>(C, r);
   } else {
     if (C.slots[0]) {   // grid barriers: a resident-sized grid (cooperative only with EIRENE_COOP=1, launch_k)
-      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, true, C, r);
+      launch_k(update_kernel, dim3(blocks), dim3(UPD_THREADS), dsm, st, true, true, C, r);
     } else {
-      launch_k(update_kernel, dim3(blocks), dim3(128), 0, st, true, false, C, r);
+      launch_k(update_kernel, dim3(blocks), dim3(UPD_THREADS), dsm, st, true, false, C, r);
     }
   }
   ++*launches;
