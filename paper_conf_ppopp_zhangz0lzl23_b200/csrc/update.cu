@@ -987,7 +987,12 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
   const Tree& t = C.t;
   for (uint32_t L = 0; L + 1 < MAX_LEVELS; ++L) {
     grid_barrier(C.ctl, gen);
-    if (ld_cg(&C.ctl->lvl_ent[L]) == 0) return;   // uniform: read after the barrier by every warp
+    // (uniform: read after the barrier, by one thread per CTA -- every thread
+    // loading the same word is an L2 same-address storm)
+    __shared__ uint32_t s_lv;
+    if (threadIdx.x == 0) s_lv = ld_cg(&C.ctl->lvl_ent[L]);
+    __syncthreads();
+    if (s_lv == 0) return;
     const uint2* sl = C.slots[L & 1];
     uint2* sn = C.slots[(L + 1) & 1];
     uint64_t* K = C.eK[L & 1];
@@ -1047,10 +1052,14 @@ __device__ void levels_up(const Ctx& C, uint32_t U, uint32_t gw, uint32_t nwarps
         }
       }
       grid_barrier(C.ctl, gen);
-      ftotal = ld_cg(&C.ctl->flat_total);
       // copy my unit into the flat list and look its entries' parents up (lanes over entries)
-      if (threadIdx.x == 0) s_cta = ld_cg(C.flat_off + blockIdx.x);
+      __shared__ uint32_t s_ft;
+      if (threadIdx.x == 0) {
+        s_ft = ld_cg(&C.ctl->flat_total);
+        s_cta = ld_cg(C.flat_off + blockIdx.x);
+      }
       __syncthreads();
+      ftotal = s_ft;
       for (uint32_t u = u0; u < u1; ++u) {   // (u == gw: my own unit)
         const uint2 su = sl[u];
         const uint32_t off = s_cta + s_woff[threadIdx.x >> 5];
