@@ -165,6 +165,26 @@ __device__ __forceinline__ void st_result(tkey_t* p, uint64_t v) {
 #endif
 }
 
+// The CTA's structural-write counts (nins, ndelp): zeroed by q_zero before the
+// first retire, added to the BatchCtl by q_flush after the last (both by every
+// thread of the CTA: they synchronise it).
+__device__ __forceinline__ uint32_t* q_counts() {
+  __shared__ uint32_t qc[2];
+  return qc;
+}
+__device__ __forceinline__ void q_zero() {
+  if (threadIdx.x < 2) q_counts()[threadIdx.x] = 0;
+  __syncthreads();
+}
+__device__ __forceinline__ void q_flush(BatchCtl* ctl) {
+  __syncthreads();
+  const uint32_t* qc = q_counts();
+  if (threadIdx.x == 0) {
+    if (qc[0]) atomicAdd(&ctl->nins, qc[0]);
+    if (qc[1]) atomicAdd(&ctl->ndelp, qc[1]);
+  }
+}
+
 __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, uint32_t nq, uint32_t node, int s,
                                        uint64_t v, tkey_t* __restrict__ results, BatchCtl* __restrict__ ctl,
                                        tkey_t* __restrict__ lvals) {
@@ -210,11 +230,13 @@ __device__ __forceinline__ void retire(const QueryIO& io, uint32_t i, bool isq, 
     // present ones) to do, and re-applies overwrites idempotently.
     if (s >= 0 && op != OP_DELETE) lvals[(size_t)node * LSTRIDE + s] = wv;
   }
-  {
+  {   // counted per CTA in shared memory (q_counts), added to ctl once per CTA (q_flush): one global
+      // atomic per warp on the same word serialised in L2 under insert-heavy batches
     const uint32_t am = __activemask();
     const uint32_t m = __ballot_sync(am, ins), md = __ballot_sync(am, delp);
-    if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&ctl->nins, (uint32_t)__popc(m));
-    if (md && (threadIdx.x & 31) == __ffs(md) - 1) atomicAdd(&ctl->ndelp, (uint32_t)__popc(md));
+    uint32_t* qc = q_counts();
+    if (m && (threadIdx.x & 31) == __ffs(m) - 1) atomicAdd(&qc[0], (uint32_t)__popc(m));
+    if (md && (threadIdx.x & 31) == __ffs(md) - 1) atomicAdd(&qc[1], (uint32_t)__popc(md));
   }
   // old[seg] (the pre-batch value) is read by the result phase for long
   // segments and by the range kernel for written keys only
@@ -260,6 +282,7 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
     if (blockIdx.x == 0 && threadIdx.x == 0) ctl->status = EIRENE_EFULL;
     return;
   }
+  q_zero();
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
   const uint64_t pl = pol_evict_last(), pf = pol_evict_first();
@@ -321,6 +344,7 @@ __device__ __forceinline__ void query_body(const uint64_t* __restrict__ qkey,
     retire(QueryIO{qseg, wseg, wop, wval, A->vals, wleaf, wslot, old, spay, pinfo, istart, longseg}, i, isq, nq, node, s, v,
            results, ctl, t.lvals);
   }
+  q_flush(ctl);
 }
 
 // End of the query kernel in graph mode (cond != 0): its last CTA decides
@@ -423,6 +447,7 @@ __device__ __forceinline__ void query_iterwarp_body(const uint64_t* __restrict__
     return;
   }
   const uint32_t rq = (nq + 31) / 32, nrg = rq + (nw + 31) / 32;
+  q_zero();
   const unsigned long long rw = t.hdr->root_word;
   const uint32_t height = (uint32_t)(rw >> 32), root = (uint32_t)rw;
   const uint32_t lane = threadIdx.x & 31;
@@ -488,6 +513,7 @@ __device__ __forceinline__ void query_iterwarp_body(const uint64_t* __restrict__
     atomicAdd(&ctl->rg_vertical, nvert);
     atomicAdd(&ctl->rg_horizontal, nhor);
   }
+  q_flush(ctl);
 }
 
 __global__ void __launch_bounds__(256, 4) query_iterwarp_kernel(const uint64_t* __restrict__ qkey,
