@@ -104,6 +104,7 @@ struct BatchCtl {
   unsigned long long uprof[24];   // diagnostic (EIRENE_UPDATE_PROF): update-kernel phase timestamps
   unsigned long long leaf_runs, retries, stm_fallbacks, leaf_splits, inner_splits, new_leaves, new_inner;
   uint32_t dbg[8];   // watchdog diagnostics
+  uint32_t ustripe[8][32];   // update kernel: level-0 chunk claims, one counter per stripe, each on its own line
 };
 
 // Device watchdog: spin / retry loops give up after this long and report

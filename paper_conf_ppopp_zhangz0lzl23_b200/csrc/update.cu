@@ -746,6 +746,12 @@ __device__ void process_run(const Ctx& C, uint32_t b, uint32_t e, uint32_t hint,
 }
 
 
+#ifndef UPD_BATCH_LAST
+#define UPD_BATCH_LAST 1   // A/B: 0 = the chunk's last run always through process_run
+#endif
+#ifndef UPD_STRIPES
+#define UPD_STRIPES 1   // level-0 chunk-claim counters (r4a: 8 striped counters: cfg4 update 508 -> 523 us)
+#endif
 constexpr uint32_t UPD_LSYNC_CH = 16;   // writes per level-0 chunk under a split storm (r3t: 32 slower on cfg1)
 // Dynamic shared memory of batched_runs: per warp, the key + value blocks of up
 // to UPD_LSYNC_CH locked leaves and the kept plan (upserts before each key)
@@ -1337,6 +1343,28 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
     // tail imbalance costs more than the claims' atomics on one address)
     const uint32_t G = 1u;
     uint32_t c_next = 0, c_end = 0;
+#if UPD_STRIPES > 1
+    // (and spread over UPD_STRIPES counters on their own lines: the chunks are
+    // cut into that many contiguous stripes, a warp starts on stripe gw % S and
+    // moves on when its stripe is exhausted -- the same dynamic balance with
+    // 1/S of the same-address atomics per counter)
+    (void)G;
+    (void)c_end;
+    const uint32_t NS = UPD_STRIPES, ssz = (nchunks + NS - 1) / NS;
+    uint32_t stripe = gw % NS, tried = 0;
+    auto next_chunk = [&]() -> uint32_t {
+      while (tried < NS) {
+        uint32_t c = 0;
+        if (lane == 0) c = atomicAdd(&C.ctl->ustripe[stripe][0], 1u);
+        c = __shfl_sync(FULL, c, 0);
+        const uint32_t ch = stripe * ssz + c;
+        if (c < ssz && ch < nchunks) return ch;
+        stripe = (stripe + 1) % NS;
+        ++tried;
+      }
+      return nchunks;   // (ends the loop: chunk * CH >= nw)
+    };
+#else
     auto next_chunk = [&]() -> uint32_t {
       if (c_next == c_end) {
         uint32_t c = 0;
@@ -1346,6 +1374,7 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
       }
       return c_next++;
     };
+#endif
     uint32_t lvl0 = 0;   // this warp's level-0 entries (one atomic per warp, not per chunk)
     for (uint32_t chunk = lsync ? next_chunk() : gw; chunk * CH < nw;
          chunk = lsync ? next_chunk() : chunk + nwarps) {
@@ -1407,7 +1436,31 @@ __device__ __forceinline__ void update_body(const Ctx& C) {
       if (lsync && !ws.leaf_root && !C.force_stm && C.threshold > 0) {
         const uint32_t later_l = allheads & ~((2u << lane) - 1u);
         bool cand = ((heads >> lane) & 1u) && later_l != 0;
-        const uint32_t eL = cand ? base + __ffs(later_l) - 1 : 0u;
+        uint32_t eL = cand ? base + __ffs(later_l) - 1 : 0u;
+#if UPD_BATCH_LAST
+        // the chunk's last run (its end may lie in the next chunk, whose warp
+        // skips it): its end found as process_run's caller would, then batched
+        // too if short -- so a chunk is one batch, not a batch and a chain
+        if (allheads) {
+          const int hl = 31 - __clz(allheads);
+          if ((heads >> hl) & 1u) {
+            const uint32_t leaf = __shfl_sync(FULL, lf, hl);
+            uint32_t e = nw;
+            for (uint32_t s2 = base + CH; s2 < nw; s2 += 32) {
+              const uint32_t jj = s2 + lane;
+              const uint32_t mk = __ballot_sync(FULL, jj < nw && C.wleaf[jj] != leaf);
+              if (mk) {
+                e = s2 + __ffs(mk) - 1;
+                break;
+              }
+            }
+            if (lane == hl) {
+              cand = true;
+              eL = e;
+            }
+          }
+        }
+#endif
         cand = cand && eL - (base + lane) <= (uint32_t)FAN;   // <= 16 writes: at most two leaves (batched_runs)
         const uint32_t bm = __ballot_sync(FULL, cand);
         if (__popc(bm) >= 2) {
