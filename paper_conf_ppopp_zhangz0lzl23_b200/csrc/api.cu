@@ -12,6 +12,7 @@
 // pipeline.  No allocation and no host synchronisation happen inside submit.
 // Graphs are captured per size bucket; pipelined handles (EIRENE_F_PIPELINE)
 // split each batch into a front and a back graph on two streams (§7.2).
+#include <algorithm>
 #include <atomic>
 #include <cstdio>
 #include <cstdlib>
@@ -669,6 +670,32 @@ static int get_graph(eirene_handle h, GraphEntry* table, uint32_t& next, uint32_
   cudaError_t ee = cudaStreamEndCapture(h->cap_stream, &e.graph);
   if (ce != cudaSuccess) return cuda_fail(ce, "capture");
   CK(ee);
+  // A/B (EIRENE_L2WIN=MB): an L2 persisting access-policy window over the
+  // first MB of the inner nodes' separator lines on every kernel node
+  static const int l2win = std::getenv("EIRENE_L2WIN") ? std::atoi(std::getenv("EIRENE_L2WIN")) : 0;
+  if (l2win > 0) {
+    int maxp = 0, maxw = 0;
+    cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, h->cfg.device);
+    cudaDeviceGetAttribute(&maxw, cudaDevAttrMaxAccessPolicyWindowSize, h->cfg.device);
+    const size_t want = std::min<size_t>({(size_t)l2win << 20, (size_t)maxp, (size_t)maxw,
+                                          (size_t)h->t.inner_cap * FAN * sizeof(tkey_t)});
+    cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
+    cudaLaunchAttributeValue v{};
+    v.accessPolicyWindow.base_ptr = h->t.ikeys;
+    v.accessPolicyWindow.num_bytes = want;
+    v.accessPolicyWindow.hitRatio = 1.0f;
+    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    size_t nn = 0;
+    CK(cudaGraphGetNodes(e.graph, nullptr, &nn));
+    std::vector<cudaGraphNode_t> nodes(nn);
+    CK(cudaGraphGetNodes(e.graph, nodes.data(), &nn));
+    for (cudaGraphNode_t nd : nodes) {
+      cudaGraphNodeType ty;
+      if (cudaGraphNodeGetType(nd, &ty) == cudaSuccess && ty == cudaGraphNodeTypeKernel)
+        CK(cudaGraphKernelNodeSetAttribute(nd, cudaLaunchAttributeAccessPolicyWindow, &v));
+    }
+  }
   CK(cudaGraphInstantiate(&e.exec, e.graph, 0));
   e.n = nk;
   e.range = range;
