@@ -228,12 +228,13 @@ def run_reference(args):
     for s in range(args.warmup + args.steps):
         ops, keys, vals = wl.batch_arrays(s)
         ops, keys, vals = ops[:sample], keys[:sample], vals[:sample]
-        a = time.perf_counter()
-        if cap:
-            t.apply_range(ops, keys, vals, cap)
-        else:
-            t.apply(ops, keys, vals)
-        dt = time.perf_counter() - a
+        with pinned_core():
+            a = time.perf_counter()
+            if cap:
+                t.apply_range(ops, keys, vals, cap)
+            else:
+                t.apply(ops, keys, vals)
+            dt = time.perf_counter() - a
         if s >= args.warmup:
             times.append(dt)
             total += sample
@@ -678,12 +679,14 @@ def run_ours(args):
         for b in range(n_check):
             ref = refs[step_tree[b]]
             o, k, v = host_batches[b]
-            a = time.perf_counter()
-            if cap:
-                want, wk, wv = ref.apply_range(o, k, v, cap)
-            else:
-                want = ref.apply(o, k, v)
-            cpu_t += time.perf_counter() - a
+            with pinned_core() as pc:
+                a = time.perf_counter()
+                if cap:
+                    want, wk, wv = ref.apply_range(o, k, v, cap)
+                else:
+                    want = ref.apply(o, k, v)
+                cpu_t += time.perf_counter() - a
+            pin_core = pc.core
             got = widen_np(results[b].cpu().numpy())
             bad += int(np.sum(got != want))
             if cap:
@@ -694,7 +697,8 @@ def run_ours(args):
         parity = {"batches_checked": n_check, "mismatches": bad, "vs": "oracle B+tree, every request, bit-exact"}
         cpu = {"value": n_check * batch_n / cpu_t / 1e9, "unit": "Greq/s", "cores": 1, "host_cores": os.cpu_count(), "kind": "oracle",
                "sample": f"first {n_check} batches of the same workload ({n_check * batch_n} requests), "
-                         f"sequential B+tree, 1 thread; bulk load {load_s:.1f}s untimed"}
+                         f"sequential B+tree, 1 thread pinned to core {pin_core} (sched_setaffinity); "
+                         f"bulk load {load_s:.1f}s untimed"}
         # roofline of the dominant kernel
         peaks = load_peaks()
         dom = int(np.argmax(stage_ms))
@@ -843,6 +847,20 @@ def run_ours(args):
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
+
+
+class pinned_core:
+    """Pin this process to one host core while the (single-threaded) oracle is timed; restore afterwards."""
+
+    def __enter__(self):
+        self.prev = os.sched_getaffinity(0)
+        self.core = max(self.prev)
+        os.sched_setaffinity(0, {self.core})
+        return self
+
+    def __exit__(self, *exc):
+        os.sched_setaffinity(0, self.prev)
+        return False
 
 
 def main():
